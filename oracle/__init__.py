@@ -1,0 +1,149 @@
+"""TEST INFRASTRUCTURE ONLY — the CPU oracle for the SpMV hot path.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
+``cpu_baseline`` / ``--impl reference`` legs may import this package. The
+product path (``paper_conf_sc_dastgeerlk12_b200``) never imports it and shares
+no code with it.
+
+Every function is a thin ctypes call into ``oracle/oracle.c`` (plain C,
+``-O2 -ffp-contract=off``); see that file's header for the paper passages each
+one follows. Pins: ``tests/test_oracle_pins.py`` (dense brute force,
+permutation, diagonal, Laplacian closed forms, exact-sum bound, power-of-two
+scaling, partition brute force) — none of them re-calls this code to make its
+expected value.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared", "-fPIC",
+          "-std=c11", "-Wall", "-Wno-unknown-pragmas"]
+
+
+def build(force: bool = False) -> str:
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", *CFLAGS, _SRC, "-o", _LIB, "-lm"])
+    return _LIB
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_LIB)
+        i64 = ctypes.c_int64
+        p = ctypes.c_void_p
+        L.oracle_spmv_seq.argtypes = [i64, i64, p, p, p, p, p]
+        L.oracle_spmv_rows_parallel.argtypes = [i64, i64, p, p, p, p, p]
+        L.oracle_spmv_row.argtypes = [i64, i64, p, p, p, p]
+        L.oracle_spmv_row.restype = ctypes.c_double
+        L.oracle_abs_rowsum.argtypes = [i64, i64, p, p, p, p, p]
+        L.oracle_spmv_iterate.argtypes = [i64, i64, i64, p, p, p, p, p, p, p]
+        L.oracle_partition_nnz.argtypes = [i64, i64, p, i64, p]
+        _lib = L
+    return _lib
+
+
+def _c(a, dt):
+    a = np.ascontiguousarray(a, dtype=dt)
+    return a
+
+
+def _args(row_ptr, col, val):
+    rp = _c(row_ptr, np.int64)
+    c = _c(col, np.int32)
+    v = _c(val, np.float64)
+    return rp, c, v
+
+
+def _ptr(a):
+    return a.ctypes.data if a.size else None
+
+
+def spmv(A, x, parallel: bool = False) -> np.ndarray:
+    """y = A·x for a CSR (gen.CSR-like: nrows, row_ptr, col, val) — the definition."""
+    rp, c, v = _args(A.row_ptr, A.col, A.val)
+    xx = _c(x, np.float64)
+    y = np.empty(A.nrows, dtype=np.float64)
+    f = lib().oracle_spmv_rows_parallel if parallel else lib().oracle_spmv_seq
+    if A.nrows:
+        f(A.nrows, int(rp[0]), _ptr(rp), _ptr(c), _ptr(v), _ptr(xx), _ptr(y))
+    return y
+
+
+def spmv_raw(nrows, first, row_ptr, col, val, x, parallel=False) -> np.ndarray:
+    rp, c, v = _args(row_ptr, col, val)
+    xx = _c(x, np.float64)
+    y = np.empty(nrows, dtype=np.float64)
+    f = lib().oracle_spmv_rows_parallel if parallel else lib().oracle_spmv_seq
+    if nrows:
+        f(nrows, first, _ptr(rp), _ptr(c), _ptr(v), _ptr(xx), _ptr(y))
+    return y
+
+
+def spmv_rows(A, x, rows) -> np.ndarray:
+    """y_i for sampled rows i only (full-size parity)."""
+    rp, c, v = _args(A.row_ptr, A.col, A.val)
+    xx = _c(x, np.float64)
+    L = lib()
+    first = int(rp[0])
+    return np.array([L.oracle_spmv_row(int(i), first, _ptr(rp), _ptr(c), _ptr(v), _ptr(xx))
+                     for i in rows], dtype=np.float64)
+
+
+def abs_rowsum(A, x) -> np.ndarray:
+    """S_i = Σ |a_ij||x_j| (bound ingredient)."""
+    rp, c, v = _args(A.row_ptr, A.col, A.val)
+    xx = _c(x, np.float64)
+    s = np.empty(A.nrows, dtype=np.float64)
+    if A.nrows:
+        lib().oracle_abs_rowsum(A.nrows, int(rp[0]), _ptr(rp), _ptr(c), _ptr(v), _ptr(xx), _ptr(s))
+    return s
+
+
+def row_lengths(A) -> np.ndarray:
+    return np.diff(np.asarray(A.row_ptr, dtype=np.int64))
+
+
+def bound(A, x) -> np.ndarray:
+    """Per-row tolerance of BASELINE.json north_star: 2·nnz_row·2^-52·Σ|a||x|."""
+    return 2.0 * row_lengths(A).astype(np.float64) * 2.0 ** -52 * abs_rowsum(A, x)
+
+
+def iterate(A, x0, K: int, with_bound: bool = False):
+    """x_K = A^K x0 (reading A11); optionally z_K = |A|^K |x0| (P7)."""
+    rp, c, v = _args(A.row_ptr, A.col, A.val)
+    x = _c(x0, np.float64).copy()
+    n = A.nrows
+    tmp = np.empty(n)
+    z = np.empty(n) if with_bound else None
+    zt = np.empty(n) if with_bound else None
+    lib().oracle_spmv_iterate(K, n, int(rp[0]), _ptr(rp), _ptr(c), _ptr(v), _ptr(x), _ptr(tmp),
+                              _ptr(z) if with_bound else None, _ptr(zt) if with_bound else None)
+    return (x, z) if with_bound else x
+
+
+def iterate_bound(A, zK: np.ndarray, K: int) -> np.ndarray:
+    """Propagated componentwise bound of P7: 2·K·γ_w·(1+γ_w)^K·(|A|^K|x0|)."""
+    w = int(row_lengths(A).max()) if A.nrows else 0
+    u = 2.0 ** -53
+    g = w * u / (1 - w * u)
+    return 2.0 * K * g * (1 + g) ** K * zK
+
+
+def partition_nnz(A, P: int) -> np.ndarray:
+    rp = _c(A.row_ptr, np.int64)
+    b = np.empty(P + 1, dtype=np.int64)
+    lib().oracle_partition_nnz(A.nrows, int(rp[0]), _ptr(rp), P, _ptr(b))
+    return b
