@@ -1,0 +1,452 @@
+#!/usr/bin/env python3
+"""Benchmark of the SpMV hot path (BASELINE.json metric: SpMV GFLOP/s and
+achieved HBM GB/s (% of HBM) at 1/2/4/8 B200).
+
+Default workload = BASELINE.json config 4: 2D 5-point Laplacian on an
+8192x8192 grid (67,108,864 rows, 335,511,552 nnz, fp64), 100 iterated SpMVs
+x_{k+1} = A·x_k per step, rows nnz-balanced over N ranks (one process per
+GPU), NCCL exchange of y between iterations. The matrix (5.4 GB of
+algorithmic bytes per SpMV) is far larger than L2 (126 MB), so no flush is
+needed between iterations. Every step goes through the C-ABI
+(pepp_spmv_exec per iteration: per-call variant selection + kernel +
+exchange + history update).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--workload lap8192|uniform1m|zipf4m|lap64] [--iters I] [--variant csr_vector:4|merge_path|sell]
+
+One JSON line on rank 0. Multi-GPU: launched by torchrun (RANK / WORLD_SIZE /
+LOCAL_RANK / MASTER_* from the environment); times are device events, max
+over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    "lap8192": dict(desc="BASELINE config 4: 2D 5-point Laplacian 8192x8192 (67.1M rows, 335.5M nnz), fp64, "
+                         "100 iterated SpMVs per step, nnz-balanced row blocks over N GPUs, NCCL exchange",
+                    iters=100, iterated=True),
+    "uniform1m": dict(desc="BASELINE config 2: uniform random 1M x 1M, 16 nnz/row (16.8M nnz), fp64",
+                      iters=20, iterated=False),
+    "zipf4m": dict(desc="BASELINE config 3: power-law rows P(k)~k^-1.5, k<=435, 4M x 4M (~67M nnz), fp64",
+                   iters=20, iterated=False),
+    "lap64": dict(desc="BASELINE config 1: 2D 5-point Laplacian 64x64 (4096 rows, 20224 nnz), fp64",
+                  iters=1000, iterated=False),
+}
+
+
+# --------------------------------------------------------------- inputs
+def make_block(workload: str, r0: int, r1: int):
+    import gen
+    if workload == "lap8192":
+        return gen.laplacian2d(8192, r0, r1)
+    if workload == "lap64":
+        return gen.laplacian2d(64, r0, r1)
+    if workload == "uniform1m":
+        return gen.uniform(1 << 20, 1 << 20, 16, seed=42, r0=r0, r1=r1)
+    if workload == "zipf4m":
+        return gen.zipf(4 << 20, 4 << 20, seed=46, r0=r0, r1=r1)
+    raise ValueError(workload)
+
+
+def global_rowptr(workload: str) -> np.ndarray:
+    import ctypes
+
+    import gen
+    if workload in ("lap8192", "lap64"):
+        n = 8192 if workload == "lap8192" else 64
+        rp = np.empty(n * n + 1, dtype=np.int64)
+        gen.lib().gen_laplacian2d_rowptr(n, 0, n * n, rp.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)))
+        return rp
+    if workload == "uniform1m":
+        return np.arange(0, ((1 << 20) + 1) * 16, 16, dtype=np.int64)
+    return gen._rowptr_global(1, 46, 4 << 20, 4 << 20, 1.5, 435, 0, 4 << 20)
+
+
+def x0_vector(workload: str, n: int) -> np.ndarray:
+    import gen
+    return gen.vector(4, gen.REAL, n)   # real x0 ~ U[-1,1) (config 4's real mode, seed 4)
+
+
+# --------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+        self.out = None
+
+    def start(self):
+        try:
+            self.out = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=self.out, stderr=subprocess.DEVNULL)
+        except (OSError, FileNotFoundError):
+            self.proc = None
+
+    def stop(self) -> dict | None:
+        if not self.proc:
+            return None
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.out.flush()
+        self.out.seek(0)
+        rows = [l.strip().split(", ") for l in self.out.read().splitlines() if l.strip()]
+        os.unlink(self.out.name)
+        if not rows:
+            return None
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        loaded = [v for v in sm if v > 0.5 * (max(mx) if mx else 1)] or sm
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            for i, nm in enumerate(names):
+                if len(r) > 5 + i and r[5 + i].strip().lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(rows)}
+
+
+# --------------------------------------------------------------- helpers
+def measured_peak() -> tuple[float, str]:
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        return float(json.load(open(p))["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except (OSError, KeyError, ValueError):
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def traffic_for(kernel: str, workload: str):
+    """dram read+write bytes per launch from the committed ncu --set full summary, if any."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        d = json.load(open(p))
+        return d.get(workload, {}).get(kernel)
+    except (OSError, ValueError):
+        return None
+
+
+def parse_variant(s: str | None):
+    import paper_conf_sc_dastgeerlk12_b200 as pepp
+    if not s:
+        return None
+    name, _, prm = s.partition(":")
+    v = {"csr_vector": pepp.V_CSR_VECTOR, "merge_path": pepp.V_MERGE_PATH, "sell": pepp.V_SELL}[name]
+    return pepp.Choice(v, int(prm) if prm else 0)
+
+
+def cpu_baseline(A, x0: np.ndarray, iters: int) -> dict:
+    """The oracle as it stands (test infrastructure), on the host cores."""
+    import oracle
+    cores = os.cpu_count()
+    t0 = time.perf_counter()
+    x = x0
+    for _ in range(iters):
+        x = oracle.spmv(A, x, parallel=True)
+    t = time.perf_counter() - t0
+    gflops = 2.0 * A.nnz * iters / t / 1e9
+    # single-core sequential oracle on one iteration (the paper's "serial C++" role, P@33595)
+    t1 = time.perf_counter()
+    oracle.spmv(A, x0, parallel=False)
+    ts = time.perf_counter() - t1
+    return {"value": round(gflops, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+            "sample": f"{iters} full-size SpMV(s) of the bench matrix ({A.nnz} nnz) with "
+                      f"oracle_spmv_rows_parallel on {cores} OpenMP threads",
+            "seq_1core_gflops": round(2.0 * A.nnz / ts / 1e9, 3)}
+
+
+# --------------------------------------------------------------- arms
+def run_reference(args, rank: int, world: int) -> None:
+    """--impl reference: the CPU oracle (no code was published with the paper)."""
+    if rank != 0:
+        return
+    import oracle
+    wl = WORKLOADS[args.workload]
+    A = make_block(args.workload, 0, len(global_rowptr(args.workload)) - 1)
+    x = x0_vector(args.workload, A.ncols)
+    for _ in range(args.warmup):
+        oracle.spmv(A, x, parallel=True)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.spmv(A, x, parallel=True)
+    t = time.perf_counter() - t0
+    flops = 2.0 * A.nnz * args.steps
+    val = flops / t / 1e9
+    cores = os.cpu_count()
+    sample = (f"each step = 1 of the {wl['iters']} SpMVs of a {args.workload} step, full matrix "
+              f"({A.nnz} nnz), oracle_spmv_rows_parallel on {cores} threads")
+    line = {"impl": "reference", "metric": "SpMV GFLOP/s (aggregate)", "value": round(val, 3), "unit": "GFLOP/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(1000 * t / args.steps, 3), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": args.workload, "desc": wl["desc"]},
+            "cpu_baseline": {"value": round(val, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": round(val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_ours(args, rank: int, world: int, local_rank: int) -> None:
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_dastgeerlk12_b200 as pepp
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    wl = WORKLOADS[args.workload]
+    iters = args.iters or wl["iters"]
+    iterated = wl["iterated"]
+
+    # ---- partition (a2) + this rank's block ----
+    rp_global = global_rowptr(args.workload)
+    R = len(rp_global) - 1
+    Z = int(rp_global[-1])
+    bounds = pepp.partition_rows(rp_global, world)
+    r0, r1 = int(bounds[rank]), int(bounds[rank + 1])
+    del rp_global
+    A = make_block(args.workload, r0, r1)
+    x0 = x0_vector(args.workload, A.ncols)
+
+    uid = None
+    if world > 1:
+        obj = [pepp.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    plan = pepp.Plan.from_csr(A, nranks=world, rank=rank, row_bounds=bounds if world > 1 else None,
+                              nccl_unique_id=uid)
+    info = plan.info()
+    force = parse_variant(args.variant)
+    flags = pepp.Y_NEXT_INPUT if iterated else pepp.Y_LOCAL
+
+    stream = torch.cuda.Stream(device=dev)
+    xs = torch.from_numpy(x0).to(dev)
+    bufs = [torch.empty(R, dtype=torch.float64, device=dev) for _ in range(2)]
+    flush = None if iterated or Z * 12 > 4 * (1 << 30) else torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+
+    ev_pool = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(iters)]
+    launches = {"n": 0}
+    used_count: dict = {}
+
+    def one_step(record: bool):
+        """`iters` SpMVs through the C-ABI. Iterated: x0 -> b0 -> b1 -> b0 ...
+        (x0 stays resident and is only read, so every step restarts from it)."""
+        kernel_ms = []
+        with torch.cuda.stream(stream):
+            src = xs
+            for k in range(iters):
+                dst = bufs[k & 1]
+                if not iterated:
+                    src = xs
+                    if flush is not None:
+                        flush.zero_()
+                a, b = ev_pool[k]
+                if record:
+                    a.record(stream)
+                u = plan.exec(src, dst, flags=flags, stream=stream, force=force)
+                if record:
+                    b.record(stream)
+                    used_count[u.name] = used_count.get(u.name, 0) + 1
+                    launches["n"] += 2 if u.variant == pepp.V_MERGE_PATH else 1
+                if iterated:
+                    src = dst
+        return kernel_ms
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for _ in range(args.warmup):
+        one_step(False)
+    torch.cuda.synchronize()
+    barrier()
+
+    # ---- timed region ----
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    time.sleep(0.3)
+    barrier()
+    torch.cuda.synchronize()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    kern_ms = []
+    t_start.record(stream)
+    for _ in range(args.steps):
+        one_step(True)
+        # harvest this step's per-launch kernel times (the events are reused next step)
+        torch.cuda.current_stream(dev).wait_stream(stream)
+        stream.synchronize()
+        kern_ms.extend(a.elapsed_time(b) for a, b in ev_pool)
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    clk = clocks.stop()
+    total_ms = t_start.elapsed_time(t_end)
+    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_ms = float(t.item())
+
+    nspmv = iters * args.steps
+    alg_bytes_global = Z * 12 + (R + 1) * 4 + A.ncols * 8 + R * 8
+    if iterated:
+        secs = total_ms / 1e3
+    else:
+        # single-SpMV workloads: L2 flushed between calls; time = sum of kernel events
+        secs = sum(kern_ms) / 1e3
+        tk = torch.tensor([secs], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tk, op=dist.ReduceOp.MAX)
+        secs = float(tk.item())
+    gflops = 2.0 * Z * nspmv / secs / 1e9
+    gbs = alg_bytes_global * nspmv / secs / 1e9
+    peak, peak_src = measured_peak()
+
+    # roofline of the dominant kernel on this rank (rank 0 reports)
+    avg_kernel_s = statistics.mean(kern_ms) / 1e3
+    local_bytes = A.nnz * 12 + (A.nrows + 1) * 4 + (A.nrows + info["halo_recv"]) * 8 + A.nrows * 8
+    if world == 1:
+        local_bytes = alg_bytes_global
+    achieved = local_bytes / avg_kernel_s / 1e9
+    chosen = max(used_count, key=used_count.get) if used_count else "?"
+
+    # ---- selector quality: every candidate timed after the timed region (same run) ----
+    sel = None
+    if not args.no_sweep:
+        per = {}
+        for c in plan.candidates():
+            f = pepp.Choice(c.variant, c.param)
+            ts = []
+            with torch.cuda.stream(stream):
+                src = xs
+                for k in range(min(iters, 10) + 2):
+                    if flush is not None:
+                        flush.zero_()
+                    a, b = ev_pool[k % len(ev_pool)]
+                    a.record(stream)
+                    plan.exec(src, bufs[k & 1], flags=flags, stream=stream, force=f)
+                    b.record(stream)
+                    b.synchronize()
+                    if k >= 2:
+                        ts.append(a.elapsed_time(b))
+                    if iterated:
+                        src = bufs[k & 1]
+            per[f.name] = statistics.median(ts) * 1e3
+        best = min(per, key=per.get)
+        sel = {"chosen": chosen, "chosen_us": round(per.get(chosen, float("nan")), 2), "best": best,
+               "best_us": round(per[best], 2), "ratio": round(per.get(chosen, float("nan")) / per[best], 4),
+               "candidates_us": {k: round(v, 2) for k, v in per.items()}}
+
+    # ---- e2e: host buffers through the C-ABI (pepp_spmv_exec_host) ----
+    xh = torch.from_numpy(x0).pin_memory().numpy() if torch.cuda.is_available() else x0
+    yh = torch.empty(R, dtype=torch.float64).pin_memory().numpy()
+    e2e_iters = iters if iterated else 1
+    e2e_flags = flags
+    plan.exec_host(xh, yh, iterations=e2e_iters, flags=e2e_flags, stream=stream)   # warm
+    barrier()
+    e2e_steps = max(1, min(args.steps, 5 if iterated else args.steps))
+    te = time.perf_counter()
+    for _ in range(e2e_steps):
+        plan.exec_host(xh, yh, iterations=e2e_iters, flags=e2e_flags, stream=stream)
+    te = time.perf_counter() - te
+    tt = torch.tensor([te], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    te = float(tt.item())
+    e2e_val = 2.0 * Z * e2e_iters * e2e_steps / te / 1e9
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(A, x0, 2 if A.nnz > 10_000_000 else 200)
+
+    if rank == 0:
+        kname = chosen
+        line = {
+            "metric": "SpMV GFLOP/s (aggregate over ranks); achieved HBM GB/s in 'hbm'",
+            "value": round(gflops, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": args.workload, "desc": wl["desc"], "spmv_per_step": iters,
+                       "rows": R, "nnz": Z, "l2": "inputs larger than L2 (5.4 GB/SpMV)" if iterated
+                       else "L2 flushed (512 MB memset) between SpMVs; kernel events only",
+                       "exchange": pepp._capi.EXCHANGE_NAMES.get(info["exchange"], "?"),
+                       "variant": args.variant or "auto (history-based per call)"},
+            "hbm": {"achieved_gbs": round(gbs, 1), "frac_of_measured": round(gbs / (world * peak), 4),
+                    "frac_of_8tbs": round(gbs / (world * 8000.0), 4), "algorithmic_bytes_per_spmv": alg_bytes_global},
+            "roofline": {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
+                         "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4),
+                         "avg_launch_us": round(avg_kernel_s * 1e6, 2), "bytes_per_launch": local_bytes,
+                         "traffic": traffic_for(kname, args.workload)},
+            "e2e": {"value": round(e2e_val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": A.ncols * 8,
+                    "d2h_bytes_per_step": A.nrows * 8, "spmv_per_step": e2e_iters,
+                    "api": "pepp_spmv_exec_host (pinned host x0 -> iterations -> host y)"},
+            "gpu_launches": launches["n"],
+            "selector": sel,
+            "clocks": clk,
+            "cpu_baseline": cpu,
+            "plan": {k: info[k] for k in ("mean_row", "cv_row", "max_row", "sell_sigma", "sell_fill",
+                                          "device_bytes", "halo_recv", "halo_send")},
+            "choices": used_count,
+        }
+        print(json.dumps(line), flush=True)
+    plan.close()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", choices=sorted(WORKLOADS), default="lap8192")
+    ap.add_argument("--iters", type=int, default=0)
+    ap.add_argument("--variant", default=None)
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        if args.impl == "reference":
+            run_reference(args, rank, world)
+        else:
+            run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

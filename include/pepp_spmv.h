@@ -1,0 +1,301 @@
+/*
+ * pepp_spmv.h — C-ABI of the B200-native SpMV hot path (libpepp_spmv.so).
+ *
+ * The operation is the PEPPHER composition example component
+ *
+ *     void spmv(float* values, int nnz, int nrows, int ncols, int first,
+ *               size_t* colidxs, size_t* rowPtr, float* x, float* y);
+ *
+ * (Dastgeer, Li, Kessler, MuCoCoS 2012, §V-A; PAPER.md P@32944 + P@31037 —
+ * the signature is split by the PDF extraction, garble G1 of SURVEY.md §0):
+ *
+ *     y[i] = Σ_{k = rowPtr[i]-first}^{rowPtr[i+1]-first-1} values[k] · x[colidxs[k]]
+ *
+ * re-designed as plan / select / exec / destroy:
+ *   - pepp_spmv_plan    ~ PEPPHER_INITIALIZE + smart-container registration
+ *                          ("register once", §IV-H P@28291–29611): validates,
+ *                          extracts the context instance (§III P@9781),
+ *                          copies the operand into device memory it owns and
+ *                          prepares every implementation variant (§II P@4772).
+ *   - pepp_spmv_select  ~ the runtime's performance-aware variant choice from
+ *                          recorded history (dynamic composition §III
+ *                          P@10254–10489; useHistoryModels P@28038, P@29611).
+ *   - pepp_spmv_exec    ~ the generated entry-wrapper (§IV-C P@16839): one call,
+ *                          asynchronous (P@17990), partitioned over ranks whose
+ *                          outputs concatenate (§IV-F P@27330–28000).
+ *   - pepp_spmv_destroy ~ PEPPHER_SHUTDOWN (P@33881).
+ *
+ * Precision and index widths (readings A2, A3): values, x, y and all
+ * sums are fp64; column indices int32; row pointers int64 at the ABI (the
+ * paper's size_t) — narrowed to int32 on the device (nnz < 2^31 required;
+ * larger blocks return PEPP_E_UNSUPPORTED).
+ *
+ * Access modes follow the paper's interface descriptor (read / write /
+ * readwrite, §II P@4233) and the const / non-const inference of the utility
+ * mode (§IV-I P@31894): every `const T*` argument is READ, `double* y` is
+ * WRITE (not read; y = A·x, not y += A·x — reading A4).
+ *
+ * Errors: every entry point returns pepp_status_t; no abort, no exception and
+ * no exit crosses the ABI. A CUDA error inside a plan is sticky for that plan
+ * (PEPP_E_CUDA on every later call), like a CUDA context error.
+ * Threading: a plan is not thread-safe; distinct plans are independent.
+ * There is NO CPU fallback: a machine without a CUDA device gets PEPP_E_CUDA
+ * from pepp_spmv_plan. The host-only utilities at the end of this header
+ * (partition, halo lists, history/selector) run without a GPU.
+ */
+#ifndef PEPP_SPMV_H
+#define PEPP_SPMV_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PEPP_ABI_VERSION 1
+
+typedef enum {
+    PEPP_OK = 0,
+    PEPP_E_INVALID = -1,      /* bad argument or malformed CSR              */
+    PEPP_E_CUDA = -2,         /* CUDA runtime error (sticky per plan)       */
+    PEPP_E_NCCL = -3,         /* NCCL missing or failed                     */
+    PEPP_E_NOMEM = -4,        /* host or device allocation failed          */
+    PEPP_E_UNSUPPORTED = -5,  /* valid but not supported (e.g. nnz >= 2^31) */
+    PEPP_E_STATE = -6         /* call not valid in the object's state       */
+} pepp_status_t;
+
+/* Implementation variants (§II P@4772: "several implementations of one
+   interface"; the paper's CUSP variant P@33595 is replaced by three
+   hand-written sm_100a kernels). */
+typedef enum {
+    PEPP_V_AUTO = -1,
+    PEPP_V_CSR_VECTOR = 0,    /* TPR lanes per row, 128-bit val/col loads, shfl_xor reduction; param = TPR */
+    PEPP_V_MERGE_PATH = 1,    /* merge-path over (row ends, nnz), smem-staged, deterministic carry fix-up */
+    PEPP_V_SELL = 2,          /* SELL-C-σ, C = 32, column-major chunks; param = σ */
+    PEPP_V_COUNT = 3
+} pepp_variant_t;
+
+/* Exchange that makes y usable as the next x when the call is partitioned */
+typedef enum {
+    PEPP_X_AUTO = -1,
+    PEPP_X_NONE = 0,          /* single rank                                          */
+    PEPP_X_ALLGATHER = 1,     /* allgatherv of y slices: every rank gets all of y     */
+    PEPP_X_HALO = 2           /* ghost (halo) exchange: only entries peers' rows read */
+} pepp_exchange_t;
+
+/* exec flags: which part of y is valid on return (once the stream completes) */
+#define PEPP_Y_LOCAL       0x0  /* own rows only: y[row_offset, row_offset+nrows)              */
+#define PEPP_Y_NEXT_INPUT  0x1  /* own rows + every entry this plan's next call reads as x     */
+#define PEPP_Y_REPLICATED  0x2  /* all global rows (allgatherv)                                */
+#define PEPP_EXEC_NO_TIMING 0x10 /* do not record event timing for this call (e.g. graph capture) */
+
+/* CSR operand (the paper's tuple, G1). Row i of this block holds entries
+   [row_ptr[i] - first, row_ptr[i+1] - first) of col_idx / values (reading
+   A1: `first` is the row-pointer base, so a rank can pass a slice of a
+   global rowPtr unchanged; column indices are 0-based and global).
+   Invariants checked by pepp_spmv_plan: row_ptr[0] == first,
+   row_ptr[nrows] - first == nnz, row_ptr non-decreasing, 0 <= col < ncols.
+   Duplicate or unsorted columns within a row are allowed and summed (A8).
+   All three arrays are READ; host memory if on_device == 0, else device
+   memory on the plan's device. The plan copies what it needs: the caller may
+   free them as soon as pepp_spmv_plan returns. */
+typedef struct {
+    int64_t nrows;            /* rows in this block                          */
+    int64_t ncols;            /* columns = length of x (global)              */
+    int64_t nnz;              /* entries in this block                       */
+    int64_t first;            /* row_ptr base (paper's `first`)              */
+    const int64_t* row_ptr;   /* [nrows + 1]                                 */
+    const int32_t* col_idx;   /* [nnz]                                       */
+    const double* values;     /* [nnz]                                       */
+    int32_t on_device;        /* 0 = host pointers, 1 = device pointers      */
+} pepp_csr_t;
+
+/* Plan options. Use pepp_spmv_opts_default() then override. */
+typedef struct {
+    uint32_t variant_mask;    /* bit v set = variant v allowed; 0 = all (the paper's disableImpls, P@16687) */
+    int32_t use_history;      /* 1 = history-based dynamic selection (default; useHistoryModels P@28038);
+                                 0 = fixed heuristic from the context instance */
+    int32_t validate;         /* 1 = full O(nnz) check of the CSR invariants (default) */
+    int32_t sell_sigma;       /* SELL sorting window σ (rows); 0 = chosen from the padding ratio */
+    int32_t device;           /* CUDA device ordinal; -1 = the caller's current device */
+    int32_t min_samples;      /* timed calls per candidate before exploiting (default 3) */
+    int32_t sample_period;    /* after calibration, time every N-th call (default 8; 0 = never) */
+    /* partitioning (§IV-F intra-component parallelism, P@27330–28000) */
+    int32_t nranks;           /* ranks the global matrix is split over (1 = unpartitioned) */
+    int32_t rank;             /* this process's rank */
+    const int64_t* row_bounds;/* [nranks + 1] global row boundaries (x is split the same way; square A);
+                                 NULL when nranks == 1. This block is rows [row_bounds[rank], row_bounds[rank+1]) */
+    void* nccl_comm;          /* borrowed ncclComm_t, or NULL */
+    const void* nccl_unique_id; /* 128-byte ncclUniqueId (same on every rank) when nccl_comm is NULL and nranks > 1 */
+    int32_t exchange;         /* pepp_exchange_t; AUTO = halo when ghosts are < 1/4 of ncols, else allgather */
+    const char* history_path; /* if set: history loaded at plan, saved at destroy (NEXT-f2 persistence) */
+} pepp_spmv_opts_t;
+
+/* Selection result. `candidate` indexes pepp_spmv_candidates(). */
+typedef struct {
+    int32_t variant;          /* pepp_variant_t */
+    int32_t param;            /* TPR (CSR_VECTOR), σ (SELL), items per thread (MERGE_PATH) */
+    int32_t nparts;           /* ranks the call runs on */
+    int32_t exchange;         /* pepp_exchange_t used when flags ask for it */
+    int32_t calibrating;      /* 1 = chosen to gather history, not the predicted best */
+    int32_t candidate;        /* index in the plan's candidate list */
+    double predicted_us;      /* history mean of this candidate (0 if unknown) */
+} pepp_choice_t;
+
+/* Context instance (§III P@9781: "a tuple of concrete values for context
+   properties that might influence callee selection") + plan facts. */
+typedef struct {
+    int64_t nrows, ncols, nnz;
+    double mean_row;          /* nnz / nrows */
+    double cv_row;            /* coefficient of variation of row lengths */
+    int64_t max_row;          /* longest row */
+    int64_t empty_rows;
+    int32_t nranks, rank;
+    int64_t row_offset;       /* global index of this block's first row */
+    uint64_t key;             /* history key derived from the bucketed context */
+    int32_t ncandidates;
+    int32_t sell_sigma;       /* σ of the prepared SELL layout (0 if not prepared) */
+    double sell_fill;         /* SELL stored slots / nnz (>= 1) */
+    int64_t device_bytes;     /* device memory owned by the plan */
+    int64_t algorithmic_bytes;/* nnz*12 + (nrows+1)*4 + ncols*8 + nrows*8 */
+    int32_t exchange;         /* resolved pepp_exchange_t */
+    int64_t halo_recv;        /* ghost entries received per exchange (halo) */
+    int64_t halo_send;        /* entries sent per exchange (halo) */
+} pepp_plan_info_t;
+
+typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */
+
+/* ---- core calls ----------------------------------------------------- */
+
+/* Human-readable name of a status code (static storage; never NULL). */
+const char* pepp_status_str(pepp_status_t s);
+
+/* Fill *opts with the defaults documented above. */
+void pepp_spmv_opts_default(pepp_spmv_opts_t* opts);
+
+/* Build a plan for A on opts->device. Copies A; the plan owns all device
+   memory it allocates. Collective over ranks when opts->nranks > 1 (every
+   rank must call it with its own row block). On error *out is NULL.
+   Errors: PEPP_E_INVALID (NULL args, broken CSR invariants, bad options),
+   PEPP_E_CUDA (no device / CUDA failure), PEPP_E_NOMEM, PEPP_E_NCCL,
+   PEPP_E_UNSUPPORTED (nnz >= 2^31 in one block, ncols >= 2^31). */
+pepp_status_t pepp_spmv_plan(const pepp_csr_t* A, const pepp_spmv_opts_t* opts,
+                             pepp_spmv_plan_t** out);
+
+/* The choice pepp_spmv_exec(force = NULL) would make now. Host only: no
+   device synchronisation; harvests finished timing events without blocking.
+   Budget: < 2 µs (the paper's runtime task overhead, P@40366). */
+pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_choice_t* out);
+
+/* y = A·x for this plan's rows, enqueued on `stream` (cudaStream_t; NULL =
+   legacy default stream) and returned without waiting (asynchronous, P@17990).
+   x: READ, device, ncols entries (global length), not modified, must not
+      overlap y.
+   y: WRITE, device, global-length buffer (row_bounds[nranks] entries when
+      partitioned, else nrows); this block's rows land at
+      y[row_offset .. row_offset+nrows). With PEPP_Y_NEXT_INPUT /
+      PEPP_Y_REPLICATED the exchange then fills ghost / all entries from the
+      other ranks (NCCL, same stream). Entries not covered by `flags` are
+      left untouched.
+   force: NULL = automatic selection; else force->variant/param (and
+      force->exchange when partitioned) select the implementation.
+   used: optional; receives the choice that ran.
+   Errors: PEPP_E_INVALID (NULL / aliasing / unknown forced variant or
+   masked-out variant), PEPP_E_CUDA, PEPP_E_NCCL, PEPP_E_STATE (exchange
+   requested on an unpartitioned plan is fine and a no-op; a plan in a sticky
+   error state returns its error). */
+pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const double* x, double* y, int flags,
+                             void* stream, const pepp_choice_t* force, pepp_choice_t* used);
+
+/* Host-buffer entry point (the paper's measurement setting, where operand
+   transfers are part of the call: Fig. 5 "communication overhead of copying
+   data back and forth to device memory is also included", P@35591–35720).
+   Copies x_host (READ, host, ncols entries; pinned memory gives full PCIe /
+   C2C speed) into a plan-owned device buffer, runs `iterations` >= 1 calls
+   x_{k+1} = A·x_k (iterations > 1 needs a square global matrix: ncols ==
+   global rows, reading A11) with the exchange `flags` asks for
+   (PEPP_Y_NEXT_INPUT is implied between iterations when partitioned), then
+   copies the final y into y_host (WRITE, host, global-length; all global rows
+   with PEPP_Y_REPLICATED, else only this rank's rows are written) and waits
+   for completion on `stream`.
+   The plan-owned device buffers are allocated on first use and kept
+   ("register once", P@29208). Errors as pepp_spmv_exec. */
+pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const double* x_host, double* y_host, int32_t iterations,
+                                  int flags, void* stream);
+
+/* Free everything the plan owns (device memory, events, an owned NCCL
+   communicator); saves history to opts.history_path if set. Waits for the
+   plan's outstanding work. NULL is a no-op. */
+pepp_status_t pepp_spmv_destroy(pepp_spmv_plan_t* p);
+
+/* ---- introspection -------------------------------------------------- */
+
+pepp_status_t pepp_spmv_plan_info(const pepp_spmv_plan_t* p, pepp_plan_info_t* out);
+
+/* Copy up to `cap` candidates (variant, param, exchange) into out; *n gets the total. */
+pepp_status_t pepp_spmv_candidates(const pepp_spmv_plan_t* p, pepp_choice_t* out, int32_t cap, int32_t* n);
+
+/* Block until every recorded timing is available and fold it into the history. */
+pepp_status_t pepp_spmv_flush_history(pepp_spmv_plan_t* p);
+
+/* History statistics of candidate `cand` for this plan's key. */
+pepp_status_t pepp_spmv_history_stats(const pepp_spmv_plan_t* p, int32_t cand,
+                                      int64_t* count, double* mean_us, double* m2);
+
+/* ---- host-only utilities (no GPU needed) ---------------------------- */
+
+/* nnz-balanced contiguous row blocks (reading A9; P@27578):
+   bounds[p] = min{ r : row_ptr[r] - first >= ceil(p*nnz/nparts) } for
+   0 < p < nparts, bounds[0] = 0, bounds[nparts] = nrows.
+   row_ptr: READ host [nrows+1]; bounds: WRITE host [nparts+1]. */
+pepp_status_t pepp_partition_rows(const int64_t* row_ptr, int64_t nrows, int64_t first,
+                                  int32_t nparts, int64_t* bounds);
+
+/* Ghost (halo) columns of one row block: the sorted distinct columns of
+   col_idx[0..nnz) that lie outside [row_bounds[rank], row_bounds[rank+1]),
+   grouped by owning rank. counts: WRITE [nranks] (count per owner; own rank
+   gets 0). ghosts: WRITE, capacity `cap` entries, sorted ascending (so
+   grouped by owner); *total gets the number of ghosts (may exceed cap, in
+   which case only counts/total are valid). Host memory only. */
+pepp_status_t pepp_halo_ghosts(const int32_t* col_idx, int64_t nnz, int32_t nranks, int32_t rank,
+                               const int64_t* row_bounds, int64_t* counts, int32_t* ghosts,
+                               int64_t cap, int64_t* total);
+
+/* ---- history / selector object (host only; the plan embeds one) ------ */
+/* A history table keyed by (context key, candidate id) with Welford
+   count / mean / M2 of measured times — the runtime's "performance history"
+   (P@10254). Exposed so the selection policy is testable without a GPU
+   (inject times with pepp_history_record). */
+typedef struct pepp_history pepp_history;
+
+pepp_status_t pepp_history_create(pepp_history** out);
+pepp_status_t pepp_history_destroy(pepp_history* h);
+pepp_status_t pepp_history_record(pepp_history* h, uint64_t key, int32_t cand, double us);
+pepp_status_t pepp_history_stats(const pepp_history* h, uint64_t key, int32_t cand,
+                                 int64_t* count, double* mean_us, double* m2);
+/* Policy (reading A10): among candidates with eligible[c] != 0, if any has
+   fewer than min_samples records, return the lowest such c with
+   *calibrating = 1; else return argmin mean time, ties within 1 % going to
+   the lower index, *calibrating = 0. *predicted_us = that candidate's mean. */
+pepp_status_t pepp_history_select(const pepp_history* h, uint64_t key, int32_t ncand,
+                                  const uint8_t* eligible, int32_t min_samples,
+                                  int32_t* cand, int32_t* calibrating, double* predicted_us);
+pepp_status_t pepp_history_save(const pepp_history* h, const char* path);
+pepp_status_t pepp_history_load(pepp_history* h, const char* path);
+
+/* Context key of a row-pointer array (host): bucketed (log2 rows, log2 nnz,
+   mean row length, CV, nparts) — the "context instance" used as history key. */
+uint64_t pepp_context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts);
+
+/* NCCL bootstrap helper: write a fresh 128-byte ncclUniqueId into id_out
+   (NCCL is loaded on demand with dlopen; PEPP_E_NCCL if unavailable). */
+pepp_status_t pepp_nccl_unique_id(void* id_out);
+
+/* ABI version (PEPP_ABI_VERSION) of the loaded library. */
+int32_t pepp_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PEPP_SPMV_H */

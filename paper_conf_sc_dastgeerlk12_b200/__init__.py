@@ -1,0 +1,262 @@
+"""B200-native SpMV hot path of the PEPPHER composition tool (Dastgeer, Li,
+Kessler, MuCoCoS 2012): y = A·x over CSR in fp64, three hand-written sm_100a
+variants, per-call history-based variant selection, nnz-balanced row
+partitioning over ranks with NCCL exchange.
+
+This module is the thin Python binding of ``include/pepp_spmv.h``: it only
+marshals arguments (pointers, sizes, the caller's CUDA stream) into
+``libpepp_spmv.so``. Every step of the path runs in that library's kernels.
+Device memory, streams and process groups come from PyTorch (plumbing).
+There is no CPU fallback: importing works without a GPU, but planning needs
+the CUDA library and a device and fails loudly otherwise.
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+from typing import Optional, Sequence
+
+import numpy as np
+
+from . import _capi as C
+from ._capi import (EXEC_NO_TIMING, PeppError, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, X_ALLGATHER, X_AUTO,
+                    X_HALO, X_NONE, Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, VARIANT_NAMES)
+
+__all__ = ["Plan", "Choice", "History", "partition_rows", "halo_ghosts", "context_key", "nccl_unique_id",
+           "lib_path", "PeppError", "V_CSR_VECTOR", "V_MERGE_PATH", "V_SELL", "X_AUTO", "X_NONE",
+           "X_ALLGATHER", "X_HALO", "Y_LOCAL", "Y_NEXT_INPUT", "Y_REPLICATED", "EXEC_NO_TIMING",
+           "VARIANT_NAMES"]
+
+lib_path = C.LIB_PATH
+
+
+@dataclass
+class Choice:
+    variant: int
+    param: int = 0
+    exchange: int = X_AUTO
+    nparts: int = 1
+    calibrating: bool = False
+    candidate: int = -1
+    predicted_us: float = 0.0
+
+    @property
+    def name(self) -> str:
+        return f"{VARIANT_NAMES.get(self.variant, self.variant)}[{self.param}]"
+
+    @staticmethod
+    def _from(c: C.CHOICE_T) -> "Choice":
+        return Choice(c.variant, c.param, c.exchange, c.nparts, bool(c.calibrating), c.candidate, c.predicted_us)
+
+    def _to(self) -> C.CHOICE_T:
+        c = C.CHOICE_T()
+        c.variant, c.param, c.exchange, c.nparts = self.variant, self.param, self.exchange, self.nparts
+        return c
+
+
+def _ptr(a) -> int:
+    """Raw address of a numpy array or torch tensor (no copy)."""
+    if a is None:
+        return 0
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data
+    return int(a.data_ptr())
+
+
+def _stream_handle(stream) -> int:
+    if stream is None:
+        import torch
+        return int(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return stream
+    return int(stream.cuda_stream)
+
+
+class Plan:
+    """pepp_spmv_plan over one CSR row block.
+
+    ``row_ptr`` (int64, global offsets: row_ptr[0] == first), ``col`` (int32),
+    ``val`` (float64): numpy host arrays, or CUDA torch tensors on the plan's
+    device (then ``on_device`` is inferred). The plan copies them.
+    """
+
+    def __init__(self, nrows: int, ncols: int, row_ptr, col, val, *, variant_mask: int = 0,
+                 use_history: bool = True, validate: bool = True, sell_sigma: int = 0,
+                 device: Optional[int] = None, min_samples: int = 3, sample_period: int = 8,
+                 nranks: int = 1, rank: int = 0, row_bounds: Optional[Sequence[int]] = None,
+                 nccl_unique_id: Optional[bytes] = None, exchange: int = X_AUTO,
+                 history_path: Optional[str] = None):
+        L = C.lib()
+        self._h = ctypes.c_void_p()
+        on_dev = not isinstance(row_ptr, np.ndarray)
+        if not on_dev:
+            row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+            col = np.ascontiguousarray(col, dtype=np.int32)
+            val = np.ascontiguousarray(val, dtype=np.float64)
+        nnz = int(col.shape[0]) if col is not None else 0
+        first = int(row_ptr[0]) if not on_dev else int(row_ptr[:1].cpu()[0])
+        A = C.CSR_T(nrows, ncols, nnz, first, _ptr(row_ptr), _ptr(col) if nnz else 0,
+                    _ptr(val) if nnz else 0, 1 if on_dev else 0)
+        o = C.OPTS_T()
+        L.pepp_spmv_opts_default(ctypes.byref(o))
+        o.variant_mask = variant_mask
+        o.use_history = 1 if use_history else 0
+        o.validate = 1 if validate else 0
+        o.sell_sigma = sell_sigma
+        o.device = -1 if device is None else device
+        o.min_samples = min_samples
+        o.sample_period = sample_period
+        o.nranks, o.rank = nranks, rank
+        self._bounds = None
+        if row_bounds is not None:
+            self._bounds = np.ascontiguousarray(row_bounds, dtype=np.int64)
+            o.row_bounds = self._bounds.ctypes.data
+        self._uid = None
+        if nccl_unique_id is not None:
+            self._uid = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+            o.nccl_unique_id = ctypes.addressof(self._uid)
+        o.exchange = exchange
+        self._hp = history_path.encode() if history_path else None
+        o.history_path = self._hp
+        C.check(L.pepp_spmv_plan(ctypes.byref(A), ctypes.byref(o), ctypes.byref(self._h)), "pepp_spmv_plan")
+        self.nrows, self.ncols, self.nnz = nrows, ncols, nnz
+
+    # ---- calls ----
+    def exec(self, x, y, flags: int = Y_LOCAL, stream=None, force: Optional[Choice] = None) -> Choice:
+        """y = A·x (x, y: CUDA float64 tensors; y global-length). Asynchronous on ``stream``."""
+        used = C.CHOICE_T()
+        f = force._to() if force is not None else None
+        C.check(C.lib().pepp_spmv_exec(self._h, _ptr(x), _ptr(y), flags, _stream_handle(stream),
+                                       ctypes.byref(f) if f is not None else None, ctypes.byref(used)),
+                "pepp_spmv_exec")
+        return Choice._from(used)
+
+    def exec_host(self, x_host: np.ndarray, y_host: np.ndarray, iterations: int = 1, flags: int = Y_LOCAL,
+                  stream=None) -> None:
+        """Host buffers in and out, transfers inside the call (synchronous)."""
+        assert x_host.dtype == np.float64 and y_host.dtype == np.float64
+        C.check(C.lib().pepp_spmv_exec_host(self._h, _ptr(x_host), _ptr(y_host), iterations, flags,
+                                            _stream_handle(stream)), "pepp_spmv_exec_host")
+
+    def select(self) -> Choice:
+        c = C.CHOICE_T()
+        C.check(C.lib().pepp_spmv_select(self._h, ctypes.byref(c)), "pepp_spmv_select")
+        return Choice._from(c)
+
+    def candidates(self) -> list[Choice]:
+        n = ctypes.c_int32()
+        C.check(C.lib().pepp_spmv_candidates(self._h, None, 0, ctypes.byref(n)), "pepp_spmv_candidates")
+        arr = (C.CHOICE_T * max(1, n.value))()
+        C.check(C.lib().pepp_spmv_candidates(self._h, arr, n.value, ctypes.byref(n)), "pepp_spmv_candidates")
+        return [Choice._from(arr[i]) for i in range(n.value)]
+
+    def info(self) -> dict:
+        i = C.INFO_T()
+        C.check(C.lib().pepp_spmv_plan_info(self._h, ctypes.byref(i)), "pepp_spmv_plan_info")
+        return i.as_dict()
+
+    def flush_history(self) -> None:
+        C.check(C.lib().pepp_spmv_flush_history(self._h), "pepp_spmv_flush_history")
+
+    def history_stats(self, cand: int) -> tuple[int, float, float]:
+        n, m, m2 = ctypes.c_int64(), ctypes.c_double(), ctypes.c_double()
+        C.check(C.lib().pepp_spmv_history_stats(self._h, cand, ctypes.byref(n), ctypes.byref(m), ctypes.byref(m2)),
+                "pepp_spmv_history_stats")
+        return n.value, m.value, m2.value
+
+    def close(self) -> None:
+        if getattr(self, "_h", None) and self._h.value:
+            C.check(C.lib().pepp_spmv_destroy(self._h), "pepp_spmv_destroy")
+            self._h = ctypes.c_void_p()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    @classmethod
+    def from_csr(cls, A, **kw) -> "Plan":
+        """From any object with nrows, ncols, row_ptr, col, val (e.g. gen.CSR)."""
+        return cls(A.nrows, A.ncols, A.row_ptr, A.col, A.val, **kw)
+
+
+class History:
+    """Stand-alone history table + selection policy (host only; see header)."""
+
+    def __init__(self):
+        self._h = ctypes.c_void_p()
+        C.check(C.lib().pepp_history_create(ctypes.byref(self._h)), "pepp_history_create")
+
+    def record(self, key: int, cand: int, us: float) -> None:
+        C.check(C.lib().pepp_history_record(self._h, key, cand, us), "pepp_history_record")
+
+    def stats(self, key: int, cand: int) -> tuple[int, float, float]:
+        n, m, m2 = ctypes.c_int64(), ctypes.c_double(), ctypes.c_double()
+        C.check(C.lib().pepp_history_stats(self._h, key, cand, ctypes.byref(n), ctypes.byref(m), ctypes.byref(m2)),
+                "pepp_history_stats")
+        return n.value, m.value, m2.value
+
+    def select(self, key: int, eligible: Sequence[bool], min_samples: int = 3) -> tuple[int, bool, float]:
+        e = np.ascontiguousarray([1 if v else 0 for v in eligible], dtype=np.uint8)
+        c, cal, pred = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_double()
+        C.check(C.lib().pepp_history_select(self._h, key, len(e), e.ctypes.data, min_samples, ctypes.byref(c),
+                                            ctypes.byref(cal), ctypes.byref(pred)), "pepp_history_select")
+        return c.value, bool(cal.value), pred.value
+
+    def save(self, path: str) -> None:
+        C.check(C.lib().pepp_history_save(self._h, path.encode()), "pepp_history_save")
+
+    def load(self, path: str) -> None:
+        C.check(C.lib().pepp_history_load(self._h, path.encode()), "pepp_history_load")
+
+    def close(self) -> None:
+        if self._h.value:
+            C.lib().pepp_history_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def partition_rows(row_ptr: np.ndarray, nparts: int) -> np.ndarray:
+    """nnz-balanced contiguous row blocks (pepp_partition_rows)."""
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    b = np.empty(nparts + 1, dtype=np.int64)
+    C.check(C.lib().pepp_partition_rows(rp.ctypes.data, len(rp) - 1, int(rp[0]), nparts, b.ctypes.data),
+            "pepp_partition_rows")
+    return b
+
+
+def halo_ghosts(col: np.ndarray, nranks: int, rank: int, row_bounds: Sequence[int]) -> tuple[np.ndarray, np.ndarray]:
+    """(counts per owner rank, sorted ghost columns) of one row block."""
+    c = np.ascontiguousarray(col, dtype=np.int32)
+    rb = np.ascontiguousarray(row_bounds, dtype=np.int64)
+    counts = np.zeros(nranks, dtype=np.int64)
+    total = ctypes.c_int64()
+    C.check(C.lib().pepp_halo_ghosts(c.ctypes.data if c.size else None, c.size, nranks, rank, rb.ctypes.data,
+                                     counts.ctypes.data, None, 0, ctypes.byref(total)), "pepp_halo_ghosts")
+    g = np.empty(max(1, total.value), dtype=np.int32)
+    C.check(C.lib().pepp_halo_ghosts(c.ctypes.data if c.size else None, c.size, nranks, rank, rb.ctypes.data,
+                                     counts.ctypes.data, g.ctypes.data, g.size, ctypes.byref(total)),
+            "pepp_halo_ghosts")
+    return counts, g[:total.value]
+
+
+def context_key(nrows: int, ncols: int, nnz: int, cv: float, nparts: int = 1) -> int:
+    return int(C.lib().pepp_context_key(nrows, ncols, nnz, cv, nparts))
+
+
+def nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    C.check(C.lib().pepp_nccl_unique_id(ctypes.addressof(buf)), "pepp_nccl_unique_id")
+    return buf.raw

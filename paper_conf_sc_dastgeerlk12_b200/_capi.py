@@ -1,0 +1,115 @@
+"""ctypes mirror of include/pepp_spmv.h (argument marshalling only).
+
+Loads the in-tree ``libpepp_spmv.so``; raises if it is missing — there is no
+CPU fallback anywhere on the product path.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libpepp_spmv.so")
+
+PEPP_OK, PEPP_E_INVALID, PEPP_E_CUDA, PEPP_E_NCCL, PEPP_E_NOMEM, PEPP_E_UNSUPPORTED, PEPP_E_STATE = 0, -1, -2, -3, -4, -5, -6
+V_AUTO, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, V_COUNT = -1, 0, 1, 2, 3
+X_AUTO, X_NONE, X_ALLGATHER, X_HALO = -1, 0, 1, 2
+Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, EXEC_NO_TIMING = 0x0, 0x1, 0x2, 0x10
+VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell"}
+EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_AUTO: "auto"}
+
+c_i32, c_i64, c_u32, c_u64, c_f64, c_vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_uint64,
+                                          ctypes.c_double, ctypes.c_void_p)
+
+
+class CSR_T(ctypes.Structure):
+    _fields_ = [("nrows", c_i64), ("ncols", c_i64), ("nnz", c_i64), ("first", c_i64),
+                ("row_ptr", c_vp), ("col_idx", c_vp), ("values", c_vp), ("on_device", c_i32)]
+
+
+class OPTS_T(ctypes.Structure):
+    _fields_ = [("variant_mask", c_u32), ("use_history", c_i32), ("validate", c_i32), ("sell_sigma", c_i32),
+                ("device", c_i32), ("min_samples", c_i32), ("sample_period", c_i32), ("nranks", c_i32),
+                ("rank", c_i32), ("row_bounds", c_vp), ("nccl_comm", c_vp), ("nccl_unique_id", c_vp),
+                ("exchange", c_i32), ("history_path", ctypes.c_char_p)]
+
+
+class CHOICE_T(ctypes.Structure):
+    _fields_ = [("variant", c_i32), ("param", c_i32), ("nparts", c_i32), ("exchange", c_i32),
+                ("calibrating", c_i32), ("candidate", c_i32), ("predicted_us", c_f64)]
+
+    def as_dict(self) -> dict:
+        return {"variant": VARIANT_NAMES.get(self.variant, str(self.variant)), "variant_id": self.variant,
+                "param": self.param, "nparts": self.nparts, "exchange": EXCHANGE_NAMES.get(self.exchange, "?"),
+                "calibrating": bool(self.calibrating), "candidate": self.candidate,
+                "predicted_us": self.predicted_us}
+
+
+class INFO_T(ctypes.Structure):
+    _fields_ = [("nrows", c_i64), ("ncols", c_i64), ("nnz", c_i64), ("mean_row", c_f64), ("cv_row", c_f64),
+                ("max_row", c_i64), ("empty_rows", c_i64), ("nranks", c_i32), ("rank", c_i32),
+                ("row_offset", c_i64), ("key", c_u64), ("ncandidates", c_i32), ("sell_sigma", c_i32),
+                ("sell_fill", c_f64), ("device_bytes", c_i64), ("algorithmic_bytes", c_i64),
+                ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64)]
+
+    def as_dict(self) -> dict:
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+# (name, restype, argtypes) for every entry point of include/pepp_spmv.h
+SIGNATURES = {
+    "pepp_status_str": (ctypes.c_char_p, [c_i32]),
+    "pepp_spmv_opts_default": (None, [ctypes.POINTER(OPTS_T)]),
+    "pepp_spmv_plan": (c_i32, [ctypes.POINTER(CSR_T), ctypes.POINTER(OPTS_T), ctypes.POINTER(c_vp)]),
+    "pepp_spmv_select": (c_i32, [c_vp, ctypes.POINTER(CHOICE_T)]),
+    "pepp_spmv_exec": (c_i32, [c_vp, c_vp, c_vp, ctypes.c_int, c_vp, ctypes.POINTER(CHOICE_T), ctypes.POINTER(CHOICE_T)]),
+    "pepp_spmv_exec_host": (c_i32, [c_vp, c_vp, c_vp, c_i32, ctypes.c_int, c_vp]),
+    "pepp_spmv_destroy": (c_i32, [c_vp]),
+    "pepp_spmv_plan_info": (c_i32, [c_vp, ctypes.POINTER(INFO_T)]),
+    "pepp_spmv_candidates": (c_i32, [c_vp, ctypes.POINTER(CHOICE_T), c_i32, ctypes.POINTER(c_i32)]),
+    "pepp_spmv_flush_history": (c_i32, [c_vp]),
+    "pepp_spmv_history_stats": (c_i32, [c_vp, c_i32, ctypes.POINTER(c_i64), ctypes.POINTER(c_f64), ctypes.POINTER(c_f64)]),
+    "pepp_partition_rows": (c_i32, [c_vp, c_i64, c_i64, c_i32, c_vp]),
+    "pepp_halo_ghosts": (c_i32, [c_vp, c_i64, c_i32, c_i32, c_vp, c_vp, c_vp, c_i64, ctypes.POINTER(c_i64)]),
+    "pepp_history_create": (c_i32, [ctypes.POINTER(c_vp)]),
+    "pepp_history_destroy": (c_i32, [c_vp]),
+    "pepp_history_record": (c_i32, [c_vp, c_u64, c_i32, c_f64]),
+    "pepp_history_stats": (c_i32, [c_vp, c_u64, c_i32, ctypes.POINTER(c_i64), ctypes.POINTER(c_f64), ctypes.POINTER(c_f64)]),
+    "pepp_history_select": (c_i32, [c_vp, c_u64, c_i32, c_vp, c_i32, ctypes.POINTER(c_i32), ctypes.POINTER(c_i32), ctypes.POINTER(c_f64)]),
+    "pepp_history_save": (c_i32, [c_vp, ctypes.c_char_p]),
+    "pepp_history_load": (c_i32, [c_vp, ctypes.c_char_p]),
+    "pepp_context_key": (c_u64, [c_i64, c_i64, c_i64, c_f64, c_i32]),
+    "pepp_nccl_unique_id": (c_i32, [c_vp]),
+    "pepp_abi_version": (c_i32, []),
+}
+
+_lib = None
+
+
+class PeppError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        super().__init__(f"{where}: {status_str(status)} ({status})")
+
+
+def lib() -> ctypes.CDLL:
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run `python build.py` (no CPU fallback exists)")
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in SIGNATURES.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def status_str(s: int) -> str:
+    return lib().pepp_status_str(s).decode()
+
+
+def check(status: int, where: str) -> None:
+    if status != PEPP_OK:
+        raise PeppError(status, where)

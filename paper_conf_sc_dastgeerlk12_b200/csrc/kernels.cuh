@@ -1,0 +1,436 @@
+// kernels.cuh — sm_100a kernels of the SpMV hot path (y = A·x over CSR, fp64).
+//
+// The paper's GPU variant was a library call into CUSP on Fermi / GT200
+// (PAPER.md P@33595, P@35591); these three hand-written variants replace it
+// (implementation variants of one interface, §II P@4772). SpMV is not a dense
+// contraction, so no tensor cores: every kernel is bound by HBM streaming of
+// val (8 B) + col (4 B) per nonzero; the design levers are
+// coalescing, 128-bit loads, bytes in flight, and keeping x in L2.
+//
+// Device CSR layout (built by plan.cu):
+//   rp[0..nrows]   int32, rp[i] = row_ptr[i] - first + pad, pad = first mod 4,
+//                  so the 4-element alignment of every entry equals its
+//                  alignment in the caller's global array (partition
+//                  invariance).
+//   col[], val[]   pad leading zeros + nnz entries + >= 4 trailing zeros
+//                  (val = 0, col = 0), 16-B aligned, so aligned 4-groups
+//                  never read out of bounds.
+//   x              global length; y points at this block's first row.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace pepp {
+namespace k {
+
+// ----------------------------------------------------------------- loads
+// Streaming loads for the matrix (read exactly once per call): non-coherent
+// path, no L1 allocation, L2 evict-first policy (createpolicy) so that x
+// keeps its L2 residency. (On sm_100a the bare .L2::evict_first qualifier is
+// only accepted on 256-bit loads; the cache_hint form works for every width.)
+__device__ __forceinline__ uint64_t evict_first_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ int4 ld_stream_i4(const int* p, uint64_t pol) {
+    int4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ double2 ld_stream_d2(const double* p, uint64_t pol) {
+    double2 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0,%1}, [%2], %3;"
+                 : "=d"(r.x), "=d"(r.y) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ double ld_stream_d(const double* p, uint64_t pol) {
+    double r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(r) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ int ld_stream_i(const int* p, uint64_t pol) {
+    int r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    return r;
+}
+// x gather: read-only path, cached in L1 and L2 (reused across rows)
+__device__ __forceinline__ double ld_x(const double* __restrict__ x, int c) { return __ldg(x + c); }
+
+// =====================================================================
+// Variant 0: vector-CSR with TPR lanes per row (TPR in {2,4,8,16,32}).
+// Each lane walks aligned 4-element groups of its row with stride TPR:
+// one int4 of columns + two double2 of values per group (3 x 16-B loads),
+// entries outside the row are masked. Partial sums are combined with a
+// __shfl_xor_sync butterfly over the TPR lanes. The row loop is warp-
+// uniform (all 32 lanes iterate together) so full-mask shuffles are legal.
+// =====================================================================
+template <int TPR, int BLOCK>
+__global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int* __restrict__ rp,
+                                                           const int* __restrict__ col,
+                                                           const double* __restrict__ val,
+                                                           const double* __restrict__ x,
+                                                           double* __restrict__ y) {
+    static_assert(TPR >= 1 && TPR <= 32 && (TPR & (TPR - 1)) == 0, "TPR must be a power of two <= 32");
+    constexpr int RPW = 32 / TPR;                 // rows per warp per step
+    const int lane = threadIdx.x & 31;
+    const int sub = lane & (TPR - 1);             // lane within the row group
+    const int grp = lane / TPR;                   // row group within the warp
+    const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
+    const int nwarps = (gridDim.x * BLOCK) >> 5;
+    const uint64_t pol = evict_first_policy();
+
+    for (int64_t base = (int64_t)warp * RPW; base < nrows; base += (int64_t)nwarps * RPW) {
+        const int64_t row = base + grp;
+        int s = 0, e = 0;
+        if (row < nrows) {
+            s = __ldg(rp + row);
+            e = __ldg(rp + row + 1);
+        }
+        double acc = 0.0;
+        const int g_end = (e + 3) >> 2;
+        int g = (s >> 2) + sub;
+        // two groups per iteration: 6 independent 16-B loads in flight per lane
+        for (; g + TPR < g_end; g += 2 * TPR) {
+            const int k0 = g << 2, k1 = (g + TPR) << 2;
+            const int4 c0 = ld_stream_i4(col + k0, pol);
+            const double2 a0 = ld_stream_d2(val + k0, pol);
+            const double2 b0 = ld_stream_d2(val + k0 + 2, pol);
+            const int4 c1 = ld_stream_i4(col + k1, pol);
+            const double2 a1 = ld_stream_d2(val + k1, pol);
+            const double2 b1 = ld_stream_d2(val + k1 + 2, pol);
+            // group g is not the row's last group: only its head can precede s
+            if (k0 + 0 >= s) acc = fma(a0.x, ld_x(x, c0.x), acc);
+            if (k0 + 1 >= s) acc = fma(a0.y, ld_x(x, c0.y), acc);
+            if (k0 + 2 >= s) acc = fma(b0.x, ld_x(x, c0.z), acc);
+            if (k0 + 3 >= s) acc = fma(b0.y, ld_x(x, c0.w), acc);
+            // group g+TPR starts after s: only its tail can pass e
+            if (k1 + 0 < e) acc = fma(a1.x, ld_x(x, c1.x), acc);
+            if (k1 + 1 < e) acc = fma(a1.y, ld_x(x, c1.y), acc);
+            if (k1 + 2 < e) acc = fma(b1.x, ld_x(x, c1.z), acc);
+            if (k1 + 3 < e) acc = fma(b1.y, ld_x(x, c1.w), acc);
+        }
+        if (g < g_end) {
+            const int k0 = g << 2;
+            const int4 c0 = ld_stream_i4(col + k0, pol);
+            const double2 a0 = ld_stream_d2(val + k0, pol);
+            const double2 b0 = ld_stream_d2(val + k0 + 2, pol);
+            if (k0 + 0 >= s && k0 + 0 < e) acc = fma(a0.x, ld_x(x, c0.x), acc);
+            if (k0 + 1 >= s && k0 + 1 < e) acc = fma(a0.y, ld_x(x, c0.y), acc);
+            if (k0 + 2 >= s && k0 + 2 < e) acc = fma(b0.x, ld_x(x, c0.z), acc);
+            if (k0 + 3 >= s && k0 + 3 < e) acc = fma(b0.y, ld_x(x, c0.w), acc);
+        }
+#pragma unroll
+        for (int off = TPR / 2; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (sub == 0 && row < nrows) y[row] = acc;
+    }
+}
+
+// =====================================================================
+// Variant 2: SELL-C-σ, C = 32. Chunk c holds the 32 (sorted) rows
+// [32c, 32c+32): slot j of lane l is at chunk_ptr[c] + 32*j + l, so a warp
+// reads 256 contiguous bytes of values and 128 of columns per slot. Each
+// lane masks slots beyond its own row length (no padding arithmetic, so
+// Inf/NaN in x behave exactly as in the CSR definition). perm maps sorted
+// position -> original row (NULL when σ = 1).
+// =====================================================================
+template <int BLOCK>
+__global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
+                                                     const int* __restrict__ chunk_len,
+                                                     const int* __restrict__ rowlen,
+                                                     const int* __restrict__ perm,
+                                                     const int* __restrict__ col,
+                                                     const double* __restrict__ val,
+                                                     const double* __restrict__ x,
+                                                     double* __restrict__ y) {
+    const int lane = threadIdx.x & 31;
+    const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
+    const int nwarps = (gridDim.x * BLOCK) >> 5;
+    const uint64_t pol = evict_first_policy();
+    for (int c = warp; c < nchunks; c += nwarps) {
+        const int r = c * 32 + lane;
+        const int len = r < nrows ? __ldg(rowlen + r) : 0;
+        const int clen = __ldg(chunk_len + c);
+        const int64_t base = __ldg(chunk_ptr + c) + lane;
+        double acc = 0.0;
+        int j = 0;
+        for (; j + 4 <= clen; j += 4) {
+            double v[4];
+            int ci[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                v[u] = 0.0; ci[u] = 0;
+                if (j + u < len) {
+                    v[u] = ld_stream_d(val + base + (int64_t)(j + u) * 32, pol);
+                    ci[u] = ld_stream_i(col + base + (int64_t)(j + u) * 32, pol);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+                if (j + u < len) acc = fma(v[u], ld_x(x, ci[u]), acc);
+        }
+        for (; j < clen; ++j)
+            if (j < len) acc = fma(ld_stream_d(val + base + (int64_t)j * 32, pol), ld_x(x, ld_stream_i(col + base + (int64_t)j * 32, pol)), acc);
+        if (r < nrows) y[perm ? __ldg(perm + r) : r] = acc;
+    }
+}
+
+// =====================================================================
+// Variant 1: merge-path CSR (balanced over rows + nonzeros).
+// The merge of the row-end list (rp[1..nrows]) with the nonzero indices is
+// cut into tiles of TILE = BLOCK*IPT items; tile start coordinates are
+// found once at plan time (merge_tile_search). Per tile: stage the tile's
+// row ends and the products val*x[col] in shared memory with coalesced
+// loads, then each thread consumes IPT merge items sequentially. Rows that
+// cross thread boundaries are joined with a deterministic block-wide
+// segmented scan; rows that cross tile boundaries leave a carry that
+// merge_fixup_kernel adds afterwards, in tile order (no fp atomics).
+// =====================================================================
+struct SegPair {
+    double v;
+    int f;  // 1 = a row ended inside this segment (resets the running sum)
+};
+__device__ __forceinline__ SegPair seg_combine(SegPair a, SegPair b) {
+    // a precedes b
+    SegPair r;
+    r.f = a.f | b.f;
+    r.v = b.f ? b.v : a.v + b.v;
+    return r;
+}
+
+template <int BLOCK, int IPT>
+__global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int* __restrict__ rp,
+                                                          const int* __restrict__ col,
+                                                          const double* __restrict__ val,
+                                                          const double* __restrict__ x,
+                                                          double* __restrict__ y,
+                                                          const int2* __restrict__ tile_coord,
+                                                          int* __restrict__ carry_row,
+                                                          double* __restrict__ carry_val) {
+    constexpr int TILE = BLOCK * IPT;
+    constexpr int NW = BLOCK / 32;
+    __shared__ int s_row_end[TILE];
+    __shared__ double s_prod[TILE];
+    __shared__ SegPair s_warp[NW];
+
+    const int tid = threadIdx.x;
+    const int tile = blockIdx.x;
+    const int2 c0 = __ldg(tile_coord + tile);
+    const int2 c1 = __ldg(tile_coord + tile + 1);
+    const int nr = c1.x - c0.x;   // row ends in this tile
+    const int nz = c1.y - c0.y;   // nonzeros in this tile
+
+    const uint64_t pol = evict_first_policy();
+    for (int i = tid; i < nr; i += BLOCK) s_row_end[i] = __ldg(rp + c0.x + 1 + i);
+    for (int j = tid; j < nz; j += BLOCK) {
+        const int k = c0.y + j;
+        s_prod[j] = ld_stream_d(val + k, pol) * ld_x(x, ld_stream_i(col + k, pol));
+    }
+    __syncthreads();
+
+    // this thread's start on the tile-local merge path
+    const int total = nr + nz;
+    const int d = min(tid * IPT, total);
+    int lo = max(0, d - nz), hi = min(d, nr);
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (s_row_end[mid] <= c0.y + d - mid - 1) lo = mid + 1;
+        else hi = mid;
+    }
+    int ri = lo, ki = d - lo;
+    const int dend = min(d + IPT, total);
+
+    double acc = 0.0, head_val = 0.0;
+    int head_row = -1;
+#pragma unroll
+    for (int it = 0; it < IPT; ++it) {
+        if (d + it < dend) {
+            const int re = ri < nr ? s_row_end[ri] : 0x7fffffff;
+            if (c0.y + ki < re) {                   // consume a nonzero
+                acc += s_prod[ki];
+                ++ki;
+            } else {                                // row ri ends here
+                if (head_row < 0) { head_row = ri; head_val = acc; }
+                else y[c0.x + ri] = acc;
+                acc = 0.0;
+                ++ri;
+            }
+        }
+    }
+
+    // block-wide inclusive segmented scan of (acc, ended-a-row)
+    SegPair me{acc, head_row >= 0 ? 1 : 0};
+    SegPair inc = me;
+    const int lane = tid & 31, wid = tid >> 5;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        SegPair o;
+        o.v = __shfl_up_sync(0xffffffffu, inc.v, off);
+        o.f = __shfl_up_sync(0xffffffffu, inc.f, off);
+        if (lane >= off) inc = seg_combine(o, inc);
+    }
+    if (lane == 31) s_warp[wid] = inc;
+    __syncthreads();
+    SegPair wpre{0.0, 0};
+    for (int w = 0; w < wid; ++w) wpre = w == 0 ? s_warp[0] : seg_combine(wpre, s_warp[w]);
+    // exclusive prefix for this thread = (warp prefix) ⊕ (inclusive of lane-1)
+    SegPair prev;
+    prev.v = __shfl_up_sync(0xffffffffu, inc.v, 1);
+    prev.f = __shfl_up_sync(0xffffffffu, inc.f, 1);
+    SegPair excl;
+    if (lane == 0) excl = wpre;
+    else excl = (wid == 0) ? prev : seg_combine(wpre, prev);
+    if (wid == 0 && lane == 0) excl = SegPair{0.0, 0};
+
+    if (head_row >= 0) y[c0.x + head_row] = excl.v + head_val;
+
+    if (tid == BLOCK - 1) {
+        const SegPair all = (wid == 0) ? inc : seg_combine(wpre, inc);
+        carry_row[tile] = c1.x;            // the row left open at the end of the tile
+        carry_val[tile] = all.v;
+    }
+}
+
+// Per tile t: if t is the first tile carrying into its row, add the carries
+// of t, t+1, ... (same row) to y[row] in tile order.
+__global__ void merge_fixup_kernel(int ntiles, int nrows, const int* __restrict__ carry_row,
+                                   const double* __restrict__ carry_val, double* __restrict__ y) {
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= ntiles) return;
+    const int row = carry_row[t];
+    if (row >= nrows) return;
+    if (t > 0 && carry_row[t - 1] == row) return;
+    double s = carry_val[t];
+    for (int u = t + 1; u < ntiles && carry_row[u] == row; ++u) s += carry_val[u];
+    y[row] = s + y[row];
+}
+
+// Plan time: tile start coordinates on the global merge path.
+__global__ void merge_tile_search_kernel(int nrows, int64_t nnz, const int* __restrict__ rp, int tile_items,
+                                         int ntiles, int2* __restrict__ tile_coord) {
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t > ntiles) return;
+    const int base = rp[0];
+    const int64_t total = (int64_t)nrows + nnz;
+    const int64_t d = min((int64_t)t * tile_items, total);
+    int64_t lo = max((int64_t)0, d - nnz), hi = min(d, (int64_t)nrows);
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if ((int64_t)rp[mid + 1] - base <= d - mid - 1) lo = mid + 1;
+        else hi = mid;
+    }
+    tile_coord[t] = make_int2((int)lo, (int)(base + (d - lo)));
+}
+
+// =====================================================================
+// plan-time helpers
+// =====================================================================
+// validation + context statistics over the caller's int64 row pointer
+struct RowStats {
+    unsigned long long sum_len2_lo;   // Σ len^2 (wraps only beyond 2^64)
+    unsigned long long max_len;
+    unsigned long long empty;
+    int bad;
+};
+
+__global__ void rowptr_check_narrow_kernel(int64_t nrows, const int64_t* __restrict__ rp64, int64_t first, int pad,
+                                           int* __restrict__ rp32, RowStats* st) {
+    unsigned long long s2 = 0, mx = 0, em = 0;
+    int bad = 0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= nrows; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t v = rp64[i];
+        rp32[i] = (int)(v - first + pad);
+        if (i < nrows) {
+            const int64_t len = rp64[i + 1] - v;
+            if (len < 0) bad = 1;
+            else {
+                s2 += (unsigned long long)len * (unsigned long long)len;
+                mx = max(mx, (unsigned long long)len);
+                em += (len == 0);
+            }
+        }
+    }
+    // warp reduce then one atomic per warp
+    for (int off = 16; off > 0; off >>= 1) {
+        s2 += __shfl_xor_sync(0xffffffffu, s2, off);
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+        em += __shfl_xor_sync(0xffffffffu, em, off);
+        bad |= __shfl_xor_sync(0xffffffffu, bad, off);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(&st->sum_len2_lo, s2);
+        atomicMax(&st->max_len, mx);
+        atomicAdd(&st->empty, em);
+        if (bad) atomicOr(&st->bad, 1);
+    }
+}
+
+__global__ void col_check_kernel(int64_t n, const int* __restrict__ col, int64_t ncols, int* bad) {
+    int b = 0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int c = col[i];
+        b |= (c < 0 || (int64_t)c >= ncols);
+    }
+    b = __any_sync(0xffffffffu, b);
+    if (b && (threadIdx.x & 31) == 0) atomicOr(bad, 1);
+}
+
+// SELL conversion -----------------------------------------------------
+// key for the σ-window sort: (window, descending length, row) packed in 64 bits
+__global__ void sell_keys_kernel(int nrows, const int* __restrict__ rp, int sigma, int maxlen,
+                                 unsigned long long* __restrict__ keys, int* __restrict__ rows) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nrows) return;
+    const int len = rp[i + 1] - rp[i];
+    const unsigned long long win = (unsigned long long)(i / sigma);
+    keys[i] = (win << 32) | (unsigned long long)(maxlen - len);
+    rows[i] = i;
+}
+
+// sorted position r -> original row perm[r]; lengths + per-chunk max
+__global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,
+                                    int* __restrict__ rowlen, int* __restrict__ chunk_len) {
+    const int r = blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = threadIdx.x & 31;
+    int len = 0;
+    if (r < nrows) {
+        const int o = perm ? perm[r] : r;
+        len = rp[o + 1] - rp[o];
+        rowlen[r] = len;
+    }
+    int m = len;
+    for (int off = 16; off > 0; off >>= 1) m = max(m, __shfl_xor_sync(0xffffffffu, m, off));
+    if (lane == 0 && r < nrows) chunk_len[r >> 5] = m;
+}
+
+__global__ void sell_fill_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,
+                                 const int* __restrict__ src_col, const double* __restrict__ src_val,
+                                 const int64_t* __restrict__ chunk_ptr, int* __restrict__ col,
+                                 double* __restrict__ val) {
+    const int r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= nrows) return;
+    const int o = perm ? perm[r] : r;
+    const int s = rp[o], e = rp[o + 1];
+    const int64_t base = chunk_ptr[r >> 5] + (r & 31);
+    for (int k = s; k < e; ++k) {
+        col[base + (int64_t)(k - s) * 32] = src_col[k];
+        val[base + (int64_t)(k - s) * 32] = src_val[k];
+    }
+}
+
+// halo pack / unpack --------------------------------------------------
+__global__ void gather_kernel(int64_t n, const int* __restrict__ idx, const double* __restrict__ src,
+                              double* __restrict__ dst) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[i] = src[idx[i]];
+}
+__global__ void scatter_kernel(int64_t n, const int* __restrict__ idx, const double* __restrict__ src,
+                               double* __restrict__ dst) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[idx[i]] = src[i];
+}
+
+}  // namespace k
+}  // namespace pepp

@@ -1,0 +1,52 @@
+// pepp_internal.h — shared declarations inside libpepp_spmv.so (not installed).
+#pragma once
+
+#include "pepp_spmv.h"
+
+#include <cstdint>
+#include <vector>
+
+#define PEPP_API __attribute__((visibility("default")))
+
+namespace pepp {
+
+struct Welford {
+    int64_t count = 0;
+    double mean = 0.0;
+    double m2 = 0.0;
+    void add(double v);
+};
+
+pepp_history* history_new();
+void history_free(pepp_history* h);
+void history_add(pepp_history* h, uint64_t key, int32_t cand, double us);
+const Welford* history_get(const pepp_history* h, uint64_t key, int32_t cand);
+int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible,
+                     int32_t min_samples, int32_t* calibrating, double* predicted_us);
+uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts);
+void halo_ghost_list(const int32_t* col, int64_t nnz, int64_t lo, int64_t hi, std::vector<int32_t>& out);
+
+// ---- NCCL, loaded on demand with dlopen (nccl_dl.cpp) ----
+// Only the handful of entry points the exchange needs; types mirror nccl.h
+// (NCCL 2.x ABI). No link-time dependency, so the library loads (and its
+// host-only utilities run) on machines without NCCL or a GPU.
+typedef struct ncclComm_opaque* ncclComm_t;
+typedef struct { char internal[128]; } ncclUniqueId;
+enum { NCCL_INT32 = 2, NCCL_INT64 = 4, NCCL_FLOAT64 = 8 };
+enum { NCCL_OP_MAX = 2 };
+struct Nccl {
+    int (*GetUniqueId)(ncclUniqueId*);
+    int (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int);
+    int (*CommDestroy)(ncclComm_t);
+    int (*CommGetAsyncError)(ncclComm_t, int*);
+    const char* (*GetErrorString)(int);
+    int (*GroupStart)();
+    int (*GroupEnd)();
+    int (*Send)(const void*, size_t, int, int, ncclComm_t, void*);
+    int (*Recv)(void*, size_t, int, int, ncclComm_t, void*);
+    int (*Broadcast)(const void*, void*, size_t, int, int, ncclComm_t, void*);
+    int (*AllReduce)(const void*, void*, size_t, int, int, ncclComm_t, void*);
+};
+const Nccl* nccl_load();                   // nullptr if libnccl cannot be loaded
+
+}  // namespace pepp

@@ -1,0 +1,818 @@
+// plan.cu — pepp_spmv_plan / _select / _exec / _destroy (see include/pepp_spmv.h).
+//
+// Steps of the hot path:
+//   a1 context extraction     -> rowptr_check_narrow_kernel (+ host CV)     [plan]
+//   a2 partition              -> caller / pepp_partition_rows; ghosts here  [plan]
+//   a3 variant preparation    -> SELL conversion, merge tile search          [plan]
+//   a4 selection              -> pepp::history_pick over the candidates      [each call, host]
+//   a5 SpMV kernel            -> kernels.cuh                                 [each call, device]
+//   a6 exchange               -> NCCL allgatherv (grouped broadcasts) / halo [each call, P > 1]
+//   a7 history update         -> lazily harvested CUDA events -> Welford     [each call, host]
+#include "pepp_internal.h"
+#include "kernels.cuh"
+
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+namespace {
+
+using pepp::Nccl;
+using pepp::ncclComm_t;
+
+constexpr int kBlock = 256;
+constexpr int kMergeBlock = 256;
+constexpr int kMergeIPT = 7;
+constexpr int kMergeTile = kMergeBlock * kMergeIPT;
+constexpr int kTimingRing = 64;
+
+struct Candidate {
+    int32_t variant;
+    int32_t param;
+};
+
+struct TimingRec {
+    cudaEvent_t start = nullptr, stop = nullptr;
+    int32_t cand = -1;
+    bool pending = false;
+};
+
+struct PeerXfer {            // halo traffic with one peer
+    int32_t peer;
+    int64_t count;
+    int64_t contig_start;    // >= 0: the entries are y[contig_start, contig_start+count)
+    int* d_idx = nullptr;    // else: global indices into y (device)
+    double* d_buf = nullptr; // pack / unpack buffer
+};
+
+}  // namespace
+
+struct pepp_spmv_plan_s {
+    pepp_spmv_opts_t opts{};
+    int device = 0;
+    int sm_count = 148;
+    pepp_status_t sticky = PEPP_OK;
+
+    int64_t nrows = 0, ncols = 0, nnz = 0, first = 0, row_offset = 0, global_rows = 0;
+    int pad = 0;
+    std::vector<int64_t> row_bounds;
+    std::string history_path;
+
+    // device CSR
+    int* d_rp = nullptr;
+    int* d_col = nullptr;
+    double* d_val = nullptr;
+    int64_t dev_bytes = 0;
+
+    // SELL-C-σ
+    int sell_sigma = 0;
+    int nchunks = 0;
+    int64_t sell_slots = 0;
+    int64_t* d_chunk_ptr = nullptr;
+    int* d_chunk_len = nullptr;
+    int* d_rowlen = nullptr;
+    int* d_perm = nullptr;
+    int* d_scol = nullptr;
+    double* d_sval = nullptr;
+
+    // merge path
+    int ntiles = 0;
+    int2* d_tile = nullptr;
+    int* d_carry_row = nullptr;
+    double* d_carry_val = nullptr;
+
+    // occupancy-derived grids
+    int grid_csr[6] = {0};   // per log2(TPR)
+    int grid_sell = 0;
+
+    // selection
+    pepp_plan_info_t info{};
+    std::vector<Candidate> cands;
+    std::vector<uint8_t> eligible;
+    pepp_history* hist = nullptr;
+    uint64_t key = 0;
+    int64_t ncalls = 0;
+
+    // timing ring
+    TimingRec ring[kTimingRing];
+    int ring_head = 0;   // oldest pending
+    int ring_count = 0;
+
+    // multi-GPU
+    const Nccl* nccl = nullptr;
+    ncclComm_t comm = nullptr;
+    bool own_comm = false;
+    int32_t exchange = PEPP_X_NONE;
+    std::vector<PeerXfer> recv_x, send_x;
+
+    // plan-owned x / y for pepp_spmv_exec_host (allocated on first use)
+    double* d_hx = nullptr;
+    double* d_hy = nullptr;
+};
+
+namespace {
+
+#define PEPP_CUDA_TRY(expr)                                   \
+    do {                                                      \
+        cudaError_t _e = (expr);                              \
+        if (_e != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; } \
+    } while (0)
+
+template <typename T>
+pepp_status_t dalloc(pepp_spmv_plan_t* p, T** ptr, int64_t n) {
+    *ptr = nullptr;
+    if (n <= 0) n = 1;
+    cudaError_t e = cudaMalloc((void**)ptr, sizeof(T) * (size_t)n);
+    if (e != cudaSuccess) { (void)cudaGetLastError(); *ptr = nullptr; return e == cudaErrorMemoryAllocation ? PEPP_E_NOMEM : PEPP_E_CUDA; }
+    p->dev_bytes += (int64_t)sizeof(T) * n;
+    return PEPP_OK;
+}
+
+void free_plan(pepp_spmv_plan_t* p) {
+    if (!p) return;
+    if (p->device >= 0) cudaSetDevice(p->device);
+    void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
+                    p->d_scol, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy};
+    for (void* b : bufs) if (b) cudaFree(b);
+    for (auto* v : {&p->recv_x, &p->send_x})
+        for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
+    for (auto& r : p->ring) { if (r.start) cudaEventDestroy(r.start); if (r.stop) cudaEventDestroy(r.stop); }
+    if (p->comm && p->own_comm && p->nccl) p->nccl->CommDestroy(p->comm);
+    if (p->hist) pepp::history_free(p->hist);
+    delete p;
+}
+
+int grid_for(const void* fn, int block, int64_t work_items, int items_per_block, int sms) {
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, block, 0) != cudaSuccess || occ < 1) occ = 1;
+    (void)cudaGetLastError();
+    const int64_t need = (work_items + items_per_block - 1) / items_per_block;
+    const int64_t cap = (int64_t)sms * occ * 4;   // 4 resident waves, grid-stride beyond
+    return (int)std::max<int64_t>(1, std::min(need, cap));
+}
+
+// ---------------------------------------------------------------- SELL prep
+pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
+    const int n = (int)p->nrows;
+    p->nchunks = (n + 31) / 32;
+    if (n == 0) return PEPP_OK;
+    pepp_status_t s;
+    if ((s = dalloc(p, &p->d_chunk_len, p->nchunks))) return s;
+    if ((s = dalloc(p, &p->d_rowlen, n))) return s;
+    if ((s = dalloc(p, &p->d_chunk_ptr, (int64_t)p->nchunks + 1))) return s;
+    const int tb = 256, gb = (n + tb - 1) / tb;
+
+    auto fill_ratio = [&](const int* perm, double* fill) -> pepp_status_t {
+        pepp::k::sell_lengths_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, perm, p->d_rowlen, p->d_chunk_len);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        std::vector<int> cl(p->nchunks);
+        PEPP_CUDA_TRY(cudaMemcpyAsync(cl.data(), p->d_chunk_len, sizeof(int) * p->nchunks, cudaMemcpyDeviceToHost, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        int64_t slots = 0;
+        std::vector<int64_t> cp(p->nchunks + 1);
+        for (int c = 0; c < p->nchunks; ++c) { cp[c] = slots; slots += (int64_t)cl[c] * 32; }
+        cp[p->nchunks] = slots;
+        p->sell_slots = slots;
+        *fill = p->nnz ? (double)slots / (double)p->nnz : 1.0;
+        PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_chunk_ptr, cp.data(), sizeof(int64_t) * (p->nchunks + 1), cudaMemcpyHostToDevice, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        return PEPP_OK;
+    };
+
+    double fill = 1.0;
+    int sigma = p->opts.sell_sigma;
+    if (sigma <= 1) {
+        if ((s = fill_ratio(nullptr, &fill))) return s;
+        sigma = 1;
+        if (p->opts.sell_sigma == 0 && fill > 1.15) sigma = 4096;   // auto: sort when σ=1 pads > 15 %
+    }
+    if (sigma > 1) {
+        // stable radix sort of (window, maxlen - len) keys -> perm
+        unsigned long long *keys = nullptr, *keys_out = nullptr;
+        int* rows = nullptr;
+        void* tmp = nullptr;
+        size_t tmp_bytes = 0;
+        const int maxlen = (int)p->info.max_row;
+        PEPP_CUDA_TRY(cudaMalloc(&keys, sizeof(unsigned long long) * n));
+        PEPP_CUDA_TRY(cudaMalloc(&keys_out, sizeof(unsigned long long) * n));
+        PEPP_CUDA_TRY(cudaMalloc(&rows, sizeof(int) * n));
+        if ((s = dalloc(p, &p->d_perm, n))) return s;
+        pepp::k::sell_keys_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, sigma, maxlen, keys, rows);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        int end_bit = 32;
+        while ((1ull << (end_bit - 32)) <= (unsigned long long)((n - 1) / sigma) && end_bit < 64) ++end_bit;
+        cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, keys, keys_out, rows, p->d_perm, n, 0, end_bit, st);
+        PEPP_CUDA_TRY(cudaMalloc(&tmp, tmp_bytes));
+        PEPP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, keys, keys_out, rows, p->d_perm, n, 0, end_bit, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        cudaFree(tmp); cudaFree(keys); cudaFree(keys_out); cudaFree(rows);
+        if ((s = fill_ratio(p->d_perm, &fill))) return s;
+    }
+    p->sell_sigma = sigma;
+    if ((s = dalloc(p, &p->d_scol, p->sell_slots + 32))) return s;
+    if ((s = dalloc(p, &p->d_sval, p->sell_slots + 32))) return s;
+    // padding slots are never read (lanes mask by row length), but keep them defined
+    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_scol, 0, sizeof(int) * (p->sell_slots + 32), st));
+    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_sval, 0, sizeof(double) * (p->sell_slots + 32), st));
+    pepp::k::sell_fill_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, p->d_col, p->d_val, p->d_chunk_ptr,
+                                                   p->d_scol, p->d_sval);
+    PEPP_CUDA_TRY(cudaGetLastError());
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    p->info.sell_sigma = sigma;
+    p->info.sell_fill = fill;
+    return PEPP_OK;
+}
+
+// ---------------------------------------------------------------- merge prep
+pepp_status_t prepare_merge(pepp_spmv_plan_t* p, cudaStream_t st) {
+    const int64_t total = p->nrows + p->nnz;
+    p->ntiles = (int)((total + kMergeTile - 1) / kMergeTile);
+    pepp_status_t s;
+    if ((s = dalloc(p, &p->d_tile, (int64_t)p->ntiles + 1))) return s;
+    if ((s = dalloc(p, &p->d_carry_row, std::max(p->ntiles, 1)))) return s;
+    if ((s = dalloc(p, &p->d_carry_val, std::max(p->ntiles, 1)))) return s;
+    const int tb = 256;
+    pepp::k::merge_tile_search_kernel<<<(p->ntiles + 1 + tb - 1) / tb, tb, 0, st>>>(
+        (int)p->nrows, p->nnz, p->d_rp, kMergeTile, p->ntiles, p->d_tile);
+    PEPP_CUDA_TRY(cudaGetLastError());
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    return PEPP_OK;
+}
+
+// ---------------------------------------------------------------- launches
+template <int TPR>
+void launch_csr_vector(const pepp_spmv_plan_t* p, const double* x, double* y, cudaStream_t st, int grid) {
+    pepp::k::csr_vector_kernel<TPR, kBlock><<<grid, kBlock, 0, st>>>((int)p->nrows, p->d_rp, p->d_col, p->d_val, x, y);
+}
+
+pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const double* x, double* y, cudaStream_t st) {
+    if (p->nrows == 0) return PEPP_OK;
+    switch (c.variant) {
+    case PEPP_V_CSR_VECTOR:
+        switch (c.param) {
+        case 2: launch_csr_vector<2>(p, x, y, st, p->grid_csr[1]); break;
+        case 4: launch_csr_vector<4>(p, x, y, st, p->grid_csr[2]); break;
+        case 8: launch_csr_vector<8>(p, x, y, st, p->grid_csr[3]); break;
+        case 16: launch_csr_vector<16>(p, x, y, st, p->grid_csr[4]); break;
+        case 32: launch_csr_vector<32>(p, x, y, st, p->grid_csr[5]); break;
+        default: return PEPP_E_INVALID;
+        }
+        break;
+    case PEPP_V_MERGE_PATH:
+        if (p->ntiles > 0) {
+            pepp::k::merge_spmv_kernel<kMergeBlock, kMergeIPT><<<p->ntiles, kMergeBlock, 0, st>>>(
+                (int)p->nrows, p->d_rp, p->d_col, p->d_val, x, y, p->d_tile, p->d_carry_row, p->d_carry_val);
+            pepp::k::merge_fixup_kernel<<<(p->ntiles + 255) / 256, 256, 0, st>>>(p->ntiles, (int)p->nrows,
+                                                                                  p->d_carry_row, p->d_carry_val, y);
+        }
+        break;
+    case PEPP_V_SELL:
+        pepp::k::sell_kernel<kBlock><<<p->grid_sell, kBlock, 0, st>>>((int)p->nrows, p->nchunks, p->d_chunk_ptr,
+                                                                       p->d_chunk_len, p->d_rowlen, p->d_perm,
+                                                                       p->d_scol, p->d_sval, x, y);
+        break;
+    default:
+        return PEPP_E_INVALID;
+    }
+    return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
+}
+
+// ---------------------------------------------------------------- history
+void harvest(pepp_spmv_plan_t* p, bool block) {
+    while (p->ring_count > 0) {
+        TimingRec& r = p->ring[p->ring_head];
+        if (block) cudaEventSynchronize(r.stop);
+        cudaError_t q = cudaEventQuery(r.stop);
+        if (q == cudaErrorNotReady) { (void)cudaGetLastError(); break; }
+        float ms = 0.f;
+        if (q == cudaSuccess && cudaEventElapsedTime(&ms, r.start, r.stop) == cudaSuccess)
+            pepp::history_add(p->hist, p->key, r.cand, (double)ms * 1000.0);
+        (void)cudaGetLastError();
+        r.pending = false;
+        p->ring_head = (p->ring_head + 1) % kTimingRing;
+        --p->ring_count;
+    }
+}
+
+int heuristic_candidate(const pepp_spmv_plan_t* p) {
+    // use_history = 0: fixed rule from the context instance (mean, CV)
+    const double mean = p->info.mean_row, cv = p->info.cv_row;
+    auto find = [&](int v, int prm) {
+        for (size_t i = 0; i < p->cands.size(); ++i)
+            if (p->cands[i].variant == v && (prm < 0 || p->cands[i].param == prm) && p->eligible[i]) return (int)i;
+        return -1;
+    };
+    int c = -1;
+    if (cv > 1.0) c = find(PEPP_V_MERGE_PATH, -1);
+    if (c < 0 && mean <= 12.0 && cv <= 0.5) c = find(PEPP_V_SELL, -1);
+    if (c < 0) {
+        const int tpr = mean <= 6 ? 2 : mean <= 12 ? 4 : mean <= 24 ? 8 : mean <= 96 ? 16 : 32;
+        c = find(PEPP_V_CSR_VECTOR, tpr);
+    }
+    for (size_t i = 0; c < 0 && i < p->cands.size(); ++i) if (p->eligible[i]) c = (int)i;
+    return c;
+}
+
+void fill_choice(const pepp_spmv_plan_t* p, int cand, int calibrating, double pred, pepp_choice_t* out) {
+    out->variant = p->cands[cand].variant;
+    out->param = p->cands[cand].param;
+    out->nparts = p->opts.nranks;
+    out->exchange = p->exchange;
+    out->calibrating = calibrating;
+    out->candidate = cand;
+    out->predicted_us = pred;
+}
+
+pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out) {
+    harvest(p, false);
+    int calibrating = 0;
+    double pred = 0.0;
+    int cand;
+    if (p->opts.use_history) {
+        cand = pepp::history_pick(p->hist, p->key, (int32_t)p->cands.size(), p->eligible.data(),
+                                  std::max(1, p->opts.min_samples), &calibrating, &pred);
+    } else {
+        cand = heuristic_candidate(p);
+    }
+    if (cand < 0) return PEPP_E_INVALID;
+    fill_choice(p, cand, calibrating, pred, out);
+    return PEPP_OK;
+}
+
+// ---------------------------------------------------------------- NCCL
+pepp_status_t nccl_ok(const pepp_spmv_plan_t* p, int r) { (void)p; return r == 0 ? PEPP_OK : PEPP_E_NCCL; }
+
+pepp_status_t exchange_allgather(pepp_spmv_plan_t* p, double* y, cudaStream_t st) {
+    const Nccl* n = p->nccl;
+    if (nccl_ok(p, n->GroupStart())) return PEPP_E_NCCL;
+    for (int r = 0; r < p->opts.nranks; ++r) {
+        const int64_t b = p->row_bounds[r], cnt = p->row_bounds[r + 1] - b;
+        if (cnt == 0) continue;
+        if (n->Broadcast(y + b, y + b, (size_t)cnt, pepp::NCCL_FLOAT64, r, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
+    }
+    return nccl_ok(p, n->GroupEnd());
+}
+
+pepp_status_t exchange_halo(pepp_spmv_plan_t* p, double* y, cudaStream_t st) {
+    const Nccl* n = p->nccl;
+    for (auto& t : p->send_x)
+        if (t.contig_start < 0 && t.count > 0)
+            pepp::k::gather_kernel<<<(int)std::min<int64_t>(1024, (t.count + 255) / 256), 256, 0, st>>>(t.count, t.d_idx, y, t.d_buf);
+    if (n->GroupStart()) return PEPP_E_NCCL;
+    for (auto& t : p->send_x) {
+        if (!t.count) continue;
+        const double* src = t.contig_start >= 0 ? y + t.contig_start : t.d_buf;
+        if (n->Send(src, (size_t)t.count, pepp::NCCL_FLOAT64, t.peer, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
+    }
+    for (auto& t : p->recv_x) {
+        if (!t.count) continue;
+        double* dst = t.contig_start >= 0 ? y + t.contig_start : t.d_buf;
+        if (n->Recv(dst, (size_t)t.count, pepp::NCCL_FLOAT64, t.peer, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
+    }
+    if (n->GroupEnd()) return PEPP_E_NCCL;
+    for (auto& t : p->recv_x)
+        if (t.contig_start < 0 && t.count > 0)
+            pepp::k::scatter_kernel<<<(int)std::min<int64_t>(1024, (t.count + 255) / 256), 256, 0, st>>>(t.count, t.d_idx, t.d_buf, y);
+    return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
+}
+
+// plan-time halo setup: ghosts (what I receive) from my columns; what I send
+// is learnt from the peers with one NCCL exchange of counts and indices.
+pepp_status_t setup_halo(pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts, cudaStream_t st) {
+    const int P = p->opts.nranks, me = p->opts.rank;
+    std::vector<int64_t> rcount(P, 0), scount(P, 0);
+    std::vector<std::vector<int32_t>> rlist(P);
+    for (int32_t c : ghosts) {
+        int q = (int)(std::upper_bound(p->row_bounds.begin(), p->row_bounds.end(), (int64_t)c) - p->row_bounds.begin()) - 1;
+        rlist[q].push_back(c);
+    }
+    for (int q = 0; q < P; ++q) rcount[q] = (int64_t)rlist[q].size();
+    // exchange counts: send rcount[q] to q, receive scount[q] from q
+    int64_t *d_rc = nullptr, *d_sc = nullptr;
+    PEPP_CUDA_TRY(cudaMalloc(&d_rc, sizeof(int64_t) * P));
+    PEPP_CUDA_TRY(cudaMalloc(&d_sc, sizeof(int64_t) * P));
+    PEPP_CUDA_TRY(cudaMemcpy(d_rc, rcount.data(), sizeof(int64_t) * P, cudaMemcpyHostToDevice));
+    PEPP_CUDA_TRY(cudaMemset(d_sc, 0, sizeof(int64_t) * P));
+    const Nccl* n = p->nccl;
+    n->GroupStart();
+    for (int q = 0; q < P; ++q) {
+        if (q == me) continue;
+        n->Send(d_rc + q, 1, pepp::NCCL_INT64, q, p->comm, st);
+        n->Recv(d_sc + q, 1, pepp::NCCL_INT64, q, p->comm, st);
+    }
+    if (n->GroupEnd()) return PEPP_E_NCCL;
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    PEPP_CUDA_TRY(cudaMemcpy(scount.data(), d_sc, sizeof(int64_t) * P, cudaMemcpyDeviceToHost));
+    cudaFree(d_rc); cudaFree(d_sc);
+    scount[me] = 0;
+    // exchange index lists
+    std::vector<int*> d_r(P, nullptr), d_s(P, nullptr);
+    for (int q = 0; q < P; ++q) {
+        if (rcount[q]) {
+            PEPP_CUDA_TRY(cudaMalloc(&d_r[q], sizeof(int) * rcount[q]));
+            PEPP_CUDA_TRY(cudaMemcpy(d_r[q], rlist[q].data(), sizeof(int) * rcount[q], cudaMemcpyHostToDevice));
+        }
+        if (scount[q]) PEPP_CUDA_TRY(cudaMalloc(&d_s[q], sizeof(int) * scount[q]));
+    }
+    n->GroupStart();
+    for (int q = 0; q < P; ++q) {
+        if (rcount[q]) n->Send(d_r[q], (size_t)rcount[q], pepp::NCCL_INT32, q, p->comm, st);
+        if (scount[q]) n->Recv(d_s[q], (size_t)scount[q], pepp::NCCL_INT32, q, p->comm, st);
+    }
+    if (n->GroupEnd()) return PEPP_E_NCCL;
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    auto make = [&](int q, std::vector<int32_t>& lst, int* d_list, std::vector<PeerXfer>& out) -> pepp_status_t {
+        PeerXfer t;
+        t.peer = q;
+        t.count = (int64_t)lst.size();
+        const bool contig = !lst.empty() && (int64_t)lst.back() - lst.front() + 1 == t.count;
+        t.contig_start = contig ? lst.front() : -1;
+        if (!contig && t.count) {
+            t.d_idx = d_list;
+            d_list = nullptr;
+            PEPP_CUDA_TRY(cudaMalloc(&t.d_buf, sizeof(double) * t.count));
+        }
+        if (d_list) cudaFree(d_list);
+        out.push_back(t);
+        return PEPP_OK;
+    };
+    for (int q = 0; q < P; ++q) {
+        if (rcount[q]) { pepp_status_t s = make(q, rlist[q], d_r[q], p->recv_x); if (s) return s; }
+        if (scount[q]) {
+            std::vector<int32_t> sl(scount[q]);
+            PEPP_CUDA_TRY(cudaMemcpy(sl.data(), d_s[q], sizeof(int) * scount[q], cudaMemcpyDeviceToHost));
+            pepp_status_t s = make(q, sl, d_s[q], p->send_x);
+            if (s) return s;
+        }
+    }
+    int64_t tr = 0, ts = 0;
+    for (auto& t : p->recv_x) tr += t.count;
+    for (auto& t : p->send_x) ts += t.count;
+    p->info.halo_recv = tr;
+    p->info.halo_send = ts;
+    return PEPP_OK;
+}
+
+pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spmv_plan_t* p) {
+    // ---- argument checks (host, O(1)) ----
+    if (A->nrows < 0 || A->ncols < 0 || A->nnz < 0 || !A->row_ptr) return PEPP_E_INVALID;
+    if (A->nnz > 0 && (!A->col_idx || !A->values)) return PEPP_E_INVALID;
+    if (o->nranks < 1 || o->rank < 0 || o->rank >= o->nranks) return PEPP_E_INVALID;
+    if (o->nranks > 1 && !o->row_bounds) return PEPP_E_INVALID;
+    if (A->nnz + 8 >= (int64_t)INT32_MAX || A->ncols >= (int64_t)INT32_MAX || A->nrows >= (int64_t)INT32_MAX)
+        return PEPP_E_UNSUPPORTED;
+    if (o->variant_mask != 0 && (o->variant_mask & ((1u << PEPP_V_COUNT) - 1)) == 0) return PEPP_E_INVALID;
+
+    p->opts = *o;
+    p->nrows = A->nrows; p->ncols = A->ncols; p->nnz = A->nnz; p->first = A->first;
+    p->pad = (int)(((A->first % 4) + 4) % 4);
+    if (o->nranks > 1) {
+        p->row_bounds.assign(o->row_bounds, o->row_bounds + o->nranks + 1);
+        for (int r = 0; r < o->nranks; ++r) if (p->row_bounds[r + 1] < p->row_bounds[r]) return PEPP_E_INVALID;
+        if (p->row_bounds[o->rank + 1] - p->row_bounds[o->rank] != A->nrows) return PEPP_E_INVALID;
+        p->row_offset = p->row_bounds[o->rank];
+        p->global_rows = p->row_bounds[o->nranks];
+    } else {
+        p->row_bounds = {0, A->nrows};
+        p->row_offset = 0;
+        p->global_rows = A->nrows;
+    }
+    if (o->history_path) p->history_path = o->history_path;
+    p->opts.history_path = nullptr;
+    p->opts.row_bounds = nullptr;
+
+    // ---- device ----
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    if (o->device >= 0) { if (o->device >= ndev) return PEPP_E_INVALID; p->device = o->device; }
+    else PEPP_CUDA_TRY(cudaGetDevice(&p->device));
+    PEPP_CUDA_TRY(cudaSetDevice(p->device));
+    PEPP_CUDA_TRY(cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device));
+    cudaStream_t st = nullptr;
+    PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+    struct StreamGuard { cudaStream_t s; ~StreamGuard() { cudaStreamDestroy(s); } } guard{st};
+
+    // row_ptr[0] == first (A1) is checked on the host (one value)
+    int64_t rp0 = 0, rpn = 0;
+    if (A->on_device) {
+        PEPP_CUDA_TRY(cudaMemcpy(&rp0, A->row_ptr, sizeof(int64_t), cudaMemcpyDeviceToHost));
+        PEPP_CUDA_TRY(cudaMemcpy(&rpn, A->row_ptr + A->nrows, sizeof(int64_t), cudaMemcpyDeviceToHost));
+    } else {
+        rp0 = A->row_ptr[0];
+        rpn = A->row_ptr[A->nrows];
+    }
+    if (rp0 != A->first || rpn - A->first != A->nnz) return PEPP_E_INVALID;
+
+    // ---- a1: copy + narrow row_ptr, validate, context statistics ----
+    pepp_status_t s;
+    const int64_t nstore = p->pad + A->nnz + 8;   // + trailing zeros for aligned 4-groups
+    if ((s = dalloc(p, &p->d_rp, A->nrows + 1))) return s;
+    if ((s = dalloc(p, &p->d_col, nstore))) return s;
+    if ((s = dalloc(p, &p->d_val, nstore))) return s;
+    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_col, 0, sizeof(int) * nstore, st));
+    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_val, 0, sizeof(double) * nstore, st));
+    const cudaMemcpyKind kind = A->on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+    if (A->nnz) {
+        PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_col + p->pad, A->col_idx, sizeof(int) * A->nnz, kind, st));
+        PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_val + p->pad, A->values, sizeof(double) * A->nnz, kind, st));
+    }
+    int64_t* d_rp64 = nullptr;
+    pepp::k::RowStats* d_stats = nullptr;
+    PEPP_CUDA_TRY(cudaMalloc(&d_rp64, sizeof(int64_t) * (A->nrows + 1)));
+    PEPP_CUDA_TRY(cudaMalloc(&d_stats, sizeof(pepp::k::RowStats)));
+    PEPP_CUDA_TRY(cudaMemsetAsync(d_stats, 0, sizeof(pepp::k::RowStats), st));
+    PEPP_CUDA_TRY(cudaMemcpyAsync(d_rp64, A->row_ptr, sizeof(int64_t) * (A->nrows + 1), kind, st));
+    {
+        const int tb = 256;
+        const int gb = (int)std::min<int64_t>((A->nrows + 1 + tb - 1) / tb, (int64_t)p->sm_count * 8);
+        pepp::k::rowptr_check_narrow_kernel<<<gb, tb, 0, st>>>(A->nrows, d_rp64, A->first, p->pad, p->d_rp, d_stats);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        if (o->validate && A->nnz) {
+            const int gc = (int)std::min<int64_t>((A->nnz + tb - 1) / tb, (int64_t)p->sm_count * 8);
+            pepp::k::col_check_kernel<<<gc, tb, 0, st>>>(A->nnz, p->d_col + p->pad, A->ncols, &d_stats->bad);
+            PEPP_CUDA_TRY(cudaGetLastError());
+        }
+    }
+    pepp::k::RowStats hs{};
+    PEPP_CUDA_TRY(cudaMemcpyAsync(&hs, d_stats, sizeof(hs), cudaMemcpyDeviceToHost, st));
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    std::vector<int32_t> ghosts;
+    if (o->nranks > 1) {
+        std::vector<int32_t> hcol(A->nnz);
+        if (A->nnz) PEPP_CUDA_TRY(cudaMemcpy(hcol.data(), p->d_col + p->pad, sizeof(int) * A->nnz, cudaMemcpyDeviceToHost));
+        pepp::halo_ghost_list(hcol.data(), A->nnz, p->row_offset, p->row_offset + A->nrows, ghosts);
+        if (!ghosts.empty() && (ghosts.front() < 0 || ghosts.back() >= p->global_rows)) hs.bad = 1;
+    }
+    cudaFree(d_rp64);
+    cudaFree(d_stats);
+    if (hs.bad) return PEPP_E_INVALID;
+
+    pepp_plan_info_t& I = p->info;
+    I.nrows = A->nrows; I.ncols = A->ncols; I.nnz = A->nnz;
+    I.mean_row = A->nrows ? (double)A->nnz / (double)A->nrows : 0.0;
+    {
+        const double m = I.mean_row;
+        const double ex2 = A->nrows ? (double)hs.sum_len2_lo / (double)A->nrows : 0.0;
+        const double var = std::max(0.0, ex2 - m * m);
+        I.cv_row = m > 0 ? std::sqrt(var) / m : 0.0;
+    }
+    I.max_row = (int64_t)hs.max_len;
+    I.empty_rows = (int64_t)hs.empty;
+    I.nranks = o->nranks; I.rank = o->rank; I.row_offset = p->row_offset;
+    I.algorithmic_bytes = A->nnz * 12 + (A->nrows + 1) * 4 + A->ncols * 8 + A->nrows * 8;
+
+    // ---- a3: candidates + variant preparation ----
+    const uint32_t mask = o->variant_mask ? o->variant_mask : 0xffffffffu;
+    if (mask & (1u << PEPP_V_CSR_VECTOR))
+        for (int tpr : {2, 4, 8, 16, 32}) p->cands.push_back({PEPP_V_CSR_VECTOR, tpr});
+    if (mask & (1u << PEPP_V_MERGE_PATH)) p->cands.push_back({PEPP_V_MERGE_PATH, kMergeIPT});
+    if (mask & (1u << PEPP_V_SELL)) {
+        if ((s = prepare_sell(p, st))) return s;
+        p->cands.push_back({PEPP_V_SELL, p->sell_sigma});
+    }
+    if (mask & (1u << PEPP_V_MERGE_PATH)) { if ((s = prepare_merge(p, st))) return s; }
+    p->eligible.assign(p->cands.size(), 1);
+    I.ncandidates = (int32_t)p->cands.size();
+
+    p->grid_csr[1] = grid_for((const void*)pepp::k::csr_vector_kernel<2, kBlock>, kBlock, A->nrows, kBlock / 2, p->sm_count);
+    p->grid_csr[2] = grid_for((const void*)pepp::k::csr_vector_kernel<4, kBlock>, kBlock, A->nrows, kBlock / 4, p->sm_count);
+    p->grid_csr[3] = grid_for((const void*)pepp::k::csr_vector_kernel<8, kBlock>, kBlock, A->nrows, kBlock / 8, p->sm_count);
+    p->grid_csr[4] = grid_for((const void*)pepp::k::csr_vector_kernel<16, kBlock>, kBlock, A->nrows, kBlock / 16, p->sm_count);
+    p->grid_csr[5] = grid_for((const void*)pepp::k::csr_vector_kernel<32, kBlock>, kBlock, A->nrows, kBlock / 32, p->sm_count);
+    p->grid_sell = grid_for((const void*)pepp::k::sell_kernel<kBlock>, kBlock, p->nchunks, kBlock / 32, p->sm_count);
+
+    // ---- history ----
+    p->key = pepp::context_key(A->nrows, A->ncols, A->nnz, I.cv_row, o->nranks);
+    I.key = p->key;
+    p->hist = pepp::history_new();
+    if (!p->hist) return PEPP_E_NOMEM;
+    if (!p->history_path.empty()) (void)pepp_history_load(p->hist, p->history_path.c_str());
+    for (auto& r : p->ring) {
+        PEPP_CUDA_TRY(cudaEventCreate(&r.start));
+        PEPP_CUDA_TRY(cudaEventCreate(&r.stop));
+    }
+
+    // ---- a2: exchange setup (partitioned calls) ----
+    p->exchange = PEPP_X_NONE;
+    if (o->nranks > 1) {
+        p->nccl = pepp::nccl_load();
+        if (!p->nccl) return PEPP_E_NCCL;
+        if (o->nccl_comm) {
+            p->comm = (ncclComm_t)o->nccl_comm;
+        } else {
+            if (!o->nccl_unique_id) return PEPP_E_INVALID;
+            pepp::ncclUniqueId id;
+            std::memcpy(&id, o->nccl_unique_id, sizeof(id));
+            if (p->nccl->CommInitRank(&p->comm, o->nranks, id, o->rank)) return PEPP_E_NCCL;
+            p->own_comm = true;
+        }
+        if ((s = setup_halo(p, ghosts, st))) return s;
+        int ex = o->exchange;
+        if (ex == PEPP_X_AUTO) {
+            // halo when every rank's ghosts are a small part of x;
+            // the decision must be identical on all ranks: max-reduce the counts.
+            int64_t *d_g = nullptr;
+            int64_t g = (int64_t)ghosts.size(), gmax = 0;
+            PEPP_CUDA_TRY(cudaMalloc(&d_g, sizeof(int64_t)));
+            PEPP_CUDA_TRY(cudaMemcpy(d_g, &g, sizeof(int64_t), cudaMemcpyHostToDevice));
+            if (p->nccl->AllReduce(d_g, d_g, 1, pepp::NCCL_INT64, pepp::NCCL_OP_MAX, p->comm, st)) { cudaFree(d_g); return PEPP_E_NCCL; }
+            PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+            PEPP_CUDA_TRY(cudaMemcpy(&gmax, d_g, sizeof(int64_t), cudaMemcpyDeviceToHost));
+            cudaFree(d_g);
+            ex = ((double)gmax < 0.25 * (double)p->global_rows) ? PEPP_X_HALO : PEPP_X_ALLGATHER;
+        }
+        p->exchange = ex;
+    }
+    I.exchange = p->exchange;
+    I.device_bytes = p->dev_bytes;
+    return PEPP_OK;
+}
+
+}  // namespace
+
+// ================================================================= C-ABI
+extern "C" PEPP_API pepp_status_t pepp_spmv_plan(const pepp_csr_t* A, const pepp_spmv_opts_t* opts,
+                                                pepp_spmv_plan_t** out) {
+    if (!out) return PEPP_E_INVALID;
+    *out = nullptr;
+    if (!A) return PEPP_E_INVALID;
+    pepp_spmv_opts_t def;
+    pepp_spmv_opts_default(&def);
+    if (!opts) opts = &def;
+    pepp_spmv_plan_t* p = new (std::nothrow) pepp_spmv_plan_t();
+    if (!p) return PEPP_E_NOMEM;
+    p->device = -1;
+    pepp_status_t s;
+    try {
+        s = plan_impl(A, opts, p);
+    } catch (const std::bad_alloc&) {
+        s = PEPP_E_NOMEM;
+    } catch (...) {
+        s = PEPP_E_INVALID;
+    }
+    if (s != PEPP_OK) { free_plan(p); return s; }
+    *out = p;
+    return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_choice_t* out) {
+    if (!p || !out) return PEPP_E_INVALID;
+    if (p->sticky) return p->sticky;
+    return select_choice(p, out);
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const double* x, double* y, int flags,
+                                                void* stream, const pepp_choice_t* force, pepp_choice_t* used) {
+    if (!p) return PEPP_E_INVALID;
+    if (p->sticky) return p->sticky;
+    if (!x || !y) return PEPP_E_INVALID;
+    {   // x [0, ncols) and y [0, global_rows) must not overlap
+        const char *xb = (const char*)x, *xe = (const char*)(x + p->ncols);
+        const char *yb = (const char*)y, *ye = (const char*)(y + p->global_rows);
+        if (xb < ye && yb < xe) return PEPP_E_INVALID;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    int cur = -1;
+    if (cudaGetDevice(&cur) != cudaSuccess || cur != p->device) {
+        (void)cudaGetLastError();
+        if (cudaSetDevice(p->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    }
+    pepp_choice_t ch{};
+    if (force) {
+        int idx = -1;
+        for (size_t i = 0; i < p->cands.size(); ++i)
+            if (p->cands[i].variant == force->variant && (force->param <= 0 || p->cands[i].param == force->param)) { idx = (int)i; break; }
+        if (idx < 0) return PEPP_E_INVALID;
+        fill_choice(p, idx, 0, 0.0, &ch);
+        if (p->opts.nranks > 1 && (force->exchange == PEPP_X_ALLGATHER || force->exchange == PEPP_X_HALO))
+            ch.exchange = force->exchange;
+        harvest(p, false);
+    } else {
+        pepp_status_t s = select_choice(p, &ch);
+        if (s) return s;
+    }
+
+    // timing: every calibration call and every forced call, then every
+    // sample_period-th call; never inside a CUDA graph capture
+    bool timed = !(flags & PEPP_EXEC_NO_TIMING);
+    if (timed) {
+        cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+        if (cudaStreamIsCapturing(st, &cs) != cudaSuccess) { (void)cudaGetLastError(); cs = cudaStreamCaptureStatusNone; }
+        if (cs != cudaStreamCaptureStatusNone) timed = false;
+    }
+    if (timed && !force && !ch.calibrating)
+        timed = p->opts.sample_period > 0 && (p->ncalls % p->opts.sample_period) == 0;
+    if (timed && p->ring_count == kTimingRing) timed = false;
+    TimingRec* rec = nullptr;
+    if (timed) {
+        rec = &p->ring[(p->ring_head + p->ring_count) % kTimingRing];
+        if (cudaEventRecord(rec->start, st) != cudaSuccess) { (void)cudaGetLastError(); rec = nullptr; }
+    }
+    pepp_status_t s = launch(p, p->cands[ch.candidate], x, y + p->row_offset, st);
+    if (s) { p->sticky = s; return s; }
+    if (rec) {
+        if (cudaEventRecord(rec->stop, st) == cudaSuccess) {
+            rec->cand = ch.candidate;
+            rec->pending = true;
+            ++p->ring_count;
+        } else {
+            (void)cudaGetLastError();
+        }
+    }
+    if (p->opts.nranks > 1 && (flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED))) {
+        const bool ag = (flags & PEPP_Y_REPLICATED) || ch.exchange == PEPP_X_ALLGATHER;
+        s = ag ? exchange_allgather(p, y, st) : exchange_halo(p, y, st);
+        if (s) { p->sticky = s; return s; }
+        ch.exchange = ag ? PEPP_X_ALLGATHER : PEPP_X_HALO;
+    } else {
+        ch.exchange = PEPP_X_NONE;
+    }
+    ++p->ncalls;
+    if (used) *used = ch;
+    return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const double* x_host, double* y_host,
+                                                     int32_t iterations, int flags, void* stream) {
+    if (!p || !x_host || !y_host || iterations < 1) return PEPP_E_INVALID;
+    if (p->sticky) return p->sticky;
+    if (iterations > 1 && p->ncols != p->global_rows) return PEPP_E_INVALID;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (cudaSetDevice(p->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    const int64_t nx = std::max<int64_t>(p->ncols, p->global_rows);
+    if (!p->d_hx) {
+        pepp_status_t s;
+        if ((s = dalloc(p, &p->d_hx, nx))) return s;
+        if ((s = dalloc(p, &p->d_hy, nx))) return s;
+    }
+    if (cudaMemcpyAsync(p->d_hx, x_host, sizeof(double) * p->ncols, cudaMemcpyHostToDevice, st) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return PEPP_E_CUDA;
+    }
+    double *xin = p->d_hx, *yout = p->d_hy;
+    for (int32_t it = 0; it < iterations; ++it) {
+        const bool last = it == iterations - 1;
+        const int f = last ? flags : (flags & PEPP_EXEC_NO_TIMING) | PEPP_Y_NEXT_INPUT;
+        pepp_status_t s = pepp_spmv_exec(p, xin, yout, f, stream, nullptr, nullptr);
+        if (s) return s;
+        if (!last) std::swap(xin, yout);
+    }
+    // rows written back: all global rows with PEPP_Y_REPLICATED, else this rank's rows
+    int64_t lo = p->row_offset, cnt = p->nrows;
+    if (p->opts.nranks > 1 && (flags & PEPP_Y_REPLICATED)) { lo = 0; cnt = p->global_rows; }
+    if (cnt > 0 && cudaMemcpyAsync(y_host + lo, yout + lo, sizeof(double) * cnt, cudaMemcpyDeviceToHost, st) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return PEPP_E_CUDA;
+    }
+    if (cudaStreamSynchronize(st) != cudaSuccess) { (void)cudaGetLastError(); p->sticky = PEPP_E_CUDA; return PEPP_E_CUDA; }
+    return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_destroy(pepp_spmv_plan_t* p) {
+    if (!p) return PEPP_OK;
+    cudaSetDevice(p->device);
+    harvest(p, true);
+    cudaDeviceSynchronize();
+    (void)cudaGetLastError();
+    pepp_status_t s = PEPP_OK;
+    if (!p->history_path.empty() && p->hist) s = pepp_history_save(p->hist, p->history_path.c_str());
+    free_plan(p);
+    return s;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_plan_info(const pepp_spmv_plan_t* p, pepp_plan_info_t* out) {
+    if (!p || !out) return PEPP_E_INVALID;
+    *out = p->info;
+    return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_candidates(const pepp_spmv_plan_t* p, pepp_choice_t* out, int32_t cap,
+                                                      int32_t* n) {
+    if (!p || !n) return PEPP_E_INVALID;
+    *n = (int32_t)p->cands.size();
+    for (int32_t i = 0; out && i < cap && i < *n; ++i) {
+        fill_choice(p, i, 0, 0.0, &out[i]);
+        const pepp::Welford* w = pepp::history_get(p->hist, p->key, i);
+        out[i].predicted_us = w ? w->mean : 0.0;
+    }
+    return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_flush_history(pepp_spmv_plan_t* p) {
+    if (!p) return PEPP_E_INVALID;
+    cudaSetDevice(p->device);
+    harvest(p, true);
+    return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_history_stats(const pepp_spmv_plan_t* p, int32_t cand, int64_t* count,
+                                                         double* mean_us, double* m2) {
+    if (!p) return PEPP_E_INVALID;
+    return pepp_history_stats(p->hist, p->key, cand, count, mean_us, m2);
+}

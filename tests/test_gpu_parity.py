@@ -1,0 +1,300 @@
+"""GPU parity: every variant of the CUDA path (through the C-ABI) against the
+CPU oracle, element by element. Integer-valued inputs -> bit-exact (==);
+real inputs -> per-row bound of BASELINE.json north_star:
+    |y - y_ref| <= 2 * nnz_row * 2^-52 * sum_j |a_ij||x_j|
+(empty rows must be exactly 0)."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_sc_dastgeerlk12_b200 as pepp  # noqa: E402
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def _run(plan, x, force=None, ylen=None, flags=0):
+    xd = _dev(x)
+    y = torch.full((ylen if ylen is not None else plan.nrows,), float("nan"), dtype=torch.float64, device="cuda")
+    used = plan.exec(xd, y, flags=flags, force=force)
+    torch.cuda.synchronize()
+    return y.cpu().numpy(), used
+
+
+def _all_forces(plan):
+    return [pepp.Choice(c.variant, c.param) for c in plan.candidates()]
+
+
+def _check(A, x, y, exact):
+    yr = oracle.spmv(A, x)
+    if exact:
+        assert np.array_equal(y, yr), np.flatnonzero(y != yr)[:10]
+    else:
+        b = oracle.bound(A, x)
+        bad = np.flatnonzero(~(np.abs(y - yr) <= b))
+        assert bad.size == 0, (bad[:10], y[bad[:5]], yr[bad[:5]], b[bad[:5]])
+
+
+CASES = {
+    "lap64_int": lambda: (gen.laplacian2d(64), gen.vector(1, gen.INT8, 4096), True),       # config 1, int mode
+    "lap64_real": lambda: (gen.laplacian2d(64), gen.vector(2, gen.REAL, 4096), False),     # config 1, real mode
+    "uniform_int": lambda: (gen.uniform(50_000, 50_000, 16, seed=43, val_mode=gen.INT4),
+                            gen.vector(44, gen.INT8, 50_000), True),
+    "uniform_real": lambda: (gen.uniform(50_000, 40_000, 16, seed=42), gen.vector(45, gen.REAL, 40_000), False),
+    "zipf_int": lambda: (gen.zipf(60_000, 60_000, seed=47, val_mode=gen.INT4), gen.vector(48, gen.INT8, 60_000), True),
+    "zipf_real": lambda: (gen.zipf(60_000, 60_000, seed=46), gen.vector(49, gen.REAL, 60_000), False),
+    "banded_real": lambda: (gen.banded(30_001, 4, seed=100), gen.vector(101, gen.REAL, 30_001), False),
+    "perm": lambda: (gen.permutation_matrix(10_007, 5), gen.vector(9, gen.REAL, 10_007), True),
+    "diag": lambda: (gen.diagonal_matrix(10_007, 6), gen.vector(10, gen.REAL, 10_007), True),
+}
+
+
+@pytest.mark.parametrize("case", sorted(CASES))
+def test_every_variant_matches_oracle(case):
+    A, x, exact = CASES[case]()
+    with pepp.Plan.from_csr(A) as plan:
+        forces = _all_forces(plan)
+        assert {f.variant for f in forces} == {pepp.V_CSR_VECTOR, pepp.V_MERGE_PATH, pepp.V_SELL}
+        for f in forces:
+            y, used = _run(plan, x, force=f)
+            assert (used.variant, used.param) == (f.variant, f.param)
+            _check(A, x, y, exact)
+
+
+def _hand(nrows, ncols, rows):
+    rp = [0]
+    cols, vals = [], []
+    for r in rows:
+        for c, v in r:
+            cols.append(c)
+            vals.append(v)
+        rp.append(len(cols))
+    return gen.CSR(nrows, ncols, np.array(rp, np.int64), np.array(cols, np.int32), np.array(vals, np.float64), 0, nrows)
+
+
+def _edge_cases():
+    rng = np.random.default_rng(0)
+    out = {}
+    out["one_row"] = _hand(1, 5, [[(0, 1.0), (4, 2.0)]])
+    out["one_empty_row"] = _hand(1, 3, [[]])
+    out["nnz0"] = _hand(100, 100, [[] for _ in range(100)])
+    out["ncols_ne_nrows"] = gen.uniform(3000, 17, 5, seed=3, val_mode=gen.INT4)
+    # one 1M-nnz row among short ones (rows longer than many merge tiles)
+    long = [(int(c), float(rng.integers(-4, 5))) for c in rng.integers(0, 5000, 1_000_000)]
+    out["one_long_row"] = _hand(5, 5000, [[(1, 1.0)], long, [], [(2, -3.0), (2, 1.0)], [(4999, 2.0)]])
+    # duplicates and unsorted columns (A8)
+    rows = []
+    for i in range(4000):
+        L = int(rng.integers(0, 40))
+        rows.append([(int(rng.integers(0, 300)), float(rng.integers(-4, 5))) for _ in range(L)])
+    out["dup_unsorted"] = _hand(4000, 300, rows)
+    # every row length 0..70 in sequence: all alignments of row starts
+    rows = [[(int((i * 7 + j) % 999), float(1 + (i + j) % 4)) for j in range(i % 71)] for i in range(5000)]
+    out["all_lengths"] = _hand(5000, 999, rows)
+    # many empty rows
+    rows = [[] if i % 3 else [(i % 50, 2.0)] for i in range(10_000)]
+    out["mostly_empty"] = _hand(10_000, 50, rows)
+    return out
+
+
+EDGE = _edge_cases()
+
+
+@pytest.mark.parametrize("name", sorted(EDGE))
+def test_edge_cases_bitwise(name):
+    A = EDGE[name]
+    x = gen.vector(11, gen.INT8, A.ncols)
+    with pepp.Plan.from_csr(A) as plan:
+        for f in _all_forces(plan):
+            y, _ = _run(plan, x, force=f)
+            _check(A, x, y, exact=True)
+            if A.nnz == 0:
+                assert np.all(y == 0)
+
+
+def test_empty_matrix_plan_and_exec():
+    A = _hand(0, 10, [])
+    with pepp.Plan.from_csr(A) as plan:
+        x = torch.ones(10, dtype=torch.float64, device="cuda")
+        y = torch.empty(0, dtype=torch.float64, device="cuda")
+        for f in _all_forces(plan):
+            plan.exec(x, y, force=f)
+        torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("first", [0, 1, 2, 3, 5, (1 << 33) + 7])
+def test_first_offset_any_alignment(first):
+    A = gen.zipf(20_000, 20_000, seed=46, val_mode=gen.INT4)
+    Ar = gen.rebase(A, first)
+    x = gen.vector(3, gen.INT8, 20_000)
+    yr = oracle.spmv(A, x)
+    with pepp.Plan.from_csr(Ar) as plan:
+        for f in _all_forces(plan):
+            y, _ = _run(plan, x, force=f)
+            assert np.array_equal(y, yr)
+
+
+def test_partition_invariance_bitwise_real():
+    """P8: row blocks with their own `first` concatenate to the P=1 result
+    bitwise for the same variant (alignment preserved by the front pad)."""
+    A = gen.zipf(40_000, 40_000, seed=46)
+    x = gen.vector(49, gen.REAL, 40_000)
+    xd = _dev(x)
+    with pepp.Plan.from_csr(A) as whole:
+        for f in _all_forces(whole):
+            if f.variant != pepp.V_CSR_VECTOR:
+                continue   # merge tiles / SELL chunks depend on the block boundaries
+            y1, _ = _run(whole, x, force=f)
+            for P in (2, 3, 8):
+                b = pepp.partition_rows(A.row_ptr, P)
+                y = torch.empty(A.nrows, dtype=torch.float64, device="cuda")
+                for r in range(P):
+                    blk = gen.row_block(A, int(b[r]), int(b[r + 1]))
+                    with pepp.Plan.from_csr(blk) as pl:
+                        pl.exec(xd, y[b[r]:b[r + 1]], force=f)
+                torch.cuda.synchronize()
+                assert np.array_equal(y.cpu().numpy(), y1)
+
+
+def test_determinism_bitwise():
+    A = gen.zipf(50_000, 50_000, seed=46)
+    x = gen.vector(49, gen.REAL, 50_000)
+    with pepp.Plan.from_csr(A) as plan:
+        for f in _all_forces(plan):
+            y1, _ = _run(plan, x, force=f)
+            y2, _ = _run(plan, x, force=f)
+            assert np.array_equal(y1, y2)
+
+
+def test_power_of_two_scaling_bitwise():
+    A = gen.uniform(20_000, 20_000, 16, seed=42)
+    x = gen.vector(45, gen.REAL, 20_000)
+    with pepp.Plan.from_csr(A) as plan:
+        for f in _all_forces(plan):
+            y, _ = _run(plan, x, force=f)
+            y8, _ = _run(plan, x * 8.0, force=f)
+            assert np.array_equal(y8, y * 8.0)
+
+
+def test_device_resident_operand_and_host_operand_agree():
+    A = gen.zipf(10_000, 10_000, seed=46, val_mode=gen.INT4)
+    x = gen.vector(3, gen.INT8, 10_000)
+    with pepp.Plan.from_csr(A) as ph, pepp.Plan(A.nrows, A.ncols, _dev(A.row_ptr), _dev(A.col), _dev(A.val)) as pd:
+        for f in _all_forces(ph):
+            assert np.array_equal(_run(ph, x, force=f)[0], _run(pd, x, force=f)[0])
+
+
+def test_iterated_laplacian_integer_bitwise_k16():
+    n = 128
+    A = gen.laplacian2d(n)
+    x0 = gen.vector(3, gen.INT8, n * n)
+    ref = oracle.iterate(A, x0, 16)
+    with pepp.Plan.from_csr(A) as plan:
+        for f in _all_forces(plan):
+            a = _dev(x0)
+            b = torch.empty_like(a)
+            for _ in range(16):
+                plan.exec(a, b, force=f)
+                a, b = b, a
+            torch.cuda.synchronize()
+            assert np.array_equal(a.cpu().numpy(), ref)
+
+
+def test_iterated_real_within_propagated_bound():
+    n, K = 64, 100
+    A = gen.laplacian2d(n)
+    x0 = gen.vector(4, gen.REAL, n * n)
+    xK, zK = oracle.iterate(A, x0, K, with_bound=True)
+    bnd = oracle.iterate_bound(A, zK, K)
+    with pepp.Plan.from_csr(A) as plan:
+        for f in _all_forces(plan):
+            a = _dev(x0)
+            b = torch.empty_like(a)
+            for _ in range(K):
+                plan.exec(a, b, force=f)
+                a, b = b, a
+            torch.cuda.synchronize()
+            assert np.all(np.abs(a.cpu().numpy() - xK) <= bnd)
+
+
+def test_exec_host_matches_device_path():
+    A = gen.laplacian2d(100)
+    x = gen.vector(3, gen.INT8, 10_000)
+    ref1 = oracle.spmv(A, x)
+    ref5 = oracle.iterate(A, x, 5)
+    with pepp.Plan.from_csr(A) as plan:
+        y = np.empty(10_000)
+        plan.exec_host(x, y, iterations=1)
+        assert np.array_equal(y, ref1)
+        plan.exec_host(x, y, iterations=5)
+        assert np.array_equal(y, ref5)
+
+
+# ------------------------------------------------------------- selector --
+def test_selector_calibrates_then_picks_fastest_measured():
+    A = gen.uniform(200_000, 200_000, 16, seed=42)
+    x = _dev(gen.vector(45, gen.REAL, 200_000))
+    y = torch.empty(200_000, dtype=torch.float64, device="cuda")
+    with pepp.Plan.from_csr(A, min_samples=3) as plan:
+        n = len(plan.candidates())
+        seen = []
+        for _ in range(3 * n):
+            u = plan.exec(x, y)
+            assert u.calibrating
+            seen.append(u.candidate)
+        assert sorted(set(seen)) == list(range(n))
+        plan.flush_history()
+        means = [plan.history_stats(c)[1] for c in range(n)]
+        ch = plan.select()
+        assert not ch.calibrating
+        best = min(means)
+        assert means[ch.candidate] <= best * 1.01 + 1e-9
+        u = plan.exec(x, y)
+        assert u.candidate == ch.candidate
+
+
+def test_variant_mask_and_static_heuristic():
+    A = gen.zipf(50_000, 50_000, seed=46)
+    x = _dev(gen.vector(45, gen.REAL, 50_000))
+    y = torch.empty(50_000, dtype=torch.float64, device="cuda")
+    with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_SELL) as plan:
+        assert [c.variant for c in plan.candidates()] == [pepp.V_SELL]
+        assert plan.exec(x, y).variant == pepp.V_SELL
+        with pytest.raises(pepp.PeppError):
+            plan.exec(x, y, force=pepp.Choice(pepp.V_MERGE_PATH))
+    with pepp.Plan.from_csr(A, use_history=False) as plan:
+        c = plan.exec(x, y)
+        assert not c.calibrating
+        assert c.variant == pepp.V_MERGE_PATH   # CV > 1 for the power-law rows
+
+
+def test_error_codes():
+    A = gen.laplacian2d(16)
+    with pepp.Plan.from_csr(A) as plan:
+        x = torch.ones(256, dtype=torch.float64, device="cuda")
+        with pytest.raises(pepp.PeppError) as e:
+            plan.exec(x, x)                       # x and y alias
+        assert e.value.status == pepp._capi.PEPP_E_INVALID
+        with pytest.raises(pepp.PeppError):
+            plan.exec(x, x[10:])                  # overlap
+    bad = gen.laplacian2d(16)
+    bad.col = bad.col.copy()
+    bad.col[7] = 256                              # column out of range
+    with pytest.raises(pepp.PeppError):
+        pepp.Plan.from_csr(bad)
+    bad = gen.laplacian2d(16)
+    bad.row_ptr = bad.row_ptr.copy()
+    bad.row_ptr[5] = bad.row_ptr[7]               # non-monotone
+    with pytest.raises(pepp.PeppError):
+        pepp.Plan.from_csr(bad)
+    bad = gen.laplacian2d(16)
+    with pytest.raises(pepp.PeppError):           # row_ptr[nrows] - first != nnz
+        pepp.Plan(bad.nrows, bad.ncols, bad.row_ptr, bad.col[:-1], bad.val[:-1])

@@ -1,0 +1,143 @@
+"""Host-side logic of the C-ABI library, CPU only: partitioner, halo ghost
+lists, performance history + selection policy (injected "fake clock" times),
+context keys. SURVEY.md §4.2 tier T2/T3 host parts."""
+from __future__ import annotations
+
+import os
+import tempfile
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+import paper_conf_sc_dastgeerlk12_b200 as pepp
+
+
+@pytest.mark.parametrize("maker", ["lap", "zipf", "uniform", "banded", "empty_rows"])
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+def test_partition_equals_oracle_definition(maker, P):
+    A = {
+        "lap": lambda: gen.laplacian2d(40),
+        "zipf": lambda: gen.zipf(3000, 3000, seed=46),
+        "uniform": lambda: gen.uniform(2000, 2000, 16, seed=42),
+        "banded": lambda: gen.banded(1500, 4, seed=100),
+        "empty_rows": lambda: gen.CSR(6, 6, np.array([0, 0, 0, 10, 10, 10, 12], dtype=np.int64),
+                                      np.zeros(12, np.int32), np.ones(12), 0, 6),
+    }[maker]()
+    b = pepp.partition_rows(A.row_ptr, P)
+    assert np.array_equal(b, oracle.partition_nnz(A, P))
+    # with a non-zero `first` (a block of a bigger matrix) the rule is unchanged
+    Ar = gen.rebase(A, 1 << 35)
+    assert np.array_equal(pepp.partition_rows(Ar.row_ptr, P), b)
+
+
+def test_partition_laplacian_8192_balanced():
+    n = 8192
+    rp = np.empty(n * n + 1, dtype=np.int64)
+    import ctypes
+    gen.lib().gen_laplacian2d_rowptr(n, 0, n * n, rp.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)))
+    for P in (2, 4, 8):
+        b = pepp.partition_rows(rp, P)
+        sizes = np.diff(rp[b])
+        assert sizes.max() - sizes.min() <= 10
+        assert abs(int(sizes.sum()) - 335_511_552) == 0
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_halo_ghosts_match_set_definition(P):
+    A = gen.zipf(2500, 2500, seed=7, kmax=60)
+    b = pepp.partition_rows(A.row_ptr, P)
+    for r in range(P):
+        blk = gen.row_block(A, int(b[r]), int(b[r + 1]))
+        counts, g = pepp.halo_ghosts(blk.col, P, r, b)
+        cols = set(int(c) for c in blk.col)
+        expect = sorted(c for c in cols if not (b[r] <= c < b[r + 1]))
+        assert g.tolist() == expect
+        assert counts[r] == 0 and counts.sum() == len(expect)
+        for q in range(P):
+            assert counts[q] == sum(1 for c in expect if b[q] <= c < b[q + 1])
+
+
+def test_halo_laplacian_is_two_grid_rows():
+    n, P = 64, 4
+    A = gen.laplacian2d(n)
+    b = pepp.partition_rows(A.row_ptr, P)
+    for r in range(P):
+        blk = gen.row_block(A, int(b[r]), int(b[r + 1]))
+        counts, g = pepp.halo_ghosts(blk.col, P, r, b)
+        # ghosts: n entries below and n above (one grid row each side), contiguous
+        if 0 < r < P - 1:
+            assert counts[r - 1] == n and counts[r + 1] == n
+        assert len(g) == (n if r in (0, P - 1) else 2 * n)
+
+
+# ------------------------------------------------------------ history ----
+def test_history_calibrates_then_exploits_argmin():
+    H = pepp.History()
+    key = 12345
+    times = [5.0, 3.0, 4.0, 3.02]      # fake clock: candidate 1 fastest; 3 within 1 %
+    elig = [True] * 4
+    order = []
+    for _ in range(100):
+        c, cal, _ = H.select(key, elig, min_samples=3)
+        if not cal:
+            break
+        order.append(c)
+        H.record(key, c, times[c])
+    # calibration visits each candidate min_samples times, lowest index first
+    assert order == [0, 0, 0, 1, 1, 1, 2, 2, 2, 3, 3, 3]
+    c, cal, pred = H.select(key, elig, min_samples=3)
+    assert (c, cal) == (1, False) and pred == pytest.approx(3.0)
+    # candidate 3 is 0.7 % slower: the tie rule keeps the lower index
+    assert H.select(key, elig)[0] == 1
+    # masking the best one out (disableImpls) picks the next best
+    assert H.select(key, [True, False, True, True])[0] == 3
+    # other keys are independent (context instances)
+    assert H.select(key + 1, elig) == (0, True, 0.0)
+
+
+def test_history_tracks_drift_and_welford():
+    H = pepp.History()
+    xs = [1.0, 2.0, 4.0, 8.0]
+    for v in xs:
+        H.record(7, 0, v)
+    n, m, m2 = H.stats(7, 0)
+    assert n == 4 and m == pytest.approx(np.mean(xs)) and m2 / (n - 1) == pytest.approx(np.var(xs, ddof=1))
+    # the choice follows the measurements when they change
+    for _ in range(3):
+        H.record(7, 1, 10.0)
+    assert H.select(7, [True, True], 3)[0] == 0
+    for _ in range(50):
+        H.record(7, 0, 100.0)
+    assert H.select(7, [True, True], 3)[0] == 1
+
+
+def test_history_save_load_merges():
+    H = pepp.History()
+    for v in (1.0, 3.0):
+        H.record(9, 2, v)
+    with tempfile.TemporaryDirectory() as d:
+        p = os.path.join(d, "h.txt")
+        H.save(p)
+        G = pepp.History()
+        G.record(9, 2, 5.0)
+        G.load(p)
+        n, m, m2 = G.stats(9, 2)
+        assert n == 3 and m == pytest.approx(3.0) and m2 == pytest.approx(np.var([1, 3, 5]) * 3)
+
+
+def test_history_rejects_bad_input():
+    H = pepp.History()
+    with pytest.raises(pepp.PeppError):
+        H.record(1, 0, float("nan"))
+    with pytest.raises(pepp.PeppError):
+        H.select(1, [False, False])
+
+
+def test_context_key_buckets():
+    k = pepp.context_key(1 << 20, 1 << 20, 16 << 20, 0.0)
+    assert k == pepp.context_key((1 << 20) + 1000, 1 << 20, (16 << 20) + 5000, 0.1)   # same bucket
+    assert k != pepp.context_key(1 << 22, 1 << 20, 16 << 20, 0.0)
+    assert k != pepp.context_key(1 << 20, 1 << 20, 16 << 20, 3.0)
+    assert k != pepp.context_key(1 << 20, 1 << 20, 16 << 20, 0.0, nparts=2)
