@@ -103,6 +103,7 @@ struct pepp_spmv_plan_s {
     TimingRec ring[kTimingRing];
     int ring_head = 0;   // oldest pending
     int ring_count = 0;
+    std::vector<int32_t> pending;   // timed calls in flight per candidate
 
     // multi-GPU
     const Nccl* nccl = nullptr;
@@ -295,6 +296,7 @@ void harvest(pepp_spmv_plan_t* p, bool block) {
             pepp::history_add(p->hist, p->key, r.cand, (double)ms * 1000.0);
         (void)cudaGetLastError();
         r.pending = false;
+        if (r.cand >= 0 && r.cand < (int)p->pending.size()) --p->pending[r.cand];
         p->ring_head = (p->ring_head + 1) % kTimingRing;
         --p->ring_count;
     }
@@ -335,8 +337,25 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out) {
     double pred = 0.0;
     int cand;
     if (p->opts.use_history) {
-        cand = pepp::history_pick(p->hist, p->key, (int32_t)p->cands.size(), p->eligible.data(),
-                                  std::max(1, p->opts.min_samples), &calibrating, &pred);
+        // Calibration counts timed calls already in flight, so the host (which
+        // runs far ahead of the GPU) moves on to the next under-sampled
+        // candidate instead of re-issuing the same one; once every candidate
+        // has min_samples calls issued, wait for them once and exploit.
+        const int32_t ms = std::max(1, p->opts.min_samples);
+        const int32_t n = (int32_t)p->cands.size();
+        cand = -1;
+        bool waiting = false;
+        for (int32_t c = 0; c < n; ++c) {
+            if (!p->eligible[c]) continue;
+            const pepp::Welford* w = pepp::history_get(p->hist, p->key, c);
+            const int64_t done = w ? w->count : 0;
+            if (done + p->pending[c] < ms) { cand = c; calibrating = 1; pred = w ? w->mean : 0.0; break; }
+            if (done < ms) waiting = true;
+        }
+        if (cand < 0) {
+            if (waiting) harvest(p, true);
+            cand = pepp::history_pick(p->hist, p->key, n, p->eligible.data(), ms, &calibrating, &pred);
+        }
     } else {
         cand = heuristic_candidate(p);
     }
@@ -578,6 +597,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     }
     if (mask & (1u << PEPP_V_MERGE_PATH)) { if ((s = prepare_merge(p, st))) return s; }
     p->eligible.assign(p->cands.size(), 1);
+    p->pending.assign(p->cands.size(), 0);
     I.ncandidates = (int32_t)p->cands.size();
 
     p->grid_csr[1] = grid_for((const void*)pepp::k::csr_vector_kernel<2, kBlock>, kBlock, A->nrows, kBlock / 2, p->sm_count);
@@ -671,8 +691,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const doub
                                                 void* stream, const pepp_choice_t* force, pepp_choice_t* used) {
     if (!p) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
-    if (!x || !y) return PEPP_E_INVALID;
-    {   // x [0, ncols) and y [0, global_rows) must not overlap
+    if ((!x && p->ncols > 0) || (!y && p->global_rows > 0)) return PEPP_E_INVALID;
+    if (x && y) {   // x [0, ncols) and y [0, global_rows) must not overlap
         const char *xb = (const char*)x, *xe = (const char*)(x + p->ncols);
         const char *yb = (const char*)y, *ye = (const char*)(y + p->global_rows);
         if (xb < ye && yb < xe) return PEPP_E_INVALID;
@@ -720,6 +740,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const doub
         if (cudaEventRecord(rec->stop, st) == cudaSuccess) {
             rec->cand = ch.candidate;
             rec->pending = true;
+            ++p->pending[ch.candidate];
             ++p->ring_count;
         } else {
             (void)cudaGetLastError();
