@@ -66,14 +66,15 @@ typedef enum {
 } pepp_status_t;
 
 /* Implementation variants (§II P@4772: "several implementations of one
-   interface"; the paper's CUSP variant P@33595 is replaced by three
+   interface"; the paper's CUSP variant P@33595 is replaced by four
    hand-written sm_100a kernels). */
 typedef enum {
     PEPP_V_AUTO = -1,
     PEPP_V_CSR_VECTOR = 0,    /* TPR lanes per row, 128-bit val/col loads, shfl_xor reduction; param = TPR */
     PEPP_V_MERGE_PATH = 1,    /* merge-path over (row ends, nnz), smem-staged, deterministic carry fix-up */
     PEPP_V_SELL = 2,          /* SELL-C-σ, C = 32, column-major chunks; param = σ */
-    PEPP_V_COUNT = 3
+    PEPP_V_CSR_STREAM = 3,    /* CSR-stream fed by a TMA (cp.async.bulk) shared-memory pipeline; param = nnz per item */
+    PEPP_V_COUNT = 4
 } pepp_variant_t;
 
 /* Exchange that makes y usable as the next x when the call is partitioned */
@@ -135,7 +136,7 @@ typedef struct {
 /* Selection result. `candidate` indexes pepp_spmv_candidates(). */
 typedef struct {
     int32_t variant;          /* pepp_variant_t */
-    int32_t param;            /* TPR (CSR_VECTOR), σ (SELL), items per thread (MERGE_PATH) */
+    int32_t param;            /* TPR (CSR_VECTOR), σ (SELL), items per thread (MERGE_PATH), nnz per item (CSR_STREAM) */
     int32_t nparts;           /* ranks the call runs on */
     int32_t exchange;         /* pepp_exchange_t used when flags ask for it */
     int32_t calibrating;      /* 1 = chosen to gather history, not the predicted best */

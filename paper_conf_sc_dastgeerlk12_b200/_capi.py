@@ -12,10 +12,10 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libpepp_spmv.so")
 
 PEPP_OK, PEPP_E_INVALID, PEPP_E_CUDA, PEPP_E_NCCL, PEPP_E_NOMEM, PEPP_E_UNSUPPORTED, PEPP_E_STATE = 0, -1, -2, -3, -4, -5, -6
-V_AUTO, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, V_COUNT = -1, 0, 1, 2, 3
+V_AUTO, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, V_CSR_STREAM, V_COUNT = -1, 0, 1, 2, 3, 4
 X_AUTO, X_NONE, X_ALLGATHER, X_HALO = -1, 0, 1, 2
 Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, EXEC_NO_TIMING = 0x0, 0x1, 0x2, 0x10
-VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell"}
+VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell", V_CSR_STREAM: "csr_stream"}
 EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_AUTO: "auto"}
 
 c_i32, c_i64, c_u32, c_u64, c_f64, c_vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_uint64,

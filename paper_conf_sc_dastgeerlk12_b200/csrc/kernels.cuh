@@ -29,6 +29,8 @@ namespace k {
 // path, no L1 allocation, L2 evict-first policy (createpolicy) so that x
 // keeps its L2 residency. (On sm_100a the bare .L2::evict_first qualifier is
 // only accepted on 256-bit loads; the cache_hint form works for every width.)
+// Not `volatile`: the matrix is read-only during a launch, and volatile asm
+// would pin the loads in program order and stop ptxas from batching them.
 __device__ __forceinline__ uint64_t evict_first_policy() {
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
@@ -36,24 +38,24 @@ __device__ __forceinline__ uint64_t evict_first_policy() {
 }
 __device__ __forceinline__ int4 ld_stream_i4(const int* p, uint64_t pol) {
     int4 r;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
                  : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
     return r;
 }
 __device__ __forceinline__ double2 ld_stream_d2(const double* p, uint64_t pol) {
     double2 r;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0,%1}, [%2], %3;"
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0,%1}, [%2], %3;"
                  : "=d"(r.x), "=d"(r.y) : "l"(p), "l"(pol));
     return r;
 }
 __device__ __forceinline__ double ld_stream_d(const double* p, uint64_t pol) {
     double r;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(r) : "l"(p), "l"(pol));
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(r) : "l"(p), "l"(pol));
     return r;
 }
 __device__ __forceinline__ int ld_stream_i(const int* p, uint64_t pol) {
     int r;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
     return r;
 }
 // x gather: read-only path, cached in L1 and L2 (reused across rows)
@@ -131,11 +133,37 @@ __global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int*
 // =====================================================================
 // Variant 2: SELL-C-σ, C = 32. Chunk c holds the 32 (sorted) rows
 // [32c, 32c+32): slot j of lane l is at chunk_ptr[c] + 32*j + l, so a warp
-// reads 256 contiguous bytes of values and 128 of columns per slot. Each
-// lane masks slots beyond its own row length (no padding arithmetic, so
-// Inf/NaN in x behave exactly as in the CSR definition). perm maps sorted
-// position -> original row (NULL when σ = 1).
+// reads 256 contiguous bytes of values and 128 of columns per slot.
+// chunk_len[c] >= 0: every row of the chunk has exactly that many entries
+// (no per-row length is read); chunk_len[c] < 0: -chunk_len[c] slots and
+// each lane masks the slots beyond its own row length rowlen[32c+l] (no
+// padding arithmetic, so Inf/NaN in x behave exactly as in the CSR
+// definition). perm maps sorted position -> original row (NULL when σ = 1).
+// The kernel is latency-bound at one chunk per warp, so each chunk's slots
+// are loaded in batches of up to 8 (all column and value loads, then all x
+// gathers, then the FMAs) with an exactly-sized tail batch.
 // =====================================================================
+// N slots of one chunk, loads issued unconditionally (all N exist for every
+// lane) before the first FMA; the per-lane row length only masks the FMA.
+template <int N>
+__device__ __forceinline__ double sell_slots(const double* __restrict__ val, const int* __restrict__ col,
+                                             const double* __restrict__ x, int64_t base, int j0, int len,
+                                             double acc, uint64_t pol) {
+    double v[N];
+    int c[N];
+#pragma unroll
+    for (int u = 0; u < N; ++u) c[u] = ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
+#pragma unroll
+    for (int u = 0; u < N; ++u) v[u] = ld_stream_d(val + base + (int64_t)(j0 + u) * 32, pol);
+    double xv[N];
+#pragma unroll
+    for (int u = 0; u < N; ++u) xv[u] = ld_x(x, c[u]);
+#pragma unroll
+    for (int u = 0; u < N; ++u)
+        if (j0 + u < len) acc = fma(v[u], xv[u], acc);
+    return acc;
+}
+
 template <int BLOCK>
 __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
                                                      const int* __restrict__ chunk_len,
@@ -150,29 +178,25 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     const int nwarps = (gridDim.x * BLOCK) >> 5;
     const uint64_t pol = evict_first_policy();
     for (int c = warp; c < nchunks; c += nwarps) {
-        const int r = c * 32 + lane;
-        const int len = r < nrows ? __ldg(rowlen + r) : 0;
-        const int clen = __ldg(chunk_len + c);
+        const int cl = __ldg(chunk_len + c);
         const int64_t base = __ldg(chunk_ptr + c) + lane;
+        const int clen = cl >= 0 ? cl : -cl;
+        const int r = c * 32 + lane;
+        const int len = cl >= 0 ? cl : (r < nrows ? __ldg(rowlen + r) : 0);
         double acc = 0.0;
         int j = 0;
-        for (; j + 4 <= clen; j += 4) {
-            double v[4];
-            int ci[4];
-#pragma unroll
-            for (int u = 0; u < 4; ++u) {
-                v[u] = 0.0; ci[u] = 0;
-                if (j + u < len) {
-                    v[u] = ld_stream_d(val + base + (int64_t)(j + u) * 32, pol);
-                    ci[u] = ld_stream_i(col + base + (int64_t)(j + u) * 32, pol);
-                }
-            }
-#pragma unroll
-            for (int u = 0; u < 4; ++u)
-                if (j + u < len) acc = fma(v[u], ld_x(x, ci[u]), acc);
+        // whole blocks of 8 slots, then one exactly-sized tail (warp-uniform switch)
+        for (; j + 8 <= clen; j += 8) acc = sell_slots<8>(val, col, x, base, j, len, acc, pol);
+        switch (clen - j) {
+        case 1: acc = sell_slots<1>(val, col, x, base, j, len, acc, pol); break;
+        case 2: acc = sell_slots<2>(val, col, x, base, j, len, acc, pol); break;
+        case 3: acc = sell_slots<3>(val, col, x, base, j, len, acc, pol); break;
+        case 4: acc = sell_slots<4>(val, col, x, base, j, len, acc, pol); break;
+        case 5: acc = sell_slots<5>(val, col, x, base, j, len, acc, pol); break;
+        case 6: acc = sell_slots<6>(val, col, x, base, j, len, acc, pol); break;
+        case 7: acc = sell_slots<7>(val, col, x, base, j, len, acc, pol); break;
+        default: break;
         }
-        for (; j < clen; ++j)
-            if (j < len) acc = fma(ld_stream_d(val + base + (int64_t)j * 32, pol), ld_x(x, ld_stream_i(col + base + (int64_t)j * 32, pol)), acc);
         if (r < nrows) y[perm ? __ldg(perm + r) : r] = acc;
     }
 }
@@ -325,6 +349,184 @@ __global__ void merge_tile_search_kernel(int nrows, int64_t nnz, const int* __re
 }
 
 // =====================================================================
+// Variant 3: CSR-stream with a TMA bulk-copy pipeline (B200-native).
+// The matrix is cut at plan time into work items of <= NB nonzeros and
+// <= RMAX rows (rows longer than NB become "pieces" of NB nonzeros). A
+// persistent CTA owns items b, b+G, b+2G, ...; one thread streams each
+// item's row_ptr slice, columns and values into a STAGES-deep shared-memory
+// ring with cp.async.bulk (completion counted on an mbarrier per stage),
+// so STAGES-1 items are in flight while the CTA computes the current one:
+//   phase 1 (balanced over nonzeros): sval[k] <- val[k] * x[col[k]]
+//   phase 2 (per row): stream items: one thread per row sums its products
+//           sequentially from +0.0 — the oracle's exact arithmetic (product
+//           rounded, then each sum rounded, ascending k), so results are
+//           bit-identical to the definition; vector items (long rows): one
+//           warp per row, shuffle tree; long-row pieces: a block-wide sum
+//           written to a carry slot, combined by csr_stream_fixup_kernel.
+// =====================================================================
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t done;
+    do {
+        asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+                     : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint64_t pol) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
+}
+
+constexpr int kStreamVecFlag = 0x40000000;   // item.y flag: warp-per-row reduction
+
+template <int NB, int RMAX>
+struct StreamStage {
+    double val[NB + 8];
+    int col[NB + 8];
+    int rp[RMAX + 8];
+};
+
+template <int BLOCK, int STAGES, int NB, int RMAX>
+__global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const int4* __restrict__ items,
+                                                               const int* __restrict__ rp,
+                                                               const int* __restrict__ col,
+                                                               const double* __restrict__ val,
+                                                               const double* __restrict__ x,
+                                                               double* __restrict__ y,
+                                                               double* __restrict__ carry) {
+    using Stage = StreamStage<NB, RMAX>;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    Stage* st = reinterpret_cast<Stage*>(smem_raw);
+    __shared__ __align__(8) uint64_t full[STAGES];
+    __shared__ double s_red[BLOCK / 32];
+
+    const int tid = threadIdx.x;
+    const int G = gridDim.x;
+    const int nmine = nitems > (int)blockIdx.x ? (nitems - (int)blockIdx.x + G - 1) / G : 0;
+
+    uint64_t pol = 0;
+    if (tid == 0) {
+        for (int s = 0; s < STAGES; ++s) mbar_init(&full[s], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        pol = evict_first_policy();
+    }
+    __syncthreads();
+
+    auto issue = [&](int j) {   // thread 0: stream local item j into stage j % STAGES
+        const int4 it = __ldg(items + blockIdx.x + (int64_t)j * G);
+        Stage& S = st[j % STAGES];
+        const int k0a = it.z & ~3, k1a = (it.w + 3) & ~3;
+        uint32_t bytes = (uint32_t)(k1a - k0a) * 12u;
+        int r0a = 0, r1a = 0;
+        if (it.y >= 0) {
+            const int r1 = it.y & ~kStreamVecFlag;
+            r0a = it.x & ~3;
+            r1a = (r1 + 1 + 3) & ~3;
+            bytes += (uint32_t)(r1a - r0a) * 4u;
+        }
+        mbar_arrive_expect_tx(&full[j % STAGES], bytes);
+        if (k1a > k0a) {
+            tma_load_1d(S.val, val + k0a, (uint32_t)(k1a - k0a) * 8u, &full[j % STAGES], pol);
+            tma_load_1d(S.col, col + k0a, (uint32_t)(k1a - k0a) * 4u, &full[j % STAGES], pol);
+        }
+        if (r1a > r0a) tma_load_1d(S.rp, rp + r0a, (uint32_t)(r1a - r0a) * 4u, &full[j % STAGES], pol);
+    };
+
+    if (tid == 0)
+        for (int j = 0; j < STAGES - 1 && j < nmine; ++j) issue(j);
+
+    for (int j = 0; j < nmine; ++j) {
+        if (tid == 0 && j + STAGES - 1 < nmine) issue(j + STAGES - 1);
+        const int4 it = __ldg(items + blockIdx.x + (int64_t)j * G);
+        Stage& S = st[j % STAGES];
+        mbar_wait(&full[j % STAGES], (uint32_t)((j / STAGES) & 1));
+
+        const int k0a = it.z & ~3;
+        const int off = it.z - k0a;
+        const int nz = it.w - it.z;
+        // phase 1: products in place, balanced over nonzeros. Batched: all of
+        // a thread's (val, col) smem reads, then all its x gathers, then the
+        // products, so the gathers overlap instead of forming a serial chain.
+        {
+            constexpr int PER = (NB + BLOCK - 1) / BLOCK;
+            double v[PER];
+            int c[PER];
+#pragma unroll
+            for (int u = 0; u < PER; ++u) {
+                const int i = tid + u * BLOCK;
+                v[u] = 0.0;
+                c[u] = 0;
+                if (i < nz) { v[u] = S.val[off + i]; c[u] = S.col[off + i]; }
+            }
+            double xv[PER];
+#pragma unroll
+            for (int u = 0; u < PER; ++u) xv[u] = (tid + u * BLOCK < nz) ? ld_x(x, c[u]) : 0.0;
+#pragma unroll
+            for (int u = 0; u < PER; ++u) {
+                const int i = tid + u * BLOCK;
+                if (i < nz) S.val[off + i] = v[u] * xv[u];
+            }
+        }
+        __syncthreads();
+        // phase 2
+        if (it.y >= 0 && !(it.y & kStreamVecFlag)) {
+            const int r0 = it.x, r1 = it.y, roff = r0 - (r0 & ~3);
+            for (int r = tid; r < r1 - r0; r += BLOCK) {
+                const int s = S.rp[roff + r] - k0a, e = S.rp[roff + r + 1] - k0a;
+                double acc = +0.0;
+                for (int k = s; k < e; ++k) acc = acc + S.val[k];
+                y[r0 + r] = acc;
+            }
+        } else if (it.y >= 0) {
+            const int r0 = it.x, r1 = it.y & ~kStreamVecFlag, roff = r0 - (r0 & ~3);
+            const int lane = tid & 31, w = tid >> 5;
+            for (int r = w; r < r1 - r0; r += BLOCK / 32) {
+                const int s = S.rp[roff + r] - k0a, e = S.rp[roff + r + 1] - k0a;
+                double acc = 0.0;
+                for (int k = s + lane; k < e; k += 32) acc += S.val[k];
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+                if (lane == 0) y[r0 + r] = acc;
+            }
+        } else {
+            // long-row piece: deterministic block sum -> carry slot
+            double acc = 0.0;
+            for (int i = tid; i < nz; i += BLOCK) acc += S.val[off + i];
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+            if ((tid & 31) == 0) s_red[tid >> 5] = acc;
+            __syncthreads();
+            if (tid == 0) {
+                double t = 0.0;
+                for (int w = 0; w < BLOCK / 32; ++w) t += s_red[w];
+                carry[-it.y - 1] = t;
+            }
+        }
+        __syncthreads();   // stage j is free; make generic-proxy writes visible to the async proxy
+        if (tid == 0) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+}
+
+// y[row] = sum of its long-row pieces, in piece order
+__global__ void csr_stream_fixup_kernel(int nlong, const int4* __restrict__ longrows, const double* __restrict__ carry,
+                                        double* __restrict__ y) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nlong) return;
+    const int4 L = longrows[i];   // (row, first piece, end piece, -)
+    double s = 0.0;
+    for (int p = L.y; p < L.z; ++p) s += carry[p];
+    y[L.x] = s;
+}
+
+// =====================================================================
 // plan-time helpers
 // =====================================================================
 // validation + context statistics over the caller's int64 row pointer
@@ -390,19 +592,24 @@ __global__ void sell_keys_kernel(int nrows, const int* __restrict__ rp, int sigm
 }
 
 // sorted position r -> original row perm[r]; lengths + per-chunk max
+// chunk_len[c] = max length if all 32 rows exist and have that length, else -max
 __global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,
                                     int* __restrict__ rowlen, int* __restrict__ chunk_len) {
     const int r = blockIdx.x * blockDim.x + threadIdx.x;
     const int lane = threadIdx.x & 31;
-    int len = 0;
+    int len = -1;
     if (r < nrows) {
         const int o = perm ? perm[r] : r;
         len = rp[o + 1] - rp[o];
         rowlen[r] = len;
     }
-    int m = len;
-    for (int off = 16; off > 0; off >>= 1) m = max(m, __shfl_xor_sync(0xffffffffu, m, off));
-    if (lane == 0 && r < nrows) chunk_len[r >> 5] = m;
+    int mx = len, mn = len;
+    for (int off = 16; off > 0; off >>= 1) {
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+        mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, off));
+    }
+    mx = max(mx, 0);
+    if (lane == 0 && r < nrows) chunk_len[r >> 5] = (mn == mx) ? mx : -mx;
 }
 
 __global__ void sell_fill_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,

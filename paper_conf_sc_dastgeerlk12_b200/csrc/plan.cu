@@ -31,6 +31,12 @@ constexpr int kMergeBlock = 256;
 constexpr int kMergeIPT = 7;
 constexpr int kMergeTile = kMergeBlock * kMergeIPT;
 constexpr int kTimingRing = 64;
+// TMA CSR-stream: items of <= kStreamNB nonzeros / <= kStreamRMAX rows, kStreamStages-deep ring
+constexpr int kStreamBlock = 256;
+constexpr int kStreamStages = 3;
+constexpr int kStreamNB = 2048;
+constexpr int kStreamRMAX = 512;
+constexpr int kStreamVecMinLen = 64;   // items whose longest row exceeds this reduce warp-per-row
 
 struct Candidate {
     int32_t variant;
@@ -87,6 +93,12 @@ struct pepp_spmv_plan_s {
     int* d_carry_row = nullptr;
     double* d_carry_val = nullptr;
 
+    // TMA CSR-stream
+    int nitems = 0, nlong = 0, grid_stream = 0;
+    int4* d_items = nullptr;
+    int4* d_longrows = nullptr;
+    double* d_stream_carry = nullptr;
+
     // occupancy-derived grids
     int grid_csr[6] = {0};   // per log2(TPR)
     int grid_sell = 0;
@@ -139,7 +151,8 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (!p) return;
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
-                    p->d_scol, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy};
+                    p->d_scol, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
+                    p->d_items, p->d_longrows, p->d_stream_carry};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -177,7 +190,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
         int64_t slots = 0;
         std::vector<int64_t> cp(p->nchunks + 1);
-        for (int c = 0; c < p->nchunks; ++c) { cp[c] = slots; slots += (int64_t)cl[c] * 32; }
+        for (int c = 0; c < p->nchunks; ++c) { cp[c] = slots; slots += (int64_t)std::abs(cl[c]) * 32; }
         cp[p->nchunks] = slots;
         p->sell_slots = slots;
         *fill = p->nnz ? (double)slots / (double)p->nnz : 1.0;
@@ -246,6 +259,59 @@ pepp_status_t prepare_merge(pepp_spmv_plan_t* p, cudaStream_t st) {
     return PEPP_OK;
 }
 
+// ---------------------------------------------------------------- CSR-stream prep
+auto stream_kernel() { return pepp::k::csr_stream_tma_kernel<kStreamBlock, kStreamStages, kStreamNB, kStreamRMAX>; }
+constexpr size_t kStreamSmem = sizeof(pepp::k::StreamStage<kStreamNB, kStreamRMAX>) * kStreamStages;
+
+pepp_status_t prepare_stream(pepp_spmv_plan_t* p, cudaStream_t st) {
+    const int64_t R = p->nrows;
+    if (R == 0) return PEPP_OK;
+    std::vector<int> rp(R + 1);
+    PEPP_CUDA_TRY(cudaMemcpyAsync(rp.data(), p->d_rp, sizeof(int) * (R + 1), cudaMemcpyDeviceToHost, st));
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    std::vector<int4> items, longrows;
+    items.reserve((size_t)(p->nnz / kStreamNB + R / kStreamRMAX + 16));
+    int piece = 0;
+    int64_t r = 0;
+    while (r < R) {
+        const int len = rp[r + 1] - rp[r];
+        if (len > kStreamNB) {   // long row -> pieces of kStreamNB nonzeros
+            const int first_piece = piece;
+            for (int k = rp[r]; k < rp[r + 1]; k += kStreamNB, ++piece)
+                items.push_back(make_int4((int)r, -(piece + 1), k, std::min(k + kStreamNB, rp[r + 1])));
+            longrows.push_back(make_int4((int)r, first_piece, piece, 0));
+            ++r;
+            continue;
+        }
+        const int64_t r0 = r;
+        const int k0 = rp[r];
+        int maxlen = 0;
+        while (r < R && r - r0 < kStreamRMAX && rp[r + 1] - k0 <= kStreamNB) {
+            maxlen = std::max(maxlen, rp[r + 1] - rp[r]);
+            ++r;
+        }
+        const int flag = maxlen > kStreamVecMinLen ? pepp::k::kStreamVecFlag : 0;
+        items.push_back(make_int4((int)r0, (int)r | flag, k0, rp[r]));
+    }
+    p->nitems = (int)items.size();
+    p->nlong = (int)longrows.size();
+    pepp_status_t s;
+    if ((s = dalloc(p, &p->d_items, p->nitems))) return s;
+    PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_items, items.data(), sizeof(int4) * items.size(), cudaMemcpyHostToDevice, st));
+    if (p->nlong) {
+        if ((s = dalloc(p, &p->d_longrows, p->nlong))) return s;
+        if ((s = dalloc(p, &p->d_stream_carry, piece))) return s;
+        PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_longrows, longrows.data(), sizeof(int4) * longrows.size(), cudaMemcpyHostToDevice, st));
+    }
+    PEPP_CUDA_TRY(cudaFuncSetAttribute(stream_kernel(), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kStreamSmem));
+    int occ = 0;
+    PEPP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, stream_kernel(), kStreamBlock, kStreamSmem));
+    if (occ < 1) return PEPP_E_UNSUPPORTED;
+    p->grid_stream = (int)std::min<int64_t>((int64_t)p->sm_count * occ, p->nitems);
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    return PEPP_OK;
+}
+
 // ---------------------------------------------------------------- launches
 template <int TPR>
 void launch_csr_vector(const pepp_spmv_plan_t* p, const double* x, double* y, cudaStream_t st, int grid) {
@@ -271,6 +337,15 @@ pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const double* x, d
                 (int)p->nrows, p->d_rp, p->d_col, p->d_val, x, y, p->d_tile, p->d_carry_row, p->d_carry_val);
             pepp::k::merge_fixup_kernel<<<(p->ntiles + 255) / 256, 256, 0, st>>>(p->ntiles, (int)p->nrows,
                                                                                   p->d_carry_row, p->d_carry_val, y);
+        }
+        break;
+    case PEPP_V_CSR_STREAM:
+        if (p->nitems > 0) {
+            stream_kernel()<<<p->grid_stream, kStreamBlock, kStreamSmem, st>>>(
+                p->nitems, p->d_items, p->d_rp, p->d_col, p->d_val, x, y, p->d_stream_carry);
+            if (p->nlong)
+                pepp::k::csr_stream_fixup_kernel<<<(p->nlong + 127) / 128, 128, 0, st>>>(p->nlong, p->d_longrows,
+                                                                                        p->d_stream_carry, y);
         }
         break;
     case PEPP_V_SELL:
@@ -531,7 +606,8 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     // ---- a1: copy + narrow row_ptr, validate, context statistics ----
     pepp_status_t s;
     const int64_t nstore = p->pad + A->nnz + 8;   // + trailing zeros for aligned 4-groups
-    if ((s = dalloc(p, &p->d_rp, A->nrows + 1))) return s;
+    if ((s = dalloc(p, &p->d_rp, A->nrows + 1 + 8))) return s;   // +8: aligned 16-B bulk copies may overrun
+    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_rp, 0, sizeof(int) * (A->nrows + 1 + 8), st));
     if ((s = dalloc(p, &p->d_col, nstore))) return s;
     if ((s = dalloc(p, &p->d_val, nstore))) return s;
     PEPP_CUDA_TRY(cudaMemsetAsync(p->d_col, 0, sizeof(int) * nstore, st));
@@ -596,6 +672,10 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         p->cands.push_back({PEPP_V_SELL, p->sell_sigma});
     }
     if (mask & (1u << PEPP_V_MERGE_PATH)) { if ((s = prepare_merge(p, st))) return s; }
+    if (mask & (1u << PEPP_V_CSR_STREAM)) {
+        if ((s = prepare_stream(p, st))) return s;
+        p->cands.push_back({PEPP_V_CSR_STREAM, kStreamNB});
+    }
     p->eligible.assign(p->cands.size(), 1);
     p->pending.assign(p->cands.size(), 0);
     I.ncandidates = (int32_t)p->cands.size();

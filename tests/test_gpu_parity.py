@@ -62,7 +62,7 @@ def test_every_variant_matches_oracle(case):
     A, x, exact = CASES[case]()
     with pepp.Plan.from_csr(A) as plan:
         forces = _all_forces(plan)
-        assert {f.variant for f in forces} == {pepp.V_CSR_VECTOR, pepp.V_MERGE_PATH, pepp.V_SELL}
+        assert {f.variant for f in forces} == {pepp.V_CSR_VECTOR, pepp.V_MERGE_PATH, pepp.V_SELL, pepp.V_CSR_STREAM}
         for f in forces:
             y, used = _run(plan, x, force=f)
             assert (used.variant, used.param) == (f.variant, f.param)
@@ -150,7 +150,7 @@ def test_partition_invariance_bitwise_real():
     xd = _dev(x)
     with pepp.Plan.from_csr(A) as whole:
         for f in _all_forces(whole):
-            if f.variant != pepp.V_CSR_VECTOR:
+            if f.variant not in (pepp.V_CSR_VECTOR, pepp.V_CSR_STREAM):
                 continue   # merge tiles / SELL chunks depend on the block boundaries
             y1, _ = _run(whole, x, force=f)
             for P in (2, 3, 8):
@@ -162,6 +162,20 @@ def test_partition_invariance_bitwise_real():
                         pl.exec(xd, y[b[r]:b[r + 1]], force=f)
                 torch.cuda.synchronize()
                 assert np.array_equal(y.cpu().numpy(), y1)
+
+
+@pytest.mark.parametrize("case", ["lap64_real", "uniform_real", "banded_real"])
+def test_csr_stream_bit_identical_to_oracle_on_real_inputs(case):
+    """CSR-stream's stream items compute exactly the oracle's arithmetic
+    (rounded product, then ascending sequential sums from +0.0), so without
+    long rows its result equals the definition bit for bit, not just within
+    the bound."""
+    A, x, _ = CASES[case]()
+    assert int(np.diff(A.row_ptr).max()) <= 64
+    with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_CSR_STREAM) as plan:
+        y, used = _run(plan, x)
+        assert used.variant == pepp.V_CSR_STREAM
+        assert np.array_equal(y, oracle.spmv(A, x))
 
 
 def test_determinism_bitwise():
