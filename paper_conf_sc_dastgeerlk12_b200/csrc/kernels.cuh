@@ -60,6 +60,13 @@ __device__ __forceinline__ int ld_stream_i(const int* p, uint64_t pol) {
 }
 // x gather: read-only path, cached in L1 and L2 (reused across rows)
 __device__ __forceinline__ double ld_x(const double* __restrict__ x, int c) { return __ldg(x + c); }
+// same gather as volatile asm: a run of these is issued back-to-back in
+// program order (ptxas may not interleave the consumers between them)
+__device__ __forceinline__ double ld_x_ordered(const double* __restrict__ x, int c) {
+    double r;
+    asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(r) : "l"(x + c));
+    return r;
+}
 
 // =====================================================================
 // Variant 0: vector-CSR with TPR lanes per row (TPR in {2,4,8,16,32}).
@@ -357,12 +364,13 @@ __global__ void merge_tile_search_kernel(int nrows, int64_t nnz, const int* __re
 // ring with cp.async.bulk (completion counted on an mbarrier per stage),
 // so STAGES-1 items are in flight while the CTA computes the current one:
 //   phase 1 (balanced over nonzeros): sval[k] <- val[k] * x[col[k]]
-//   phase 2 (per row): stream items: one thread per row sums its products
-//           sequentially from +0.0 — the oracle's exact arithmetic (product
-//           rounded, then each sum rounded, ascending k), so results are
-//           bit-identical to the definition; vector items (long rows): one
-//           warp per row, shuffle tree; long-row pieces: a block-wide sum
-//           written to a carry slot, combined by csr_stream_fixup_kernel.
+//   phase 2 (per row): rows of <= VEC entries: one thread sums the row's
+//           products sequentially from +0.0 — the oracle's exact arithmetic
+//           (product rounded, then each sum rounded, ascending k), so those
+//           rows are bit-identical to the definition; rows of VEC..NB
+//           entries: one warp per row, lane-strided + shuffle tree; rows
+//           longer than NB: NB-sized pieces, each a block-wide sum written to
+//           a carry slot, combined in piece order by csr_stream_fixup_kernel.
 // =====================================================================
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -385,7 +393,7 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
                  ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
 }
 
-constexpr int kStreamVecFlag = 0x40000000;   // item.y flag: warp-per-row reduction
+constexpr int kStreamVecFlag = 0x40000000;   // item.y flag: the item holds a row longer than VEC
 
 template <int NB, int RMAX>
 struct StreamStage {
@@ -394,7 +402,7 @@ struct StreamStage {
     int rp[RMAX + 8];
 };
 
-template <int BLOCK, int STAGES, int NB, int RMAX>
+template <int BLOCK, int STAGES, int NB, int RMAX, int VEC>
 __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const int4* __restrict__ items,
                                                                const int* __restrict__ rp,
                                                                const int* __restrict__ col,
@@ -468,7 +476,7 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
             }
             double xv[PER];
 #pragma unroll
-            for (int u = 0; u < PER; ++u) xv[u] = (tid + u * BLOCK < nz) ? ld_x(x, c[u]) : 0.0;
+            for (int u = 0; u < PER; ++u) xv[u] = (tid + u * BLOCK < nz) ? ld_x_ordered(x, c[u]) : 0.0;
 #pragma unroll
             for (int u = 0; u < PER; ++u) {
                 const int i = tid + u * BLOCK;
@@ -476,25 +484,31 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
             }
         }
         __syncthreads();
-        // phase 2
-        if (it.y >= 0 && !(it.y & kStreamVecFlag)) {
-            const int r0 = it.x, r1 = it.y, roff = r0 - (r0 & ~3);
+        // phase 2: the reduction order is a property of the row alone (not of
+        // the item it landed in), so results do not depend on item or rank
+        // boundaries: rows of <= VEC entries are summed sequentially by one
+        // thread (the oracle's order); longer rows lane-strided by a warp.
+        if (it.y >= 0) {
+            const bool has_long = (it.y & kStreamVecFlag) != 0;
+            const int r0 = it.x, r1 = it.y & ~kStreamVecFlag, roff = r0 - (r0 & ~3);
             for (int r = tid; r < r1 - r0; r += BLOCK) {
                 const int s = S.rp[roff + r] - k0a, e = S.rp[roff + r + 1] - k0a;
+                if (e - s > VEC) continue;
                 double acc = +0.0;
                 for (int k = s; k < e; ++k) acc = acc + S.val[k];
                 y[r0 + r] = acc;
             }
-        } else if (it.y >= 0) {
-            const int r0 = it.x, r1 = it.y & ~kStreamVecFlag, roff = r0 - (r0 & ~3);
-            const int lane = tid & 31, w = tid >> 5;
-            for (int r = w; r < r1 - r0; r += BLOCK / 32) {
-                const int s = S.rp[roff + r] - k0a, e = S.rp[roff + r + 1] - k0a;
-                double acc = 0.0;
-                for (int k = s + lane; k < e; k += 32) acc += S.val[k];
+            if (has_long) {
+                const int lane = tid & 31, w = tid >> 5;
+                for (int r = w; r < r1 - r0; r += BLOCK / 32) {
+                    const int s = S.rp[roff + r] - k0a, e = S.rp[roff + r + 1] - k0a;
+                    if (e - s <= VEC) continue;
+                    double acc = 0.0;
+                    for (int k = s + lane; k < e; k += 32) acc += S.val[k];
 #pragma unroll
-                for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-                if (lane == 0) y[r0 + r] = acc;
+                    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+                    if (lane == 0) y[r0 + r] = acc;
+                }
             }
         } else {
             // long-row piece: deterministic block sum -> carry slot

@@ -33,7 +33,7 @@ constexpr int kMergeTile = kMergeBlock * kMergeIPT;
 constexpr int kTimingRing = 64;
 // TMA CSR-stream: items of <= kStreamNB nonzeros / <= kStreamRMAX rows, kStreamStages-deep ring
 constexpr int kStreamBlock = 256;
-constexpr int kStreamStages = 3;
+constexpr int kStreamStages = 2;   // 2 x 26.7 KB per CTA -> 4 CTAs (32 warps) per SM
 constexpr int kStreamNB = 2048;
 constexpr int kStreamRMAX = 512;
 constexpr int kStreamVecMinLen = 64;   // items whose longest row exceeds this reduce warp-per-row
@@ -260,7 +260,7 @@ pepp_status_t prepare_merge(pepp_spmv_plan_t* p, cudaStream_t st) {
 }
 
 // ---------------------------------------------------------------- CSR-stream prep
-auto stream_kernel() { return pepp::k::csr_stream_tma_kernel<kStreamBlock, kStreamStages, kStreamNB, kStreamRMAX>; }
+auto stream_kernel() { return pepp::k::csr_stream_tma_kernel<kStreamBlock, kStreamStages, kStreamNB, kStreamRMAX, kStreamVecMinLen>; }
 constexpr size_t kStreamSmem = sizeof(pepp::k::StreamStage<kStreamNB, kStreamRMAX>) * kStreamStages;
 
 pepp_status_t prepare_stream(pepp_spmv_plan_t* p, cudaStream_t st) {

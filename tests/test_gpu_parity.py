@@ -164,18 +164,21 @@ def test_partition_invariance_bitwise_real():
                 assert np.array_equal(y.cpu().numpy(), y1)
 
 
-@pytest.mark.parametrize("case", ["lap64_real", "uniform_real", "banded_real"])
-def test_csr_stream_bit_identical_to_oracle_on_real_inputs(case):
-    """CSR-stream's stream items compute exactly the oracle's arithmetic
-    (rounded product, then ascending sequential sums from +0.0), so without
-    long rows its result equals the definition bit for bit, not just within
-    the bound."""
+@pytest.mark.parametrize("case", ["lap64_real", "uniform_real", "zipf_real", "banded_real"])
+def test_csr_stream_bit_identical_to_oracle_on_short_rows(case):
+    """CSR-stream sums every row of <= 64 entries with exactly the oracle's
+    arithmetic (rounded product, then ascending sequential sums from +0.0),
+    so those rows equal the definition bit for bit, not just within the
+    bound; longer rows (warp-strided order) stay within the bound."""
     A, x, _ = CASES[case]()
-    assert int(np.diff(A.row_ptr).max()) <= 64
     with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_CSR_STREAM) as plan:
         y, used = _run(plan, x)
         assert used.variant == pepp.V_CSR_STREAM
-        assert np.array_equal(y, oracle.spmv(A, x))
+    yr = oracle.spmv(A, x)
+    short = np.diff(A.row_ptr) <= 64
+    assert np.array_equal(y[short], yr[short])
+    b = oracle.bound(A, x)
+    assert np.all(np.abs(y - yr) <= b)
 
 
 def test_determinism_bitwise():
