@@ -17,7 +17,7 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 
 def main(paths):
     for p in paths:
-        out = subprocess.run(["ncu", "-i", p, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+        out = subprocess.run(["ncu", "-i", p, "--page", "raw", "--csv", "--print-units", "base"], capture_output=True, text=True).stdout
         rows = list(csv.reader(out.splitlines()))
         if not rows:
             continue
