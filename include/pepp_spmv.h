@@ -209,6 +209,15 @@ pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_choice_t* out);
 pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const double* x, double* y, int flags,
                              void* stream, const pepp_choice_t* force, pepp_choice_t* used);
 
+/* The exchange step alone: make this rank's rows of y
+   usable by the other ranks' next call, on `stream`. flags as in
+   pepp_spmv_exec (PEPP_Y_NEXT_INPUT: the plan's exchange, halo or
+   allgatherv; PEPP_Y_REPLICATED: allgatherv). y: READWRITE device buffer,
+   global length; own rows are read, other rows written. exec(flags) ==
+   exec(PEPP_Y_LOCAL) followed by exchange(flags). A no-op when nranks == 1.
+   Errors: PEPP_E_INVALID, PEPP_E_NCCL, PEPP_E_CUDA. */
+pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, double* y, int flags, void* stream);
+
 /* Host-buffer entry point (the paper's measurement setting, where operand
    transfers are part of the call: Fig. 5 "communication overhead of copying
    data back and forth to device memory is also included", P@35591–35720).

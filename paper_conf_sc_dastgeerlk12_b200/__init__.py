@@ -131,6 +131,10 @@ class Plan:
                 "pepp_spmv_exec")
         return Choice._from(used)
 
+    def exchange(self, y, flags: int = Y_NEXT_INPUT, stream=None) -> None:
+        """The exchange step alone (no-op on an unpartitioned plan)."""
+        C.check(C.lib().pepp_spmv_exchange(self._h, _ptr(y), flags, _stream_handle(stream)), "pepp_spmv_exchange")
+
     def exec_host(self, x_host: np.ndarray, y_host: np.ndarray, iterations: int = 1, flags: int = Y_LOCAL,
                   stream=None) -> None:
         """Host buffers in and out, transfers inside the call (synchronous)."""

@@ -826,17 +826,31 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const doub
             (void)cudaGetLastError();
         }
     }
+    ch.exchange = PEPP_X_NONE;
     if (p->opts.nranks > 1 && (flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED))) {
-        const bool ag = (flags & PEPP_Y_REPLICATED) || ch.exchange == PEPP_X_ALLGATHER;
-        s = ag ? exchange_allgather(p, y, st) : exchange_halo(p, y, st);
+        const bool ag = (flags & PEPP_Y_REPLICATED) || p->exchange == PEPP_X_ALLGATHER;
+        const int ex = (force && (force->exchange == PEPP_X_ALLGATHER || force->exchange == PEPP_X_HALO))
+                           ? force->exchange : (ag ? PEPP_X_ALLGATHER : PEPP_X_HALO);
+        s = ex == PEPP_X_ALLGATHER ? exchange_allgather(p, y, st) : exchange_halo(p, y, st);
         if (s) { p->sticky = s; return s; }
-        ch.exchange = ag ? PEPP_X_ALLGATHER : PEPP_X_HALO;
-    } else {
-        ch.exchange = PEPP_X_NONE;
+        ch.exchange = ex;
     }
     ++p->ncalls;
     if (used) *used = ch;
     return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, double* y, int flags, void* stream) {
+    if (!p) return PEPP_E_INVALID;
+    if (p->sticky) return p->sticky;
+    if (p->opts.nranks == 1 || !(flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED))) return PEPP_OK;
+    if (!y) return PEPP_E_INVALID;
+    if (cudaSetDevice(p->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    cudaStream_t st = (cudaStream_t)stream;
+    const bool ag = (flags & PEPP_Y_REPLICATED) || p->exchange == PEPP_X_ALLGATHER;
+    pepp_status_t s = ag ? exchange_allgather(p, y, st) : exchange_halo(p, y, st);
+    if (s) p->sticky = s;
+    return s;
 }
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const double* x_host, double* y_host,
