@@ -45,6 +45,8 @@ WORKLOADS = {
                    iters=20, iterated=False),
     "lap64": dict(desc="BASELINE config 1: 2D 5-point Laplacian 64x64 (4096 rows, 20224 nnz), fp64",
                   iters=1000, iterated=False),
+    "skew": dict(desc="heavy-tailed rows (not a BASELINE config): P(k)~k^-2, k<=4M, 4M x 4M, fp64 — rows up to ~1e6 nnz",
+                 iters=20, iterated=False),
 }
 
 
@@ -59,6 +61,8 @@ def make_block(workload: str, r0: int, r1: int):
         return gen.uniform(1 << 20, 1 << 20, 16, seed=42, r0=r0, r1=r1)
     if workload == "zipf4m":
         return gen.zipf(4 << 20, 4 << 20, seed=46, r0=r0, r1=r1)
+    if workload == "skew":
+        return gen.zipf(4 << 20, 4 << 20, seed=50, alpha=2.0, kmax=4 << 20, r0=r0, r1=r1)
     raise ValueError(workload)
 
 
@@ -73,6 +77,8 @@ def global_rowptr(workload: str) -> np.ndarray:
         return rp
     if workload == "uniform1m":
         return np.arange(0, ((1 << 20) + 1) * 16, 16, dtype=np.int64)
+    if workload == "skew":
+        return gen._rowptr_global(1, 50, 4 << 20, 4 << 20, 2.0, 4 << 20, 0, 4 << 20)
     return gen._rowptr_global(1, 46, 4 << 20, 4 << 20, 1.5, 435, 0, 4 << 20)
 
 
@@ -267,11 +273,14 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
                 a, b = ev_pool[k]
                 if record:
                     a.record(stream)
-                u = plan.exec(src, dst, flags=flags, stream=stream, force=force)
+                # kernel (events bracket it alone), then the exchange step
+                u = plan.exec(src, dst, flags=pepp.Y_LOCAL, stream=stream, force=force)
                 if record:
                     b.record(stream)
                     used_count[u.name] = used_count.get(u.name, 0) + 1
                     launches["n"] += 2 if u.variant == pepp.V_MERGE_PATH else 1
+                if flags != pepp.Y_LOCAL and world > 1:
+                    plan.exchange(dst, flags, stream=stream)
                 if iterated:
                     src = dst
         return kernel_ms

@@ -131,6 +131,11 @@ typedef struct {
     const void* nccl_unique_id; /* 128-byte ncclUniqueId (same on every rank) when nccl_comm is NULL and nranks > 1 */
     int32_t exchange;         /* pepp_exchange_t; AUTO = halo when ghosts are < 1/4 of ncols, else allgather */
     const char* history_path; /* if set: history loaded at plan, saved at destroy (NEXT-f2 persistence) */
+    int32_t prune;            /* 1 (default) = multi-stage composition (P@10489): statically narrow the
+                                 candidates from the context instance before the runtime choice —
+                                 vector-CSR only if max_row <= max(4096, 256*mean), SELL only if
+                                 max_row <= max(256, 16*mean); merge-path and CSR-stream always.
+                                 0 = every variant is a candidate (variant_mask still applies). */
 } pepp_spmv_opts_t;
 
 /* Selection result. `candidate` indexes pepp_spmv_candidates(). */
@@ -284,10 +289,15 @@ pepp_status_t pepp_history_destroy(pepp_history* h);
 pepp_status_t pepp_history_record(pepp_history* h, uint64_t key, int32_t cand, double us);
 pepp_status_t pepp_history_stats(const pepp_history* h, uint64_t key, int32_t cand,
                                  int64_t* count, double* mean_us, double* m2);
-/* Policy (reading A10): among candidates with eligible[c] != 0, if any has
-   fewer than min_samples records, return the lowest such c with
-   *calibrating = 1; else return argmin mean time, ties within 1 % going to
-   the lower index, *calibrating = 0. *predicted_us = that candidate's mean. */
+/* Policy (reading A10): calibration runs in rounds r = 1..min_samples —
+   the lowest eligible candidate with fewer than r records is returned with
+   *calibrating = 1, except that a candidate whose samples already average
+   more than 4x the best mean seen so far is not sampled again (early
+   abandonment: one sample rules it out). When every candidate is
+   calibrated or abandoned, return argmin mean time, ties within 1 % going
+   to the lower index, *calibrating = 0. *predicted_us = that candidate's
+   mean. (pepp_spmv_exec applies the same policy and also counts timed calls
+   still in flight.) */
 pepp_status_t pepp_history_select(const pepp_history* h, uint64_t key, int32_t ncand,
                                   const uint8_t* eligible, int32_t min_samples,
                                   int32_t* cand, int32_t* calibrating, double* predicted_us);

@@ -31,7 +31,7 @@ class OPTS_T(ctypes.Structure):
     _fields_ = [("variant_mask", c_u32), ("use_history", c_i32), ("validate", c_i32), ("sell_sigma", c_i32),
                 ("device", c_i32), ("min_samples", c_i32), ("sample_period", c_i32), ("nranks", c_i32),
                 ("rank", c_i32), ("row_bounds", c_vp), ("nccl_comm", c_vp), ("nccl_unique_id", c_vp),
-                ("exchange", c_i32), ("history_path", ctypes.c_char_p)]
+                ("exchange", c_i32), ("history_path", ctypes.c_char_p), ("prune", c_i32)]
 
 
 class CHOICE_T(ctypes.Structure):

@@ -49,6 +49,7 @@ extern "C" PEPP_API void pepp_spmv_opts_default(pepp_spmv_opts_t* o) {
     o->nccl_unique_id = nullptr;
     o->exchange = PEPP_X_AUTO;
     o->history_path = nullptr;
+    o->prune = 1;
 }
 
 // ---------------------------------------------------------------- partition
@@ -141,16 +142,34 @@ const Welford* history_get(const pepp_history* h, uint64_t key, int32_t cand) {
     return it == h->table.end() ? nullptr : &it->second;
 }
 
-int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible,
-                     int32_t min_samples, int32_t* calibrating, double* predicted_us) {
-    // 1) calibration: the lowest eligible candidate with too few samples
+double history_best_mean(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible) {
+    double best = -1.0;
     for (int32_t c = 0; c < ncand; ++c) {
         if (!eligible[c]) continue;
         const Welford* w = history_get(h, key, c);
-        if (!w || w->count < min_samples) {
-            *calibrating = 1;
-            *predicted_us = w ? w->mean : 0.0;
-            return c;
+        if (w && w->count > 0 && (best < 0 || w->mean < best)) best = w->mean;
+    }
+    return best;
+}
+
+bool history_abandoned(const Welford* w, double best_mean) {
+    return w && w->count > 0 && best_mean > 0 && w->mean > kAbandonFactor * best_mean;
+}
+
+int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible,
+                     int32_t min_samples, int32_t* calibrating, double* predicted_us) {
+    const double best_mean = history_best_mean(h, key, ncand, eligible);
+    // 1) calibration in rounds: round r gives every candidate its r-th sample
+    //    (lowest index first), skipping candidates already ruled out
+    for (int32_t r = 1; r <= min_samples; ++r) {
+        for (int32_t c = 0; c < ncand; ++c) {
+            if (!eligible[c]) continue;
+            const Welford* w = history_get(h, key, c);
+            if ((!w || w->count < r) && !history_abandoned(w, best_mean)) {
+                *calibrating = 1;
+                *predicted_us = w ? w->mean : 0.0;
+                return c;
+            }
         }
     }
     // 2) exploitation: argmin of the mean, ties within 1 % -> lower index (A10)
@@ -158,7 +177,9 @@ int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const u
     double best_t = 0.0;
     for (int32_t c = 0; c < ncand; ++c) {
         if (!eligible[c]) continue;
-        const double t = history_get(h, key, c)->mean;
+        const Welford* w = history_get(h, key, c);
+        if (!w || w->count == 0) continue;
+        const double t = w->mean;
         if (best < 0 || t < best_t * 0.99) { best = c; best_t = t; }
     }
     *calibrating = 0;

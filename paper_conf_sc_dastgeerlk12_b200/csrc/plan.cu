@@ -419,18 +419,28 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out) {
         const int32_t ms = std::max(1, p->opts.min_samples);
         const int32_t n = (int32_t)p->cands.size();
         cand = -1;
-        bool waiting = false;
-        for (int32_t c = 0; c < n; ++c) {
-            if (!p->eligible[c]) continue;
-            const pepp::Welford* w = pepp::history_get(p->hist, p->key, c);
-            const int64_t done = w ? w->count : 0;
-            if (done + p->pending[c] < ms) { cand = c; calibrating = 1; pred = w ? w->mean : 0.0; break; }
-            if (done < ms) waiting = true;
+        for (int32_t r = 1; r <= ms && cand < 0; ++r) {
+            // round r: every candidate not yet ruled out gets its r-th timed call
+            // (calls still in flight count, so the host can run ahead of the GPU)
+            for (int pass = 0; pass < 2 && cand < 0; ++pass) {
+                const double best_mean = pepp::history_best_mean(p->hist, p->key, n, p->eligible.data());
+                bool waiting = false;
+                for (int32_t c = 0; c < n; ++c) {
+                    if (!p->eligible[c]) continue;
+                    const pepp::Welford* w = pepp::history_get(p->hist, p->key, c);
+                    if (pepp::history_abandoned(w, best_mean)) continue;
+                    const int64_t done = w ? w->count : 0;
+                    if (done + p->pending[c] < r) { cand = c; calibrating = 1; pred = w ? w->mean : 0.0; break; }
+                    if (done < r) waiting = true;
+                }
+                // the round is fully issued but not measured: wait for it once, so
+                // the next round can rule out candidates from their timings
+                if (cand < 0 && waiting) harvest(p, true);
+                else break;
+            }
         }
-        if (cand < 0) {
-            if (waiting) harvest(p, true);
+        if (cand < 0)
             cand = pepp::history_pick(p->hist, p->key, n, p->eligible.data(), ms, &calibrating, &pred);
-        }
     } else {
         cand = heuristic_candidate(p);
     }
@@ -663,7 +673,16 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     I.algorithmic_bytes = A->nnz * 12 + (A->nrows + 1) * 4 + A->ncols * 8 + A->nrows * 8;
 
     // ---- a3: candidates + variant preparation ----
-    const uint32_t mask = o->variant_mask ? o->variant_mask : 0xffffffffu;
+    // multi-stage composition (P@10489): static narrowing from the context
+    // instance, then the runtime's history-based choice among the rest
+    uint32_t mask = o->variant_mask ? o->variant_mask : 0xffffffffu;
+    if (o->prune) {
+        const double mean = I.mean_row;
+        uint32_t keep = mask;
+        if ((double)I.max_row > std::max(4096.0, 256.0 * mean)) keep &= ~(1u << PEPP_V_CSR_VECTOR);
+        if ((double)I.max_row > std::max(256.0, 16.0 * mean)) keep &= ~(1u << PEPP_V_SELL);
+        if (keep & ((1u << PEPP_V_COUNT) - 1)) mask = keep;   // never prune everything
+    }
     if (mask & (1u << PEPP_V_CSR_VECTOR))
         for (int tpr : {2, 4, 8, 16, 32}) p->cands.push_back({PEPP_V_CSR_VECTOR, tpr});
     if (mask & (1u << PEPP_V_MERGE_PATH)) p->cands.push_back({PEPP_V_MERGE_PATH, kMergeIPT});

@@ -63,7 +63,7 @@ int main(void) {
   printf("csr %zu\nopts %zu\nchoice %zu\ninfo %zu\n", sizeof(pepp_csr_t), sizeof(pepp_spmv_opts_t),
          sizeof(pepp_choice_t), sizeof(pepp_plan_info_t));
   P(pepp_csr_t, on_device) P(pepp_spmv_opts_t, row_bounds) P(pepp_spmv_opts_t, exchange)
-  P(pepp_spmv_opts_t, history_path) P(pepp_choice_t, predicted_us) P(pepp_plan_info_t, key)
+  P(pepp_spmv_opts_t, history_path) P(pepp_spmv_opts_t, prune) P(pepp_choice_t, predicted_us) P(pepp_plan_info_t, key)
   P(pepp_plan_info_t, sell_fill) P(pepp_plan_info_t, halo_send)
   return 0;
 }
@@ -82,6 +82,7 @@ int main(void) {
     assert int(vals["pepp_spmv_opts_t.row_bounds"]) == C.OPTS_T.row_bounds.offset
     assert int(vals["pepp_spmv_opts_t.exchange"]) == C.OPTS_T.exchange.offset
     assert int(vals["pepp_spmv_opts_t.history_path"]) == C.OPTS_T.history_path.offset
+    assert int(vals["pepp_spmv_opts_t.prune"]) == C.OPTS_T.prune.offset
     assert int(vals["pepp_choice_t.predicted_us"]) == C.CHOICE_T.predicted_us.offset
     assert int(vals["pepp_plan_info_t.key"]) == C.INFO_T.key.offset
     assert int(vals["pepp_plan_info_t.sell_fill"]) == C.INFO_T.sell_fill.offset

@@ -60,7 +60,7 @@ CASES = {
 @pytest.mark.parametrize("case", sorted(CASES))
 def test_every_variant_matches_oracle(case):
     A, x, exact = CASES[case]()
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         forces = _all_forces(plan)
         assert {f.variant for f in forces} == {pepp.V_CSR_VECTOR, pepp.V_MERGE_PATH, pepp.V_SELL, pepp.V_CSR_STREAM}
         for f in forces:
@@ -112,7 +112,7 @@ EDGE = _edge_cases()
 def test_edge_cases_bitwise(name):
     A = EDGE[name]
     x = gen.vector(11, gen.INT8, A.ncols)
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         for f in _all_forces(plan):
             y, _ = _run(plan, x, force=f)
             _check(A, x, y, exact=True)
@@ -122,7 +122,7 @@ def test_edge_cases_bitwise(name):
 
 def test_empty_matrix_plan_and_exec():
     A = _hand(0, 10, [])
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         x = torch.ones(10, dtype=torch.float64, device="cuda")
         y = torch.empty(0, dtype=torch.float64, device="cuda")
         for f in _all_forces(plan):
@@ -136,7 +136,7 @@ def test_first_offset_any_alignment(first):
     Ar = gen.rebase(A, first)
     x = gen.vector(3, gen.INT8, 20_000)
     yr = oracle.spmv(A, x)
-    with pepp.Plan.from_csr(Ar) as plan:
+    with pepp.Plan.from_csr(Ar, prune=False) as plan:
         for f in _all_forces(plan):
             y, _ = _run(plan, x, force=f)
             assert np.array_equal(y, yr)
@@ -148,7 +148,7 @@ def test_partition_invariance_bitwise_real():
     A = gen.zipf(40_000, 40_000, seed=46)
     x = gen.vector(49, gen.REAL, 40_000)
     xd = _dev(x)
-    with pepp.Plan.from_csr(A) as whole:
+    with pepp.Plan.from_csr(A, prune=False) as whole:
         for f in _all_forces(whole):
             if f.variant not in (pepp.V_CSR_VECTOR, pepp.V_CSR_STREAM):
                 continue   # merge tiles / SELL chunks depend on the block boundaries
@@ -184,7 +184,7 @@ def test_csr_stream_bit_identical_to_oracle_on_short_rows(case):
 def test_determinism_bitwise():
     A = gen.zipf(50_000, 50_000, seed=46)
     x = gen.vector(49, gen.REAL, 50_000)
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         for f in _all_forces(plan):
             y1, _ = _run(plan, x, force=f)
             y2, _ = _run(plan, x, force=f)
@@ -194,7 +194,7 @@ def test_determinism_bitwise():
 def test_power_of_two_scaling_bitwise():
     A = gen.uniform(20_000, 20_000, 16, seed=42)
     x = gen.vector(45, gen.REAL, 20_000)
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         for f in _all_forces(plan):
             y, _ = _run(plan, x, force=f)
             y8, _ = _run(plan, x * 8.0, force=f)
@@ -204,7 +204,8 @@ def test_power_of_two_scaling_bitwise():
 def test_device_resident_operand_and_host_operand_agree():
     A = gen.zipf(10_000, 10_000, seed=46, val_mode=gen.INT4)
     x = gen.vector(3, gen.INT8, 10_000)
-    with pepp.Plan.from_csr(A) as ph, pepp.Plan(A.nrows, A.ncols, _dev(A.row_ptr), _dev(A.col), _dev(A.val)) as pd:
+    with pepp.Plan.from_csr(A, prune=False) as ph, \
+            pepp.Plan(A.nrows, A.ncols, _dev(A.row_ptr), _dev(A.col), _dev(A.val), prune=False) as pd:
         for f in _all_forces(ph):
             assert np.array_equal(_run(ph, x, force=f)[0], _run(pd, x, force=f)[0])
 
@@ -214,7 +215,7 @@ def test_iterated_laplacian_integer_bitwise_k16():
     A = gen.laplacian2d(n)
     x0 = gen.vector(3, gen.INT8, n * n)
     ref = oracle.iterate(A, x0, 16)
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         for f in _all_forces(plan):
             a = _dev(x0)
             b = torch.empty_like(a)
@@ -231,7 +232,7 @@ def test_iterated_real_within_propagated_bound():
     x0 = gen.vector(4, gen.REAL, n * n)
     xK, zK = oracle.iterate(A, x0, K, with_bound=True)
     bnd = oracle.iterate_bound(A, zK, K)
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         for f in _all_forces(plan):
             a = _dev(x0)
             b = torch.empty_like(a)
@@ -247,7 +248,7 @@ def test_exec_host_matches_device_path():
     x = gen.vector(3, gen.INT8, 10_000)
     ref1 = oracle.spmv(A, x)
     ref5 = oracle.iterate(A, x, 5)
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         y = np.empty(10_000)
         plan.exec_host(x, y, iterations=1)
         assert np.array_equal(y, ref1)
@@ -260,14 +261,17 @@ def test_selector_calibrates_then_picks_fastest_measured():
     A = gen.uniform(200_000, 200_000, 16, seed=42)
     x = _dev(gen.vector(45, gen.REAL, 200_000))
     y = torch.empty(200_000, dtype=torch.float64, device="cuda")
-    with pepp.Plan.from_csr(A, min_samples=3) as plan:
+    with pepp.Plan.from_csr(A, min_samples=3, prune=False) as plan:
         n = len(plan.candidates())
         seen = []
-        for _ in range(3 * n):
+        for _ in range(10 * n):
             u = plan.exec(x, y)
-            assert u.calibrating
+            if not u.calibrating:
+                break
             seen.append(u.candidate)
-        assert sorted(set(seen)) == list(range(n))
+        # round 1 visits every candidate; later rounds skip the ones ruled out
+        assert seen[:n] == list(range(n))
+        assert len(seen) <= 3 * n
         plan.flush_history()
         means = [plan.history_stats(c)[1] for c in range(n)]
         ch = plan.select()
@@ -295,7 +299,7 @@ def test_variant_mask_and_static_heuristic():
 
 def test_error_codes():
     A = gen.laplacian2d(16)
-    with pepp.Plan.from_csr(A) as plan:
+    with pepp.Plan.from_csr(A, prune=False) as plan:
         x = torch.ones(256, dtype=torch.float64, device="cuda")
         with pytest.raises(pepp.PeppError) as e:
             plan.exec(x, x)                       # x and y alias
@@ -315,3 +319,35 @@ def test_error_codes():
     bad = gen.laplacian2d(16)
     with pytest.raises(pepp.PeppError):           # row_ptr[nrows] - first != nnz
         pepp.Plan(bad.nrows, bad.ncols, bad.row_ptr, bad.col[:-1], bad.val[:-1])
+
+
+def test_select_overhead_within_paper_budget():
+    """pepp_spmv_select is host-only and must fit the runtime's per-task
+    overhead the paper quotes: < 2 us (P@40366-40402). Measured through
+    ctypes, so the C call itself is cheaper still."""
+    import ctypes
+    import time
+    A = gen.laplacian2d(64)
+    with pepp.Plan.from_csr(A, prune=False) as plan:
+        L = pepp._capi.lib()
+        c = pepp._capi.CHOICE_T()
+        ref = ctypes.byref(c)
+        h = plan._h
+        for _ in range(1000):
+            L.pepp_spmv_select(h, ref)
+        n = 20000
+        t = time.perf_counter()
+        for _ in range(n):
+            L.pepp_spmv_select(h, ref)
+        per_call_us = (time.perf_counter() - t) / n * 1e6
+        assert per_call_us < 2.0, per_call_us
+
+
+def test_exchange_is_noop_unpartitioned():
+    A = gen.laplacian2d(16)
+    with pepp.Plan.from_csr(A, prune=False) as plan:
+        y = torch.zeros(256, dtype=torch.float64, device="cuda")
+        plan.exchange(y, pepp.Y_NEXT_INPUT)
+        plan.exchange(y, pepp.Y_REPLICATED)
+        torch.cuda.synchronize()
+        assert torch.all(y == 0)

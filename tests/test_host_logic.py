@@ -85,8 +85,8 @@ def test_history_calibrates_then_exploits_argmin():
             break
         order.append(c)
         H.record(key, c, times[c])
-    # calibration visits each candidate min_samples times, lowest index first
-    assert order == [0, 0, 0, 1, 1, 1, 2, 2, 2, 3, 3, 3]
+    # calibration runs in rounds: every candidate once per round, lowest index first
+    assert order == [0, 1, 2, 3] * 3
     c, cal, pred = H.select(key, elig, min_samples=3)
     assert (c, cal) == (1, False) and pred == pytest.approx(3.0)
     # candidate 3 is 0.7 % slower: the tie rule keeps the lower index
@@ -95,6 +95,24 @@ def test_history_calibrates_then_exploits_argmin():
     assert H.select(key, [True, False, True, True])[0] == 3
     # other keys are independent (context instances)
     assert H.select(key + 1, elig) == (0, True, 0.0)
+
+
+def test_history_early_abandonment():
+    """A candidate > 4x slower than the best after round 1 is not sampled again."""
+    H = pepp.History()
+    key = 99
+    times = [10.0, 1.0, 300.0, 1.5]
+    order = []
+    for _ in range(100):
+        c, cal, _ = H.select(key, [True] * 4, min_samples=3)
+        if not cal:
+            break
+        order.append(c)
+        H.record(key, c, times[c])
+    # round 1 samples everyone; candidates 0 (10x) and 2 (300x) are then dropped
+    assert order == [0, 1, 2, 3, 1, 3, 1, 3]
+    assert H.select(key, [True] * 4)[:2] == (1, False)
+    assert H.stats(key, 2)[0] == 1 and H.stats(key, 0)[0] == 1
 
 
 def test_history_tracks_drift_and_welford():
