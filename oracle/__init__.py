@@ -49,6 +49,8 @@ def lib():
         L.oracle_spmv_row.argtypes = [i64, i64, p, p, p, p]
         L.oracle_spmv_row.restype = ctypes.c_double
         L.oracle_abs_rowsum.argtypes = [i64, i64, p, p, p, p, p]
+        L.oracle_abs_row.argtypes = [i64, i64, p, p, p, p]
+        L.oracle_abs_row.restype = ctypes.c_double
         L.oracle_spmv_iterate.argtypes = [i64, i64, i64, p, p, p, p, p, p, p]
         L.oracle_partition_nnz.argtypes = [i64, i64, p, i64, p]
         _lib = L
@@ -100,6 +102,19 @@ def spmv_rows(A, x, rows) -> np.ndarray:
     first = int(rp[0])
     return np.array([L.oracle_spmv_row(int(i), first, _ptr(rp), _ptr(c), _ptr(v), _ptr(xx))
                      for i in rows], dtype=np.float64)
+
+
+def bound_rows(A, x, rows) -> np.ndarray:
+    """The per-row tolerance of `bound` for sampled rows only."""
+    rp, c, v = _args(A.row_ptr, A.col, A.val)
+    xx = _c(x, np.float64)
+    L = lib()
+    first = int(rp[0])
+    out = np.empty(len(rows))
+    for j, i in enumerate(rows):
+        n = int(rp[i + 1] - rp[i])
+        out[j] = 2.0 * n * 2.0 ** -52 * L.oracle_abs_row(int(i), first, _ptr(rp), _ptr(c), _ptr(v), _ptr(xx))
+    return out
 
 
 def abs_rowsum(A, x) -> np.ndarray:

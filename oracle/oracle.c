@@ -79,6 +79,15 @@ ORACLE_EXPORT double oracle_spmv_row(int64_t i, int64_t first, const int64_t* ro
     return acc;
 }
 
+/* S_i for one row i (sampled bound checks at full size) */
+ORACLE_EXPORT double oracle_abs_row(int64_t i, int64_t first, const int64_t* row_ptr,
+                                    const int32_t* col, const double* val, const double* x) {
+    double acc = 0.0;
+    for (int64_t k = row_ptr[i] - first; k < row_ptr[i + 1] - first; ++k)
+        acc = acc + fabs(val[k]) * fabs(x[col[k]]);
+    return acc;
+}
+
 /* S_i = sum |a_ik| |x_col|  (bound ingredient, P6) */
 ORACLE_EXPORT void oracle_abs_rowsum(int64_t nrows, int64_t first, const int64_t* row_ptr,
                                      const int32_t* col, const double* val,

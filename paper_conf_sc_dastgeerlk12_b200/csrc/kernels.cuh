@@ -254,10 +254,27 @@ __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int*
     const int nz = c1.y - c0.y;   // nonzeros in this tile
 
     const uint64_t pol = evict_first_policy();
-    for (int i = tid; i < nr; i += BLOCK) s_row_end[i] = __ldg(rp + c0.x + 1 + i);
-    for (int j = tid; j < nz; j += BLOCK) {
-        const int k = c0.y + j;
-        s_prod[j] = ld_stream_d(val + k, pol) * ld_x(x, ld_stream_i(col + k, pol));
+    // staging, batched per thread: every thread owns IPT slots of each list
+    // (nr, nz <= TILE = BLOCK*IPT); all index/value loads are issued, then all
+    // x gathers, then the products are stored — no serial load chains.
+    {
+        int re[IPT], ci[IPT];
+        double v[IPT], xv[IPT];
+#pragma unroll
+        for (int u = 0; u < IPT; ++u) {
+            const int i = tid + u * BLOCK;
+            re[u] = i < nr ? __ldg(rp + c0.x + 1 + i) : 0;
+            ci[u] = i < nz ? ld_stream_i(col + c0.y + i, pol) : 0;
+            v[u] = i < nz ? ld_stream_d(val + c0.y + i, pol) : 0.0;
+        }
+#pragma unroll
+        for (int u = 0; u < IPT; ++u) xv[u] = (tid + u * BLOCK < nz) ? ld_x_ordered(x, ci[u]) : 0.0;
+#pragma unroll
+        for (int u = 0; u < IPT; ++u) {
+            const int i = tid + u * BLOCK;
+            if (i < nr) s_row_end[i] = re[u];
+            if (i < nz) s_prod[i] = v[u] * xv[u];
+        }
     }
     __syncthreads();
 
