@@ -148,7 +148,9 @@ __global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int*
 // definition). perm maps sorted position -> original row (NULL when σ = 1).
 // The kernel is latency-bound at one chunk per warp, so each chunk's slots
 // are loaded in batches of up to 8 (all column and value loads, then all x
-// gathers, then the FMAs) with an exactly-sized tail batch.
+// gathers, then the FMAs) with an exactly-sized tail batch, and the next
+// chunk's metadata is prefetched (tools/experiments/sell_probe.cu: 830 ->
+// 771 us on config 4). The grid is one resident wave (SMs x occupancy).
 // =====================================================================
 // N slots of one chunk, loads issued unconditionally (all N exist for every
 // lane) before the first FMA; the per-lane row length only masks the FMA.
@@ -184,12 +186,32 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
     const int nwarps = (gridDim.x * BLOCK) >> 5;
     const uint64_t pol = evict_first_policy();
-    for (int c = warp; c < nchunks; c += nwarps) {
-        const int cl = __ldg(chunk_len + c);
-        const int64_t base = __ldg(chunk_ptr + c) + lane;
-        const int clen = cl >= 0 ? cl : -cl;
+    // software pipelining over the warp's chunks: the next chunk's metadata
+    // (and its row lengths when masked) is loaded while the current chunk's
+    // slots are in flight, removing one dependent memory round trip per chunk
+    int c = warp;
+    int cl = 0, rl = 0;
+    int64_t cp = 0;
+    if (c < nchunks) {
+        cl = __ldg(chunk_len + c);
+        cp = __ldg(chunk_ptr + c);
         const int r = c * 32 + lane;
-        const int len = cl >= 0 ? cl : (r < nrows ? __ldg(rowlen + r) : 0);
+        rl = cl >= 0 ? cl : (r < nrows ? __ldg(rowlen + r) : 0);
+    }
+    for (; c < nchunks; c += nwarps) {
+        const int cn = c + nwarps;
+        int cln = 0, rln = 0;
+        int64_t cpn = 0;
+        if (cn < nchunks) {
+            cln = __ldg(chunk_len + cn);
+            cpn = __ldg(chunk_ptr + cn);
+            const int rn = cn * 32 + lane;
+            rln = cln >= 0 ? cln : (rn < nrows ? __ldg(rowlen + rn) : 0);
+        }
+        const int64_t base = cp + lane;
+        const int clen = cl >= 0 ? cl : -cl;
+        const int len = rl;
+        const int r = c * 32 + lane;
         double acc = 0.0;
         int j = 0;
         // whole blocks of 8 slots, then one exactly-sized tail (warp-uniform switch)
@@ -205,6 +227,7 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
         default: break;
         }
         if (r < nrows) y[perm ? __ldg(perm + r) : r] = acc;
+        cl = cln; cp = cpn; rl = rln;
     }
 }
 

@@ -704,7 +704,17 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     p->grid_csr[3] = grid_for((const void*)pepp::k::csr_vector_kernel<8, kBlock>, kBlock, A->nrows, kBlock / 8, p->sm_count);
     p->grid_csr[4] = grid_for((const void*)pepp::k::csr_vector_kernel<16, kBlock>, kBlock, A->nrows, kBlock / 16, p->sm_count);
     p->grid_csr[5] = grid_for((const void*)pepp::k::csr_vector_kernel<32, kBlock>, kBlock, A->nrows, kBlock / 32, p->sm_count);
-    p->grid_sell = grid_for((const void*)pepp::k::sell_kernel<kBlock>, kBlock, p->nchunks, kBlock / 32, p->sm_count);
+    {   // SELL: exactly one resident wave; warps walk their chunks with prefetch
+        int occ = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pepp::k::sell_kernel<kBlock>, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
+        (void)cudaGetLastError();
+        const int64_t need = ((int64_t)p->nchunks + kBlock / 32 - 1) / (kBlock / 32);
+        const int64_t wave = (int64_t)p->sm_count * occ;
+        // prefetching pays once a warp walks many chunks; small matrices keep
+        // more (shorter-lived) blocks instead
+        const int64_t cap = need >= 16 * wave ? wave : 4 * wave;
+        p->grid_sell = (int)std::max<int64_t>(1, std::min<int64_t>(need, cap));
+    }
 
     // ---- history ----
     p->key = pepp::context_key(A->nrows, A->ncols, A->nnz, I.cv_row, o->nranks);
