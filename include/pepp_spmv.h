@@ -168,6 +168,7 @@ typedef struct {
     int32_t exchange;         /* resolved pepp_exchange_t */
     int64_t halo_recv;        /* ghost entries received per exchange (halo) */
     int64_t halo_send;        /* entries sent per exchange (halo) */
+    double sell_col16_frac;   /* fraction of SELL chunks storing 16-bit column deltas */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

@@ -53,6 +53,11 @@ __device__ __forceinline__ double ld_stream_d(const double* p, uint64_t pol) {
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(r) : "l"(p), "l"(pol));
     return r;
 }
+__device__ __forceinline__ int ld_stream_i16(const int16_t* p, uint64_t pol) {
+    int r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s16 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    return r;
+}
 __device__ __forceinline__ int ld_stream_i(const int* p, uint64_t pol) {
     int r;
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
@@ -152,16 +157,28 @@ __global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int*
 // chunk's metadata is prefetched (tools/experiments/sell_probe.cu: 830 ->
 // 771 us on config 4). The grid is one resident wave (SMs x occupancy).
 // =====================================================================
+// Chunk descriptor bits in chunk_len[c]: low 29 bits = slots in the chunk;
+// bit 30 = masked (rows of the chunk have different lengths: read rowlen);
+// bit 29 = 16-bit columns (col16 holds col - row, row = the original index of
+// the lane's row; every delta of the chunk fits in int16).
+constexpr int kSellMasked = 1 << 30;
+constexpr int kSellCol16 = 1 << 29;
+constexpr int kSellLenMask = (1 << 29) - 1;
+
 // N slots of one chunk, loads issued unconditionally (all N exist for every
 // lane) before the first FMA; the per-lane row length only masks the FMA.
-template <int N>
+// C16: columns stored as int16 deltas from the lane's row index `row0`.
+template <int N, bool C16>
 __device__ __forceinline__ double sell_slots(const double* __restrict__ val, const int* __restrict__ col,
+                                             const int16_t* __restrict__ col16, int row0,
                                              const double* __restrict__ x, int64_t base, int j0, int len,
                                              double acc, uint64_t pol) {
     double v[N];
     int c[N];
 #pragma unroll
-    for (int u = 0; u < N; ++u) c[u] = ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
+    for (int u = 0; u < N; ++u)
+        c[u] = C16 ? row0 + ld_stream_i16(col16 + base + (int64_t)(j0 + u) * 32, pol)
+                   : ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
 #pragma unroll
     for (int u = 0; u < N; ++u) v[u] = ld_stream_d(val + base + (int64_t)(j0 + u) * 32, pol);
     double xv[N];
@@ -173,12 +190,34 @@ __device__ __forceinline__ double sell_slots(const double* __restrict__ val, con
     return acc;
 }
 
+template <bool C16>
+__device__ __forceinline__ double sell_chunk(const double* __restrict__ val, const int* __restrict__ col,
+                                             const int16_t* __restrict__ col16, int row0, const double* __restrict__ x,
+                                             int64_t base, int clen, int len, uint64_t pol) {
+    double acc = 0.0;
+    int j = 0;
+    // whole blocks of 8 slots, then one exactly-sized tail (warp-uniform switch)
+    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, C16>(val, col, col16, row0, x, base, j, len, acc, pol);
+    switch (clen - j) {
+    case 1: acc = sell_slots<1, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 2: acc = sell_slots<2, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 3: acc = sell_slots<3, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 4: acc = sell_slots<4, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 5: acc = sell_slots<5, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 6: acc = sell_slots<6, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 7: acc = sell_slots<7, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    default: break;
+    }
+    return acc;
+}
+
 template <int BLOCK>
 __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
                                                      const int* __restrict__ chunk_len,
                                                      const int* __restrict__ rowlen,
                                                      const int* __restrict__ perm,
                                                      const int* __restrict__ col,
+                                                     const int16_t* __restrict__ col16,
                                                      const double* __restrict__ val,
                                                      const double* __restrict__ x,
                                                      double* __restrict__ y) {
@@ -187,47 +226,31 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     const int nwarps = (gridDim.x * BLOCK) >> 5;
     const uint64_t pol = evict_first_policy();
     // software pipelining over the warp's chunks: the next chunk's metadata
-    // (and its row lengths when masked) is loaded while the current chunk's
-    // slots are in flight, removing one dependent memory round trip per chunk
-    int c = warp;
-    int cl = 0, rl = 0;
-    int64_t cp = 0;
-    if (c < nchunks) {
-        cl = __ldg(chunk_len + c);
+    // (its row lengths when masked, its original row indices when sorted) is
+    // loaded while the current chunk's slots are in flight, removing one
+    // dependent memory round trip per chunk
+    auto meta = [&](int c, int& d, int64_t& cp, int& len, int& orow) {
+        d = __ldg(chunk_len + c);
         cp = __ldg(chunk_ptr + c);
         const int r = c * 32 + lane;
-        rl = cl >= 0 ? cl : (r < nrows ? __ldg(rowlen + r) : 0);
-    }
+        len = !(d & kSellMasked) ? (d & kSellLenMask) : (r < nrows ? __ldg(rowlen + r) : 0);
+        orow = (perm && r < nrows) ? __ldg(perm + r) : r;
+    };
+    int c = warp;
+    int d = 0, len = 0, orow = 0;
+    int64_t cp = 0;
+    if (c < nchunks) meta(c, d, cp, len, orow);
     for (; c < nchunks; c += nwarps) {
         const int cn = c + nwarps;
-        int cln = 0, rln = 0;
+        int dn = 0, lenn = 0, orown = 0;
         int64_t cpn = 0;
-        if (cn < nchunks) {
-            cln = __ldg(chunk_len + cn);
-            cpn = __ldg(chunk_ptr + cn);
-            const int rn = cn * 32 + lane;
-            rln = cln >= 0 ? cln : (rn < nrows ? __ldg(rowlen + rn) : 0);
-        }
+        if (cn < nchunks) meta(cn, dn, cpn, lenn, orown);
         const int64_t base = cp + lane;
-        const int clen = cl >= 0 ? cl : -cl;
-        const int len = rl;
-        const int r = c * 32 + lane;
-        double acc = 0.0;
-        int j = 0;
-        // whole blocks of 8 slots, then one exactly-sized tail (warp-uniform switch)
-        for (; j + 8 <= clen; j += 8) acc = sell_slots<8>(val, col, x, base, j, len, acc, pol);
-        switch (clen - j) {
-        case 1: acc = sell_slots<1>(val, col, x, base, j, len, acc, pol); break;
-        case 2: acc = sell_slots<2>(val, col, x, base, j, len, acc, pol); break;
-        case 3: acc = sell_slots<3>(val, col, x, base, j, len, acc, pol); break;
-        case 4: acc = sell_slots<4>(val, col, x, base, j, len, acc, pol); break;
-        case 5: acc = sell_slots<5>(val, col, x, base, j, len, acc, pol); break;
-        case 6: acc = sell_slots<6>(val, col, x, base, j, len, acc, pol); break;
-        case 7: acc = sell_slots<7>(val, col, x, base, j, len, acc, pol); break;
-        default: break;
-        }
-        if (r < nrows) y[perm ? __ldg(perm + r) : r] = acc;
-        cl = cln; cp = cpn; rl = rln;
+        const int clen = d & kSellLenMask;
+        const double acc = (d & kSellCol16) ? sell_chunk<true>(val, col, col16, orow, x, base, clen, len, pol)
+                                            : sell_chunk<false>(val, col, col16, orow, x, base, clen, len, pol);
+        if (c * 32 + lane < nrows) y[orow] = acc;
+        d = dn; cp = cpn; len = lenn; orow = orown;
     }
 }
 
@@ -646,7 +669,7 @@ __global__ void sell_keys_kernel(int nrows, const int* __restrict__ rp, int sigm
 }
 
 // sorted position r -> original row perm[r]; lengths + per-chunk max
-// chunk_len[c] = max length if all 32 rows exist and have that length, else -max
+// chunk_len[c] = max length, | kSellMasked unless all 32 rows exist with that length
 __global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,
                                     int* __restrict__ rowlen, int* __restrict__ chunk_len) {
     const int r = blockIdx.x * blockDim.x + threadIdx.x;
@@ -663,7 +686,7 @@ __global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const
         mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, off));
     }
     mx = max(mx, 0);
-    if (lane == 0 && r < nrows) chunk_len[r >> 5] = (mn == mx) ? mx : -mx;
+    if (lane == 0 && r < nrows) chunk_len[r >> 5] = (mn == mx) ? mx : (mx | kSellMasked);
 }
 
 __global__ void sell_fill_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,
@@ -678,6 +701,37 @@ __global__ void sell_fill_kernel(int nrows, const int* __restrict__ rp, const in
     for (int k = s; k < e; ++k) {
         col[base + (int64_t)(k - s) * 32] = src_col[k];
         val[base + (int64_t)(k - s) * 32] = src_val[k];
+    }
+}
+
+// 16-bit column deltas: one warp per chunk; if every stored column of the
+// chunk is within int16 of its row's original index, write col16 and set
+// kSellCol16 in chunk_len.
+__global__ void sell_col16_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
+                                  int* __restrict__ chunk_len, const int* __restrict__ rowlen,
+                                  const int* __restrict__ perm, const int* __restrict__ col,
+                                  int16_t* __restrict__ col16, unsigned long long* __restrict__ n16) {
+    const int lane = threadIdx.x & 31;
+    const int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (c >= nchunks) return;
+    const int d = chunk_len[c];
+    const int clen = d & kSellLenMask;
+    const int r = c * 32 + lane;
+    const int len = r < nrows ? rowlen[r] : 0;
+    const int orow = (perm && r < nrows) ? perm[r] : r;
+    const int64_t base = chunk_ptr[c] + lane;
+    bool ok = true;
+    for (int j = 0; j < len; ++j) {
+        const int dl = col[base + (int64_t)j * 32] - orow;
+        ok &= (dl >= -32768 && dl <= 32767);
+    }
+    ok = __all_sync(0xffffffffu, ok);
+    if (!ok) return;
+    for (int j = 0; j < clen; ++j)
+        col16[base + (int64_t)j * 32] = (int16_t)(j < len ? col[base + (int64_t)j * 32] - orow : 0);
+    if (lane == 0) {
+        chunk_len[c] = d | kSellCol16;
+        atomicAdd(n16, 1ull);
     }
 }
 

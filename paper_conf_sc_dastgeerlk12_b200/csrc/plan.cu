@@ -85,6 +85,8 @@ struct pepp_spmv_plan_s {
     int* d_rowlen = nullptr;
     int* d_perm = nullptr;
     int* d_scol = nullptr;
+    int16_t* d_scol16 = nullptr;
+    int64_t sell_col16_chunks = 0;
     double* d_sval = nullptr;
 
     // merge path
@@ -151,7 +153,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (!p) return;
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
-                    p->d_scol, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
+                    p->d_scol, p->d_scol16, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
                     p->d_items, p->d_longrows, p->d_stream_carry};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
@@ -190,7 +192,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
         int64_t slots = 0;
         std::vector<int64_t> cp(p->nchunks + 1);
-        for (int c = 0; c < p->nchunks; ++c) { cp[c] = slots; slots += (int64_t)std::abs(cl[c]) * 32; }
+        for (int c = 0; c < p->nchunks; ++c) { cp[c] = slots; slots += (int64_t)(cl[c] & pepp::k::kSellLenMask) * 32; }
         cp[p->nchunks] = slots;
         p->sell_slots = slots;
         *fill = p->nnz ? (double)slots / (double)p->nnz : 1.0;
@@ -237,8 +239,28 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     pepp::k::sell_fill_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, p->d_col, p->d_val, p->d_chunk_ptr,
                                                    p->d_scol, p->d_sval);
     PEPP_CUDA_TRY(cudaGetLastError());
+    // 16-bit column deltas where a whole chunk allows them (banded / stencil
+    // structure): 2 instead of 4 bytes of index per stored slot
+    {
+        if ((s = dalloc(p, &p->d_scol16, p->sell_slots + 32))) return s;
+        PEPP_CUDA_TRY(cudaMemsetAsync(p->d_scol16, 0, sizeof(int16_t) * (p->sell_slots + 32), st));
+        unsigned long long* d_n16 = nullptr;
+        PEPP_CUDA_TRY(cudaMalloc(&d_n16, sizeof(unsigned long long)));
+        PEPP_CUDA_TRY(cudaMemsetAsync(d_n16, 0, sizeof(unsigned long long), st));
+        const int wb = 256, wg = (int)(((int64_t)p->nchunks * 32 + wb - 1) / wb);
+        pepp::k::sell_col16_kernel<<<wg, wb, 0, st>>>(n, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen,
+                                                       p->d_perm, p->d_scol, p->d_scol16, d_n16);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        unsigned long long n16 = 0;
+        PEPP_CUDA_TRY(cudaMemcpyAsync(&n16, d_n16, sizeof(n16), cudaMemcpyDeviceToHost, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        cudaFree(d_n16);
+        p->sell_col16_chunks = (int64_t)n16;
+        if (n16 == 0) { cudaFree(p->d_scol16); p->d_scol16 = nullptr; p->dev_bytes -= (int64_t)sizeof(int16_t) * (p->sell_slots + 32); }
+    }
     PEPP_CUDA_TRY(cudaStreamSynchronize(st));
     p->info.sell_sigma = sigma;
+    p->info.sell_col16_frac = p->nchunks ? (double)p->sell_col16_chunks / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
     return PEPP_OK;
 }
@@ -351,7 +373,7 @@ pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const double* x, d
     case PEPP_V_SELL:
         pepp::k::sell_kernel<kBlock><<<p->grid_sell, kBlock, 0, st>>>((int)p->nrows, p->nchunks, p->d_chunk_ptr,
                                                                        p->d_chunk_len, p->d_rowlen, p->d_perm,
-                                                                       p->d_scol, p->d_sval, x, y);
+                                                                       p->d_scol, p->d_scol16, p->d_sval, x, y);
         break;
     default:
         return PEPP_E_INVALID;

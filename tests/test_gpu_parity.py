@@ -351,3 +351,30 @@ def test_exchange_is_noop_unpartitioned():
         plan.exchange(y, pepp.Y_REPLICATED)
         torch.cuda.synchronize()
         assert torch.all(y == 0)
+
+
+def test_sell_col16_used_and_exact_on_stencils():
+    """Banded / Laplacian chunks store 16-bit column deltas; mixed matrices
+    keep 32-bit chunks where deltas do not fit; results stay bit-exact."""
+    for A, expect in ((gen.laplacian2d(200), 1.0), (gen.banded(50_000, 4, seed=1, val_mode=gen.INT4), 1.0)):
+        x = gen.vector(3, gen.INT8, A.ncols)
+        with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_SELL) as plan:
+            assert plan.info()["sell_col16_frac"] == expect
+            y, _ = _run(plan, x)
+        assert np.array_equal(y, oracle.spmv(A, x))
+    # uniform random over 100k columns: deltas do not fit in int16 for most chunks
+    A = gen.uniform(20_000, 100_000, 8, seed=2, val_mode=gen.INT4)
+    x = gen.vector(3, gen.INT8, A.ncols)
+    with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_SELL, prune=False) as plan:
+        assert plan.info()["sell_col16_frac"] < 0.5
+        y, _ = _run(plan, x)
+    assert np.array_equal(y, oracle.spmv(A, x))
+    # a matrix whose chunks mix both kinds: near-diagonal rows + far rows
+    rows = [[(i, 2.0), ((i * 7919) % 70_000, 1.0)] if i % 64 == 0 else [(i, 3.0)] for i in range(70_000)]
+    B = _hand(70_000, 70_000, [sorted(r) for r in rows])
+    x = gen.vector(5, gen.INT8, B.ncols)
+    with pepp.Plan.from_csr(B, variant_mask=1 << pepp.V_SELL, prune=False) as plan:
+        f = plan.info()["sell_col16_frac"]
+        assert 0.0 < f < 1.0
+        y, _ = _run(plan, x)
+    assert np.array_equal(y, oracle.spmv(B, x))
