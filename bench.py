@@ -155,6 +155,21 @@ def traffic_for(kernel: str, workload: str):
         return None
 
 
+def roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, workload) -> dict:
+    """Roofline of the dominant kernel: algorithmic bytes / launch time vs the
+    measured peak; `traffic` = ncu DRAM bytes per launch (may be below the
+    algorithmic bytes when the variant stores a compressed layout, e.g. SELL
+    16-bit column deltas), with the DRAM-traffic fraction beside it."""
+    traffic = traffic_for(kname, workload)
+    d = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "peak_source": peak_src,
+         "unit": "GB/s", "frac": round(achieved / peak, 4), "avg_launch_us": round(avg_kernel_s * 1e6, 2),
+         "bytes_per_launch": local_bytes, "traffic": traffic}
+    if traffic:
+        d["traffic_gbs"] = round(traffic / avg_kernel_s / 1e9, 1)
+        d["traffic_frac"] = round(traffic / avg_kernel_s / 1e9 / peak, 4)
+    return d
+
+
 def parse_variant(s: str | None):
     import paper_conf_sc_dastgeerlk12_b200 as pepp
     if not s:
@@ -406,10 +421,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
                        "variant": args.variant or "auto (history-based per call)"},
             "hbm": {"achieved_gbs": round(gbs, 1), "frac_of_measured": round(gbs / (world * peak), 4),
                     "frac_of_8tbs": round(gbs / (world * 8000.0), 4), "algorithmic_bytes_per_spmv": alg_bytes_global},
-            "roofline": {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
-                         "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4),
-                         "avg_launch_us": round(avg_kernel_s * 1e6, 2), "bytes_per_launch": local_bytes,
-                         "traffic": traffic_for(kname, args.workload)},
+            "roofline": roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, args.workload),
             "e2e": {"value": round(e2e_val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": A.ncols * 8,
                     "d2h_bytes_per_step": A.nrows * 8, "spmv_per_step": e2e_iters,
                     "api": "pepp_spmv_exec_host (pinned host x0 -> iterations -> host y)"},
