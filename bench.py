@@ -259,7 +259,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
     plan = pepp.Plan.from_csr(A, nranks=world, rank=rank, row_bounds=bounds if world > 1 else None,
-                              nccl_unique_id=uid)
+                              nccl_unique_id=uid, prune=not args.no_prune)
     info = plan.info()
     force = parse_variant(args.variant)
     flags = pepp.Y_NEXT_INPUT if iterated else pepp.Y_LOCAL
@@ -448,6 +448,7 @@ def main():
     ap.add_argument("--variant", default=None)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-sweep", action="store_true")
+    ap.add_argument("--no-prune", action="store_true", help="every variant is a candidate (no static narrowing)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
 

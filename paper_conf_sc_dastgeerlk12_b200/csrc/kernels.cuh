@@ -96,12 +96,21 @@ __global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int*
     const int nwarps = (gridDim.x * BLOCK) >> 5;
     const uint64_t pol = evict_first_policy();
 
-    for (int64_t base = (int64_t)warp * RPW; base < nrows; base += (int64_t)nwarps * RPW) {
+    // the next row's [s, e) is prefetched while the current row's entries
+    // are in flight (one dependent round trip less per row)
+    const int64_t step = (int64_t)nwarps * RPW;
+    int64_t base = (int64_t)warp * RPW;
+    int sn = 0, en = 0;
+    if (base + grp < nrows) {
+        sn = __ldg(rp + base + grp);
+        en = __ldg(rp + base + grp + 1);
+    }
+    for (; base < nrows; base += step) {
         const int64_t row = base + grp;
-        int s = 0, e = 0;
-        if (row < nrows) {
-            s = __ldg(rp + row);
-            e = __ldg(rp + row + 1);
+        const int s = sn, e = en;
+        if (row + step < nrows) {
+            sn = __ldg(rp + row + step);
+            en = __ldg(rp + row + step + 1);
         }
         double acc = 0.0;
         const int g_end = (e + 3) >> 2;
