@@ -396,8 +396,106 @@ __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int*
     }
 }
 
-// Per tile t: if t is the first tile carrying into its row, add the carries
-// of t, t+1, ... (same row) to y[row] in tile order.
+// Warp-granular merge-path: the same decomposition with tiles of 32*IPT
+// merge items owned by ONE warp (row ends + products staged in that warp's
+// slice of shared memory, warp-only segmented scan): no block barriers, so
+// every warp streams independently (latency hiding by warp count).
+template <int IPT, int WARPS>
+__global__ void __launch_bounds__(WARPS * 32) merge_warp_kernel(int nrows, int ntiles, const int* __restrict__ rp,
+                                                               const int* __restrict__ col,
+                                                               const double* __restrict__ val,
+                                                               const double* __restrict__ x,
+                                                               double* __restrict__ y,
+                                                               const int2* __restrict__ tile_coord,
+                                                               int* __restrict__ carry_row,
+                                                               double* __restrict__ carry_val) {
+    constexpr int TILE = 32 * IPT;
+    __shared__ int s_row_end_all[WARPS][TILE];
+    __shared__ double s_prod_all[WARPS][TILE];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int tile = blockIdx.x * WARPS + w;
+    if (tile >= ntiles) return;
+    int* s_row_end = s_row_end_all[w];
+    double* s_prod = s_prod_all[w];
+    const uint64_t pol = evict_first_policy();
+    const int2 c0 = __ldg(tile_coord + tile);
+    const int2 c1 = __ldg(tile_coord + tile + 1);
+    const int nr = c1.x - c0.x, nz = c1.y - c0.y;
+    {
+        int re[IPT], ci[IPT];
+        double v[IPT], xv[IPT];
+#pragma unroll
+        for (int u = 0; u < IPT; ++u) {
+            const int i = lane + u * 32;
+            re[u] = i < nr ? __ldg(rp + c0.x + 1 + i) : 0;
+            ci[u] = i < nz ? ld_stream_i(col + c0.y + i, pol) : 0;
+            v[u] = i < nz ? ld_stream_d(val + c0.y + i, pol) : 0.0;
+        }
+#pragma unroll
+        for (int u = 0; u < IPT; ++u) xv[u] = (lane + u * 32 < nz) ? ld_x_ordered(x, ci[u]) : 0.0;
+#pragma unroll
+        for (int u = 0; u < IPT; ++u) {
+            const int i = lane + u * 32;
+            if (i < nr) s_row_end[i] = re[u];
+            if (i < nz) s_prod[i] = v[u] * xv[u];
+        }
+    }
+    __syncwarp();
+    const int total = nr + nz;
+    const int d = min(lane * IPT, total);
+    int lo = max(0, d - nz), hi = min(d, nr);
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (s_row_end[mid] <= c0.y + d - mid - 1) lo = mid + 1;
+        else hi = mid;
+    }
+    int ri = lo, kabs = c0.y + d - lo;
+    const int dend = min(d + IPT, total);
+    int re = ri < nr ? s_row_end[ri] : 0x7fffffff;
+    double acc = 0.0, head_val = 0.0;
+    int head_row = -1;
+#pragma unroll
+    for (int it = 0; it < IPT; ++it) {
+        if (d + it < dend) {
+            if (kabs < re) {
+                acc += s_prod[kabs - c0.y];
+                ++kabs;
+            } else {
+                if (head_row < 0) { head_row = ri; head_val = acc; }
+                else y[c0.x + ri] = acc;
+                acc = 0.0;
+                ++ri;
+                re = ri < nr ? s_row_end[ri] : 0x7fffffff;
+            }
+        }
+    }
+    // warp inclusive segmented scan of (acc, ended-a-row)
+    SegPair inc{acc, head_row >= 0 ? 1 : 0};
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        SegPair o;
+        o.v = __shfl_up_sync(0xffffffffu, inc.v, off);
+        o.f = __shfl_up_sync(0xffffffffu, inc.f, off);
+        if (lane >= off) inc = seg_combine(o, inc);
+    }
+    double excl = __shfl_up_sync(0xffffffffu, inc.v, 1);
+    if (lane == 0) excl = 0.0;
+    if (head_row >= 0) y[c0.x + head_row] = excl + head_val;
+    if (lane == 31) {
+        carry_row[tile] = c1.x;
+        carry_val[tile] = inc.v;
+    }
+}
+
+// Carry fix-up. Tile t leaves carry_val[t] for row carry_row[t] (the row
+// open at its end); a run of consecutive tiles carrying into one row is
+// summed in tile order and added to y[row] once (deterministic, no fp
+// atomics). Runs are fixed by the matrix structure, so the plan lists the
+// long ones (>= kLongRun tiles, rows spanning many tiles): those go to
+// merge_fixup_long_kernel (one warp per run, lane-strided + fixed shuffle
+// tree); merge_fixup_kernel (one thread per tile) handles the short ones.
+constexpr int kLongRun = 32;
+
 __global__ void merge_fixup_kernel(int ntiles, int nrows, const int* __restrict__ carry_row,
                                    const double* __restrict__ carry_val, double* __restrict__ y) {
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
@@ -406,8 +504,24 @@ __global__ void merge_fixup_kernel(int ntiles, int nrows, const int* __restrict_
     if (row >= nrows) return;
     if (t > 0 && carry_row[t - 1] == row) return;
     double s = carry_val[t];
-    for (int u = t + 1; u < ntiles && carry_row[u] == row; ++u) s += carry_val[u];
+    int u = t + 1;
+    for (; u < ntiles && u - t < kLongRun && carry_row[u] == row; ++u) s += carry_val[u];
+    if (u - t >= kLongRun) return;   // a long run: merge_fixup_long_kernel adds it
     y[row] = s + y[row];
+}
+
+// runs[i] = (first tile, number of tiles, row)
+__global__ void merge_fixup_long_kernel(int nruns, const int4* __restrict__ runs, const double* __restrict__ carry_val,
+                                        double* __restrict__ y) {
+    const int lane = threadIdx.x & 31;
+    const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    if (i >= nruns) return;
+    const int4 r = runs[i];
+    double s = 0.0;
+    for (int u = lane; u < r.y; u += 32) s += carry_val[r.x + u];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) y[r.z] = s + y[r.z];
 }
 
 // Plan time: tile start coordinates on the global merge path.
@@ -601,15 +715,19 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
     }
 }
 
-// y[row] = sum of its long-row pieces, in piece order
+// y[row] = sum of its long-row pieces: one warp per long row, lane-strided
+// over the pieces then a fixed shuffle tree (deterministic)
 __global__ void csr_stream_fixup_kernel(int nlong, const int4* __restrict__ longrows, const double* __restrict__ carry,
                                         double* __restrict__ y) {
-    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = threadIdx.x & 31;
+    const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
     if (i >= nlong) return;
     const int4 L = longrows[i];   // (row, first piece, end piece, -)
     double s = 0.0;
-    for (int p = L.y; p < L.z; ++p) s += carry[p];
-    y[L.x] = s;
+    for (int p = L.y + lane; p < L.z; p += 32) s += carry[p];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) y[L.x] = s;
 }
 
 // =====================================================================

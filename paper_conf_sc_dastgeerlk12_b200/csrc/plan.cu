@@ -30,6 +30,11 @@ constexpr int kBlock = 256;
 constexpr int kMergeBlock = 256;
 constexpr int kMergeIPT = 7;
 constexpr int kMergeTile = kMergeBlock * kMergeIPT;
+// warp-granular merge-path: tiles of 32 x kMergeWarpIPT items, kMergeWarps warps per CTA
+constexpr int kMergeWarpIPT = 7;
+constexpr int kMergeWarps = 8;
+constexpr int kMergeWarpTile = 32 * kMergeWarpIPT;
+constexpr int kMergeWarpParam = 1000 + kMergeWarpIPT;   // candidate param of the warp-granular kernel
 constexpr int kTimingRing = 64;
 // TMA CSR-stream: items of <= kStreamNB nonzeros / <= kStreamRMAX rows, kStreamStages-deep ring
 constexpr int kStreamBlock = 256;
@@ -94,6 +99,13 @@ struct pepp_spmv_plan_s {
     int2* d_tile = nullptr;
     int* d_carry_row = nullptr;
     double* d_carry_val = nullptr;
+    int nlongruns = 0, nlongruns_w = 0;
+    int4* d_longruns = nullptr;
+    int4* d_longruns_w = nullptr;
+    int ntiles_w = 0;
+    int2* d_tile_w = nullptr;
+    int* d_carry_row_w = nullptr;
+    double* d_carry_val_w = nullptr;
 
     // TMA CSR-stream
     int nitems = 0, nlong = 0, grid_stream = 0;
@@ -154,7 +166,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
-                    p->d_items, p->d_longrows, p->d_stream_carry};
+                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -266,6 +278,29 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
 }
 
 // ---------------------------------------------------------------- merge prep
+// Runs of >= kLongRun consecutive tiles that carry into the same row (the row
+// open at a tile's end is tile_coord[t+1].x, fixed by the structure).
+pepp_status_t long_runs(pepp_spmv_plan_t* p, const int2* d_tile, int ntiles, int4** out, int* nout) {
+    *nout = 0;
+    if (ntiles <= 0) return PEPP_OK;
+    std::vector<int2> tc(ntiles + 1);
+    PEPP_CUDA_TRY(cudaMemcpy(tc.data(), d_tile, sizeof(int2) * (ntiles + 1), cudaMemcpyDeviceToHost));
+    std::vector<int4> runs;
+    for (int t = 0; t < ntiles;) {
+        const int row = tc[t + 1].x;
+        int u = t + 1;
+        while (u < ntiles && tc[u + 1].x == row) ++u;
+        if (row < p->nrows && u - t >= pepp::k::kLongRun) runs.push_back(make_int4(t, u - t, row, 0));
+        t = u;
+    }
+    if (runs.empty()) return PEPP_OK;
+    pepp_status_t s;
+    if ((s = dalloc(p, out, (int64_t)runs.size()))) return s;
+    PEPP_CUDA_TRY(cudaMemcpy(*out, runs.data(), sizeof(int4) * runs.size(), cudaMemcpyHostToDevice));
+    *nout = (int)runs.size();
+    return PEPP_OK;
+}
+
 pepp_status_t prepare_merge(pepp_spmv_plan_t* p, cudaStream_t st) {
     const int64_t total = p->nrows + p->nnz;
     p->ntiles = (int)((total + kMergeTile - 1) / kMergeTile);
@@ -277,7 +312,16 @@ pepp_status_t prepare_merge(pepp_spmv_plan_t* p, cudaStream_t st) {
     pepp::k::merge_tile_search_kernel<<<(p->ntiles + 1 + tb - 1) / tb, tb, 0, st>>>(
         (int)p->nrows, p->nnz, p->d_rp, kMergeTile, p->ntiles, p->d_tile);
     PEPP_CUDA_TRY(cudaGetLastError());
+    p->ntiles_w = (int)((total + kMergeWarpTile - 1) / kMergeWarpTile);
+    if ((s = dalloc(p, &p->d_tile_w, (int64_t)p->ntiles_w + 1))) return s;
+    if ((s = dalloc(p, &p->d_carry_row_w, std::max(p->ntiles_w, 1)))) return s;
+    if ((s = dalloc(p, &p->d_carry_val_w, std::max(p->ntiles_w, 1)))) return s;
+    pepp::k::merge_tile_search_kernel<<<(p->ntiles_w + 1 + tb - 1) / tb, tb, 0, st>>>(
+        (int)p->nrows, p->nnz, p->d_rp, kMergeWarpTile, p->ntiles_w, p->d_tile_w);
+    PEPP_CUDA_TRY(cudaGetLastError());
     PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    if ((s = long_runs(p, p->d_tile, p->ntiles, &p->d_longruns, &p->nlongruns))) return s;
+    if ((s = long_runs(p, p->d_tile_w, p->ntiles_w, &p->d_longruns_w, &p->nlongruns_w))) return s;
     return PEPP_OK;
 }
 
@@ -354,11 +398,28 @@ pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const double* x, d
         }
         break;
     case PEPP_V_MERGE_PATH:
+        if (c.param == kMergeWarpParam) {
+            if (p->ntiles_w > 0) {
+                pepp::k::merge_warp_kernel<kMergeWarpIPT, kMergeWarps>
+                    <<<(p->ntiles_w + kMergeWarps - 1) / kMergeWarps, kMergeWarps * 32, 0, st>>>(
+                        (int)p->nrows, p->ntiles_w, p->d_rp, p->d_col, p->d_val, x, y, p->d_tile_w, p->d_carry_row_w,
+                        p->d_carry_val_w);
+                pepp::k::merge_fixup_kernel<<<(p->ntiles_w + 255) / 256, 256, 0, st>>>(
+                    p->ntiles_w, (int)p->nrows, p->d_carry_row_w, p->d_carry_val_w, y);
+                if (p->nlongruns_w)
+                    pepp::k::merge_fixup_long_kernel<<<(p->nlongruns_w * 32 + 255) / 256, 256, 0, st>>>(
+                        p->nlongruns_w, p->d_longruns_w, p->d_carry_val_w, y);
+            }
+            break;
+        }
         if (p->ntiles > 0) {
             pepp::k::merge_spmv_kernel<kMergeBlock, kMergeIPT><<<p->ntiles, kMergeBlock, 0, st>>>(
                 (int)p->nrows, p->d_rp, p->d_col, p->d_val, x, y, p->d_tile, p->d_carry_row, p->d_carry_val);
-            pepp::k::merge_fixup_kernel<<<(p->ntiles + 255) / 256, 256, 0, st>>>(p->ntiles, (int)p->nrows,
-                                                                                  p->d_carry_row, p->d_carry_val, y);
+            pepp::k::merge_fixup_kernel<<<(p->ntiles + 255) / 256, 256, 0, st>>>(
+                p->ntiles, (int)p->nrows, p->d_carry_row, p->d_carry_val, y);
+            if (p->nlongruns)
+                pepp::k::merge_fixup_long_kernel<<<(p->nlongruns * 32 + 255) / 256, 256, 0, st>>>(
+                    p->nlongruns, p->d_longruns, p->d_carry_val, y);
         }
         break;
     case PEPP_V_CSR_STREAM:
@@ -366,8 +427,8 @@ pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const double* x, d
             stream_kernel()<<<p->grid_stream, kStreamBlock, kStreamSmem, st>>>(
                 p->nitems, p->d_items, p->d_rp, p->d_col, p->d_val, x, y, p->d_stream_carry);
             if (p->nlong)
-                pepp::k::csr_stream_fixup_kernel<<<(p->nlong + 127) / 128, 128, 0, st>>>(p->nlong, p->d_longrows,
-                                                                                        p->d_stream_carry, y);
+                pepp::k::csr_stream_fixup_kernel<<<(p->nlong * 32 + 255) / 256, 256, 0, st>>>(p->nlong, p->d_longrows,
+                                                                                              p->d_stream_carry, y);
         }
         break;
     case PEPP_V_SELL:
@@ -707,7 +768,10 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     }
     if (mask & (1u << PEPP_V_CSR_VECTOR))
         for (int tpr : {2, 4, 8, 16, 32}) p->cands.push_back({PEPP_V_CSR_VECTOR, tpr});
-    if (mask & (1u << PEPP_V_MERGE_PATH)) p->cands.push_back({PEPP_V_MERGE_PATH, kMergeIPT});
+    if (mask & (1u << PEPP_V_MERGE_PATH)) {
+        p->cands.push_back({PEPP_V_MERGE_PATH, kMergeIPT});
+        p->cands.push_back({PEPP_V_MERGE_PATH, kMergeWarpParam});
+    }
     if (mask & (1u << PEPP_V_SELL)) {
         if ((s = prepare_sell(p, st))) return s;
         p->cands.push_back({PEPP_V_SELL, p->sell_sigma});
