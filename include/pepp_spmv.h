@@ -134,7 +134,7 @@ typedef struct {
     int32_t prune;            /* 1 (default) = multi-stage composition (P@10489): statically narrow the
                                  candidates from the context instance before the runtime choice —
                                  vector-CSR only if max_row <= max(4096, 256*mean), SELL only if
-                                 max_row <= max(256, 16*mean); merge-path and CSR-stream always.
+                                 max_row <= 4096; merge-path and CSR-stream always.
                                  0 = every variant is a candidate (variant_mask still applies). */
 } pepp_spmv_opts_t;
 

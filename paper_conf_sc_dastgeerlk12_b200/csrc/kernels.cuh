@@ -220,7 +220,7 @@ __device__ __forceinline__ double sell_chunk(const double* __restrict__ val, con
     return acc;
 }
 
-template <int BLOCK>
+template <int BLOCK, bool SORTED>
 __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
                                                      const int* __restrict__ chunk_len,
                                                      const int* __restrict__ rowlen,
@@ -229,37 +229,48 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
                                                      const int16_t* __restrict__ col16,
                                                      const double* __restrict__ val,
                                                      const double* __restrict__ x,
-                                                     double* __restrict__ y) {
+                                                     double* __restrict__ y,
+                                                     int cpw) {
     const int lane = threadIdx.x & 31;
     const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
     const int nwarps = (gridDim.x * BLOCK) >> 5;
     const uint64_t pol = evict_first_policy();
-    // software pipelining over the warp's chunks: the next chunk's metadata
-    // (its row lengths when masked, its original row indices when sorted) is
-    // loaded while the current chunk's slots are in flight, removing one
-    // dependent memory round trip per chunk
+    // chunk order: warp w walks i = w, w + nwarps, ...; chunk = i when the
+    // chunks are uniform (σ = 1). When σ > 1 sorted the rows, chunk lengths
+    // repeat a long-to-short pattern in every window of cpw = σ/32 chunks and
+    // a plain stride can hand a warp only the longest chunks; the order is
+    // then transposed (window-major -> position-major) over the full windows,
+    // a bijection that walks every warp through all positions.
+    const int nfull = SORTED ? (nchunks / cpw) * cpw : 0;
+    const int nwin = SORTED ? nchunks / cpw : 1;
+    auto chunk_of = [&](int i) -> int {
+        if (!SORTED) return i;
+        return i < nfull ? (i % nwin) * cpw + i / nwin : i;
+    };
     auto meta = [&](int c, int& d, int64_t& cp, int& len, int& orow) {
         d = __ldg(chunk_len + c);
         cp = __ldg(chunk_ptr + c);
         const int r = c * 32 + lane;
         len = !(d & kSellMasked) ? (d & kSellLenMask) : (r < nrows ? __ldg(rowlen + r) : 0);
-        orow = (perm && r < nrows) ? __ldg(perm + r) : r;
+        orow = (SORTED && r < nrows) ? __ldg(perm + r) : r;
     };
-    int c = warp;
+    int i = warp;
+    int c = i < nchunks ? chunk_of(i) : 0;
     int d = 0, len = 0, orow = 0;
     int64_t cp = 0;
-    if (c < nchunks) meta(c, d, cp, len, orow);
-    for (; c < nchunks; c += nwarps) {
-        const int cn = c + nwarps;
+    if (i < nchunks) meta(c, d, cp, len, orow);
+    for (; i < nchunks; i += nwarps) {
+        const int in = i + nwarps;
+        const int cn = in < nchunks ? chunk_of(in) : 0;
         int dn = 0, lenn = 0, orown = 0;
         int64_t cpn = 0;
-        if (cn < nchunks) meta(cn, dn, cpn, lenn, orown);
+        if (in < nchunks) meta(cn, dn, cpn, lenn, orown);
         const int64_t base = cp + lane;
         const int clen = d & kSellLenMask;
         const double acc = (d & kSellCol16) ? sell_chunk<true>(val, col, col16, orow, x, base, clen, len, pol)
                                             : sell_chunk<false>(val, col, col16, orow, x, base, clen, len, pol);
         if (c * 32 + lane < nrows) y[orow] = acc;
-        d = dn; cp = cpn; len = lenn; orow = orown;
+        c = cn; d = dn; cp = cpn; len = lenn; orow = orown;
     }
 }
 

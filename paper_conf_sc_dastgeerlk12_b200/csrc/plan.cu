@@ -91,6 +91,7 @@ struct pepp_spmv_plan_s {
     int* d_perm = nullptr;
     int* d_scol = nullptr;
     int16_t* d_scol16 = nullptr;
+    int sell_cpw = 1;            // chunks per σ window (chunk order is transposed when > 1)
     int64_t sell_col16_chunks = 0;
     double* d_sval = nullptr;
 
@@ -271,6 +272,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
         if (n16 == 0) { cudaFree(p->d_scol16); p->d_scol16 = nullptr; p->dev_bytes -= (int64_t)sizeof(int16_t) * (p->sell_slots + 32); }
     }
     PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    p->sell_cpw = sigma > 1 ? std::max(1, sigma / 32) : 1;
     p->info.sell_sigma = sigma;
     p->info.sell_col16_frac = p->nchunks ? (double)p->sell_col16_chunks / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
@@ -432,9 +434,14 @@ pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const double* x, d
         }
         break;
     case PEPP_V_SELL:
-        pepp::k::sell_kernel<kBlock><<<p->grid_sell, kBlock, 0, st>>>((int)p->nrows, p->nchunks, p->d_chunk_ptr,
-                                                                       p->d_chunk_len, p->d_rowlen, p->d_perm,
-                                                                       p->d_scol, p->d_scol16, p->d_sval, x, y);
+        if (p->d_perm)
+            pepp::k::sell_kernel<kBlock, true><<<p->grid_sell, kBlock, 0, st>>>(
+                (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
+                p->d_scol16, p->d_sval, x, y, p->sell_cpw);
+        else
+            pepp::k::sell_kernel<kBlock, false><<<p->grid_sell, kBlock, 0, st>>>(
+                (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr, p->d_scol,
+                p->d_scol16, p->d_sval, x, y, 1);
         break;
     default:
         return PEPP_E_INVALID;
@@ -763,7 +770,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         const double mean = I.mean_row;
         uint32_t keep = mask;
         if ((double)I.max_row > std::max(4096.0, 256.0 * mean)) keep &= ~(1u << PEPP_V_CSR_VECTOR);
-        if ((double)I.max_row > std::max(256.0, 16.0 * mean)) keep &= ~(1u << PEPP_V_SELL);
+        if (I.max_row > 4096) keep &= ~(1u << PEPP_V_SELL);   // one lane would own a whole huge row
         if (keep & ((1u << PEPP_V_COUNT) - 1)) mask = keep;   // never prune everything
     }
     if (mask & (1u << PEPP_V_CSR_VECTOR))
@@ -792,7 +799,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     p->grid_csr[5] = grid_for((const void*)pepp::k::csr_vector_kernel<32, kBlock>, kBlock, A->nrows, kBlock / 32, p->sm_count);
     {   // SELL: exactly one resident wave; warps walk their chunks with prefetch
         int occ = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pepp::k::sell_kernel<kBlock>, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pepp::k::sell_kernel<kBlock, false>, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
         (void)cudaGetLastError();
         const int64_t need = ((int64_t)p->nchunks + kBlock / 32 - 1) / (kBlock / 32);
         const int64_t wave = (int64_t)p->sm_count * occ;
