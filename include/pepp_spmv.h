@@ -259,6 +259,56 @@ pepp_status_t pepp_spmv_flush_history(pepp_spmv_plan_t* p);
 pepp_status_t pepp_spmv_history_stats(const pepp_spmv_plan_t* p, int32_t cand,
                                       int64_t* count, double* mean_us, double* m2);
 
+/* ---- smart containers (paper §IV-D P@20045–21195) --
+   A vector whose payload may live in host memory (the master copy) and in
+   device memory at the same time, with a valid / outdated state per copy.
+   Copies move only when an access needs them (paper Fig. 3, P@22400–26903):
+     - device access for a component call: READ or READWRITE copies host ->
+       device if the device copy is outdated; WRITE-only copies nothing
+       ("the first component call only writes the data and hence no copy is
+       made", P@23793); any write marks the host copy outdated;
+     - host access (the paper's [] operator, element-wise R/W proxies): copies
+       device -> host if the host copy is outdated (also before a host write:
+       "data is copied back ... before the actual operation takes place");
+       a host write marks the device copy outdated.
+   Fig. 3's program (write, host read, readwrite, read, read, host write)
+   therefore makes 2 copies, where copying around every call makes 7.
+   Access modes: */
+#define PEPP_ACCESS_READ      1
+#define PEPP_ACCESS_WRITE     2
+#define PEPP_ACCESS_READWRITE 3
+#define PEPP_DEVICE_SIMULATED (-2)  /* state machine + counters only, no CUDA (CPU tests) */
+
+typedef struct pepp_vector_s pepp_vector_t;
+
+/* n fp64 elements. host: the master copy (borrowed, must outlive the vector)
+   or NULL to allocate one (pinned). device: CUDA ordinal, -1 = current, or
+   PEPP_DEVICE_SIMULATED. The device copy is allocated on first device use.
+   Errors: PEPP_E_INVALID, PEPP_E_NOMEM, PEPP_E_CUDA. */
+pepp_status_t pepp_vector_create(int64_t n, double* host, int32_t device, pepp_vector_t** out);
+/* Waits for outstanding device work on the vector, frees what it owns. NULL is a no-op. */
+pepp_status_t pepp_vector_destroy(pepp_vector_t* v);
+/* Host access with `mode`; *host receives the master copy, valid for `mode`
+   on return (blocks until any device work that uses the vector completed). */
+pepp_status_t pepp_vector_acquire_host(pepp_vector_t* v, int32_t mode, double** host);
+/* Device access with `mode` for work the caller enqueues on `stream`; the
+   needed copy (if any) is enqueued on `stream`; *dev receives the device copy
+   (NULL for a simulated vector). Call pepp_vector_release_device after
+   enqueueing the work. */
+pepp_status_t pepp_vector_acquire_device(pepp_vector_t* v, int32_t mode, void* stream, double** dev);
+/* Records the end of the device work on `stream` that used the vector. */
+pepp_status_t pepp_vector_release_device(pepp_vector_t* v, void* stream);
+/* Copies made so far (host->device, device->host) and bytes moved. */
+pepp_status_t pepp_vector_counters(const pepp_vector_t* v, int64_t* h2d, int64_t* d2h, int64_t* bytes);
+/* Current state: 1 = that copy is valid. */
+pepp_status_t pepp_vector_state(const pepp_vector_t* v, int32_t* host_valid, int32_t* device_valid);
+/* A READWRITE component on a vector: v = alpha * v on the device (stream-ordered). */
+pepp_status_t pepp_vector_scale(pepp_vector_t* v, double alpha, void* stream);
+/* y = A·x through containers: x READ, y WRITE (see pepp_spmv_exec for flags,
+   force, used). x and y must be distinct vectors of length ncols / global rows. */
+pepp_status_t pepp_spmv_exec_vec(pepp_spmv_plan_t* p, pepp_vector_t* x, pepp_vector_t* y, int flags,
+                                 void* stream, const pepp_choice_t* force, pepp_choice_t* used);
+
 /* ---- host-only utilities (no GPU needed) ---------------------------- */
 
 /* nnz-balanced contiguous row blocks (reading A9; P@27578):
