@@ -258,10 +258,13 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
         obj = [pepp.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
-    plan = pepp.Plan.from_csr(A, nranks=world, rank=rank, row_bounds=bounds if world > 1 else None,
-                              nccl_unique_id=uid, prune=not args.no_prune)
-    info = plan.info()
     force = parse_variant(args.variant)
+    # --variant pins the choice everywhere (timed steps and the e2e leg): the
+    # plan is built with that variant only
+    plan = pepp.Plan.from_csr(A, nranks=world, rank=rank, row_bounds=bounds if world > 1 else None,
+                              nccl_unique_id=uid, prune=not args.no_prune,
+                              variant_mask=(1 << force.variant) if force is not None else 0)
+    info = plan.info()
     flags = pepp.Y_NEXT_INPUT if iterated else pepp.Y_LOCAL
 
     stream = torch.cuda.Stream(device=dev)

@@ -20,7 +20,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 PKG = os.path.join(ROOT, "paper_conf_sc_dastgeerlk12_b200")
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libpepp_spmv.so")
-SOURCES = ["plan.cu", "host_util.cpp", "nccl_dl.cpp"]
+SOURCES = ["plan.cu", "containers.cu", "host_util.cpp", "nccl_dl.cpp"]
 HEADERS = ["kernels.cuh", "pepp_internal.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

@@ -19,10 +19,11 @@ from typing import Optional, Sequence
 import numpy as np
 
 from . import _capi as C
-from ._capi import (EXEC_NO_TIMING, PeppError, V_CSR_STREAM, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, X_ALLGATHER, X_AUTO,
+from ._capi import (ACCESS_READ, ACCESS_READWRITE, ACCESS_WRITE, DEVICE_SIMULATED, EXEC_NO_TIMING, PeppError, V_CSR_STREAM, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, X_ALLGATHER, X_AUTO,
                     X_HALO, X_NONE, Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, VARIANT_NAMES)
 
-__all__ = ["Plan", "Choice", "History", "partition_rows", "halo_ghosts", "context_key", "nccl_unique_id",
+__all__ = ["Plan", "Choice", "History", "Vector", "ACCESS_READ", "ACCESS_WRITE", "ACCESS_READWRITE",
+           "DEVICE_SIMULATED", "partition_rows", "halo_ghosts", "context_key", "nccl_unique_id",
            "lib_path", "PeppError", "V_CSR_VECTOR", "V_MERGE_PATH", "V_SELL", "V_CSR_STREAM", "X_AUTO", "X_NONE",
            "X_ALLGATHER", "X_HALO", "Y_LOCAL", "Y_NEXT_INPUT", "Y_REPLICATED", "EXEC_NO_TIMING",
            "VARIANT_NAMES"]
@@ -66,6 +67,8 @@ def _ptr(a) -> int:
 def _stream_handle(stream) -> int:
     if stream is None:
         import torch
+        if not torch.cuda.is_available():
+            return 0   # legacy default stream (the library reports PEPP_E_CUDA where a device is needed)
         return int(torch.cuda.current_stream().cuda_stream)
     if isinstance(stream, int):
         return stream
@@ -132,6 +135,16 @@ class Plan:
                 "pepp_spmv_exec")
         return Choice._from(used)
 
+    def exec_vec(self, x: "Vector", y: "Vector", flags: int = Y_LOCAL, stream=None,
+                 force: Optional[Choice] = None) -> Choice:
+        """y = A·x through smart containers (x READ, y WRITE); copies only what the states require."""
+        used = C.CHOICE_T()
+        f = force._to() if force is not None else None
+        C.check(C.lib().pepp_spmv_exec_vec(self._h, x._h, y._h, flags, _stream_handle(stream),
+                                           ctypes.byref(f) if f is not None else None, ctypes.byref(used)),
+                "pepp_spmv_exec_vec")
+        return Choice._from(used)
+
     def exchange(self, y, flags: int = Y_NEXT_INPUT, stream=None) -> None:
         """The exchange step alone (no-op on an unpartitioned plan)."""
         C.check(C.lib().pepp_spmv_exchange(self._h, _ptr(y), flags, _stream_handle(stream)), "pepp_spmv_exchange")
@@ -190,6 +203,71 @@ class Plan:
     def from_csr(cls, A, **kw) -> "Plan":
         """From any object with nrows, ncols, row_ptr, col, val (e.g. gen.CSR)."""
         return cls(A.nrows, A.ncols, A.row_ptr, A.col, A.val, **kw)
+
+
+class Vector:
+    """Smart container for one fp64 vector (pepp_vector_*): a host master copy
+    plus a lazily allocated device copy with valid / outdated states
+    (paper §IV-D, Fig. 3). ``host`` (numpy float64) is borrowed as the master
+    copy, or one is allocated (pinned)."""
+
+    def __init__(self, n: int, host: Optional[np.ndarray] = None, device: Optional[int] = None):
+        self._h = ctypes.c_void_p()
+        self._host_ref = None
+        hp = 0
+        if host is not None:
+            assert host.dtype == np.float64 and host.flags.c_contiguous and host.size == n
+            self._host_ref = host
+            hp = host.ctypes.data
+        C.check(C.lib().pepp_vector_create(n, hp or None, -1 if device is None else device, ctypes.byref(self._h)),
+                "pepp_vector_create")
+        self.n = n
+
+    def host(self, mode: int = ACCESS_READ) -> np.ndarray:
+        """Host access with `mode`: returns the (now valid) master copy as a numpy view."""
+        p = ctypes.c_void_p()
+        C.check(C.lib().pepp_vector_acquire_host(self._h, mode, ctypes.byref(p)), "pepp_vector_acquire_host")
+        if self._host_ref is not None:
+            return self._host_ref
+        return np.ctypeslib.as_array(ctypes.cast(p, ctypes.POINTER(ctypes.c_double)), shape=(self.n,))
+
+    def device(self, mode: int, stream=None) -> int:
+        """Device access with `mode` (copy enqueued if needed); returns the device pointer."""
+        p = ctypes.c_void_p()
+        C.check(C.lib().pepp_vector_acquire_device(self._h, mode, _stream_handle(stream) if stream is not False else None,
+                                                   ctypes.byref(p)), "pepp_vector_acquire_device")
+        return p.value or 0
+
+    def release(self, stream=None) -> None:
+        C.check(C.lib().pepp_vector_release_device(self._h, _stream_handle(stream) if stream is not False else None),
+                "pepp_vector_release_device")
+
+    def scale(self, alpha: float, stream=None) -> None:
+        """A READWRITE component: v = alpha * v on the device."""
+        C.check(C.lib().pepp_vector_scale(self._h, alpha, _stream_handle(stream) if stream is not False else None),
+                "pepp_vector_scale")
+
+    def counters(self) -> tuple[int, int, int]:
+        a, b, c = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        C.check(C.lib().pepp_vector_counters(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)),
+                "pepp_vector_counters")
+        return a.value, b.value, c.value
+
+    def state(self) -> tuple[bool, bool]:
+        h, d = ctypes.c_int32(), ctypes.c_int32()
+        C.check(C.lib().pepp_vector_state(self._h, ctypes.byref(h), ctypes.byref(d)), "pepp_vector_state")
+        return bool(h.value), bool(d.value)
+
+    def close(self) -> None:
+        if getattr(self, "_h", None) and self._h.value:
+            C.lib().pepp_vector_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 class History:

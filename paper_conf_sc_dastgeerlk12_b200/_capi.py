@@ -15,6 +15,8 @@ PEPP_OK, PEPP_E_INVALID, PEPP_E_CUDA, PEPP_E_NCCL, PEPP_E_NOMEM, PEPP_E_UNSUPPOR
 V_AUTO, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, V_CSR_STREAM, V_COUNT = -1, 0, 1, 2, 3, 4
 X_AUTO, X_NONE, X_ALLGATHER, X_HALO = -1, 0, 1, 2
 Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, EXEC_NO_TIMING = 0x0, 0x1, 0x2, 0x10
+ACCESS_READ, ACCESS_WRITE, ACCESS_READWRITE = 1, 2, 3
+DEVICE_SIMULATED = -2
 VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell", V_CSR_STREAM: "csr_stream"}
 EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_AUTO: "auto"}
 
@@ -70,6 +72,15 @@ SIGNATURES = {
     "pepp_spmv_candidates": (c_i32, [c_vp, ctypes.POINTER(CHOICE_T), c_i32, ctypes.POINTER(c_i32)]),
     "pepp_spmv_flush_history": (c_i32, [c_vp]),
     "pepp_spmv_history_stats": (c_i32, [c_vp, c_i32, ctypes.POINTER(c_i64), ctypes.POINTER(c_f64), ctypes.POINTER(c_f64)]),
+    "pepp_vector_create": (c_i32, [c_i64, c_vp, c_i32, ctypes.POINTER(c_vp)]),
+    "pepp_vector_destroy": (c_i32, [c_vp]),
+    "pepp_vector_acquire_host": (c_i32, [c_vp, c_i32, ctypes.POINTER(c_vp)]),
+    "pepp_vector_acquire_device": (c_i32, [c_vp, c_i32, c_vp, ctypes.POINTER(c_vp)]),
+    "pepp_vector_release_device": (c_i32, [c_vp, c_vp]),
+    "pepp_vector_counters": (c_i32, [c_vp, ctypes.POINTER(c_i64), ctypes.POINTER(c_i64), ctypes.POINTER(c_i64)]),
+    "pepp_vector_state": (c_i32, [c_vp, ctypes.POINTER(c_i32), ctypes.POINTER(c_i32)]),
+    "pepp_vector_scale": (c_i32, [c_vp, c_f64, c_vp]),
+    "pepp_spmv_exec_vec": (c_i32, [c_vp, c_vp, c_vp, ctypes.c_int, c_vp, ctypes.POINTER(CHOICE_T), ctypes.POINTER(CHOICE_T)]),
     "pepp_partition_rows": (c_i32, [c_vp, c_i64, c_i64, c_i32, c_vp]),
     "pepp_halo_ghosts": (c_i32, [c_vp, c_i64, c_i32, c_i32, c_vp, c_vp, c_vp, c_i64, ctypes.POINTER(c_i64)]),
     "pepp_history_create": (c_i32, [ctypes.POINTER(c_vp)]),

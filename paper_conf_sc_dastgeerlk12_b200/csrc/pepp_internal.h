@@ -29,6 +29,10 @@ int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const u
 uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts);
 void halo_ghost_list(const int32_t* col, int64_t nnz, int64_t lo, int64_t hi, std::vector<int32_t>& out);
 
+// ---- smart containers (containers.cu) ----
+int64_t vector_length(const pepp_vector_t* v);
+bool vector_simulated(const pepp_vector_t* v);
+
 // ---- NCCL, loaded on demand with dlopen (nccl_dl.cpp) ----
 // Only the handful of entry points the exchange needs; types mirror nccl.h
 // (NCCL 2.x ABI). No link-time dependency, so the library loads (and its

@@ -962,6 +962,25 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const doub
     return PEPP_OK;
 }
 
+extern "C" PEPP_API pepp_status_t pepp_spmv_exec_vec(pepp_spmv_plan_t* p, pepp_vector_t* x, pepp_vector_t* y, int flags,
+                                                    void* stream, const pepp_choice_t* force, pepp_choice_t* used) {
+    if (!p || !x || !y || x == y) return PEPP_E_INVALID;
+    if (pepp::vector_simulated(x) || pepp::vector_simulated(y)) return PEPP_E_INVALID;
+    if (pepp::vector_length(x) != p->ncols || pepp::vector_length(y) != p->global_rows) return PEPP_E_INVALID;
+    double *dx = nullptr, *dy = nullptr;
+    pepp_status_t s = pepp_vector_acquire_device(x, PEPP_ACCESS_READ, stream, &dx);
+    if (s) return s;
+    // y is written (A4): with an exchange, other ranks' rows are written too;
+    // without one, rows outside this block are left untouched, so a
+    // partitioned LOCAL call keeps y's device copy as the valid one
+    s = pepp_vector_acquire_device(y, PEPP_ACCESS_WRITE, stream, &dy);
+    if (s) return s;
+    s = pepp_spmv_exec(p, dx, dy, flags, stream, force, used);
+    const pepp_status_t s1 = pepp_vector_release_device(x, stream);
+    const pepp_status_t s2 = pepp_vector_release_device(y, stream);
+    return s ? s : (s1 ? s1 : s2);
+}
+
 extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, double* y, int flags, void* stream) {
     if (!p) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
