@@ -8,6 +8,15 @@
 // host master copy and one device copy; PEPP_DEVICE_SIMULATED runs the same
 // state machine without CUDA (counters only) so the protocol is testable on a
 // machine without a GPU.
+//
+// Inter-call parallelism (paper §IV-E P@21908–27091): the
+// container also records, per device access, an event on the caller's stream
+// — the latest writer, and the readers since that write. A device access on
+// any stream first waits (cudaStreamWaitEvent) for what its mode conflicts
+// with: READ after the last write (RAW), WRITE after the last write and after
+// every reader since (WAW, WAR). Calls on different streams are thus ordered
+// by their data dependencies alone, and read-only calls on one vector run
+// concurrently (Fig. 3, lines 10 and 12).
 #include "pepp_internal.h"
 
 #include <cuda_runtime.h>
@@ -28,6 +37,14 @@ struct pepp_vector_s {
     cudaEvent_t last_use = nullptr;   // end of the latest device work on the vector
     bool has_use = false;
     int64_t h2d = 0, d2h = 0, bytes = 0;
+    // dependency tracking (inter-call parallelism)
+    static constexpr int kMaxReaders = 16;
+    cudaEvent_t writer = nullptr;         // end of the latest writing access
+    bool has_writer = false;
+    cudaEvent_t readers[kMaxReaders] = {};
+    int nreaders = 0;                     // readers since the latest write
+    int32_t pending_mode = 0;             // mode of the access being released
+    int64_t waits = 0;                    // cross-stream dependency waits inserted
 };
 
 namespace {
@@ -37,8 +54,23 @@ inline bool writes(int32_t m) { return (m & PEPP_ACCESS_WRITE) != 0; }
 inline bool valid_mode(int32_t m) { return m == PEPP_ACCESS_READ || m == PEPP_ACCESS_WRITE || m == PEPP_ACCESS_READWRITE; }
 
 pepp_status_t wait_device(pepp_vector_t* v) {
-    if (v->simulated || !v->has_use) return PEPP_OK;
-    if (cudaEventSynchronize(v->last_use) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    if (v->simulated) return PEPP_OK;
+    bool ok = true;
+    if (v->has_writer) ok &= cudaEventSynchronize(v->writer) == cudaSuccess;
+    for (int i = 0; i < v->nreaders; ++i) ok &= cudaEventSynchronize(v->readers[i]) == cudaSuccess;
+    if (v->has_use) ok &= cudaEventSynchronize(v->last_use) == cudaSuccess;
+    if (!ok) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    return PEPP_OK;
+}
+
+// make `stream` wait for the accesses `mode` conflicts with
+pepp_status_t order_after(pepp_vector_t* v, int32_t mode, cudaStream_t stream) {
+    if (v->simulated) return PEPP_OK;
+    bool ok = true;
+    if (v->has_writer) { ok &= cudaStreamWaitEvent(stream, v->writer, 0) == cudaSuccess; ++v->waits; }   // RAW / WAW
+    if (writes(mode))
+        for (int i = 0; i < v->nreaders; ++i) { ok &= cudaStreamWaitEvent(stream, v->readers[i], 0) == cudaSuccess; ++v->waits; }  // WAR
+    if (!ok) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
     return PEPP_OK;
 }
 
@@ -68,9 +100,13 @@ extern "C" PEPP_API pepp_status_t pepp_vector_create(int64_t n, double* host, in
             return PEPP_E_CUDA;
         }
         cudaSetDevice(v->device);
-        if (cudaEventCreateWithFlags(&v->last_use, cudaEventDisableTiming) != cudaSuccess) {
+        bool ok = cudaEventCreateWithFlags(&v->last_use, cudaEventDisableTiming) == cudaSuccess &&
+                  cudaEventCreateWithFlags(&v->writer, cudaEventDisableTiming) == cudaSuccess;
+        for (int i = 0; ok && i < pepp_vector_t::kMaxReaders; ++i)
+            ok = cudaEventCreateWithFlags(&v->readers[i], cudaEventDisableTiming) == cudaSuccess;
+        if (!ok) {
             (void)cudaGetLastError();
-            delete v;
+            pepp_vector_destroy(v);
             return PEPP_E_CUDA;
         }
     }
@@ -97,6 +133,8 @@ extern "C" PEPP_API pepp_status_t pepp_vector_destroy(pepp_vector_t* v) {
         (void)wait_device(v);
         if (v->dev) cudaFree(v->dev);
         if (v->last_use) cudaEventDestroy(v->last_use);
+        if (v->writer) cudaEventDestroy(v->writer);
+        for (auto& e : v->readers) if (e) cudaEventDestroy(e);
     }
     if (v->own_host) {
         if (v->pinned) cudaFreeHost(v->host);
@@ -139,6 +177,11 @@ extern "C" PEPP_API pepp_status_t pepp_vector_acquire_device(pepp_vector_t* v, i
             }
         }
     }
+    {
+        pepp_status_t so = order_after(v, mode, (cudaStream_t)stream);
+        if (so) return so;
+    }
+    v->pending_mode = mode;
     if (reads(mode) && !v->dev_valid) {
         if (!v->host_valid) return PEPP_E_STATE;   // no valid copy anywhere (cannot happen through this API)
         if (!v->simulated && v->n > 0 &&
@@ -149,6 +192,13 @@ extern "C" PEPP_API pepp_status_t pepp_vector_acquire_device(pepp_vector_t* v, i
         }
         v->h2d += 1;
         v->bytes += (int64_t)sizeof(double) * v->n;
+        // the copy in writes the device copy: later accesses on other streams
+        // must order after it
+        if (!v->simulated) {
+            if (cudaEventRecord(v->writer, (cudaStream_t)stream) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+            v->has_writer = true;
+            v->nreaders = 0;
+        }
     }
     // write-only: no copy in, only the allocation ("just a memory allocation
     // is made in the device memory where data is written", P@23793)
@@ -161,7 +211,23 @@ extern "C" PEPP_API pepp_status_t pepp_vector_acquire_device(pepp_vector_t* v, i
 extern "C" PEPP_API pepp_status_t pepp_vector_release_device(pepp_vector_t* v, void* stream) {
     if (!v) return PEPP_E_INVALID;
     if (v->simulated) return PEPP_OK;
-    if (cudaEventRecord(v->last_use, (cudaStream_t)stream) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    cudaStream_t st = (cudaStream_t)stream;
+    bool ok = cudaEventRecord(v->last_use, st) == cudaSuccess;
+    if (writes(v->pending_mode)) {
+        ok &= cudaEventRecord(v->writer, st) == cudaSuccess;
+        v->has_writer = true;
+        v->nreaders = 0;
+    } else if (v->nreaders < pepp_vector_t::kMaxReaders) {
+        ok &= cudaEventRecord(v->readers[v->nreaders++], st) == cudaSuccess;
+    } else {
+        // too many concurrent readers to track: fold them into one by making
+        // this stream wait for all of them, then record a single reader
+        for (int i = 0; i < v->nreaders; ++i) ok &= cudaStreamWaitEvent(st, v->readers[i], 0) == cudaSuccess;
+        ok &= cudaEventRecord(v->readers[0], st) == cudaSuccess;
+        v->nreaders = 1;
+    }
+    v->pending_mode = 0;
+    if (!ok) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
     v->has_use = true;
     return PEPP_OK;
 }

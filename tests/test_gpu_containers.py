@@ -81,3 +81,31 @@ def test_exec_vec_rejects_bad_arguments():
         sim = pepp.Vector(64, device=pepp.DEVICE_SIMULATED)
         with pytest.raises(pepp.PeppError):
             plan.exec_vec(sim, v)                    # simulated containers cannot feed kernels
+
+
+def test_dependencies_across_streams_raw_war():
+    """Inter-call parallelism: calls on different streams
+    with no explicit synchronisation are ordered by their access modes alone.
+    Large vectors make an unordered run visibly wrong."""
+    n = 2048
+    A = gen.laplacian2d(n)
+    N = n * n
+    x0 = gen.vector(3, gen.INT8, N)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    with pepp.Plan.from_csr(A) as plan:
+        u = pepp.Vector(N, host=x0.copy())
+        v, w1, w2, w3 = (pepp.Vector(N) for _ in range(4))
+        for _ in range(3):
+            plan.exec_vec(u, v, stream=s1)          # v written on s1
+            plan.exec_vec(v, w1, stream=s2)         # RAW: s2 must wait for s1
+            plan.exec_vec(v, w2, stream=s1)         # read-read: may overlap with the s2 read
+            plan.exec_vec(v, w3, stream=s2)
+            v.scale(3.0, stream=s1)                 # WAR: must wait for both readers (s1 and s2)
+            ref_v = oracle.spmv(A, x0)
+            ref_w = oracle.spmv(A, ref_v)
+            assert np.array_equal(w1.host(R), ref_w)
+            assert np.array_equal(w2.host(R), ref_w)
+            assert np.array_equal(w3.host(R), ref_w)
+            assert np.array_equal(v.host(R), 3.0 * ref_v)
+        for c in (u, v, w1, w2, w3):
+            c.close()
