@@ -259,6 +259,26 @@ pepp_status_t pepp_spmv_flush_history(pepp_spmv_plan_t* p);
 pepp_status_t pepp_spmv_history_stats(const pepp_spmv_plan_t* p, int32_t cand,
                                       int64_t* count, double* mean_us, double* m2);
 
+/* ---- CUDA graphs for launch-bound calls --------------------------------
+   Small matrices (BASELINE config 1: 20 K nonzeros, a few µs of work) are
+   bound by launch and host overhead, like the paper's ODE solver making
+   10,613 small component calls (Fig. 7, P@41298). A graph captures
+   `iterations` calls once — the variant the selector would choose now, with
+   its exchange — and replays them with one launch.
+   mode 0 (repeat): every call computes y = A·x (same x, same y).
+   mode 1 (iterate): x_{k+1} = A·x_k, ping-pong between y and `work`
+   (device, same length as y; x is read only by the first call); the result
+   of the last call is in y when `iterations` is odd, else in work.
+   x, y, work: device buffers that must stay valid while the graph exists.
+   Timing events are not recorded inside graphs (history is not updated by
+   replays). Errors: PEPP_E_INVALID, PEPP_E_CUDA, PEPP_E_NCCL. */
+typedef struct pepp_spmv_graph_s pepp_spmv_graph_t;
+pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, const double* x, double* y, double* work,
+                                     int32_t iterations, int32_t mode, int flags, void* stream,
+                                     pepp_spmv_graph_t** out);
+pepp_status_t pepp_spmv_graph_launch(pepp_spmv_graph_t* g, void* stream);
+pepp_status_t pepp_spmv_graph_destroy(pepp_spmv_graph_t* g);
+
 /* ---- smart containers (paper §IV-D P@20045–21195) --
    A vector whose payload may live in host memory (the master copy) and in
    device memory at the same time, with a valid / outdated state per copy.

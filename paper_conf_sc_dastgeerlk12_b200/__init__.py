@@ -145,6 +145,15 @@ class Plan:
                 "pepp_spmv_exec_vec")
         return Choice._from(used)
 
+    def graph(self, x, y, iterations: int = 1, mode: int = 0, work=None, flags: int = Y_LOCAL,
+              stream=None) -> "Graph":
+        """Capture `iterations` calls into a CUDA graph (mode 0: repeat y = A·x;
+        mode 1: iterate, ping-pong y / work)."""
+        g = ctypes.c_void_p()
+        C.check(C.lib().pepp_spmv_graph_create(self._h, _ptr(x), _ptr(y), _ptr(work), iterations, mode, flags,
+                                               _stream_handle(stream), ctypes.byref(g)), "pepp_spmv_graph_create")
+        return Graph(g, (x, y, work))
+
     def exchange(self, y, flags: int = Y_NEXT_INPUT, stream=None) -> None:
         """The exchange step alone (no-op on an unpartitioned plan)."""
         C.check(C.lib().pepp_spmv_exchange(self._h, _ptr(y), flags, _stream_handle(stream)), "pepp_spmv_exchange")
@@ -203,6 +212,28 @@ class Plan:
     def from_csr(cls, A, **kw) -> "Plan":
         """From any object with nrows, ncols, row_ptr, col, val (e.g. gen.CSR)."""
         return cls(A.nrows, A.ncols, A.row_ptr, A.col, A.val, **kw)
+
+
+class Graph:
+    """A captured sequence of SpMV calls (pepp_spmv_graph_*)."""
+
+    def __init__(self, h, keep):
+        self._h = h
+        self._keep = keep   # the buffers the graph reads / writes must stay alive
+
+    def launch(self, stream=None) -> None:
+        C.check(C.lib().pepp_spmv_graph_launch(self._h, _stream_handle(stream)), "pepp_spmv_graph_launch")
+
+    def close(self) -> None:
+        if self._h and self._h.value:
+            C.lib().pepp_spmv_graph_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 class Vector:

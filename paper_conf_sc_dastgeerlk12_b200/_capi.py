@@ -72,6 +72,9 @@ SIGNATURES = {
     "pepp_spmv_candidates": (c_i32, [c_vp, ctypes.POINTER(CHOICE_T), c_i32, ctypes.POINTER(c_i32)]),
     "pepp_spmv_flush_history": (c_i32, [c_vp]),
     "pepp_spmv_history_stats": (c_i32, [c_vp, c_i32, ctypes.POINTER(c_i64), ctypes.POINTER(c_f64), ctypes.POINTER(c_f64)]),
+    "pepp_spmv_graph_create": (c_i32, [c_vp, c_vp, c_vp, c_vp, c_i32, c_i32, ctypes.c_int, c_vp, ctypes.POINTER(c_vp)]),
+    "pepp_spmv_graph_launch": (c_i32, [c_vp, c_vp]),
+    "pepp_spmv_graph_destroy": (c_i32, [c_vp]),
     "pepp_vector_create": (c_i32, [c_i64, c_vp, c_i32, ctypes.POINTER(c_vp)]),
     "pepp_vector_destroy": (c_i32, [c_vp]),
     "pepp_vector_acquire_host": (c_i32, [c_vp, c_i32, ctypes.POINTER(c_vp)]),

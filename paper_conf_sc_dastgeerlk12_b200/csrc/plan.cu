@@ -962,6 +962,81 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const doub
     return PEPP_OK;
 }
 
+struct pepp_spmv_graph_s {
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
+    int device = 0;
+};
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, const double* x, double* y, double* work,
+                                                        int32_t iterations, int32_t mode, int flags, void* stream,
+                                                        pepp_spmv_graph_t** out) {
+    if (!out) return PEPP_E_INVALID;
+    *out = nullptr;
+    if (!p || iterations < 1 || (mode != 0 && mode != 1) || (mode == 1 && iterations > 1 && !work)) return PEPP_E_INVALID;
+    if (mode == 1 && p->ncols != p->global_rows) return PEPP_E_INVALID;
+    if (p->sticky) return p->sticky;
+    if (cudaSetDevice(p->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    // choose once, outside the capture (calibration calls would not be timed)
+    pepp_choice_t ch{};
+    pepp_status_t s = select_choice(p, &ch);
+    if (s) return s;
+    cudaStream_t st = (cudaStream_t)stream;
+    cudaStream_t cap = nullptr;
+    if (cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    pepp_spmv_graph_t* g = new (std::nothrow) pepp_spmv_graph_t();
+    if (!g) { cudaStreamDestroy(cap); return PEPP_E_NOMEM; }
+    g->device = p->device;
+    bool ok = cudaStreamBeginCapture(cap, cudaStreamCaptureModeRelaxed) == cudaSuccess;
+    const double* in = x;
+    double* outb = y;
+    for (int32_t it = 0; ok && it < iterations; ++it) {
+        s = pepp_spmv_exec(p, in, outb, flags | PEPP_EXEC_NO_TIMING, cap, &ch, nullptr);
+        if (s) ok = false;
+        if (mode == 1) {
+            in = outb;
+            outb = (outb == y) ? work : y;
+        }
+    }
+    cudaGraph_t graph = nullptr;
+    const bool ended = cudaStreamEndCapture(cap, &graph) == cudaSuccess;
+    cudaStreamDestroy(cap);
+    if (!ok || !ended || !graph) {
+        (void)cudaGetLastError();
+        if (graph) cudaGraphDestroy(graph);
+        delete g;
+        return s ? s : PEPP_E_CUDA;
+    }
+    g->graph = graph;
+    if (cudaGraphInstantiate(&g->exec, graph, 0) != cudaSuccess) {
+        (void)cudaGetLastError();
+        cudaGraphDestroy(graph);
+        delete g;
+        return PEPP_E_CUDA;
+    }
+    if (cudaGraphUpload(g->exec, st) != cudaSuccess) (void)cudaGetLastError();   // pre-stage on the caller's stream
+    *out = g;
+    return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_graph_launch(pepp_spmv_graph_t* g, void* stream) {
+    if (!g) return PEPP_E_INVALID;
+    if (cudaSetDevice(g->device) != cudaSuccess || cudaGraphLaunch(g->exec, (cudaStream_t)stream) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return PEPP_E_CUDA;
+    }
+    return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_graph_destroy(pepp_spmv_graph_t* g) {
+    if (!g) return PEPP_OK;
+    cudaSetDevice(g->device);
+    if (g->exec) cudaGraphExecDestroy(g->exec);
+    if (g->graph) cudaGraphDestroy(g->graph);
+    delete g;
+    return PEPP_OK;
+}
+
 extern "C" PEPP_API pepp_status_t pepp_spmv_exec_vec(pepp_spmv_plan_t* p, pepp_vector_t* x, pepp_vector_t* y, int flags,
                                                     void* stream, const pepp_choice_t* force, pepp_choice_t* used) {
     if (!p || !x || !y || x == y) return PEPP_E_INVALID;

@@ -378,3 +378,28 @@ def test_sell_col16_used_and_exact_on_stencils():
         assert 0.0 < f < 1.0
         y, _ = _run(plan, x)
     assert np.array_equal(y, oracle.spmv(B, x))
+
+
+def test_graph_repeat_and_iterate_match_oracle():
+    A = gen.laplacian2d(64)
+    x0 = gen.vector(1, gen.INT8, 4096)
+    with pepp.Plan.from_csr(A) as plan:
+        x = _dev(x0)
+        y = torch.empty(4096, dtype=torch.float64, device="cuda")
+        w = torch.empty_like(y)
+        g = plan.graph(x, y, iterations=100, mode=0)
+        for _ in range(3):
+            g.launch()
+        torch.cuda.synchronize()
+        assert np.array_equal(y.cpu().numpy(), oracle.spmv(A, x0))
+        g.close()
+        for K in (1, 15, 16):
+            g = plan.graph(x, y, iterations=K, mode=1, work=w)
+            g.launch()
+            g.launch()   # replays are idempotent: x is only read by the first call
+            torch.cuda.synchronize()
+            res = (y if K % 2 == 1 else w).cpu().numpy()
+            assert np.array_equal(res, oracle.iterate(A, x0, K))
+            g.close()
+        with pytest.raises(pepp.PeppError):
+            plan.graph(x, y, iterations=4, mode=1)   # iterate needs a work buffer
