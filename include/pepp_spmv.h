@@ -138,7 +138,9 @@ typedef struct {
                                  0 = every variant is a candidate (variant_mask still applies). */
 } pepp_spmv_opts_t;
 
-/* Selection result. `candidate` indexes pepp_spmv_candidates(). */
+/* Selection result. `candidate` indexes pepp_spmv_candidates(). The plan's
+   history records each candidate under the stable id (variant << 20 | param),
+   so a persisted history (history_path) means the same across plans. */
 typedef struct {
     int32_t variant;          /* pepp_variant_t */
     int32_t param;            /* TPR (CSR_VECTOR), σ (SELL), items per thread (MERGE_PATH), nnz per item (CSR_STREAM) */
@@ -169,6 +171,7 @@ typedef struct {
     int64_t halo_recv;        /* ghost entries received per exchange (halo) */
     int64_t halo_send;        /* entries sent per exchange (halo) */
     double sell_col16_frac;   /* fraction of SELL chunks storing 16-bit column deltas */
+    uint64_t prior_key;       /* context key the cold-start prior came from (0 = none) */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */
@@ -372,6 +375,15 @@ pepp_status_t pepp_history_stats(const pepp_history* h, uint64_t key, int32_t ca
 pepp_status_t pepp_history_select(const pepp_history* h, uint64_t key, int32_t ncand,
                                   const uint8_t* eligible, int32_t min_samples,
                                   int32_t* cand, int32_t* calibrating, double* predicted_us);
+/* Cold-start prior (static composition from recorded runs, P@10069, P@10489):
+   the nearest context key to `key` (L1 distance over the bucket fields of
+   pepp_context_key; same rank count) that has samples for some of the
+   candidate ids ids[0..n); prior[c] = that key's mean for ids[c] (-1 if it
+   has none). PEPP_E_STATE if no such key exists. A plan with an unseen key
+   uses this prior (from a loaded history_path) to calibrate the predicted
+   best candidate first and to skip candidates predicted > 4x slower. */
+pepp_status_t pepp_history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t* ids,
+                                 double* prior, uint64_t* from_key);
 pepp_status_t pepp_history_save(const pepp_history* h, const char* path);
 pepp_status_t pepp_history_load(pepp_history* h, const char* path);
 

@@ -324,6 +324,17 @@ class History:
                                             ctypes.byref(cal), ctypes.byref(pred)), "pepp_history_select")
         return c.value, bool(cal.value), pred.value
 
+    def prior(self, key: int, ids: Sequence[int]):
+        """(prior means per id or -1, source key) from the nearest recorded context, or None."""
+        a = np.ascontiguousarray(ids, dtype=np.int32)
+        out = np.empty(len(a), dtype=np.float64)
+        k = ctypes.c_uint64()
+        st = C.lib().pepp_history_prior(self._h, key, len(a), a.ctypes.data, out.ctypes.data, ctypes.byref(k))
+        if st == C.PEPP_E_STATE:
+            return None
+        C.check(st, "pepp_history_prior")
+        return out, k.value
+
     def save(self, path: str) -> None:
         C.check(C.lib().pepp_history_save(self._h, path.encode()), "pepp_history_save")
 

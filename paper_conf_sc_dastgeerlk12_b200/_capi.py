@@ -52,7 +52,8 @@ class INFO_T(ctypes.Structure):
                 ("max_row", c_i64), ("empty_rows", c_i64), ("nranks", c_i32), ("rank", c_i32),
                 ("row_offset", c_i64), ("key", c_u64), ("ncandidates", c_i32), ("sell_sigma", c_i32),
                 ("sell_fill", c_f64), ("device_bytes", c_i64), ("algorithmic_bytes", c_i64),
-                ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64)]
+                ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64),
+                ("prior_key", c_u64)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -91,6 +92,7 @@ SIGNATURES = {
     "pepp_history_record": (c_i32, [c_vp, c_u64, c_i32, c_f64]),
     "pepp_history_stats": (c_i32, [c_vp, c_u64, c_i32, ctypes.POINTER(c_i64), ctypes.POINTER(c_f64), ctypes.POINTER(c_f64)]),
     "pepp_history_select": (c_i32, [c_vp, c_u64, c_i32, c_vp, c_i32, ctypes.POINTER(c_i32), ctypes.POINTER(c_i32), ctypes.POINTER(c_f64)]),
+    "pepp_history_prior": (c_i32, [c_vp, c_u64, c_i32, c_vp, c_vp, ctypes.POINTER(c_u64)]),
     "pepp_history_save": (c_i32, [c_vp, ctypes.c_char_p]),
     "pepp_history_load": (c_i32, [c_vp, ctypes.c_char_p]),
     "pepp_context_key": (c_u64, [c_i64, c_i64, c_i64, c_f64, c_i32]),

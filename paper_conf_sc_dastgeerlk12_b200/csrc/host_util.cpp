@@ -187,6 +187,38 @@ int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const u
     return best;
 }
 
+// Cold start (static composition from recorded runs, P@10069 / P@10489): the
+// nearest context key (bucket distance; same tag and rank count) that has
+// samples for some of the given candidate ids; their means become a prior.
+bool history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t* ids, double* prior,
+                   uint64_t* from_key) {
+    auto field = [](uint64_t k, int shift, uint64_t mask) { return (int64_t)((k >> shift) & mask); };
+    auto dist = [&](uint64_t a, uint64_t b) -> int64_t {
+        if ((a >> 27) != (b >> 27)) return -1;   // ranks + tag must match
+        return std::llabs(field(a, 0, 0x7f) - field(b, 0, 0x7f)) + std::llabs(field(a, 7, 0x7f) - field(b, 7, 0x7f)) +
+               std::llabs(field(a, 14, 0x7f) - field(b, 14, 0x7f)) + std::llabs(field(a, 21, 0x3f) - field(b, 21, 0x3f));
+    };
+    int64_t best_d = -1;
+    uint64_t best_k = 0;
+    for (const auto& kv : h->table) {
+        const uint64_t k = kv.first.key;
+        if (k == key || kv.second.count == 0) continue;
+        bool ours = false;
+        for (int32_t c = 0; c < n && !ours; ++c) ours = ids[c] == kv.first.cand;
+        if (!ours) continue;
+        const int64_t d = dist(key, k);
+        if (d < 0) continue;
+        if (best_d < 0 || d < best_d || (d == best_d && k < best_k)) { best_d = d; best_k = k; }
+    }
+    if (best_d < 0) return false;
+    for (int32_t c = 0; c < n; ++c) {
+        const Welford* w = history_get(h, best_k, ids[c]);
+        prior[c] = (w && w->count > 0) ? w->mean : -1.0;
+    }
+    if (from_key) *from_key = best_k;
+    return true;
+}
+
 uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts) {
     // bucketed context instance: half-octave buckets of rows / cols / nnz,
     // quarter buckets of the row-length CV (capped), and the partition count.
@@ -240,6 +272,12 @@ extern "C" PEPP_API pepp_status_t pepp_history_select(const pepp_history* h, uin
     if (!any) return PEPP_E_INVALID;
     *cand = pepp::history_pick(h, key, ncand, eligible, min_samples < 1 ? 1 : min_samples, calibrating, predicted_us);
     return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t* ids,
+                                                    double* prior, uint64_t* from_key) {
+    if (!h || n < 0 || (n > 0 && (!ids || !prior))) return PEPP_E_INVALID;
+    return pepp::history_prior(h, key, n, ids, prior, from_key) ? PEPP_OK : PEPP_E_STATE;
 }
 
 extern "C" PEPP_API pepp_status_t pepp_history_save(const pepp_history* h, const char* path) {

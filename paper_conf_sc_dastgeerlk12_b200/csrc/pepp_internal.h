@@ -27,6 +27,8 @@ bool history_abandoned(const Welford* w, double best_mean);
 int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible,
                      int32_t min_samples, int32_t* calibrating, double* predicted_us);
 uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts);
+bool history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t* ids, double* prior,
+                   uint64_t* from_key);
 void halo_ghost_list(const int32_t* col, int64_t nnz, int64_t lo, int64_t hi, std::vector<int32_t>& out);
 
 // ---- smart containers (containers.cu) ----

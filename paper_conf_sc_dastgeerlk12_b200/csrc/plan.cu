@@ -131,6 +131,10 @@ struct pepp_spmv_plan_s {
     int ring_head = 0;   // oldest pending
     int ring_count = 0;
     std::vector<int32_t> pending;   // timed calls in flight per candidate
+    std::vector<int32_t> uids;      // stable candidate identity in the history: variant << 20 | param
+    std::vector<double> prior;      // cold-start means from the nearest recorded context (-1 = none)
+    std::vector<int32_t> order;     // calibration order (predicted best first)
+    uint64_t prior_key = 0;
 
     // multi-GPU
     const Nccl* nccl = nullptr;
@@ -458,7 +462,7 @@ void harvest(pepp_spmv_plan_t* p, bool block) {
         if (q == cudaErrorNotReady) { (void)cudaGetLastError(); break; }
         float ms = 0.f;
         if (q == cudaSuccess && cudaEventElapsedTime(&ms, r.start, r.stop) == cudaSuccess)
-            pepp::history_add(p->hist, p->key, r.cand, (double)ms * 1000.0);
+            pepp::history_add(p->hist, p->key, p->uids[r.cand], (double)ms * 1000.0);
         (void)cudaGetLastError();
         r.pending = false;
         if (r.cand >= 0 && r.cand < (int)p->pending.size()) --p->pending[r.cand];
@@ -508,29 +512,65 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out) {
         // has min_samples calls issued, wait for them once and exploit.
         const int32_t ms = std::max(1, p->opts.min_samples);
         const int32_t n = (int32_t)p->cands.size();
+        auto hget = [&](int32_t c) { return pepp::history_get(p->hist, p->key, p->uids[c]); };
+        double best_mean = -1.0;
+        for (int32_t c = 0; c < n; ++c) {
+            const pepp::Welford* w = hget(c);
+            if (p->eligible[c] && w && w->count > 0 && (best_mean < 0 || w->mean < best_mean)) best_mean = w->mean;
+        }
+        double prior_best = -1.0;
+        for (int32_t c = 0; c < n; ++c)
+            if (p->eligible[c] && p->prior[c] > 0 && (prior_best < 0 || p->prior[c] < prior_best)) prior_best = p->prior[c];
+        // ruled out: own samples > 4x the best own mean, or (never sampled) a
+        // prior > 4x the best prior from the nearest recorded context
+        auto ruled_out = [&](int32_t c, const pepp::Welford* w) {
+            if (pepp::history_abandoned(w, best_mean)) return true;
+            return (!w || w->count == 0) && prior_best > 0 && p->prior[c] > pepp::kAbandonFactor * prior_best;
+        };
         cand = -1;
         for (int32_t r = 1; r <= ms && cand < 0; ++r) {
             // round r: every candidate not yet ruled out gets its r-th timed call
             // (calls still in flight count, so the host can run ahead of the GPU)
             for (int pass = 0; pass < 2 && cand < 0; ++pass) {
-                const double best_mean = pepp::history_best_mean(p->hist, p->key, n, p->eligible.data());
                 bool waiting = false;
-                for (int32_t c = 0; c < n; ++c) {
+                for (int32_t oi = 0; oi < n; ++oi) {
+                    const int32_t c = p->order[oi];
                     if (!p->eligible[c]) continue;
-                    const pepp::Welford* w = pepp::history_get(p->hist, p->key, c);
-                    if (pepp::history_abandoned(w, best_mean)) continue;
+                    const pepp::Welford* w = hget(c);
+                    if (ruled_out(c, w)) continue;
                     const int64_t done = w ? w->count : 0;
-                    if (done + p->pending[c] < r) { cand = c; calibrating = 1; pred = w ? w->mean : 0.0; break; }
+                    if (done + p->pending[c] < r) {
+                        cand = c; calibrating = 1;
+                        pred = w && w->count ? w->mean : (p->prior[c] > 0 ? p->prior[c] : 0.0);
+                        break;
+                    }
                     if (done < r) waiting = true;
                 }
                 // the round is fully issued but not measured: wait for it once, so
                 // the next round can rule out candidates from their timings
-                if (cand < 0 && waiting) harvest(p, true);
-                else break;
+                if (cand < 0 && waiting) {
+                    harvest(p, true);
+                    best_mean = -1.0;
+                    for (int32_t c = 0; c < n; ++c) {
+                        const pepp::Welford* w = hget(c);
+                        if (p->eligible[c] && w && w->count > 0 && (best_mean < 0 || w->mean < best_mean)) best_mean = w->mean;
+                    }
+                } else {
+                    break;
+                }
             }
         }
-        if (cand < 0)
-            cand = pepp::history_pick(p->hist, p->key, n, p->eligible.data(), ms, &calibrating, &pred);
+        if (cand < 0) {
+            // exploitation: argmin of the measured means, ties within 1 % -> lower index (A10)
+            double bt = 0.0;
+            for (int32_t c = 0; c < n; ++c) {
+                const pepp::Welford* w = hget(c);
+                if (!p->eligible[c] || !w || w->count == 0) continue;
+                if (cand < 0 || w->mean < bt * 0.99) { cand = c; bt = w->mean; }
+            }
+            calibrating = 0;
+            pred = bt;
+        }
     } else {
         cand = heuristic_candidate(p);
     }
@@ -815,6 +855,21 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     p->hist = pepp::history_new();
     if (!p->hist) return PEPP_E_NOMEM;
     if (!p->history_path.empty()) (void)pepp_history_load(p->hist, p->history_path.c_str());
+    {
+        const int32_t n = (int32_t)p->cands.size();
+        p->uids.resize(n);
+        for (int32_t c = 0; c < n; ++c) p->uids[c] = (p->cands[c].variant << 20) | (p->cands[c].param & 0xFFFFF);
+        p->prior.assign(n, -1.0);
+        p->order.resize(n);
+        for (int32_t c = 0; c < n; ++c) p->order[c] = c;
+        if (n && pepp::history_prior(p->hist, p->key, n, p->uids.data(), p->prior.data(), &p->prior_key)) {
+            p->info.prior_key = p->prior_key;
+            std::stable_sort(p->order.begin(), p->order.end(), [&](int32_t a, int32_t b) {
+                const double pa = p->prior[a] > 0 ? p->prior[a] : 1e300, pb = p->prior[b] > 0 ? p->prior[b] : 1e300;
+                return pa < pb;
+            });
+        }
+    }
     for (auto& r : p->ring) {
         PEPP_CUDA_TRY(cudaEventCreate(&r.start));
         PEPP_CUDA_TRY(cudaEventCreate(&r.stop));
@@ -1129,7 +1184,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_candidates(const pepp_spmv_plan_t* p
     *n = (int32_t)p->cands.size();
     for (int32_t i = 0; out && i < cap && i < *n; ++i) {
         fill_choice(p, i, 0, 0.0, &out[i]);
-        const pepp::Welford* w = pepp::history_get(p->hist, p->key, i);
+        const pepp::Welford* w = pepp::history_get(p->hist, p->key, p->uids[i]);
         out[i].predicted_us = w ? w->mean : 0.0;
     }
     return PEPP_OK;
@@ -1144,6 +1199,6 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_flush_history(pepp_spmv_plan_t* p) {
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_history_stats(const pepp_spmv_plan_t* p, int32_t cand, int64_t* count,
                                                          double* mean_us, double* m2) {
-    if (!p) return PEPP_E_INVALID;
-    return pepp_history_stats(p->hist, p->key, cand, count, mean_us, m2);
+    if (!p || cand < 0 || cand >= (int32_t)p->cands.size()) return PEPP_E_INVALID;
+    return pepp_history_stats(p->hist, p->key, p->uids[cand], count, mean_us, m2);
 }

@@ -403,3 +403,31 @@ def test_graph_repeat_and_iterate_match_oracle():
             g.close()
         with pytest.raises(pepp.PeppError):
             plan.graph(x, y, iterations=4, mode=1)   # iterate needs a work buffer
+
+
+def test_cold_start_from_persisted_history(tmp_path):
+    """A plan on an unseen context, loading a history file recorded on a
+    similar matrix, calibrates the predicted best first and skips candidates
+    the neighbour measured > 4x slower."""
+    hist = str(tmp_path / "h.txt")
+    A = gen.laplacian2d(1024)                # wide vector-CSR variants are 7-13x slower here
+    x = _dev(gen.vector(45, gen.REAL, A.nrows))
+    y = torch.empty(A.nrows, dtype=torch.float64, device="cuda")
+    with pepp.Plan.from_csr(A, history_path=hist) as plan:
+        assert plan.info()["prior_key"] == 0
+        calls_a = 0
+        while plan.exec(x, y).calibrating:
+            calls_a += 1
+        best_a = plan.select()
+    B = gen.laplacian2d(1200)
+    xb = _dev(gen.vector(46, gen.REAL, B.nrows))
+    yb = torch.empty(B.nrows, dtype=torch.float64, device="cuda")
+    with pepp.Plan.from_csr(B, history_path=hist) as plan:
+        info = plan.info()
+        assert info["prior_key"] != 0 and info["key"] != info["prior_key"]
+        first = plan.exec(xb, yb)
+        assert first.calibrating and (first.variant, first.param) == (best_a.variant, best_a.param)
+        calls_b = 1
+        while plan.exec(xb, yb).calibrating:
+            calls_b += 1
+        assert calls_b < calls_a          # the prior ruled some candidates out

@@ -159,3 +159,31 @@ def test_context_key_buckets():
     assert k != pepp.context_key(1 << 22, 1 << 20, 16 << 20, 0.0)
     assert k != pepp.context_key(1 << 20, 1 << 20, 16 << 20, 3.0)
     assert k != pepp.context_key(1 << 20, 1 << 20, 16 << 20, 0.0, nparts=2)
+
+
+def test_cold_start_prior_from_nearest_context():
+    """Static composition from recorded runs: an unseen context borrows the
+    means of the nearest recorded context (bucket distance, same rank count)."""
+    H = pepp.History()
+    k_small = pepp.context_key(1 << 16, 1 << 16, 16 << 16, 0.0)
+    k_big = pepp.context_key(1 << 24, 1 << 24, 16 << 24, 0.0)
+    k_other_ranks = pepp.context_key(1 << 20, 1 << 20, 16 << 20, 0.0, nparts=2)
+    ids = [10, 20, 30]
+    for cid, t in zip(ids, (5.0, 2.0, 9.0)):
+        H.record(k_small, cid, t)
+    for cid, t in zip(ids, (50.0, 80.0, 20.0)):
+        H.record(k_big, cid, t)
+    H.record(k_other_ranks, 10, 1.0)
+    q = pepp.context_key(1 << 17, 1 << 17, 16 << 17, 0.1)        # nearer to k_small
+    prior, src = H.prior(q, ids)
+    assert src == k_small and prior.tolist() == [5.0, 2.0, 9.0]
+    q2 = pepp.context_key(1 << 23, 1 << 23, 16 << 23, 0.0)       # nearer to k_big
+    prior, src = H.prior(q2, ids)
+    assert src == k_big and prior.tolist() == [50.0, 80.0, 20.0]
+    # ids the neighbour never ran get -1; unknown ids only -> no prior
+    prior, _ = H.prior(q, [20, 99])
+    assert prior.tolist() == [2.0, -1.0]
+    assert H.prior(q, [99]) is None
+    # a context with a different rank count never serves as a prior
+    q3 = pepp.context_key(1 << 20, 1 << 20, 16 << 20, 0.0, nparts=4)
+    assert H.prior(q3, ids) is None

@@ -5,7 +5,9 @@ For banded (half-bandwidth 4) and uniform-random (16/row) square matrices
 with 10^4 ... 10^8 rows, build one plan, let the history-based selector
 calibrate through ordinary automatic calls, then compare its choice with an
 exhaustive per-candidate timing in the same process (median of several
-calls, L2 flushed between calls). One JSON line per matrix.
+calls, L2 flushed between calls). Also reports the cold pick: the first call
+of a fresh plan whose history file holds the previously swept matrices
+(nearest-context prior; the first matrix has none). One JSON line per matrix.
 
   python tools/sweep.py [--max-rows 1e8] [--out gpurun_out/sweep.jsonl]
 """
@@ -41,6 +43,11 @@ def main():
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
     fo = open(a.out, "w")
+    # one history file shared by the whole sweep: every plan loads what the
+    # previous matrices recorded (a cold start borrows the nearest context)
+    hist_path = os.path.join(os.path.dirname(a.out), "sweep_history.txt")
+    if os.path.exists(hist_path):
+        os.unlink(hist_path)
     for idx, R in enumerate(sizes):
         for kind in a.kinds.split(","):
             t0 = time.perf_counter()
@@ -50,7 +57,7 @@ def main():
             x = torch.from_numpy(gen.vector(seed + 50, gen.REAL, R)).cuda()
             y = torch.empty(R, dtype=torch.float64, device="cuda")
             t0 = time.perf_counter()
-            plan = pepp.Plan.from_csr(A)
+            plan = pepp.Plan.from_csr(A, history_path=hist_path)
             tplan = time.perf_counter() - t0
             del A
             ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.reps)]
@@ -66,11 +73,15 @@ def main():
                     ts.append(e0.elapsed_time(e1) * 1e3)
                 return statistics.median(ts), u
 
-            # calibration through ordinary automatic calls (flush between calls)
+            # calibration through ordinary automatic calls (flush between calls);
+            # the first call is the cold pick (predicted best from the prior)
             calib_calls = 0
+            cold = None
             while True:
                 flush.zero_()
                 u = plan.exec(x, y)
+                if cold is None:
+                    cold = u
                 calib_calls += 1
                 if not u.calibrating or calib_calls > 200:
                     break
@@ -88,6 +99,8 @@ def main():
                    "chosen": choice.name, "chosen_us": round(per[choice.name], 2), "auto_us": round(t_auto, 2),
                    "best": best, "best_us": round(per[best], 2),
                    "ratio": round(per[choice.name] / per[best], 4), "calibration_calls": calib_calls,
+                   "cold_chosen": cold.name, "cold_ratio": round(per[cold.name] / per[best], 4),
+                   "prior_key": info["prior_key"],
                    "candidates_us": {k: round(v, 2) for k, v in per.items()},
                    "gen_s": round(tgen, 1), "plan_s": round(tplan, 2),
                    "alg_gbs_best": round(info["algorithmic_bytes"] / per[best] / 1e3, 1)}
