@@ -156,6 +156,19 @@ namespace {
         if (_e != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; } \
     } while (0)
 
+// plan-time scratch device buffer, freed on every exit path
+template <typename T>
+struct DevTmp {
+    T* p = nullptr;
+    DevTmp() = default;
+    DevTmp(const DevTmp&) = delete;
+    DevTmp& operator=(const DevTmp&) = delete;
+    DevTmp(DevTmp&& o) noexcept : p(o.p) { o.p = nullptr; }
+    ~DevTmp() { if (p) cudaFree(p); }
+    cudaError_t alloc(size_t n) { return cudaMalloc((void**)&p, sizeof(T) * (n ? n : 1)); }
+    T* release() { T* r = p; p = nullptr; return r; }
+};
+
 template <typename T>
 pepp_status_t dalloc(pepp_spmv_plan_t* p, T** ptr, int64_t n) {
     *ptr = nullptr;
@@ -227,24 +240,23 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     }
     if (sigma > 1) {
         // stable radix sort of (window, maxlen - len) keys -> perm
-        unsigned long long *keys = nullptr, *keys_out = nullptr;
-        int* rows = nullptr;
-        void* tmp = nullptr;
+        DevTmp<unsigned long long> keys, keys_out;
+        DevTmp<int> rows;
+        DevTmp<unsigned char> tmp;
         size_t tmp_bytes = 0;
         const int maxlen = (int)p->info.max_row;
-        PEPP_CUDA_TRY(cudaMalloc(&keys, sizeof(unsigned long long) * n));
-        PEPP_CUDA_TRY(cudaMalloc(&keys_out, sizeof(unsigned long long) * n));
-        PEPP_CUDA_TRY(cudaMalloc(&rows, sizeof(int) * n));
+        PEPP_CUDA_TRY(keys.alloc(n));
+        PEPP_CUDA_TRY(keys_out.alloc(n));
+        PEPP_CUDA_TRY(rows.alloc(n));
         if ((s = dalloc(p, &p->d_perm, n))) return s;
-        pepp::k::sell_keys_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, sigma, maxlen, keys, rows);
+        pepp::k::sell_keys_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, sigma, maxlen, keys.p, rows.p);
         PEPP_CUDA_TRY(cudaGetLastError());
         int end_bit = 32;
         while ((1ull << (end_bit - 32)) <= (unsigned long long)((n - 1) / sigma) && end_bit < 64) ++end_bit;
-        cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, keys, keys_out, rows, p->d_perm, n, 0, end_bit, st);
-        PEPP_CUDA_TRY(cudaMalloc(&tmp, tmp_bytes));
-        PEPP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, keys, keys_out, rows, p->d_perm, n, 0, end_bit, st));
+        cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, keys.p, keys_out.p, rows.p, p->d_perm, n, 0, end_bit, st);
+        PEPP_CUDA_TRY(tmp.alloc(tmp_bytes));
+        PEPP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp.p, tmp_bytes, keys.p, keys_out.p, rows.p, p->d_perm, n, 0, end_bit, st));
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-        cudaFree(tmp); cudaFree(keys); cudaFree(keys_out); cudaFree(rows);
         if ((s = fill_ratio(p->d_perm, &fill))) return s;
     }
     p->sell_sigma = sigma;
@@ -261,17 +273,16 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     {
         if ((s = dalloc(p, &p->d_scol16, p->sell_slots + 32))) return s;
         PEPP_CUDA_TRY(cudaMemsetAsync(p->d_scol16, 0, sizeof(int16_t) * (p->sell_slots + 32), st));
-        unsigned long long* d_n16 = nullptr;
-        PEPP_CUDA_TRY(cudaMalloc(&d_n16, sizeof(unsigned long long)));
-        PEPP_CUDA_TRY(cudaMemsetAsync(d_n16, 0, sizeof(unsigned long long), st));
+        DevTmp<unsigned long long> d_n16;
+        PEPP_CUDA_TRY(d_n16.alloc(1));
+        PEPP_CUDA_TRY(cudaMemsetAsync(d_n16.p, 0, sizeof(unsigned long long), st));
         const int wb = 256, wg = (int)(((int64_t)p->nchunks * 32 + wb - 1) / wb);
         pepp::k::sell_col16_kernel<<<wg, wb, 0, st>>>(n, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen,
-                                                       p->d_perm, p->d_scol, p->d_scol16, d_n16);
+                                                       p->d_perm, p->d_scol, p->d_scol16, d_n16.p);
         PEPP_CUDA_TRY(cudaGetLastError());
         unsigned long long n16 = 0;
-        PEPP_CUDA_TRY(cudaMemcpyAsync(&n16, d_n16, sizeof(n16), cudaMemcpyDeviceToHost, st));
+        PEPP_CUDA_TRY(cudaMemcpyAsync(&n16, d_n16.p, sizeof(n16), cudaMemcpyDeviceToHost, st));
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-        cudaFree(d_n16);
         p->sell_col16_chunks = (int64_t)n16;
         if (n16 == 0) { cudaFree(p->d_scol16); p->d_scol16 = nullptr; p->dev_bytes -= (int64_t)sizeof(int16_t) * (p->sell_slots + 32); }
     }
@@ -628,51 +639,50 @@ pepp_status_t setup_halo(pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts
     }
     for (int q = 0; q < P; ++q) rcount[q] = (int64_t)rlist[q].size();
     // exchange counts: send rcount[q] to q, receive scount[q] from q
-    int64_t *d_rc = nullptr, *d_sc = nullptr;
-    PEPP_CUDA_TRY(cudaMalloc(&d_rc, sizeof(int64_t) * P));
-    PEPP_CUDA_TRY(cudaMalloc(&d_sc, sizeof(int64_t) * P));
-    PEPP_CUDA_TRY(cudaMemcpy(d_rc, rcount.data(), sizeof(int64_t) * P, cudaMemcpyHostToDevice));
-    PEPP_CUDA_TRY(cudaMemset(d_sc, 0, sizeof(int64_t) * P));
+    DevTmp<int64_t> d_rc, d_sc;
+    PEPP_CUDA_TRY(d_rc.alloc(P));
+    PEPP_CUDA_TRY(d_sc.alloc(P));
+    PEPP_CUDA_TRY(cudaMemcpy(d_rc.p, rcount.data(), sizeof(int64_t) * P, cudaMemcpyHostToDevice));
+    PEPP_CUDA_TRY(cudaMemset(d_sc.p, 0, sizeof(int64_t) * P));
     const Nccl* n = p->nccl;
-    n->GroupStart();
+    if (n->GroupStart()) return PEPP_E_NCCL;
     for (int q = 0; q < P; ++q) {
         if (q == me) continue;
-        n->Send(d_rc + q, 1, pepp::NCCL_INT64, q, p->comm, st);
-        n->Recv(d_sc + q, 1, pepp::NCCL_INT64, q, p->comm, st);
+        n->Send(d_rc.p + q, 1, pepp::NCCL_INT64, q, p->comm, st);
+        n->Recv(d_sc.p + q, 1, pepp::NCCL_INT64, q, p->comm, st);
     }
     if (n->GroupEnd()) return PEPP_E_NCCL;
     PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-    PEPP_CUDA_TRY(cudaMemcpy(scount.data(), d_sc, sizeof(int64_t) * P, cudaMemcpyDeviceToHost));
-    cudaFree(d_rc); cudaFree(d_sc);
+    PEPP_CUDA_TRY(cudaMemcpy(scount.data(), d_sc.p, sizeof(int64_t) * P, cudaMemcpyDeviceToHost));
     scount[me] = 0;
     // exchange index lists
-    std::vector<int*> d_r(P, nullptr), d_s(P, nullptr);
+    std::vector<DevTmp<int>> d_r(P), d_s(P);
     for (int q = 0; q < P; ++q) {
         if (rcount[q]) {
-            PEPP_CUDA_TRY(cudaMalloc(&d_r[q], sizeof(int) * rcount[q]));
-            PEPP_CUDA_TRY(cudaMemcpy(d_r[q], rlist[q].data(), sizeof(int) * rcount[q], cudaMemcpyHostToDevice));
+            PEPP_CUDA_TRY(d_r[q].alloc(rcount[q]));
+            PEPP_CUDA_TRY(cudaMemcpy(d_r[q].p, rlist[q].data(), sizeof(int) * rcount[q], cudaMemcpyHostToDevice));
         }
-        if (scount[q]) PEPP_CUDA_TRY(cudaMalloc(&d_s[q], sizeof(int) * scount[q]));
+        if (scount[q]) PEPP_CUDA_TRY(d_s[q].alloc(scount[q]));
     }
-    n->GroupStart();
+    if (n->GroupStart()) return PEPP_E_NCCL;
     for (int q = 0; q < P; ++q) {
-        if (rcount[q]) n->Send(d_r[q], (size_t)rcount[q], pepp::NCCL_INT32, q, p->comm, st);
-        if (scount[q]) n->Recv(d_s[q], (size_t)scount[q], pepp::NCCL_INT32, q, p->comm, st);
+        if (rcount[q]) n->Send(d_r[q].p, (size_t)rcount[q], pepp::NCCL_INT32, q, p->comm, st);
+        if (scount[q]) n->Recv(d_s[q].p, (size_t)scount[q], pepp::NCCL_INT32, q, p->comm, st);
     }
     if (n->GroupEnd()) return PEPP_E_NCCL;
     PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-    auto make = [&](int q, std::vector<int32_t>& lst, int* d_list, std::vector<PeerXfer>& out) -> pepp_status_t {
+    auto make = [&](int q, std::vector<int32_t>& lst, DevTmp<int>& d_list, std::vector<PeerXfer>& out) -> pepp_status_t {
         PeerXfer t;
         t.peer = q;
         t.count = (int64_t)lst.size();
         const bool contig = !lst.empty() && (int64_t)lst.back() - lst.front() + 1 == t.count;
         t.contig_start = contig ? lst.front() : -1;
         if (!contig && t.count) {
-            t.d_idx = d_list;
-            d_list = nullptr;
-            PEPP_CUDA_TRY(cudaMalloc(&t.d_buf, sizeof(double) * t.count));
+            DevTmp<double> buf;
+            PEPP_CUDA_TRY(buf.alloc(t.count));
+            t.d_idx = d_list.release();
+            t.d_buf = buf.release();
         }
-        if (d_list) cudaFree(d_list);
         out.push_back(t);
         return PEPP_OK;
     };
@@ -680,7 +690,7 @@ pepp_status_t setup_halo(pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts
         if (rcount[q]) { pepp_status_t s = make(q, rlist[q], d_r[q], p->recv_x); if (s) return s; }
         if (scount[q]) {
             std::vector<int32_t> sl(scount[q]);
-            PEPP_CUDA_TRY(cudaMemcpy(sl.data(), d_s[q], sizeof(int) * scount[q], cudaMemcpyDeviceToHost));
+            PEPP_CUDA_TRY(cudaMemcpy(sl.data(), d_s[q].p, sizeof(int) * scount[q], cudaMemcpyDeviceToHost));
             pepp_status_t s = make(q, sl, d_s[q], p->send_x);
             if (s) return s;
         }
@@ -757,10 +767,12 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_col + p->pad, A->col_idx, sizeof(int) * A->nnz, kind, st));
         PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_val + p->pad, A->values, sizeof(double) * A->nnz, kind, st));
     }
-    int64_t* d_rp64 = nullptr;
-    pepp::k::RowStats* d_stats = nullptr;
-    PEPP_CUDA_TRY(cudaMalloc(&d_rp64, sizeof(int64_t) * (A->nrows + 1)));
-    PEPP_CUDA_TRY(cudaMalloc(&d_stats, sizeof(pepp::k::RowStats)));
+    DevTmp<int64_t> rp64;
+    DevTmp<pepp::k::RowStats> stats;
+    PEPP_CUDA_TRY(rp64.alloc(A->nrows + 1));
+    PEPP_CUDA_TRY(stats.alloc(1));
+    int64_t* d_rp64 = rp64.p;
+    pepp::k::RowStats* d_stats = stats.p;
     PEPP_CUDA_TRY(cudaMemsetAsync(d_stats, 0, sizeof(pepp::k::RowStats), st));
     PEPP_CUDA_TRY(cudaMemcpyAsync(d_rp64, A->row_ptr, sizeof(int64_t) * (A->nrows + 1), kind, st));
     {
@@ -784,8 +796,6 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         pepp::halo_ghost_list(hcol.data(), A->nnz, p->row_offset, p->row_offset + A->nrows, ghosts);
         if (!ghosts.empty() && (ghosts.front() < 0 || ghosts.back() >= p->global_rows)) hs.bad = 1;
     }
-    cudaFree(d_rp64);
-    cudaFree(d_stats);
     if (hs.bad) return PEPP_E_INVALID;
 
     pepp_plan_info_t& I = p->info;
@@ -894,14 +904,13 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         if (ex == PEPP_X_AUTO) {
             // halo when every rank's ghosts are a small part of x;
             // the decision must be identical on all ranks: max-reduce the counts.
-            int64_t *d_g = nullptr;
+            DevTmp<int64_t> d_g;
             int64_t g = (int64_t)ghosts.size(), gmax = 0;
-            PEPP_CUDA_TRY(cudaMalloc(&d_g, sizeof(int64_t)));
-            PEPP_CUDA_TRY(cudaMemcpy(d_g, &g, sizeof(int64_t), cudaMemcpyHostToDevice));
-            if (p->nccl->AllReduce(d_g, d_g, 1, pepp::NCCL_INT64, pepp::NCCL_OP_MAX, p->comm, st)) { cudaFree(d_g); return PEPP_E_NCCL; }
+            PEPP_CUDA_TRY(d_g.alloc(1));
+            PEPP_CUDA_TRY(cudaMemcpy(d_g.p, &g, sizeof(int64_t), cudaMemcpyHostToDevice));
+            if (p->nccl->AllReduce(d_g.p, d_g.p, 1, pepp::NCCL_INT64, pepp::NCCL_OP_MAX, p->comm, st)) return PEPP_E_NCCL;
             PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-            PEPP_CUDA_TRY(cudaMemcpy(&gmax, d_g, sizeof(int64_t), cudaMemcpyDeviceToHost));
-            cudaFree(d_g);
+            PEPP_CUDA_TRY(cudaMemcpy(&gmax, d_g.p, sizeof(int64_t), cudaMemcpyDeviceToHost));
             ex = ((double)gmax < 0.25 * (double)p->global_rows) ? PEPP_X_HALO : PEPP_X_ALLGATHER;
         }
         p->exchange = ex;
