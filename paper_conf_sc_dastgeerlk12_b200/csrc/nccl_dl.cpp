@@ -5,6 +5,7 @@
 #include "pepp_internal.h"
 
 #include <dlfcn.h>
+#include <cstdlib>
 #include <mutex>
 
 namespace pepp {
@@ -15,13 +16,14 @@ static std::once_flag g_once;
 
 const Nccl* nccl_load() {
     std::call_once(g_once, [] {
-        // Prefer the copy already mapped into the process (torch's), then the system one.
+        // PEPP_NCCL_LIB (an explicit path) wins — tests point it at a
+        // same-ABI stand-in (tests/support/fake_nccl.c) to run several ranks
+        // on one GPU; else the copy already mapped into the process (torch's),
+        // then the system one.
         const char* names[] = {"libnccl.so.2", "libnccl.so"};
         void* h = nullptr;
-        for (const char* n : names) {
-            h = dlopen(n, RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
-            if (h) break;
-        }
+        if (const char* path = std::getenv("PEPP_NCCL_LIB")) h = dlopen(path, RTLD_NOW | RTLD_LOCAL);
+        for (int i = 0; !h && i < 2; ++i) h = dlopen(names[i], RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
         for (int i = 0; !h && i < 2; ++i) h = dlopen(names[i], RTLD_NOW | RTLD_GLOBAL);
         if (!h) return;
 #define PEPP_SYM(field, name) g_nccl.field = reinterpret_cast<decltype(g_nccl.field)>(dlsym(h, name)); if (!g_nccl.field) return;

@@ -1,0 +1,125 @@
+"""The partitioned path end to end with two ranks on ONE GPU:
+the library's own plan-time halo setup (counts, index lists, the AllReduce
+that makes every rank agree on the exchange), per-iteration halo exchange
+(contiguous ranges and pack/unpack) and allgatherv, exec(PEPP_Y_NEXT_INPUT /
+PEPP_Y_REPLICATED), pepp_spmv_exchange and the partitioned exec_host. Real
+NCCL refuses two ranks on one device, so the library is pointed (through
+PEPP_NCCL_LIB) at tests/support/fake_nccl.c, which implements the same C ABI
+with NCCL's matching semantics over a shared host mapping; everything else
+is the production code. Results: iterated SpMV over the concatenated row
+blocks equals the unpartitioned oracle bit for bit (integer-valued inputs)."""
+from __future__ import annotations
+
+import os
+import shutil
+import subprocess
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+SRC = os.path.join(HERE, "support", "fake_nccl.c")
+LIB = os.path.join(HERE, "support", "libfake_nccl.so")
+
+
+def _build_fake() -> str:
+    if not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
+        nvcc = shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc"
+        subprocess.check_call([nvcc, "-O2", "-shared", "-Xcompiler", "-fPIC", "-cudart=static", SRC, "-o", LIB])
+    return LIB
+
+
+def _matrix(name):
+    import gen
+    if name == "lap":
+        return gen.laplacian2d(96)
+    if name == "zipf":
+        return gen.zipf(6000, 6000, seed=47, kmax=40, val_mode=gen.INT4)
+    if name == "banded":
+        return gen.banded(5000, 4, seed=100, val_mode=gen.INT4)
+    raise ValueError(name)
+
+
+def _worker(rank, world, lib, uid, name, exchange, K, outq):
+    os.environ["PEPP_NCCL_LIB"] = lib
+    try:
+        import sys
+        sys.path.insert(0, os.path.dirname(HERE))
+        import torch
+
+        import gen
+        import oracle
+        import paper_conf_sc_dastgeerlk12_b200 as pepp
+        torch.cuda.set_device(0)
+        A = _matrix(name)
+        n = A.nrows
+        bounds = pepp.partition_rows(A.row_ptr, world)
+        blk = gen.row_block(A, int(bounds[rank]), int(bounds[rank + 1]))
+        x0 = gen.vector(3, gen.INT8, n)
+        res = {}
+        with pepp.Plan.from_csr(blk, nranks=world, rank=rank, row_bounds=bounds, nccl_unique_id=uid,
+                                exchange=exchange) as plan:
+            info = plan.info()
+            a = torch.from_numpy(x0).cuda()
+            b = torch.full_like(a, float("nan"))
+            c = torch.full_like(a, float("nan"))
+            src, dst = a, b
+            for k in range(K):
+                if k % 2 == 0:
+                    plan.exec(src, dst, flags=pepp.Y_NEXT_INPUT)
+                else:   # kernel and exchange as separate calls
+                    plan.exec(src, dst, flags=pepp.Y_LOCAL)
+                    plan.exchange(dst, pepp.Y_NEXT_INPUT)
+                src, dst = dst, (c if dst is b else b)
+            plan.exec(src, dst, flags=pepp.Y_REPLICATED)   # iteration K+1, all rows on every rank
+            torch.cuda.synchronize()
+            res["iter"] = bool(np.array_equal(dst.cpu().numpy(), oracle.iterate(A, x0, K + 1)))
+            # host-buffer entry point, partitioned: iterations with the exchange inside
+            yh = np.full(n, np.nan)
+            plan.exec_host(x0, yh, iterations=K, flags=pepp.Y_REPLICATED)
+            res["host"] = bool(np.array_equal(yh, oracle.iterate(A, x0, K)))
+            res["exchange"] = info["exchange"]
+            res["halo_recv"] = info["halo_recv"]
+            res["halo_send"] = info["halo_send"]
+        outq.put((rank, res))
+    except Exception as e:
+        import traceback
+        outq.put((rank, {"error": repr(e) + traceback.format_exc()}))
+
+
+def _run(name, exchange, K=6):
+    import torch.multiprocessing as mp
+    lib = _build_fake()
+    uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_{exchange}".encode() + b"\0" * 128)[:128]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker, args=(r, 2, lib, uid, name, exchange, K, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = {}
+    for _ in range(2):
+        r, res = q.get(timeout=300)
+        out[r] = res
+    for p in procs:
+        p.join(timeout=60)
+    for r in range(2):
+        assert "error" not in out[r], out[r]["error"]
+    return out
+
+
+@pytest.mark.parametrize("name,exchange", [("lap", 2), ("lap", 1), ("zipf", 2), ("zipf", 1), ("banded", -1),
+                                           ("zipf", -1)])
+def test_two_ranks_one_gpu_iterated_spmv_bitwise(name, exchange):
+    import paper_conf_sc_dastgeerlk12_b200 as pepp
+    out = _run(name, exchange)
+    for r in range(2):
+        assert out[r]["iter"] and out[r]["host"], (r, out[r])
+    ex = {out[0]["exchange"], out[1]["exchange"]}
+    assert len(ex) == 1                       # every rank resolved the same exchange
+    if exchange != -1:
+        assert ex == {exchange}
+    if name == "lap" and exchange == pepp.X_HALO:
+        assert out[0]["halo_recv"] == 96 and out[1]["halo_send"] == 96   # one grid row each way
