@@ -26,9 +26,13 @@
  *   - pepp_spmv_destroy ~ PEPPHER_SHUTDOWN (P@33881).
  *
  * Precision and index widths (readings A2, A3): values, x, y and all
- * sums are fp64; column indices int32; row pointers int64 at the ABI (the
- * paper's size_t) — narrowed to int32 on the device (nnz < 2^31 required;
- * larger blocks return PEPP_E_UNSUPPORTED).
+ * sums are fp64 (PEPP_VALUE_F64, the default) or — the paper's own `float`
+ * signature (P@32944), SURVEY §8(f) f3 — fp32 throughout (PEPP_VALUE_F32:
+ * fp32 values, x, y, products and sums); the value type is a property of the
+ * plan and every value pointer below (x, y, work, host buffers) points to
+ * elements of that type. Column indices int32; row pointers int64 at the ABI
+ * (the paper's size_t) — narrowed to int32 on the device (nnz < 2^31
+ * required; larger blocks return PEPP_E_UNSUPPORTED).
  *
  * Access modes follow the paper's interface descriptor (read / write /
  * readwrite, §II P@4233) and the const / non-const inference of the utility
@@ -85,6 +89,10 @@ typedef enum {
     PEPP_X_HALO = 2           /* ghost (halo) exchange: only entries peers' rows read */
 } pepp_exchange_t;
 
+/* value types (pepp_csr_t.value_type) */
+#define PEPP_VALUE_F64 0
+#define PEPP_VALUE_F32 1
+
 /* exec flags: which part of y is valid on return (once the stream completes) */
 #define PEPP_Y_LOCAL       0x0  /* own rows only: y[row_offset, row_offset+nrows)              */
 #define PEPP_Y_NEXT_INPUT  0x1  /* own rows + every entry this plan's next call reads as x     */
@@ -108,8 +116,9 @@ typedef struct {
     int64_t first;            /* row_ptr base (paper's `first`)              */
     const int64_t* row_ptr;   /* [nrows + 1]                                 */
     const int32_t* col_idx;   /* [nnz]                                       */
-    const double* values;     /* [nnz]                                       */
+    const void* values;       /* [nnz] of value_type                         */
     int32_t on_device;        /* 0 = host pointers, 1 = device pointers      */
+    int32_t value_type;       /* PEPP_VALUE_F64 (0, default) or PEPP_VALUE_F32 */
 } pepp_csr_t;
 
 /* Plan options. Use pepp_spmv_opts_default() then override. */
@@ -215,7 +224,7 @@ pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_choice_t* out);
    masked-out variant), PEPP_E_CUDA, PEPP_E_NCCL, PEPP_E_STATE (exchange
    requested on an unpartitioned plan is fine and a no-op; a plan in a sticky
    error state returns its error). */
-pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const double* x, double* y, int flags,
+pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void* x, void* y, int flags,
                              void* stream, const pepp_choice_t* force, pepp_choice_t* used);
 
 /* The exchange step alone: make this rank's rows of y
@@ -225,7 +234,7 @@ pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const double* x, double* y, in
    global length; own rows are read, other rows written. exec(flags) ==
    exec(PEPP_Y_LOCAL) followed by exchange(flags). A no-op when nranks == 1.
    Errors: PEPP_E_INVALID, PEPP_E_NCCL, PEPP_E_CUDA. */
-pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, double* y, int flags, void* stream);
+pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* y, int flags, void* stream);
 
 /* Host-buffer entry point (the paper's measurement setting, where operand
    transfers are part of the call: Fig. 5 "communication overhead of copying
@@ -240,7 +249,7 @@ pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, double* y, int flags, void
    for completion on `stream`.
    The plan-owned device buffers are allocated on first use and kept
    ("register once", P@29208). Errors as pepp_spmv_exec. */
-pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const double* x_host, double* y_host, int32_t iterations,
+pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const void* x_host, void* y_host, int32_t iterations,
                                   int flags, void* stream);
 
 /* Free everything the plan owns (device memory, events, an owned NCCL
@@ -276,7 +285,7 @@ pepp_status_t pepp_spmv_history_stats(const pepp_spmv_plan_t* p, int32_t cand,
    Timing events are not recorded inside graphs (history is not updated by
    replays). Errors: PEPP_E_INVALID, PEPP_E_CUDA, PEPP_E_NCCL. */
 typedef struct pepp_spmv_graph_s pepp_spmv_graph_t;
-pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, const double* x, double* y, double* work,
+pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, const void* x, void* y, void* work,
                                      int32_t iterations, int32_t mode, int flags, void* stream,
                                      pepp_spmv_graph_t** out);
 pepp_status_t pepp_spmv_graph_launch(pepp_spmv_graph_t* g, void* stream);
@@ -328,7 +337,8 @@ pepp_status_t pepp_vector_state(const pepp_vector_t* v, int32_t* host_valid, int
 /* A READWRITE component on a vector: v = alpha * v on the device (stream-ordered). */
 pepp_status_t pepp_vector_scale(pepp_vector_t* v, double alpha, void* stream);
 /* y = A·x through containers: x READ, y WRITE (see pepp_spmv_exec for flags,
-   force, used). x and y must be distinct vectors of length ncols / global rows. */
+   force, used). x and y must be distinct vectors of length ncols / global rows.
+   Containers hold fp64: an fp32 plan returns PEPP_E_UNSUPPORTED. */
 pepp_status_t pepp_spmv_exec_vec(pepp_spmv_plan_t* p, pepp_vector_t* x, pepp_vector_t* y, int flags,
                                  void* stream, const pepp_choice_t* force, pepp_choice_t* used);
 

@@ -53,6 +53,9 @@ def lib():
         L.oracle_abs_row.restype = ctypes.c_double
         L.oracle_spmv_iterate.argtypes = [i64, i64, i64, p, p, p, p, p, p, p]
         L.oracle_partition_nnz.argtypes = [i64, i64, p, i64, p]
+        L.oracle_spmv_seq_f32.argtypes = [i64, i64, p, p, p, p, p]
+        L.oracle_spmv_rows_parallel_f32.argtypes = [i64, i64, p, p, p, p, p]
+        L.oracle_abs_rowsum_f32.argtypes = [i64, i64, p, p, p, p, p]
         _lib = L
     return _lib
 
@@ -74,7 +77,10 @@ def _ptr(a):
 
 
 def spmv(A, x, parallel: bool = False) -> np.ndarray:
-    """y = A·x for a CSR (gen.CSR-like: nrows, row_ptr, col, val) — the definition."""
+    """y = A·x for a CSR (gen.CSR-like: nrows, row_ptr, col, val) — the definition.
+    float32 values select the fp32 instance (fp32 x, products and sums)."""
+    if np.asarray(A.val).dtype == np.float32:
+        return spmv_f32(A, x, parallel)
     rp, c, v = _args(A.row_ptr, A.col, A.val)
     xx = _c(x, np.float64)
     y = np.empty(A.nrows, dtype=np.float64)
@@ -82,6 +88,32 @@ def spmv(A, x, parallel: bool = False) -> np.ndarray:
     if A.nrows:
         f(A.nrows, int(rp[0]), _ptr(rp), _ptr(c), _ptr(v), _ptr(xx), _ptr(y))
     return y
+
+
+def spmv_f32(A, x, parallel: bool = False) -> np.ndarray:
+    """The fp32 instance of the definition (paper's `float` signature)."""
+    rp = _c(A.row_ptr, np.int64)
+    c = _c(A.col, np.int32)
+    v = _c(A.val, np.float32)
+    xx = _c(x, np.float32)
+    y = np.empty(A.nrows, dtype=np.float32)
+    f = lib().oracle_spmv_rows_parallel_f32 if parallel else lib().oracle_spmv_seq_f32
+    if A.nrows:
+        f(A.nrows, int(rp[0]), _ptr(rp), _ptr(c), _ptr(v), _ptr(xx), _ptr(y))
+    return y
+
+
+def bound_f32(A, x) -> np.ndarray:
+    """Per-row tolerance for the fp32 instance: 2·nnz_row·2^-23·Σ|a||x|
+    (the north-star bound with fp32's unit roundoff 2^-24 in place of 2^-53)."""
+    rp = _c(A.row_ptr, np.int64)
+    c = _c(A.col, np.int32)
+    v = _c(A.val, np.float32)
+    xx = _c(x, np.float32)
+    s = np.empty(A.nrows, dtype=np.float64)
+    if A.nrows:
+        lib().oracle_abs_rowsum_f32(A.nrows, int(rp[0]), _ptr(rp), _ptr(c), _ptr(v), _ptr(xx), _ptr(s))
+    return 2.0 * row_lengths(A).astype(np.float64) * 2.0 ** -23 * s
 
 
 def spmv_raw(nrows, first, row_ptr, col, val, x, parallel=False) -> np.ndarray:

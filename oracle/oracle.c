@@ -79,6 +79,47 @@ ORACLE_EXPORT double oracle_spmv_row(int64_t i, int64_t first, const int64_t* ro
     return acc;
 }
 
+/* ---- fp32 instance: the paper's own `float` signature (P@32944), SURVEY
+   §8(f) f3. Same definition with float values, float x and a float
+   accumulator: product rounded to float, then sum rounded to float,
+   ascending k (SSE single precision, no FMA: -ffp-contract=off). */
+ORACLE_EXPORT void oracle_spmv_seq_f32(int64_t nrows, int64_t first, const int64_t* row_ptr,
+                                       const int32_t* col, const float* val, const float* x, float* y) {
+    for (int64_t i = 0; i < nrows; ++i) {
+        float acc = +0.0f;
+        for (int64_t k = row_ptr[i] - first; k < row_ptr[i + 1] - first; ++k) {
+            float prod = val[k] * x[col[k]];
+            acc = acc + prod;
+        }
+        y[i] = acc;
+    }
+}
+
+ORACLE_EXPORT void oracle_spmv_rows_parallel_f32(int64_t nrows, int64_t first, const int64_t* row_ptr,
+                                                 const int32_t* col, const float* val, const float* x, float* y) {
+    #pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < nrows; ++i) {
+        float acc = +0.0f;
+        for (int64_t k = row_ptr[i] - first; k < row_ptr[i + 1] - first; ++k) {
+            float prod = val[k] * x[col[k]];
+            acc = acc + prod;
+        }
+        y[i] = acc;
+    }
+}
+
+/* S_i = sum |a| |x| of an fp32 matrix, accumulated in double (bound only) */
+ORACLE_EXPORT void oracle_abs_rowsum_f32(int64_t nrows, int64_t first, const int64_t* row_ptr,
+                                         const int32_t* col, const float* val, const float* x, double* s) {
+    #pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < nrows; ++i) {
+        double acc = 0.0;
+        for (int64_t k = row_ptr[i] - first; k < row_ptr[i + 1] - first; ++k)
+            acc = acc + fabs((double)val[k]) * fabs((double)x[col[k]]);
+        s[i] = acc;
+    }
+}
+
 /* S_i for one row i (sampled bound checks at full size) */
 ORACLE_EXPORT double oracle_abs_row(int64_t i, int64_t first, const int64_t* row_ptr,
                                     const int32_t* col, const double* val, const double* x) {

@@ -79,8 +79,10 @@ class Plan:
     """pepp_spmv_plan over one CSR row block.
 
     ``row_ptr`` (int64, global offsets: row_ptr[0] == first), ``col`` (int32),
-    ``val`` (float64): numpy host arrays, or CUDA torch tensors on the plan's
-    device (then ``on_device`` is inferred). The plan copies them.
+    ``val`` (float64, or float32 for the fp32 instance — the value type of
+    the plan, and of every x / y passed to it): numpy host arrays, or CUDA
+    torch tensors on the plan's device (then ``on_device`` is inferred). The
+    plan copies them.
     """
 
     def __init__(self, nrows: int, ncols: int, row_ptr, col, val, *, variant_mask: int = 0,
@@ -93,13 +95,18 @@ class Plan:
         self._h = ctypes.c_void_p()
         on_dev = not isinstance(row_ptr, np.ndarray)
         if not on_dev:
+            f32 = np.asarray(val).dtype == np.float32
             row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
             col = np.ascontiguousarray(col, dtype=np.int32)
-            val = np.ascontiguousarray(val, dtype=np.float64)
+            val = np.ascontiguousarray(val, dtype=np.float32 if f32 else np.float64)
+        else:
+            import torch
+            f32 = val.dtype == torch.float32
         nnz = int(col.shape[0]) if col is not None else 0
         first = int(row_ptr[0]) if not on_dev else int(row_ptr[:1].cpu()[0])
+        self.value_type = C.VALUE_F32 if f32 else C.VALUE_F64
         A = C.CSR_T(nrows, ncols, nnz, first, _ptr(row_ptr), _ptr(col) if nnz else 0,
-                    _ptr(val) if nnz else 0, 1 if on_dev else 0)
+                    _ptr(val) if nnz else 0, 1 if on_dev else 0, self.value_type)
         o = C.OPTS_T()
         L.pepp_spmv_opts_default(ctypes.byref(o))
         o.variant_mask = variant_mask
@@ -161,7 +168,8 @@ class Plan:
     def exec_host(self, x_host: np.ndarray, y_host: np.ndarray, iterations: int = 1, flags: int = Y_LOCAL,
                   stream=None) -> None:
         """Host buffers in and out, transfers inside the call (synchronous)."""
-        assert x_host.dtype == np.float64 and y_host.dtype == np.float64
+        want = np.float32 if self.value_type == C.VALUE_F32 else np.float64
+        assert x_host.dtype == want and y_host.dtype == want
         C.check(C.lib().pepp_spmv_exec_host(self._h, _ptr(x_host), _ptr(y_host), iterations, flags,
                                             _stream_handle(stream)), "pepp_spmv_exec_host")
 

@@ -16,6 +16,7 @@ V_AUTO, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, V_CSR_STREAM, V_COUNT = -1, 0, 1, 2,
 X_AUTO, X_NONE, X_ALLGATHER, X_HALO = -1, 0, 1, 2
 Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, EXEC_NO_TIMING = 0x0, 0x1, 0x2, 0x10
 ACCESS_READ, ACCESS_WRITE, ACCESS_READWRITE = 1, 2, 3
+VALUE_F64, VALUE_F32 = 0, 1
 DEVICE_SIMULATED = -2
 VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell", V_CSR_STREAM: "csr_stream"}
 EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_AUTO: "auto"}
@@ -26,7 +27,7 @@ c_i32, c_i64, c_u32, c_u64, c_f64, c_vp = (ctypes.c_int32, ctypes.c_int64, ctype
 
 class CSR_T(ctypes.Structure):
     _fields_ = [("nrows", c_i64), ("ncols", c_i64), ("nnz", c_i64), ("first", c_i64),
-                ("row_ptr", c_vp), ("col_idx", c_vp), ("values", c_vp), ("on_device", c_i32)]
+                ("row_ptr", c_vp), ("col_idx", c_vp), ("values", c_vp), ("on_device", c_i32), ("value_type", c_i32)]
 
 
 class OPTS_T(ctypes.Structure):

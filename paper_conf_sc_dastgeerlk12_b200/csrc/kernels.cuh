@@ -63,13 +63,44 @@ __device__ __forceinline__ int ld_stream_i(const int* p, uint64_t pol) {
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
     return r;
 }
+__device__ __forceinline__ float ld_stream_f(const float* p, uint64_t pol) {
+    float r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(r) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ float4 ld_stream_f4(const float* p, uint64_t pol) {
+    float4 r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+        : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p), "l"(pol));
+    return r;
+}
+// value-type generic forms (T = double for the fp64 path, float for the
+// fp32 instance of the paper's `float` signature)
+__device__ __forceinline__ double ld_stream_v(const double* p, uint64_t pol) { return ld_stream_d(p, pol); }
+__device__ __forceinline__ float ld_stream_v(const float* p, uint64_t pol) { return ld_stream_f(p, pol); }
+// four consecutive values starting at a 4-element-aligned position (16 B for
+// float: one load; 32 B for double: two)
+__device__ __forceinline__ void ld_stream_4(const double* p, uint64_t pol, double v[4]) {
+    const double2 a = ld_stream_d2(p, pol), b = ld_stream_d2(p + 2, pol);
+    v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+}
+__device__ __forceinline__ void ld_stream_4(const float* p, uint64_t pol, float v[4]) {
+    const float4 a = ld_stream_f4(p, pol);
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+}
 // x gather: read-only path, cached in L1 and L2 (reused across rows)
-__device__ __forceinline__ double ld_x(const double* __restrict__ x, int c) { return __ldg(x + c); }
+template <typename T>
+__device__ __forceinline__ T ld_x(const T* __restrict__ x, int c) { return __ldg(x + c); }
 // same gather as volatile asm: a run of these is issued back-to-back in
 // program order (ptxas may not interleave the consumers between them)
 __device__ __forceinline__ double ld_x_ordered(const double* __restrict__ x, int c) {
     double r;
     asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(r) : "l"(x + c));
+    return r;
+}
+__device__ __forceinline__ float ld_x_ordered(const float* __restrict__ x, int c) {
+    float r;
+    asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(r) : "l"(x + c));
     return r;
 }
 
@@ -81,12 +112,12 @@ __device__ __forceinline__ double ld_x_ordered(const double* __restrict__ x, int
 // __shfl_xor_sync butterfly over the TPR lanes. The row loop is warp-
 // uniform (all 32 lanes iterate together) so full-mask shuffles are legal.
 // =====================================================================
-template <int TPR, int BLOCK>
+template <int TPR, int BLOCK, typename T>
 __global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int* __restrict__ rp,
                                                            const int* __restrict__ col,
-                                                           const double* __restrict__ val,
-                                                           const double* __restrict__ x,
-                                                           double* __restrict__ y) {
+                                                           const T* __restrict__ val,
+                                                           const T* __restrict__ x,
+                                                           T* __restrict__ y) {
     static_assert(TPR >= 1 && TPR <= 32 && (TPR & (TPR - 1)) == 0, "TPR must be a power of two <= 32");
     constexpr int RPW = 32 / TPR;                 // rows per warp per step
     const int lane = threadIdx.x & 31;
@@ -112,38 +143,37 @@ __global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int*
             sn = __ldg(rp + row + step);
             en = __ldg(rp + row + step + 1);
         }
-        double acc = 0.0;
+        T acc = T(0);
         const int g_end = (e + 3) >> 2;
         int g = (s >> 2) + sub;
-        // two groups per iteration: 6 independent 16-B loads in flight per lane
+        // two groups per iteration: up to 6 independent 16-B loads in flight per lane
         for (; g + TPR < g_end; g += 2 * TPR) {
             const int k0 = g << 2, k1 = (g + TPR) << 2;
             const int4 c0 = ld_stream_i4(col + k0, pol);
-            const double2 a0 = ld_stream_d2(val + k0, pol);
-            const double2 b0 = ld_stream_d2(val + k0 + 2, pol);
+            T v0[4], v1[4];
+            ld_stream_4(val + k0, pol, v0);
             const int4 c1 = ld_stream_i4(col + k1, pol);
-            const double2 a1 = ld_stream_d2(val + k1, pol);
-            const double2 b1 = ld_stream_d2(val + k1 + 2, pol);
+            ld_stream_4(val + k1, pol, v1);
             // group g is not the row's last group: only its head can precede s
-            if (k0 + 0 >= s) acc = fma(a0.x, ld_x(x, c0.x), acc);
-            if (k0 + 1 >= s) acc = fma(a0.y, ld_x(x, c0.y), acc);
-            if (k0 + 2 >= s) acc = fma(b0.x, ld_x(x, c0.z), acc);
-            if (k0 + 3 >= s) acc = fma(b0.y, ld_x(x, c0.w), acc);
+            if (k0 + 0 >= s) acc = fma(v0[0], ld_x(x, c0.x), acc);
+            if (k0 + 1 >= s) acc = fma(v0[1], ld_x(x, c0.y), acc);
+            if (k0 + 2 >= s) acc = fma(v0[2], ld_x(x, c0.z), acc);
+            if (k0 + 3 >= s) acc = fma(v0[3], ld_x(x, c0.w), acc);
             // group g+TPR starts after s: only its tail can pass e
-            if (k1 + 0 < e) acc = fma(a1.x, ld_x(x, c1.x), acc);
-            if (k1 + 1 < e) acc = fma(a1.y, ld_x(x, c1.y), acc);
-            if (k1 + 2 < e) acc = fma(b1.x, ld_x(x, c1.z), acc);
-            if (k1 + 3 < e) acc = fma(b1.y, ld_x(x, c1.w), acc);
+            if (k1 + 0 < e) acc = fma(v1[0], ld_x(x, c1.x), acc);
+            if (k1 + 1 < e) acc = fma(v1[1], ld_x(x, c1.y), acc);
+            if (k1 + 2 < e) acc = fma(v1[2], ld_x(x, c1.z), acc);
+            if (k1 + 3 < e) acc = fma(v1[3], ld_x(x, c1.w), acc);
         }
         if (g < g_end) {
             const int k0 = g << 2;
             const int4 c0 = ld_stream_i4(col + k0, pol);
-            const double2 a0 = ld_stream_d2(val + k0, pol);
-            const double2 b0 = ld_stream_d2(val + k0 + 2, pol);
-            if (k0 + 0 >= s && k0 + 0 < e) acc = fma(a0.x, ld_x(x, c0.x), acc);
-            if (k0 + 1 >= s && k0 + 1 < e) acc = fma(a0.y, ld_x(x, c0.y), acc);
-            if (k0 + 2 >= s && k0 + 2 < e) acc = fma(b0.x, ld_x(x, c0.z), acc);
-            if (k0 + 3 >= s && k0 + 3 < e) acc = fma(b0.y, ld_x(x, c0.w), acc);
+            T v0[4];
+            ld_stream_4(val + k0, pol, v0);
+            if (k0 + 0 >= s && k0 + 0 < e) acc = fma(v0[0], ld_x(x, c0.x), acc);
+            if (k0 + 1 >= s && k0 + 1 < e) acc = fma(v0[1], ld_x(x, c0.y), acc);
+            if (k0 + 2 >= s && k0 + 2 < e) acc = fma(v0[2], ld_x(x, c0.z), acc);
+            if (k0 + 3 >= s && k0 + 3 < e) acc = fma(v0[3], ld_x(x, c0.w), acc);
         }
 #pragma unroll
         for (int off = TPR / 2; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
@@ -177,20 +207,20 @@ constexpr int kSellLenMask = (1 << 29) - 1;
 // N slots of one chunk, loads issued unconditionally (all N exist for every
 // lane) before the first FMA; the per-lane row length only masks the FMA.
 // C16: columns stored as int16 deltas from the lane's row index `row0`.
-template <int N, bool C16>
-__device__ __forceinline__ double sell_slots(const double* __restrict__ val, const int* __restrict__ col,
-                                             const int16_t* __restrict__ col16, int row0,
-                                             const double* __restrict__ x, int64_t base, int j0, int len,
-                                             double acc, uint64_t pol) {
-    double v[N];
+template <int N, bool C16, typename T>
+__device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __restrict__ col,
+                                        const int16_t* __restrict__ col16, int row0,
+                                        const T* __restrict__ x, int64_t base, int j0, int len,
+                                        T acc, uint64_t pol) {
+    T v[N];
     int c[N];
 #pragma unroll
     for (int u = 0; u < N; ++u)
         c[u] = C16 ? row0 + ld_stream_i16(col16 + base + (int64_t)(j0 + u) * 32, pol)
                    : ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
 #pragma unroll
-    for (int u = 0; u < N; ++u) v[u] = ld_stream_d(val + base + (int64_t)(j0 + u) * 32, pol);
-    double xv[N];
+    for (int u = 0; u < N; ++u) v[u] = ld_stream_v(val + base + (int64_t)(j0 + u) * 32, pol);
+    T xv[N];
 #pragma unroll
     for (int u = 0; u < N; ++u) xv[u] = ld_x(x, c[u]);
 #pragma unroll
@@ -199,37 +229,37 @@ __device__ __forceinline__ double sell_slots(const double* __restrict__ val, con
     return acc;
 }
 
-template <bool C16>
-__device__ __forceinline__ double sell_chunk(const double* __restrict__ val, const int* __restrict__ col,
-                                             const int16_t* __restrict__ col16, int row0, const double* __restrict__ x,
-                                             int64_t base, int clen, int len, uint64_t pol) {
-    double acc = 0.0;
+template <bool C16, typename T>
+__device__ __forceinline__ T sell_chunk(const T* __restrict__ val, const int* __restrict__ col,
+                                        const int16_t* __restrict__ col16, int row0, const T* __restrict__ x,
+                                        int64_t base, int clen, int len, uint64_t pol) {
+    T acc = T(0);
     int j = 0;
     // whole blocks of 8 slots, then one exactly-sized tail (warp-uniform switch)
-    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, C16>(val, col, col16, row0, x, base, j, len, acc, pol);
+    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol);
     switch (clen - j) {
-    case 1: acc = sell_slots<1, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 2: acc = sell_slots<2, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 3: acc = sell_slots<3, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 4: acc = sell_slots<4, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 5: acc = sell_slots<5, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 6: acc = sell_slots<6, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 7: acc = sell_slots<7, C16>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 1: acc = sell_slots<1, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 2: acc = sell_slots<2, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 3: acc = sell_slots<3, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 4: acc = sell_slots<4, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 5: acc = sell_slots<5, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 6: acc = sell_slots<6, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 7: acc = sell_slots<7, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
     default: break;
     }
     return acc;
 }
 
-template <int BLOCK, bool SORTED>
+template <int BLOCK, bool SORTED, typename T>
 __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
                                                      const int* __restrict__ chunk_len,
                                                      const int* __restrict__ rowlen,
                                                      const int* __restrict__ perm,
                                                      const int* __restrict__ col,
                                                      const int16_t* __restrict__ col16,
-                                                     const double* __restrict__ val,
-                                                     const double* __restrict__ x,
-                                                     double* __restrict__ y,
+                                                     const T* __restrict__ val,
+                                                     const T* __restrict__ x,
+                                                     T* __restrict__ y,
                                                      int cpw) {
     const int lane = threadIdx.x & 31;
     const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
@@ -267,8 +297,8 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
         if (in < nchunks) meta(cn, dn, cpn, lenn, orown);
         const int64_t base = cp + lane;
         const int clen = d & kSellLenMask;
-        const double acc = (d & kSellCol16) ? sell_chunk<true>(val, col, col16, orow, x, base, clen, len, pol)
-                                            : sell_chunk<false>(val, col, col16, orow, x, base, clen, len, pol);
+        const T acc = (d & kSellCol16) ? sell_chunk<true, T>(val, col, col16, orow, x, base, clen, len, pol)
+                                       : sell_chunk<false, T>(val, col, col16, orow, x, base, clen, len, pol);
         if (c * 32 + lane < nrows) y[orow] = acc;
         c = cn; d = dn; cp = cpn; len = lenn; orow = orown;
     }
@@ -285,31 +315,34 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
 // segmented scan; rows that cross tile boundaries leave a carry that
 // merge_fixup_kernel adds afterwards, in tile order (no fp atomics).
 // =====================================================================
-struct SegPair {
-    double v;
+template <typename T>
+struct SegPairT {
+    T v;
     int f;  // 1 = a row ended inside this segment (resets the running sum)
 };
-__device__ __forceinline__ SegPair seg_combine(SegPair a, SegPair b) {
+template <typename T>
+__device__ __forceinline__ SegPairT<T> seg_combine(SegPairT<T> a, SegPairT<T> b) {
     // a precedes b
-    SegPair r;
+    SegPairT<T> r;
     r.f = a.f | b.f;
     r.v = b.f ? b.v : a.v + b.v;
     return r;
 }
 
-template <int BLOCK, int IPT>
+template <int BLOCK, int IPT, typename T>
 __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int* __restrict__ rp,
                                                           const int* __restrict__ col,
-                                                          const double* __restrict__ val,
-                                                          const double* __restrict__ x,
-                                                          double* __restrict__ y,
+                                                          const T* __restrict__ val,
+                                                          const T* __restrict__ x,
+                                                          T* __restrict__ y,
                                                           const int2* __restrict__ tile_coord,
                                                           int* __restrict__ carry_row,
-                                                          double* __restrict__ carry_val) {
+                                                          T* __restrict__ carry_val) {
+    using SegPair = SegPairT<T>;
     constexpr int TILE = BLOCK * IPT;
     constexpr int NW = BLOCK / 32;
     __shared__ int s_row_end[TILE];
-    __shared__ double s_prod[TILE];
+    __shared__ T s_prod[TILE];
     __shared__ SegPair s_warp[NW];
 
     const int tid = threadIdx.x;
@@ -325,16 +358,16 @@ __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int*
     // x gathers, then the products are stored — no serial load chains.
     {
         int re[IPT], ci[IPT];
-        double v[IPT], xv[IPT];
+        T v[IPT], xv[IPT];
 #pragma unroll
         for (int u = 0; u < IPT; ++u) {
             const int i = tid + u * BLOCK;
             re[u] = i < nr ? __ldg(rp + c0.x + 1 + i) : 0;
             ci[u] = i < nz ? ld_stream_i(col + c0.y + i, pol) : 0;
-            v[u] = i < nz ? ld_stream_d(val + c0.y + i, pol) : 0.0;
+            v[u] = i < nz ? ld_stream_v(val + c0.y + i, pol) : T(0);
         }
 #pragma unroll
-        for (int u = 0; u < IPT; ++u) xv[u] = (tid + u * BLOCK < nz) ? ld_x_ordered(x, ci[u]) : 0.0;
+        for (int u = 0; u < IPT; ++u) xv[u] = (tid + u * BLOCK < nz) ? ld_x_ordered(x, ci[u]) : T(0);
 #pragma unroll
         for (int u = 0; u < IPT; ++u) {
             const int i = tid + u * BLOCK;
@@ -356,7 +389,7 @@ __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int*
     int ri = lo, ki = d - lo;
     const int dend = min(d + IPT, total);
 
-    double acc = 0.0, head_val = 0.0;
+    T acc = T(0), head_val = T(0);
     int head_row = -1;
 #pragma unroll
     for (int it = 0; it < IPT; ++it) {
@@ -368,7 +401,7 @@ __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int*
             } else {                                // row ri ends here
                 if (head_row < 0) { head_row = ri; head_val = acc; }
                 else y[c0.x + ri] = acc;
-                acc = 0.0;
+                acc = T(0);
                 ++ri;
             }
         }
@@ -387,7 +420,7 @@ __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int*
     }
     if (lane == 31) s_warp[wid] = inc;
     __syncthreads();
-    SegPair wpre{0.0, 0};
+    SegPair wpre{T(0), 0};
     for (int w = 0; w < wid; ++w) wpre = w == 0 ? s_warp[0] : seg_combine(wpre, s_warp[w]);
     // exclusive prefix for this thread = (warp prefix) ⊕ (inclusive of lane-1)
     SegPair prev;
@@ -396,7 +429,7 @@ __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int*
     SegPair excl;
     if (lane == 0) excl = wpre;
     else excl = (wid == 0) ? prev : seg_combine(wpre, prev);
-    if (wid == 0 && lane == 0) excl = SegPair{0.0, 0};
+    if (wid == 0 && lane == 0) excl = SegPair{T(0), 0};
 
     if (head_row >= 0) y[c0.x + head_row] = excl.v + head_val;
 
@@ -411,39 +444,40 @@ __global__ void __launch_bounds__(BLOCK) merge_spmv_kernel(int nrows, const int*
 // merge items owned by ONE warp (row ends + products staged in that warp's
 // slice of shared memory, warp-only segmented scan): no block barriers, so
 // every warp streams independently (latency hiding by warp count).
-template <int IPT, int WARPS>
+template <int IPT, int WARPS, typename T>
 __global__ void __launch_bounds__(WARPS * 32) merge_warp_kernel(int nrows, int ntiles, const int* __restrict__ rp,
                                                                const int* __restrict__ col,
-                                                               const double* __restrict__ val,
-                                                               const double* __restrict__ x,
-                                                               double* __restrict__ y,
+                                                               const T* __restrict__ val,
+                                                               const T* __restrict__ x,
+                                                               T* __restrict__ y,
                                                                const int2* __restrict__ tile_coord,
                                                                int* __restrict__ carry_row,
-                                                               double* __restrict__ carry_val) {
+                                                               T* __restrict__ carry_val) {
+    using SegPair = SegPairT<T>;
     constexpr int TILE = 32 * IPT;
     __shared__ int s_row_end_all[WARPS][TILE];
-    __shared__ double s_prod_all[WARPS][TILE];
+    __shared__ T s_prod_all[WARPS][TILE];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int tile = blockIdx.x * WARPS + w;
     if (tile >= ntiles) return;
     int* s_row_end = s_row_end_all[w];
-    double* s_prod = s_prod_all[w];
+    T* s_prod = s_prod_all[w];
     const uint64_t pol = evict_first_policy();
     const int2 c0 = __ldg(tile_coord + tile);
     const int2 c1 = __ldg(tile_coord + tile + 1);
     const int nr = c1.x - c0.x, nz = c1.y - c0.y;
     {
         int re[IPT], ci[IPT];
-        double v[IPT], xv[IPT];
+        T v[IPT], xv[IPT];
 #pragma unroll
         for (int u = 0; u < IPT; ++u) {
             const int i = lane + u * 32;
             re[u] = i < nr ? __ldg(rp + c0.x + 1 + i) : 0;
             ci[u] = i < nz ? ld_stream_i(col + c0.y + i, pol) : 0;
-            v[u] = i < nz ? ld_stream_d(val + c0.y + i, pol) : 0.0;
+            v[u] = i < nz ? ld_stream_v(val + c0.y + i, pol) : T(0);
         }
 #pragma unroll
-        for (int u = 0; u < IPT; ++u) xv[u] = (lane + u * 32 < nz) ? ld_x_ordered(x, ci[u]) : 0.0;
+        for (int u = 0; u < IPT; ++u) xv[u] = (lane + u * 32 < nz) ? ld_x_ordered(x, ci[u]) : T(0);
 #pragma unroll
         for (int u = 0; u < IPT; ++u) {
             const int i = lane + u * 32;
@@ -463,7 +497,7 @@ __global__ void __launch_bounds__(WARPS * 32) merge_warp_kernel(int nrows, int n
     int ri = lo, kabs = c0.y + d - lo;
     const int dend = min(d + IPT, total);
     int re = ri < nr ? s_row_end[ri] : 0x7fffffff;
-    double acc = 0.0, head_val = 0.0;
+    T acc = T(0), head_val = T(0);
     int head_row = -1;
 #pragma unroll
     for (int it = 0; it < IPT; ++it) {
@@ -474,7 +508,7 @@ __global__ void __launch_bounds__(WARPS * 32) merge_warp_kernel(int nrows, int n
             } else {
                 if (head_row < 0) { head_row = ri; head_val = acc; }
                 else y[c0.x + ri] = acc;
-                acc = 0.0;
+                acc = T(0);
                 ++ri;
                 re = ri < nr ? s_row_end[ri] : 0x7fffffff;
             }
@@ -489,8 +523,8 @@ __global__ void __launch_bounds__(WARPS * 32) merge_warp_kernel(int nrows, int n
         o.f = __shfl_up_sync(0xffffffffu, inc.f, off);
         if (lane >= off) inc = seg_combine(o, inc);
     }
-    double excl = __shfl_up_sync(0xffffffffu, inc.v, 1);
-    if (lane == 0) excl = 0.0;
+    T excl = __shfl_up_sync(0xffffffffu, inc.v, 1);
+    if (lane == 0) excl = T(0);
     if (head_row >= 0) y[c0.x + head_row] = excl + head_val;
     if (lane == 31) {
         carry_row[tile] = c1.x;
@@ -507,14 +541,15 @@ __global__ void __launch_bounds__(WARPS * 32) merge_warp_kernel(int nrows, int n
 // tree); merge_fixup_kernel (one thread per tile) handles the short ones.
 constexpr int kLongRun = 32;
 
+template <typename T>
 __global__ void merge_fixup_kernel(int ntiles, int nrows, const int* __restrict__ carry_row,
-                                   const double* __restrict__ carry_val, double* __restrict__ y) {
+                                   const T* __restrict__ carry_val, T* __restrict__ y) {
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= ntiles) return;
     const int row = carry_row[t];
     if (row >= nrows) return;
     if (t > 0 && carry_row[t - 1] == row) return;
-    double s = carry_val[t];
+    T s = carry_val[t];
     int u = t + 1;
     for (; u < ntiles && u - t < kLongRun && carry_row[u] == row; ++u) s += carry_val[u];
     if (u - t >= kLongRun) return;   // a long run: merge_fixup_long_kernel adds it
@@ -522,13 +557,14 @@ __global__ void merge_fixup_kernel(int ntiles, int nrows, const int* __restrict_
 }
 
 // runs[i] = (first tile, number of tiles, row)
-__global__ void merge_fixup_long_kernel(int nruns, const int4* __restrict__ runs, const double* __restrict__ carry_val,
-                                        double* __restrict__ y) {
+template <typename T>
+__global__ void merge_fixup_long_kernel(int nruns, const int4* __restrict__ runs, const T* __restrict__ carry_val,
+                                        T* __restrict__ y) {
     const int lane = threadIdx.x & 31;
     const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
     if (i >= nruns) return;
     const int4 r = runs[i];
-    double s = 0.0;
+    T s = T(0);
     for (int u = lane; u < r.y; u += 32) s += carry_val[r.x + u];
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
@@ -592,26 +628,26 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
 
 constexpr int kStreamVecFlag = 0x40000000;   // item.y flag: the item holds a row longer than VEC
 
-template <int NB, int RMAX>
+template <int NB, int RMAX, typename T>
 struct StreamStage {
-    double val[NB + 8];
+    T val[NB + 8];
     int col[NB + 8];
     int rp[RMAX + 8];
 };
 
-template <int BLOCK, int STAGES, int NB, int RMAX, int VEC>
+template <int BLOCK, int STAGES, int NB, int RMAX, int VEC, typename T>
 __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const int4* __restrict__ items,
                                                                const int* __restrict__ rp,
                                                                const int* __restrict__ col,
-                                                               const double* __restrict__ val,
-                                                               const double* __restrict__ x,
-                                                               double* __restrict__ y,
-                                                               double* __restrict__ carry) {
-    using Stage = StreamStage<NB, RMAX>;
+                                                               const T* __restrict__ val,
+                                                               const T* __restrict__ x,
+                                                               T* __restrict__ y,
+                                                               T* __restrict__ carry) {
+    using Stage = StreamStage<NB, RMAX, T>;
     extern __shared__ __align__(128) unsigned char smem_raw[];
     Stage* st = reinterpret_cast<Stage*>(smem_raw);
     __shared__ __align__(8) uint64_t full[STAGES];
-    __shared__ double s_red[BLOCK / 32];
+    __shared__ T s_red[BLOCK / 32];
 
     const int tid = threadIdx.x;
     const int G = gridDim.x;
@@ -629,7 +665,7 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
         const int4 it = __ldg(items + blockIdx.x + (int64_t)j * G);
         Stage& S = st[j % STAGES];
         const int k0a = it.z & ~3, k1a = (it.w + 3) & ~3;
-        uint32_t bytes = (uint32_t)(k1a - k0a) * 12u;
+        uint32_t bytes = (uint32_t)(k1a - k0a) * (uint32_t)(sizeof(T) + 4);
         int r0a = 0, r1a = 0;
         if (it.y >= 0) {
             const int r1 = it.y & ~kStreamVecFlag;
@@ -639,7 +675,7 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
         }
         mbar_arrive_expect_tx(&full[j % STAGES], bytes);
         if (k1a > k0a) {
-            tma_load_1d(S.val, val + k0a, (uint32_t)(k1a - k0a) * 8u, &full[j % STAGES], pol);
+            tma_load_1d(S.val, val + k0a, (uint32_t)(k1a - k0a) * (uint32_t)sizeof(T), &full[j % STAGES], pol);
             tma_load_1d(S.col, col + k0a, (uint32_t)(k1a - k0a) * 4u, &full[j % STAGES], pol);
         }
         if (r1a > r0a) tma_load_1d(S.rp, rp + r0a, (uint32_t)(r1a - r0a) * 4u, &full[j % STAGES], pol);
@@ -662,18 +698,18 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
         // products, so the gathers overlap instead of forming a serial chain.
         {
             constexpr int PER = (NB + BLOCK - 1) / BLOCK;
-            double v[PER];
+            T v[PER];
             int c[PER];
 #pragma unroll
             for (int u = 0; u < PER; ++u) {
                 const int i = tid + u * BLOCK;
-                v[u] = 0.0;
+                v[u] = T(0);
                 c[u] = 0;
                 if (i < nz) { v[u] = S.val[off + i]; c[u] = S.col[off + i]; }
             }
-            double xv[PER];
+            T xv[PER];
 #pragma unroll
-            for (int u = 0; u < PER; ++u) xv[u] = (tid + u * BLOCK < nz) ? ld_x_ordered(x, c[u]) : 0.0;
+            for (int u = 0; u < PER; ++u) xv[u] = (tid + u * BLOCK < nz) ? ld_x_ordered(x, c[u]) : T(0);
 #pragma unroll
             for (int u = 0; u < PER; ++u) {
                 const int i = tid + u * BLOCK;
@@ -691,7 +727,7 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
             for (int r = tid; r < r1 - r0; r += BLOCK) {
                 const int s = S.rp[roff + r] - k0a, e = S.rp[roff + r + 1] - k0a;
                 if (e - s > VEC) continue;
-                double acc = +0.0;
+                T acc = T(+0.0);
                 for (int k = s; k < e; ++k) acc = acc + S.val[k];
                 y[r0 + r] = acc;
             }
@@ -700,7 +736,7 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
                 for (int r = w; r < r1 - r0; r += BLOCK / 32) {
                     const int s = S.rp[roff + r] - k0a, e = S.rp[roff + r + 1] - k0a;
                     if (e - s <= VEC) continue;
-                    double acc = 0.0;
+                    T acc = T(0);
                     for (int k = s + lane; k < e; k += 32) acc += S.val[k];
 #pragma unroll
                     for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
@@ -709,14 +745,14 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
             }
         } else {
             // long-row piece: deterministic block sum -> carry slot
-            double acc = 0.0;
+            T acc = T(0);
             for (int i = tid; i < nz; i += BLOCK) acc += S.val[off + i];
 #pragma unroll
             for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
             if ((tid & 31) == 0) s_red[tid >> 5] = acc;
             __syncthreads();
             if (tid == 0) {
-                double t = 0.0;
+                T t = T(0);
                 for (int w = 0; w < BLOCK / 32; ++w) t += s_red[w];
                 carry[-it.y - 1] = t;
             }
@@ -728,13 +764,14 @@ __global__ void __launch_bounds__(BLOCK) csr_stream_tma_kernel(int nitems, const
 
 // y[row] = sum of its long-row pieces: one warp per long row, lane-strided
 // over the pieces then a fixed shuffle tree (deterministic)
-__global__ void csr_stream_fixup_kernel(int nlong, const int4* __restrict__ longrows, const double* __restrict__ carry,
-                                        double* __restrict__ y) {
+template <typename T>
+__global__ void csr_stream_fixup_kernel(int nlong, const int4* __restrict__ longrows, const T* __restrict__ carry,
+                                        T* __restrict__ y) {
     const int lane = threadIdx.x & 31;
     const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
     if (i >= nlong) return;
     const int4 L = longrows[i];   // (row, first piece, end piece, -)
-    double s = 0.0;
+    T s = T(0);
     for (int p = L.y + lane; p < L.z; p += 32) s += carry[p];
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
@@ -827,10 +864,11 @@ __global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const
     if (lane == 0 && r < nrows) chunk_len[r >> 5] = (mn == mx) ? mx : (mx | kSellMasked);
 }
 
+template <typename T>
 __global__ void sell_fill_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,
-                                 const int* __restrict__ src_col, const double* __restrict__ src_val,
+                                 const int* __restrict__ src_col, const T* __restrict__ src_val,
                                  const int64_t* __restrict__ chunk_ptr, int* __restrict__ col,
-                                 double* __restrict__ val) {
+                                 T* __restrict__ val) {
     const int r = blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= nrows) return;
     const int o = perm ? perm[r] : r;
@@ -874,13 +912,15 @@ __global__ void sell_col16_kernel(int nrows, int nchunks, const int64_t* __restr
 }
 
 // halo pack / unpack --------------------------------------------------
-__global__ void gather_kernel(int64_t n, const int* __restrict__ idx, const double* __restrict__ src,
-                              double* __restrict__ dst) {
+template <typename T>
+__global__ void gather_kernel(int64_t n, const int* __restrict__ idx, const T* __restrict__ src,
+                              T* __restrict__ dst) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         dst[i] = src[idx[i]];
 }
-__global__ void scatter_kernel(int64_t n, const int* __restrict__ idx, const double* __restrict__ src,
-                               double* __restrict__ dst) {
+template <typename T>
+__global__ void scatter_kernel(int64_t n, const int* __restrict__ idx, const T* __restrict__ src,
+                               T* __restrict__ dst) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         dst[idx[i]] = src[i];
 }

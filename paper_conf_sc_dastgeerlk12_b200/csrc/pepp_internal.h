@@ -41,7 +41,7 @@ bool vector_simulated(const pepp_vector_t* v);
 // host-only utilities run) on machines without NCCL or a GPU.
 typedef struct ncclComm_opaque* ncclComm_t;
 typedef struct { char internal[128]; } ncclUniqueId;
-enum { NCCL_INT32 = 2, NCCL_INT64 = 4, NCCL_FLOAT64 = 8 };
+enum { NCCL_INT32 = 2, NCCL_INT64 = 4, NCCL_FLOAT32 = 7, NCCL_FLOAT64 = 8 };
 enum { NCCL_OP_MAX = 2 };
 struct Nccl {
     int (*GetUniqueId)(ncclUniqueId*);

@@ -59,7 +59,7 @@ struct PeerXfer {            // halo traffic with one peer
     int64_t count;
     int64_t contig_start;    // >= 0: the entries are y[contig_start, contig_start+count)
     int* d_idx = nullptr;    // else: global indices into y (device)
-    double* d_buf = nullptr; // pack / unpack buffer
+    void* d_buf = nullptr;   // pack / unpack buffer (value type)
 };
 
 }  // namespace
@@ -78,7 +78,9 @@ struct pepp_spmv_plan_s {
     // device CSR
     int* d_rp = nullptr;
     int* d_col = nullptr;
-    double* d_val = nullptr;
+    void* d_val = nullptr;      // value_type elements (fp64 or fp32)
+    int vt = PEPP_VALUE_F64;     // value type of the plan
+    size_t esz = 8;              // bytes per value
     int64_t dev_bytes = 0;
 
     // SELL-C-σ
@@ -93,26 +95,26 @@ struct pepp_spmv_plan_s {
     int16_t* d_scol16 = nullptr;
     int sell_cpw = 1;            // chunks per σ window (chunk order is transposed when > 1)
     int64_t sell_col16_chunks = 0;
-    double* d_sval = nullptr;
+    void* d_sval = nullptr;
 
     // merge path
     int ntiles = 0;
     int2* d_tile = nullptr;
     int* d_carry_row = nullptr;
-    double* d_carry_val = nullptr;
+    void* d_carry_val = nullptr;   // carries are stored in the plan's value type (8 B slots)
     int nlongruns = 0, nlongruns_w = 0;
     int4* d_longruns = nullptr;
     int4* d_longruns_w = nullptr;
     int ntiles_w = 0;
     int2* d_tile_w = nullptr;
     int* d_carry_row_w = nullptr;
-    double* d_carry_val_w = nullptr;
+    void* d_carry_val_w = nullptr;
 
     // TMA CSR-stream
     int nitems = 0, nlong = 0, grid_stream = 0;
     int4* d_items = nullptr;
     int4* d_longrows = nullptr;
-    double* d_stream_carry = nullptr;
+    void* d_stream_carry = nullptr;
 
     // occupancy-derived grids
     int grid_csr[6] = {0};   // per log2(TPR)
@@ -144,8 +146,8 @@ struct pepp_spmv_plan_s {
     std::vector<PeerXfer> recv_x, send_x;
 
     // plan-owned x / y for pepp_spmv_exec_host (allocated on first use)
-    double* d_hx = nullptr;
-    double* d_hy = nullptr;
+    void* d_hx = nullptr;
+    void* d_hy = nullptr;
 };
 
 namespace {
@@ -155,6 +157,16 @@ namespace {
         cudaError_t _e = (expr);                              \
         if (_e != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; } \
     } while (0)
+
+// device buffer of `bytes` bytes owned by the plan (value-typed arrays)
+pepp_status_t dalloc_bytes(pepp_spmv_plan_t* p, void** ptr, int64_t bytes) {
+    *ptr = nullptr;
+    if (bytes <= 0) bytes = 8;
+    cudaError_t e = cudaMalloc(ptr, (size_t)bytes);
+    if (e != cudaSuccess) { (void)cudaGetLastError(); *ptr = nullptr; return e == cudaErrorMemoryAllocation ? PEPP_E_NOMEM : PEPP_E_CUDA; }
+    p->dev_bytes += bytes;
+    return PEPP_OK;
+}
 
 // plan-time scratch device buffer, freed on every exit path
 template <typename T>
@@ -261,12 +273,16 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     }
     p->sell_sigma = sigma;
     if ((s = dalloc(p, &p->d_scol, p->sell_slots + 32))) return s;
-    if ((s = dalloc(p, &p->d_sval, p->sell_slots + 32))) return s;
+    if ((s = dalloc_bytes(p, &p->d_sval, (p->sell_slots + 32) * (int64_t)p->esz))) return s;
     // padding slots are never read (lanes mask by row length), but keep them defined
     PEPP_CUDA_TRY(cudaMemsetAsync(p->d_scol, 0, sizeof(int) * (p->sell_slots + 32), st));
-    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_sval, 0, sizeof(double) * (p->sell_slots + 32), st));
-    pepp::k::sell_fill_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, p->d_col, p->d_val, p->d_chunk_ptr,
-                                                   p->d_scol, p->d_sval);
+    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_sval, 0, p->esz * (p->sell_slots + 32), st));
+    if (p->vt == PEPP_VALUE_F32)
+        pepp::k::sell_fill_kernel<float><<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, p->d_col, (const float*)p->d_val,
+                                                            p->d_chunk_ptr, p->d_scol, (float*)p->d_sval);
+    else
+        pepp::k::sell_fill_kernel<double><<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, p->d_col, (const double*)p->d_val,
+                                                             p->d_chunk_ptr, p->d_scol, (double*)p->d_sval);
     PEPP_CUDA_TRY(cudaGetLastError());
     // 16-bit column deltas where a whole chunk allows them (banded / stencil
     // structure): 2 instead of 4 bytes of index per stored slot
@@ -324,7 +340,7 @@ pepp_status_t prepare_merge(pepp_spmv_plan_t* p, cudaStream_t st) {
     pepp_status_t s;
     if ((s = dalloc(p, &p->d_tile, (int64_t)p->ntiles + 1))) return s;
     if ((s = dalloc(p, &p->d_carry_row, std::max(p->ntiles, 1)))) return s;
-    if ((s = dalloc(p, &p->d_carry_val, std::max(p->ntiles, 1)))) return s;
+    if ((s = dalloc_bytes(p, &p->d_carry_val, 8 * (int64_t)std::max(p->ntiles, 1)))) return s;
     const int tb = 256;
     pepp::k::merge_tile_search_kernel<<<(p->ntiles + 1 + tb - 1) / tb, tb, 0, st>>>(
         (int)p->nrows, p->nnz, p->d_rp, kMergeTile, p->ntiles, p->d_tile);
@@ -332,7 +348,7 @@ pepp_status_t prepare_merge(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->ntiles_w = (int)((total + kMergeWarpTile - 1) / kMergeWarpTile);
     if ((s = dalloc(p, &p->d_tile_w, (int64_t)p->ntiles_w + 1))) return s;
     if ((s = dalloc(p, &p->d_carry_row_w, std::max(p->ntiles_w, 1)))) return s;
-    if ((s = dalloc(p, &p->d_carry_val_w, std::max(p->ntiles_w, 1)))) return s;
+    if ((s = dalloc_bytes(p, &p->d_carry_val_w, 8 * (int64_t)std::max(p->ntiles_w, 1)))) return s;
     pepp::k::merge_tile_search_kernel<<<(p->ntiles_w + 1 + tb - 1) / tb, tb, 0, st>>>(
         (int)p->nrows, p->nnz, p->d_rp, kMergeWarpTile, p->ntiles_w, p->d_tile_w);
     PEPP_CUDA_TRY(cudaGetLastError());
@@ -343,8 +359,17 @@ pepp_status_t prepare_merge(pepp_spmv_plan_t* p, cudaStream_t st) {
 }
 
 // ---------------------------------------------------------------- CSR-stream prep
-auto stream_kernel() { return pepp::k::csr_stream_tma_kernel<kStreamBlock, kStreamStages, kStreamNB, kStreamRMAX, kStreamVecMinLen>; }
-constexpr size_t kStreamSmem = sizeof(pepp::k::StreamStage<kStreamNB, kStreamRMAX>) * kStreamStages;
+template <typename T>
+auto stream_kernel() { return pepp::k::csr_stream_tma_kernel<kStreamBlock, kStreamStages, kStreamNB, kStreamRMAX, kStreamVecMinLen, T>; }
+template <typename T>
+constexpr size_t stream_smem() { return sizeof(pepp::k::StreamStage<kStreamNB, kStreamRMAX, T>) * kStreamStages; }
+
+template <typename T>
+pepp_status_t stream_occupancy(int* occ) {
+    PEPP_CUDA_TRY(cudaFuncSetAttribute(stream_kernel<T>(), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)stream_smem<T>()));
+    PEPP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, stream_kernel<T>(), kStreamBlock, stream_smem<T>()));
+    return PEPP_OK;
+}
 
 pepp_status_t prepare_stream(pepp_spmv_plan_t* p, cudaStream_t st) {
     const int64_t R = p->nrows;
@@ -383,12 +408,11 @@ pepp_status_t prepare_stream(pepp_spmv_plan_t* p, cudaStream_t st) {
     PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_items, items.data(), sizeof(int4) * items.size(), cudaMemcpyHostToDevice, st));
     if (p->nlong) {
         if ((s = dalloc(p, &p->d_longrows, p->nlong))) return s;
-        if ((s = dalloc(p, &p->d_stream_carry, piece))) return s;
+        if ((s = dalloc_bytes(p, &p->d_stream_carry, 8 * (int64_t)piece))) return s;
         PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_longrows, longrows.data(), sizeof(int4) * longrows.size(), cudaMemcpyHostToDevice, st));
     }
-    PEPP_CUDA_TRY(cudaFuncSetAttribute(stream_kernel(), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kStreamSmem));
     int occ = 0;
-    PEPP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, stream_kernel(), kStreamBlock, kStreamSmem));
+    if ((s = p->vt == PEPP_VALUE_F32 ? stream_occupancy<float>(&occ) : stream_occupancy<double>(&occ))) return s;
     if (occ < 1) return PEPP_E_UNSUPPORTED;
     p->grid_stream = (int)std::min<int64_t>((int64_t)p->sm_count * occ, p->nitems);
     PEPP_CUDA_TRY(cudaStreamSynchronize(st));
@@ -396,72 +420,80 @@ pepp_status_t prepare_stream(pepp_spmv_plan_t* p, cudaStream_t st) {
 }
 
 // ---------------------------------------------------------------- launches
-template <int TPR>
-void launch_csr_vector(const pepp_spmv_plan_t* p, const double* x, double* y, cudaStream_t st, int grid) {
-    pepp::k::csr_vector_kernel<TPR, kBlock><<<grid, kBlock, 0, st>>>((int)p->nrows, p->d_rp, p->d_col, p->d_val, x, y);
+template <int TPR, typename T>
+void launch_csr_vector(const pepp_spmv_plan_t* p, const T* x, T* y, cudaStream_t st, int grid) {
+    pepp::k::csr_vector_kernel<TPR, kBlock, T><<<grid, kBlock, 0, st>>>((int)p->nrows, p->d_rp, p->d_col,
+                                                                        (const T*)p->d_val, x, y);
 }
 
-pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const double* x, double* y, cudaStream_t st) {
+template <typename T>
+pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y, cudaStream_t st) {
     if (p->nrows == 0) return PEPP_OK;
+    const T* val = (const T*)p->d_val;
     switch (c.variant) {
     case PEPP_V_CSR_VECTOR:
         switch (c.param) {
-        case 2: launch_csr_vector<2>(p, x, y, st, p->grid_csr[1]); break;
-        case 4: launch_csr_vector<4>(p, x, y, st, p->grid_csr[2]); break;
-        case 8: launch_csr_vector<8>(p, x, y, st, p->grid_csr[3]); break;
-        case 16: launch_csr_vector<16>(p, x, y, st, p->grid_csr[4]); break;
-        case 32: launch_csr_vector<32>(p, x, y, st, p->grid_csr[5]); break;
+        case 2: launch_csr_vector<2, T>(p, x, y, st, p->grid_csr[1]); break;
+        case 4: launch_csr_vector<4, T>(p, x, y, st, p->grid_csr[2]); break;
+        case 8: launch_csr_vector<8, T>(p, x, y, st, p->grid_csr[3]); break;
+        case 16: launch_csr_vector<16, T>(p, x, y, st, p->grid_csr[4]); break;
+        case 32: launch_csr_vector<32, T>(p, x, y, st, p->grid_csr[5]); break;
         default: return PEPP_E_INVALID;
         }
         break;
     case PEPP_V_MERGE_PATH:
         if (c.param == kMergeWarpParam) {
             if (p->ntiles_w > 0) {
-                pepp::k::merge_warp_kernel<kMergeWarpIPT, kMergeWarps>
+                pepp::k::merge_warp_kernel<kMergeWarpIPT, kMergeWarps, T>
                     <<<(p->ntiles_w + kMergeWarps - 1) / kMergeWarps, kMergeWarps * 32, 0, st>>>(
-                        (int)p->nrows, p->ntiles_w, p->d_rp, p->d_col, p->d_val, x, y, p->d_tile_w, p->d_carry_row_w,
-                        p->d_carry_val_w);
-                pepp::k::merge_fixup_kernel<<<(p->ntiles_w + 255) / 256, 256, 0, st>>>(
-                    p->ntiles_w, (int)p->nrows, p->d_carry_row_w, p->d_carry_val_w, y);
+                        (int)p->nrows, p->ntiles_w, p->d_rp, p->d_col, val, x, y, p->d_tile_w, p->d_carry_row_w,
+                        (T*)p->d_carry_val_w);
+                pepp::k::merge_fixup_kernel<T><<<(p->ntiles_w + 255) / 256, 256, 0, st>>>(
+                    p->ntiles_w, (int)p->nrows, p->d_carry_row_w, (const T*)p->d_carry_val_w, y);
                 if (p->nlongruns_w)
-                    pepp::k::merge_fixup_long_kernel<<<(p->nlongruns_w * 32 + 255) / 256, 256, 0, st>>>(
-                        p->nlongruns_w, p->d_longruns_w, p->d_carry_val_w, y);
+                    pepp::k::merge_fixup_long_kernel<T><<<(p->nlongruns_w * 32 + 255) / 256, 256, 0, st>>>(
+                        p->nlongruns_w, p->d_longruns_w, (const T*)p->d_carry_val_w, y);
             }
             break;
         }
         if (p->ntiles > 0) {
-            pepp::k::merge_spmv_kernel<kMergeBlock, kMergeIPT><<<p->ntiles, kMergeBlock, 0, st>>>(
-                (int)p->nrows, p->d_rp, p->d_col, p->d_val, x, y, p->d_tile, p->d_carry_row, p->d_carry_val);
-            pepp::k::merge_fixup_kernel<<<(p->ntiles + 255) / 256, 256, 0, st>>>(
-                p->ntiles, (int)p->nrows, p->d_carry_row, p->d_carry_val, y);
+            pepp::k::merge_spmv_kernel<kMergeBlock, kMergeIPT, T><<<p->ntiles, kMergeBlock, 0, st>>>(
+                (int)p->nrows, p->d_rp, p->d_col, val, x, y, p->d_tile, p->d_carry_row, (T*)p->d_carry_val);
+            pepp::k::merge_fixup_kernel<T><<<(p->ntiles + 255) / 256, 256, 0, st>>>(
+                p->ntiles, (int)p->nrows, p->d_carry_row, (const T*)p->d_carry_val, y);
             if (p->nlongruns)
-                pepp::k::merge_fixup_long_kernel<<<(p->nlongruns * 32 + 255) / 256, 256, 0, st>>>(
-                    p->nlongruns, p->d_longruns, p->d_carry_val, y);
+                pepp::k::merge_fixup_long_kernel<T><<<(p->nlongruns * 32 + 255) / 256, 256, 0, st>>>(
+                    p->nlongruns, p->d_longruns, (const T*)p->d_carry_val, y);
         }
         break;
     case PEPP_V_CSR_STREAM:
         if (p->nitems > 0) {
-            stream_kernel()<<<p->grid_stream, kStreamBlock, kStreamSmem, st>>>(
-                p->nitems, p->d_items, p->d_rp, p->d_col, p->d_val, x, y, p->d_stream_carry);
+            stream_kernel<T>()<<<p->grid_stream, kStreamBlock, stream_smem<T>(), st>>>(
+                p->nitems, p->d_items, p->d_rp, p->d_col, val, x, y, (T*)p->d_stream_carry);
             if (p->nlong)
-                pepp::k::csr_stream_fixup_kernel<<<(p->nlong * 32 + 255) / 256, 256, 0, st>>>(p->nlong, p->d_longrows,
-                                                                                              p->d_stream_carry, y);
+                pepp::k::csr_stream_fixup_kernel<T><<<(p->nlong * 32 + 255) / 256, 256, 0, st>>>(
+                    p->nlong, p->d_longrows, (const T*)p->d_stream_carry, y);
         }
         break;
     case PEPP_V_SELL:
         if (p->d_perm)
-            pepp::k::sell_kernel<kBlock, true><<<p->grid_sell, kBlock, 0, st>>>(
+            pepp::k::sell_kernel<kBlock, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
-                p->d_scol16, p->d_sval, x, y, p->sell_cpw);
+                p->d_scol16, (const T*)p->d_sval, x, y, p->sell_cpw);
         else
-            pepp::k::sell_kernel<kBlock, false><<<p->grid_sell, kBlock, 0, st>>>(
+            pepp::k::sell_kernel<kBlock, false, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr, p->d_scol,
-                p->d_scol16, p->d_sval, x, y, 1);
+                p->d_scol16, (const T*)p->d_sval, x, y, 1);
         break;
     default:
         return PEPP_E_INVALID;
     }
     return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
+}
+
+pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const void* x, void* y, cudaStream_t st) {
+    if (p->vt == PEPP_VALUE_F32) return launch_t<float>(p, c, (const float*)x, (float*)y, st);
+    return launch_t<double>(p, c, (const double*)x, (double*)y, st);
 }
 
 // ---------------------------------------------------------------- history
@@ -593,37 +625,51 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out) {
 // ---------------------------------------------------------------- NCCL
 pepp_status_t nccl_ok(const pepp_spmv_plan_t* p, int r) { (void)p; return r == 0 ? PEPP_OK : PEPP_E_NCCL; }
 
-pepp_status_t exchange_allgather(pepp_spmv_plan_t* p, double* y, cudaStream_t st) {
+int nccl_value_type(const pepp_spmv_plan_t* p) { return p->vt == PEPP_VALUE_F32 ? pepp::NCCL_FLOAT32 : pepp::NCCL_FLOAT64; }
+
+pepp_status_t exchange_allgather(pepp_spmv_plan_t* p, void* y, cudaStream_t st) {
     const Nccl* n = p->nccl;
+    char* yb = (char*)y;
     if (nccl_ok(p, n->GroupStart())) return PEPP_E_NCCL;
     for (int r = 0; r < p->opts.nranks; ++r) {
         const int64_t b = p->row_bounds[r], cnt = p->row_bounds[r + 1] - b;
         if (cnt == 0) continue;
-        if (n->Broadcast(y + b, y + b, (size_t)cnt, pepp::NCCL_FLOAT64, r, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
+        char* at = yb + b * (int64_t)p->esz;
+        if (n->Broadcast(at, at, (size_t)cnt, nccl_value_type(p), r, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
     }
     return nccl_ok(p, n->GroupEnd());
 }
 
-pepp_status_t exchange_halo(pepp_spmv_plan_t* p, double* y, cudaStream_t st) {
+template <typename T>
+void pack_unpack(pepp_spmv_plan_t* p, T* y, bool pack, cudaStream_t st) {
+    for (auto& t : pack ? p->send_x : p->recv_x) {
+        if (t.contig_start >= 0 || t.count == 0) continue;
+        const int g = (int)std::min<int64_t>(1024, (t.count + 255) / 256);
+        if (pack) pepp::k::gather_kernel<T><<<g, 256, 0, st>>>(t.count, t.d_idx, y, (T*)t.d_buf);
+        else pepp::k::scatter_kernel<T><<<g, 256, 0, st>>>(t.count, t.d_idx, (const T*)t.d_buf, y);
+    }
+}
+
+pepp_status_t exchange_halo(pepp_spmv_plan_t* p, void* y, cudaStream_t st) {
     const Nccl* n = p->nccl;
-    for (auto& t : p->send_x)
-        if (t.contig_start < 0 && t.count > 0)
-            pepp::k::gather_kernel<<<(int)std::min<int64_t>(1024, (t.count + 255) / 256), 256, 0, st>>>(t.count, t.d_idx, y, t.d_buf);
+    char* yb = (char*)y;
+    const int64_t es = (int64_t)p->esz;
+    if (p->vt == PEPP_VALUE_F32) pack_unpack<float>(p, (float*)y, true, st);
+    else pack_unpack<double>(p, (double*)y, true, st);
     if (n->GroupStart()) return PEPP_E_NCCL;
     for (auto& t : p->send_x) {
         if (!t.count) continue;
-        const double* src = t.contig_start >= 0 ? y + t.contig_start : t.d_buf;
-        if (n->Send(src, (size_t)t.count, pepp::NCCL_FLOAT64, t.peer, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
+        const void* src = t.contig_start >= 0 ? (const void*)(yb + t.contig_start * es) : t.d_buf;
+        if (n->Send(src, (size_t)t.count, nccl_value_type(p), t.peer, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
     }
     for (auto& t : p->recv_x) {
         if (!t.count) continue;
-        double* dst = t.contig_start >= 0 ? y + t.contig_start : t.d_buf;
-        if (n->Recv(dst, (size_t)t.count, pepp::NCCL_FLOAT64, t.peer, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
+        void* dst = t.contig_start >= 0 ? (void*)(yb + t.contig_start * es) : t.d_buf;
+        if (n->Recv(dst, (size_t)t.count, nccl_value_type(p), t.peer, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
     }
     if (n->GroupEnd()) return PEPP_E_NCCL;
-    for (auto& t : p->recv_x)
-        if (t.contig_start < 0 && t.count > 0)
-            pepp::k::scatter_kernel<<<(int)std::min<int64_t>(1024, (t.count + 255) / 256), 256, 0, st>>>(t.count, t.d_idx, t.d_buf, y);
+    if (p->vt == PEPP_VALUE_F32) pack_unpack<float>(p, (float*)y, false, st);
+    else pack_unpack<double>(p, (double*)y, false, st);
     return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
 }
 
@@ -678,7 +724,7 @@ pepp_status_t setup_halo(pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts
         const bool contig = !lst.empty() && (int64_t)lst.back() - lst.front() + 1 == t.count;
         t.contig_start = contig ? lst.front() : -1;
         if (!contig && t.count) {
-            DevTmp<double> buf;
+            DevTmp<double> buf;   // 8-byte slots hold either value type
             PEPP_CUDA_TRY(buf.alloc(t.count));
             t.d_idx = d_list.release();
             t.d_buf = buf.release();
@@ -707,6 +753,9 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     // ---- argument checks (host, O(1)) ----
     if (A->nrows < 0 || A->ncols < 0 || A->nnz < 0 || !A->row_ptr) return PEPP_E_INVALID;
     if (A->nnz > 0 && (!A->col_idx || !A->values)) return PEPP_E_INVALID;
+    if (A->value_type != PEPP_VALUE_F64 && A->value_type != PEPP_VALUE_F32) return PEPP_E_INVALID;
+    p->vt = A->value_type;
+    p->esz = p->vt == PEPP_VALUE_F32 ? sizeof(float) : sizeof(double);
     if (o->nranks < 1 || o->rank < 0 || o->rank >= o->nranks) return PEPP_E_INVALID;
     if (o->nranks > 1 && !o->row_bounds) return PEPP_E_INVALID;
     if (A->nnz + 8 >= (int64_t)INT32_MAX || A->ncols >= (int64_t)INT32_MAX || A->nrows >= (int64_t)INT32_MAX)
@@ -759,13 +808,13 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     if ((s = dalloc(p, &p->d_rp, A->nrows + 1 + 8))) return s;   // +8: aligned 16-B bulk copies may overrun
     PEPP_CUDA_TRY(cudaMemsetAsync(p->d_rp, 0, sizeof(int) * (A->nrows + 1 + 8), st));
     if ((s = dalloc(p, &p->d_col, nstore))) return s;
-    if ((s = dalloc(p, &p->d_val, nstore))) return s;
+    if ((s = dalloc_bytes(p, &p->d_val, nstore * (int64_t)p->esz))) return s;
     PEPP_CUDA_TRY(cudaMemsetAsync(p->d_col, 0, sizeof(int) * nstore, st));
-    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_val, 0, sizeof(double) * nstore, st));
+    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_val, 0, p->esz * nstore, st));
     const cudaMemcpyKind kind = A->on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
     if (A->nnz) {
         PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_col + p->pad, A->col_idx, sizeof(int) * A->nnz, kind, st));
-        PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_val + p->pad, A->values, sizeof(double) * A->nnz, kind, st));
+        PEPP_CUDA_TRY(cudaMemcpyAsync((char*)p->d_val + p->pad * p->esz, A->values, p->esz * A->nnz, kind, st));
     }
     DevTmp<int64_t> rp64;
     DevTmp<pepp::k::RowStats> stats;
@@ -842,14 +891,14 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     p->pending.assign(p->cands.size(), 0);
     I.ncandidates = (int32_t)p->cands.size();
 
-    p->grid_csr[1] = grid_for((const void*)pepp::k::csr_vector_kernel<2, kBlock>, kBlock, A->nrows, kBlock / 2, p->sm_count);
-    p->grid_csr[2] = grid_for((const void*)pepp::k::csr_vector_kernel<4, kBlock>, kBlock, A->nrows, kBlock / 4, p->sm_count);
-    p->grid_csr[3] = grid_for((const void*)pepp::k::csr_vector_kernel<8, kBlock>, kBlock, A->nrows, kBlock / 8, p->sm_count);
-    p->grid_csr[4] = grid_for((const void*)pepp::k::csr_vector_kernel<16, kBlock>, kBlock, A->nrows, kBlock / 16, p->sm_count);
-    p->grid_csr[5] = grid_for((const void*)pepp::k::csr_vector_kernel<32, kBlock>, kBlock, A->nrows, kBlock / 32, p->sm_count);
+    p->grid_csr[1] = grid_for((const void*)pepp::k::csr_vector_kernel<2, kBlock, double>, kBlock, A->nrows, kBlock / 2, p->sm_count);
+    p->grid_csr[2] = grid_for((const void*)pepp::k::csr_vector_kernel<4, kBlock, double>, kBlock, A->nrows, kBlock / 4, p->sm_count);
+    p->grid_csr[3] = grid_for((const void*)pepp::k::csr_vector_kernel<8, kBlock, double>, kBlock, A->nrows, kBlock / 8, p->sm_count);
+    p->grid_csr[4] = grid_for((const void*)pepp::k::csr_vector_kernel<16, kBlock, double>, kBlock, A->nrows, kBlock / 16, p->sm_count);
+    p->grid_csr[5] = grid_for((const void*)pepp::k::csr_vector_kernel<32, kBlock, double>, kBlock, A->nrows, kBlock / 32, p->sm_count);
     {   // SELL: exactly one resident wave; warps walk their chunks with prefetch
         int occ = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pepp::k::sell_kernel<kBlock, false>, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pepp::k::sell_kernel<kBlock, false, double>, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
         (void)cudaGetLastError();
         const int64_t need = ((int64_t)p->nchunks + kBlock / 32 - 1) / (kBlock / 32);
         const int64_t wave = (int64_t)p->sm_count * occ;
@@ -953,14 +1002,14 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_cho
     return select_choice(p, out);
 }
 
-extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const double* x, double* y, int flags,
+extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void* x, void* y, int flags,
                                                 void* stream, const pepp_choice_t* force, pepp_choice_t* used) {
     if (!p) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
     if ((!x && p->ncols > 0) || (!y && p->global_rows > 0)) return PEPP_E_INVALID;
     if (x && y) {   // x [0, ncols) and y [0, global_rows) must not overlap
-        const char *xb = (const char*)x, *xe = (const char*)(x + p->ncols);
-        const char *yb = (const char*)y, *ye = (const char*)(y + p->global_rows);
+        const char *xb = (const char*)x, *xe = xb + p->ncols * (int64_t)p->esz;
+        const char *yb = (const char*)y, *ye = yb + p->global_rows * (int64_t)p->esz;
         if (xb < ye && yb < xe) return PEPP_E_INVALID;
     }
     cudaStream_t st = (cudaStream_t)stream;
@@ -1000,7 +1049,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const doub
         rec = &p->ring[(p->ring_head + p->ring_count) % kTimingRing];
         if (cudaEventRecord(rec->start, st) != cudaSuccess) { (void)cudaGetLastError(); rec = nullptr; }
     }
-    pepp_status_t s = launch(p, p->cands[ch.candidate], x, y + p->row_offset, st);
+    pepp_status_t s = launch(p, p->cands[ch.candidate], x, (char*)y + p->row_offset * (int64_t)p->esz, st);
     if (s) { p->sticky = s; return s; }
     if (rec) {
         if (cudaEventRecord(rec->stop, st) == cudaSuccess) {
@@ -1032,7 +1081,7 @@ struct pepp_spmv_graph_s {
     int device = 0;
 };
 
-extern "C" PEPP_API pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, const double* x, double* y, double* work,
+extern "C" PEPP_API pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, const void* x, void* y, void* work,
                                                         int32_t iterations, int32_t mode, int flags, void* stream,
                                                         pepp_spmv_graph_t** out) {
     if (!out) return PEPP_E_INVALID;
@@ -1052,8 +1101,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, co
     if (!g) { cudaStreamDestroy(cap); return PEPP_E_NOMEM; }
     g->device = p->device;
     bool ok = cudaStreamBeginCapture(cap, cudaStreamCaptureModeRelaxed) == cudaSuccess;
-    const double* in = x;
-    double* outb = y;
+    const void* in = x;
+    void* outb = y;
     for (int32_t it = 0; ok && it < iterations; ++it) {
         s = pepp_spmv_exec(p, in, outb, flags | PEPP_EXEC_NO_TIMING, cap, &ch, nullptr);
         if (s) ok = false;
@@ -1104,6 +1153,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_graph_destroy(pepp_spmv_graph_t* g) 
 extern "C" PEPP_API pepp_status_t pepp_spmv_exec_vec(pepp_spmv_plan_t* p, pepp_vector_t* x, pepp_vector_t* y, int flags,
                                                     void* stream, const pepp_choice_t* force, pepp_choice_t* used) {
     if (!p || !x || !y || x == y) return PEPP_E_INVALID;
+    if (p->vt != PEPP_VALUE_F64) return PEPP_E_UNSUPPORTED;   // containers hold fp64
     if (pepp::vector_simulated(x) || pepp::vector_simulated(y)) return PEPP_E_INVALID;
     if (pepp::vector_length(x) != p->ncols || pepp::vector_length(y) != p->global_rows) return PEPP_E_INVALID;
     double *dx = nullptr, *dy = nullptr;
@@ -1120,7 +1170,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_vec(pepp_spmv_plan_t* p, pepp_v
     return s ? s : (s1 ? s1 : s2);
 }
 
-extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, double* y, int flags, void* stream) {
+extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* y, int flags, void* stream) {
     if (!p) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
     if (p->opts.nranks == 1 || !(flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED))) return PEPP_OK;
@@ -1133,7 +1183,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, double
     return s;
 }
 
-extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const double* x_host, double* y_host,
+extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const void* x_host, void* y_host,
                                                      int32_t iterations, int flags, void* stream) {
     if (!p || !x_host || !y_host || iterations < 1) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
@@ -1143,14 +1193,14 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const
     const int64_t nx = std::max<int64_t>(p->ncols, p->global_rows);
     if (!p->d_hx) {
         pepp_status_t s;
-        if ((s = dalloc(p, &p->d_hx, nx))) return s;
-        if ((s = dalloc(p, &p->d_hy, nx))) return s;
+        if ((s = dalloc_bytes(p, &p->d_hx, nx * (int64_t)p->esz))) return s;
+        if ((s = dalloc_bytes(p, &p->d_hy, nx * (int64_t)p->esz))) return s;
     }
-    if (cudaMemcpyAsync(p->d_hx, x_host, sizeof(double) * p->ncols, cudaMemcpyHostToDevice, st) != cudaSuccess) {
+    if (cudaMemcpyAsync(p->d_hx, x_host, p->esz * p->ncols, cudaMemcpyHostToDevice, st) != cudaSuccess) {
         (void)cudaGetLastError();
         return PEPP_E_CUDA;
     }
-    double *xin = p->d_hx, *yout = p->d_hy;
+    void *xin = p->d_hx, *yout = p->d_hy;
     for (int32_t it = 0; it < iterations; ++it) {
         const bool last = it == iterations - 1;
         const int f = last ? flags : (flags & PEPP_EXEC_NO_TIMING) | PEPP_Y_NEXT_INPUT;
@@ -1161,7 +1211,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const
     // rows written back: all global rows with PEPP_Y_REPLICATED, else this rank's rows
     int64_t lo = p->row_offset, cnt = p->nrows;
     if (p->opts.nranks > 1 && (flags & PEPP_Y_REPLICATED)) { lo = 0; cnt = p->global_rows; }
-    if (cnt > 0 && cudaMemcpyAsync(y_host + lo, yout + lo, sizeof(double) * cnt, cudaMemcpyDeviceToHost, st) != cudaSuccess) {
+    if (cnt > 0 && cudaMemcpyAsync((char*)y_host + lo * (int64_t)p->esz, (const char*)yout + lo * (int64_t)p->esz,
+                                   p->esz * cnt, cudaMemcpyDeviceToHost, st) != cudaSuccess) {
         (void)cudaGetLastError();
         return PEPP_E_CUDA;
     }

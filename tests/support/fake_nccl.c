@@ -76,7 +76,15 @@ static void barrier(Comm* c) {
     }
 }
 
-static size_t dsize(int dtype) { return dtype == 2 || dtype == 3 ? 4 : dtype == 4 || dtype == 5 || dtype == 8 ? 8 : 1; }
+/* ncclDataType_t: 0/1 int8/uint8, 2/3 int32/uint32, 4/5 int64/uint64, 6 half, 7 float, 8 double, 9 bf16 */
+static size_t dsize(int dtype) {
+    switch (dtype) {
+    case 2: case 3: case 7: return 4;
+    case 4: case 5: case 8: return 8;
+    case 6: case 9: return 2;
+    default: return 1;
+    }
+}
 
 EXPORT const char* ncclGetErrorString(int r) { return r ? "fake nccl error" : "no error"; }
 
@@ -164,10 +172,16 @@ static int flush(Comm* c) {
                 double dv = 0; int64_t iv = 0;
                 for (int r = 0; r < c->nranks; ++r) {
                     const unsigned char* src = arslot(c, r) + arc + k * dsize(o->dtype);
-                    if (o->dtype == 8) { double v; memcpy(&v, src, 8); dv = r == 0 ? v : (o->redop == 2 ? (v > dv ? v : dv) : dv + v); }
+                    if (o->dtype == 8 || o->dtype == 7) {
+                        double v;
+                        if (o->dtype == 8) memcpy(&v, src, 8); else { float f; memcpy(&f, src, 4); v = f; }
+                        dv = r == 0 ? v : (o->redop == 2 ? (v > dv ? v : dv) : dv + v);
+                    }
                     else { int64_t v = 0; memcpy(&v, src, dsize(o->dtype)); iv = r == 0 ? v : (o->redop == 2 ? (v > iv ? v : iv) : iv + v); }
                 }
-                if (o->dtype == 8) memcpy(tmp + k * 8, &dv, 8); else memcpy(tmp + k * dsize(o->dtype), &iv, dsize(o->dtype));
+                if (o->dtype == 8) memcpy(tmp + k * 8, &dv, 8);
+                else if (o->dtype == 7) { float f = (float)dv; memcpy(tmp + k * 4, &f, 4); }
+                else memcpy(tmp + k * dsize(o->dtype), &iv, dsize(o->dtype));
             }
             cudaMemcpy(o->rbuf, tmp, o->bytes, cudaMemcpyHostToDevice);
             arc += o->bytes;

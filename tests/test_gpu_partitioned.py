@@ -43,7 +43,7 @@ def _matrix(name):
     raise ValueError(name)
 
 
-def _worker(rank, world, lib, uid, name, exchange, K, outq):
+def _worker(rank, world, lib, uid, name, exchange, K, outq, f32=False):
     os.environ["PEPP_NCCL_LIB"] = lib
     try:
         import sys
@@ -57,8 +57,10 @@ def _worker(rank, world, lib, uid, name, exchange, K, outq):
         A = _matrix(name)
         n = A.nrows
         bounds = pepp.partition_rows(A.row_ptr, world)
+        if f32:   # fp32 instance: the same integer values, stored as float
+            A = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float32), A.r0, A.global_nrows)
         blk = gen.row_block(A, int(bounds[rank]), int(bounds[rank + 1]))
-        x0 = gen.vector(3, gen.INT8, n)
+        x0 = gen.vector(3, gen.INT8, n).astype(np.float32 if f32 else np.float64)
         res = {}
         with pepp.Plan.from_csr(blk, nranks=world, rank=rank, row_bounds=bounds, nccl_unique_id=uid,
                                 exchange=exchange) as plan:
@@ -76,11 +78,15 @@ def _worker(rank, world, lib, uid, name, exchange, K, outq):
                 src, dst = dst, (c if dst is b else b)
             plan.exec(src, dst, flags=pepp.Y_REPLICATED)   # iteration K+1, all rows on every rank
             torch.cuda.synchronize()
-            res["iter"] = bool(np.array_equal(dst.cpu().numpy(), oracle.iterate(A, x0, K + 1)))
+            ref = x0.astype(np.float64)
+            for _ in range(K + 1):   # integer values: the fp64 oracle is exact, and so is fp32 below 2^24
+                ref = oracle.spmv(gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float64)), ref)
+            res["iter"] = bool(np.array_equal(dst.cpu().numpy().astype(np.float64), ref))
             # host-buffer entry point, partitioned: iterations with the exchange inside
-            yh = np.full(n, np.nan)
+            yh = np.full(n, np.nan, dtype=x0.dtype)
             plan.exec_host(x0, yh, iterations=K, flags=pepp.Y_REPLICATED)
-            res["host"] = bool(np.array_equal(yh, oracle.iterate(A, x0, K)))
+            A64 = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float64))
+            res["host"] = bool(np.array_equal(yh.astype(np.float64), oracle.iterate(A64, x0.astype(np.float64), K)))
             res["exchange"] = info["exchange"]
             res["halo_recv"] = info["halo_recv"]
             res["halo_send"] = info["halo_send"]
@@ -90,13 +96,13 @@ def _worker(rank, world, lib, uid, name, exchange, K, outq):
         outq.put((rank, {"error": repr(e) + traceback.format_exc()}))
 
 
-def _run(name, exchange, K=6):
+def _run(name, exchange, K=6, f32=False):
     import torch.multiprocessing as mp
     lib = _build_fake()
     uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_{exchange}".encode() + b"\0" * 128)[:128]
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker, args=(r, 2, lib, uid, name, exchange, K, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, lib, uid, name, exchange, K, q, f32)) for r in range(2)]
     for p in procs:
         p.start()
     out = {}
@@ -123,3 +129,11 @@ def test_two_ranks_one_gpu_iterated_spmv_bitwise(name, exchange):
         assert ex == {exchange}
     if name == "lap" and exchange == pepp.X_HALO:
         assert out[0]["halo_recv"] == 96 and out[1]["halo_send"] == 96   # one grid row each way
+
+
+@pytest.mark.parametrize("name,exchange", [("lap", 2), ("zipf", 1)])
+def test_two_ranks_one_gpu_fp32(name, exchange):
+    """fp32 plans exchange fp32 payloads (ncclFloat32)."""
+    out = _run(name, exchange, K=3, f32=True)
+    for r in range(2):
+        assert out[r]["iter"] and out[r]["host"], (r, out[r])

@@ -29,7 +29,8 @@ class _M:
         self.nrows, self.ncols = nrows, ncols
         self.row_ptr = np.asarray(row_ptr, dtype=np.int64)
         self.col = np.asarray(col, dtype=np.int32)
-        self.val = np.asarray(val, dtype=np.float64)
+        f32 = isinstance(val, np.ndarray) and val.dtype == np.float32
+        self.val = val if f32 else np.asarray(val, dtype=np.float64)
 
 
 def _random_csr(rng: random.Random, m, n, first, int_vals=True, dup=True, unsorted=True, pempty=0.2):
@@ -269,3 +270,42 @@ def test_partition_rule_properties(P):
     bl = oracle.partition_nnz(L, 4)
     sizes = np.diff(L.row_ptr[bl])
     assert sizes.max() - sizes.min() <= 2 * 5   # each boundary within one row (<=5 nnz)
+
+
+# ------------------------------------------------- fp32 instance (f3) ----
+@pytest.mark.parametrize("seed", range(6))
+def test_f32_oracle_integer_exact_and_real_single_order_bound(seed):
+    """The fp32 oracle (paper's `float` signature): exact on small integers
+    (all partial sums < 2^24), and within one fp32 summation order of the
+    exact rational result on real inputs; it is NOT the fp64 result."""
+    rng = random.Random(200 + seed)
+    m, n = rng.randint(1, 50), rng.randint(1, 50)
+    A = _random_csr(rng, m, n, rng.choice([0, 5]))
+    A32 = _M(m, n, A.row_ptr, A.col, A.val.astype(np.float32))
+    x = np.array([float(rng.randint(-8, 8)) for _ in range(n)], dtype=np.float32)
+    y = oracle.spmv(A32, x)
+    assert y.dtype == np.float32
+    exact = _dense_exact(A, x.astype(np.float64))
+    assert all(Fraction(float(a)) == b for a, b in zip(y, exact))
+    # real values: float products and sums, error vs exact within gamma_n(fp32) * S
+    R = _random_csr(rng, m, n, 0, int_vals=False)
+    R32 = _M(m, n, R.row_ptr, R.col, R.val.astype(np.float32))
+    xr = np.array([rng.uniform(-1, 1) for _ in range(n)], dtype=np.float32)
+    yr = oracle.spmv(R32, xr)
+    ex = _dense_exact(_M(m, n, R.row_ptr, R.col, R32.val.astype(np.float64)), xr.astype(np.float64))
+    u = 2.0 ** -24
+    for i in range(m):
+        L = int(R.row_ptr[i + 1] - R.row_ptr[i])
+        S = sum(abs(float(R32.val[k])) * abs(float(xr[R.col[k]])) for k in range(int(R.row_ptr[i]), int(R.row_ptr[i + 1])))
+        g = (L * u / (1 - L * u)) if L else 0.0
+        assert abs(Fraction(float(yr[i])) - ex[i]) <= Fraction(g * S * (1 + 1e-9))
+
+
+def test_f32_oracle_rounds_like_float():
+    """A case where float and double sums differ: 1 + 2^-24 + 2^-24 is 1 in
+    float (each addition rounds) but 1 + 2^-23 in double."""
+    A = _M(1, 3, [0, 3], [0, 1, 2], np.array([1.0, 1.0, 1.0], dtype=np.float32))
+    x = np.array([1.0, 2.0 ** -24, 2.0 ** -24], dtype=np.float32)
+    assert oracle.spmv(A, x)[0] == np.float32(1.0)
+    A64 = _M(1, 3, [0, 3], [0, 1, 2], np.array([1.0, 1.0, 1.0]))
+    assert oracle.spmv(A64, x.astype(np.float64))[0] == 1.0 + 2.0 ** -23
