@@ -252,6 +252,13 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     del rp_global
     A = make_block(args.workload, r0, r1)
     x0 = x0_vector(args.workload, A.ncols)
+    f32 = args.dtype == "f32"
+    if f32:   # the fp32 instance (paper's `float` signature): same matrix, values rounded to float
+        import gen
+        A = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float32), A.r0, A.global_nrows, A.name)
+        x0 = x0.astype(np.float32)
+    tdt = torch.float32 if f32 else torch.float64
+    esz = 4 if f32 else 8
 
     uid = None
     if world > 1:
@@ -269,7 +276,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
 
     stream = torch.cuda.Stream(device=dev)
     xs = torch.from_numpy(x0).to(dev)
-    bufs = [torch.empty(R, dtype=torch.float64, device=dev) for _ in range(2)]
+    bufs = [torch.empty(R, dtype=tdt, device=dev) for _ in range(2)]
     flush = None if iterated or Z * 12 > 4 * (1 << 30) else torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     ev_pool = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(iters)]
@@ -339,7 +346,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     total_ms = float(t.item())
 
     nspmv = iters * args.steps
-    alg_bytes_global = Z * 12 + (R + 1) * 4 + A.ncols * 8 + R * 8
+    alg_bytes_global = Z * (4 + esz) + (R + 1) * 4 + A.ncols * esz + R * esz
     if iterated:
         secs = total_ms / 1e3
     else:
@@ -355,7 +362,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
 
     # roofline of the dominant kernel on this rank (rank 0 reports)
     avg_kernel_s = statistics.mean(kern_ms) / 1e3
-    local_bytes = A.nnz * 12 + (A.nrows + 1) * 4 + (A.nrows + info["halo_recv"]) * 8 + A.nrows * 8
+    local_bytes = A.nnz * (4 + esz) + (A.nrows + 1) * 4 + (A.nrows + info["halo_recv"]) * esz + A.nrows * esz
     if world == 1:
         local_bytes = alg_bytes_global
     achieved = local_bytes / avg_kernel_s / 1e9
@@ -410,7 +417,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
 
     # ---- e2e: host buffers through the C-ABI (pepp_spmv_exec_host) ----
     xh = torch.from_numpy(x0).pin_memory().numpy() if torch.cuda.is_available() else x0
-    yh = torch.empty(R, dtype=torch.float64).pin_memory().numpy()
+    yh = torch.empty(R, dtype=tdt).pin_memory().numpy()
     e2e_iters = iters if iterated else 1
     e2e_flags = flags
     plan.exec_host(xh, yh, iterations=e2e_iters, flags=e2e_flags, stream=stream)   # warm
@@ -427,7 +434,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     e2e_val = 2.0 * Z * e2e_iters * e2e_steps / te / 1e9
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu:
+    if rank == 0 and world == 1 and not args.no_cpu and not f32:
         cpu = cpu_baseline(A, x0, 2 if A.nnz > 10_000_000 else 200)
 
     if rank == 0:
@@ -436,7 +443,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             "metric": "SpMV GFLOP/s (aggregate over ranks); achieved HBM GB/s in 'hbm'",
             "value": round(gflops, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
             "config": {"workload": args.workload, "desc": wl["desc"], "spmv_per_step": iters,
                        "rows": R, "nnz": Z, "l2": "inputs larger than L2 (5.4 GB/SpMV)" if iterated
                        else "L2 flushed (512 MB memset) between SpMVs; kernel events only",
@@ -445,8 +452,8 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             "hbm": {"achieved_gbs": round(gbs, 1), "frac_of_measured": round(gbs / (world * peak), 4),
                     "frac_of_8tbs": round(gbs / (world * 8000.0), 4), "algorithmic_bytes_per_spmv": alg_bytes_global},
             "roofline": roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, args.workload),
-            "e2e": {"value": round(e2e_val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": A.ncols * 8,
-                    "d2h_bytes_per_step": A.nrows * 8, "spmv_per_step": e2e_iters,
+            "e2e": {"value": round(e2e_val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": A.ncols * esz,
+                    "d2h_bytes_per_step": A.nrows * esz, "spmv_per_step": e2e_iters,
                     "api": "pepp_spmv_exec_host (pinned host x0 -> iterations -> host y)"},
             "gpu_launches": launches["n"],
             "graph": graph_info,
@@ -473,6 +480,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-prune", action="store_true", help="every variant is a candidate (no static narrowing)")
+    ap.add_argument("--dtype", choices=["f64", "f32"], default="f64",
+                    help="f64 = BASELINE's precision (default); f32 = the paper's float instance")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
 
