@@ -181,6 +181,7 @@ typedef struct {
     int64_t halo_send;        /* entries sent per exchange (halo) */
     double sell_col16_frac;   /* fraction of SELL chunks storing 16-bit column deltas */
     uint64_t prior_key;       /* context key the cold-start prior came from (0 = none) */
+    double sell_stencil_frac; /* fraction of SELL chunks stored as stencil (one offset per slot per chunk) */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

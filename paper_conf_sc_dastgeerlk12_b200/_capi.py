@@ -54,7 +54,7 @@ class INFO_T(ctypes.Structure):
                 ("row_offset", c_i64), ("key", c_u64), ("ncandidates", c_i32), ("sell_sigma", c_i32),
                 ("sell_fill", c_f64), ("device_bytes", c_i64), ("algorithmic_bytes", c_i64),
                 ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64),
-                ("prior_key", c_u64)]
+                ("prior_key", c_u64), ("sell_stencil_frac", c_f64)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}

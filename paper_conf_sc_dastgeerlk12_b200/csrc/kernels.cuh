@@ -196,28 +196,35 @@ __global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int*
 // chunk's metadata is prefetched (tools/experiments/sell_probe.cu: 830 ->
 // 771 us on config 4). The grid is one resident wave (SMs x occupancy).
 // =====================================================================
-// Chunk descriptor bits in chunk_len[c]: low 29 bits = slots in the chunk;
+// Chunk descriptor bits in chunk_len[c]: low 28 bits = slots in the chunk;
 // bit 30 = masked (rows of the chunk have different lengths: read rowlen);
 // bit 29 = 16-bit columns (col16 holds col - row, row = the original index of
-// the lane's row; every delta of the chunk fits in int16).
+// the lane's row; every delta of the chunk fits in int16);
+// bit 28 = stencil chunk (every lane has the same column offsets relative to
+// its row: soff[chunk_ptr[c]/32 + j] holds the offset of slot j once for the
+// whole chunk — a per-chunk diagonal (DIA) layout; no column stream at all).
 constexpr int kSellMasked = 1 << 30;
 constexpr int kSellCol16 = 1 << 29;
-constexpr int kSellLenMask = (1 << 29) - 1;
+constexpr int kSellStencil = 1 << 28;
+constexpr int kSellLenMask = (1 << 28) - 1;
+enum { kIdx32 = 0, kIdx16 = 1, kIdxStencil = 2 };
 
 // N slots of one chunk, loads issued unconditionally (all N exist for every
 // lane) before the first FMA; the per-lane row length only masks the FMA.
-// C16: columns stored as int16 deltas from the lane's row index `row0`.
-template <int N, bool C16, typename T>
+// IDX: kIdx32 columns; kIdx16 int16 deltas from the lane's row index `row0`;
+// kIdxStencil one offset per slot for the whole chunk (soff + sbase).
+template <int N, int IDX, typename T>
 __device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __restrict__ col,
-                                        const int16_t* __restrict__ col16, int row0,
-                                        const T* __restrict__ x, int64_t base, int j0, int len,
-                                        T acc, uint64_t pol) {
+                                        const int16_t* __restrict__ col16, const int* __restrict__ soff,
+                                        int64_t sbase, int row0, const T* __restrict__ x, int64_t base, int j0,
+                                        int len, T acc, uint64_t pol) {
     T v[N];
     int c[N];
 #pragma unroll
     for (int u = 0; u < N; ++u)
-        c[u] = C16 ? row0 + ld_stream_i16(col16 + base + (int64_t)(j0 + u) * 32, pol)
-                   : ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
+        c[u] = IDX == kIdxStencil ? row0 + __ldg(soff + sbase + j0 + u)
+             : IDX == kIdx16      ? row0 + ld_stream_i16(col16 + base + (int64_t)(j0 + u) * 32, pol)
+                                  : ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
 #pragma unroll
     for (int u = 0; u < N; ++u) v[u] = ld_stream_v(val + base + (int64_t)(j0 + u) * 32, pol);
     T xv[N];
@@ -229,22 +236,23 @@ __device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __
     return acc;
 }
 
-template <bool C16, typename T>
+template <int IDX, typename T>
 __device__ __forceinline__ T sell_chunk(const T* __restrict__ val, const int* __restrict__ col,
-                                        const int16_t* __restrict__ col16, int row0, const T* __restrict__ x,
+                                        const int16_t* __restrict__ col16, const int* __restrict__ soff,
+                                        int64_t sbase, int row0, const T* __restrict__ x,
                                         int64_t base, int clen, int len, uint64_t pol) {
     T acc = T(0);
     int j = 0;
     // whole blocks of 8 slots, then one exactly-sized tail (warp-uniform switch)
-    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol);
+    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol);
     switch (clen - j) {
-    case 1: acc = sell_slots<1, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 2: acc = sell_slots<2, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 3: acc = sell_slots<3, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 4: acc = sell_slots<4, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 5: acc = sell_slots<5, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 6: acc = sell_slots<6, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
-    case 7: acc = sell_slots<7, C16, T>(val, col, col16, row0, x, base, j, len, acc, pol); break;
+    case 1: acc = sell_slots<1, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
+    case 2: acc = sell_slots<2, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
+    case 3: acc = sell_slots<3, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
+    case 4: acc = sell_slots<4, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
+    case 5: acc = sell_slots<5, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
+    case 6: acc = sell_slots<6, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
+    case 7: acc = sell_slots<7, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
     default: break;
     }
     return acc;
@@ -257,6 +265,7 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
                                                      const int* __restrict__ perm,
                                                      const int* __restrict__ col,
                                                      const int16_t* __restrict__ col16,
+                                                     const int* __restrict__ soff,
                                                      const T* __restrict__ val,
                                                      const T* __restrict__ x,
                                                      T* __restrict__ y,
@@ -297,8 +306,11 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
         if (in < nchunks) meta(cn, dn, cpn, lenn, orown);
         const int64_t base = cp + lane;
         const int clen = d & kSellLenMask;
-        const T acc = (d & kSellCol16) ? sell_chunk<true, T>(val, col, col16, orow, x, base, clen, len, pol)
-                                       : sell_chunk<false, T>(val, col, col16, orow, x, base, clen, len, pol);
+        const int64_t sbase = cp >> 5;   // this chunk's slot offsets in soff (stencil chunks)
+        T acc;
+        if (d & kSellStencil) acc = sell_chunk<kIdxStencil, T>(val, col, col16, soff, sbase, orow, x, base, clen, len, pol);
+        else if (d & kSellCol16) acc = sell_chunk<kIdx16, T>(val, col, col16, soff, sbase, orow, x, base, clen, len, pol);
+        else acc = sell_chunk<kIdx32, T>(val, col, col16, soff, sbase, orow, x, base, clen, len, pol);
         if (c * 32 + lane < nrows) y[orow] = acc;
         c = cn; d = dn; cp = cpn; len = lenn; orow = orown;
     }
@@ -891,6 +903,7 @@ __global__ void sell_col16_kernel(int nrows, int nchunks, const int64_t* __restr
     const int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (c >= nchunks) return;
     const int d = chunk_len[c];
+    if (d & kSellStencil) return;       // already needs no column stream
     const int clen = d & kSellLenMask;
     const int r = c * 32 + lane;
     const int len = r < nrows ? rowlen[r] : 0;
@@ -908,6 +921,36 @@ __global__ void sell_col16_kernel(int nrows, int nchunks, const int64_t* __restr
     if (lane == 0) {
         chunk_len[c] = d | kSellCol16;
         atomicAdd(n16, 1ull);
+    }
+}
+
+// Stencil chunks: one warp per chunk; a uniform chunk (all 32 rows present,
+// all of length clen) whose slot-j column offsets (col - row) are equal in
+// every lane stores those clen offsets once: soff[chunk_ptr[c]/32 + j].
+__global__ void sell_stencil_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
+                                    int* __restrict__ chunk_len, const int* __restrict__ perm,
+                                    const int* __restrict__ col, int* __restrict__ soff,
+                                    unsigned long long* __restrict__ nst) {
+    const int lane = threadIdx.x & 31;
+    const int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (c >= nchunks) return;
+    const int d = chunk_len[c];
+    if (d & kSellMasked) return;        // rows of different lengths (or a partial chunk)
+    const int clen = d & kSellLenMask;
+    const int r = c * 32 + lane;
+    const int orow = perm ? perm[r] : r;
+    const int64_t base = chunk_ptr[c] + lane;
+    bool same = true;
+    for (int j = 0; j < clen; ++j) {
+        const int dl = col[base + (int64_t)j * 32] - orow;
+        same &= dl == __shfl_sync(0xffffffffu, dl, 0);
+    }
+    if (!__all_sync(0xffffffffu, same)) return;
+    const int64_t sb = chunk_ptr[c] >> 5;
+    for (int j = lane; j < clen; j += 32) soff[sb + j] = col[chunk_ptr[c] + (int64_t)j * 32] - (perm ? perm[c * 32] : c * 32);
+    if (lane == 0) {
+        chunk_len[c] = d | kSellStencil;
+        atomicAdd(nst, 1ull);
     }
 }
 

@@ -93,6 +93,8 @@ struct pepp_spmv_plan_s {
     int* d_perm = nullptr;
     int* d_scol = nullptr;
     int16_t* d_scol16 = nullptr;
+    int* d_soff = nullptr;           // stencil-chunk slot offsets
+    int64_t sell_stencil_chunks = 0;
     int sell_cpw = 1;            // chunks per σ window (chunk order is transposed when > 1)
     int64_t sell_col16_chunks = 0;
     void* d_sval = nullptr;
@@ -195,7 +197,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (!p) return;
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
-                    p->d_scol, p->d_scol16, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
+                    p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
                     p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
@@ -284,6 +286,21 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
         pepp::k::sell_fill_kernel<double><<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, p->d_col, (const double*)p->d_val,
                                                              p->d_chunk_ptr, p->d_scol, (double*)p->d_sval);
     PEPP_CUDA_TRY(cudaGetLastError());
+    // stencil chunks: one offset per slot for the whole chunk (no column stream)
+    {
+        if ((s = dalloc(p, &p->d_soff, p->sell_slots / 32 + 8))) return s;
+        DevTmp<unsigned long long> d_nst;
+        PEPP_CUDA_TRY(d_nst.alloc(1));
+        PEPP_CUDA_TRY(cudaMemsetAsync(d_nst.p, 0, sizeof(unsigned long long), st));
+        const int wb = 256, wg = (int)(((int64_t)p->nchunks * 32 + wb - 1) / wb);
+        pepp::k::sell_stencil_kernel<<<wg, wb, 0, st>>>(n, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_perm,
+                                                         p->d_scol, p->d_soff, d_nst.p);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        unsigned long long nst = 0;
+        PEPP_CUDA_TRY(cudaMemcpyAsync(&nst, d_nst.p, sizeof(nst), cudaMemcpyDeviceToHost, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        p->sell_stencil_chunks = (int64_t)nst;
+    }
     // 16-bit column deltas where a whole chunk allows them (banded / stencil
     // structure): 2 instead of 4 bytes of index per stored slot
     {
@@ -306,6 +323,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->sell_cpw = sigma > 1 ? std::max(1, sigma / 32) : 1;
     p->info.sell_sigma = sigma;
     p->info.sell_col16_frac = p->nchunks ? (double)p->sell_col16_chunks / (double)p->nchunks : 0.0;
+    p->info.sell_stencil_frac = p->nchunks ? (double)p->sell_stencil_chunks / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
     return PEPP_OK;
 }
@@ -479,11 +497,11 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
         if (p->d_perm)
             pepp::k::sell_kernel<kBlock, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
-                p->d_scol16, (const T*)p->d_sval, x, y, p->sell_cpw);
+                p->d_scol16, p->d_soff, (const T*)p->d_sval, x, y, p->sell_cpw);
         else
             pepp::k::sell_kernel<kBlock, false, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr, p->d_scol,
-                p->d_scol16, (const T*)p->d_sval, x, y, 1);
+                p->d_scol16, p->d_soff, (const T*)p->d_sval, x, y, 1);
         break;
     default:
         return PEPP_E_INVALID;
