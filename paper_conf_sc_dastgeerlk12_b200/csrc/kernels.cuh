@@ -212,17 +212,17 @@ enum { kIdx32 = 0, kIdx16 = 1, kIdxStencil = 2 };
 // N slots of one chunk, loads issued unconditionally (all N exist for every
 // lane) before the first FMA; the per-lane row length only masks the FMA.
 // IDX: kIdx32 columns; kIdx16 int16 deltas from the lane's row index `row0`;
-// kIdxStencil one offset per slot for the whole chunk (soff + sbase).
+// kIdxStencil one offset per slot for the whole chunk (lane j's `offl`).
 template <int N, int IDX, typename T>
 __device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __restrict__ col,
-                                        const int16_t* __restrict__ col16, const int* __restrict__ soff,
-                                        int64_t sbase, int row0, const T* __restrict__ x, int64_t base, int j0,
+                                        const int16_t* __restrict__ col16, int offl,
+                                        int row0, const T* __restrict__ x, int64_t base, int j0,
                                         int len, T acc, uint64_t pol) {
     T v[N];
     int c[N];
 #pragma unroll
     for (int u = 0; u < N; ++u)
-        c[u] = IDX == kIdxStencil ? row0 + __ldg(soff + sbase + j0 + u)
+        c[u] = IDX == kIdxStencil ? row0 + __shfl_sync(0xffffffffu, offl, j0 + u)   // lane j holds slot j's offset
              : IDX == kIdx16      ? row0 + ld_stream_i16(col16 + base + (int64_t)(j0 + u) * 32, pol)
                                   : ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
 #pragma unroll
@@ -238,21 +238,20 @@ __device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __
 
 template <int IDX, typename T>
 __device__ __forceinline__ T sell_chunk(const T* __restrict__ val, const int* __restrict__ col,
-                                        const int16_t* __restrict__ col16, const int* __restrict__ soff,
-                                        int64_t sbase, int row0, const T* __restrict__ x,
-                                        int64_t base, int clen, int len, uint64_t pol) {
+                                        const int16_t* __restrict__ col16, int offl, int row0,
+                                        const T* __restrict__ x, int64_t base, int clen, int len, uint64_t pol) {
     T acc = T(0);
     int j = 0;
     // whole blocks of 8 slots, then one exactly-sized tail (warp-uniform switch)
-    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol);
+    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol);
     switch (clen - j) {
-    case 1: acc = sell_slots<1, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
-    case 2: acc = sell_slots<2, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
-    case 3: acc = sell_slots<3, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
-    case 4: acc = sell_slots<4, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
-    case 5: acc = sell_slots<5, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
-    case 6: acc = sell_slots<6, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
-    case 7: acc = sell_slots<7, IDX, T>(val, col, col16, soff, sbase, row0, x, base, j, len, acc, pol); break;
+    case 1: acc = sell_slots<1, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 2: acc = sell_slots<2, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 3: acc = sell_slots<3, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 4: acc = sell_slots<4, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 5: acc = sell_slots<5, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 6: acc = sell_slots<6, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 7: acc = sell_slots<7, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
     default: break;
     }
     return acc;
@@ -286,33 +285,43 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
         if (!SORTED) return i;
         return i < nfull ? (i % nwin) * cpw + i / nwin : i;
     };
-    auto meta = [&](int c, int& d, int64_t& cp, int& len, int& orow) {
-        d = __ldg(chunk_len + c);
-        cp = __ldg(chunk_ptr + c);
+    // Two-deep software pipelining over the warp's chunks (latency-bound
+    // kernel): while chunk i computes, chunk i+1's dependent per-lane loads
+    // (row length if masked, original row if sorted, the stencil offsets —
+    // lane j loads slot j's offset once, broadcast later with shuffles) and
+    // chunk i+2's descriptor (length/flags, slot pointer) are in flight.
+    struct Desc { int d; int64_t cp; };
+    struct Lane { int len; int orow; int offl; };
+    auto desc = [&](int i) -> Desc {
+        Desc q{0, 0};
+        if (i < nchunks) { const int c = chunk_of(i); q.d = __ldg(chunk_len + c); q.cp = __ldg(chunk_ptr + c); }
+        return q;
+    };
+    auto lanes = [&](int i, const Desc& q) -> Lane {
+        Lane l{0, 0, 0};
+        if (i >= nchunks) return l;
+        const int c = chunk_of(i);
         const int r = c * 32 + lane;
-        len = !(d & kSellMasked) ? (d & kSellLenMask) : (r < nrows ? __ldg(rowlen + r) : 0);
-        orow = (SORTED && r < nrows) ? __ldg(perm + r) : r;
+        l.len = !(q.d & kSellMasked) ? (q.d & kSellLenMask) : (r < nrows ? __ldg(rowlen + r) : 0);
+        l.orow = (SORTED && r < nrows) ? __ldg(perm + r) : r;
+        if ((q.d & kSellStencil) && lane < (q.d & kSellLenMask)) l.offl = __ldg(soff + (q.cp >> 5) + lane);
+        return l;
     };
     int i = warp;
-    int c = i < nchunks ? chunk_of(i) : 0;
-    int d = 0, len = 0, orow = 0;
-    int64_t cp = 0;
-    if (i < nchunks) meta(c, d, cp, len, orow);
+    Desc q0 = desc(i), q1 = desc(i + nwarps);
+    Lane l0 = lanes(i, q0);
     for (; i < nchunks; i += nwarps) {
-        const int in = i + nwarps;
-        const int cn = in < nchunks ? chunk_of(in) : 0;
-        int dn = 0, lenn = 0, orown = 0;
-        int64_t cpn = 0;
-        if (in < nchunks) meta(cn, dn, cpn, lenn, orown);
-        const int64_t base = cp + lane;
-        const int clen = d & kSellLenMask;
-        const int64_t sbase = cp >> 5;   // this chunk's slot offsets in soff (stencil chunks)
+        const Desc q2 = desc(i + 2 * nwarps);
+        const Lane l1 = lanes(i + nwarps, q1);
+        const int c = chunk_of(i);
+        const int64_t base = q0.cp + lane;
+        const int clen = q0.d & kSellLenMask;
         T acc;
-        if (d & kSellStencil) acc = sell_chunk<kIdxStencil, T>(val, col, col16, soff, sbase, orow, x, base, clen, len, pol);
-        else if (d & kSellCol16) acc = sell_chunk<kIdx16, T>(val, col, col16, soff, sbase, orow, x, base, clen, len, pol);
-        else acc = sell_chunk<kIdx32, T>(val, col, col16, soff, sbase, orow, x, base, clen, len, pol);
-        if (c * 32 + lane < nrows) y[orow] = acc;
-        c = cn; d = dn; cp = cpn; len = lenn; orow = orown;
+        if (q0.d & kSellStencil) acc = sell_chunk<kIdxStencil, T>(val, col, col16, l0.offl, l0.orow, x, base, clen, l0.len, pol);
+        else if (q0.d & kSellCol16) acc = sell_chunk<kIdx16, T>(val, col, col16, 0, l0.orow, x, base, clen, l0.len, pol);
+        else acc = sell_chunk<kIdx32, T>(val, col, col16, 0, l0.orow, x, base, clen, l0.len, pol);
+        if (c * 32 + lane < nrows) y[l0.orow] = acc;
+        q0 = q1; q1 = q2; l0 = l1;
     }
 }
 
@@ -937,6 +946,7 @@ __global__ void sell_stencil_kernel(int nrows, int nchunks, const int64_t* __res
     const int d = chunk_len[c];
     if (d & kSellMasked) return;        // rows of different lengths (or a partial chunk)
     const int clen = d & kSellLenMask;
+    if (clen > 32) return;              // the kernel keeps slot offsets one per lane
     const int r = c * 32 + lane;
     const int orow = perm ? perm[r] : r;
     const int64_t base = chunk_ptr[c] + lane;
