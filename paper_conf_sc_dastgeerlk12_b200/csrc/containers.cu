@@ -49,6 +49,17 @@ struct pepp_vector_s {
 
 namespace {
 
+// works on the vector's device, restores the caller's current device
+struct DevScope {
+    int prev = -1;
+    explicit DevScope(const pepp_vector_t* v);
+    ~DevScope() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+        (void)cudaGetLastError();
+    }
+};
+
 inline bool reads(int32_t m) { return (m & PEPP_ACCESS_READ) != 0; }
 inline bool writes(int32_t m) { return (m & PEPP_ACCESS_WRITE) != 0; }
 inline bool valid_mode(int32_t m) { return m == PEPP_ACCESS_READ || m == PEPP_ACCESS_WRITE || m == PEPP_ACCESS_READWRITE; }
@@ -79,6 +90,12 @@ __global__ void scale_kernel(int64_t n, double alpha, double* __restrict__ v) {
         v[i] = alpha * v[i];
 }
 
+DevScope::DevScope(const pepp_vector_t* v) {
+    if (v->simulated) return;
+    if (cudaGetDevice(&prev) != cudaSuccess) { (void)cudaGetLastError(); prev = -1; }
+    if (prev != v->device) cudaSetDevice(v->device);
+}
+
 }  // namespace
 
 extern "C" PEPP_API pepp_status_t pepp_vector_create(int64_t n, double* host, int32_t device, pepp_vector_t** out) {
@@ -99,7 +116,7 @@ extern "C" PEPP_API pepp_status_t pepp_vector_create(int64_t n, double* host, in
             delete v;
             return PEPP_E_CUDA;
         }
-        cudaSetDevice(v->device);
+        DevScope scope(v);
         bool ok = cudaEventCreateWithFlags(&v->last_use, cudaEventDisableTiming) == cudaSuccess &&
                   cudaEventCreateWithFlags(&v->writer, cudaEventDisableTiming) == cudaSuccess;
         for (int i = 0; ok && i < pepp_vector_t::kMaxReaders; ++i)
@@ -128,8 +145,8 @@ extern "C" PEPP_API pepp_status_t pepp_vector_create(int64_t n, double* host, in
 
 extern "C" PEPP_API pepp_status_t pepp_vector_destroy(pepp_vector_t* v) {
     if (!v) return PEPP_OK;
+    DevScope scope(v);
     if (!v->simulated) {
-        cudaSetDevice(v->device);
         (void)wait_device(v);
         if (v->dev) cudaFree(v->dev);
         if (v->last_use) cudaEventDestroy(v->last_use);
@@ -146,7 +163,7 @@ extern "C" PEPP_API pepp_status_t pepp_vector_destroy(pepp_vector_t* v) {
 
 extern "C" PEPP_API pepp_status_t pepp_vector_acquire_host(pepp_vector_t* v, int32_t mode, double** host) {
     if (!v || !valid_mode(mode)) return PEPP_E_INVALID;
-    if (!v->simulated) cudaSetDevice(v->device);
+    DevScope scope(v);
     // element-wise access through the [] proxies: any host access needs the
     // latest data, and a host write must not race device work that reads it
     pepp_status_t s = wait_device(v);
@@ -168,8 +185,8 @@ extern "C" PEPP_API pepp_status_t pepp_vector_acquire_host(pepp_vector_t* v, int
 
 extern "C" PEPP_API pepp_status_t pepp_vector_acquire_device(pepp_vector_t* v, int32_t mode, void* stream, double** dev) {
     if (!v || !valid_mode(mode)) return PEPP_E_INVALID;
+    DevScope scope(v);
     if (!v->simulated) {
-        if (cudaSetDevice(v->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
         if (!v->dev) {
             if (cudaMalloc((void**)&v->dev, sizeof(double) * (v->n > 0 ? v->n : 1)) != cudaSuccess) {
                 (void)cudaGetLastError();

@@ -160,6 +160,23 @@ namespace {
         if (_e != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; } \
     } while (0)
 
+// Every entry point works on the plan's device and leaves the caller's
+// current device as it found it.
+struct DeviceScope {
+    int prev = -1;
+    bool ok = false;
+    explicit DeviceScope(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) { (void)cudaGetLastError(); prev = -1; }
+        ok = prev == dev || cudaSetDevice(dev) == cudaSuccess;
+        if (!ok) (void)cudaGetLastError();
+    }
+    ~DeviceScope() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+        (void)cudaGetLastError();
+    }
+};
+
 // device buffer of `bytes` bytes owned by the plan (value-typed arrays)
 pepp_status_t dalloc_bytes(pepp_spmv_plan_t* p, void** ptr, int64_t bytes) {
     *ptr = nullptr;
@@ -1001,6 +1018,9 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_plan(const pepp_csr_t* A, const pepp
     pepp_spmv_plan_t* p = new (std::nothrow) pepp_spmv_plan_t();
     if (!p) return PEPP_E_NOMEM;
     p->device = -1;
+    int caller_dev = -1;
+    if (cudaGetDevice(&caller_dev) != cudaSuccess) { (void)cudaGetLastError(); caller_dev = -1; }
+    struct Restore { int d; ~Restore() { if (d >= 0) cudaSetDevice(d); (void)cudaGetLastError(); } } restore{caller_dev};
     pepp_status_t s;
     try {
         s = plan_impl(A, opts, p);
@@ -1031,11 +1051,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         if (xb < ye && yb < xe) return PEPP_E_INVALID;
     }
     cudaStream_t st = (cudaStream_t)stream;
-    int cur = -1;
-    if (cudaGetDevice(&cur) != cudaSuccess || cur != p->device) {
-        (void)cudaGetLastError();
-        if (cudaSetDevice(p->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
-    }
+    DeviceScope dscope(p->device);
+    if (!dscope.ok) return PEPP_E_CUDA;
     pepp_choice_t ch{};
     if (force) {
         int idx = -1;
@@ -1107,7 +1124,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, co
     if (!p || iterations < 1 || (mode != 0 && mode != 1) || (mode == 1 && iterations > 1 && !work)) return PEPP_E_INVALID;
     if (mode == 1 && p->ncols != p->global_rows) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
-    if (cudaSetDevice(p->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    DeviceScope dscope(p->device);
+    if (!dscope.ok) return PEPP_E_CUDA;
     // choose once, outside the capture (calibration calls would not be timed)
     pepp_choice_t ch{};
     pepp_status_t s = select_choice(p, &ch);
@@ -1152,7 +1170,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, co
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_graph_launch(pepp_spmv_graph_t* g, void* stream) {
     if (!g) return PEPP_E_INVALID;
-    if (cudaSetDevice(g->device) != cudaSuccess || cudaGraphLaunch(g->exec, (cudaStream_t)stream) != cudaSuccess) {
+    DeviceScope dscope(g->device);
+    if (!dscope.ok || cudaGraphLaunch(g->exec, (cudaStream_t)stream) != cudaSuccess) {
         (void)cudaGetLastError();
         return PEPP_E_CUDA;
     }
@@ -1161,7 +1180,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_graph_launch(pepp_spmv_graph_t* g, v
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_graph_destroy(pepp_spmv_graph_t* g) {
     if (!g) return PEPP_OK;
-    cudaSetDevice(g->device);
+    DeviceScope dscope(g->device);
     if (g->exec) cudaGraphExecDestroy(g->exec);
     if (g->graph) cudaGraphDestroy(g->graph);
     delete g;
@@ -1193,7 +1212,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* 
     if (p->sticky) return p->sticky;
     if (p->opts.nranks == 1 || !(flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED))) return PEPP_OK;
     if (!y) return PEPP_E_INVALID;
-    if (cudaSetDevice(p->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    DeviceScope dscope(p->device);
+    if (!dscope.ok) return PEPP_E_CUDA;
     cudaStream_t st = (cudaStream_t)stream;
     const bool ag = (flags & PEPP_Y_REPLICATED) || p->exchange == PEPP_X_ALLGATHER;
     pepp_status_t s = ag ? exchange_allgather(p, y, st) : exchange_halo(p, y, st);
@@ -1207,7 +1227,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const
     if (p->sticky) return p->sticky;
     if (iterations > 1 && p->ncols != p->global_rows) return PEPP_E_INVALID;
     cudaStream_t st = (cudaStream_t)stream;
-    if (cudaSetDevice(p->device) != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    DeviceScope dscope(p->device);
+    if (!dscope.ok) return PEPP_E_CUDA;
     const int64_t nx = std::max<int64_t>(p->ncols, p->global_rows);
     if (!p->d_hx) {
         pepp_status_t s;
@@ -1240,7 +1261,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_destroy(pepp_spmv_plan_t* p) {
     if (!p) return PEPP_OK;
-    cudaSetDevice(p->device);
+    DeviceScope dscope(p->device);
     harvest(p, true);
     cudaDeviceSynchronize();
     (void)cudaGetLastError();
@@ -1270,7 +1291,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_candidates(const pepp_spmv_plan_t* p
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_flush_history(pepp_spmv_plan_t* p) {
     if (!p) return PEPP_E_INVALID;
-    cudaSetDevice(p->device);
+    DeviceScope dscope(p->device);
     harvest(p, true);
     return PEPP_OK;
 }

@@ -132,3 +132,16 @@ def test_invalid_arguments_rejected_on_host():
     rp = np.array([0, 2, 1], dtype=np.int64)
     b = np.zeros(3, dtype=np.int64)
     assert L.pepp_partition_rows(rp.ctypes.data, 2, 5, 2, b.ctypes.data) == C.PEPP_E_INVALID  # row_ptr[0] != first
+
+
+def test_oversized_block_refused_before_touching_memory():
+    """nnz >= 2^31 in one block is refused (PEPP_E_UNSUPPORTED, reading A3)
+    by the argument checks, before any pointer is dereferenced."""
+    from paper_conf_sc_dastgeerlk12_b200 import _capi as C
+    L = C.lib()
+    dummy = np.zeros(4, dtype=np.int64)
+    A = C.CSR_T(10, 10, 1 << 31, 0, dummy.ctypes.data, dummy.ctypes.data, dummy.ctypes.data, 0, 0)
+    h = ctypes.c_void_p()
+    assert L.pepp_spmv_plan(ctypes.byref(A), None, ctypes.byref(h)) == C.PEPP_E_UNSUPPORTED
+    A.nnz, A.value_type = 4, 7                      # unknown value type
+    assert L.pepp_spmv_plan(ctypes.byref(A), None, ctypes.byref(h)) == C.PEPP_E_INVALID

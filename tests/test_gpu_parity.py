@@ -434,3 +434,24 @@ def test_cold_start_from_persisted_history(tmp_path):
         while plan.exec(xb, yb).calibrating:
             calls_b += 1
         assert calls_b < calls_a          # the prior ruled some candidates out
+
+
+def test_entry_points_restore_the_callers_device():
+    """Every entry point works on the plan's device and leaves the caller's
+    current device unchanged (checked on device 0 with device 0 plans; on a
+    multi-GPU box a plan on device 1 is used from device 0)."""
+    A = gen.laplacian2d(32)
+    ndev = torch.cuda.device_count()
+    dev = 1 if ndev > 1 else 0
+    torch.cuda.set_device(0)
+    with pepp.Plan.from_csr(A, device=dev) as plan:
+        assert torch.cuda.current_device() == 0
+        x = torch.ones(A.ncols, dtype=torch.float64, device=f"cuda:{dev}")
+        y = torch.empty(A.nrows, dtype=torch.float64, device=f"cuda:{dev}")
+        with torch.cuda.device(dev):
+            s = torch.cuda.current_stream()
+        plan.exec(x, y, stream=s)
+        assert torch.cuda.current_device() == 0
+        plan.exec_host(np.ones(A.ncols), np.empty(A.nrows))
+        assert torch.cuda.current_device() == 0
+    assert torch.cuda.current_device() == 0
