@@ -3,8 +3,9 @@
 // Steps of the hot path:
 //   a1 context extraction     -> rowptr_check_narrow_kernel (+ host CV)     [plan]
 //   a2 partition              -> caller / pepp_partition_rows; ghosts here  [plan]
-//   a3 variant preparation    -> SELL conversion, merge tile search          [plan]
-//   a4 selection              -> pepp::history_pick over the candidates      [each call, host]
+//   a3 variant preparation    -> SELL conversion (+ stencil / 16-bit index compression),
+//                                merge tile search, CSR-stream item table     [plan]
+//   a4 selection              -> select_choice: calibration rounds / argmin  [each call, host]
 //   a5 SpMV kernel            -> kernels.cuh                                 [each call, device]
 //   a6 exchange               -> NCCL allgatherv (grouped broadcasts) / halo [each call, P > 1]
 //   a7 history update         -> lazily harvested CUDA events -> Welford     [each call, host]
@@ -812,7 +813,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         p->global_rows = A->nrows;
     }
     if (o->history_path) p->history_path = o->history_path;
-    p->opts.history_path = nullptr;
+    p->opts.history_path = nullptr;   // borrowed pointers are not kept past this call
     p->opts.row_bounds = nullptr;
 
     // ---- device ----
@@ -983,6 +984,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
             if (p->nccl->CommInitRank(&p->comm, o->nranks, id, o->rank)) return PEPP_E_NCCL;
             p->own_comm = true;
         }
+        p->opts.nccl_unique_id = nullptr;
         if ((s = setup_halo(p, ghosts, st))) return s;
         int ex = o->exchange;
         if (ex == PEPP_X_AUTO) {
