@@ -44,6 +44,8 @@ WORKLOADS = {
                    iters=20, iterated=False),
     "lap64": dict(desc="BASELINE config 1: 2D 5-point Laplacian 64x64 (4096 rows, 20224 nnz), fp64",
                   iters=1000, iterated=False),
+    "lap2048": dict(desc="test-sized Laplacian 2048x2048 (4.2M rows), iterated like config 4 (not a BASELINE config)",
+                    iters=100, iterated=True),
     "skew": dict(desc="heavy-tailed rows (not a BASELINE config): P(k)~k^-2, k<=4M, 4M x 4M, fp64 — rows up to ~1e6 nnz",
                  iters=20, iterated=False),
 }
@@ -56,6 +58,8 @@ def make_block(workload: str, r0: int, r1: int):
         return gen.laplacian2d(8192, r0, r1)
     if workload == "lap64":
         return gen.laplacian2d(64, r0, r1)
+    if workload == "lap2048":
+        return gen.laplacian2d(2048, r0, r1)
     if workload == "uniform1m":
         return gen.uniform(1 << 20, 1 << 20, 16, seed=42, r0=r0, r1=r1)
     if workload == "zipf4m":
@@ -69,8 +73,8 @@ def global_rowptr(workload: str) -> np.ndarray:
     import ctypes
 
     import gen
-    if workload in ("lap8192", "lap64"):
-        n = 8192 if workload == "lap8192" else 64
+    if workload in ("lap8192", "lap64", "lap2048"):
+        n = {"lap8192": 8192, "lap64": 64, "lap2048": 2048}[workload]
         rp = np.empty(n * n + 1, dtype=np.int64)
         gen.lib().gen_laplacian2d_rowptr(n, 0, n * n, rp.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)))
         return rp
@@ -313,6 +317,15 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
         if world > 1:
             dist.barrier()
 
+    def allmax(v: float) -> float:
+        """max over ranks (device tensor for NCCL, host tensor for gloo)"""
+        if world == 1:
+            return v
+        on_dev = dist.get_backend() == "nccl"
+        t = torch.tensor([v], dtype=torch.float64, device=dev if on_dev else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
     for _ in range(args.warmup):
         one_step(False)
     torch.cuda.synchronize()
@@ -338,11 +351,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     torch.cuda.synchronize()
     barrier()
     clk = clocks.stop()
-    total_ms = t_start.elapsed_time(t_end)
-    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    total_ms = float(t.item())
+    total_ms = allmax(t_start.elapsed_time(t_end))
 
     nspmv = iters * args.steps
     alg_bytes_global = Z * (4 + esz) + (R + 1) * 4 + A.ncols * esz + R * esz
@@ -350,11 +359,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
         secs = total_ms / 1e3
     else:
         # single-SpMV workloads: L2 flushed between calls; time = sum of kernel events
-        secs = sum(kern_ms) / 1e3
-        tk = torch.tensor([secs], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(tk, op=dist.ReduceOp.MAX)
-        secs = float(tk.item())
+        secs = allmax(sum(kern_ms) / 1e3)
     gflops = 2.0 * Z * nspmv / secs / 1e9
     gbs = alg_bytes_global * nspmv / secs / 1e9
     peak, peak_src = measured_peak()
@@ -425,11 +430,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     te = time.perf_counter()
     for _ in range(e2e_steps):
         plan.exec_host(xh, yh, iterations=e2e_iters, flags=e2e_flags, stream=stream)
-    te = time.perf_counter() - te
-    tt = torch.tensor([te], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-    te = float(tt.item())
+    te = allmax(time.perf_counter() - te)
     e2e_val = 2.0 * Z * e2e_iters * e2e_steps / te / 1e9
 
     cpu = None
@@ -487,11 +488,20 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    # Test-only knobs (tests/test_gpu_bench_multirank.py): run every rank on one
+    # device with gloo for torch.distributed (the library then needs
+    # PEPP_NCCL_LIB pointing at the NCCL stand-in). Never set by the driver.
+    if os.environ.get("PEPP_BENCH_ONE_DEVICE"):
+        local_rank = 0
     if world > 1:
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        backend = os.environ.get("PEPP_BENCH_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:
+            dist.init_process_group(backend)
     try:
         if args.impl == "reference":
             run_reference(args, rank, world)
