@@ -145,6 +145,14 @@ typedef struct {
                                  vector-CSR only if max_row <= max(4096, 256*mean), SELL only if
                                  max_row <= 4096; merge-path and CSR-stream always.
                                  0 = every variant is a candidate (variant_mask still applies). */
+    int32_t overlap;          /* partitioned halo plans (nranks > 1): 1 (default) = when the rows this
+                                 rank sends lie in a short head and tail of its block (stencils, banded
+                                 matrices), a PEPP_Y_NEXT_INPUT call computes head and tail first, then
+                                 runs the halo exchange on a plan-owned side stream while the interior
+                                 rows compute, and joins before returning (the paper's overlap of
+                                 communication with computation in partitioned execution, §IV-F
+                                 P@27330–28000). Costs a second device copy of the block (head,
+                                 interior and tail sub-plans). 0 = kernel, then exchange, in order. */
 } pepp_spmv_opts_t;
 
 /* Selection result. `candidate` indexes pepp_spmv_candidates(). The plan's
@@ -182,6 +190,9 @@ typedef struct {
     double sell_col16_frac;   /* fraction of SELL chunks storing 16-bit column deltas */
     uint64_t prior_key;       /* context key the cold-start prior came from (0 = none) */
     double sell_stencil_frac; /* fraction of SELL chunks stored as stencil (one offset per slot per chunk) */
+    int32_t overlap;          /* 1 = NEXT_INPUT calls overlap the halo exchange with the interior rows */
+    int64_t overlap_head;     /* rows [0, overlap_head) and [nrows - overlap_tail, nrows) are computed */
+    int64_t overlap_tail;     /*   before the exchange starts (0 / 0 when overlap == 0) */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

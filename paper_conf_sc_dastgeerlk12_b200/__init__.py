@@ -90,7 +90,7 @@ class Plan:
                  device: Optional[int] = None, min_samples: int = 3, sample_period: int = 8,
                  nranks: int = 1, rank: int = 0, row_bounds: Optional[Sequence[int]] = None,
                  nccl_unique_id: Optional[bytes] = None, exchange: int = X_AUTO,
-                 history_path: Optional[str] = None, prune: bool = True):
+                 history_path: Optional[str] = None, prune: bool = True, overlap: bool = True):
         L = C.lib()
         self._h = ctypes.c_void_p()
         on_dev = not isinstance(row_ptr, np.ndarray)
@@ -129,6 +129,7 @@ class Plan:
         self._hp = history_path.encode() if history_path else None
         o.history_path = self._hp
         o.prune = 1 if prune else 0
+        o.overlap = 1 if overlap else 0
         C.check(L.pepp_spmv_plan(ctypes.byref(A), ctypes.byref(o), ctypes.byref(self._h)), "pepp_spmv_plan")
         self.nrows, self.ncols, self.nnz = nrows, ncols, nnz
 

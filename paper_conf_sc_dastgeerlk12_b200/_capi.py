@@ -34,7 +34,8 @@ class OPTS_T(ctypes.Structure):
     _fields_ = [("variant_mask", c_u32), ("use_history", c_i32), ("validate", c_i32), ("sell_sigma", c_i32),
                 ("device", c_i32), ("min_samples", c_i32), ("sample_period", c_i32), ("nranks", c_i32),
                 ("rank", c_i32), ("row_bounds", c_vp), ("nccl_comm", c_vp), ("nccl_unique_id", c_vp),
-                ("exchange", c_i32), ("history_path", ctypes.c_char_p), ("prune", c_i32)]
+                ("exchange", c_i32), ("history_path", ctypes.c_char_p), ("prune", c_i32),
+                ("overlap", c_i32)]
 
 
 class CHOICE_T(ctypes.Structure):
@@ -54,7 +55,8 @@ class INFO_T(ctypes.Structure):
                 ("row_offset", c_i64), ("key", c_u64), ("ncandidates", c_i32), ("sell_sigma", c_i32),
                 ("sell_fill", c_f64), ("device_bytes", c_i64), ("algorithmic_bytes", c_i64),
                 ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64),
-                ("prior_key", c_u64), ("sell_stencil_frac", c_f64)]
+                ("prior_key", c_u64), ("sell_stencil_frac", c_f64),
+                ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}

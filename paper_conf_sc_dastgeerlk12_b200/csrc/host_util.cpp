@@ -50,6 +50,7 @@ extern "C" PEPP_API void pepp_spmv_opts_default(pepp_spmv_opts_t* o) {
     o->exchange = PEPP_X_AUTO;
     o->history_path = nullptr;
     o->prune = 1;
+    o->overlap = 1;
 }
 
 // ---------------------------------------------------------------- partition

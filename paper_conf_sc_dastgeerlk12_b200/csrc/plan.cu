@@ -43,6 +43,7 @@ constexpr int kStreamStages = 2;   // 2 x 26.7 KB per CTA -> 4 CTAs (32 warps) p
 constexpr int kStreamNB = 2048;
 constexpr int kStreamRMAX = 512;
 constexpr int kStreamVecMinLen = 64;   // items whose longest row exceeds this reduce warp-per-row
+constexpr int kReserveSms = 2;         // SMs the interior sub-plan's persistent grid leaves to the exchange
 
 struct Candidate {
     int32_t variant;
@@ -148,6 +149,14 @@ struct pepp_spmv_plan_s {
     int32_t exchange = PEPP_X_NONE;
     std::vector<PeerXfer> recv_x, send_x;
 
+    // halo / interior overlap (opts.overlap): head [0, h), interior, tail [R - t, R)
+    pepp_spmv_plan_t* sub[3] = {nullptr, nullptr, nullptr};
+    int64_t sub_r0[3] = {0, 0, 0};
+    cudaStream_t side = nullptr;                 // exchange stream (highest priority)
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    int reserve_sms = 0;                         // SMs a persistent grid leaves free (interior sub-plan)
+    std::vector<int64_t> send_local;             // plan time: local rows the peers receive
+
     // plan-owned x / y for pepp_spmv_exec_host (allocated on first use)
     void* d_hx = nullptr;
     void* d_hy = nullptr;
@@ -223,6 +232,10 @@ void free_plan(pepp_spmv_plan_t* p) {
     for (auto& r : p->ring) { if (r.start) cudaEventDestroy(r.start); if (r.stop) cudaEventDestroy(r.stop); }
     if (p->comm && p->own_comm && p->nccl) p->nccl->CommDestroy(p->comm);
     if (p->hist) pepp::history_free(p->hist);
+    for (auto* q : p->sub) free_plan(q);
+    if (p->ev_fork) cudaEventDestroy(p->ev_fork);
+    if (p->ev_join) cudaEventDestroy(p->ev_join);
+    if (p->side) cudaStreamDestroy(p->side);
     delete p;
 }
 
@@ -773,6 +786,7 @@ pepp_status_t setup_halo(pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts
         if (scount[q]) {
             std::vector<int32_t> sl(scount[q]);
             PEPP_CUDA_TRY(cudaMemcpy(sl.data(), d_s[q].p, sizeof(int) * scount[q], cudaMemcpyDeviceToHost));
+            for (int32_t v : sl) p->send_local.push_back((int64_t)v - p->row_offset);
             pepp_status_t s = make(q, sl, d_s[q], p->send_x);
             if (s) return s;
         }
@@ -782,6 +796,76 @@ pepp_status_t setup_halo(pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts
     for (auto& t : p->send_x) ts += t.count;
     p->info.halo_recv = tr;
     p->info.halo_send = ts;
+    return PEPP_OK;
+}
+
+pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spmv_plan_t* p);
+
+// rows [r0, r1) of this block as a plan of their own (unpartitioned, same
+// options); the slice shares A's arrays, offset by row_ptr[r0] - first
+pepp_status_t make_sub(const pepp_csr_t* A, const pepp_spmv_opts_t* o, const pepp_spmv_plan_t* p, int64_t r0,
+                       int64_t r1, int reserve, pepp_spmv_plan_t** out) {
+    *out = nullptr;
+    int64_t b0 = 0, b1 = 0;
+    if (A->on_device) {
+        PEPP_CUDA_TRY(cudaMemcpy(&b0, A->row_ptr + r0, sizeof(int64_t), cudaMemcpyDeviceToHost));
+        PEPP_CUDA_TRY(cudaMemcpy(&b1, A->row_ptr + r1, sizeof(int64_t), cudaMemcpyDeviceToHost));
+    } else {
+        b0 = A->row_ptr[r0];
+        b1 = A->row_ptr[r1];
+    }
+    pepp_csr_t S = *A;
+    S.nrows = r1 - r0;
+    S.nnz = b1 - b0;
+    S.first = b0;
+    S.row_ptr = A->row_ptr + r0;
+    if (A->nnz) {
+        S.col_idx = A->col_idx + (b0 - A->first);
+        S.values = (const char*)A->values + (b0 - A->first) * (int64_t)p->esz;
+    }
+    pepp_spmv_opts_t so = *o;
+    so.nranks = 1; so.rank = 0; so.row_bounds = nullptr;
+    so.nccl_comm = nullptr; so.nccl_unique_id = nullptr; so.exchange = PEPP_X_NONE;
+    so.history_path = nullptr; so.overlap = 0;
+    so.validate = 0;          // the whole block was validated
+    so.device = p->device;
+    pepp_spmv_plan_t* q = new (std::nothrow) pepp_spmv_plan_t();
+    if (!q) return PEPP_E_NOMEM;
+    q->device = -1;
+    q->reserve_sms = reserve;
+    pepp_status_t s = plan_impl(&S, &so, q);
+    if (s) { free_plan(q); return s; }
+    *out = q;
+    return PEPP_OK;
+}
+
+// Overlap of the halo exchange with the interior rows (opts.overlap). The
+// rows peers receive must lie in a head [0, h) and a tail [R - t, R) with
+// h + t <= R / 2; else the block keeps the in-order kernel -> exchange path.
+pepp_status_t setup_overlap(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spmv_plan_t* p) {
+    const int64_t R = p->nrows;
+    int64_t h = 0, t = 0;
+    for (int64_t v : p->send_local) {
+        if (v < 0 || v >= R) return PEPP_OK;   // not a row of this block: no overlap
+        if (v < R / 2) h = std::max(h, v + 1);
+        else t = std::max(t, R - v);
+    }
+    if (R < 2 || h + t > R / 2) return PEPP_OK;
+    pepp_status_t s;
+    const int64_t bnd[4] = {0, h, R - t, R};
+    for (int i = 0; i < 3; ++i) {
+        p->sub_r0[i] = bnd[i];
+        if (bnd[i + 1] > bnd[i] && (s = make_sub(A, o, p, bnd[i], bnd[i + 1], i == 1 ? kReserveSms : 0, &p->sub[i])))
+            return s;
+    }
+    int lo = 0, hi = 0;
+    PEPP_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    PEPP_CUDA_TRY(cudaStreamCreateWithPriority(&p->side, cudaStreamNonBlocking, hi));
+    PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming));
+    PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_join, cudaEventDisableTiming));
+    p->info.overlap = 1;
+    p->info.overlap_head = h;
+    p->info.overlap_tail = t;
     return PEPP_OK;
 }
 
@@ -937,7 +1021,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pepp::k::sell_kernel<kBlock, false, double>, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
         (void)cudaGetLastError();
         const int64_t need = ((int64_t)p->nchunks + kBlock / 32 - 1) / (kBlock / 32);
-        const int64_t wave = (int64_t)p->sm_count * occ;
+        const int64_t wave = (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ;
         // prefetching pays once a warp walks many chunks; small matrices keep
         // more (shorter-lived) blocks instead
         const int64_t cap = need >= 16 * wave ? wave : 4 * wave;
@@ -1002,13 +1086,48 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         p->exchange = ex;
     }
     I.exchange = p->exchange;
+    if (p->exchange == PEPP_X_HALO && o->overlap && !p->send_local.empty())
+        if ((s = setup_overlap(A, o, p))) return s;
+    p->send_local.clear();
+    p->send_local.shrink_to_fit();
     I.device_bytes = p->dev_bytes;
+    for (auto* q : p->sub) if (q) I.device_bytes += q->dev_bytes;
     return PEPP_OK;
 }
 
 }  // namespace
 
 // ================================================================= C-ABI
+extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void* x, void* y, int flags,
+                                                void* stream, const pepp_choice_t* force, pepp_choice_t* used);
+
+namespace {
+// head and tail rows, then (side stream) the halo exchange, which reads only
+// those rows and writes only other ranks' rows of y, while the interior rows
+// compute on the caller's stream; the caller's stream joins the exchange.
+pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flags, cudaStream_t st,
+                           pepp_choice_t* used) {
+    char* yb = (char*)y + p->row_offset * (int64_t)p->esz;
+    const int sf = flags & PEPP_EXEC_NO_TIMING;
+    pepp_status_t s;
+    for (int i : {0, 2})
+        if (p->sub[i] && (s = pepp_spmv_exec(p->sub[i], x, yb + p->sub_r0[i] * (int64_t)p->esz, sf, st, nullptr, nullptr)))
+            return s;
+    PEPP_CUDA_TRY(cudaEventRecord(p->ev_fork, st));
+    PEPP_CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_fork, 0));
+    pepp_status_t sx = exchange_halo(p, y, p->side);
+    pepp_choice_t u{};
+    s = sx ? sx : pepp_spmv_exec(p->sub[1], x, yb + p->sub_r0[1] * (int64_t)p->esz, sf, st, nullptr, &u);
+    PEPP_CUDA_TRY(cudaEventRecord(p->ev_join, p->side));   // join whatever reached the side stream
+    PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_join, 0));
+    if (s) return s;
+    u.nparts = p->opts.nranks;
+    u.exchange = PEPP_X_HALO;
+    if (used) *used = u;
+    return PEPP_OK;
+}
+}  // namespace
+
 extern "C" PEPP_API pepp_status_t pepp_spmv_plan(const pepp_csr_t* A, const pepp_spmv_opts_t* opts,
                                                 pepp_spmv_plan_t** out) {
     if (!out) return PEPP_E_INVALID;
@@ -1055,6 +1174,12 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
     cudaStream_t st = (cudaStream_t)stream;
     DeviceScope dscope(p->device);
     if (!dscope.ok) return PEPP_E_CUDA;
+    if (!force && p->sub[1] && (flags & PEPP_Y_NEXT_INPUT) && !(flags & PEPP_Y_REPLICATED) && p->exchange == PEPP_X_HALO) {
+        pepp_status_t s = exec_overlap(p, x, y, flags, st, used);
+        if (s) p->sticky = s;
+        else ++p->ncalls;
+        return s;
+    }
     pepp_choice_t ch{};
     if (force) {
         int idx = -1;
@@ -1295,6 +1420,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_flush_history(pepp_spmv_plan_t* p) {
     if (!p) return PEPP_E_INVALID;
     DeviceScope dscope(p->device);
     harvest(p, true);
+    for (auto* q : p->sub) if (q) harvest(q, true);
     return PEPP_OK;
 }
 

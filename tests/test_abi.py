@@ -65,6 +65,7 @@ int main(void) {
   P(pepp_csr_t, on_device) P(pepp_spmv_opts_t, row_bounds) P(pepp_spmv_opts_t, exchange)
   P(pepp_spmv_opts_t, history_path) P(pepp_spmv_opts_t, prune) P(pepp_choice_t, predicted_us) P(pepp_plan_info_t, key)
   P(pepp_plan_info_t, sell_fill) P(pepp_plan_info_t, halo_send) P(pepp_plan_info_t, sell_col16_frac) P(pepp_plan_info_t, prior_key) P(pepp_plan_info_t, sell_stencil_frac)
+  P(pepp_spmv_opts_t, overlap) P(pepp_plan_info_t, overlap) P(pepp_plan_info_t, overlap_head) P(pepp_plan_info_t, overlap_tail)
   return 0;
 }
 """
@@ -90,6 +91,9 @@ int main(void) {
     assert int(vals["pepp_plan_info_t.sell_col16_frac"]) == C.INFO_T.sell_col16_frac.offset
     assert int(vals["pepp_plan_info_t.prior_key"]) == C.INFO_T.prior_key.offset
     assert int(vals["pepp_plan_info_t.sell_stencil_frac"]) == C.INFO_T.sell_stencil_frac.offset
+    for f in ("overlap", "overlap_head", "overlap_tail"):
+        assert int(vals["pepp_plan_info_t." + f]) == getattr(C.INFO_T, f).offset
+    assert int(vals["pepp_spmv_opts_t.overlap"]) == C.OPTS_T.overlap.offset
 
 
 def test_sm100a_cubin_present():

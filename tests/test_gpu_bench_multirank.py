@@ -42,5 +42,8 @@ def test_bench_two_ranks_one_gpu():
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["steps"] == 1 and d["value"] > 0
     assert d["config"]["exchange"] == "halo"
-    assert d["e2e"]["value"] > 0 and d["gpu_launches"] == 100
+    # rank 0's block sends its last grid row: tail + interior kernels per SpMV, exchange overlapped
+    assert d["plan"]["overlap"] == 1 and d["plan"]["overlap_head"] == 0 and d["plan"]["overlap_tail"] == 2048
+    assert d["e2e"]["value"] > 0 and d["gpu_launches"] >= 200
+    assert "launch_includes" in d["roofline"]
     assert d["cpu_baseline"] is None          # rank 0 at N = 1 only

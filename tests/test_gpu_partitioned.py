@@ -43,7 +43,7 @@ def _matrix(name):
     raise ValueError(name)
 
 
-def _worker(rank, world, lib, uid, name, exchange, K, outq, f32=False):
+def _worker(rank, world, lib, uid, name, exchange, K, outq, f32=False, overlap=True):
     os.environ["PEPP_NCCL_LIB"] = lib
     try:
         import sys
@@ -63,7 +63,7 @@ def _worker(rank, world, lib, uid, name, exchange, K, outq, f32=False):
         x0 = gen.vector(3, gen.INT8, n).astype(np.float32 if f32 else np.float64)
         res = {}
         with pepp.Plan.from_csr(blk, nranks=world, rank=rank, row_bounds=bounds, nccl_unique_id=uid,
-                                exchange=exchange) as plan:
+                                exchange=exchange, overlap=overlap) as plan:
             info = plan.info()
             a = torch.from_numpy(x0).cuda()
             b = torch.full_like(a, float("nan"))
@@ -90,19 +90,20 @@ def _worker(rank, world, lib, uid, name, exchange, K, outq, f32=False):
             res["exchange"] = info["exchange"]
             res["halo_recv"] = info["halo_recv"]
             res["halo_send"] = info["halo_send"]
+            res["overlap"] = (info["overlap"], info["overlap_head"], info["overlap_tail"])
         outq.put((rank, res))
     except Exception as e:
         import traceback
         outq.put((rank, {"error": repr(e) + traceback.format_exc()}))
 
 
-def _run(name, exchange, K=6, f32=False):
+def _run(name, exchange, K=6, f32=False, overlap=True):
     import torch.multiprocessing as mp
     lib = _build_fake()
     uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_{exchange}".encode() + b"\0" * 128)[:128]
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker, args=(r, 2, lib, uid, name, exchange, K, q, f32)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, lib, uid, name, exchange, K, q, f32, overlap)) for r in range(2)]
     for p in procs:
         p.start()
     out = {}
@@ -129,6 +130,20 @@ def test_two_ranks_one_gpu_iterated_spmv_bitwise(name, exchange):
         assert ex == {exchange}
     if name == "lap" and exchange == pepp.X_HALO:
         assert out[0]["halo_recv"] == 96 and out[1]["halo_send"] == 96   # one grid row each way
+        # the rows each rank sends are one grid row at the block's edge: head / tail sub-plans
+        assert out[0]["overlap"] == (1, 0, 96) and out[1]["overlap"] == (1, 96, 0)
+    if name == "zipf" and exchange == pepp.X_HALO:
+        assert out[0]["overlap"][0] == 0   # random columns: the sent rows are everywhere
+
+
+@pytest.mark.parametrize("name,exchange,overlap", [("lap", 2, False), ("banded", 2, True), ("banded", 2, False)])
+def test_two_ranks_halo_overlap_on_off(name, exchange, overlap):
+    """opts.overlap: the head / interior / tail split with the exchange on the
+    side stream gives the same bits as the in-order kernel -> exchange path."""
+    out = _run(name, exchange, overlap=overlap)
+    for r in range(2):
+        assert out[r]["iter"] and out[r]["host"], (r, out[r])
+        assert out[r]["overlap"][0] == (1 if overlap else 0)
 
 
 @pytest.mark.parametrize("name,exchange", [("lap", 2), ("zipf", 1)])
