@@ -592,12 +592,23 @@ void fill_choice(const pepp_spmv_plan_t* p, int cand, int calibrating, double pr
     out->predicted_us = pred;
 }
 
-pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out) {
-    harvest(p, false);
+// frozen: the call is being captured into a CUDA graph — no event queries (a
+// global-mode capture forbids them) and no calibration (nothing is timed):
+// the best measured candidate so far, else the heuristic
+pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out, bool frozen = false) {
+    if (!frozen) harvest(p, false);
     int calibrating = 0;
     double pred = 0.0;
     int cand;
-    if (p->opts.use_history) {
+    if (frozen) {
+        cand = -1;
+        for (int32_t c = 0; c < (int32_t)p->cands.size(); ++c) {
+            const pepp::Welford* w = pepp::history_get(p->hist, p->key, p->uids[c]);
+            if (!p->eligible[c] || !w || w->count == 0) continue;
+            if (cand < 0 || w->mean < pred * 0.99) { cand = c; pred = w->mean; }
+        }
+        if (cand < 0) cand = heuristic_candidate(p);
+    } else if (p->opts.use_history) {
         // Calibration counts timed calls already in flight, so the host (which
         // runs far ahead of the GPU) moves on to the next under-sampled
         // candidate instead of re-issuing the same one; once every candidate
@@ -1174,6 +1185,12 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
     cudaStream_t st = (cudaStream_t)stream;
     DeviceScope dscope(p->device);
     if (!dscope.ok) return PEPP_E_CUDA;
+    bool capturing = false;
+    {
+        cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+        if (cudaStreamIsCapturing(st, &cs) != cudaSuccess) { (void)cudaGetLastError(); cs = cudaStreamCaptureStatusNone; }
+        capturing = cs != cudaStreamCaptureStatusNone;
+    }
     if (!force && p->sub[1] && (flags & PEPP_Y_NEXT_INPUT) && !(flags & PEPP_Y_REPLICATED) && p->exchange == PEPP_X_HALO) {
         pepp_status_t s = exec_overlap(p, x, y, flags, st, used);
         if (s) p->sticky = s;
@@ -1189,20 +1206,15 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         fill_choice(p, idx, 0, 0.0, &ch);
         if (p->opts.nranks > 1 && (force->exchange == PEPP_X_ALLGATHER || force->exchange == PEPP_X_HALO))
             ch.exchange = force->exchange;
-        harvest(p, false);
+        if (!capturing) harvest(p, false);
     } else {
-        pepp_status_t s = select_choice(p, &ch);
+        pepp_status_t s = select_choice(p, &ch, capturing);
         if (s) return s;
     }
 
     // timing: every calibration call and every forced call, then every
     // sample_period-th call; never inside a CUDA graph capture
-    bool timed = !(flags & PEPP_EXEC_NO_TIMING);
-    if (timed) {
-        cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-        if (cudaStreamIsCapturing(st, &cs) != cudaSuccess) { (void)cudaGetLastError(); cs = cudaStreamCaptureStatusNone; }
-        if (cs != cudaStreamCaptureStatusNone) timed = false;
-    }
+    bool timed = !(flags & PEPP_EXEC_NO_TIMING) && !capturing;
     if (timed && !force && !ch.calibrating)
         timed = p->opts.sample_period > 0 && (p->ncalls % p->opts.sample_period) == 0;
     if (timed && p->ring_count == kTimingRing) timed = false;

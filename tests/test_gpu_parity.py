@@ -408,6 +408,39 @@ def test_graph_repeat_and_iterate_match_oracle():
             plan.graph(x, y, iterations=4, mode=1)   # iterate needs a work buffer
 
 
+@pytest.mark.parametrize("calibrate", [False, True])
+def test_torch_graph_capture_global_mode(calibrate):
+    """plan.exec inside torch.cuda.graph (global capture mode, which forbids
+    event queries): the selection freezes to the best measured candidate (or
+    the heuristic before any timing), nothing is timed, replays are exact."""
+    A = gen.uniform(20_000, 20_000, 12, seed=61, val_mode=gen.INT4)
+    x0 = gen.vector(62, gen.INT8, 20_000)
+    with pepp.Plan.from_csr(A) as plan:
+        x = _dev(x0)
+        y = torch.full((20_000,), float("nan"), dtype=torch.float64, device="cuda")
+        if calibrate:
+            for _ in range(40):
+                plan.exec(x, y)
+            plan.flush_history()
+        before = [plan.history_stats(c)[0] for c in range(len(plan.candidates()))]
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.stream(s):
+            with torch.cuda.graph(g, stream=s):
+                u = plan.exec(x, y, stream=s)
+        assert not u.calibrating
+        if calibrate:
+            assert u.name == plan.select().name
+        y.fill_(float("nan"))
+        g.replay()
+        g.replay()
+        torch.cuda.synchronize()
+        assert np.array_equal(y.cpu().numpy(), oracle.spmv(A, x0))
+        plan.flush_history()
+        assert [plan.history_stats(c)[0] for c in range(len(plan.candidates()))] == before
+
+
 def test_cold_start_from_persisted_history(tmp_path):
     """A plan on an unseen context, loading a history file recorded on a
     similar matrix, calibrates the predicted best first and skips candidates
