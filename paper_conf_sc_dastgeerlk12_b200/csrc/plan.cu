@@ -17,6 +17,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -894,6 +895,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     if (o->variant_mask != 0 && (o->variant_mask & ((1u << PEPP_V_COUNT) - 1)) == 0) return PEPP_E_INVALID;
 
     p->opts = *o;
+    if (const char* e = std::getenv("PEPP_RESERVE_SMS")) p->reserve_sms = std::atoi(e);   // experiments only (tools/overlap_cost.py)
     p->nrows = A->nrows; p->ncols = A->ncols; p->nnz = A->nnz; p->first = A->first;
     p->pad = (int)(((A->first % 4) + 4) % 4);
     if (o->nranks > 1) {
@@ -1113,22 +1115,26 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
                                                 void* stream, const pepp_choice_t* force, pepp_choice_t* used);
 
 namespace {
-// head and tail rows, then (side stream) the halo exchange, which reads only
-// those rows and writes only other ranks' rows of y, while the interior rows
-// compute on the caller's stream; the caller's stream joins the exchange.
+// The interior rows compute on the caller's stream while a high-priority side
+// stream computes the head and tail rows (into the SMs the interior's
+// persistent grid leaves free) and then runs the halo exchange, which reads
+// only head / tail rows and writes only other ranks' rows of y; the caller's
+// stream joins the side stream. Critical path: max(interior, head + tail +
+// exchange) instead of kernel + exchange.
 pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flags, cudaStream_t st,
                            pepp_choice_t* used) {
     char* yb = (char*)y + p->row_offset * (int64_t)p->esz;
     const int sf = flags & PEPP_EXEC_NO_TIMING;
-    pepp_status_t s;
-    for (int i : {0, 2})
-        if (p->sub[i] && (s = pepp_spmv_exec(p->sub[i], x, yb + p->sub_r0[i] * (int64_t)p->esz, sf, st, nullptr, nullptr)))
-            return s;
+    // the side stream starts after everything the caller queued (x is ready)
     PEPP_CUDA_TRY(cudaEventRecord(p->ev_fork, st));
     PEPP_CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_fork, 0));
-    pepp_status_t sx = exchange_halo(p, y, p->side);
+    // interior first (the host may block inside a synchronous exchange)
     pepp_choice_t u{};
-    s = sx ? sx : pepp_spmv_exec(p->sub[1], x, yb + p->sub_r0[1] * (int64_t)p->esz, sf, st, nullptr, &u);
+    pepp_status_t s = pepp_spmv_exec(p->sub[1], x, yb + p->sub_r0[1] * (int64_t)p->esz, sf, st, nullptr, &u);
+    for (int i : {0, 2})
+        if (!s && p->sub[i])
+            s = pepp_spmv_exec(p->sub[i], x, yb + p->sub_r0[i] * (int64_t)p->esz, sf, p->side, nullptr, nullptr);
+    if (!s) s = exchange_halo(p, y, p->side);
     PEPP_CUDA_TRY(cudaEventRecord(p->ev_join, p->side));   // join whatever reached the side stream
     PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_join, 0));
     if (s) return s;

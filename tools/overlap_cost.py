@@ -5,8 +5,10 @@ For the config-4 Laplacian (8192^2) partitioned over P ranks, take a middle
 rank's row block (it sends one grid row at each end) and time, back to back
 on one stream with the L2-exceeding block:
   whole : the block as one plan (the in-order path's kernel)
-  split : head (n rows) + tail (n rows) + interior as three plans, in the
-          order the overlapped call issues them
+  split : head (n rows) + tail (n rows) + interior as three plans, one
+          after the other
+  concurrent_rK : interior on the caller's stream with K SMs left free,
+          head + tail on a high-priority side stream (the overlapped call)
 The difference is what the overlap costs on the critical path; what it saves
 is the exchange time, which runs beside the interior kernel (not measurable
 with one GPU). One JSON line per P.
@@ -83,6 +85,29 @@ def main():
                 res["each_us"] = [round(timed([c], a.reps), 2) for c in calls]
             res[name + "_choices"] = [p.select().name for p, _, _ in plans]
             for p, _, _ in plans:
+                p.close()
+        # as the overlapped call runs it: interior on the caller's stream (its
+        # persistent grid leaving `reserve` SMs), head + tail on a high-priority
+        # side stream, fork / join (the exchange itself is not modelled)
+        side = torch.cuda.Stream(priority=-1)
+        for reserve in (0, 2, 4):
+            os.environ["PEPP_RESERVE_SMS"] = str(reserve)
+            inner = pepp.Plan.from_csr(gen.row_block(A, r0 + n, r1 - n))
+            del os.environ["PEPP_RESERVE_SMS"]
+            edges = [(pepp.Plan.from_csr(gen.row_block(A, s, e)), s, e) for s, e in [(r0, r0 + n), (r1 - n, r1)]]
+
+            def conc():
+                main = torch.cuda.current_stream()
+                side.wait_stream(main)
+                inner.exec(x, y[r0 + n:r1 - n], stream=main)
+                for p, s, e in edges:
+                    p.exec(x, y[s:e], stream=side)
+                main.wait_stream(side)
+            res[f"concurrent_r{reserve}_us"] = round(timed([conc], a.reps), 2)
+            res[f"interior_r{reserve}_us"] = round(timed([lambda: inner.exec(x, y[r0 + n:r1 - n],
+                                                                          stream=torch.cuda.current_stream())], a.reps), 2)
+            inner.close()
+            for p, _, _ in edges:
                 p.close()
         res["split_cost_us"] = round(res["split_us"] - res["whole_us"], 2)
         print(json.dumps(res), flush=True)
