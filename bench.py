@@ -200,7 +200,24 @@ def cpu_baseline(A, x0: np.ndarray, iters: int) -> dict:
     return {"value": round(gflops, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
             "sample": f"{iters} full-size SpMV(s) of the bench matrix ({A.nnz} nnz) with "
                       f"oracle_spmv_rows_parallel on {cores} OpenMP threads",
-            "seq_1core_gflops": round(2.0 * A.nnz / ts / 1e9, 3)}
+            "seq_1core_gflops": round(2.0 * A.nnz / ts / 1e9, 3), "host": host_cpu()}
+
+
+def host_cpu() -> dict:
+    """CPU model and socket count of the host the oracle ran on."""
+    model, sockets = None, set()
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                k, _, v = line.partition(":")
+                k = k.strip()
+                if k == "model name" and model is None:
+                    model = v.strip()
+                elif k == "physical id":
+                    sockets.add(v.strip())
+    except OSError:
+        pass
+    return {"model": model, "sockets": len(sockets) or None, "nproc": os.cpu_count()}
 
 
 # --------------------------------------------------------------- arms
@@ -229,7 +246,7 @@ def run_reference(args, rank: int, world: int) -> None:
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": args.workload, "desc": wl["desc"]},
             "cpu_baseline": {"value": round(val, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
-                             "sample": sample},
+                             "sample": sample, "host": host_cpu()},
             "e2e": {"value": round(val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 

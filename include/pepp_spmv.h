@@ -121,6 +121,19 @@ typedef struct {
     int32_t value_type;       /* PEPP_VALUE_F64 (0, default) or PEPP_VALUE_F32 */
 } pepp_csr_t;
 
+struct pepp_plan_info_s;   /* = pepp_plan_info_t, below */
+
+/* Performance prediction function (the component descriptor's "reference to a
+   (usually, programmer provided) performance prediction function that is
+   called with a given context descriptor data structure", §II P@6887–7157).
+   Called at plan time, once per candidate, with the plan's context instance
+   (`context`: sizes, row statistics, key; the candidate list is not final
+   yet) and the candidate's variant and tunable; returns the predicted time of
+   one call in µs, or <= 0 for "no prediction". Must not call back into the
+   plan. `user` is opts.predict_user. */
+typedef double (*pepp_predict_fn)(const struct pepp_plan_info_s* context, int32_t variant, int32_t param,
+                                  void* user);
+
 /* Plan options. Use pepp_spmv_opts_default() then override. */
 typedef struct {
     uint32_t variant_mask;    /* bit v set = variant v allowed; 0 = all (the paper's disableImpls, P@16687) */
@@ -153,6 +166,15 @@ typedef struct {
                                  communication with computation in partitioned execution, §IV-F
                                  P@27330–28000). Costs a second device copy of the block (head,
                                  interior and tail sub-plans). 0 = kernel, then exchange, in order. */
+    pepp_predict_fn predict;  /* optional (NULL = none). Its predictions stand in where no recorded
+                                 history exists: with use_history = 1 they order the calibration
+                                 (predicted best first) and rule out candidates predicted > 4x the
+                                 best prediction, exactly like a cold-start prior from a recorded
+                                 context (which takes precedence when both exist); with
+                                 use_history = 0 every call dispatches to the argmin of the
+                                 predictions (static composition through the prediction function,
+                                 P@10069) instead of the built-in heuristic. */
+    void* predict_user;       /* passed to predict; borrowed, used only during pepp_spmv_plan */
 } pepp_spmv_opts_t;
 
 /* Selection result. `candidate` indexes pepp_spmv_candidates(). The plan's
@@ -170,7 +192,7 @@ typedef struct {
 
 /* Context instance (§III P@9781: "a tuple of concrete values for context
    properties that might influence callee selection") + plan facts. */
-typedef struct {
+typedef struct pepp_plan_info_s {
     int64_t nrows, ncols, nnz;
     double mean_row;          /* nnz / nrows */
     double cv_row;            /* coefficient of variation of row lengths */
@@ -193,6 +215,7 @@ typedef struct {
     int32_t overlap;          /* 1 = NEXT_INPUT calls overlap the halo exchange with the interior rows */
     int64_t overlap_head;     /* rows [0, overlap_head) and [nrows - overlap_tail, nrows) are computed */
     int64_t overlap_tail;     /*   before the exchange starts (0 / 0 when overlap == 0) */
+    int32_t predicted;        /* candidates with a prediction from opts.predict (0 = none / no function) */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

@@ -90,7 +90,8 @@ class Plan:
                  device: Optional[int] = None, min_samples: int = 3, sample_period: int = 8,
                  nranks: int = 1, rank: int = 0, row_bounds: Optional[Sequence[int]] = None,
                  nccl_unique_id: Optional[bytes] = None, exchange: int = X_AUTO,
-                 history_path: Optional[str] = None, prune: bool = True, overlap: bool = True):
+                 history_path: Optional[str] = None, prune: bool = True, overlap: bool = True,
+                 predict=None):
         L = C.lib()
         self._h = ctypes.c_void_p()
         on_dev = not isinstance(row_ptr, np.ndarray)
@@ -130,6 +131,17 @@ class Plan:
         o.history_path = self._hp
         o.prune = 1 if prune else 0
         o.overlap = 1 if overlap else 0
+        cb = None
+        if predict is not None:
+            # predict(context: dict, variant: int, param: int) -> µs (<= 0: no prediction);
+            # called only inside pepp_spmv_plan (the descriptor's prediction function, P@6887)
+            def _cb(info_p, variant, param, _user):
+                try:
+                    return float(predict(info_p.contents.as_dict(), int(variant), int(param)))
+                except Exception:   # never unwind through the C caller
+                    return -1.0
+            cb = C.PREDICT_FN(_cb)
+            o.predict = cb
         C.check(L.pepp_spmv_plan(ctypes.byref(A), ctypes.byref(o), ctypes.byref(self._h)), "pepp_spmv_plan")
         self.nrows, self.ncols, self.nnz = nrows, ncols, nnz
 

@@ -30,12 +30,29 @@ class CSR_T(ctypes.Structure):
                 ("row_ptr", c_vp), ("col_idx", c_vp), ("values", c_vp), ("on_device", c_i32), ("value_type", c_i32)]
 
 
+class INFO_T(ctypes.Structure):
+    _fields_ = [("nrows", c_i64), ("ncols", c_i64), ("nnz", c_i64), ("mean_row", c_f64), ("cv_row", c_f64),
+                ("max_row", c_i64), ("empty_rows", c_i64), ("nranks", c_i32), ("rank", c_i32),
+                ("row_offset", c_i64), ("key", c_u64), ("ncandidates", c_i32), ("sell_sigma", c_i32),
+                ("sell_fill", c_f64), ("device_bytes", c_i64), ("algorithmic_bytes", c_i64),
+                ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64),
+                ("prior_key", c_u64), ("sell_stencil_frac", c_f64),
+                ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64), ("predicted", c_i32)]
+
+    def as_dict(self) -> dict:
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+# pepp_predict_fn: double (*)(const pepp_plan_info_t*, int32_t variant, int32_t param, void* user)
+PREDICT_FN = ctypes.CFUNCTYPE(c_f64, ctypes.POINTER(INFO_T), c_i32, c_i32, c_vp)
+
+
 class OPTS_T(ctypes.Structure):
     _fields_ = [("variant_mask", c_u32), ("use_history", c_i32), ("validate", c_i32), ("sell_sigma", c_i32),
                 ("device", c_i32), ("min_samples", c_i32), ("sample_period", c_i32), ("nranks", c_i32),
                 ("rank", c_i32), ("row_bounds", c_vp), ("nccl_comm", c_vp), ("nccl_unique_id", c_vp),
                 ("exchange", c_i32), ("history_path", ctypes.c_char_p), ("prune", c_i32),
-                ("overlap", c_i32)]
+                ("overlap", c_i32), ("predict", PREDICT_FN), ("predict_user", c_vp)]
 
 
 class CHOICE_T(ctypes.Structure):
@@ -47,19 +64,6 @@ class CHOICE_T(ctypes.Structure):
                 "param": self.param, "nparts": self.nparts, "exchange": EXCHANGE_NAMES.get(self.exchange, "?"),
                 "calibrating": bool(self.calibrating), "candidate": self.candidate,
                 "predicted_us": self.predicted_us}
-
-
-class INFO_T(ctypes.Structure):
-    _fields_ = [("nrows", c_i64), ("ncols", c_i64), ("nnz", c_i64), ("mean_row", c_f64), ("cv_row", c_f64),
-                ("max_row", c_i64), ("empty_rows", c_i64), ("nranks", c_i32), ("rank", c_i32),
-                ("row_offset", c_i64), ("key", c_u64), ("ncandidates", c_i32), ("sell_sigma", c_i32),
-                ("sell_fill", c_f64), ("device_bytes", c_i64), ("algorithmic_bytes", c_i64),
-                ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64),
-                ("prior_key", c_u64), ("sell_stencil_frac", c_f64),
-                ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64)]
-
-    def as_dict(self) -> dict:
-        return {f: getattr(self, f) for f, _ in self._fields_}
 
 
 # (name, restype, argtypes) for every entry point of include/pepp_spmv.h

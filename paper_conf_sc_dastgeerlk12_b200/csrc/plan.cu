@@ -141,6 +141,7 @@ struct pepp_spmv_plan_s {
     std::vector<int32_t> uids;      // stable candidate identity in the history: variant << 20 | param
     std::vector<double> prior;      // cold-start means from the nearest recorded context (-1 = none)
     std::vector<int32_t> order;     // calibration order (predicted best first)
+    std::vector<double> predicted;  // opts.predict per candidate (-1 = none)
     uint64_t prior_key = 0;
 
     // multi-GPU
@@ -565,7 +566,16 @@ void harvest(pepp_spmv_plan_t* p, bool block) {
 }
 
 int heuristic_candidate(const pepp_spmv_plan_t* p) {
-    // use_history = 0: fixed rule from the context instance (mean, CV)
+    // use_history = 0: the argmin of the user's prediction function when it
+    // predicted anything (ties -> lower index), else a fixed rule from the
+    // context instance (mean, CV)
+    {
+        int c = -1;
+        double best = 0.0;
+        for (size_t i = 0; i < p->predicted.size(); ++i)
+            if (p->eligible[i] && p->predicted[i] > 0 && (c < 0 || p->predicted[i] < best)) { c = (int)i; best = p->predicted[i]; }
+        if (c >= 0) return c;
+    }
     const double mean = p->info.mean_row, cv = p->info.cv_row;
     auto find = [&](int v, int prm) {
         for (size_t i = 0; i < p->cands.size(); ++i)
@@ -1054,8 +1064,17 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         p->prior.assign(n, -1.0);
         p->order.resize(n);
         for (int32_t c = 0; c < n; ++c) p->order[c] = c;
-        if (n && pepp::history_prior(p->hist, p->key, n, p->uids.data(), p->prior.data(), &p->prior_key)) {
-            p->info.prior_key = p->prior_key;
+        bool have_prior = n && pepp::history_prior(p->hist, p->key, n, p->uids.data(), p->prior.data(), &p->prior_key);
+        if (have_prior) p->info.prior_key = p->prior_key;
+        if (o->predict) {   // the descriptor's prediction function (M6, P@6887)
+            p->predicted.assign(n, -1.0);
+            for (int32_t c = 0; c < n; ++c) {
+                const double v = o->predict(&p->info, p->cands[c].variant, p->cands[c].param, o->predict_user);
+                if (v > 0 && std::isfinite(v)) { p->predicted[c] = v; ++p->info.predicted; }
+            }
+            if (!have_prior && p->info.predicted) { p->prior = p->predicted; have_prior = true; }
+        }
+        if (have_prior) {
             std::stable_sort(p->order.begin(), p->order.end(), [&](int32_t a, int32_t b) {
                 const double pa = p->prior[a] > 0 ? p->prior[a] : 1e300, pb = p->prior[b] > 0 ? p->prior[b] : 1e300;
                 return pa < pb;
@@ -1429,7 +1448,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_candidates(const pepp_spmv_plan_t* p
     for (int32_t i = 0; out && i < cap && i < *n; ++i) {
         fill_choice(p, i, 0, 0.0, &out[i]);
         const pepp::Welford* w = pepp::history_get(p->hist, p->key, p->uids[i]);
-        out[i].predicted_us = w ? w->mean : 0.0;
+        out[i].predicted_us = w ? w->mean : (p->prior[i] > 0 ? p->prior[i] : 0.0);
     }
     return PEPP_OK;
 }

@@ -66,6 +66,7 @@ int main(void) {
   P(pepp_spmv_opts_t, history_path) P(pepp_spmv_opts_t, prune) P(pepp_choice_t, predicted_us) P(pepp_plan_info_t, key)
   P(pepp_plan_info_t, sell_fill) P(pepp_plan_info_t, halo_send) P(pepp_plan_info_t, sell_col16_frac) P(pepp_plan_info_t, prior_key) P(pepp_plan_info_t, sell_stencil_frac)
   P(pepp_spmv_opts_t, overlap) P(pepp_plan_info_t, overlap) P(pepp_plan_info_t, overlap_head) P(pepp_plan_info_t, overlap_tail)
+  P(pepp_spmv_opts_t, predict) P(pepp_spmv_opts_t, predict_user) P(pepp_plan_info_t, predicted)
   return 0;
 }
 """
@@ -94,6 +95,9 @@ int main(void) {
     for f in ("overlap", "overlap_head", "overlap_tail"):
         assert int(vals["pepp_plan_info_t." + f]) == getattr(C.INFO_T, f).offset
     assert int(vals["pepp_spmv_opts_t.overlap"]) == C.OPTS_T.overlap.offset
+    assert int(vals["pepp_spmv_opts_t.predict"]) == C.OPTS_T.predict.offset
+    assert int(vals["pepp_spmv_opts_t.predict_user"]) == C.OPTS_T.predict_user.offset
+    assert int(vals["pepp_plan_info_t.predicted"]) == C.INFO_T.predicted.offset
 
 
 def test_sm100a_cubin_present():

@@ -441,6 +441,63 @@ def test_torch_graph_capture_global_mode(calibrate):
         assert [plan.history_stats(c)[0] for c in range(len(plan.candidates()))] == before
 
 
+def test_prediction_function_static_dispatch():
+    """use_history = 0 + opts.predict: every call dispatches to the argmin of
+    the user's predictions (P@6887 / P@10069), which see the context instance."""
+    A = gen.uniform(30_000, 30_000, 10, seed=63, val_mode=gen.INT4)
+    x0 = gen.vector(64, gen.INT8, 30_000)
+    seen = []
+
+    def predict(ctx, variant, param):
+        seen.append((ctx["nnz"], ctx["nrows"], round(ctx["mean_row"], 6), variant, param))
+        return 1.0 if (variant, param) == (pepp.V_CSR_VECTOR, 32) else 50.0
+
+    with pepp.Plan.from_csr(A, use_history=False, predict=predict) as plan:
+        cands = plan.candidates()
+        assert plan.info()["predicted"] == len(cands)
+        assert {(v, p) for *_, v, p in seen} == {(c.variant, c.param) for c in cands}
+        assert all(s[:3] == (A.nnz, A.nrows, round(A.nnz / A.nrows, 6)) for s in seen)
+        for _ in range(3):
+            y, u = _run(plan, x0)
+            assert (u.variant, u.param) == (pepp.V_CSR_VECTOR, 32) and not u.calibrating
+            _check(A, x0, y, True)
+    # no prediction (<= 0 everywhere): the built-in heuristic, same as without a function
+    with pepp.Plan.from_csr(A, use_history=False, predict=lambda c, v, p: 0.0) as plan, \
+            pepp.Plan.from_csr(A, use_history=False) as ref:
+        assert plan.info()["predicted"] == 0
+        assert _run(plan, x0)[1].name == _run(ref, x0)[1].name
+
+
+def test_prediction_function_orders_calibration():
+    """use_history = 1: the predictions act as a cold-start prior — the
+    predicted best is calibrated first and candidates predicted > 4x the best
+    are never timed; the final choice still comes from measurements."""
+    A = gen.laplacian2d(512)
+    x = _dev(gen.vector(65, gen.REAL, A.nrows))
+    y = torch.empty(A.nrows, dtype=torch.float64, device="cuda")
+    pred = {(pepp.V_MERGE_PATH, 7): 10.0, (pepp.V_SELL, 1): 12.0}
+
+    def predict(ctx, variant, param):
+        return pred.get((variant, param), 100.0)
+
+    with pepp.Plan.from_csr(A, predict=predict) as plan:
+        cands = plan.candidates()
+        assert all(c.predicted_us == pred.get((c.variant, c.param), 100.0) for c in cands)
+        first = plan.exec(x, y)
+        assert (first.variant, first.param) == (pepp.V_MERGE_PATH, 7) and first.calibrating
+        for _ in range(40):
+            plan.exec(x, y)
+        plan.flush_history()
+        for i, c in enumerate(cands):
+            n = plan.history_stats(i)[0]
+            if (c.variant, c.param) in pred:
+                assert n >= 3, (c.name, n)
+            else:
+                assert n == 0, (c.name, n)
+        best = plan.select()
+        assert (best.variant, best.param) in pred and not best.calibrating
+
+
 def test_cold_start_from_persisted_history(tmp_path):
     """A plan on an unseen context, loading a history file recorded on a
     similar matrix, calibrates the predicted best first and skips candidates
