@@ -268,7 +268,8 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
                                                      const T* __restrict__ val,
                                                      const T* __restrict__ x,
                                                      T* __restrict__ y,
-                                                     int cpw) {
+                                                     int cpw,
+                                                     const int* __restrict__ wstart) {
     const int lane = threadIdx.x & 31;
     const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
     const int nwarps = (gridDim.x * BLOCK) >> 5;
@@ -277,8 +278,10 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     // chunks are uniform (σ = 1). When σ > 1 sorted the rows, chunk lengths
     // repeat a long-to-short pattern in every window of cpw = σ/32 chunks and
     // a plain stride can hand a warp only the longest chunks; the order is
-    // then transposed (window-major -> position-major) over the full windows,
-    // a bijection that walks every warp through all positions.
+    // then transposed (window-major -> position-major) over the full windows
+    // (longest first), and warp w walks the contiguous range
+    // [wstart[w], wstart[w+1]) of that order, cut at plan time so that every
+    // warp gets the same number of slots.
     const int nfull = SORTED ? (nchunks / cpw) * cpw : 0;
     const int nwin = SORTED ? nchunks / cpw : 1;
     auto chunk_of = [&](int i) -> int {
@@ -292,14 +295,16 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     // chunk i+2's descriptor (length/flags, slot pointer) are in flight.
     struct Desc { int d; int64_t cp; };
     struct Lane { int len; int orow; int offl; };
+    int i = warp, end = nchunks, step = nwarps;
+    if (SORTED) { i = __ldg(wstart + warp); end = __ldg(wstart + warp + 1); step = 1; }
     auto desc = [&](int i) -> Desc {
         Desc q{0, 0};
-        if (i < nchunks) { const int c = chunk_of(i); q.d = __ldg(chunk_len + c); q.cp = __ldg(chunk_ptr + c); }
+        if (i < end) { const int c = chunk_of(i); q.d = __ldg(chunk_len + c); q.cp = __ldg(chunk_ptr + c); }
         return q;
     };
     auto lanes = [&](int i, const Desc& q) -> Lane {
         Lane l{0, 0, 0};
-        if (i >= nchunks) return l;
+        if (i >= end) return l;
         const int c = chunk_of(i);
         const int r = c * 32 + lane;
         l.len = !(q.d & kSellMasked) ? (q.d & kSellLenMask) : (r < nrows ? __ldg(rowlen + r) : 0);
@@ -307,12 +312,11 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
         if ((q.d & kSellStencil) && lane < (q.d & kSellLenMask)) l.offl = __ldg(soff + (q.cp >> 5) + lane);
         return l;
     };
-    int i = warp;
-    Desc q0 = desc(i), q1 = desc(i + nwarps);
+    Desc q0 = desc(i), q1 = desc(i + step);
     Lane l0 = lanes(i, q0);
-    for (; i < nchunks; i += nwarps) {
-        const Desc q2 = desc(i + 2 * nwarps);
-        const Lane l1 = lanes(i + nwarps, q1);
+    for (; i < end; i += step) {
+        const Desc q2 = desc(i + 2 * step);
+        const Lane l1 = lanes(i + step, q1);
         const int c = chunk_of(i);
         const int64_t base = q0.cp + lane;
         const int clen = q0.d & kSellLenMask;

@@ -99,6 +99,7 @@ struct pepp_spmv_plan_s {
     int* d_soff = nullptr;           // stencil-chunk slot offsets
     int64_t sell_stencil_chunks = 0;
     int sell_cpw = 1;            // chunks per σ window (chunk order is transposed when > 1)
+    int* d_sell_ws = nullptr;    // σ > 1: per-warp ranges of the transposed chunk order, equal slots
     int64_t sell_col16_chunks = 0;
     void* d_sval = nullptr;
 
@@ -227,7 +228,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
-                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w};
+                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -251,6 +252,35 @@ int grid_for(const void* fn, int block, int64_t work_items, int items_per_block,
 }
 
 // ---------------------------------------------------------------- SELL prep
+// σ > 1: cut the transposed chunk order (the kernel's chunk_of) into one
+// contiguous range per warp of the grid with equal cost (slots + a per-chunk
+// overhead), so that the few long chunks of every window do not pile up on
+// the warps a cyclic stride would hand them to.
+pepp_status_t sell_warp_ranges(pepp_spmv_plan_t* p) {
+    const int nc = p->nchunks, cpw = p->sell_cpw;
+    const int W = p->grid_sell * (kBlock / 32);
+    std::vector<int> len(nc > 0 ? nc : 1);
+    if (nc > 0) PEPP_CUDA_TRY(cudaMemcpy(len.data(), p->d_chunk_len, sizeof(int) * nc, cudaMemcpyDeviceToHost));
+    const int nwin = nc / cpw, nfull = nwin * cpw;
+    auto chunk_of = [&](int i) { return i < nfull ? (i % nwin) * cpw + i / nwin : i; };
+    int64_t kChunkOverhead = 4;   // descriptor + per-lane loads + y store, in slot-equivalents
+    if (const char* e = std::getenv("PEPP_SELL_CHUNK_COST")) kChunkOverhead = std::atoi(e);   // experiments only
+    int64_t total = 0;
+    for (int i = 0; i < nc; ++i) total += (len[chunk_of(i)] & pepp::k::kSellLenMask) + kChunkOverhead;
+    std::vector<int> ws(W + 1, nc);
+    ws[0] = 0;
+    int64_t acc = 0;
+    int w = 1;
+    for (int i = 0; i < nc && w < W; ++i) {
+        acc += (len[chunk_of(i)] & pepp::k::kSellLenMask) + kChunkOverhead;
+        while (w < W && acc * W >= total * w) ws[w++] = i + 1;
+    }
+    pepp_status_t s;
+    if ((s = dalloc(p, &p->d_sell_ws, W + 1))) return s;
+    PEPP_CUDA_TRY(cudaMemcpy(p->d_sell_ws, ws.data(), sizeof(int) * (W + 1), cudaMemcpyHostToDevice));
+    return PEPP_OK;
+}
+
 pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     const int n = (int)p->nrows;
     p->nchunks = (n + 31) / 32;
@@ -530,11 +560,11 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
         if (p->d_perm)
             pepp::k::sell_kernel<kBlock, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
-                p->d_scol16, p->d_soff, (const T*)p->d_sval, x, y, p->sell_cpw);
+                p->d_scol16, p->d_soff, (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws);
         else
             pepp::k::sell_kernel<kBlock, false, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr, p->d_scol,
-                p->d_scol16, p->d_soff, (const T*)p->d_sval, x, y, 1);
+                p->d_scol16, p->d_soff, (const T*)p->d_sval, x, y, 1, nullptr);
         break;
     default:
         return PEPP_E_INVALID;
@@ -1049,6 +1079,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         // more (shorter-lived) blocks instead
         const int64_t cap = need >= 16 * wave ? wave : 4 * wave;
         p->grid_sell = (int)std::max<int64_t>(1, std::min<int64_t>(need, cap));
+        if (p->d_perm && (s = sell_warp_ranges(p))) return s;
     }
 
     // ---- history ----
