@@ -440,6 +440,16 @@ uint64_t pepp_context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, 
    (NCCL is loaded on demand with dlopen; PEPP_E_NCCL if unavailable). */
 pepp_status_t pepp_nccl_unique_id(void* id_out);
 
+/* NCCL self-test on `device` (-1 = current): a one-rank communicator runs
+   every NCCL call the partitioned path makes — grouped ncclSend/ncclRecv to
+   itself (int32, int64, fp32, fp64), in-place ncclBroadcast, ncclAllReduce
+   (max) — and checks the bytes that arrive. Verifies that the NCCL found at
+   run time (dlopen: PEPP_NCCL_LIB, else the copy already loaded, else the
+   system one) matches the calling convention this library was built against.
+   PEPP_OK, PEPP_E_NCCL (unavailable, an NCCL error, or wrong data), or
+   PEPP_E_CUDA. Synchronous; allocates and frees its own buffers. */
+pepp_status_t pepp_nccl_selftest(int32_t device);
+
 /* ABI version (PEPP_ABI_VERSION) of the loaded library. */
 int32_t pepp_abi_version(void);
 

@@ -406,3 +406,9 @@ def nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     C.check(C.lib().pepp_nccl_unique_id(ctypes.addressof(buf)), "pepp_nccl_unique_id")
     return buf.raw
+
+
+def nccl_selftest(device: int = -1) -> None:
+    """Run every NCCL call of the partitioned path on a one-rank communicator
+    and check the data (pepp_nccl_selftest); raises PeppError on mismatch."""
+    C.check(C.lib().pepp_nccl_selftest(device), "pepp_nccl_selftest")

@@ -104,6 +104,7 @@ SIGNATURES = {
     "pepp_history_load": (c_i32, [c_vp, ctypes.c_char_p]),
     "pepp_context_key": (c_u64, [c_i64, c_i64, c_i64, c_f64, c_i32]),
     "pepp_nccl_unique_id": (c_i32, [c_vp]),
+    "pepp_nccl_selftest": (c_i32, [c_i32]),
     "pepp_abi_version": (c_i32, []),
 }
 

@@ -152,3 +152,19 @@ def test_two_ranks_one_gpu_fp32(name, exchange):
     out = _run(name, exchange, K=3, f32=True)
     for r in range(2):
         assert out[r]["iter"] and out[r]["host"], (r, out[r])
+
+
+def test_real_nccl_selftest():
+    """The REAL NCCL (torch's libnccl, found by dlopen RTLD_NOLOAD) driven by
+    the library's own function table: grouped self send/recv in all four
+    value types, in-place broadcast, max all-reduce — data checked. One GPU
+    cannot host a multi-rank NCCL communicator; this pins the calling
+    convention the multi-GPU exchange relies on."""
+    import torch
+    import paper_conf_sc_dastgeerlk12_b200 as pepp
+    assert "PEPP_NCCL_LIB" not in os.environ
+    torch.cuda.init()
+    pepp.nccl_selftest(0)
+    with open("/proc/self/maps") as f:
+        maps = f.read()
+    assert "libnccl" in maps and "fake_nccl" not in maps
