@@ -290,7 +290,8 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     # plan is built with that variant only
     plan = pepp.Plan.from_csr(A, nranks=world, rank=rank, row_bounds=bounds if world > 1 else None,
                               nccl_unique_id=uid, prune=not args.no_prune,
-                              variant_mask=(1 << force.variant) if force is not None else 0)
+                              variant_mask=(1 << force.variant) if force is not None else 0,
+                              compress_values=not args.no_value_compression)
     info = plan.info()
     flags = pepp.Y_NEXT_INPUT if iterated else pepp.Y_LOCAL
     overlapped = bool(world > 1 and iterated and force is None and info["overlap"])
@@ -463,6 +464,8 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
 
     if rank == 0:
         kname = chosen
+        if kname.startswith("sell") and info["sell_constval_frac"] > 0:
+            kname += "+constval"   # value-compressed layout: its own ncu traffic entry
         line = {
             "metric": "SpMV GFLOP/s (aggregate over ranks); achieved HBM GB/s in 'hbm'",
             "value": round(gflops, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
@@ -487,6 +490,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             "clocks": clk,
             "cpu_baseline": cpu,
             "plan": {k: info[k] for k in ("mean_row", "cv_row", "max_row", "sell_sigma", "sell_fill",
+                                          "sell_stencil_frac", "sell_constval_frac", "sell_col16_frac",
                                           "device_bytes", "halo_recv", "halo_send", "overlap",
                                           "overlap_head", "overlap_tail")},
             "choices": used_count,
@@ -507,6 +511,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-prune", action="store_true", help="every variant is a candidate (no static narrowing)")
+    ap.add_argument("--no-value-compression", action="store_true",
+                    help="stream every stored SELL value (opts.compress_values = 0)")
     ap.add_argument("--dtype", choices=["f64", "f32"], default="f64",
                     help="f64 = BASELINE's precision (default); f32 = the paper's float instance")
     args = ap.parse_args()

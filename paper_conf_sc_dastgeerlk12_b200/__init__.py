@@ -91,7 +91,7 @@ class Plan:
                  nranks: int = 1, rank: int = 0, row_bounds: Optional[Sequence[int]] = None,
                  nccl_unique_id: Optional[bytes] = None, exchange: int = X_AUTO,
                  history_path: Optional[str] = None, prune: bool = True, overlap: bool = True,
-                 predict=None):
+                 predict=None, compress_values: bool = True):
         L = C.lib()
         self._h = ctypes.c_void_p()
         on_dev = not isinstance(row_ptr, np.ndarray)
@@ -131,6 +131,7 @@ class Plan:
         o.history_path = self._hp
         o.prune = 1 if prune else 0
         o.overlap = 1 if overlap else 0
+        o.compress_values = 1 if compress_values else 0
         cb = None
         if predict is not None:
             # predict(context: dict, variant: int, param: int) -> µs (<= 0: no prediction);

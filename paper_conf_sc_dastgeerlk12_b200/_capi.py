@@ -37,7 +37,8 @@ class INFO_T(ctypes.Structure):
                 ("sell_fill", c_f64), ("device_bytes", c_i64), ("algorithmic_bytes", c_i64),
                 ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64),
                 ("prior_key", c_u64), ("sell_stencil_frac", c_f64),
-                ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64), ("predicted", c_i32)]
+                ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64), ("predicted", c_i32),
+                ("sell_constval_frac", c_f64)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -52,7 +53,8 @@ class OPTS_T(ctypes.Structure):
                 ("device", c_i32), ("min_samples", c_i32), ("sample_period", c_i32), ("nranks", c_i32),
                 ("rank", c_i32), ("row_bounds", c_vp), ("nccl_comm", c_vp), ("nccl_unique_id", c_vp),
                 ("exchange", c_i32), ("history_path", ctypes.c_char_p), ("prune", c_i32),
-                ("overlap", c_i32), ("predict", PREDICT_FN), ("predict_user", c_vp)]
+                ("overlap", c_i32), ("predict", PREDICT_FN), ("predict_user", c_vp),
+                ("compress_values", c_i32)]
 
 
 class CHOICE_T(ctypes.Structure):
@@ -117,6 +119,9 @@ class PeppError(RuntimeError):
         super().__init__(f"{where}: {status_str(status)} ({status})")
 
 
+ABI_VERSION = 2   # PEPP_ABI_VERSION of include/pepp_spmv.h
+
+
 def lib() -> ctypes.CDLL:
     global _lib
     if _lib is None:
@@ -127,6 +132,9 @@ def lib() -> ctypes.CDLL:
             f = getattr(L, name)
             f.restype = res
             f.argtypes = args
+        if L.pepp_abi_version() != ABI_VERSION:   # the structs below mirror one header version
+            raise ImportError(f"{LIB_PATH} has ABI {L.pepp_abi_version()}, the binding expects {ABI_VERSION}: "
+                              "rebuild with `python build.py`")
         _lib = L
     return _lib
 

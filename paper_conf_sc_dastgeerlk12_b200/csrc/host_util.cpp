@@ -51,6 +51,7 @@ extern "C" PEPP_API void pepp_spmv_opts_default(pepp_spmv_opts_t* o) {
     o->history_path = nullptr;
     o->prune = 1;
     o->overlap = 1;
+    o->compress_values = 1;
 }
 
 // ---------------------------------------------------------------- partition

@@ -97,6 +97,8 @@ struct pepp_spmv_plan_s {
     int* d_scol = nullptr;
     int16_t* d_scol16 = nullptr;
     int* d_soff = nullptr;           // stencil-chunk slot offsets
+    void* d_sconst = nullptr;        // constant-value stencil chunks: one value per slot (value type)
+    int64_t sell_const_chunks = 0;
     int64_t sell_stencil_chunks = 0;
     int sell_cpw = 1;            // chunks per σ window (chunk order is transposed when > 1)
     int* d_sell_ws = nullptr;    // σ > 1: per-warp ranges of the transposed chunk order, equal slots
@@ -228,7 +230,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
-                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws};
+                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_sconst};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -352,17 +354,29 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     // stencil chunks: one offset per slot for the whole chunk (no column stream)
     {
         if ((s = dalloc(p, &p->d_soff, p->sell_slots / 32 + 8))) return s;
+        const int64_t nconst_slots = p->sell_slots / 32 + 8;
+        if (p->opts.compress_values && (s = dalloc_bytes(p, &p->d_sconst, nconst_slots * (int64_t)p->esz))) return s;
         DevTmp<unsigned long long> d_nst;
-        PEPP_CUDA_TRY(d_nst.alloc(1));
-        PEPP_CUDA_TRY(cudaMemsetAsync(d_nst.p, 0, sizeof(unsigned long long), st));
+        PEPP_CUDA_TRY(d_nst.alloc(2));
+        PEPP_CUDA_TRY(cudaMemsetAsync(d_nst.p, 0, 2 * sizeof(unsigned long long), st));
         const int wb = 256, wg = (int)(((int64_t)p->nchunks * 32 + wb - 1) / wb);
-        pepp::k::sell_stencil_kernel<<<wg, wb, 0, st>>>(n, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_perm,
-                                                         p->d_scol, p->d_soff, d_nst.p);
+        if (p->vt == PEPP_VALUE_F32)
+            pepp::k::sell_stencil_kernel<float><<<wg, wb, 0, st>>>(n, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_perm,
+                p->d_scol, p->d_soff, d_nst.p, (const float*)p->d_sval, (float*)p->d_sconst, d_nst.p + 1);
+        else
+            pepp::k::sell_stencil_kernel<double><<<wg, wb, 0, st>>>(n, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_perm,
+                p->d_scol, p->d_soff, d_nst.p, (const double*)p->d_sval, (double*)p->d_sconst, d_nst.p + 1);
         PEPP_CUDA_TRY(cudaGetLastError());
-        unsigned long long nst = 0;
-        PEPP_CUDA_TRY(cudaMemcpyAsync(&nst, d_nst.p, sizeof(nst), cudaMemcpyDeviceToHost, st));
+        unsigned long long nst[2] = {0, 0};
+        PEPP_CUDA_TRY(cudaMemcpyAsync(nst, d_nst.p, sizeof(nst), cudaMemcpyDeviceToHost, st));
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-        p->sell_stencil_chunks = (int64_t)nst;
+        p->sell_stencil_chunks = (int64_t)nst[0];
+        p->sell_const_chunks = (int64_t)nst[1];
+        if (p->d_sconst && nst[1] == 0) {
+            cudaFree(p->d_sconst);
+            p->d_sconst = nullptr;
+            p->dev_bytes -= nconst_slots * (int64_t)p->esz;
+        }
     }
     // 16-bit column deltas where a whole chunk allows them (banded / stencil
     // structure): 2 instead of 4 bytes of index per stored slot
@@ -387,6 +401,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->info.sell_sigma = sigma;
     p->info.sell_col16_frac = p->nchunks ? (double)p->sell_col16_chunks / (double)p->nchunks : 0.0;
     p->info.sell_stencil_frac = p->nchunks ? (double)p->sell_stencil_chunks / (double)p->nchunks : 0.0;
+    p->info.sell_constval_frac = p->nchunks ? (double)p->sell_const_chunks / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
     return PEPP_OK;
 }
@@ -560,11 +575,11 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
         if (p->d_perm)
             pepp::k::sell_kernel<kBlock, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
-                p->d_scol16, p->d_soff, (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws);
+                p->d_scol16, p->d_soff, (const T*)p->d_sconst, (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws);
         else
             pepp::k::sell_kernel<kBlock, false, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr, p->d_scol,
-                p->d_scol16, p->d_soff, (const T*)p->d_sval, x, y, 1, nullptr);
+                p->d_scol16, p->d_soff, (const T*)p->d_sconst, (const T*)p->d_sval, x, y, 1, nullptr);
         break;
     default:
         return PEPP_E_INVALID;
@@ -1051,6 +1066,8 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         p->cands.push_back({PEPP_V_MERGE_PATH, kMergeIPT});
         p->cands.push_back({PEPP_V_MERGE_PATH, kMergeWarpParam});
     }
+    if (I.max_row > pepp::k::kSellLenMask) mask &= ~(1u << PEPP_V_SELL);   // chunk length field width
+    if ((mask & ((1u << PEPP_V_COUNT) - 1)) == 0) return PEPP_E_UNSUPPORTED;
     if (mask & (1u << PEPP_V_SELL)) {
         if ((s = prepare_sell(p, st))) return s;
         p->cands.push_back({PEPP_V_SELL, p->sell_sigma});

@@ -353,6 +353,47 @@ def test_exchange_is_noop_unpartitioned():
         assert torch.all(y == 0)
 
 
+def _sell_y(A, x, compress):
+    with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_SELL, prune=False, compress_values=compress) as plan:
+        y, u = _run(plan, x)
+        return y, plan.info()
+
+
+def test_value_compression_lossless():
+    """opts.compress_values: stencil chunks whose every slot holds one
+    bitwise-identical value store it once; y is bit-identical to the streamed
+    layout (same products, same order), and chunks with any differing bit
+    (even +0.0 vs -0.0) stay streamed."""
+    A = gen.laplacian2d(200)                           # {4, -1}: constant coefficients
+    for x in (gen.vector(3, gen.INT8, A.ncols), gen.vector(4, gen.REAL, A.ncols)):
+        y1, i1 = _sell_y(A, x, True)
+        y0, i0 = _sell_y(A, x, False)
+        assert i1["sell_constval_frac"] >= 0.75 and i0["sell_constval_frac"] == 0.0
+        assert i1["sell_constval_frac"] <= i1["sell_stencil_frac"]
+        assert i1["device_bytes"] > i0["device_bytes"] - 1   # the value table is extra, never less
+        assert np.array_equal(y1.view(np.int64), y0.view(np.int64))
+        _check(A, x, y1, x.dtype == np.float64 and np.all(x == np.round(x)))
+    # random values: nothing to compress
+    B = gen.banded(20_000, 4, seed=5, val_mode=gen.INT4)
+    x = gen.vector(6, gen.INT8, B.ncols)
+    y1, i1 = _sell_y(B, x, True)
+    assert i1["sell_constval_frac"] == 0.0 and np.array_equal(y1, oracle.spmv(B, x))
+    # tridiagonal (+0.0, 2, +0.0) — explicit zeros — with one diagonal one ulp
+    # off and one -0.0 entry: exactly the two chunks holding them are streamed
+    n = 32 * 40
+    rows = [[(j, 0.0 if j != i else 2.0) for j in (i - 1, i, i + 1) if 0 <= j < n] for i in range(n)]
+    rows[37 + 32][1] = (37 + 32, 2.0000000000000004)
+    rows[5 * 32 + 3][0] = (5 * 32 + 2, -0.0)
+    C = _hand(n, n, rows)
+    x = gen.vector(7, gen.REAL, n)
+    y1, i1 = _sell_y(C, x, True)
+    y0, _ = _sell_y(C, x, False)
+    interior = 40 - 2                                  # first / last chunk hold the ragged boundary rows
+    assert i1["sell_constval_frac"] == pytest.approx((interior - 2) / 40)
+    assert np.array_equal(y1.view(np.int64), y0.view(np.int64))
+    _check(C, x, y1, False)
+
+
 def test_sell_col16_used_and_exact_on_stencils():
     """Stencil / banded chunks with identical column offsets in every lane are
     stored as per-chunk offsets (no column stream); the remaining chunks whose
