@@ -177,10 +177,12 @@ typedef struct {
     void* predict_user;       /* passed to predict; borrowed, used only during pepp_spmv_plan */
     int32_t compress_values;  /* 1 (default) = value compression in the SELL layout: a stencil chunk
                                  (32 rows sharing their column offsets) whose every slot holds one
-                                 bitwise-identical value for all 32 rows stores that value once
-                                 (constant-coefficient stencils, unweighted graphs). Lossless: the
-                                 same products and sums in the same order (bit-identical y); only the
-                                 bytes read change. 0 = every stored slot's value is streamed. */
+                                 bitwise-identical value for all 32 rows becomes an id into a small
+                                 per-plan pattern table (<= 32 patterns of <= 8 slots, passed to the
+                                 kernel by value): the chunk then reads only x and writes y
+                                 (constant-coefficient stencils). Lossless: the same products and
+                                 sums in the same order (bit-identical y); only the bytes read
+                                 change. 0 = every stored slot's value is streamed. */
 } pepp_spmv_opts_t;
 
 /* Selection result. `candidate` indexes pepp_spmv_candidates(). The plan's
@@ -222,7 +224,7 @@ typedef struct pepp_plan_info_s {
     int64_t overlap_head;     /* rows [0, overlap_head) and [nrows - overlap_tail, nrows) are computed */
     int64_t overlap_tail;     /*   before the exchange starts (0 / 0 when overlap == 0) */
     int32_t predicted;        /* candidates with a prediction from opts.predict (0 = none / no function) */
-    double sell_constval_frac;/* fraction of SELL chunks stored value-compressed (one value per slot) */
+    double sell_constval_frac;/* fraction of SELL chunks stored as a pattern-table id (compress_values) */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

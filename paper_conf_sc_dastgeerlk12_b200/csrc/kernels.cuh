@@ -206,33 +206,28 @@ __global__ void __launch_bounds__(BLOCK) csr_vector_kernel(int nrows, const int*
 constexpr int kSellMasked = 1 << 30;
 constexpr int kSellCol16 = 1 << 29;
 constexpr int kSellStencil = 1 << 28;
-constexpr int kSellConstVal = 1 << 27;   // stencil chunk whose every slot holds one value for all 32 rows
+constexpr int kSellPattern = 1 << 27;    // chunk = one entry of the plan's pattern table (offsets + values)
 constexpr int kSellLenMask = (1 << 27) - 1;
-enum { kIdx32 = 0, kIdx16 = 1, kIdxStencil = 2, kIdxStencilConst = 3 };
+enum { kIdx32 = 0, kIdx16 = 1, kIdxStencil = 2 };
 
 // N slots of one chunk, loads issued unconditionally (all N exist for every
 // lane) before the first FMA; the per-lane row length only masks the FMA.
 // IDX: kIdx32 columns; kIdx16 int16 deltas from the lane's row index `row0`;
-// kIdxStencil one offset per slot for the whole chunk (lane j's `offl`);
-// kIdxStencilConst additionally one value per slot (lane j's `vall`): no
-// value stream at all (value compression of constant-coefficient stencils).
+// kIdxStencil one offset per slot for the whole chunk (lane j's `offl`).
 template <int N, int IDX, typename T>
 __device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __restrict__ col,
-                                        const int16_t* __restrict__ col16, int offl, T vall,
+                                        const int16_t* __restrict__ col16, int offl,
                                         int row0, const T* __restrict__ x, int64_t base, int j0,
                                         int len, T acc, uint64_t pol) {
-    constexpr bool kStencil = IDX == kIdxStencil || IDX == kIdxStencilConst;
     T v[N];
     int c[N];
 #pragma unroll
     for (int u = 0; u < N; ++u)
-        c[u] = kStencil      ? row0 + __shfl_sync(0xffffffffu, offl, j0 + u)   // lane j holds slot j's offset
-             : IDX == kIdx16 ? row0 + ld_stream_i16(col16 + base + (int64_t)(j0 + u) * 32, pol)
-                             : ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
+        c[u] = IDX == kIdxStencil ? row0 + __shfl_sync(0xffffffffu, offl, j0 + u)   // lane j holds slot j's offset
+             : IDX == kIdx16      ? row0 + ld_stream_i16(col16 + base + (int64_t)(j0 + u) * 32, pol)
+                                  : ld_stream_i(col + base + (int64_t)(j0 + u) * 32, pol);
 #pragma unroll
-    for (int u = 0; u < N; ++u)
-        v[u] = IDX == kIdxStencilConst ? __shfl_sync(0xffffffffu, vall, j0 + u)   // lane j holds slot j's value
-                                       : ld_stream_v(val + base + (int64_t)(j0 + u) * 32, pol);
+    for (int u = 0; u < N; ++u) v[u] = ld_stream_v(val + base + (int64_t)(j0 + u) * 32, pol);
     T xv[N];
 #pragma unroll
     for (int u = 0; u < N; ++u) xv[u] = ld_x(x, c[u]);
@@ -244,23 +239,68 @@ __device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __
 
 template <int IDX, typename T>
 __device__ __forceinline__ T sell_chunk(const T* __restrict__ val, const int* __restrict__ col,
-                                        const int16_t* __restrict__ col16, int offl, T vall, int row0,
+                                        const int16_t* __restrict__ col16, int offl, int row0,
                                         const T* __restrict__ x, int64_t base, int clen, int len, uint64_t pol) {
     T acc = T(0);
     int j = 0;
     // whole blocks of 8 slots, then one exactly-sized tail (warp-uniform switch)
-    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, IDX, T>(val, col, col16, offl, vall, row0, x, base, j, len, acc, pol);
+    for (; j + 8 <= clen; j += 8) acc = sell_slots<8, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol);
     switch (clen - j) {
-    case 1: acc = sell_slots<1, IDX, T>(val, col, col16, offl, vall, row0, x, base, j, len, acc, pol); break;
-    case 2: acc = sell_slots<2, IDX, T>(val, col, col16, offl, vall, row0, x, base, j, len, acc, pol); break;
-    case 3: acc = sell_slots<3, IDX, T>(val, col, col16, offl, vall, row0, x, base, j, len, acc, pol); break;
-    case 4: acc = sell_slots<4, IDX, T>(val, col, col16, offl, vall, row0, x, base, j, len, acc, pol); break;
-    case 5: acc = sell_slots<5, IDX, T>(val, col, col16, offl, vall, row0, x, base, j, len, acc, pol); break;
-    case 6: acc = sell_slots<6, IDX, T>(val, col, col16, offl, vall, row0, x, base, j, len, acc, pol); break;
-    case 7: acc = sell_slots<7, IDX, T>(val, col, col16, offl, vall, row0, x, base, j, len, acc, pol); break;
+    case 1: acc = sell_slots<1, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 2: acc = sell_slots<2, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 3: acc = sell_slots<3, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 4: acc = sell_slots<4, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 5: acc = sell_slots<5, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 6: acc = sell_slots<6, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
+    case 7: acc = sell_slots<7, IDX, T>(val, col, col16, offl, row0, x, base, j, len, acc, pol); break;
     default: break;
     }
     return acc;
+}
+
+// Pattern table (value + index compression): chunks whose 32 rows share
+// their column offsets AND whose every slot holds one bitwise-identical value
+// (constant-coefficient stencils) are stored as an id into this table, passed
+// by value as a kernel parameter (constant bank: uniform LDC reads, no
+// memory stream). The chunk reads only x and writes y.
+constexpr int kSellMaxPatterns = 32;
+constexpr int kSellMaxPatternLen = 8;
+template <typename T>
+struct SellPatterns {
+    int len[kSellMaxPatterns];
+    int off[kSellMaxPatterns][kSellMaxPatternLen];
+    T val[kSellMaxPatterns][kSellMaxPatternLen];
+};
+
+template <int N, typename T>
+__device__ __forceinline__ T sell_pattern_slots(const SellPatterns<T>& pt, int pid, int row0,
+                                                const T* __restrict__ x) {
+    int c[N];
+    T xv[N];
+#pragma unroll
+    for (int u = 0; u < N; ++u) c[u] = row0 + pt.off[pid][u];
+#pragma unroll
+    for (int u = 0; u < N; ++u) xv[u] = ld_x(x, c[u]);
+    T acc = T(0);
+#pragma unroll
+    for (int u = 0; u < N; ++u) acc = fma(pt.val[pid][u], xv[u], acc);   // slot order = the row's CSR order
+    return acc;
+}
+
+template <typename T>
+__device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int pid, int row0,
+                                                const T* __restrict__ x) {
+    switch (pt.len[pid]) {
+    case 1: return sell_pattern_slots<1, T>(pt, pid, row0, x);
+    case 2: return sell_pattern_slots<2, T>(pt, pid, row0, x);
+    case 3: return sell_pattern_slots<3, T>(pt, pid, row0, x);
+    case 4: return sell_pattern_slots<4, T>(pt, pid, row0, x);
+    case 5: return sell_pattern_slots<5, T>(pt, pid, row0, x);
+    case 6: return sell_pattern_slots<6, T>(pt, pid, row0, x);
+    case 7: return sell_pattern_slots<7, T>(pt, pid, row0, x);
+    case 8: return sell_pattern_slots<8, T>(pt, pid, row0, x);
+    default: return T(0);
+    }
 }
 
 template <int BLOCK, bool SORTED, typename T>
@@ -271,7 +311,7 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
                                                      const int* __restrict__ col,
                                                      const int16_t* __restrict__ col16,
                                                      const int* __restrict__ soff,
-                                                     const T* __restrict__ sconst,
+                                                     const __grid_constant__ SellPatterns<T> pt,
                                                      const T* __restrict__ val,
                                                      const T* __restrict__ x,
                                                      T* __restrict__ y,
@@ -301,7 +341,7 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     // lane j loads slot j's offset once, broadcast later with shuffles) and
     // chunk i+2's descriptor (length/flags, slot pointer) are in flight.
     struct Desc { int d; int64_t cp; };
-    struct Lane { int len; int orow; int offl; T vall; };
+    struct Lane { int len; int orow; int offl; };
     int i = warp, end = nchunks, step = nwarps;
     if (SORTED) { i = __ldg(wstart + warp); end = __ldg(wstart + warp + 1); step = 1; }
     auto desc = [&](int i) -> Desc {
@@ -310,16 +350,13 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
         return q;
     };
     auto lanes = [&](int i, const Desc& q) -> Lane {
-        Lane l{0, 0, 0, T(0)};
+        Lane l{0, 0, 0};
         if (i >= end) return l;
         const int c = chunk_of(i);
         const int r = c * 32 + lane;
         l.len = !(q.d & kSellMasked) ? (q.d & kSellLenMask) : (r < nrows ? __ldg(rowlen + r) : 0);
         l.orow = (SORTED && r < nrows) ? __ldg(perm + r) : r;
-        if ((q.d & kSellStencil) && lane < (q.d & kSellLenMask)) {
-            l.offl = __ldg(soff + (q.cp >> 5) + lane);
-            if (q.d & kSellConstVal) l.vall = __ldg(sconst + (q.cp >> 5) + lane);
-        }
+        if ((q.d & kSellStencil) && lane < (q.d & kSellLenMask)) l.offl = __ldg(soff + (q.cp >> 5) + lane);
         return l;
     };
     Desc q0 = desc(i), q1 = desc(i + step);
@@ -331,10 +368,10 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
         const int64_t base = q0.cp + lane;
         const int clen = q0.d & kSellLenMask;
         T acc;
-        if (q0.d & kSellConstVal) acc = sell_chunk<kIdxStencilConst, T>(val, col, col16, l0.offl, l0.vall, l0.orow, x, base, clen, l0.len, pol);
-        else if (q0.d & kSellStencil) acc = sell_chunk<kIdxStencil, T>(val, col, col16, l0.offl, T(0), l0.orow, x, base, clen, l0.len, pol);
-        else if (q0.d & kSellCol16) acc = sell_chunk<kIdx16, T>(val, col, col16, 0, T(0), l0.orow, x, base, clen, l0.len, pol);
-        else acc = sell_chunk<kIdx32, T>(val, col, col16, 0, T(0), l0.orow, x, base, clen, l0.len, pol);
+        if (q0.d & kSellPattern) acc = sell_pattern_chunk<T>(pt, (int)q0.cp, l0.orow, x);   // cp holds the pattern id
+        else if (q0.d & kSellStencil) acc = sell_chunk<kIdxStencil, T>(val, col, col16, l0.offl, l0.orow, x, base, clen, l0.len, pol);
+        else if (q0.d & kSellCol16) acc = sell_chunk<kIdx16, T>(val, col, col16, 0, l0.orow, x, base, clen, l0.len, pol);
+        else acc = sell_chunk<kIdx32, T>(val, col, col16, 0, l0.orow, x, base, clen, l0.len, pol);
         if (c * 32 + lane < nrows) y[l0.orow] = acc;
         q0 = q1; q1 = q2; l0 = l1;
     }
@@ -927,7 +964,7 @@ __global__ void sell_col16_kernel(int nrows, int nchunks, const int64_t* __restr
     const int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (c >= nchunks) return;
     const int d = chunk_len[c];
-    if (d & kSellStencil) return;       // already needs no column stream
+    if (d & (kSellStencil | kSellPattern)) return;   // already needs no column stream
     const int clen = d & kSellLenMask;
     const int r = c * 32 + lane;
     const int len = r < nrows ? rowlen[r] : 0;
@@ -960,7 +997,7 @@ __global__ void sell_stencil_kernel(int nrows, int nchunks, const int64_t* __res
                                     const int* __restrict__ col, int* __restrict__ soff,
                                     unsigned long long* __restrict__ nst,
                                     const T* __restrict__ val, T* __restrict__ sconst,
-                                    unsigned long long* __restrict__ nconst) {
+                                    unsigned char* __restrict__ cflag, unsigned long long* __restrict__ nconst) {
     const int lane = threadIdx.x & 31;
     const int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (c >= nchunks) return;
@@ -986,10 +1023,13 @@ __global__ void sell_stencil_kernel(int nrows, int nchunks, const int64_t* __res
         const T v = val[base + (int64_t)j * 32];
         cval = __all_sync(0xffffffffu, bits_equal(v, __shfl_sync(0xffffffffu, v, 0)));
     }
+    // constant chunk: cflag[c] = 1 and sconst[sb + j] = slot j's value (the
+    // plan dedupes (offsets, values) into its pattern table on the host)
     if (cval)
         for (int j = lane; j < clen; j += 32) sconst[sb + j] = val[chunk_ptr[c] + (int64_t)j * 32];
+    if (cflag && lane == 0) cflag[c] = cval ? 1 : 0;
     if (lane == 0) {
-        chunk_len[c] = d | kSellStencil | (cval ? kSellConstVal : 0);
+        chunk_len[c] = d | kSellStencil;
         atomicAdd(nst, 1ull);
         if (cval) atomicAdd(nconst, 1ull);
     }

@@ -97,8 +97,9 @@ struct pepp_spmv_plan_s {
     int* d_scol = nullptr;
     int16_t* d_scol16 = nullptr;
     int* d_soff = nullptr;           // stencil-chunk slot offsets
-    void* d_sconst = nullptr;        // constant-value stencil chunks: one value per slot (value type)
-    int64_t sell_const_chunks = 0;
+    int64_t sell_const_chunks = 0;   // chunks stored as a pattern-table id (value + index compression)
+    pepp::k::SellPatterns<double> pat64{};   // the pattern table, passed by value to the SELL kernel
+    pepp::k::SellPatterns<float> pat32{};
     int64_t sell_stencil_chunks = 0;
     int sell_cpw = 1;            // chunks per σ window (chunk order is transposed when > 1)
     int* d_sell_ws = nullptr;    // σ > 1: per-warp ranges of the transposed chunk order, equal slots
@@ -230,7 +231,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
-                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_sconst};
+                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -280,6 +281,57 @@ pepp_status_t sell_warp_ranges(pepp_spmv_plan_t* p) {
     pepp_status_t s;
     if ((s = dalloc(p, &p->d_sell_ws, W + 1))) return s;
     PEPP_CUDA_TRY(cudaMemcpy(p->d_sell_ws, ws.data(), sizeof(int) * (W + 1), cudaMemcpyHostToDevice));
+    return PEPP_OK;
+}
+
+// Value + index compression: constant stencil chunks (cflag) with the same
+// (length, offsets, value bits) become one entry of the pattern table; the
+// chunk keeps its length, trades kSellStencil for kSellPattern, and its
+// chunk_ptr entry becomes the pattern id. At most kSellMaxPatterns patterns
+// of at most kSellMaxPatternLen slots; other chunks stay as they are.
+template <typename T>
+pepp_status_t sell_patterns(pepp_spmv_plan_t* p, int64_t nsb, const void* d_sconst, const unsigned char* d_cflag,
+                            pepp::k::SellPatterns<T>* pt) {
+    using pepp::k::kSellLenMask;
+    const int nc = p->nchunks;
+    std::vector<unsigned char> cflag(nc);
+    std::vector<int> clen(nc), soff(nsb);
+    std::vector<int64_t> cp(nc + 1);
+    std::vector<T> sval(nsb);
+    PEPP_CUDA_TRY(cudaMemcpy(cflag.data(), d_cflag, nc, cudaMemcpyDeviceToHost));
+    PEPP_CUDA_TRY(cudaMemcpy(clen.data(), p->d_chunk_len, sizeof(int) * nc, cudaMemcpyDeviceToHost));
+    PEPP_CUDA_TRY(cudaMemcpy(cp.data(), p->d_chunk_ptr, sizeof(int64_t) * (nc + 1), cudaMemcpyDeviceToHost));
+    PEPP_CUDA_TRY(cudaMemcpy(soff.data(), p->d_soff, sizeof(int) * nsb, cudaMemcpyDeviceToHost));
+    PEPP_CUDA_TRY(cudaMemcpy(sval.data(), d_sconst, sizeof(T) * nsb, cudaMemcpyDeviceToHost));
+    *pt = pepp::k::SellPatterns<T>{};
+    int npat = 0;
+    int64_t used = 0;
+    for (int c = 0; c < nc; ++c) {
+        if (!cflag[c]) continue;
+        const int len = clen[c] & kSellLenMask;
+        if (len < 1 || len > pepp::k::kSellMaxPatternLen) continue;
+        const int64_t sb = cp[c] >> 5;
+        int pid = -1;
+        for (int q = 0; q < npat && pid < 0; ++q) {
+            bool same = pt->len[q] == len;
+            for (int j = 0; same && j < len; ++j)
+                same = pt->off[q][j] == soff[sb + j] && std::memcmp(&pt->val[q][j], &sval[sb + j], sizeof(T)) == 0;
+            if (same) pid = q;
+        }
+        if (pid < 0) {
+            if (npat == pepp::k::kSellMaxPatterns) continue;
+            pid = npat++;
+            pt->len[pid] = len;
+            for (int j = 0; j < len; ++j) { pt->off[pid][j] = soff[sb + j]; pt->val[pid][j] = sval[sb + j]; }
+        }
+        clen[c] = (clen[c] & ~pepp::k::kSellStencil) | pepp::k::kSellPattern;
+        cp[c] = pid;
+        ++used;
+    }
+    if (!used) return PEPP_OK;
+    PEPP_CUDA_TRY(cudaMemcpy(p->d_chunk_len, clen.data(), sizeof(int) * nc, cudaMemcpyHostToDevice));
+    PEPP_CUDA_TRY(cudaMemcpy(p->d_chunk_ptr, cp.data(), sizeof(int64_t) * nc, cudaMemcpyHostToDevice));
+    p->sell_const_chunks = used;
     return PEPP_OK;
 }
 
@@ -354,28 +406,33 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     // stencil chunks: one offset per slot for the whole chunk (no column stream)
     {
         if ((s = dalloc(p, &p->d_soff, p->sell_slots / 32 + 8))) return s;
-        const int64_t nconst_slots = p->sell_slots / 32 + 8;
-        if (p->opts.compress_values && (s = dalloc_bytes(p, &p->d_sconst, nconst_slots * (int64_t)p->esz))) return s;
+        const int64_t nsb = p->sell_slots / 32 + 8;   // per-chunk slot tables are indexed by chunk_ptr / 32
+        DevTmp<double> d_sconst;                      // 8-byte slots hold either value type
+        DevTmp<unsigned char> d_cflag;
+        if (p->opts.compress_values) {
+            PEPP_CUDA_TRY(d_sconst.alloc(nsb));
+            PEPP_CUDA_TRY(d_cflag.alloc(p->nchunks));
+            PEPP_CUDA_TRY(cudaMemsetAsync(d_cflag.p, 0, p->nchunks, st));
+        }
         DevTmp<unsigned long long> d_nst;
         PEPP_CUDA_TRY(d_nst.alloc(2));
         PEPP_CUDA_TRY(cudaMemsetAsync(d_nst.p, 0, 2 * sizeof(unsigned long long), st));
         const int wb = 256, wg = (int)(((int64_t)p->nchunks * 32 + wb - 1) / wb);
         if (p->vt == PEPP_VALUE_F32)
             pepp::k::sell_stencil_kernel<float><<<wg, wb, 0, st>>>(n, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_perm,
-                p->d_scol, p->d_soff, d_nst.p, (const float*)p->d_sval, (float*)p->d_sconst, d_nst.p + 1);
+                p->d_scol, p->d_soff, d_nst.p, (const float*)p->d_sval, (float*)d_sconst.p, d_cflag.p, d_nst.p + 1);
         else
             pepp::k::sell_stencil_kernel<double><<<wg, wb, 0, st>>>(n, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_perm,
-                p->d_scol, p->d_soff, d_nst.p, (const double*)p->d_sval, (double*)p->d_sconst, d_nst.p + 1);
+                p->d_scol, p->d_soff, d_nst.p, (const double*)p->d_sval, d_sconst.p, d_cflag.p, d_nst.p + 1);
         PEPP_CUDA_TRY(cudaGetLastError());
         unsigned long long nst[2] = {0, 0};
         PEPP_CUDA_TRY(cudaMemcpyAsync(nst, d_nst.p, sizeof(nst), cudaMemcpyDeviceToHost, st));
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
         p->sell_stencil_chunks = (int64_t)nst[0];
-        p->sell_const_chunks = (int64_t)nst[1];
-        if (p->d_sconst && nst[1] == 0) {
-            cudaFree(p->d_sconst);
-            p->d_sconst = nullptr;
-            p->dev_bytes -= nconst_slots * (int64_t)p->esz;
+        if (nst[1] > 0) {
+            if (p->vt == PEPP_VALUE_F32) s = sell_patterns<float>(p, nsb, d_sconst.p, d_cflag.p, &p->pat32);
+            else s = sell_patterns<double>(p, nsb, d_sconst.p, d_cflag.p, &p->pat64);
+            if (s) return s;
         }
     }
     // 16-bit column deltas where a whole chunk allows them (banded / stencil
@@ -522,6 +579,10 @@ void launch_csr_vector(const pepp_spmv_plan_t* p, const T* x, T* y, cudaStream_t
                                                                         (const T*)p->d_val, x, y);
 }
 
+template <typename T> const pepp::k::SellPatterns<T>& sell_pattern_table(const pepp_spmv_plan_t* p);
+template <> const pepp::k::SellPatterns<double>& sell_pattern_table<double>(const pepp_spmv_plan_t* p) { return p->pat64; }
+template <> const pepp::k::SellPatterns<float>& sell_pattern_table<float>(const pepp_spmv_plan_t* p) { return p->pat32; }
+
 template <typename T>
 pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y, cudaStream_t st) {
     if (p->nrows == 0) return PEPP_OK;
@@ -575,11 +636,11 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
         if (p->d_perm)
             pepp::k::sell_kernel<kBlock, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
-                p->d_scol16, p->d_soff, (const T*)p->d_sconst, (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws);
+                p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws);
         else
             pepp::k::sell_kernel<kBlock, false, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr, p->d_scol,
-                p->d_scol16, p->d_soff, (const T*)p->d_sconst, (const T*)p->d_sval, x, y, 1, nullptr);
+                p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr);
         break;
     default:
         return PEPP_E_INVALID;
