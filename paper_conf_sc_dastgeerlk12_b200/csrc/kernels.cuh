@@ -316,11 +316,28 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
                                                      const T* __restrict__ x,
                                                      T* __restrict__ y,
                                                      int cpw,
-                                                     const int* __restrict__ wstart) {
+                                                     const int* __restrict__ wstart,
+                                                     const int* __restrict__ patlist, int npatc,
+                                                     const int* __restrict__ genlist) {
     const int lane = threadIdx.x & 31;
     const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
     const int nwarps = (gridDim.x * BLOCK) >> 5;
     const uint64_t pol = evict_first_policy();
+    // Phase A (σ = 1 plans with pattern chunks): the pattern chunks, listed
+    // as (chunk << 5 | pattern id), in a tight loop — no descriptor, no
+    // per-lane loads: 1 list entry (prefetched one step ahead), the x
+    // gathers, the FMAs and the y store per chunk. Phase B below then walks
+    // only the other chunks (`genlist`, `nchunks` of them).
+    if (!SORTED && npatc > 0) {
+        int k = warp;
+        int e = k < npatc ? __ldg(patlist + k) : 0;
+        for (; k < npatc; k += nwarps) {
+            const int en = k + nwarps < npatc ? __ldg(patlist + k + nwarps) : 0;
+            const int r = (e >> 5) * 32 + lane;
+            y[r] = sell_pattern_chunk<T>(pt, e & 31, r, x);
+            e = en;
+        }
+    }
     // chunk order: warp w walks i = w, w + nwarps, ...; chunk = i when the
     // chunks are uniform (σ = 1). When σ > 1 sorted the rows, chunk lengths
     // repeat a long-to-short pattern in every window of cpw = σ/32 chunks and
@@ -332,7 +349,7 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     const int nfull = SORTED ? (nchunks / cpw) * cpw : 0;
     const int nwin = SORTED ? nchunks / cpw : 1;
     auto chunk_of = [&](int i) -> int {
-        if (!SORTED) return i;
+        if (!SORTED) return genlist ? __ldg(genlist + i) : i;
         return i < nfull ? (i % nwin) * cpw + i / nwin : i;
     };
     // Two-deep software pipelining over the warp's chunks (latency-bound

@@ -98,6 +98,9 @@ struct pepp_spmv_plan_s {
     int16_t* d_scol16 = nullptr;
     int* d_soff = nullptr;           // stencil-chunk slot offsets
     int64_t sell_const_chunks = 0;   // chunks stored as a pattern-table id (value + index compression)
+    int* d_patlist = nullptr;        // σ = 1: pattern chunks as (chunk << 5 | id), phase A of the kernel
+    int* d_genlist = nullptr;        // σ = 1: the other chunks, phase B
+    int npatc = 0, ngen = 0;
     pepp::k::SellPatterns<double> pat64{};   // the pattern table, passed by value to the SELL kernel
     pepp::k::SellPatterns<float> pat32{};
     int64_t sell_stencil_chunks = 0;
@@ -231,7 +234,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
-                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws};
+                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -332,6 +335,22 @@ pepp_status_t sell_patterns(pepp_spmv_plan_t* p, int64_t nsb, const void* d_scon
     PEPP_CUDA_TRY(cudaMemcpy(p->d_chunk_len, clen.data(), sizeof(int) * nc, cudaMemcpyHostToDevice));
     PEPP_CUDA_TRY(cudaMemcpy(p->d_chunk_ptr, cp.data(), sizeof(int64_t) * nc, cudaMemcpyHostToDevice));
     p->sell_const_chunks = used;
+    if (!p->d_perm) {   // σ = 1: split the chunks into the kernel's two phases
+        std::vector<int> pat, gen;
+        pat.reserve(used);
+        gen.reserve(nc - used);
+        for (int c = 0; c < nc; ++c) {
+            if (clen[c] & pepp::k::kSellPattern) pat.push_back((c << 5) | (int)cp[c]);
+            else gen.push_back(c);
+        }
+        pepp_status_t s;
+        if ((s = dalloc(p, &p->d_patlist, (int64_t)pat.size()))) return s;
+        if ((s = dalloc(p, &p->d_genlist, (int64_t)gen.size()))) return s;
+        PEPP_CUDA_TRY(cudaMemcpy(p->d_patlist, pat.data(), sizeof(int) * pat.size(), cudaMemcpyHostToDevice));
+        if (!gen.empty()) PEPP_CUDA_TRY(cudaMemcpy(p->d_genlist, gen.data(), sizeof(int) * gen.size(), cudaMemcpyHostToDevice));
+        p->npatc = (int)pat.size();
+        p->ngen = (int)gen.size();
+    }
     return PEPP_OK;
 }
 
@@ -636,11 +655,13 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
         if (p->d_perm)
             pepp::k::sell_kernel<kBlock, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
-                p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws);
+                p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws,
+                nullptr, 0, nullptr);
         else
             pepp::k::sell_kernel<kBlock, false, T><<<p->grid_sell, kBlock, 0, st>>>(
-                (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr, p->d_scol,
-                p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr);
+                (int)p->nrows, p->d_patlist ? p->ngen : p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
+                p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
+                p->d_patlist, p->npatc, p->d_patlist ? p->d_genlist : nullptr);
         break;
     default:
         return PEPP_E_INVALID;
