@@ -287,6 +287,21 @@ __device__ __forceinline__ T sell_pattern_slots(const SellPatterns<T>& pt, int p
     return acc;
 }
 
+// Phase A form: the pattern's offsets / values already in registers (loaded
+// once per pattern change; reading the kernel-parameter table per chunk
+// would issue indexed LDCs, which run on the narrow ADU pipe).
+template <int N, typename T>
+__device__ __forceinline__ T sell_pattern_regs(const int (&o)[kSellMaxPatternLen], const T (&v)[kSellMaxPatternLen],
+                                               int row0, const T* __restrict__ x) {
+    T xv[N];
+#pragma unroll
+    for (int u = 0; u < N; ++u) xv[u] = ld_x(x, row0 + o[u]);
+    T acc = T(0);
+#pragma unroll
+    for (int u = 0; u < N; ++u) acc = fma(v[u], xv[u], acc);   // slot order = the row's CSR order
+    return acc;
+}
+
 template <typename T>
 __device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int pid, int row0,
                                                 const T* __restrict__ x) {
@@ -331,10 +346,31 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     if (!SORTED && npatc > 0) {
         int k = warp;
         int e = k < npatc ? __ldg(patlist + k) : 0;
+        int cur = -1, plen = 0;
+        int o[kSellMaxPatternLen];
+        T v[kSellMaxPatternLen];
         for (; k < npatc; k += nwarps) {
             const int en = k + nwarps < npatc ? __ldg(patlist + k + nwarps) : 0;
+            const int pid = e & 31;
+            if (pid != cur) {   // the list is sorted by pattern: rare
+                cur = pid;
+                plen = pt.len[pid];
+#pragma unroll
+                for (int u = 0; u < kSellMaxPatternLen; ++u) { o[u] = pt.off[pid][u]; v[u] = pt.val[pid][u]; }
+            }
             const int r = (e >> 5) * 32 + lane;
-            y[r] = sell_pattern_chunk<T>(pt, e & 31, r, x);
+            T acc;
+            switch (plen) {
+            case 1: acc = sell_pattern_regs<1, T>(o, v, r, x); break;
+            case 2: acc = sell_pattern_regs<2, T>(o, v, r, x); break;
+            case 3: acc = sell_pattern_regs<3, T>(o, v, r, x); break;
+            case 4: acc = sell_pattern_regs<4, T>(o, v, r, x); break;
+            case 5: acc = sell_pattern_regs<5, T>(o, v, r, x); break;
+            case 6: acc = sell_pattern_regs<6, T>(o, v, r, x); break;
+            case 7: acc = sell_pattern_regs<7, T>(o, v, r, x); break;
+            default: acc = sell_pattern_regs<8, T>(o, v, r, x); break;
+            }
+            y[r] = acc;
             e = en;
         }
     }

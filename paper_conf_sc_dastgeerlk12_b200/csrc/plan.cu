@@ -343,6 +343,9 @@ pepp_status_t sell_patterns(pepp_spmv_plan_t* p, int64_t nsb, const void* d_scon
             if (clen[c] & pepp::k::kSellPattern) pat.push_back((c << 5) | (int)cp[c]);
             else gen.push_back(c);
         }
+        // grouped by pattern (the kernel reloads its register copy of the
+        // pattern only when the id changes), chunk order within a pattern
+        std::stable_sort(pat.begin(), pat.end(), [](int a, int b) { return (a & 31) < (b & 31); });
         pepp_status_t s;
         if ((s = dalloc(p, &p->d_patlist, (int64_t)pat.size()))) return s;
         if ((s = dalloc(p, &p->d_genlist, (int64_t)gen.size()))) return s;
