@@ -50,6 +50,7 @@ def build_cuda(force: bool = False, verbose: bool = False) -> str:
               "-Xcompiler", "-fPIC,-fvisibility=hidden,-Wall", "--expt-relaxed-constexpr"]
     if verbose:
         common += ["-Xptxas", "-v"]
+    common += os.environ.get("PEPP_NVCC_EXTRA", "").split()   # experiments only (e.g. -DPEPP_PAT_U=4)
     objs = []
     for s in SOURCES:
         src = os.path.join(CSRC, s)

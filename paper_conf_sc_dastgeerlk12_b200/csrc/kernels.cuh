@@ -302,6 +302,32 @@ __device__ __forceinline__ T sell_pattern_regs(const int (&o)[kSellMaxPatternLen
     return acc;
 }
 
+// kPatU pattern chunks (list entries q[u], -1 = none) with the pattern in
+// registers: all loads first, then each row's FMAs in slot order, then stores.
+#ifndef PEPP_PAT_U
+#define PEPP_PAT_U 4
+#endif
+constexpr int kPatU = PEPP_PAT_U;
+template <int N, typename T>
+__device__ __forceinline__ void sell_pattern_group(const int (&o)[kSellMaxPatternLen], const T (&v)[kSellMaxPatternLen],
+                                                   const int (&q)[kPatU], int lane, const T* __restrict__ x,
+                                                   T* __restrict__ y) {
+    T xv[kPatU][N];
+#pragma unroll
+    for (int u = 0; u < kPatU; ++u) {
+        const int r = (q[u] >> 5) * 32 + lane;
+#pragma unroll
+        for (int j = 0; j < N; ++j) xv[u][j] = q[u] >= 0 ? ld_x(x, r + o[j]) : T(0);
+    }
+#pragma unroll
+    for (int u = 0; u < kPatU; ++u) {
+        T acc = T(0);
+#pragma unroll
+        for (int j = 0; j < N; ++j) acc = fma(v[j], xv[u][j], acc);   // slot order = the row's CSR order
+        if (q[u] >= 0) y[(q[u] >> 5) * 32 + lane] = acc;
+    }
+}
+
 template <typename T>
 __device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int pid, int row0,
                                                 const T* __restrict__ x) {
@@ -344,44 +370,55 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     // gathers, the FMAs and the y store per chunk. Phase B below then walks
     // only the other chunks (`genlist`, `nchunks` of them).
     if (!SORTED && npatc > 0) {
-        int k = warp;
-        int e = k < npatc ? __ldg(patlist + k) : 0;
+        // kPatU chunks per iteration (warp stride apart) so that kPatU x N
+        // gathers are in flight per warp; the next group's list entries are
+        // prefetched. Groups that straddle two patterns (the list is sorted
+        // by id, so at most a few per warp) take the one-chunk path.
+        int e[kPatU], en[kPatU];
+        auto load_e = [&](int k0, int (&q)[kPatU]) {
+#pragma unroll
+            for (int u = 0; u < kPatU; ++u) { const int kk = k0 + u * nwarps; q[u] = kk < npatc ? __ldg(patlist + kk) : -1; }
+        };
         int cur = -1, plen = 0;
         int o[kSellMaxPatternLen];
         T v[kSellMaxPatternLen];
-        for (; k < npatc; k += nwarps) {
-            const int en = k + nwarps < npatc ? __ldg(patlist + k + nwarps) : 0;
-            const int pid = e & 31;
-            if (pid != cur) {   // the list is sorted by pattern: rare
-                cur = pid;
-                plen = pt.len[pid];
+        auto reload = [&](int pid) {
+            cur = pid;
+            plen = pt.len[pid];
 #pragma unroll
-                for (int u = 0; u < kSellMaxPatternLen; ++u) { o[u] = pt.off[pid][u]; v[u] = pt.val[pid][u]; }
+            for (int u = 0; u < kSellMaxPatternLen; ++u) { o[u] = pt.off[pid][u]; v[u] = pt.val[pid][u]; }
+        };
+        load_e(warp, e);
+        for (int k0 = warp; k0 < npatc; k0 += kPatU * nwarps) {
+            load_e(k0 + kPatU * nwarps, en);
+            const int pid = e[0] & 31;
+            bool uni = true;
+#pragma unroll
+            for (int u = 1; u < kPatU; ++u) uni &= e[u] < 0 || (e[u] & 31) == pid;
+            if (pid != cur) reload(pid);
+            if (uni) {
+                switch (plen) {
+                case 1: sell_pattern_group<1, T>(o, v, e, lane, x, y); break;
+                case 2: sell_pattern_group<2, T>(o, v, e, lane, x, y); break;
+                case 3: sell_pattern_group<3, T>(o, v, e, lane, x, y); break;
+                case 4: sell_pattern_group<4, T>(o, v, e, lane, x, y); break;
+                case 5: sell_pattern_group<5, T>(o, v, e, lane, x, y); break;
+                case 6: sell_pattern_group<6, T>(o, v, e, lane, x, y); break;
+                case 7: sell_pattern_group<7, T>(o, v, e, lane, x, y); break;
+                default: sell_pattern_group<8, T>(o, v, e, lane, x, y); break;
+                }
+            } else {
+                for (int u = 0; u < kPatU; ++u) {
+                    if (e[u] < 0) continue;
+                    if ((e[u] & 31) != cur) reload(e[u] & 31);
+                    const int r = (e[u] >> 5) * 32 + lane;
+                    y[r] = sell_pattern_chunk<T>(pt, cur, r, x);
+                }
             }
-            const int r = (e >> 5) * 32 + lane;
-            T acc;
-            switch (plen) {
-            case 1: acc = sell_pattern_regs<1, T>(o, v, r, x); break;
-            case 2: acc = sell_pattern_regs<2, T>(o, v, r, x); break;
-            case 3: acc = sell_pattern_regs<3, T>(o, v, r, x); break;
-            case 4: acc = sell_pattern_regs<4, T>(o, v, r, x); break;
-            case 5: acc = sell_pattern_regs<5, T>(o, v, r, x); break;
-            case 6: acc = sell_pattern_regs<6, T>(o, v, r, x); break;
-            case 7: acc = sell_pattern_regs<7, T>(o, v, r, x); break;
-            default: acc = sell_pattern_regs<8, T>(o, v, r, x); break;
-            }
-            y[r] = acc;
-            e = en;
+#pragma unroll
+            for (int u = 0; u < kPatU; ++u) e[u] = en[u];
         }
     }
-    // chunk order: warp w walks i = w, w + nwarps, ...; chunk = i when the
-    // chunks are uniform (σ = 1). When σ > 1 sorted the rows, chunk lengths
-    // repeat a long-to-short pattern in every window of cpw = σ/32 chunks and
-    // a plain stride can hand a warp only the longest chunks; the order is
-    // then transposed (window-major -> position-major) over the full windows
-    // (longest first), and warp w walks the contiguous range
-    // [wstart[w], wstart[w+1]) of that order, cut at plan time so that every
-    // warp gets the same number of slots.
     const int nfull = SORTED ? (nchunks / cpw) * cpw : 0;
     const int nwin = SORTED ? nchunks / cpw : 1;
     auto chunk_of = [&](int i) -> int {
