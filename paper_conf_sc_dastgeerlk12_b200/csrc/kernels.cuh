@@ -287,45 +287,57 @@ __device__ __forceinline__ T sell_pattern_slots(const SellPatterns<T>& pt, int p
     return acc;
 }
 
-// Phase A form: the pattern's offsets / values already in registers (loaded
-// once per pattern change; reading the kernel-parameter table per chunk
-// would issue indexed LDCs, which run on the narrow ADU pipe).
-template <int N, typename T>
-__device__ __forceinline__ T sell_pattern_regs(const int (&o)[kSellMaxPatternLen], const T (&v)[kSellMaxPatternLen],
-                                               int row0, const T* __restrict__ x) {
-    T xv[N];
-#pragma unroll
-    for (int u = 0; u < N; ++u) xv[u] = ld_x(x, row0 + o[u]);
-    T acc = T(0);
-#pragma unroll
-    for (int u = 0; u < N; ++u) acc = fma(v[u], xv[u], acc);   // slot order = the row's CSR order
-    return acc;
-}
-
-// kPatU pattern chunks (list entries q[u], -1 = none) with the pattern in
-// registers: all loads first, then each row's FMAs in slot order, then stores.
 #ifndef PEPP_PAT_U
 #define PEPP_PAT_U 4
 #endif
-constexpr int kPatU = PEPP_PAT_U;
+constexpr int kPatU = PEPP_PAT_U;   // pattern chunks per warp iteration in phase A
+
+// list entries k0, k0 + stride, ... (kPatU of them; -1 past the end)
+__device__ __forceinline__ void sell_pattern_ids(const int* __restrict__ patlist, int npatc, int k0, int stride,
+                                                 int (&q)[kPatU]) {
+#pragma unroll
+    for (int u = 0; u < kPatU; ++u) { const int kk = k0 + u * stride; q[u] = kk < npatc ? __ldg(patlist + kk) : -1; }
+}
+
+// Groups of kPatU chunks of pattern `pid` (N slots) starting at list index
+// k0 (entries already in q), the next group's entries prefetched: the
+// pattern is read from the parameter table once into registers (indexed LDCs
+// per chunk would run on the narrow ADU pipe); all loads of the group are
+// issued before the first FMA. Returns the list index of the first group that
+// is not all `pid` (q then holds it), or >= npatc when the warp is done.
 template <int N, typename T>
-__device__ __forceinline__ void sell_pattern_group(const int (&o)[kSellMaxPatternLen], const T (&v)[kSellMaxPatternLen],
-                                                   const int (&q)[kPatU], int lane, const T* __restrict__ x,
-                                                   T* __restrict__ y) {
-    T xv[kPatU][N];
+__device__ __forceinline__ int sell_pattern_run(const SellPatterns<T>& pt, int pid, const int* __restrict__ patlist,
+                                             int npatc, int k0, int stride, int (&q)[kPatU], int lane,
+                                             const T* __restrict__ x, T* __restrict__ y) {
+    int o[N];
+    T v[N];
 #pragma unroll
-    for (int u = 0; u < kPatU; ++u) {
-        const int r = (q[u] >> 5) * 32 + lane;
+    for (int j = 0; j < N; ++j) { o[j] = pt.off[pid][j]; v[j] = pt.val[pid][j]; }
+    for (; k0 < npatc; k0 += kPatU * stride) {
+        bool uni = true;
 #pragma unroll
-        for (int j = 0; j < N; ++j) xv[u][j] = q[u] >= 0 ? ld_x(x, r + o[j]) : T(0);
+        for (int u = 0; u < kPatU; ++u) uni &= q[u] < 0 || (q[u] & 31) == pid;
+        if (!uni) return k0;
+        int qn[kPatU];
+        sell_pattern_ids(patlist, npatc, k0 + kPatU * stride, stride, qn);
+        T xv[kPatU][N];
+#pragma unroll
+        for (int u = 0; u < kPatU; ++u) {
+            const int r = (q[u] >> 5) * 32 + lane;
+#pragma unroll
+            for (int j = 0; j < N; ++j) xv[u][j] = q[u] >= 0 ? ld_x(x, r + o[j]) : T(0);
+        }
+#pragma unroll
+        for (int u = 0; u < kPatU; ++u) {
+            T acc = T(0);
+#pragma unroll
+            for (int j = 0; j < N; ++j) acc = fma(v[j], xv[u][j], acc);   // slot order = the row's CSR order
+            if (q[u] >= 0) y[(q[u] >> 5) * 32 + lane] = acc;
+        }
+#pragma unroll
+        for (int u = 0; u < kPatU; ++u) q[u] = qn[u];
     }
-#pragma unroll
-    for (int u = 0; u < kPatU; ++u) {
-        T acc = T(0);
-#pragma unroll
-        for (int j = 0; j < N; ++j) acc = fma(v[j], xv[u][j], acc);   // slot order = the row's CSR order
-        if (q[u] >= 0) y[(q[u] >> 5) * 32 + lane] = acc;
-    }
+    return k0;
 }
 
 template <typename T>
@@ -370,53 +382,33 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     // gathers, the FMAs and the y store per chunk. Phase B below then walks
     // only the other chunks (`genlist`, `nchunks` of them).
     if (!SORTED && npatc > 0) {
-        // kPatU chunks per iteration (warp stride apart) so that kPatU x N
-        // gathers are in flight per warp; the next group's list entries are
-        // prefetched. Groups that straddle two patterns (the list is sorted
-        // by id, so at most a few per warp) take the one-chunk path.
-        int e[kPatU], en[kPatU];
-        auto load_e = [&](int k0, int (&q)[kPatU]) {
-#pragma unroll
-            for (int u = 0; u < kPatU; ++u) { const int kk = k0 + u * nwarps; q[u] = kk < npatc ? __ldg(patlist + kk) : -1; }
-        };
-        int cur = -1, plen = 0;
-        int o[kSellMaxPatternLen];
-        T v[kSellMaxPatternLen];
-        auto reload = [&](int pid) {
-            cur = pid;
-            plen = pt.len[pid];
-#pragma unroll
-            for (int u = 0; u < kSellMaxPatternLen; ++u) { o[u] = pt.off[pid][u]; v[u] = pt.val[pid][u]; }
-        };
-        load_e(warp, e);
-        for (int k0 = warp; k0 < npatc; k0 += kPatU * nwarps) {
-            load_e(k0 + kPatU * nwarps, en);
+        // Runs of one pattern go through sell_pattern_run<N> (no per-chunk
+        // branch on the pattern length); a group of list entries that
+        // straddles two patterns (the list is sorted by id: at most one per
+        // pattern change per warp) takes the one-chunk path.
+        int e[kPatU];
+        int k0 = warp;
+        sell_pattern_ids(patlist, npatc, k0, nwarps, e);
+        while (k0 < npatc) {
             const int pid = e[0] & 31;
-            bool uni = true;
-#pragma unroll
-            for (int u = 1; u < kPatU; ++u) uni &= e[u] < 0 || (e[u] & 31) == pid;
-            if (pid != cur) reload(pid);
-            if (uni) {
-                switch (plen) {
-                case 1: sell_pattern_group<1, T>(o, v, e, lane, x, y); break;
-                case 2: sell_pattern_group<2, T>(o, v, e, lane, x, y); break;
-                case 3: sell_pattern_group<3, T>(o, v, e, lane, x, y); break;
-                case 4: sell_pattern_group<4, T>(o, v, e, lane, x, y); break;
-                case 5: sell_pattern_group<5, T>(o, v, e, lane, x, y); break;
-                case 6: sell_pattern_group<6, T>(o, v, e, lane, x, y); break;
-                case 7: sell_pattern_group<7, T>(o, v, e, lane, x, y); break;
-                default: sell_pattern_group<8, T>(o, v, e, lane, x, y); break;
-                }
-            } else {
-                for (int u = 0; u < kPatU; ++u) {
-                    if (e[u] < 0) continue;
-                    if ((e[u] & 31) != cur) reload(e[u] & 31);
-                    const int r = (e[u] >> 5) * 32 + lane;
-                    y[r] = sell_pattern_chunk<T>(pt, cur, r, x);
-                }
+            switch (pt.len[pid]) {
+            case 1: k0 = sell_pattern_run<1, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 2: k0 = sell_pattern_run<2, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 3: k0 = sell_pattern_run<3, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 4: k0 = sell_pattern_run<4, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 5: k0 = sell_pattern_run<5, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 6: k0 = sell_pattern_run<6, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 7: k0 = sell_pattern_run<7, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            default: k0 = sell_pattern_run<8, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
             }
-#pragma unroll
-            for (int u = 0; u < kPatU; ++u) e[u] = en[u];
+            if (k0 >= npatc) break;
+            for (int u = 0; u < kPatU; ++u) {   // the mixed group
+                if (e[u] < 0) continue;
+                const int r = (e[u] >> 5) * 32 + lane;
+                y[r] = sell_pattern_chunk<T>(pt, e[u] & 31, r, x);
+            }
+            k0 += kPatU * nwarps;
+            sell_pattern_ids(patlist, npatc, k0, nwarps, e);
         }
     }
     const int nfull = SORTED ? (nchunks / cpw) * cpw : 0;
