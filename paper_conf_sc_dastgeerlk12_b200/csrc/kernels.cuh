@@ -21,6 +21,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <type_traits>
+
 namespace pepp {
 namespace k {
 
@@ -356,7 +358,13 @@ __device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int p
     }
 }
 
-template <int BLOCK, bool SORTED, typename T>
+struct NoPatterns {};
+template <bool PAT, typename T>
+using SellPatternArg = std::conditional_t<PAT, SellPatterns<T>, NoPatterns>;
+
+// PAT: the plan has pattern chunks (phase A + genlist); PAT = false compiles
+// the general kernel without them (no extra registers, no 3 KB parameter).
+template <int BLOCK, bool SORTED, bool PAT, typename T>
 __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
                                                      const int* __restrict__ chunk_len,
                                                      const int* __restrict__ rowlen,
@@ -364,7 +372,7 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
                                                      const int* __restrict__ col,
                                                      const int16_t* __restrict__ col16,
                                                      const int* __restrict__ soff,
-                                                     const __grid_constant__ SellPatterns<T> pt,
+                                                     const __grid_constant__ SellPatternArg<PAT, T> pt,
                                                      const T* __restrict__ val,
                                                      const T* __restrict__ x,
                                                      T* __restrict__ y,
@@ -381,7 +389,7 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     // per-lane loads: 1 list entry (prefetched one step ahead), the x
     // gathers, the FMAs and the y store per chunk. Phase B below then walks
     // only the other chunks (`genlist`, `nchunks` of them).
-    if (!SORTED && npatc > 0) {
+    if constexpr (!SORTED && PAT) if (npatc > 0) {
         // Runs of one pattern go through sell_pattern_run<N> (no per-chunk
         // branch on the pattern length); a group of list entries that
         // straddles two patterns (the list is sorted by id: at most one per
@@ -414,7 +422,7 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     const int nfull = SORTED ? (nchunks / cpw) * cpw : 0;
     const int nwin = SORTED ? nchunks / cpw : 1;
     auto chunk_of = [&](int i) -> int {
-        if (!SORTED) return genlist ? __ldg(genlist + i) : i;
+        if (!SORTED) return PAT ? __ldg(genlist + i) : i;
         return i < nfull ? (i % nwin) * cpw + i / nwin : i;
     };
     // Two-deep software pipelining over the warp's chunks (latency-bound
@@ -450,8 +458,13 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
         const int64_t base = q0.cp + lane;
         const int clen = q0.d & kSellLenMask;
         T acc;
-        if (q0.d & kSellPattern) acc = sell_pattern_chunk<T>(pt, (int)q0.cp, l0.orow, x);   // cp holds the pattern id
-        else if (q0.d & kSellStencil) acc = sell_chunk<kIdxStencil, T>(val, col, col16, l0.offl, l0.orow, x, base, clen, l0.len, pol);
+        bool pat_chunk = false;
+        if constexpr (PAT) {
+            pat_chunk = (q0.d & kSellPattern) != 0;
+            if (pat_chunk) acc = sell_pattern_chunk<T>(pt, (int)q0.cp, l0.orow, x);   // cp holds the pattern id
+        }
+        if (pat_chunk) {
+        } else if (q0.d & kSellStencil) acc = sell_chunk<kIdxStencil, T>(val, col, col16, l0.offl, l0.orow, x, base, clen, l0.len, pol);
         else if (q0.d & kSellCol16) acc = sell_chunk<kIdx16, T>(val, col, col16, 0, l0.orow, x, base, clen, l0.len, pol);
         else acc = sell_chunk<kIdx32, T>(val, col, col16, 0, l0.orow, x, base, clen, l0.len, pol);
         if (c * 32 + lane < nrows) y[l0.orow] = acc;

@@ -655,16 +655,26 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
         }
         break;
     case PEPP_V_SELL:
-        if (p->d_perm)
-            pepp::k::sell_kernel<kBlock, true, T><<<p->grid_sell, kBlock, 0, st>>>(
+        if (p->d_perm && p->sell_const_chunks)   // σ > 1: pattern chunks inline in the sorted walk
+            pepp::k::sell_kernel<kBlock, true, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
                 p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws,
                 nullptr, 0, nullptr);
-        else
-            pepp::k::sell_kernel<kBlock, false, T><<<p->grid_sell, kBlock, 0, st>>>(
-                (int)p->nrows, p->d_patlist ? p->ngen : p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
+        else if (p->d_perm)
+            pepp::k::sell_kernel<kBlock, true, false, T><<<p->grid_sell, kBlock, 0, st>>>(
+                (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
+                p->d_scol16, p->d_soff, pepp::k::NoPatterns{}, (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws,
+                nullptr, 0, nullptr);
+        else if (p->d_patlist)   // pattern chunks (value compression): phase A + the rest through genlist
+            pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, st>>>(
+                (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
-                p->d_patlist, p->npatc, p->d_patlist ? p->d_genlist : nullptr);
+                p->d_patlist, p->npatc, p->d_genlist);
+        else
+            pepp::k::sell_kernel<kBlock, false, false, T><<<p->grid_sell, kBlock, 0, st>>>(
+                (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
+                p->d_scol, p->d_scol16, p->d_soff, pepp::k::NoPatterns{}, (const T*)p->d_sval, x, y, 1, nullptr,
+                nullptr, 0, nullptr);
         break;
     default:
         return PEPP_E_INVALID;
@@ -1173,7 +1183,12 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     p->grid_csr[5] = grid_for((const void*)pepp::k::csr_vector_kernel<32, kBlock, double>, kBlock, A->nrows, kBlock / 32, p->sm_count);
     {   // SELL: exactly one resident wave; warps walk their chunks with prefetch
         int occ = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pepp::k::sell_kernel<kBlock, false, double>, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
+        const bool srt = p->d_perm != nullptr, pat = p->sell_const_chunks > 0, f32 = p->vt == PEPP_VALUE_F32;
+        const void* fn = f32 ? (srt ? (pat ? (const void*)pepp::k::sell_kernel<kBlock, true, true, float> : (const void*)pepp::k::sell_kernel<kBlock, true, false, float>)
+                                    : (pat ? (const void*)pepp::k::sell_kernel<kBlock, false, true, float> : (const void*)pepp::k::sell_kernel<kBlock, false, false, float>))
+                             : (srt ? (pat ? (const void*)pepp::k::sell_kernel<kBlock, true, true, double> : (const void*)pepp::k::sell_kernel<kBlock, true, false, double>)
+                                    : (pat ? (const void*)pepp::k::sell_kernel<kBlock, false, true, double> : (const void*)pepp::k::sell_kernel<kBlock, false, false, double>));
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
         (void)cudaGetLastError();
         const int64_t need = ((int64_t)p->nchunks + kBlock / 32 - 1) / (kBlock / 32);
         const int64_t wave = (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ;
