@@ -357,7 +357,14 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
 
     stream = torch.cuda.Stream(device=dev)
     xs = torch.from_numpy(x0).to(dev)
-    bufs = [torch.empty(R, dtype=tdt, device=dev) for _ in range(2)]
+    p2p = overlapped and not args.no_p2p
+    if p2p:
+        # symmetric buffers: the boundary kernel pushes the halo straight into
+        # the neighbours' copies over peer memory (PEPP_X_P2P), no NCCL per iteration
+        bufs = plan.p2p_buffers(2)
+        kernels_per_call = 2
+    else:
+        bufs = [torch.empty(R, dtype=tdt, device=dev) for _ in range(2)]
     flush = None if iterated or Z * 12 > 4 * (1 << 30) else torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     ev_pool = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(iters)]
@@ -537,12 +544,14 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             "config": {"workload": args.workload, "desc": wl["desc"], "spmv_per_step": iters,
                        "rows": R, "nnz": Z, "l2": "inputs larger than L2 (5.4 GB/SpMV)" if iterated
                        else "L2 flushed (512 MB memset) between SpMVs; kernel events only",
-                       "exchange": pepp._capi.EXCHANGE_NAMES.get(info["exchange"], "?"),
+                       "exchange": "p2p (fused boundary kernel, peer-memory stores)" if p2p
+                       else pepp._capi.EXCHANGE_NAMES.get(info["exchange"], "?"),
                        "variant": args.variant or "auto (history-based per call)"},
             "hbm": {"achieved_gbs": round(gbs, 1), "frac_of_measured": round(gbs / (world * peak), 4),
                     "frac_of_8tbs": round(gbs / (world * 8000.0), 4), "algorithmic_bytes_per_spmv": alg_bytes_global},
             "roofline": dict(roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, args.workload),
-                             **({"launch_includes": "head + interior + tail kernels and the overlapped halo exchange"}
+                             **({"launch_includes": "interior kernel + the fused boundary/push kernel (P2P halo)"
+                                 if p2p else "head + interior + tail kernels and the overlapped halo exchange"}
                                 if overlapped else {})),
             "e2e": {"value": round(e2e_val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": A.ncols * esz,
                     "d2h_bytes_per_step": A.nrows * esz, "spmv_per_step": e2e_iters,
@@ -581,6 +590,8 @@ def main():
                          "streamed and the compressed plan is reported separately under 'value_compressed'")
     ap.add_argument("--no-value-compression", action="store_true", help=argparse.SUPPRESS)   # the default now
     ap.add_argument("--no-vc-leg", action="store_true", help="skip the value-compressed leg")
+    ap.add_argument("--no-p2p", action="store_true",
+                    help="N > 1: NCCL halo per iteration instead of the fused peer-memory push (PEPP_X_P2P)")
     ap.add_argument("--dtype", choices=["f64", "f32"], default="f64",
                     help="f64 = BASELINE's precision (default); f32 = the paper's float instance")
     args = ap.parse_args()

@@ -57,7 +57,7 @@
 extern "C" {
 #endif
 
-#define PEPP_ABI_VERSION 2
+#define PEPP_ABI_VERSION 3
 
 typedef enum {
     PEPP_OK = 0,
@@ -86,7 +86,13 @@ typedef enum {
     PEPP_X_AUTO = -1,
     PEPP_X_NONE = 0,          /* single rank                                          */
     PEPP_X_ALLGATHER = 1,     /* allgatherv of y slices: every rank gets all of y     */
-    PEPP_X_HALO = 2           /* ghost (halo) exchange: only entries peers' rows read */
+    PEPP_X_HALO = 2,          /* ghost (halo) exchange: only entries peers' rows read */
+    PEPP_X_P2P = 3            /* halo written by the boundary-row kernel itself straight into the
+                                 peers' registered buffers over peer memory (CUDA IPC mappings:
+                                 NVLink / NVSwitch stores), signalled with flags in peer memory —
+                                 compute and exchange in one kernel, no NCCL on the data path.
+                                 Used (never requested) by PEPP_Y_NEXT_INPUT calls whose y is one
+                                 of the plan's pepp_spmv_p2p_buffers; reported in pepp_choice_t */
 } pepp_exchange_t;
 
 /* value types (pepp_csr_t.value_type) */
@@ -225,6 +231,7 @@ typedef struct pepp_plan_info_s {
     int64_t overlap_tail;     /*   before the exchange starts (0 / 0 when overlap == 0) */
     int32_t predicted;        /* candidates with a prediction from opts.predict (0 = none / no function) */
     double sell_constval_frac;/* fraction of SELL chunks stored as a pattern-table id (compress_values) */
+    int32_t p2p_buffers;      /* symmetric buffers registered by pepp_spmv_p2p_buffers (0 = none) */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */
@@ -279,6 +286,38 @@ pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void* x, void* y, int fl
    exec(PEPP_Y_LOCAL) followed by exchange(flags). A no-op when nranks == 1.
    Errors: PEPP_E_INVALID, PEPP_E_NCCL, PEPP_E_CUDA. */
 pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* y, int flags, void* stream);
+
+/* Symmetric buffers for the fused peer-memory halo (PEPP_X_P2P).
+   The paper partitions a component call into sub-tasks whose outputs are
+   concatenated (§IV-F P@27330–28000) and overlaps their communication with
+   computation; on B200s joined by NVSwitch the concatenation can be done by
+   the kernel that produces the rows: it stores them into the neighbours'
+   memory directly (SURVEY §8(e) "Stretch": fuse the ghost push into the
+   SpMV). Collective over the plan's ranks (every rank calls it with the
+   same nbuf). Allocates nbuf (1..4) device buffers of row_bounds[nranks]
+   elements of the plan's value type (zeroed) plus a small signal block,
+   exports them with CUDA IPC, all-gathers the handles over the plan's
+   communicator and maps the buffers of the ranks this rank sends to
+   (cudaIpcMemLazyEnablePeerAccess). bufs: WRITE, host array of nbuf
+   pointers that receive this rank's buffers (owned by the plan, valid until
+   pepp_spmv_destroy, which is then collective too).
+   Afterwards a pepp_spmv_exec(flags = PEPP_Y_NEXT_INPUT, force = NULL) whose
+   y is bufs[i] — the same i on every rank, every rank making the same
+   sequence of such calls — computes the interior rows on `stream` and, on
+   the plan's side stream, runs ONE kernel that computes the head / tail rows,
+   writes them to y and to the peers' bufs[i], and signals / waits on the
+   peers (protocol in kernels.cuh, halo_push_kernel); the call's stream work
+   completes when own rows and every ghost are in y, as with the NCCL halo.
+   Rows of this block outside the ghosts a peer reads may also be written
+   into that peer's buffer (with their correct values). Calls with any other
+   y use the NCCL exchange. Boundary rows are summed in the oracle's order
+   (no FMA). Requires nranks > 1, the halo exchange and the head / interior /
+   tail split (pepp_plan_info_t.overlap == 1), else PEPP_E_UNSUPPORTED;
+   PEPP_E_STATE if already registered. A peer that stops calling makes the
+   waiting kernel give up after 20 s and the plan's next call return
+   PEPP_E_NCCL. Errors: PEPP_E_INVALID, PEPP_E_CUDA (IPC unavailable),
+   PEPP_E_NCCL, PEPP_E_NOMEM. */
+pepp_status_t pepp_spmv_p2p_buffers(pepp_spmv_plan_t* p, int32_t nbuf, void** bufs);
 
 /* Host-buffer entry point (the paper's measurement setting, where operand
    transfers are part of the call: Fig. 5 "communication overhead of copying
@@ -458,6 +497,11 @@ pepp_status_t pepp_nccl_unique_id(void* id_out);
    PEPP_OK, PEPP_E_NCCL (unavailable, an NCCL error, or wrong data), or
    PEPP_E_CUDA. Synchronous; allocates and frees its own buffers. */
 pepp_status_t pepp_nccl_selftest(int32_t device);
+
+/* Text of the last CUDA failure that made a call on this thread return
+   PEPP_E_CUDA: the CUDA error string, the failing runtime call and its
+   source line ("" if none yet). Thread-local, static storage, never NULL. */
+const char* pepp_last_error(void);
 
 /* ABI version (PEPP_ABI_VERSION) of the loaded library. */
 int32_t pepp_abi_version(void);

@@ -20,12 +20,12 @@ import numpy as np
 
 from . import _capi as C
 from ._capi import (ACCESS_READ, ACCESS_READWRITE, ACCESS_WRITE, DEVICE_SIMULATED, EXEC_NO_TIMING, PeppError, V_CSR_STREAM, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, X_ALLGATHER, X_AUTO,
-                    X_HALO, X_NONE, Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, VARIANT_NAMES)
+                    X_HALO, X_NONE, X_P2P, Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, VARIANT_NAMES)
 
 __all__ = ["Plan", "Choice", "History", "Vector", "ACCESS_READ", "ACCESS_WRITE", "ACCESS_READWRITE",
            "DEVICE_SIMULATED", "partition_rows", "halo_ghosts", "context_key", "nccl_unique_id",
            "lib_path", "PeppError", "V_CSR_VECTOR", "V_MERGE_PATH", "V_SELL", "V_CSR_STREAM", "X_AUTO", "X_NONE",
-           "X_ALLGATHER", "X_HALO", "Y_LOCAL", "Y_NEXT_INPUT", "Y_REPLICATED", "EXEC_NO_TIMING",
+           "X_ALLGATHER", "X_HALO", "X_P2P", "Y_LOCAL", "Y_NEXT_INPUT", "Y_REPLICATED", "EXEC_NO_TIMING",
            "VARIANT_NAMES"]
 
 lib_path = C.LIB_PATH
@@ -179,6 +179,25 @@ class Plan:
         """The exchange step alone (no-op on an unpartitioned plan)."""
         C.check(C.lib().pepp_spmv_exchange(self._h, _ptr(y), flags, _stream_handle(stream)), "pepp_spmv_exchange")
 
+    def p2p_buffers(self, nbuf: int = 2) -> list:
+        """pepp_spmv_p2p_buffers (collective): `nbuf` plan-owned symmetric
+        device buffers (global length, the plan's value type) as CUDA tensors.
+        PEPP_Y_NEXT_INPUT calls whose y is one of them push the halo from the
+        boundary kernel straight into the peers' copies (PEPP_X_P2P). The
+        tensors borrow the plan's memory: they keep the Plan object alive, and
+        must not be used after close()."""
+        import torch
+        arr = (ctypes.c_void_p * nbuf)()
+        C.check(C.lib().pepp_spmv_p2p_buffers(self._h, nbuf, arr), "pepp_spmv_p2p_buffers")
+        n = int(self._bounds[-1]) if self._bounds is not None else self.nrows
+        f32 = self.value_type == C.VALUE_F32
+        dev = torch.cuda.current_device()
+        out = []
+        for i in range(nbuf):
+            ref = _DeviceArray(arr[i], n, "<f4" if f32 else "<f8", self)
+            out.append(torch.as_tensor(ref, device=torch.device("cuda", dev)))
+        return out
+
     def exec_host(self, x_host: np.ndarray, y_host: np.ndarray, iterations: int = 1, flags: int = Y_LOCAL,
                   stream=None) -> None:
         """Host buffers in and out, transfers inside the call (synchronous)."""
@@ -234,6 +253,16 @@ class Plan:
     def from_csr(cls, A, **kw) -> "Plan":
         """From any object with nrows, ncols, row_ptr, col, val (e.g. gen.CSR)."""
         return cls(A.nrows, A.ncols, A.row_ptr, A.col, A.val, **kw)
+
+
+class _DeviceArray:
+    """__cuda_array_interface__ view of plan-owned device memory (no copy);
+    holds the plan so the memory outlives every tensor made from it."""
+
+    def __init__(self, ptr: int, n: int, typestr: str, owner):
+        self._owner = owner
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
 
 
 class Graph:

@@ -13,13 +13,13 @@ LIB_PATH = os.path.join(_HERE, "libpepp_spmv.so")
 
 PEPP_OK, PEPP_E_INVALID, PEPP_E_CUDA, PEPP_E_NCCL, PEPP_E_NOMEM, PEPP_E_UNSUPPORTED, PEPP_E_STATE = 0, -1, -2, -3, -4, -5, -6
 V_AUTO, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, V_CSR_STREAM, V_COUNT = -1, 0, 1, 2, 3, 4
-X_AUTO, X_NONE, X_ALLGATHER, X_HALO = -1, 0, 1, 2
+X_AUTO, X_NONE, X_ALLGATHER, X_HALO, X_P2P = -1, 0, 1, 2, 3
 Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, EXEC_NO_TIMING = 0x0, 0x1, 0x2, 0x10
 ACCESS_READ, ACCESS_WRITE, ACCESS_READWRITE = 1, 2, 3
 VALUE_F64, VALUE_F32 = 0, 1
 DEVICE_SIMULATED = -2
 VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell", V_CSR_STREAM: "csr_stream"}
-EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_AUTO: "auto"}
+EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_P2P: "p2p", X_AUTO: "auto"}
 
 c_i32, c_i64, c_u32, c_u64, c_f64, c_vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_uint64,
                                           ctypes.c_double, ctypes.c_void_p)
@@ -38,7 +38,7 @@ class INFO_T(ctypes.Structure):
                 ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64),
                 ("prior_key", c_u64), ("sell_stencil_frac", c_f64),
                 ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64), ("predicted", c_i32),
-                ("sell_constval_frac", c_f64)]
+                ("sell_constval_frac", c_f64), ("p2p_buffers", c_i32)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -77,6 +77,7 @@ SIGNATURES = {
     "pepp_spmv_exec": (c_i32, [c_vp, c_vp, c_vp, ctypes.c_int, c_vp, ctypes.POINTER(CHOICE_T), ctypes.POINTER(CHOICE_T)]),
     "pepp_spmv_exec_host": (c_i32, [c_vp, c_vp, c_vp, c_i32, ctypes.c_int, c_vp]),
     "pepp_spmv_exchange": (c_i32, [c_vp, c_vp, ctypes.c_int, c_vp]),
+    "pepp_spmv_p2p_buffers": (c_i32, [c_vp, c_i32, ctypes.POINTER(c_vp)]),
     "pepp_spmv_destroy": (c_i32, [c_vp]),
     "pepp_spmv_plan_info": (c_i32, [c_vp, ctypes.POINTER(INFO_T)]),
     "pepp_spmv_candidates": (c_i32, [c_vp, ctypes.POINTER(CHOICE_T), c_i32, ctypes.POINTER(c_i32)]),
@@ -108,6 +109,7 @@ SIGNATURES = {
     "pepp_nccl_unique_id": (c_i32, [c_vp]),
     "pepp_nccl_selftest": (c_i32, [c_i32]),
     "pepp_abi_version": (c_i32, []),
+    "pepp_last_error": (ctypes.c_char_p, []),
 }
 
 _lib = None
@@ -116,10 +118,16 @@ _lib = None
 class PeppError(RuntimeError):
     def __init__(self, status: int, where: str):
         self.status = status
-        super().__init__(f"{where}: {status_str(status)} ({status})")
+        detail = ""
+        if status == PEPP_E_CUDA:
+            try:
+                detail = lib().pepp_last_error().decode()
+            except Exception:
+                pass
+        super().__init__(f"{where}: {status_str(status)} ({status})" + (f": {detail}" if detail else ""))
 
 
-ABI_VERSION = 2   # PEPP_ABI_VERSION of include/pepp_spmv.h
+ABI_VERSION = 3   # PEPP_ABI_VERSION of include/pepp_spmv.h
 
 
 def lib() -> ctypes.CDLL:

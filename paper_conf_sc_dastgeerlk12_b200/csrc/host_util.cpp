@@ -17,6 +17,16 @@
 #include <unordered_map>
 #include <vector>
 
+namespace {
+thread_local char g_last_error[512] = "";
+}
+
+void pepp::set_last_error(const char* msg, const char* expr, int line) {
+    std::snprintf(g_last_error, sizeof(g_last_error), "%s (%s, plan.cu:%d)", msg ? msg : "?", expr ? expr : "?", line);
+}
+
+extern "C" PEPP_API const char* pepp_last_error(void) { return g_last_error; }
+
 extern "C" PEPP_API const char* pepp_status_str(pepp_status_t s) {
     switch (s) {
     case PEPP_OK: return "PEPP_OK";

@@ -1144,5 +1144,131 @@ __global__ void scatter_kernel(int64_t n, const int* __restrict__ idx, const T* 
         dst[idx[i]] = src[i];
 }
 
+
+// =====================================================================
+// Fused compute + halo exchange over peer memory (exchange PEPP_X_P2P).
+// One kernel per partitioned iteration computes the rows the neighbours read
+// (the head [0, h) and tail [R - t, R) of the block), stores each result in
+// the local y AND straight into every receiving peer's copy of the same
+// buffer (CUDA-IPC mapped peer memory: NVLink / NVSwitch stores), then
+// signals the peers with release stores to flags in their memory and waits
+// (acquire) until every peer this rank receives from has signalled. Replaces
+// head/tail SpMV kernels + NCCL send/recv + pack/unpack of the in-order path.
+//
+// Protocol (per plan, `epoch` e = number of P2P calls so far, device
+// resident so CUDA graphs replay it correctly). Flags live in the receiver's
+// signal block, one slot per sender:
+//   ready[q]  = e+1 : rank q began call e, so everything q's streams did
+//                   before (calls < e, which read q's buffers — e.g. the
+//                   previous x — and the caller's own writes, e.g. filling
+//                   x_0) is complete: q's y of call e may now be written;
+//   arrive[q] = e+1 : rank q's rows of call e have landed in this rank's y.
+// Call e on rank r: every CTA writes ready = e+1 into each send-peer's block
+// (idempotent; no CTA waits for another CTA of the grid), waits for the
+// send-peers' ready >= e+1, computes its rows and pushes them; the last CTA
+// (grid-wide counter) fences, writes arrive = e+1 into each send-peer's
+// block, waits for arrive >= e+1 from every receive-peer, resets the counter
+// and bumps the epoch. Kernel completion therefore means exactly what the
+// NCCL halo's stream completion means: own rows and every ghost are in y.
+// Every wait is bounded (%globaltimer, timeout_ns: 20 s, PEPP_P2P_TIMEOUT_MS): a peer that never
+// arrives sets *err (host-mapped) instead of hanging the GPU.
+//
+// Row sums are the oracle's arithmetic (sequential in CSR order, product
+// rounded then sum rounded: __dmul_rn / __dadd_rn, no FMA), one thread per
+// row: boundary rows of stencils / banded matrices are short.
+// =====================================================================
+constexpr int kP2PMaxPeers = 8;
+constexpr int kP2PMaxPush = 16;
+
+template <typename T>
+struct P2PArgs {
+    int64_t seg_lo[2], seg_hi[2];      // local rows computed here: head, tail
+    int64_t row_offset;                // global index of local row 0
+    int npush;                         // push ranges: local rows [lo, hi) -> peer buffer base
+    int64_t push_lo[kP2PMaxPush], push_hi[kP2PMaxPush];
+    T* push_dst[kP2PMaxPush];          // the peer's buffer (global indexing)
+    int nsend;                         // peers this rank writes to
+    unsigned long long* peer_ready[kP2PMaxPeers];    // &peer.ready[me]
+    unsigned long long* peer_arrive[kP2PMaxPeers];   // &peer.arrive[me]
+    unsigned long long* my_ready[kP2PMaxPeers];      // &my.ready[send peer]
+    int nrecv;                         // peers this rank receives from
+    unsigned long long* my_arrive[kP2PMaxPeers];     // &my.arrive[recv peer]
+    unsigned long long* epoch;         // my signal block
+    unsigned int* done;                // my signal block: CTAs finished this call
+    int* err;                          // host-mapped error flag
+    unsigned long long timeout_ns;     // bound on every wait
+};
+
+__device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long global_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// spin until *p >= v (bounded); false on timeout
+__device__ __forceinline__ bool wait_geq(const unsigned long long* p, unsigned long long v, unsigned long long t0,
+                                         unsigned long long timeout_ns) {
+    while (ld_acquire_sys(p) < v) {
+        if (global_ns() - t0 > timeout_ns) return false;
+        __nanosleep(64);
+    }
+    return true;
+}
+
+__device__ __forceinline__ double mul_rn(double a, double b) { return __dmul_rn(a, b); }
+__device__ __forceinline__ double add_rn(double a, double b) { return __dadd_rn(a, b); }
+__device__ __forceinline__ float mul_rn(float a, float b) { return __fmul_rn(a, b); }
+__device__ __forceinline__ float add_rn(float a, float b) { return __fadd_rn(a, b); }
+
+template <typename T>
+__global__ void __launch_bounds__(256) halo_push_kernel(const int* __restrict__ rp, const int* __restrict__ col,
+                                                        const T* __restrict__ val, const T* __restrict__ x,
+                                                        T* __restrict__ y, const __grid_constant__ P2PArgs<T> a) {
+    __shared__ unsigned long long s_epoch;
+    __shared__ int s_last;
+    const unsigned long long t0 = global_ns();
+    if (threadIdx.x == 0) {
+        const unsigned long long e = *(volatile unsigned long long*)a.epoch;
+        s_epoch = e;
+        for (int j = 0; j < a.nsend; ++j) st_release_sys(a.peer_ready[j], e + 1);
+        bool ok = true;
+        for (int j = 0; j < a.nsend; ++j) ok &= wait_geq(a.my_ready[j], e + 1, t0, a.timeout_ns);
+        if (!ok) atomicExch(a.err, 1);
+    }
+    __syncthreads();
+    const int64_t n0 = a.seg_hi[0] - a.seg_lo[0], n = n0 + (a.seg_hi[1] - a.seg_lo[1]);
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = t < n0 ? a.seg_lo[0] + t : a.seg_lo[1] + (t - n0);
+        T acc = T(0);
+        for (int k = rp[i]; k < rp[i + 1]; ++k) acc = add_rn(acc, mul_rn(val[k], x[col[k]]));
+        const int64_t g = a.row_offset + i;
+        y[g] = acc;
+        for (int j = 0; j < a.npush; ++j)
+            if (i >= a.push_lo[j] && i < a.push_hi[j]) a.push_dst[j][g] = acc;
+    }
+    // publish: every CTA's stores before the last CTA's arrive flags
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) s_last = atomicAdd(a.done, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (!s_last || threadIdx.x != 0) return;
+    __threadfence_system();
+    const unsigned long long e = s_epoch;
+    for (int j = 0; j < a.nsend; ++j) st_release_sys(a.peer_arrive[j], e + 1);
+    bool ok = true;
+    for (int j = 0; j < a.nrecv; ++j) ok &= wait_geq(a.my_arrive[j], e + 1, global_ns(), a.timeout_ns);
+    if (!ok) atomicExch(a.err, 1);
+    *a.done = 0u;
+    *(volatile unsigned long long*)a.epoch = e + 1;
+    __threadfence();
+}
+
 }  // namespace k
 }  // namespace pepp

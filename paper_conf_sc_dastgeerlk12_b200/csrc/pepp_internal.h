@@ -31,6 +31,9 @@ bool history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t
                    uint64_t* from_key);
 void halo_ghost_list(const int32_t* col, int64_t nnz, int64_t lo, int64_t hi, std::vector<int32_t>& out);
 
+// last CUDA failure of this thread (pepp_last_error): message, failing expression, plan.cu line
+void set_last_error(const char* msg, const char* expr, int line);
+
 // ---- smart containers (containers.cu) ----
 int64_t vector_length(const pepp_vector_t* v);
 bool vector_simulated(const pepp_vector_t* v);
@@ -41,7 +44,7 @@ bool vector_simulated(const pepp_vector_t* v);
 // host-only utilities run) on machines without NCCL or a GPU.
 typedef struct ncclComm_opaque* ncclComm_t;
 typedef struct { char internal[128]; } ncclUniqueId;
-enum { NCCL_INT32 = 2, NCCL_INT64 = 4, NCCL_FLOAT32 = 7, NCCL_FLOAT64 = 8 };
+enum { NCCL_INT8 = 0, NCCL_INT32 = 2, NCCL_INT64 = 4, NCCL_FLOAT32 = 7, NCCL_FLOAT64 = 8 };
 enum { NCCL_OP_MAX = 2 };
 struct Nccl {
     int (*GetUniqueId)(ncclUniqueId*);

@@ -17,6 +17,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <new>
@@ -45,6 +46,7 @@ constexpr int kStreamNB = 2048;
 constexpr int kStreamRMAX = 512;
 constexpr int kStreamVecMinLen = 64;   // items whose longest row exceeds this reduce warp-per-row
 constexpr int kReserveSms = 2;         // SMs the interior sub-plan's persistent grid leaves to the exchange
+constexpr int kP2PMaxBuf = 4;          // symmetric buffers per plan (pepp_spmv_p2p_buffers)
 
 struct Candidate {
     int32_t variant;
@@ -166,6 +168,26 @@ struct pepp_spmv_plan_s {
     int reserve_sms = 0;                         // SMs a persistent grid leaves free (interior sub-plan)
     std::vector<int64_t> send_local;             // plan time: local rows the peers receive
 
+    // fused peer-memory halo (PEPP_X_P2P, pepp_spmv_p2p_buffers)
+    struct SendRange { int32_t peer; int64_t lo, hi; };   // local rows [lo, hi) some peer receives
+    std::vector<SendRange> send_rng;             // plan time (setup_halo)
+    int p2p_nbuf = 0;
+    void* p2p_buf[kP2PMaxBuf] = {};              // this rank's symmetric buffers (global length)
+    unsigned long long* d_sig = nullptr;         // signal block: ready[P], arrive[P], epoch, done
+    int* h_err = nullptr;                        // host-mapped error flag (a peer never arrived)
+    int* d_err = nullptr;
+    std::vector<void*> p2p_opened;               // IPC mappings of peers' buffers / signal blocks
+    int p2p_npush = 0;
+    int64_t p2p_push_lo[pepp::k::kP2PMaxPush] = {}, p2p_push_hi[pepp::k::kP2PMaxPush] = {};
+    void* p2p_push_dst[kP2PMaxBuf][pepp::k::kP2PMaxPush] = {};
+    int p2p_nsend = 0, p2p_nrecv = 0;
+    unsigned long long* p2p_peer_ready[pepp::k::kP2PMaxPeers] = {};
+    unsigned long long* p2p_peer_arrive[pepp::k::kP2PMaxPeers] = {};
+    unsigned long long* p2p_my_ready[pepp::k::kP2PMaxPeers] = {};
+    unsigned long long* p2p_my_arrive[pepp::k::kP2PMaxPeers] = {};
+    int p2p_grid = 1;
+    unsigned long long p2p_timeout_ns = 20ull * 1000 * 1000 * 1000;
+
     // plan-owned x / y for pepp_spmv_exec_host (allocated on first use)
     void* d_hx = nullptr;
     void* d_hy = nullptr;
@@ -176,7 +198,11 @@ namespace {
 #define PEPP_CUDA_TRY(expr)                                   \
     do {                                                      \
         cudaError_t _e = (expr);                              \
-        if (_e != cudaSuccess) { (void)cudaGetLastError(); return PEPP_E_CUDA; } \
+        if (_e != cudaSuccess) {                              \
+            pepp::set_last_error(cudaGetErrorString(_e), #expr, __LINE__); \
+            (void)cudaGetLastError();                         \
+            return PEPP_E_CUDA;                               \
+        }                                                     \
     } while (0)
 
 // Every entry point works on the plan's device and leaves the caller's
@@ -201,7 +227,7 @@ pepp_status_t dalloc_bytes(pepp_spmv_plan_t* p, void** ptr, int64_t bytes) {
     *ptr = nullptr;
     if (bytes <= 0) bytes = 8;
     cudaError_t e = cudaMalloc(ptr, (size_t)bytes);
-    if (e != cudaSuccess) { (void)cudaGetLastError(); *ptr = nullptr; return e == cudaErrorMemoryAllocation ? PEPP_E_NOMEM : PEPP_E_CUDA; }
+    if (e != cudaSuccess) { pepp::set_last_error(cudaGetErrorString(e), "cudaMalloc", __LINE__); (void)cudaGetLastError(); *ptr = nullptr; return e == cudaErrorMemoryAllocation ? PEPP_E_NOMEM : PEPP_E_CUDA; }
     p->dev_bytes += bytes;
     return PEPP_OK;
 }
@@ -224,7 +250,7 @@ pepp_status_t dalloc(pepp_spmv_plan_t* p, T** ptr, int64_t n) {
     *ptr = nullptr;
     if (n <= 0) n = 1;
     cudaError_t e = cudaMalloc((void**)ptr, sizeof(T) * (size_t)n);
-    if (e != cudaSuccess) { (void)cudaGetLastError(); *ptr = nullptr; return e == cudaErrorMemoryAllocation ? PEPP_E_NOMEM : PEPP_E_CUDA; }
+    if (e != cudaSuccess) { pepp::set_last_error(cudaGetErrorString(e), "cudaMalloc", __LINE__); (void)cudaGetLastError(); *ptr = nullptr; return e == cudaErrorMemoryAllocation ? PEPP_E_NOMEM : PEPP_E_CUDA; }
     p->dev_bytes += (int64_t)sizeof(T) * n;
     return PEPP_OK;
 }
@@ -239,6 +265,10 @@ void free_plan(pepp_spmv_plan_t* p) {
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
     for (auto& r : p->ring) { if (r.start) cudaEventDestroy(r.start); if (r.stop) cudaEventDestroy(r.stop); }
+    for (void* m : p->p2p_opened) cudaIpcCloseMemHandle(m);
+    for (void* b : p->p2p_buf) if (b) cudaFree(b);
+    if (p->d_sig) cudaFree(p->d_sig);
+    if (p->h_err) cudaFreeHost(p->h_err);
     if (p->comm && p->own_comm && p->nccl) p->nccl->CommDestroy(p->comm);
     if (p->hist) pepp::history_free(p->hist);
     for (auto* q : p->sub) free_plan(q);
@@ -948,7 +978,13 @@ pepp_status_t setup_halo(pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts
         if (scount[q]) {
             std::vector<int32_t> sl(scount[q]);
             PEPP_CUDA_TRY(cudaMemcpy(sl.data(), d_s[q].p, sizeof(int) * scount[q], cudaMemcpyDeviceToHost));
-            for (int32_t v : sl) p->send_local.push_back((int64_t)v - p->row_offset);
+            int64_t lo = INT64_MAX, hi = INT64_MIN;
+            for (int32_t v : sl) {
+                p->send_local.push_back((int64_t)v - p->row_offset);
+                lo = std::min<int64_t>(lo, (int64_t)v - p->row_offset);
+                hi = std::max<int64_t>(hi, (int64_t)v - p->row_offset + 1);
+            }
+            p->send_rng.push_back({q, lo, hi});
             pepp_status_t s = make(q, sl, d_s[q], p->send_x);
             if (s) return s;
         }
@@ -1029,6 +1065,180 @@ pepp_status_t setup_overlap(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp
     p->info.overlap_head = h;
     p->info.overlap_tail = t;
     return PEPP_OK;
+}
+
+// ---------------------------------------------------------------- P2P
+// Fused peer-memory halo (pepp_spmv_p2p_buffers): symmetric buffers and a
+// signal block per rank, exported with CUDA IPC, their handles all-gathered
+// over the plan's communicator (grouped broadcasts of bytes), the peers' ones
+// opened (cudaIpcMemLazyEnablePeerAccess: NVLink / NVSwitch mappings).
+struct P2PHandles {
+    cudaIpcMemHandle_t buf[kP2PMaxBuf];
+    cudaIpcMemHandle_t sig;
+    int64_t ok;                              // 1 = this rank's export succeeded
+};
+
+// max over ranks of v (an all-reduce that doubles as a barrier)
+pepp_status_t nccl_allmax(pepp_spmv_plan_t* p, cudaStream_t st, int64_t* v) {
+    DevTmp<int64_t> d;
+    PEPP_CUDA_TRY(d.alloc(1));
+    PEPP_CUDA_TRY(cudaMemcpyAsync(d.p, v, sizeof(int64_t), cudaMemcpyHostToDevice, st));
+    if (p->nccl->AllReduce(d.p, d.p, 1, pepp::NCCL_INT64, pepp::NCCL_OP_MAX, p->comm, st)) return PEPP_E_NCCL;
+    PEPP_CUDA_TRY(cudaMemcpyAsync(v, d.p, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    return PEPP_OK;
+}
+
+pepp_status_t nccl_barrier(pepp_spmv_plan_t* p, cudaStream_t st) {
+    int64_t v = 0;
+    return nccl_allmax(p, st, &v);
+}
+
+// this rank's half: buffers, signal block, error flag, IPC export
+pepp_status_t p2p_export(pepp_spmv_plan_t* p, int nbuf, cudaStream_t st, P2PHandles* mine) {
+    const int P = p->opts.nranks;
+    pepp_status_t s;
+    // symmetric buffers + signal block (zeroed before any peer can see them)
+    for (int b = 0; b < nbuf; ++b) {
+        if ((s = dalloc_bytes(p, &p->p2p_buf[b], p->global_rows * (int64_t)p->esz))) return s;
+        PEPP_CUDA_TRY(cudaMemsetAsync(p->p2p_buf[b], 0, p->global_rows * p->esz, st));
+    }
+    if ((s = dalloc(p, &p->d_sig, 2 * (int64_t)P + 2))) return s;
+    PEPP_CUDA_TRY(cudaMemsetAsync(p->d_sig, 0, sizeof(unsigned long long) * (2 * P + 2), st));
+    PEPP_CUDA_TRY(cudaHostAlloc((void**)&p->h_err, sizeof(int), cudaHostAllocMapped));
+    *p->h_err = 0;
+    PEPP_CUDA_TRY(cudaHostGetDevicePointer((void**)&p->d_err, p->h_err, 0));
+    for (int b = 0; b < nbuf; ++b) PEPP_CUDA_TRY(cudaIpcGetMemHandle(&mine->buf[b], p->p2p_buf[b]));
+    PEPP_CUDA_TRY(cudaIpcGetMemHandle(&mine->sig, p->d_sig));
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    mine->ok = 1;
+    return PEPP_OK;
+}
+
+// map the send-peers' buffers and signal blocks; build the push ranges
+pepp_status_t p2p_import(pepp_spmv_plan_t* p, int nbuf, const std::vector<P2PHandles>& all) {
+    const int P = p->opts.nranks, me = p->opts.rank;
+    std::vector<int> sendp, recvp;   // peers this rank writes to (its send list) / receives from
+    for (auto& t : p->send_x) if (t.count) sendp.push_back(t.peer);
+    for (auto& t : p->recv_x) if (t.count) recvp.push_back(t.peer);
+    std::sort(sendp.begin(), sendp.end());
+    sendp.erase(std::unique(sendp.begin(), sendp.end()), sendp.end());
+    std::sort(recvp.begin(), recvp.end());
+    recvp.erase(std::unique(recvp.begin(), recvp.end()), recvp.end());
+    if ((int)sendp.size() > pepp::k::kP2PMaxPeers || (int)recvp.size() > pepp::k::kP2PMaxPeers) return PEPP_E_UNSUPPORTED;
+    std::vector<std::vector<void*>> peer_buf(P);
+    for (size_t j = 0; j < sendp.size(); ++j) {
+        const int q = sendp[j];
+        peer_buf[q].assign(nbuf, nullptr);
+        for (int b = 0; b < nbuf; ++b) {
+            PEPP_CUDA_TRY(cudaIpcOpenMemHandle(&peer_buf[q][b], all[q].buf[b], cudaIpcMemLazyEnablePeerAccess));
+            p->p2p_opened.push_back(peer_buf[q][b]);
+        }
+        void* sig = nullptr;
+        PEPP_CUDA_TRY(cudaIpcOpenMemHandle(&sig, all[q].sig, cudaIpcMemLazyEnablePeerAccess));
+        p->p2p_opened.push_back(sig);
+        auto* qs = (unsigned long long*)sig;
+        p->p2p_peer_ready[j] = qs + me;            // q's ready[me]
+        p->p2p_peer_arrive[j] = qs + P + me;       // q's arrive[me]
+        p->p2p_my_ready[j] = p->d_sig + q;         // my ready[q]
+    }
+    for (size_t j = 0; j < recvp.size(); ++j) p->p2p_my_arrive[j] = p->d_sig + P + recvp[j];
+    p->p2p_nsend = (int)sendp.size();
+    p->p2p_nrecv = (int)recvp.size();
+    // push ranges: each peer's send range cut to the head and the tail segments
+    const int64_t R = p->nrows, h = p->info.overlap_head, t = p->info.overlap_tail;
+    int np = 0;
+    for (auto& sr : p->send_rng) {
+        for (int seg = 0; seg < 2; ++seg) {
+            const int64_t lo = std::max(sr.lo, seg ? R - t : 0), hi = std::min(sr.hi, seg ? R : h);
+            if (lo >= hi) continue;
+            if (np == pepp::k::kP2PMaxPush) return PEPP_E_UNSUPPORTED;
+            p->p2p_push_lo[np] = lo;
+            p->p2p_push_hi[np] = hi;
+            for (int b = 0; b < nbuf; ++b) p->p2p_push_dst[b][np] = peer_buf[sr.peer][b];
+            ++np;
+        }
+    }
+    p->p2p_npush = np;
+    p->p2p_grid = (int)std::max<int64_t>(1, std::min<int64_t>((h + t + 255) / 256, 8 * kReserveSms));
+    return PEPP_OK;
+}
+
+// Collective on every path: a rank whose export or import fails still takes
+// part in the handle all-gather and the final agreement, so no peer is left
+// waiting inside a collective; every rank returns an error if any failed.
+pepp_status_t p2p_register(pepp_spmv_plan_t* p, int nbuf, cudaStream_t st) {
+    const int P = p->opts.nranks, me = p->opts.rank;
+    std::vector<P2PHandles> all(P);
+    std::memset(all.data(), 0, sizeof(P2PHandles) * P);
+    pepp_status_t s = p2p_export(p, nbuf, st, &all[me]);
+    // all-gather the IPC handles (bytes) over the plan's communicator
+    DevTmp<unsigned char> d_h;
+    PEPP_CUDA_TRY(d_h.alloc(sizeof(P2PHandles) * P));
+    PEPP_CUDA_TRY(cudaMemcpyAsync(d_h.p, all.data(), sizeof(P2PHandles) * P, cudaMemcpyHostToDevice, st));
+    if (p->nccl->GroupStart()) return PEPP_E_NCCL;
+    for (int r = 0; r < P; ++r) {
+        unsigned char* at = d_h.p + sizeof(P2PHandles) * r;
+        if (p->nccl->Broadcast(at, at, sizeof(P2PHandles), pepp::NCCL_INT8, r, p->comm, st)) { p->nccl->GroupEnd(); return PEPP_E_NCCL; }
+    }
+    if (p->nccl->GroupEnd()) return PEPP_E_NCCL;
+    PEPP_CUDA_TRY(cudaMemcpyAsync(all.data(), d_h.p, sizeof(P2PHandles) * P, cudaMemcpyDeviceToHost, st));
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    bool all_ok = true;
+    for (int r = 0; r < P; ++r) all_ok &= all[r].ok == 1;
+    if (std::getenv("PEPP_DEBUG"))
+        for (int r = 0; r < P; ++r)
+            std::fprintf(stderr, "[pepp p2p] rank %d: slot %d ok=%lld first bytes %02x%02x%02x%02x local status %d\n", me, r,
+                         (long long)all[r].ok, (unsigned char)all[r].sig.reserved[0], (unsigned char)all[r].sig.reserved[1],
+                         (unsigned char)all[r].sig.reserved[2], (unsigned char)all[r].sig.reserved[3], (int)s);
+    if (!s && all_ok) s = p2p_import(p, nbuf, all);
+    else if (!s) { s = PEPP_E_CUDA; pepp::set_last_error("a peer rank could not export its buffers", "p2p_register", __LINE__); }
+    if (const char* e = std::getenv("PEPP_P2P_TIMEOUT_MS")) p->p2p_timeout_ns = 1000000ull * (unsigned long long)std::atoll(e);
+    // agreement (and the barrier after which pushes may start: every rank has
+    // mapped its peers and zeroed its flags)
+    int64_t fail = s ? 1 : 0;
+    pepp_status_t sb = nccl_allmax(p, st, &fail);
+    if (s) return s;
+    if (sb) return sb;
+    if (fail) { pepp::set_last_error("a peer rank could not map its peers' buffers", "p2p_register", __LINE__); return PEPP_E_CUDA; }
+    p->p2p_nbuf = nbuf;
+    return PEPP_OK;
+}
+
+template <typename T>
+pepp_status_t p2p_launch_t(pepp_spmv_plan_t* p, int b, const T* x, T* y, cudaStream_t st) {
+    pepp::k::P2PArgs<T> a{};
+    const int64_t R = p->nrows, h = p->info.overlap_head, t = p->info.overlap_tail;
+    a.seg_lo[0] = 0; a.seg_hi[0] = h;
+    a.seg_lo[1] = R - t; a.seg_hi[1] = R;
+    a.row_offset = p->row_offset;
+    a.npush = p->p2p_npush;
+    for (int j = 0; j < a.npush; ++j) {
+        a.push_lo[j] = p->p2p_push_lo[j];
+        a.push_hi[j] = p->p2p_push_hi[j];
+        a.push_dst[j] = (T*)p->p2p_push_dst[b][j];
+    }
+    a.nsend = p->p2p_nsend;
+    for (int j = 0; j < a.nsend; ++j) {
+        a.peer_ready[j] = p->p2p_peer_ready[j];
+        a.peer_arrive[j] = p->p2p_peer_arrive[j];
+        a.my_ready[j] = p->p2p_my_ready[j];
+    }
+    a.nrecv = p->p2p_nrecv;
+    for (int j = 0; j < a.nrecv; ++j) a.my_arrive[j] = p->p2p_my_arrive[j];
+    const int P = p->opts.nranks;
+    a.epoch = p->d_sig + 2 * P;
+    a.done = (unsigned int*)(p->d_sig + 2 * P + 1);
+    a.err = p->d_err;
+    a.timeout_ns = p->p2p_timeout_ns;
+    pepp::k::halo_push_kernel<T><<<p->p2p_grid, 256, 0, st>>>(p->d_rp, p->d_col, (const T*)p->d_val, x, y, a);
+    return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
+}
+
+// index of the registered buffer y points to, -1 if none
+int p2p_index(const pepp_spmv_plan_t* p, const void* y) {
+    for (int b = 0; b < p->p2p_nbuf; ++b) if (p->p2p_buf[b] == y) return b;
+    return -1;
 }
 
 pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spmv_plan_t* p) {
@@ -1298,15 +1508,23 @@ pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flag
     // interior first (the host may block inside a synchronous exchange)
     pepp_choice_t u{};
     pepp_status_t s = pepp_spmv_exec(p->sub[1], x, yb + p->sub_r0[1] * (int64_t)p->esz, sf, st, nullptr, &u);
-    for (int i : {0, 2})
-        if (!s && p->sub[i])
-            s = pepp_spmv_exec(p->sub[i], x, yb + p->sub_r0[i] * (int64_t)p->esz, sf, p->side, nullptr, nullptr);
-    if (!s) s = exchange_halo(p, y, p->side);
+    const int b = p2p_index(p, y);
+    if (b >= 0) {
+        // fused: head + tail rows computed, pushed into the peers' buffer b and
+        // signalled by one kernel (PEPP_X_P2P)
+        if (!s) s = p->vt == PEPP_VALUE_F32 ? p2p_launch_t<float>(p, b, (const float*)x, (float*)y, p->side)
+                                            : p2p_launch_t<double>(p, b, (const double*)x, (double*)y, p->side);
+    } else {
+        for (int i : {0, 2})
+            if (!s && p->sub[i])
+                s = pepp_spmv_exec(p->sub[i], x, yb + p->sub_r0[i] * (int64_t)p->esz, sf, p->side, nullptr, nullptr);
+        if (!s) s = exchange_halo(p, y, p->side);
+    }
     PEPP_CUDA_TRY(cudaEventRecord(p->ev_join, p->side));   // join whatever reached the side stream
     PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_join, 0));
     if (s) return s;
     u.nparts = p->opts.nranks;
-    u.exchange = PEPP_X_HALO;
+    u.exchange = b >= 0 ? PEPP_X_P2P : PEPP_X_HALO;
     if (used) *used = u;
     return PEPP_OK;
 }
@@ -1355,6 +1573,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         const char *yb = (const char*)y, *ye = yb + p->global_rows * (int64_t)p->esz;
         if (xb < ye && yb < xe) return PEPP_E_INVALID;
     }
+    if (p->h_err && *(volatile int*)p->h_err) return p->sticky = PEPP_E_NCCL;   // a peer never arrived (P2P)
     cudaStream_t st = (cudaStream_t)stream;
     DeviceScope dscope(p->device);
     if (!dscope.ok) return PEPP_E_CUDA;
@@ -1578,9 +1797,36 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_destroy(pepp_spmv_plan_t* p) {
     cudaDeviceSynchronize();
     (void)cudaGetLastError();
     pepp_status_t s = PEPP_OK;
+    if (p->p2p_nbuf && p->nccl && p->comm) {   // peers may still write into this rank's buffers
+        cudaStream_t st = nullptr;
+        if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) == cudaSuccess) {
+            s = nccl_barrier(p, st);
+            cudaStreamDestroy(st);
+        }
+        (void)cudaGetLastError();
+    }
     if (!p->history_path.empty() && p->hist) s = pepp_history_save(p->hist, p->history_path.c_str());
     free_plan(p);
     return s;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_spmv_p2p_buffers(pepp_spmv_plan_t* p, int32_t nbuf, void** bufs) {
+    if (!p || !bufs || nbuf < 1 || nbuf > kP2PMaxBuf) return PEPP_E_INVALID;
+    if (p->sticky) return p->sticky;
+    if (p->p2p_nbuf) return PEPP_E_STATE;
+    if (p->opts.nranks < 2 || p->exchange != PEPP_X_HALO || !p->sub[1]) return PEPP_E_UNSUPPORTED;
+    DeviceScope dscope(p->device);
+    if (!dscope.ok) { pepp::set_last_error("cannot select the plan's device", "DeviceScope", __LINE__); return PEPP_E_CUDA; }
+    cudaStream_t st = nullptr;
+    PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+    pepp_status_t s = p2p_register(p, nbuf, st);
+    cudaStreamDestroy(st);
+    if (s) { p->sticky = s; return s; }
+    for (int b = 0; b < nbuf; ++b) bufs[b] = p->p2p_buf[b];
+    p->info.p2p_buffers = nbuf;
+    p->info.device_bytes = p->dev_bytes;
+    for (auto* q : p->sub) if (q) p->info.device_bytes += q->dev_bytes;
+    return PEPP_OK;
 }
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_plan_info(const pepp_spmv_plan_t* p, pepp_plan_info_t* out) {

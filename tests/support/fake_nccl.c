@@ -187,6 +187,10 @@ static int flush(Comm* c) {
             arc += o->bytes;
         }
     }
+    /* pageable H2D cudaMemcpy may return before its DMA lands: make the data
+       visible to work the caller enqueues next on any stream (real NCCL
+       orders it on the op's stream) */
+    if (cudaDeviceSynchronize() != cudaSuccess) return 1;
     barrier(c);
     c->nops = 0;
     return cudaGetLastError() == cudaSuccess ? 0 : 1;

@@ -2,8 +2,8 @@
 ranks, gloo for torch.distributed, the library pointed at the NCCL stand-in
 (tests/support/fake_nccl.c) and every rank on device 0 (test-only knobs
 PEPP_BENCH_ONE_DEVICE / PEPP_BENCH_DIST_BACKEND). Checks the contract, not
-the numbers: exactly one JSON line from rank 0, n_gpus = 2, the halo
-exchange resolved, the max-over-ranks timing and the e2e leg present."""
+the numbers: exactly one JSON line from rank 0, n_gpus = 2, the fused
+peer-memory halo (PEPP_X_P2P) in use, the max-over-ranks timing and the e2e leg present."""
 from __future__ import annotations
 
 import json
@@ -41,8 +41,9 @@ def test_bench_two_ranks_one_gpu():
     assert len(lines) == 1, out.stdout[-2000:]
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["steps"] == 1 and d["value"] > 0
-    assert d["config"]["exchange"] == "halo"
-    # rank 0's block sends its last grid row: tail + interior kernels per SpMV, exchange overlapped
+    # halo pushed by the fused boundary kernel into the peer's buffer (PEPP_X_P2P, CUDA IPC on one device)
+    assert d["config"]["exchange"].startswith("p2p")
+    # rank 0's block sends its last grid row: interior kernel + the fused tail/push kernel per SpMV
     assert d["plan"]["overlap"] == 1 and d["plan"]["overlap_head"] == 0 and d["plan"]["overlap_tail"] == 2048
     assert d["e2e"]["value"] > 0 and d["gpu_launches"] >= 200
     assert "launch_includes" in d["roofline"]

@@ -107,11 +107,16 @@ def _run(name, exchange, K=6, f32=False, overlap=True):
     for p in procs:
         p.start()
     out = {}
-    for _ in range(2):
-        r, res = q.get(timeout=300)
-        out[r] = res
-    for p in procs:
-        p.join(timeout=60)
+    try:
+        for _ in range(2):
+            r, res = q.get(timeout=300)
+            out[r] = res
+    finally:   # never leave a worker (and its GPU context) behind
+        for p in procs:
+            p.join(timeout=60)
+            if p.is_alive():
+                p.kill()
+                p.join(10)
     for r in range(2):
         assert "error" not in out[r], out[r]["error"]
     return out
@@ -168,3 +173,119 @@ def test_real_nccl_selftest():
     with open("/proc/self/maps") as f:
         maps = f.read()
     assert "libnccl" in maps and "fake_nccl" not in maps
+
+
+# ---------------------------------------------------------------- fused peer-memory halo (PEPP_X_P2P)
+def _worker_p2p(rank, world, lib, uid, name, K, outq, f32=False, real=False):
+    os.environ["PEPP_NCCL_LIB"] = lib
+    try:
+        import sys
+        sys.path.insert(0, os.path.dirname(HERE))
+        import torch
+
+        import gen
+        import oracle
+        import paper_conf_sc_dastgeerlk12_b200 as pepp
+        torch.cuda.set_device(0)
+        A = _matrix(name)
+        if real:
+            A = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, gen.vector(77, gen.REAL, A.nnz), A.r0, A.global_nrows)
+        n = A.nrows
+        bounds = pepp.partition_rows(A.row_ptr, world)
+        r0, r1 = int(bounds[rank]), int(bounds[rank + 1])
+        dt = np.float32 if f32 else np.float64
+        Ad = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(dt), A.r0, A.global_nrows)
+        blk = gen.row_block(Ad, r0, r1)
+        x0 = (gen.vector(5, gen.REAL, n) if real else gen.vector(3, gen.INT8, n)).astype(dt)
+        res = {}
+        with pepp.Plan.from_csr(blk, nranks=world, rank=rank, row_bounds=bounds, nccl_unique_id=uid,
+                                exchange=pepp.X_HALO) as plan:
+            info = plan.info()
+            bufs = plan.p2p_buffers(2)
+            res["p2p_buffers"] = plan.info()["p2p_buffers"]
+            bufs[0].copy_(torch.from_numpy(x0).cuda())
+            bufs[1].fill_(float("nan"))          # every ghost must come from a peer's push
+            torch.cuda.synchronize()
+            src, dst = bufs[0], bufs[1]
+            used = set()
+            xs = [x0.astype(np.float64)]
+            for k in range(K):
+                u = plan.exec(src, dst, flags=pepp.Y_NEXT_INPUT)
+                used.add(u.exchange)
+                torch.cuda.synchronize()
+                xs.append(dst.cpu().numpy().astype(np.float64))
+                src, dst = dst, src
+            res["used"] = sorted(used)
+            # what this rank reads next: own rows + the ghosts its rows reference
+            _, ghosts = pepp.halo_ghosts(blk.col, world, rank, bounds)
+            rows = np.concatenate([np.arange(r0, r1), ghosts.astype(np.int64)])
+            A64 = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, Ad.val.astype(np.float64))
+            if not real:   # integer-valued: exact, bit for bit
+                ref = xs[0]
+                ok = True
+                for k in range(1, K + 1):
+                    ref = oracle.spmv(A64, ref) if not f32 else oracle.spmv_f32(A64, ref.astype(np.float32)).astype(np.float64)
+                    ok &= bool(np.array_equal(xs[k][rows], ref[rows]))
+                res["ok"] = ok
+            else:          # real: every step within the north-star bound of the oracle applied to the GPU's own x_{k-1}
+                ok = True
+                for k in range(1, K + 1):
+                    xp = xs[k - 1].copy()
+                    xp[~np.isfinite(xp)] = 0.0   # never read: rows outside own + ghosts
+                    ref, tol = oracle.spmv(A64, xp), oracle.bound(A64, xp)
+                    ok &= bool(np.all(np.abs(xs[k][r0:r1] - ref[r0:r1]) <= tol[r0:r1]))
+                res["ok"] = ok
+            # the ghosts pushed into this rank == the owner's own rows, bit for bit (checked by the caller)
+            res["own"] = (r0, xs[K][r0:r1])
+            res["ghosts"] = (ghosts.astype(np.int64), xs[K][ghosts.astype(np.int64)])
+            res["overlap"] = (info["overlap"], info["overlap_head"], info["overlap_tail"])
+        outq.put((rank, res))
+    except Exception as e:
+        import traceback
+        outq.put((rank, {"error": repr(e) + traceback.format_exc()}))
+
+
+def _run_p2p(name, K=6, f32=False, real=False):
+    import torch.multiprocessing as mp
+    lib = _build_fake()
+    uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_p2p_{int(f32)}{int(real)}".encode() + b"\0" * 128)[:128]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker_p2p, args=(r, 2, lib, uid, name, K, q, f32, real)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = {}
+    try:
+        for _ in range(2):
+            r, res = q.get(timeout=300)
+            out[r] = res
+    finally:   # never leave a worker (and its GPU context) behind
+        for p in procs:
+            p.join(timeout=60)
+            if p.is_alive():
+                p.kill()
+                p.join(10)
+    for r in range(2):
+        assert "error" not in out[r], out[r]["error"]
+    return out
+
+
+@pytest.mark.parametrize("name,f32,real", [("lap", False, False), ("banded", False, False), ("lap", True, False),
+                                           ("lap", False, True)])
+def test_two_ranks_p2p_fused_halo(name, f32, real):
+    """pepp_spmv_p2p_buffers + PEPP_Y_NEXT_INPUT calls: the boundary rows are
+    computed, pushed into the peer's buffer over CUDA-IPC peer memory and
+    signalled by one kernel (halo_push_kernel) — no NCCL on the data path.
+    Two processes on one GPU (IPC within a device); NaN-initialised output
+    buffers, so every ghost must have been pushed. Integer inputs: own rows +
+    ghosts bit-exact vs the oracle after every iteration; real inputs: within
+    the north-star bound per step."""
+    import paper_conf_sc_dastgeerlk12_b200 as pepp
+    out = _run_p2p(name, f32=f32, real=real)
+    for r in range(2):
+        assert out[r]["ok"], (r, out[r]["used"])
+        gi, gv = out[r]["ghosts"]
+        o0, ov = out[1 - r]["own"]
+        assert len(gi) > 0 and np.array_equal(gv, ov[gi - o0])   # what arrived is what the owner computed
+        assert out[r]["used"] == [pepp.X_P2P], out[r]
+        assert out[r]["p2p_buffers"] == 2
