@@ -148,22 +148,23 @@ def measured_peak() -> tuple[float, str]:
         return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-def traffic_for(kernel: str, workload: str):
-    """dram read+write bytes per launch from the committed ncu --set full summary, if any."""
+def traffic_for(kernel: str, workload: str, dtype: str = "f64"):
+    """dram read+write bytes per launch from the committed ncu --set full
+    summary, if any (entries are per workload and fp64 unless keyed 'name:f32')."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     try:
         d = json.load(open(p))
-        return d.get(workload, {}).get(kernel)
+        return d.get(workload, {}).get(kernel if dtype == "f64" else f"{kernel}:{dtype}")
     except (OSError, ValueError):
         return None
 
 
-def roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, workload) -> dict:
+def roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, workload, dtype="f64") -> dict:
     """Roofline of the dominant kernel: algorithmic bytes / launch time vs the
     measured peak; `traffic` = ncu DRAM bytes per launch (may be below the
     algorithmic bytes when the variant stores a compressed layout, e.g. SELL
     16-bit column deltas), with the DRAM-traffic fraction beside it."""
-    traffic = traffic_for(kname, workload)
+    traffic = traffic_for(kname, workload, dtype)
     d = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "peak_source": peak_src,
          "unit": "GB/s", "frac": round(achieved / peak, 4), "avg_launch_us": round(avg_kernel_s * 1e6, 2),
          "bytes_per_launch": local_bytes, "traffic": traffic}
@@ -220,6 +221,38 @@ def host_cpu() -> dict:
     return {"model": model, "sockets": len(sockets) or None, "nproc": os.cpu_count()}
 
 
+def library_baseline(A, xs, stream, iterated, flush, ours_us: float) -> dict:
+    """cuSPARSE CSR SpMV (through torch.sparse_csr_tensor @ x) on the same
+    matrix and x, timed with CUDA events on the same stream: context for the
+    hand-written kernels, never on the product path."""
+    import torch
+    dev = xs.device
+    it = torch.int32 if A.nnz < (1 << 31) - 1 else torch.int64
+    crow = torch.from_numpy(A.row_ptr - A.row_ptr[0]).to(device=dev, dtype=it)
+    col = torch.from_numpy(A.col).to(device=dev, dtype=it)
+    val = torch.from_numpy(A.val).to(dev)
+    M = torch.sparse_csr_tensor(crow, col, val, size=(A.nrows, A.ncols))
+    del crow, col, val
+    n = 10 if A.nnz > 10_000_000 else 50
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
+    with torch.cuda.stream(stream):
+        y = M @ xs   # warm-up (cuSPARSE buffer + analysis)
+        for a, b in ev:
+            if flush is not None:
+                flush.zero_()
+            a.record(stream)
+            y = M @ xs
+            b.record(stream)
+    stream.synchronize()
+    us = statistics.median(a.elapsed_time(b) for a, b in ev) * 1e3
+    del M, y
+    torch.cuda.empty_cache()
+    return {"name": "cuSPARSE CSR SpMV (torch.sparse_csr_tensor @ x, torch " + torch.__version__ + ")",
+            "us_per_spmv": round(us, 2), "gflops": round(2.0 * A.nnz / (us * 1e-6) / 1e9, 3),
+            "speedup_ours": round(us / ours_us, 3),
+            "note": "same matrix / x / stream, median of %d calls%s" % (n, "" if flush is None else ", L2 flushed")}
+
+
 def value_compressed_leg(args, A, xs, bufs, stream, iters, iterated, flush, peak):
     """The same SpMVs with opts.compress_values = 1: SELL chunks whose 32 rows
     share their column offsets and whose slots hold one constant value per
@@ -265,7 +298,7 @@ def value_compressed_leg(args, A, xs, bufs, stream, iters, iterated, flush, peak
         avg_s = statistics.mean(ms) / 1e3
         chosen = max(used, key=used.get)
         kname = chosen + ("+constval" if chosen.startswith("sell") else "")
-        traffic = traffic_for(kname, args.workload)
+        traffic = traffic_for(kname, args.workload, args.dtype)
         d = {"applies": True, "kernel": kname, "constval_frac": info["sell_constval_frac"],
              "avg_launch_us": round(avg_s * 1e6, 2), "gflops": round(2.0 * A.nnz / avg_s / 1e9, 3),
              "traffic": traffic, "choices": used,
@@ -467,6 +500,14 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     if world == 1 and not args.value_compression and force is None and not args.no_vc_leg:
         vc = value_compressed_leg(args, A, xs, bufs, stream, iters, iterated, flush, peak)
 
+    # ---- cuSPARSE on the same matrix (context, not the product path) ----
+    lib_base = None
+    if world == 1 and not args.no_library:
+        try:
+            lib_base = library_baseline(A, xs, stream, iterated, flush, avg_kernel_s * 1e6)
+        except Exception as e:   # context only: never fail the bench line over it
+            lib_base = {"unavailable": repr(e)[:200]}
+
     # ---- selector quality: every candidate timed after the timed region (same run) ----
     sel = None
     if not args.no_sweep:
@@ -549,7 +590,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
                        "variant": args.variant or "auto (history-based per call)"},
             "hbm": {"achieved_gbs": round(gbs, 1), "frac_of_measured": round(gbs / (world * peak), 4),
                     "frac_of_8tbs": round(gbs / (world * 8000.0), 4), "algorithmic_bytes_per_spmv": alg_bytes_global},
-            "roofline": dict(roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, args.workload),
+            "roofline": dict(roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, args.workload, args.dtype),
                              **({"launch_includes": "interior kernel + the fused boundary/push kernel (P2P halo)"
                                  if p2p else "head + interior + tail kernels and the overlapped halo exchange"}
                                 if overlapped else {})),
@@ -560,6 +601,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             "graph": graph_info,
             "selector": sel,
             "value_compressed": vc,
+            "library_baseline": lib_base,
             "clocks": clk,
             "cpu_baseline": cpu,
             "plan": {k: info[k] for k in ("mean_row", "cv_row", "max_row", "sell_sigma", "sell_fill",
@@ -590,6 +632,7 @@ def main():
                          "streamed and the compressed plan is reported separately under 'value_compressed'")
     ap.add_argument("--no-value-compression", action="store_true", help=argparse.SUPPRESS)   # the default now
     ap.add_argument("--no-vc-leg", action="store_true", help="skip the value-compressed leg")
+    ap.add_argument("--no-library", action="store_true", help="skip the cuSPARSE context measurement")
     ap.add_argument("--no-p2p", action="store_true",
                     help="N > 1: NCCL halo per iteration instead of the fused peer-memory push (PEPP_X_P2P)")
     ap.add_argument("--dtype", choices=["f64", "f32"], default="f64",

@@ -38,7 +38,8 @@ class INFO_T(ctypes.Structure):
                 ("exchange", c_i32), ("halo_recv", c_i64), ("halo_send", c_i64), ("sell_col16_frac", c_f64),
                 ("prior_key", c_u64), ("sell_stencil_frac", c_f64),
                 ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64), ("predicted", c_i32),
-                ("sell_constval_frac", c_f64), ("p2p_buffers", c_i32)]
+                ("sell_constval_frac", c_f64), ("p2p_buffers", c_i32),
+                ("sell_long_rows", c_i64)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}

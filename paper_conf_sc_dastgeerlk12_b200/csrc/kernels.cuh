@@ -1001,11 +1001,14 @@ __global__ void col_check_kernel(int64_t n, const int* __restrict__ col, int64_t
 
 // SELL conversion -----------------------------------------------------
 // key for the σ-window sort: (window, descending length, row) packed in 64 bits
-__global__ void sell_keys_kernel(int nrows, const int* __restrict__ rp, int sigma, int maxlen,
+// Rows longer than `cap` are left out of the SELL layout (length 0 there) and
+// summed by sell_long_kernel instead (hybrid SELL for heavy-tailed rows).
+__global__ void sell_keys_kernel(int nrows, const int* __restrict__ rp, int sigma, int maxlen, int cap,
                                  unsigned long long* __restrict__ keys, int* __restrict__ rows) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= nrows) return;
-    const int len = rp[i + 1] - rp[i];
+    int len = rp[i + 1] - rp[i];
+    if (len > cap) len = 0;
     const unsigned long long win = (unsigned long long)(i / sigma);
     keys[i] = (win << 32) | (unsigned long long)(maxlen - len);
     rows[i] = i;
@@ -1013,7 +1016,7 @@ __global__ void sell_keys_kernel(int nrows, const int* __restrict__ rp, int sigm
 
 // sorted position r -> original row perm[r]; lengths + per-chunk max
 // chunk_len[c] = max length, | kSellMasked unless all 32 rows exist with that length
-__global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,
+__global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm, int cap,
                                     int* __restrict__ rowlen, int* __restrict__ chunk_len) {
     const int r = blockIdx.x * blockDim.x + threadIdx.x;
     const int lane = threadIdx.x & 31;
@@ -1021,6 +1024,7 @@ __global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const
     if (r < nrows) {
         const int o = perm ? perm[r] : r;
         len = rp[o + 1] - rp[o];
+        if (len > cap) len = 0;
         rowlen[r] = len;
     }
     int mx = len, mn = len;
@@ -1033,7 +1037,7 @@ __global__ void sell_lengths_kernel(int nrows, const int* __restrict__ rp, const
 }
 
 template <typename T>
-__global__ void sell_fill_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm,
+__global__ void sell_fill_kernel(int nrows, const int* __restrict__ rp, const int* __restrict__ perm, int cap,
                                  const int* __restrict__ src_col, const T* __restrict__ src_val,
                                  const int64_t* __restrict__ chunk_ptr, int* __restrict__ col,
                                  T* __restrict__ val) {
@@ -1041,10 +1045,67 @@ __global__ void sell_fill_kernel(int nrows, const int* __restrict__ rp, const in
     if (r >= nrows) return;
     const int o = perm ? perm[r] : r;
     const int s = rp[o], e = rp[o + 1];
+    if (e - s > cap) return;   // a long row: sell_long_kernel's
     const int64_t base = chunk_ptr[r >> 5] + (r & 31);
     for (int k = s; k < e; ++k) {
         col[base + (int64_t)(k - s) * 32] = src_col[k];
         val[base + (int64_t)(k - s) * 32] = src_val[k];
+    }
+}
+
+// Long rows of a hybrid SELL plan (length > cap): segments of up to
+// kSellLongSeg nonzeros, one CTA per segment (seg = {row, k begin, k end,
+// long-row index}; lrow = {first segment, segment count}). Each thread sums a
+// strided subsequence of the segment (coalesced val / col streams, 4 loads
+// in flight), the CTA reduces in a fixed tree, thread 0 stores the segment's
+// partial; the CTA that completes a row's last segment (per-row counter,
+// reset for the next call) adds the row's partials in segment order and
+// writes y. No fp atomics: the result does not depend on scheduling.
+// Launched after sell_kernel, which wrote 0 for these rows.
+constexpr int kSellLongSeg = 4096;
+template <int BLOCK, typename T>
+__global__ void __launch_bounds__(BLOCK) sell_long_kernel(const int4* __restrict__ seg, const int2* __restrict__ lrow,
+                                                          unsigned int* __restrict__ cnt, T* __restrict__ part,
+                                                          const int* __restrict__ col, const T* __restrict__ val,
+                                                          const T* __restrict__ x, T* __restrict__ y) {
+    constexpr int NW = BLOCK / 32;
+    __shared__ T s_w[NW];
+    __shared__ bool s_last;
+    const int4 g = seg[blockIdx.x];
+    const uint64_t pol = evict_first_policy();
+    T a0 = T(0), a1 = T(0), a2 = T(0), a3 = T(0);
+    int k = g.y + threadIdx.x;
+    for (; k + 3 * BLOCK < g.z; k += 4 * BLOCK) {
+        const int c0 = ld_stream_i(col + k, pol), c1 = ld_stream_i(col + k + BLOCK, pol);
+        const int c2 = ld_stream_i(col + k + 2 * BLOCK, pol), c3 = ld_stream_i(col + k + 3 * BLOCK, pol);
+        const T v0 = ld_stream_v(val + k, pol), v1 = ld_stream_v(val + k + BLOCK, pol);
+        const T v2 = ld_stream_v(val + k + 2 * BLOCK, pol), v3 = ld_stream_v(val + k + 3 * BLOCK, pol);
+        a0 = fma(v0, ld_x(x, c0), a0);
+        a1 = fma(v1, ld_x(x, c1), a1);
+        a2 = fma(v2, ld_x(x, c2), a2);
+        a3 = fma(v3, ld_x(x, c3), a3);
+    }
+    for (; k < g.z; k += BLOCK) a0 = fma(ld_stream_v(val + k, pol), ld_x(x, ld_stream_i(col + k, pol)), a0);
+    T acc = (a0 + a1) + (a2 + a3);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = acc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        T t = s_w[0];
+#pragma unroll
+        for (int w = 1; w < NW; ++w) t += s_w[w];
+        part[blockIdx.x] = t;
+        __threadfence();
+        const int2 lr = lrow[g.w];
+        s_last = atomicAdd(cnt + g.w, 1u) == (unsigned)(lr.y - 1);
+        if (s_last) {
+            __threadfence();
+            T r = T(0);
+            for (int j = 0; j < lr.y; ++j) r += __ldcg(part + lr.x + j);
+            y[g.x] = r;
+            cnt[g.w] = 0u;
+        }
     }
 }
 

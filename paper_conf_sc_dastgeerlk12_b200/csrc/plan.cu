@@ -110,6 +110,13 @@ struct pepp_spmv_plan_s {
     int* d_sell_ws = nullptr;    // σ > 1: per-warp ranges of the transposed chunk order, equal slots
     int64_t sell_col16_chunks = 0;
     void* d_sval = nullptr;
+    // hybrid SELL: rows longer than sell_cap are summed by sell_long_kernel
+    int sell_cap = INT32_MAX;
+    int nsell_seg = 0, nsell_long = 0;
+    int4* d_sell_seg = nullptr;      // {row, k begin, k end, long-row index} per segment
+    int2* d_sell_lrow = nullptr;     // {first segment, segments} per long row
+    unsigned int* d_sell_cnt = nullptr;
+    void* d_sell_part = nullptr;     // segment partials (8-byte slots)
 
     // merge path
     int ntiles = 0;
@@ -260,7 +267,8 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
-                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist};
+                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist,
+                    p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, p->d_sell_part};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -387,6 +395,45 @@ pepp_status_t sell_patterns(pepp_spmv_plan_t* p, int64_t nsb, const void* d_scon
     return PEPP_OK;
 }
 
+// Hybrid SELL for heavy-tailed rows: when the longest row exceeds
+// max(kSellCapMin, 32 x mean), rows above that cap leave the SELL layout (one
+// lane would otherwise walk a whole huge row, and the chunk would pad 31
+// others to its length) and are cut into segments for sell_long_kernel.
+constexpr int kSellCapMin = 1024;
+pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
+    *nnz_long = 0;
+    const double mean = p->info.mean_row;
+    const int64_t cap = std::max<int64_t>(kSellCapMin, (int64_t)std::ceil(32.0 * mean));
+    if (p->info.max_row <= cap) return PEPP_OK;
+    p->sell_cap = (int)cap;
+    const int64_t n = p->nrows;
+    std::vector<int> rp(n + 1);
+    PEPP_CUDA_TRY(cudaMemcpy(rp.data(), p->d_rp, sizeof(int) * (n + 1), cudaMemcpyDeviceToHost));
+    std::vector<int4> seg;
+    std::vector<int2> lrow;
+    for (int64_t r = 0; r < n; ++r) {
+        const int b = rp[r], e = rp[r + 1];
+        if (e - b <= cap) continue;
+        const int li = (int)lrow.size();
+        lrow.push_back(make_int2((int)seg.size(), 0));
+        for (int k = b; k < e; k += pepp::k::kSellLongSeg)
+            seg.push_back(make_int4((int)r, k, std::min(e, k + pepp::k::kSellLongSeg), li));
+        lrow.back().y = (int)seg.size() - lrow.back().x;
+        *nnz_long += e - b;
+    }
+    pepp_status_t s;
+    if ((s = dalloc(p, &p->d_sell_seg, (int64_t)seg.size()))) return s;
+    if ((s = dalloc(p, &p->d_sell_lrow, (int64_t)lrow.size()))) return s;
+    if ((s = dalloc(p, &p->d_sell_cnt, (int64_t)lrow.size()))) return s;
+    if ((s = dalloc_bytes(p, &p->d_sell_part, 8 * (int64_t)seg.size()))) return s;
+    PEPP_CUDA_TRY(cudaMemcpy(p->d_sell_seg, seg.data(), sizeof(int4) * seg.size(), cudaMemcpyHostToDevice));
+    PEPP_CUDA_TRY(cudaMemcpy(p->d_sell_lrow, lrow.data(), sizeof(int2) * lrow.size(), cudaMemcpyHostToDevice));
+    PEPP_CUDA_TRY(cudaMemset(p->d_sell_cnt, 0, sizeof(unsigned int) * lrow.size()));
+    p->nsell_seg = (int)seg.size();
+    p->nsell_long = (int)lrow.size();
+    return PEPP_OK;
+}
+
 pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     const int n = (int)p->nrows;
     p->nchunks = (n + 31) / 32;
@@ -396,9 +443,12 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     if ((s = dalloc(p, &p->d_rowlen, n))) return s;
     if ((s = dalloc(p, &p->d_chunk_ptr, (int64_t)p->nchunks + 1))) return s;
     const int tb = 256, gb = (n + tb - 1) / tb;
+    int64_t nnz_long = 0;
+    if ((s = prepare_sell_long(p, &nnz_long))) return s;
+    const int cap = p->sell_cap;
 
     auto fill_ratio = [&](const int* perm, double* fill) -> pepp_status_t {
-        pepp::k::sell_lengths_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, perm, p->d_rowlen, p->d_chunk_len);
+        pepp::k::sell_lengths_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, perm, cap, p->d_rowlen, p->d_chunk_len);
         PEPP_CUDA_TRY(cudaGetLastError());
         std::vector<int> cl(p->nchunks);
         PEPP_CUDA_TRY(cudaMemcpyAsync(cl.data(), p->d_chunk_len, sizeof(int) * p->nchunks, cudaMemcpyDeviceToHost, st));
@@ -408,7 +458,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
         for (int c = 0; c < p->nchunks; ++c) { cp[c] = slots; slots += (int64_t)(cl[c] & pepp::k::kSellLenMask) * 32; }
         cp[p->nchunks] = slots;
         p->sell_slots = slots;
-        *fill = p->nnz ? (double)slots / (double)p->nnz : 1.0;
+        *fill = p->nnz - nnz_long > 0 ? (double)slots / (double)(p->nnz - nnz_long) : 1.0;
         PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_chunk_ptr, cp.data(), sizeof(int64_t) * (p->nchunks + 1), cudaMemcpyHostToDevice, st));
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
         return PEPP_OK;
@@ -426,21 +476,29 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
         DevTmp<unsigned long long> keys, keys_out;
         DevTmp<int> rows;
         DevTmp<unsigned char> tmp;
-        size_t tmp_bytes = 0;
+        size_t tmp_cap = 0;
         const int maxlen = (int)p->info.max_row;
         PEPP_CUDA_TRY(keys.alloc(n));
         PEPP_CUDA_TRY(keys_out.alloc(n));
         PEPP_CUDA_TRY(rows.alloc(n));
         if ((s = dalloc(p, &p->d_perm, n))) return s;
-        pepp::k::sell_keys_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, sigma, maxlen, keys.p, rows.p);
-        PEPP_CUDA_TRY(cudaGetLastError());
-        int end_bit = 32;
-        while ((1ull << (end_bit - 32)) <= (unsigned long long)((n - 1) / sigma) && end_bit < 64) ++end_bit;
-        cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, keys.p, keys_out.p, rows.p, p->d_perm, n, 0, end_bit, st);
-        PEPP_CUDA_TRY(tmp.alloc(tmp_bytes));
-        PEPP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp.p, tmp_bytes, keys.p, keys_out.p, rows.p, p->d_perm, n, 0, end_bit, st));
-        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-        if ((s = fill_ratio(p->d_perm, &fill))) return s;
+        auto sort_for = [&](int sg, double* f) -> pepp_status_t {
+            size_t tmp_bytes = 0;
+            pepp::k::sell_keys_kernel<<<gb, tb, 0, st>>>(n, p->d_rp, sg, maxlen, cap, keys.p, rows.p);
+            PEPP_CUDA_TRY(cudaGetLastError());
+            int end_bit = 32;
+            while ((1ull << (end_bit - 32)) <= (unsigned long long)((n - 1) / sg) && end_bit < 64) ++end_bit;
+            cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, keys.p, keys_out.p, rows.p, p->d_perm, n, 0, end_bit, st);
+            if (!tmp.p || tmp_bytes > tmp_cap) {
+                if (tmp.p) { cudaFree(tmp.p); tmp.p = nullptr; }
+                PEPP_CUDA_TRY(tmp.alloc(tmp_bytes));
+                tmp_cap = tmp_bytes;
+            }
+            PEPP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp.p, tmp_bytes, keys.p, keys_out.p, rows.p, p->d_perm, n, 0, end_bit, st));
+            PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+            return fill_ratio(p->d_perm, f);
+        };
+        if ((s = sort_for(sigma, &fill))) return s;
     }
     p->sell_sigma = sigma;
     if ((s = dalloc(p, &p->d_scol, p->sell_slots + 32))) return s;
@@ -449,10 +507,10 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     PEPP_CUDA_TRY(cudaMemsetAsync(p->d_scol, 0, sizeof(int) * (p->sell_slots + 32), st));
     PEPP_CUDA_TRY(cudaMemsetAsync(p->d_sval, 0, p->esz * (p->sell_slots + 32), st));
     if (p->vt == PEPP_VALUE_F32)
-        pepp::k::sell_fill_kernel<float><<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, p->d_col, (const float*)p->d_val,
+        pepp::k::sell_fill_kernel<float><<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, cap, p->d_col, (const float*)p->d_val,
                                                             p->d_chunk_ptr, p->d_scol, (float*)p->d_sval);
     else
-        pepp::k::sell_fill_kernel<double><<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, p->d_col, (const double*)p->d_val,
+        pepp::k::sell_fill_kernel<double><<<gb, tb, 0, st>>>(n, p->d_rp, p->d_perm, cap, p->d_col, (const double*)p->d_val,
                                                              p->d_chunk_ptr, p->d_scol, (double*)p->d_sval);
     PEPP_CUDA_TRY(cudaGetLastError());
     // stencil chunks: one offset per slot for the whole chunk (no column stream)
@@ -512,6 +570,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->info.sell_stencil_frac = p->nchunks ? (double)p->sell_stencil_chunks / (double)p->nchunks : 0.0;
     p->info.sell_constval_frac = p->nchunks ? (double)p->sell_const_chunks / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
+    p->info.sell_long_rows = p->nsell_long;
     return PEPP_OK;
 }
 
@@ -705,6 +764,9 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, pepp::k::NoPatterns{}, (const T*)p->d_sval, x, y, 1, nullptr,
                 nullptr, 0, nullptr);
+        if (p->nsell_seg)   // hybrid: the long rows, after sell_kernel wrote 0 for them
+            pepp::k::sell_long_kernel<256, T><<<p->nsell_seg, 256, 0, st>>>(
+                p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, (T*)p->d_sell_part, p->d_col, val, x, y);
         break;
     default:
         return PEPP_E_INVALID;
@@ -1362,7 +1424,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         const double mean = I.mean_row;
         uint32_t keep = mask;
         if ((double)I.max_row > std::max(4096.0, 256.0 * mean)) keep &= ~(1u << PEPP_V_CSR_VECTOR);
-        if (I.max_row > 4096) keep &= ~(1u << PEPP_V_SELL);   // one lane would own a whole huge row
+
         if (keep & ((1u << PEPP_V_COUNT) - 1)) mask = keep;   // never prune everything
     }
     if (mask & (1u << PEPP_V_CSR_VECTOR))
@@ -1371,7 +1433,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         p->cands.push_back({PEPP_V_MERGE_PATH, kMergeIPT});
         p->cands.push_back({PEPP_V_MERGE_PATH, kMergeWarpParam});
     }
-    if (I.max_row > pepp::k::kSellLenMask) mask &= ~(1u << PEPP_V_SELL);   // chunk length field width
+    // (SELL chunk lengths stay below kSellLenMask: rows above the hybrid cap leave the layout)
     if ((mask & ((1u << PEPP_V_COUNT) - 1)) == 0) return PEPP_E_UNSUPPORTED;
     if (mask & (1u << PEPP_V_SELL)) {
         if ((s = prepare_sell(p, st))) return s;

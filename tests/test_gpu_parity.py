@@ -586,3 +586,38 @@ def test_entry_points_restore_the_callers_device():
         plan.exec_host(np.ones(A.ncols), np.empty(A.nrows))
         assert torch.cuda.current_device() == 0
     assert torch.cuda.current_device() == 0
+
+
+def _skew_with_boundary_rows(val_mode):
+    """Heavy-tailed rows plus long rows whose lengths sit on the long-row
+    kernel's segment boundaries (kSellLongSeg = 4096) and on the SELL cap."""
+    A = gen.zipf(40_000, 40_000, seed=51, alpha=2.0, kmax=40_000, val_mode=val_mode)
+    rng = np.random.default_rng(5)
+    L = np.diff(A.row_ptr).astype(np.int64)
+    for i, n in zip([7, 1000, 2047, 30_000, 39_999], [1024, 1025, 4096, 4097, 8193]):
+        L[i] = n
+    rp = np.concatenate([[0], np.cumsum(L)]).astype(np.int64)
+    col = np.concatenate([np.sort(rng.choice(40_000, int(n), replace=False)) for n in L]).astype(np.int32)
+    val = (rng.integers(-4, 5, rp[-1]).astype(np.float64) if val_mode == gen.INT4
+           else rng.uniform(-1, 1, rp[-1]))
+    return gen.CSR(40_000, 40_000, rp, col, val, 0, 40_000)
+
+
+@pytest.mark.parametrize("exact", [True, False])
+def test_hybrid_sell_long_rows(exact):
+    """Rows longer than max(1024, 32 x mean) leave the SELL layout for the
+    segmented long-row kernel (per-row counters, partials added in segment
+    order): integer inputs bit-exact, real inputs within the bound, the same
+    bits on every call (no fp atomics), for σ = 1 and the sorted layout."""
+    A = _skew_with_boundary_rows(gen.INT4 if exact else gen.REAL)
+    x = gen.vector(12, gen.INT8 if exact else gen.REAL, A.ncols)
+    for sigma in (1, 0):
+        with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_SELL, sell_sigma=sigma) as plan:
+            info = plan.info()
+            L = np.diff(A.row_ptr)
+            cap = max(1024, int(np.ceil(32 * A.nnz / A.nrows)))
+            assert info["sell_long_rows"] == int((L > cap).sum()) > 0
+            y1, _ = _run(plan, x)
+            _check(A, x, y1, exact)
+            y2, _ = _run(plan, x)
+            assert np.array_equal(y1, y2)

@@ -21,6 +21,8 @@ def main():
     ap.add_argument("--workload", default="lap8192")
     ap.add_argument("--variants", default="")
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--compress", type=int, default=0,
+                    help="opts.compress_values (0 = the bench headline's layout, 1 = pattern-table chunks)")
     a = ap.parse_args()
     import torch
 
@@ -29,7 +31,7 @@ def main():
     R = len(rp) - 1
     A = bench.make_block(a.workload, 0, R)
     x0 = bench.x0_vector(a.workload, A.ncols)
-    plan = pepp.Plan.from_csr(A)
+    plan = pepp.Plan.from_csr(A, compress_values=bool(a.compress))
     xs = torch.from_numpy(x0).cuda()
     y = torch.empty(R, dtype=torch.float64, device="cuda")
     vs = [bench.parse_variant(v) for v in a.variants.split(",") if v] or \
