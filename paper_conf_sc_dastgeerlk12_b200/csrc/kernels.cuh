@@ -322,19 +322,27 @@ __device__ __forceinline__ int sell_pattern_run(const SellPatterns<T>& pt, int p
         if (!uni) return k0;
         int qn[kPatU];
         sell_pattern_ids(patlist, npatc, k0 + kPatU * stride, stride, qn);
-        T xv[kPatU][N];
+        // at most ~20 gathers in flight per lane: long patterns take the
+        // group in sub-groups of H chunks (keeps the kernel at 48 registers)
+        constexpr int H = N * kPatU > 20 ? (20 / N > 0 ? 20 / N : 1) : kPatU;
 #pragma unroll
-        for (int u = 0; u < kPatU; ++u) {
-            const int r = (q[u] >> 5) * 32 + lane;
+        for (int u0 = 0; u0 < kPatU; u0 += H) {
+            T xv[H][N];
 #pragma unroll
-            for (int j = 0; j < N; ++j) xv[u][j] = q[u] >= 0 ? ld_x(x, r + o[j]) : T(0);
-        }
+            for (int u = 0; u < H; ++u) {
+                const int qq = u0 + u < kPatU ? q[u0 + u] : -1;
+                const int r = (qq >> 5) * 32 + lane;
 #pragma unroll
-        for (int u = 0; u < kPatU; ++u) {
-            T acc = T(0);
+                for (int j = 0; j < N; ++j) xv[u][j] = qq >= 0 ? ld_x(x, r + o[j]) : T(0);
+            }
 #pragma unroll
-            for (int j = 0; j < N; ++j) acc = fma(v[j], xv[u][j], acc);   // slot order = the row's CSR order
-            if (q[u] >= 0) y[(q[u] >> 5) * 32 + lane] = acc;
+            for (int u = 0; u < H; ++u) {
+                const int qq = u0 + u < kPatU ? q[u0 + u] : -1;
+                T acc = T(0);
+#pragma unroll
+                for (int j = 0; j < N; ++j) acc = fma(v[j], xv[u][j], acc);   // slot order = the row's CSR order
+                if (qq >= 0) y[(qq >> 5) * 32 + lane] = acc;
+            }
         }
 #pragma unroll
         for (int u = 0; u < kPatU; ++u) q[u] = qn[u];

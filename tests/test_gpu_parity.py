@@ -621,3 +621,54 @@ def test_hybrid_sell_long_rows(exact):
             _check(A, x, y1, exact)
             y2, _ = _run(plan, x)
             assert np.array_equal(y1, y2)
+
+
+def _stencil_grid(n, offsets, center, off_val, dims=2):
+    """Constant-coefficient stencil on an n^dims grid (Dirichlet: absent
+    neighbours dropped), rows in CSR column order."""
+    N = n ** dims
+    idx = np.arange(N)
+    coords = [(idx // n ** (dims - 1 - d)) % n for d in range(dims)]
+    cols, vals, rp = [], [], [0]
+    entries = []
+    for off in offsets:
+        ok = np.ones(N, bool)
+        delta = 0
+        for d in range(dims):
+            c = coords[d] + off[d]
+            ok &= (c >= 0) & (c < n)
+            delta += off[d] * n ** (dims - 1 - d)
+        entries.append((delta, ok, center if all(o == 0 for o in off) else off_val))
+    entries.sort(key=lambda e: e[0])
+    per_row = np.zeros(N, np.int64)
+    for _, ok, _ in entries:
+        per_row += ok
+    rp = np.concatenate([[0], np.cumsum(per_row)]).astype(np.int64)
+    col = np.empty(rp[-1], np.int32)
+    val = np.empty(rp[-1], np.float64)
+    pos = rp[:-1].copy()
+    for delta, ok, v in entries:
+        r = idx[ok]
+        col[pos[r]] = r + delta
+        val[pos[r]] = v
+        pos[r] += 1
+    return gen.CSR(N, N, rp, col, val, 0, N)
+
+
+@pytest.mark.parametrize("name", ["lap3d_7pt", "grid_8pt"])
+def test_value_compression_long_patterns(name):
+    """Pattern chunks of 7 and 8 slots (3-D 7-point Laplacian; a 3x3 stencil
+    without one corner) go through the sub-grouped phase-A path: bit-identical
+    to the streamed layout and to the oracle on integer inputs."""
+    if name == "lap3d_7pt":
+        offs = [(0, 0, 0), (-1, 0, 0), (1, 0, 0), (0, -1, 0), (0, 1, 0), (0, 0, -1), (0, 0, 1)]
+        A = _stencil_grid(160, offs, 6.0, -1.0, dims=3)   # lines of 160 rows: 3 of 5 chunks interior
+    else:
+        offs = [(a, b) for a in (-1, 0, 1) for b in (-1, 0, 1) if (a, b) != (1, 1)]
+        A = _stencil_grid(300, offs, 8.0, -1.0)
+    for x in (gen.vector(3, gen.INT8, A.ncols), gen.vector(4, gen.REAL, A.ncols)):
+        y1, i1 = _sell_y(A, x, True)
+        y0, _ = _sell_y(A, x, False)
+        assert i1["sell_constval_frac"] >= 0.5
+        assert np.array_equal(y1.view(np.int64), y0.view(np.int64))
+        _check(A, x, y1, bool(np.all(x == np.round(x))))
