@@ -43,6 +43,12 @@
  * no exit crosses the ABI. A CUDA error inside a plan is sticky for that plan
  * (PEPP_E_CUDA on every later call), like a CUDA context error.
  * Threading: a plan is not thread-safe; distinct plans are independent.
+ * Streams: one plan may be called on several streams with no synchronisation
+ * in between. Candidates that use the plan's device scratch (merge-path and
+ * CSR-stream carries, hybrid-SELL partial sums, halo buffers) are ordered
+ * across streams by the plan (each such call waits for the previous one on
+ * another stream); scratch-free calls overlap (inter-call parallelism,
+ * P@21908–27091). Inside a CUDA graph capture that ordering is the graph's.
  * There is NO CPU fallback: a machine without a CUDA device gets PEPP_E_CUDA
  * from pepp_spmv_plan. The host-only utilities at the end of this header
  * (partition, halo lists, history/selector) run without a GPU.

@@ -172,6 +172,10 @@ struct pepp_spmv_plan_s {
     int64_t sub_r0[3] = {0, 0, 0};
     cudaStream_t side = nullptr;                 // exchange stream (highest priority)
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    // scratch ordering across streams (scratch_acquire / scratch_release)
+    cudaEvent_t ev_scratch = nullptr;
+    cudaStream_t scratch_stream = nullptr;
+    bool scratch_used = false;
     int reserve_sms = 0;                         // SMs a persistent grid leaves free (interior sub-plan)
     std::vector<int64_t> send_local;             // plan time: local rows the peers receive
 
@@ -282,6 +286,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     for (auto* q : p->sub) free_plan(q);
     if (p->ev_fork) cudaEventDestroy(p->ev_fork);
     if (p->ev_join) cudaEventDestroy(p->ev_join);
+    if (p->ev_scratch) cudaEventDestroy(p->ev_scratch);
     if (p->side) cudaStreamDestroy(p->side);
     delete p;
 }
@@ -1554,6 +1559,33 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
                                                 void* stream, const pepp_choice_t* force, pepp_choice_t* used);
 
 namespace {
+// Per-plan device scratch — merge-path / CSR-stream carries, hybrid-SELL
+// partial sums and row counters, halo pack buffers and the side stream — is
+// shared by all of the plan's calls. Calls on one stream are ordered by the
+// stream; a call that uses scratch on another stream than the previous user
+// first waits for that user (an event), so two in-flight calls never
+// interleave on it. Scratch-free candidates (vector-CSR, SELL without long
+// rows, no exchange) skip this and keep overlapping across streams (inter-
+// call parallelism, §IV-E P@21908–27091). Not applied under graph capture:
+// a captured call's ordering is the graph's.
+bool uses_scratch(const pepp_spmv_plan_t* p, const Candidate& c) {
+    if (c.variant == PEPP_V_MERGE_PATH || c.variant == PEPP_V_CSR_STREAM) return true;
+    return c.variant == PEPP_V_SELL && p->nsell_seg > 0;
+}
+
+pepp_status_t scratch_acquire(pepp_spmv_plan_t* p, cudaStream_t st) {
+    if (!p->ev_scratch) PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_scratch, cudaEventDisableTiming));
+    if (p->scratch_used && p->scratch_stream != st) PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_scratch, 0));
+    return PEPP_OK;
+}
+
+pepp_status_t scratch_release(pepp_spmv_plan_t* p, cudaStream_t st) {
+    PEPP_CUDA_TRY(cudaEventRecord(p->ev_scratch, st));
+    p->scratch_stream = st;
+    p->scratch_used = true;
+    return PEPP_OK;
+}
+
 // The interior rows compute on the caller's stream while a high-priority side
 // stream computes the head and tail rows (into the SMs the interior's
 // persistent grid leaves free) and then runs the halo exchange, which reads
@@ -1646,7 +1678,9 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         capturing = cs != cudaStreamCaptureStatusNone;
     }
     if (!force && p->sub[1] && (flags & PEPP_Y_NEXT_INPUT) && !(flags & PEPP_Y_REPLICATED) && p->exchange == PEPP_X_HALO) {
-        pepp_status_t s = exec_overlap(p, x, y, flags, st, used);
+        pepp_status_t s = capturing ? PEPP_OK : scratch_acquire(p, st);
+        if (!s) s = exec_overlap(p, x, y, flags, st, used);
+        if (!s && !capturing) s = scratch_release(p, st);
         if (s) p->sticky = s;
         else ++p->ncalls;
         return s;
@@ -1666,6 +1700,13 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         if (s) return s;
     }
 
+    // scratch ordering first: a wait for another stream is not the call's time
+    const bool exchanging = p->opts.nranks > 1 && (flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED));
+    const bool scr = !capturing && (exchanging || uses_scratch(p, p->cands[ch.candidate]));
+    if (scr) {
+        pepp_status_t s = scratch_acquire(p, st);
+        if (s) { p->sticky = s; return s; }
+    }
     // timing: every calibration call and every forced call, then every
     // sample_period-th call; never inside a CUDA graph capture
     bool timed = !(flags & PEPP_EXEC_NO_TIMING) && !capturing;
@@ -1690,7 +1731,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         }
     }
     ch.exchange = PEPP_X_NONE;
-    if (p->opts.nranks > 1 && (flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED))) {
+    if (exchanging) {
         const bool ag = (flags & PEPP_Y_REPLICATED) || p->exchange == PEPP_X_ALLGATHER;
         const int ex = (force && (force->exchange == PEPP_X_ALLGATHER || force->exchange == PEPP_X_HALO))
                            ? force->exchange : (ag ? PEPP_X_ALLGATHER : PEPP_X_HALO);
@@ -1698,6 +1739,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         if (s) { p->sticky = s; return s; }
         ch.exchange = ex;
     }
+    if (scr && (s = scratch_release(p, st))) { p->sticky = s; return s; }
     ++p->ncalls;
     if (used) *used = ch;
     return PEPP_OK;

@@ -1,0 +1,52 @@
+"""One plan, calls on several streams at once (inter-call parallelism,
+SURVEY §8(f) f4, paper §IV-E P@21908–27091): the candidates that keep
+per-plan device scratch (merge-path and CSR-stream carries, hybrid-SELL
+partial sums and their row counters, halo pack buffers) must not let two
+in-flight calls interleave on it. Every candidate is forced, four right-hand
+sides alternate over two streams with no synchronisation in between, and
+every result is compared with the oracle bit for bit (integer-valued
+inputs)."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_sc_dastgeerlk12_b200 as pepp  # noqa: E402
+
+
+def _concurrent(A, nrhs=4, reps=3):
+    xs = [gen.vector(20 + i, gen.INT8, A.ncols) for i in range(nrhs)]
+    refs = [oracle.spmv(A, x) for x in xs]
+    streams = [torch.cuda.Stream() for _ in range(2)]
+    with pepp.Plan.from_csr(A) as plan:
+        for c in plan.candidates():
+            f = pepp.Choice(c.variant, c.param)
+            xd = [torch.from_numpy(x).cuda() for x in xs]
+            ys = [torch.full((A.nrows,), float("nan"), dtype=torch.float64, device="cuda") for _ in xs]
+            torch.cuda.synchronize()
+            for _ in range(reps):
+                for i in range(nrhs):
+                    plan.exec(xd[i], ys[i], force=f, stream=streams[i % 2])
+            torch.cuda.synchronize()
+            for i in range(nrhs):
+                y = ys[i].cpu().numpy()
+                bad = np.flatnonzero(y != refs[i])
+                assert bad.size == 0, (f.name, i, bad[:8], y[bad[:4]], refs[i][bad[:4]])
+
+
+def test_two_streams_heavy_tail():
+    """Heavy-tailed rows (P(k) ~ k^-2 up to 2^20): merge-path long runs,
+    CSR-stream long rows and hybrid-SELL long rows all use plan scratch."""
+    A = gen.zipf(1 << 20, 1 << 20, seed=50, alpha=2.0, kmax=1 << 20, val_mode=gen.INT4)
+    _concurrent(A)
+
+
+def test_two_streams_uniform():
+    A = gen.uniform(1 << 21, 1 << 21, 16, seed=43, val_mode=gen.INT4)
+    _concurrent(A)
