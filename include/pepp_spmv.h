@@ -344,6 +344,28 @@ pepp_status_t pepp_spmv_p2p_buffers(pepp_spmv_plan_t* p, int32_t nbuf, void** bu
 pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const void* x_host, void* y_host, int32_t iterations,
                                   int flags, void* stream);
 
+/* pepp_spmv_exec_host over `nbatch` independent right-hand sides: item k
+   reads x_hosts[k] (READ, host, ncols entries) and writes y_hosts[k] (WRITE,
+   host, rows as in pepp_spmv_exec_host), with `iterations` and `flags` as
+   there. The transfers overlap the computation — item k+1's input copy and
+   item k-1's output copy run on the copy engines while item k computes —
+   the data-transfer overlap the runtime is meant to provide for
+   GPU-resident operands (§IV-E, P@21908–27091; transfer-inclusive timing of
+   Fig. 5, P@35591–35720). Results equal nbatch separate pepp_spmv_exec_host
+   calls. Work starts after everything queued on `stream`; the call returns
+   when every y_hosts[k] is written. Host buffers must be pinned for the
+   copies to overlap (pageable buffers are correct, only serialised). Entries
+   may repeat: output copies run in item order, so a repeated y buffer ends
+   with its last item's result; a y buffer must not overlap an x buffer of
+   the batch. Two slots of plan-owned device buffers (4 vectors
+   of max(ncols, global rows) entries) and two copy streams are created on
+   first use and kept. nbatch = 0 is a no-op; nbatch = 1 is
+   pepp_spmv_exec_host. Errors: PEPP_E_INVALID (NULL arrays or entries,
+   nbatch < 0, iterations < 1 or > 1 on a non-square matrix), otherwise as
+   pepp_spmv_exec. */
+pepp_status_t pepp_spmv_exec_host_batch(pepp_spmv_plan_t* p, int32_t nbatch, const void* const* x_hosts,
+                                        void* const* y_hosts, int32_t iterations, int flags, void* stream);
+
 /* Free everything the plan owns (device memory, events, an owned NCCL
    communicator); saves history to opts.history_path if set. Waits for the
    plan's outstanding work. NULL is a no-op. */

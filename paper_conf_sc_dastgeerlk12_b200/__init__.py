@@ -206,6 +206,19 @@ class Plan:
         C.check(C.lib().pepp_spmv_exec_host(self._h, _ptr(x_host), _ptr(y_host), iterations, flags,
                                             _stream_handle(stream)), "pepp_spmv_exec_host")
 
+    def exec_host_batch(self, x_hosts: Sequence[np.ndarray], y_hosts: Sequence[np.ndarray], iterations: int = 1,
+                        flags: int = Y_LOCAL, stream=None) -> None:
+        """exec_host over independent right-hand sides, transfers overlapped
+        with the computation (synchronous)."""
+        want = np.float32 if self.value_type == C.VALUE_F32 else np.float64
+        assert len(x_hosts) == len(y_hosts)
+        assert all(a.dtype == want for a in x_hosts) and all(a.dtype == want for a in y_hosts)
+        n = len(x_hosts)
+        xs = (ctypes.c_void_p * max(n, 1))(*[_ptr(a) for a in x_hosts])
+        ys = (ctypes.c_void_p * max(n, 1))(*[_ptr(a) for a in y_hosts])
+        C.check(C.lib().pepp_spmv_exec_host_batch(self._h, n, xs, ys, iterations, flags, _stream_handle(stream)),
+                "pepp_spmv_exec_host_batch")
+
     def select(self) -> Choice:
         c = C.CHOICE_T()
         C.check(C.lib().pepp_spmv_select(self._h, ctypes.byref(c)), "pepp_spmv_select")

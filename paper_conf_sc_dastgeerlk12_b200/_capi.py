@@ -77,6 +77,7 @@ SIGNATURES = {
     "pepp_spmv_select": (c_i32, [c_vp, ctypes.POINTER(CHOICE_T)]),
     "pepp_spmv_exec": (c_i32, [c_vp, c_vp, c_vp, ctypes.c_int, c_vp, ctypes.POINTER(CHOICE_T), ctypes.POINTER(CHOICE_T)]),
     "pepp_spmv_exec_host": (c_i32, [c_vp, c_vp, c_vp, c_i32, ctypes.c_int, c_vp]),
+    "pepp_spmv_exec_host_batch": (c_i32, [c_vp, c_i32, c_vp, c_vp, c_i32, ctypes.c_int, c_vp]),
     "pepp_spmv_exchange": (c_i32, [c_vp, c_vp, ctypes.c_int, c_vp]),
     "pepp_spmv_p2p_buffers": (c_i32, [c_vp, c_i32, ctypes.POINTER(c_vp)]),
     "pepp_spmv_destroy": (c_i32, [c_vp]),

@@ -202,6 +202,11 @@ struct pepp_spmv_plan_s {
     // plan-owned x / y for pepp_spmv_exec_host (allocated on first use)
     void* d_hx = nullptr;
     void* d_hy = nullptr;
+    // pepp_spmv_exec_host_batch: two slots of (x, y) device buffers, copy
+    // streams and their events (created on first use)
+    void* d_hb[4] = {};
+    cudaStream_t cs_in = nullptr, cs_out = nullptr;
+    cudaEvent_t ev_start = nullptr, ev_end = nullptr, ev_in[2] = {}, ev_out[2] = {}, ev_free[2] = {};
 };
 
 namespace {
@@ -288,6 +293,11 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->ev_join) cudaEventDestroy(p->ev_join);
     if (p->ev_scratch) cudaEventDestroy(p->ev_scratch);
     if (p->side) cudaStreamDestroy(p->side);
+    for (void* b : p->d_hb) if (b) cudaFree(b);
+    for (cudaEvent_t e : {p->ev_start, p->ev_end, p->ev_in[0], p->ev_in[1], p->ev_out[0], p->ev_out[1], p->ev_free[0], p->ev_free[1]})
+        if (e) cudaEventDestroy(e);
+    if (p->cs_in) cudaStreamDestroy(p->cs_in);
+    if (p->cs_out) cudaStreamDestroy(p->cs_out);
     delete p;
 }
 
@@ -1856,6 +1866,31 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* 
     return s;
 }
 
+namespace {
+// `iterations` calls x_{k+1} = A·x_k starting from device buffer a (b is the
+// other iteration buffer); *out gets the buffer holding the final y
+pepp_status_t host_iterations(pepp_spmv_plan_t* p, void* a, void* b, int32_t iterations, int flags, cudaStream_t st,
+                              void** out) {
+    void *xin = a, *yout = b;
+    for (int32_t it = 0; it < iterations; ++it) {
+        const bool last = it == iterations - 1;
+        const int f = last ? flags : (flags & PEPP_EXEC_NO_TIMING) | PEPP_Y_NEXT_INPUT;
+        pepp_status_t s = pepp_spmv_exec(p, xin, yout, f, st, nullptr, nullptr);
+        if (s) return s;
+        if (!last) std::swap(xin, yout);
+    }
+    *out = yout;
+    return PEPP_OK;
+}
+
+// rows copied back: all global rows with PEPP_Y_REPLICATED, else this rank's rows
+void host_rows(const pepp_spmv_plan_t* p, int flags, int64_t* lo, int64_t* cnt) {
+    *lo = p->row_offset;
+    *cnt = p->nrows;
+    if (p->opts.nranks > 1 && (flags & PEPP_Y_REPLICATED)) { *lo = 0; *cnt = p->global_rows; }
+}
+}  // namespace
+
 extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const void* x_host, void* y_host,
                                                      int32_t iterations, int flags, void* stream) {
     if (!p || !x_host || !y_host || iterations < 1) return PEPP_E_INVALID;
@@ -1874,22 +1909,74 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const
         (void)cudaGetLastError();
         return PEPP_E_CUDA;
     }
-    void *xin = p->d_hx, *yout = p->d_hy;
-    for (int32_t it = 0; it < iterations; ++it) {
-        const bool last = it == iterations - 1;
-        const int f = last ? flags : (flags & PEPP_EXEC_NO_TIMING) | PEPP_Y_NEXT_INPUT;
-        pepp_status_t s = pepp_spmv_exec(p, xin, yout, f, stream, nullptr, nullptr);
-        if (s) return s;
-        if (!last) std::swap(xin, yout);
-    }
-    // rows written back: all global rows with PEPP_Y_REPLICATED, else this rank's rows
-    int64_t lo = p->row_offset, cnt = p->nrows;
-    if (p->opts.nranks > 1 && (flags & PEPP_Y_REPLICATED)) { lo = 0; cnt = p->global_rows; }
+    void* yout = nullptr;
+    pepp_status_t s = host_iterations(p, p->d_hx, p->d_hy, iterations, flags, st, &yout);
+    if (s) return s;
+    int64_t lo, cnt;
+    host_rows(p, flags, &lo, &cnt);
     if (cnt > 0 && cudaMemcpyAsync((char*)y_host + lo * (int64_t)p->esz, (const char*)yout + lo * (int64_t)p->esz,
                                    p->esz * cnt, cudaMemcpyDeviceToHost, st) != cudaSuccess) {
         (void)cudaGetLastError();
         return PEPP_E_CUDA;
     }
+    if (cudaStreamSynchronize(st) != cudaSuccess) { (void)cudaGetLastError(); p->sticky = PEPP_E_CUDA; return PEPP_E_CUDA; }
+    return PEPP_OK;
+}
+
+// Software pipeline over independent right-hand sides: item k's host->device
+// copy (stream cs_in), its iterations (the caller's stream) and its
+// device->host copy (stream cs_out) use slot k % 2, so item k+1's input copy
+// and item k-1's output copy run on the copy engines while item k computes.
+// A slot is refilled only after its previous output copy finished (ev_free).
+extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host_batch(pepp_spmv_plan_t* p, int32_t nbatch,
+                                                           const void* const* x_hosts, void* const* y_hosts,
+                                                           int32_t iterations, int flags, void* stream) {
+    if (!p || nbatch < 0 || (nbatch > 0 && (!x_hosts || !y_hosts)) || iterations < 1) return PEPP_E_INVALID;
+    for (int32_t k = 0; k < nbatch; ++k) if (!x_hosts[k] || !y_hosts[k]) return PEPP_E_INVALID;
+    if (p->sticky) return p->sticky;
+    if (iterations > 1 && p->ncols != p->global_rows) return PEPP_E_INVALID;
+    if (nbatch == 0) return PEPP_OK;
+    if (nbatch == 1) return pepp_spmv_exec_host(p, x_hosts[0], y_hosts[0], iterations, flags, stream);
+    cudaStream_t st = (cudaStream_t)stream;
+    DeviceScope dscope(p->device);
+    if (!dscope.ok) return PEPP_E_CUDA;
+    const int64_t nx = std::max<int64_t>(p->ncols, p->global_rows);
+    if (!p->cs_in) {
+        for (void*& b : p->d_hb) {
+            pepp_status_t s = dalloc_bytes(p, &b, nx * (int64_t)p->esz);
+            if (s) return s;
+        }
+        PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->cs_in, cudaStreamNonBlocking));
+        PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->cs_out, cudaStreamNonBlocking));
+        for (cudaEvent_t* e : {&p->ev_start, &p->ev_end, &p->ev_in[0], &p->ev_in[1], &p->ev_out[0], &p->ev_out[1],
+                               &p->ev_free[0], &p->ev_free[1]})
+            PEPP_CUDA_TRY(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+    }
+    int64_t lo, cnt;
+    host_rows(p, flags, &lo, &cnt);
+    // the copies start after everything the caller queued on its stream
+    PEPP_CUDA_TRY(cudaEventRecord(p->ev_start, st));
+    PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_in, p->ev_start, 0));
+    PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_out, p->ev_start, 0));
+    for (int32_t k = 0; k < nbatch; ++k) {
+        const int b = k & 1;
+        void *xa = p->d_hb[2 * b], *xb = p->d_hb[2 * b + 1];
+        if (k >= 2) PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_in, p->ev_free[b], 0));
+        PEPP_CUDA_TRY(cudaMemcpyAsync(xa, x_hosts[k], p->esz * p->ncols, cudaMemcpyHostToDevice, p->cs_in));
+        PEPP_CUDA_TRY(cudaEventRecord(p->ev_in[b], p->cs_in));
+        PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_in[b], 0));
+        void* yout = nullptr;
+        pepp_status_t s = host_iterations(p, xa, xb, iterations, flags, st, &yout);
+        if (s) return s;
+        PEPP_CUDA_TRY(cudaEventRecord(p->ev_out[b], st));
+        PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_out, p->ev_out[b], 0));
+        if (cnt > 0)
+            PEPP_CUDA_TRY(cudaMemcpyAsync((char*)y_hosts[k] + lo * (int64_t)p->esz, (const char*)yout + lo * (int64_t)p->esz,
+                                          p->esz * cnt, cudaMemcpyDeviceToHost, p->cs_out));
+        PEPP_CUDA_TRY(cudaEventRecord(p->ev_free[b], p->cs_out));
+    }
+    PEPP_CUDA_TRY(cudaEventRecord(p->ev_end, p->cs_out));
+    PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_end, 0));
     if (cudaStreamSynchronize(st) != cudaSuccess) { (void)cudaGetLastError(); p->sticky = PEPP_E_CUDA; return PEPP_E_CUDA; }
     return PEPP_OK;
 }

@@ -256,6 +256,37 @@ def test_exec_host_matches_device_path():
         assert np.array_equal(y, ref5)
 
 
+@pytest.mark.parametrize("iterations", [1, 5])
+def test_exec_host_batch_overlapped(iterations):
+    """pepp_spmv_exec_host_batch: independent right-hand sides with the
+    transfers overlapped (two device slots, copy streams) equal separate
+    exec_host calls, bit for bit, on pinned and pageable host buffers."""
+    n = 512
+    A = gen.laplacian2d(n)
+    N = n * n
+    xs = [gen.vector(30 + k, gen.INT8, N) for k in range(5)]
+    refs = [oracle.iterate(A, x, iterations) if iterations > 1 else oracle.spmv(A, x) for x in xs]
+    with pepp.Plan.from_csr(A) as plan:
+        for pinned in (True, False):
+            if pinned:
+                xh = [torch.from_numpy(x).pin_memory().numpy() for x in xs]
+                yh = [torch.full((N,), float("nan"), dtype=torch.float64).pin_memory().numpy() for _ in xs]
+            else:
+                xh = [x.copy() for x in xs]
+                yh = [np.full(N, np.nan) for _ in xs]
+            for nb in (0, 1, 2, 5):
+                for y in yh:
+                    y.fill(np.nan)
+                plan.exec_host_batch(xh[:nb], yh[:nb], iterations=iterations)
+                for k in range(nb):
+                    assert np.array_equal(yh[k], refs[k]), (pinned, nb, k)
+                for k in range(nb, len(xs)):
+                    assert np.all(np.isnan(yh[k]))
+        L = pepp._capi.lib()
+        assert L.pepp_spmv_exec_host_batch(plan._h, -1, None, None, 1, 0, None) == pepp._capi.PEPP_E_INVALID
+        assert L.pepp_spmv_exec_host_batch(plan._h, 2, None, None, 1, 0, None) == pepp._capi.PEPP_E_INVALID
+
+
 # ------------------------------------------------------------- selector --
 def test_selector_calibrates_then_picks_fastest_measured():
     A = gen.uniform(200_000, 200_000, 16, seed=42)
