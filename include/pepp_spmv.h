@@ -63,7 +63,7 @@
 extern "C" {
 #endif
 
-#define PEPP_ABI_VERSION 3
+#define PEPP_ABI_VERSION 4
 
 typedef enum {
     PEPP_OK = 0,
@@ -169,7 +169,7 @@ typedef struct {
                                  candidates from the context instance before the runtime choice —
                                  vector-CSR only if max_row <= max(4096, 256*mean); SELL, merge-path
                                  and CSR-stream always (SELL moves rows longer than
-                                 max(1024, 32*mean) to its segmented long-row kernel).
+                                 info.sell_cap to its segmented long-row kernel).
                                  0 = every variant is a candidate (variant_mask still applies). */
     int32_t overlap;          /* partitioned halo plans (nranks > 1): 1 (default) = when the rows this
                                  rank sends lie in a short head and tail of its block (stencils, banded
@@ -239,8 +239,10 @@ typedef struct pepp_plan_info_s {
     int32_t predicted;        /* candidates with a prediction from opts.predict (0 = none / no function) */
     double sell_constval_frac;/* fraction of SELL chunks stored as a pattern-table id (compress_values) */
     int32_t p2p_buffers;      /* symmetric buffers registered by pepp_spmv_p2p_buffers (0 = none) */
-    int64_t sell_long_rows;   /* hybrid SELL: rows longer than max(1024, 32 x mean) summed by the
-                                 segmented long-row kernel instead of the SELL layout (0 = none) */
+    int64_t sell_long_rows;   /* hybrid SELL: rows longer than sell_cap summed by the segmented
+                                 long-row kernel instead of the SELL layout (0 = none) */
+    int64_t sell_cap;         /* hybrid SELL cap: max(128, one warp's share of the SELL work =
+                                 (nnz/32 + 4 x chunks) / warps of one resident wave) */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

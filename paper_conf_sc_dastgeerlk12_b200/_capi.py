@@ -39,7 +39,7 @@ class INFO_T(ctypes.Structure):
                 ("prior_key", c_u64), ("sell_stencil_frac", c_f64),
                 ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64), ("predicted", c_i32),
                 ("sell_constval_frac", c_f64), ("p2p_buffers", c_i32),
-                ("sell_long_rows", c_i64)]
+                ("sell_long_rows", c_i64), ("sell_cap", c_i64)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -129,7 +129,7 @@ class PeppError(RuntimeError):
         super().__init__(f"{where}: {status_str(status)} ({status})" + (f": {detail}" if detail else ""))
 
 
-ABI_VERSION = 3   # PEPP_ABI_VERSION of include/pepp_spmv.h
+ABI_VERSION = 4   # PEPP_ABI_VERSION of include/pepp_spmv.h
 
 
 def lib() -> ctypes.CDLL:

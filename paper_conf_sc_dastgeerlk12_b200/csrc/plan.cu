@@ -30,6 +30,8 @@ using pepp::Nccl;
 using pepp::ncclComm_t;
 
 constexpr int kBlock = 256;
+constexpr int kSellCapMin = 128;      // hybrid SELL: rows above max(this, a warp's share) leave the layout
+constexpr int64_t kChunkCost = 4;     // SELL per-chunk overhead in slot-equivalents (warp ranges, hybrid cap)
 constexpr int kMergeBlock = 256;
 constexpr int kMergeIPT = 7;
 constexpr int kMergeTile = kMergeBlock * kMergeIPT;
@@ -322,7 +324,7 @@ pepp_status_t sell_warp_ranges(pepp_spmv_plan_t* p) {
     if (nc > 0) PEPP_CUDA_TRY(cudaMemcpy(len.data(), p->d_chunk_len, sizeof(int) * nc, cudaMemcpyDeviceToHost));
     const int nwin = nc / cpw, nfull = nwin * cpw;
     auto chunk_of = [&](int i) { return i < nfull ? (i % nwin) * cpw + i / nwin : i; };
-    int64_t kChunkOverhead = 4;   // descriptor + per-lane loads + y store, in slot-equivalents
+    int64_t kChunkOverhead = kChunkCost;   // descriptor + per-lane loads + y store, in slot-equivalents
     if (const char* e = std::getenv("PEPP_SELL_CHUNK_COST")) kChunkOverhead = std::atoi(e);   // experiments only
     int64_t total = 0;
     for (int i = 0; i < nc; ++i) total += (len[chunk_of(i)] & pepp::k::kSellLenMask) + kChunkOverhead;
@@ -410,17 +412,32 @@ pepp_status_t sell_patterns(pepp_spmv_plan_t* p, int64_t nsb, const void* d_scon
     return PEPP_OK;
 }
 
-// Hybrid SELL for heavy-tailed rows: when the longest row exceeds
-// max(kSellCapMin, 32 x mean), rows above that cap leave the SELL layout (one
-// lane would otherwise walk a whole huge row, and the chunk would pad 31
-// others to its length) and are cut into segments for sell_long_kernel.
-constexpr int kSellCapMin = 1024;
+// Hybrid SELL for heavy-tailed rows. One warp walks a whole chunk, so a
+// chunk of L slots is a chain of L dependent slot steps on one warp; once L
+// exceeds a warp's share of the work (Σ cost / warps of one resident wave,
+// cost = slots + kChunkCost per chunk, as sell_warp_ranges counts it) that
+// warp is the kernel's critical path whatever the other warps do. Rows longer
+// than cap = max(kSellCapMin, that share) therefore leave the SELL layout and
+// are cut into segments for sell_long_kernel (measured on the heavy-tailed
+// `skew` matrix: cap 1024 → 373 µs, 512 → 272, 256 → 262, 128 → 248; config 3,
+// whose share exceeds its longest row, keeps every row in SELL).
 pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
     *nnz_long = 0;
-    const double mean = p->info.mean_row;
-    const int64_t cap = std::max<int64_t>(kSellCapMin, (int64_t)std::ceil(32.0 * mean));
+    int64_t cap = kSellCapMin;
+    {
+        int occ = 0;
+        const void* fn = p->vt == PEPP_VALUE_F32 ? (const void*)pepp::k::sell_kernel<kBlock, true, false, float>
+                                                 : (const void*)pepp::k::sell_kernel<kBlock, true, false, double>;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
+        (void)cudaGetLastError();
+        const int64_t warps = (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ * (kBlock / 32);
+        const int64_t nchunks = (p->nrows + 31) / 32;
+        const int64_t share = (p->info.nnz / 32 + kChunkCost * nchunks + warps - 1) / warps;
+        cap = std::max<int64_t>(cap, share);
+    }
+    if (const char* e = std::getenv("PEPP_SELL_CAP")) cap = std::max(1, std::atoi(e));   // experiments only
+    p->sell_cap = (int)std::min<int64_t>(cap, INT32_MAX);
     if (p->info.max_row <= cap) return PEPP_OK;
-    p->sell_cap = (int)cap;
     const int64_t n = p->nrows;
     std::vector<int> rp(n + 1);
     PEPP_CUDA_TRY(cudaMemcpy(rp.data(), p->d_rp, sizeof(int) * (n + 1), cudaMemcpyDeviceToHost));
@@ -586,6 +603,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->info.sell_constval_frac = p->nchunks ? (double)p->sell_const_chunks / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
     p->info.sell_long_rows = p->nsell_long;
+    p->info.sell_cap = p->sell_cap == INT32_MAX ? 0 : p->sell_cap;
     return PEPP_OK;
 }
 

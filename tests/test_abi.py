@@ -47,7 +47,7 @@ def test_library_exports_every_declared_symbol():
 def test_abi_version_and_status_strings():
     from paper_conf_sc_dastgeerlk12_b200 import _capi
     L = _capi.lib()
-    assert L.pepp_abi_version() == _capi.ABI_VERSION == 3
+    assert L.pepp_abi_version() == _capi.ABI_VERSION == 4
     for s in [0, -1, -2, -3, -4, -5, -6]:
         assert L.pepp_status_str(s).decode().startswith("PEPP_")
 
@@ -67,7 +67,7 @@ int main(void) {
   P(pepp_plan_info_t, sell_fill) P(pepp_plan_info_t, halo_send) P(pepp_plan_info_t, sell_col16_frac) P(pepp_plan_info_t, prior_key) P(pepp_plan_info_t, sell_stencil_frac)
   P(pepp_spmv_opts_t, overlap) P(pepp_plan_info_t, overlap) P(pepp_plan_info_t, overlap_head) P(pepp_plan_info_t, overlap_tail)
   P(pepp_spmv_opts_t, predict) P(pepp_spmv_opts_t, predict_user) P(pepp_plan_info_t, predicted)
-  P(pepp_spmv_opts_t, compress_values) P(pepp_plan_info_t, sell_constval_frac) P(pepp_plan_info_t, p2p_buffers) P(pepp_plan_info_t, sell_long_rows)
+  P(pepp_spmv_opts_t, compress_values) P(pepp_plan_info_t, sell_constval_frac) P(pepp_plan_info_t, p2p_buffers) P(pepp_plan_info_t, sell_long_rows) P(pepp_plan_info_t, sell_cap)
   printf("x_p2p %d\n", (int)PEPP_X_P2P);
   return 0;
 }
@@ -104,6 +104,7 @@ int main(void) {
     assert int(vals["pepp_plan_info_t.sell_constval_frac"]) == C.INFO_T.sell_constval_frac.offset
     assert int(vals["pepp_plan_info_t.p2p_buffers"]) == C.INFO_T.p2p_buffers.offset
     assert int(vals["pepp_plan_info_t.sell_long_rows"]) == C.INFO_T.sell_long_rows.offset
+    assert int(vals["pepp_plan_info_t.sell_cap"]) == C.INFO_T.sell_cap.offset
     assert int(vals["x_p2p"]) == C.X_P2P
 
 

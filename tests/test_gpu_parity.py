@@ -619,13 +619,14 @@ def test_entry_points_restore_the_callers_device():
     assert torch.cuda.current_device() == 0
 
 
-def _skew_with_boundary_rows(val_mode):
+def _skew_with_boundary_rows(val_mode, at=()):
     """Heavy-tailed rows plus long rows whose lengths sit on the long-row
-    kernel's segment boundaries (kSellLongSeg = 4096) and on the SELL cap."""
+    kernel's segment boundaries (kSellLongSeg = 4096) and on `at` (the SELL
+    cap and cap + 1)."""
     A = gen.zipf(40_000, 40_000, seed=51, alpha=2.0, kmax=40_000, val_mode=val_mode)
     rng = np.random.default_rng(5)
     L = np.diff(A.row_ptr).astype(np.int64)
-    for i, n in zip([7, 1000, 2047, 30_000, 39_999], [1024, 1025, 4096, 4097, 8193]):
+    for i, n in zip([7, 1000, 2047, 30_000, 39_999, 11, 12], [1024, 1025, 4096, 4097, 8193, *at]):
         L[i] = n
     rp = np.concatenate([[0], np.cumsum(L)]).astype(np.int64)
     col = np.concatenate([np.sort(rng.choice(40_000, int(n), replace=False)) for n in L]).astype(np.int32)
@@ -636,17 +637,24 @@ def _skew_with_boundary_rows(val_mode):
 
 @pytest.mark.parametrize("exact", [True, False])
 def test_hybrid_sell_long_rows(exact):
-    """Rows longer than max(1024, 32 x mean) leave the SELL layout for the
-    segmented long-row kernel (per-row counters, partials added in segment
-    order): integer inputs bit-exact, real inputs within the bound, the same
-    bits on every call (no fp atomics), for σ = 1 and the sorted layout."""
-    A = _skew_with_boundary_rows(gen.INT4 if exact else gen.REAL)
+    """Rows longer than the plan's cap (max(128, one warp's share of the SELL
+    work)) leave the SELL layout for the segmented long-row kernel (per-row
+    counters, partials added in segment order): integer inputs bit-exact,
+    real inputs within the bound, the same bits on every call (no fp
+    atomics), for σ = 1 and the sorted layout; rows of exactly cap and cap + 1
+    entries sit on either side of the split."""
+    vm = gen.INT4 if exact else gen.REAL
+    with pepp.Plan.from_csr(_skew_with_boundary_rows(vm), variant_mask=1 << pepp.V_SELL) as plan:
+        cap0 = plan.info()["sell_cap"]
+    assert cap0 >= 128
+    A = _skew_with_boundary_rows(vm, at=(cap0, cap0 + 1))
     x = gen.vector(12, gen.INT8 if exact else gen.REAL, A.ncols)
+    L = np.diff(A.row_ptr)
     for sigma in (1, 0):
         with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_SELL, sell_sigma=sigma) as plan:
             info = plan.info()
-            L = np.diff(A.row_ptr)
-            cap = max(1024, int(np.ceil(32 * A.nnz / A.nrows)))
+            cap = info["sell_cap"]
+            assert abs(cap - cap0) <= 1
             assert info["sell_long_rows"] == int((L > cap).sum()) > 0
             y1, _ = _run(plan, x)
             _check(A, x, y1, exact)
