@@ -241,8 +241,10 @@ typedef struct pepp_plan_info_s {
     int32_t p2p_buffers;      /* symmetric buffers registered by pepp_spmv_p2p_buffers (0 = none) */
     int64_t sell_long_rows;   /* hybrid SELL: rows longer than sell_cap summed by the segmented
                                  long-row kernel instead of the SELL layout (0 = none) */
-    int64_t sell_cap;         /* hybrid SELL cap: max(128, one warp's share of the SELL work =
-                                 (nnz/32 + 4 x chunks) / warps of one resident wave) */
+    int64_t sell_cap;         /* hybrid SELL cap: max(64, min(share, 8 x mean)), share = one warp's
+                                 part of the SELL work = (nnz/32 + 4 x chunks) / warps of one
+                                 resident wave; rows up to 1024 long above it: one warp each,
+                                 longer: 4096-entry segments */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

@@ -1117,6 +1117,41 @@ __global__ void __launch_bounds__(BLOCK) sell_long_kernel(const int4* __restrict
     }
 }
 
+// Mid-length rows of a hybrid SELL plan (cap < length <= kSellLongSeg): one
+// warp per listed row, lanes strided over the row (4 col / val pairs, then 4
+// x gathers in flight per lane), a fixed-order shuffle reduction, lane 0
+// writes y — no scratch, deterministic. Launched after sell_kernel, which
+// wrote 0 for these rows.
+template <int BLOCK, typename T>
+__global__ void __launch_bounds__(BLOCK) sell_mid_kernel(int n, const int* __restrict__ rows,
+                                                         const int* __restrict__ rp, const int* __restrict__ col,
+                                                         const T* __restrict__ val, const T* __restrict__ x,
+                                                         T* __restrict__ y) {
+    const int lane = threadIdx.x & 31;
+    const int w = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
+    if (w >= n) return;
+    const int r = __ldg(rows + w);
+    const int s = __ldg(rp + r), e = __ldg(rp + r + 1);
+    const uint64_t pol = evict_first_policy();
+    T a0 = T(0), a1 = T(0), a2 = T(0), a3 = T(0);
+    int k = s + lane;
+    for (; k + 96 < e; k += 128) {
+        const int c0 = ld_stream_i(col + k, pol), c1 = ld_stream_i(col + k + 32, pol);
+        const int c2 = ld_stream_i(col + k + 64, pol), c3 = ld_stream_i(col + k + 96, pol);
+        const T v0 = ld_stream_v(val + k, pol), v1 = ld_stream_v(val + k + 32, pol);
+        const T v2 = ld_stream_v(val + k + 64, pol), v3 = ld_stream_v(val + k + 96, pol);
+        a0 = fma(v0, ld_x(x, c0), a0);
+        a1 = fma(v1, ld_x(x, c1), a1);
+        a2 = fma(v2, ld_x(x, c2), a2);
+        a3 = fma(v3, ld_x(x, c3), a3);
+    }
+    for (; k < e; k += 32) a0 = fma(ld_stream_v(val + k, pol), ld_x(x, ld_stream_i(col + k, pol)), a0);
+    T acc = (a0 + a1) + (a2 + a3);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) y[r] = acc;
+}
+
 // 16-bit column deltas: one warp per chunk; if every stored column of the
 // chunk is within int16 of its row's original index, write col16 and set
 // kSellCol16 in chunk_len.

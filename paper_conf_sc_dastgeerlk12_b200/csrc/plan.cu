@@ -30,8 +30,9 @@ using pepp::Nccl;
 using pepp::ncclComm_t;
 
 constexpr int kBlock = 256;
-constexpr int kSellCapMin = 128;      // hybrid SELL: rows above max(this, a warp's share) leave the layout
+constexpr int kSellCapMin = 64;       // hybrid SELL: floor of the cap (prepare_sell_long)
 constexpr int64_t kChunkCost = 4;     // SELL per-chunk overhead in slot-equivalents (warp ranges, hybrid cap)
+constexpr int64_t kSellMidMax = 1024; // hybrid rows up to this length: one warp each (sell_mid_kernel)
 constexpr int kMergeBlock = 256;
 constexpr int kMergeIPT = 7;
 constexpr int kMergeTile = kMergeBlock * kMergeIPT;
@@ -118,6 +119,8 @@ struct pepp_spmv_plan_s {
     int4* d_sell_seg = nullptr;      // {row, k begin, k end, long-row index} per segment
     int2* d_sell_lrow = nullptr;     // {first segment, segments} per long row
     unsigned int* d_sell_cnt = nullptr;
+    int nsell_mid = 0;
+    int* d_sell_mid = nullptr;       // rows of cap < length <= kSellLongSeg: sell_mid_kernel, warp per row
     void* d_sell_part = nullptr;     // segment partials (8-byte slots)
 
     // merge path
@@ -279,7 +282,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
                     p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist,
-                    p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, p->d_sell_part};
+                    p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, p->d_sell_part, p->d_sell_mid};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -413,14 +416,17 @@ pepp_status_t sell_patterns(pepp_spmv_plan_t* p, int64_t nsb, const void* d_scon
 }
 
 // Hybrid SELL for heavy-tailed rows. One warp walks a whole chunk, so a
-// chunk of L slots is a chain of L dependent slot steps on one warp; once L
-// exceeds a warp's share of the work (Σ cost / warps of one resident wave,
-// cost = slots + kChunkCost per chunk, as sell_warp_ranges counts it) that
-// warp is the kernel's critical path whatever the other warps do. Rows longer
-// than cap = max(kSellCapMin, that share) therefore leave the SELL layout and
-// are cut into segments for sell_long_kernel (measured on the heavy-tailed
-// `skew` matrix: cap 1024 → 373 µs, 512 → 272, 256 → 262, 128 → 248; config 3,
-// whose share exceeds its longest row, keeps every row in SELL).
+// chunk of L slots is a chain of L dependent slot steps on one warp, and in a
+// sorted window the chunk holding the window's longest rows is padded to its
+// longest row with mostly masked lanes. Rows longer than
+//   cap = max(kSellCapMin, min(share, 8 x mean)),
+// share = one warp's part of the SELL work ((nnz/32 + kChunkCost x chunks) /
+// warps of one resident wave), leave the layout: up to kSellMidMax entries
+// one warp each (sell_mid_kernel), longer ones cut into segments of
+// kSellLongSeg for sell_long_kernel. Measured (tools/gpu_cap4.sh, `skew` /
+// config 3, µs): cap 1024 and no mid kernel 373 / 359; share 276 / 359;
+// 128 241 / 352; 64 236 / 361 — the rule gives 73 on `skew` and 128 on
+// config 3.
 pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
     *nnz_long = 0;
     int64_t cap = kSellCapMin;
@@ -433,7 +439,8 @@ pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
         const int64_t warps = (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ * (kBlock / 32);
         const int64_t nchunks = (p->nrows + 31) / 32;
         const int64_t share = (p->info.nnz / 32 + kChunkCost * nchunks + warps - 1) / warps;
-        cap = std::max<int64_t>(cap, share);
+        const int64_t rel = (int64_t)std::ceil(8.0 * p->info.mean_row);
+        cap = std::max<int64_t>(cap, std::min(share, rel));
     }
     if (const char* e = std::getenv("PEPP_SELL_CAP")) cap = std::max(1, std::atoi(e));   // experiments only
     p->sell_cap = (int)std::min<int64_t>(cap, INT32_MAX);
@@ -443,17 +450,27 @@ pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
     PEPP_CUDA_TRY(cudaMemcpy(rp.data(), p->d_rp, sizeof(int) * (n + 1), cudaMemcpyDeviceToHost));
     std::vector<int4> seg;
     std::vector<int2> lrow;
+    std::vector<int> mid;
+    int64_t mid_max = kSellMidMax;
+    if (const char* e = std::getenv("PEPP_SELL_MIDMAX")) mid_max = std::atoi(e);   // experiments only
     for (int64_t r = 0; r < n; ++r) {
         const int b = rp[r], e = rp[r + 1];
         if (e - b <= cap) continue;
+        *nnz_long += e - b;
+        if (e - b <= mid_max) { mid.push_back((int)r); continue; }
         const int li = (int)lrow.size();
         lrow.push_back(make_int2((int)seg.size(), 0));
         for (int k = b; k < e; k += pepp::k::kSellLongSeg)
             seg.push_back(make_int4((int)r, k, std::min(e, k + pepp::k::kSellLongSeg), li));
         lrow.back().y = (int)seg.size() - lrow.back().x;
-        *nnz_long += e - b;
     }
     pepp_status_t s;
+    if (!mid.empty()) {
+        if ((s = dalloc(p, &p->d_sell_mid, (int64_t)mid.size()))) return s;
+        PEPP_CUDA_TRY(cudaMemcpy(p->d_sell_mid, mid.data(), sizeof(int) * mid.size(), cudaMemcpyHostToDevice));
+        p->nsell_mid = (int)mid.size();
+    }
+    if (seg.empty()) return PEPP_OK;
     if ((s = dalloc(p, &p->d_sell_seg, (int64_t)seg.size()))) return s;
     if ((s = dalloc(p, &p->d_sell_lrow, (int64_t)lrow.size()))) return s;
     if ((s = dalloc(p, &p->d_sell_cnt, (int64_t)lrow.size()))) return s;
@@ -602,7 +619,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->info.sell_stencil_frac = p->nchunks ? (double)p->sell_stencil_chunks / (double)p->nchunks : 0.0;
     p->info.sell_constval_frac = p->nchunks ? (double)p->sell_const_chunks / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
-    p->info.sell_long_rows = p->nsell_long;
+    p->info.sell_long_rows = p->nsell_long + p->nsell_mid;
     p->info.sell_cap = p->sell_cap == INT32_MAX ? 0 : p->sell_cap;
     return PEPP_OK;
 }
@@ -797,6 +814,9 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, pepp::k::NoPatterns{}, (const T*)p->d_sval, x, y, 1, nullptr,
                 nullptr, 0, nullptr);
+        if (p->nsell_mid)   // hybrid: the mid-length rows, after sell_kernel wrote 0 for them
+            pepp::k::sell_mid_kernel<256, T><<<(p->nsell_mid + 7) / 8, 256, 0, st>>>(
+                p->nsell_mid, p->d_sell_mid, p->d_rp, p->d_col, val, x, y);
         if (p->nsell_seg)   // hybrid: the long rows, after sell_kernel wrote 0 for them
             pepp::k::sell_long_kernel<256, T><<<p->nsell_seg, 256, 0, st>>>(
                 p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, (T*)p->d_sell_part, p->d_col, val, x, y);

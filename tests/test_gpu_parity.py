@@ -637,16 +637,17 @@ def _skew_with_boundary_rows(val_mode, at=()):
 
 @pytest.mark.parametrize("exact", [True, False])
 def test_hybrid_sell_long_rows(exact):
-    """Rows longer than the plan's cap (max(128, one warp's share of the SELL
-    work)) leave the SELL layout for the segmented long-row kernel (per-row
-    counters, partials added in segment order): integer inputs bit-exact,
+    """Rows longer than the plan's cap (max(64, min(one warp's share of the
+    SELL work, 8 x mean))) leave the SELL layout: up to 1024 entries one warp
+    each, longer ones for the segmented long-row kernel (per-row counters,
+    partials added in segment order; 1024 / 1025 sit on that split): integer inputs bit-exact,
     real inputs within the bound, the same bits on every call (no fp
     atomics), for σ = 1 and the sorted layout; rows of exactly cap and cap + 1
     entries sit on either side of the split."""
     vm = gen.INT4 if exact else gen.REAL
     with pepp.Plan.from_csr(_skew_with_boundary_rows(vm), variant_mask=1 << pepp.V_SELL) as plan:
         cap0 = plan.info()["sell_cap"]
-    assert cap0 >= 128
+    assert cap0 >= 64
     A = _skew_with_boundary_rows(vm, at=(cap0, cap0 + 1))
     x = gen.vector(12, gen.INT8 if exact else gen.REAL, A.ncols)
     L = np.diff(A.row_ptr)
