@@ -39,6 +39,8 @@ def main() -> int:
         rp.append(len(cols))
     mats.append(gen.CSR(len(rows), 3000, np.array(rp, np.int64), np.array(cols, np.int32), np.array(vals), 0, len(rows)))
     mats.append(gen.rebase(mats[1], 7))
+    # heavy tail: hybrid SELL with mid-length (warp per row) and segmented long rows
+    mats.append(gen.zipf(20_000, 20_000, seed=51, alpha=2.0, kmax=20_000, val_mode=gen.INT4))
     bad = 0
     for A in mats:
         x = gen.vector(3, gen.INT8, A.ncols)
@@ -71,6 +73,13 @@ def main() -> int:
         bad += 0 if np.array_equal(w.host(pepp.ACCESS_READ), oracle.spmv(A, oracle.spmv(A, x0))) else 1
         for c in (u, v, w):
             c.close()
+    # overlapped host batch (copy streams, two device slots)
+    with pepp.Plan.from_csr(A) as plan:
+        xs = [gen.vector(30 + k, gen.INT8, A.nrows) for k in range(3)]
+        ys = [np.full(A.nrows, np.nan) for _ in xs]
+        plan.exec_host_batch(xs, ys, iterations=2)
+        for xk, yk in zip(xs, ys):
+            bad += 0 if np.array_equal(yk, oracle.spmv(A, oracle.spmv(A, xk))) else 1
     print("sanitize_run: mismatches =", bad)
     return 1 if bad else 0
 
