@@ -293,6 +293,9 @@ __device__ __forceinline__ T sell_pattern_slots(const SellPatterns<T>& pt, int p
 #define PEPP_PAT_U 4
 #endif
 constexpr int kPatU = PEPP_PAT_U;   // pattern chunks per warp iteration in phase A
+#ifndef PEPP_PAT_PREFETCH
+#define PEPP_PAT_PREFETCH 1   // L2 prefetch distance in groups (0 = off; 1 measured best: 265 -> 254 us on config 4)
+#endif
 
 // list entries k0, k0 + stride, ... (kPatU of them; -1 past the end)
 __device__ __forceinline__ void sell_pattern_ids(const int* __restrict__ patlist, int npatc, int k0, int stride,
@@ -322,6 +325,23 @@ __device__ __forceinline__ int sell_pattern_run(const SellPatterns<T>& pt, int p
         if (!uni) return k0;
         int qn[kPatU];
         sell_pattern_ids(patlist, npatc, k0 + kPatU * stride, stride, qn);
+#if PEPP_PAT_PREFETCH
+        // the rows of x of the group PEPP_PAT_PREFETCH steps ahead: the band
+        // of chunks the whole grid works on then touches them first (DRAM),
+        // so pull them into L2 now
+        {
+            int qp[kPatU];
+            if (PEPP_PAT_PREFETCH == 1) {
+#pragma unroll
+                for (int u = 0; u < kPatU; ++u) qp[u] = qn[u];
+            } else {
+                sell_pattern_ids(patlist, npatc, k0 + PEPP_PAT_PREFETCH * kPatU * stride, stride, qp);
+            }
+#pragma unroll
+            for (int u = 0; u < kPatU; ++u)
+                if (qp[u] >= 0) asm volatile("prefetch.global.L2 [%0];" ::"l"(x + (qp[u] >> 5) * 32 + lane));
+        }
+#endif
         // at most ~20 gathers in flight per lane: long patterns take the
         // group in sub-groups of H chunks (keeps the kernel at 48 registers)
         constexpr int H = N * kPatU > 20 ? (20 / N > 0 ? 20 / N : 1) : kPatU;
