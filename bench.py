@@ -397,7 +397,6 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     info = plan.info()
     flags = pepp.Y_NEXT_INPUT if iterated else pepp.Y_LOCAL
     overlapped = bool(world > 1 and iterated and force is None and info["overlap"])
-    kernels_per_call = (1 + (info["overlap_head"] > 0) + (info["overlap_tail"] > 0)) if overlapped else 1
 
     stream = torch.cuda.Stream(device=dev)
     xs = torch.from_numpy(x0).to(dev)
@@ -406,7 +405,6 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
         # symmetric buffers: the boundary kernel pushes the halo straight into
         # the neighbours' copies over peer memory (PEPP_X_P2P), no NCCL per iteration
         bufs = plan.p2p_buffers(2)
-        kernels_per_call = 2
     else:
         bufs = [torch.empty(R, dtype=tdt, device=dev) for _ in range(2)]
     flush = None if iterated or Z * 12 > 4 * (1 << 30) else torch.empty(512 << 20, dtype=torch.uint8, device=dev)
@@ -440,7 +438,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
                 if record:
                     b.record(stream)
                     used_count[u.name] = used_count.get(u.name, 0) + 1
-                    launches["n"] += (2 if u.variant == pepp.V_MERGE_PATH else 1) * kernels_per_call
+                    launches["n"] += u.launches   # the library's own count of its kernels in this call
                 if not overlapped and flags != pepp.Y_LOCAL and world > 1:
                     plan.exchange(dst, flags, stream=stream)
                 if iterated:

@@ -63,7 +63,7 @@
 extern "C" {
 #endif
 
-#define PEPP_ABI_VERSION 4
+#define PEPP_ABI_VERSION 5
 
 typedef enum {
     PEPP_OK = 0,
@@ -209,6 +209,9 @@ typedef struct {
     int32_t calibrating;      /* 1 = chosen to gather history, not the predicted best */
     int32_t candidate;        /* index in the plan's candidate list */
     double predicted_us;      /* history mean of this candidate (0 if unknown) */
+    int32_t launches;         /* exec only: kernels of this library the call launched (SpMV kernels,
+                                 fix-ups, halo pack/unpack or the fused push; NCCL's own not counted) */
+    int32_t reserved;
 } pepp_choice_t;
 
 /* Context instance (§III P@9781: "a tuple of concrete values for context

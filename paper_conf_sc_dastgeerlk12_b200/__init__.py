@@ -40,6 +40,7 @@ class Choice:
     calibrating: bool = False
     candidate: int = -1
     predicted_us: float = 0.0
+    launches: int = 0
 
     @property
     def name(self) -> str:
@@ -47,7 +48,8 @@ class Choice:
 
     @staticmethod
     def _from(c: C.CHOICE_T) -> "Choice":
-        return Choice(c.variant, c.param, c.exchange, c.nparts, bool(c.calibrating), c.candidate, c.predicted_us)
+        return Choice(c.variant, c.param, c.exchange, c.nparts, bool(c.calibrating), c.candidate, c.predicted_us,
+                      c.launches)
 
     def _to(self) -> C.CHOICE_T:
         c = C.CHOICE_T()

@@ -60,13 +60,14 @@ class OPTS_T(ctypes.Structure):
 
 class CHOICE_T(ctypes.Structure):
     _fields_ = [("variant", c_i32), ("param", c_i32), ("nparts", c_i32), ("exchange", c_i32),
-                ("calibrating", c_i32), ("candidate", c_i32), ("predicted_us", c_f64)]
+                ("calibrating", c_i32), ("candidate", c_i32), ("predicted_us", c_f64),
+                ("launches", c_i32), ("reserved", c_i32)]
 
     def as_dict(self) -> dict:
         return {"variant": VARIANT_NAMES.get(self.variant, str(self.variant)), "variant_id": self.variant,
                 "param": self.param, "nparts": self.nparts, "exchange": EXCHANGE_NAMES.get(self.exchange, "?"),
                 "calibrating": bool(self.calibrating), "candidate": self.candidate,
-                "predicted_us": self.predicted_us}
+                "predicted_us": self.predicted_us, "launches": self.launches}
 
 
 # (name, restype, argtypes) for every entry point of include/pepp_spmv.h
@@ -129,7 +130,7 @@ class PeppError(RuntimeError):
         super().__init__(f"{where}: {status_str(status)} ({status})" + (f": {detail}" if detail else ""))
 
 
-ABI_VERSION = 4   # PEPP_ABI_VERSION of include/pepp_spmv.h
+ABI_VERSION = 5   # PEPP_ABI_VERSION of include/pepp_spmv.h
 
 
 def lib() -> ctypes.CDLL:

@@ -827,6 +827,28 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
     return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
 }
 
+// kernels launch_t enqueues for candidate c (mirrors its conditions)
+int launches_for(const pepp_spmv_plan_t* p, const Candidate& c) {
+    if (p->nrows == 0) return 0;
+    switch (c.variant) {
+    case PEPP_V_CSR_VECTOR: return 1;
+    case PEPP_V_MERGE_PATH:
+        if (c.param == kMergeWarpParam) return p->ntiles_w > 0 ? 2 + (p->nlongruns_w > 0) : 0;
+        return p->ntiles > 0 ? 2 + (p->nlongruns > 0) : 0;
+    case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
+    case PEPP_V_SELL: return 1 + (p->nsell_mid > 0) + (p->nsell_seg > 0);
+    default: return 0;
+    }
+}
+
+// gather / scatter kernels one halo exchange launches (pack_unpack)
+int halo_kernels(const pepp_spmv_plan_t* p) {
+    int n = 0;
+    for (const auto* v : {&p->send_x, &p->recv_x})
+        for (const auto& t : *v) n += t.contig_start < 0 && t.count > 0;
+    return n;
+}
+
 pepp_status_t launch(pepp_spmv_plan_t* p, const Candidate& c, const void* x, void* y, cudaStream_t st) {
     if (p->vt == PEPP_VALUE_F32) return launch_t<float>(p, c, (const float*)x, (float*)y, st);
     return launch_t<double>(p, c, (const double*)x, (double*)y, st);
@@ -1656,11 +1678,16 @@ pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flag
         // signalled by one kernel (PEPP_X_P2P)
         if (!s) s = p->vt == PEPP_VALUE_F32 ? p2p_launch_t<float>(p, b, (const float*)x, (float*)y, p->side)
                                             : p2p_launch_t<double>(p, b, (const double*)x, (double*)y, p->side);
+        u.launches += 1;
     } else {
         for (int i : {0, 2})
-            if (!s && p->sub[i])
-                s = pepp_spmv_exec(p->sub[i], x, yb + p->sub_r0[i] * (int64_t)p->esz, sf, p->side, nullptr, nullptr);
+            if (!s && p->sub[i]) {
+                pepp_choice_t ui{};
+                s = pepp_spmv_exec(p->sub[i], x, yb + p->sub_r0[i] * (int64_t)p->esz, sf, p->side, nullptr, &ui);
+                u.launches += ui.launches;
+            }
         if (!s) s = exchange_halo(p, y, p->side);
+        u.launches += halo_kernels(p);
     }
     PEPP_CUDA_TRY(cudaEventRecord(p->ev_join, p->side));   // join whatever reached the side stream
     PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_join, 0));
@@ -1768,6 +1795,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
     }
     pepp_status_t s = launch(p, p->cands[ch.candidate], x, (char*)y + p->row_offset * (int64_t)p->esz, st);
     if (s) { p->sticky = s; return s; }
+    ch.launches = launches_for(p, p->cands[ch.candidate]);
     if (rec) {
         if (cudaEventRecord(rec->stop, st) == cudaSuccess) {
             rec->cand = ch.candidate;
@@ -1786,6 +1814,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         s = ex == PEPP_X_ALLGATHER ? exchange_allgather(p, y, st) : exchange_halo(p, y, st);
         if (s) { p->sticky = s; return s; }
         ch.exchange = ex;
+        if (ex == PEPP_X_HALO) ch.launches += halo_kernels(p);
     }
     if (scr && (s = scratch_release(p, st))) { p->sticky = s; return s; }
     ++p->ncalls;

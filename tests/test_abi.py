@@ -47,7 +47,7 @@ def test_library_exports_every_declared_symbol():
 def test_abi_version_and_status_strings():
     from paper_conf_sc_dastgeerlk12_b200 import _capi
     L = _capi.lib()
-    assert L.pepp_abi_version() == _capi.ABI_VERSION == 4
+    assert L.pepp_abi_version() == _capi.ABI_VERSION == 5
     for s in [0, -1, -2, -3, -4, -5, -6]:
         assert L.pepp_status_str(s).decode().startswith("PEPP_")
 
@@ -63,7 +63,7 @@ int main(void) {
   printf("csr %zu\nopts %zu\nchoice %zu\ninfo %zu\n", sizeof(pepp_csr_t), sizeof(pepp_spmv_opts_t),
          sizeof(pepp_choice_t), sizeof(pepp_plan_info_t));
   P(pepp_csr_t, on_device) P(pepp_spmv_opts_t, row_bounds) P(pepp_spmv_opts_t, exchange)
-  P(pepp_spmv_opts_t, history_path) P(pepp_spmv_opts_t, prune) P(pepp_choice_t, predicted_us) P(pepp_plan_info_t, key)
+  P(pepp_spmv_opts_t, history_path) P(pepp_spmv_opts_t, prune) P(pepp_choice_t, predicted_us) P(pepp_choice_t, launches) P(pepp_plan_info_t, key)
   P(pepp_plan_info_t, sell_fill) P(pepp_plan_info_t, halo_send) P(pepp_plan_info_t, sell_col16_frac) P(pepp_plan_info_t, prior_key) P(pepp_plan_info_t, sell_stencil_frac)
   P(pepp_spmv_opts_t, overlap) P(pepp_plan_info_t, overlap) P(pepp_plan_info_t, overlap_head) P(pepp_plan_info_t, overlap_tail)
   P(pepp_spmv_opts_t, predict) P(pepp_spmv_opts_t, predict_user) P(pepp_plan_info_t, predicted)
@@ -88,6 +88,7 @@ int main(void) {
     assert int(vals["pepp_spmv_opts_t.history_path"]) == C.OPTS_T.history_path.offset
     assert int(vals["pepp_spmv_opts_t.prune"]) == C.OPTS_T.prune.offset
     assert int(vals["pepp_choice_t.predicted_us"]) == C.CHOICE_T.predicted_us.offset
+    assert int(vals["pepp_choice_t.launches"]) == C.CHOICE_T.launches.offset
     assert int(vals["pepp_plan_info_t.key"]) == C.INFO_T.key.offset
     assert int(vals["pepp_plan_info_t.sell_fill"]) == C.INFO_T.sell_fill.offset
     assert int(vals["pepp_plan_info_t.halo_send"]) == C.INFO_T.halo_send.offset

@@ -50,3 +50,24 @@ def test_two_streams_heavy_tail():
 def test_two_streams_uniform():
     A = gen.uniform(1 << 21, 1 << 21, 16, seed=43, val_mode=gen.INT4)
     _concurrent(A)
+
+
+def test_reported_launches_match_profiler():
+    """pepp_choice_t.launches (the bench's gpu_launches) equals the library
+    kernels CUPTI sees for the call, for every candidate of a heavy-tailed
+    plan (hybrid SELL: SELL + mid-row + segmented kernels; merge fix-ups;
+    CSR-stream fix-up) and of the Laplacian (one SELL kernel)."""
+    from torch.profiler import ProfilerActivity, profile
+    for A in (gen.zipf(1 << 18, 1 << 18, seed=50, alpha=2.0, kmax=1 << 18, val_mode=gen.INT4), gen.laplacian2d(256)):
+        x = torch.from_numpy(gen.vector(3, gen.INT8, A.ncols)).cuda()
+        y = torch.empty(A.nrows, dtype=torch.float64, device="cuda")
+        with pepp.Plan.from_csr(A, prune=False) as plan:
+            for c in plan.candidates():
+                f = pepp.Choice(c.variant, c.param)
+                plan.exec(x, y, force=f)   # warm
+                torch.cuda.synchronize()
+                with profile(activities=[ProfilerActivity.CUDA]) as prof:
+                    u = plan.exec(x, y, force=f)
+                    torch.cuda.synchronize()
+                seen = sum(e.count for e in prof.key_averages() if "pepp::" in e.key)
+                assert u.launches == seen > 0, (A.name, f.name, u.launches, seen)
