@@ -523,21 +523,25 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
         per = {}
         for c in plan.candidates():
             f = pepp.Choice(c.variant, c.param)
-            ts = []
+            # issued back to back like the timed region (events around each
+            # call, no host sync in between): small matrices get more calls,
+            # their per-call times are a few microseconds
+            ncall = min(iters, 10 if A.nnz > 10_000_000 else 100) + 2
+            pairs = []
             with torch.cuda.stream(stream):
                 src = xs
-                for k in range(min(iters, 10) + 2):
+                for k in range(ncall):
                     if flush is not None:
                         flush.zero_()
-                    a, b = ev_pool[k % len(ev_pool)]
+                    a, b = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                     a.record(stream)
                     plan.exec(src, bufs[k & 1], flags=flags, stream=stream, force=f)
                     b.record(stream)
-                    b.synchronize()
-                    if k >= 2:
-                        ts.append(a.elapsed_time(b))
+                    pairs.append((a, b))
                     if iterated:
                         src = bufs[k & 1]
+            stream.synchronize()
+            ts = [a.elapsed_time(b) for a, b in pairs[2:]]
             per[f.name] = statistics.median(ts) * 1e3
         best = min(per, key=per.get)
         sel = {"chosen": chosen, "chosen_us": round(per.get(chosen, float("nan")), 2), "best": best,

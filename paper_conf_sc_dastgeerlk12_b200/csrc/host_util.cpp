@@ -168,15 +168,27 @@ bool history_abandoned(const Welford* w, double best_mean) {
     return w && w->count > 0 && best_mean > 0 && w->mean > kAbandonFactor * best_mean;
 }
 
+bool history_contender(const Welford* w, double best_mean) {
+    return w && w->count > 0 && best_mean > 0 && w->mean <= kContendFactor * best_mean;
+}
+
 int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible,
                      int32_t min_samples, int32_t* calibrating, double* predicted_us) {
     const double best_mean = history_best_mean(h, key, ncand, eligible);
     // 1) calibration in rounds: round r gives every candidate its r-th sample
-    //    (lowest index first), skipping candidates already ruled out
-    for (int32_t r = 1; r <= min_samples; ++r) {
+    //    (lowest index first), skipping candidates already ruled out; rounds
+    //    past min_samples (refinement) only for the contenders, those within
+    //    kContendFactor of the best mean, when there are at least two — where
+    //    measurement noise can flip the choice (short calls: event times come
+    //    in ~2 µs steps)
+    int32_t ncontend = 0;
+    for (int32_t c = 0; c < ncand; ++c) ncontend += eligible[c] && history_contender(history_get(h, key, c), best_mean);
+    const int32_t rounds = ncontend >= 2 ? kRefineRounds * min_samples : min_samples;
+    for (int32_t r = 1; r <= rounds; ++r) {
         for (int32_t c = 0; c < ncand; ++c) {
             if (!eligible[c]) continue;
             const Welford* w = history_get(h, key, c);
+            if (r > min_samples && !history_contender(w, best_mean)) continue;
             if ((!w || w->count < r) && !history_abandoned(w, best_mean)) {
                 *calibrating = 1;
                 *predicted_us = w ? w->mean : 0.0;

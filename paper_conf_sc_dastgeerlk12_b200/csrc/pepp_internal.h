@@ -24,6 +24,11 @@ const Welford* history_get(const pepp_history* h, uint64_t key, int32_t cand);
 constexpr double kAbandonFactor = 4.0;   // calibration stops sampling a candidate this much slower than the best
 double history_best_mean(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible);
 bool history_abandoned(const Welford* w, double best_mean);
+// refinement: after min_samples rounds, candidates whose mean is within
+// kContendFactor of the best get rounds up to kRefineRounds x min_samples
+constexpr double kContendFactor = 1.10;
+constexpr int32_t kRefineRounds = 3;
+bool history_contender(const Welford* w, double best_mean);
 int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible,
                      int32_t min_samples, int32_t* calibrating, double* predicted_us);
 uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts);

@@ -948,10 +948,17 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out, bool frozen
             if (pepp::history_abandoned(w, best_mean)) return true;
             return (!w || w->count == 0) && prior_best > 0 && p->prior[c] > pepp::kAbandonFactor * prior_best;
         };
+        auto rounds = [&]() {   // refinement only while two or more contenders exist
+            int32_t k = 0;
+            for (int32_t c = 0; c < n; ++c) k += p->eligible[c] && pepp::history_contender(hget(c), best_mean);
+            return k >= 2 ? pepp::kRefineRounds * ms : ms;
+        };
         cand = -1;
-        for (int32_t r = 1; r <= ms && cand < 0; ++r) {
+        for (int32_t r = 1; r <= rounds() && cand < 0; ++r) {
             // round r: every candidate not yet ruled out gets its r-th timed call
-            // (calls still in flight count, so the host can run ahead of the GPU)
+            // (calls still in flight count, so the host can run ahead of the GPU);
+            // rounds past ms refine only the contenders (within kContendFactor
+            // of the best mean), as pepp::history_pick does
             for (int pass = 0; pass < 2 && cand < 0; ++pass) {
                 bool waiting = false;
                 for (int32_t oi = 0; oi < n; ++oi) {
@@ -959,6 +966,7 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out, bool frozen
                     if (!p->eligible[c]) continue;
                     const pepp::Welford* w = hget(c);
                     if (ruled_out(c, w)) continue;
+                    if (r > ms && !pepp::history_contender(w, best_mean)) continue;
                     const int64_t done = w ? w->count : 0;
                     if (done + p->pending[c] < r) {
                         cand = c; calibrating = 1;

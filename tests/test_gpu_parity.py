@@ -300,9 +300,10 @@ def test_selector_calibrates_then_picks_fastest_measured():
             if not u.calibrating:
                 break
             seen.append(u.candidate)
-        # round 1 visits every candidate; later rounds skip the ones ruled out
+        # round 1 visits every candidate; later rounds skip the ones ruled out,
+        # rounds 4..9 (refinement) only the contenders within 10 % of the best
         assert seen[:n] == list(range(n))
-        assert len(seen) <= 3 * n
+        assert len(seen) <= 9 * n
         plan.flush_history()
         means = [plan.history_stats(c)[1] for c in range(n)]
         ch = plan.select()

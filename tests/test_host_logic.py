@@ -85,8 +85,10 @@ def test_history_calibrates_then_exploits_argmin():
             break
         order.append(c)
         H.record(key, c, times[c])
-    # calibration runs in rounds: every candidate once per round, lowest index first
-    assert order == [0, 1, 2, 3] * 3
+    # calibration runs in rounds: every candidate once per round, lowest index
+    # first; then refinement rounds (up to 3 x min_samples) for the contenders
+    # within 10 % of the best mean: candidates 1 and 3
+    assert order == [0, 1, 2, 3] * 3 + [1, 3] * 6
     c, cal, pred = H.select(key, elig, min_samples=3)
     assert (c, cal) == (1, False) and pred == pytest.approx(3.0)
     # candidate 3 is 0.7 % slower: the tie rule keeps the lower index
@@ -109,7 +111,8 @@ def test_history_early_abandonment():
             break
         order.append(c)
         H.record(key, c, times[c])
-    # round 1 samples everyone; candidates 0 (10x) and 2 (300x) are then dropped
+    # round 1 samples everyone; candidates 0 (10x) and 2 (300x) are then
+    # dropped; no refinement rounds (3 is 50 % slower: the best has no contender)
     assert order == [0, 1, 2, 3, 1, 3, 1, 3]
     assert H.select(key, [True] * 4)[:2] == (1, False)
     assert H.stats(key, 2)[0] == 1 and H.stats(key, 0)[0] == 1

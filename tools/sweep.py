@@ -63,14 +63,18 @@ def main():
             ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.reps)]
 
             def timed(force=None):
-                ts = []
+                # calls issued back to back (no host sync in between): each L2
+                # flush keeps the GPU busy while the host queues the next call,
+                # so an event pair brackets the SpMV's device time only, not the
+                # host's submission gap (which a per-call sync would add)
+                u = None
                 for e0, e1 in ev:
                     flush.zero_()
                     e0.record()
                     u = plan.exec(x, y, force=force)
                     e1.record()
-                    e1.synchronize()
-                    ts.append(e0.elapsed_time(e1) * 1e3)
+                torch.cuda.synchronize()
+                ts = [e0.elapsed_time(e1) * 1e3 for e0, e1 in ev]
                 return statistics.median(ts), u
 
             # calibration through ordinary automatic calls (flush between calls);
