@@ -1980,22 +1980,22 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const
         if ((s = dalloc_bytes(p, &p->d_hx, nx * (int64_t)p->esz))) return s;
         if ((s = dalloc_bytes(p, &p->d_hy, nx * (int64_t)p->esz))) return s;
     }
-    if (cudaMemcpyAsync(p->d_hx, x_host, p->esz * p->ncols, cudaMemcpyHostToDevice, st) != cudaSuccess) {
-        (void)cudaGetLastError();
-        return PEPP_E_CUDA;
-    }
-    void* yout = nullptr;
-    pepp_status_t s = host_iterations(p, p->d_hx, p->d_hy, iterations, flags, st, &yout);
-    if (s) return s;
-    int64_t lo, cnt;
-    host_rows(p, flags, &lo, &cnt);
-    if (cnt > 0 && cudaMemcpyAsync((char*)y_host + lo * (int64_t)p->esz, (const char*)yout + lo * (int64_t)p->esz,
-                                   p->esz * cnt, cudaMemcpyDeviceToHost, st) != cudaSuccess) {
-        (void)cudaGetLastError();
-        return PEPP_E_CUDA;
-    }
+    auto enqueue = [&]() -> pepp_status_t {
+        PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_hx, x_host, p->esz * p->ncols, cudaMemcpyHostToDevice, st));
+        void* yout = nullptr;
+        pepp_status_t s = host_iterations(p, p->d_hx, p->d_hy, iterations, flags, st, &yout);
+        if (s) return s;
+        int64_t lo, cnt;
+        host_rows(p, flags, &lo, &cnt);
+        if (cnt > 0)
+            PEPP_CUDA_TRY(cudaMemcpyAsync((char*)y_host + lo * (int64_t)p->esz, (const char*)yout + lo * (int64_t)p->esz,
+                                          p->esz * cnt, cudaMemcpyDeviceToHost, st));
+        return PEPP_OK;
+    };
+    const pepp_status_t s = enqueue();
+    // also on failure: nothing queued may still touch the caller's host buffers
     if (cudaStreamSynchronize(st) != cudaSuccess) { (void)cudaGetLastError(); p->sticky = PEPP_E_CUDA; return PEPP_E_CUDA; }
-    return PEPP_OK;
+    return s;
 }
 
 // Software pipeline over independent right-hand sides: item k's host->device
@@ -2016,44 +2016,57 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host_batch(pepp_spmv_plan_t* p,
     DeviceScope dscope(p->device);
     if (!dscope.ok) return PEPP_E_CUDA;
     const int64_t nx = std::max<int64_t>(p->ncols, p->global_rows);
-    if (!p->cs_in) {
-        for (void*& b : p->d_hb) {
+    // first use: slots, copy streams, events (each created once; a failed
+    // attempt leaves what it made for the next one, nothing leaks)
+    for (void*& b : p->d_hb)
+        if (!b) {
             pepp_status_t s = dalloc_bytes(p, &b, nx * (int64_t)p->esz);
             if (s) return s;
         }
-        PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->cs_in, cudaStreamNonBlocking));
-        PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->cs_out, cudaStreamNonBlocking));
-        for (cudaEvent_t* e : {&p->ev_start, &p->ev_end, &p->ev_in[0], &p->ev_in[1], &p->ev_out[0], &p->ev_out[1],
-                               &p->ev_free[0], &p->ev_free[1]})
-            PEPP_CUDA_TRY(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
-    }
+    for (cudaStream_t* q : {&p->cs_in, &p->cs_out})
+        if (!*q) PEPP_CUDA_TRY(cudaStreamCreateWithFlags(q, cudaStreamNonBlocking));
+    for (cudaEvent_t* e : {&p->ev_start, &p->ev_end, &p->ev_in[0], &p->ev_in[1], &p->ev_out[0], &p->ev_out[1],
+                           &p->ev_free[0], &p->ev_free[1]})
+        if (!*e) PEPP_CUDA_TRY(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
     int64_t lo, cnt;
     host_rows(p, flags, &lo, &cnt);
-    // the copies start after everything the caller queued on its stream
-    PEPP_CUDA_TRY(cudaEventRecord(p->ev_start, st));
-    PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_in, p->ev_start, 0));
-    PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_out, p->ev_start, 0));
-    for (int32_t k = 0; k < nbatch; ++k) {
-        const int b = k & 1;
-        void *xa = p->d_hb[2 * b], *xb = p->d_hb[2 * b + 1];
-        if (k >= 2) PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_in, p->ev_free[b], 0));
-        PEPP_CUDA_TRY(cudaMemcpyAsync(xa, x_hosts[k], p->esz * p->ncols, cudaMemcpyHostToDevice, p->cs_in));
-        PEPP_CUDA_TRY(cudaEventRecord(p->ev_in[b], p->cs_in));
-        PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_in[b], 0));
-        void* yout = nullptr;
-        pepp_status_t s = host_iterations(p, xa, xb, iterations, flags, st, &yout);
-        if (s) return s;
-        PEPP_CUDA_TRY(cudaEventRecord(p->ev_out[b], st));
-        PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_out, p->ev_out[b], 0));
-        if (cnt > 0)
-            PEPP_CUDA_TRY(cudaMemcpyAsync((char*)y_hosts[k] + lo * (int64_t)p->esz, (const char*)yout + lo * (int64_t)p->esz,
-                                          p->esz * cnt, cudaMemcpyDeviceToHost, p->cs_out));
-        PEPP_CUDA_TRY(cudaEventRecord(p->ev_free[b], p->cs_out));
+    auto enqueue = [&]() -> pepp_status_t {
+        // the copies start after everything the caller queued on its stream
+        PEPP_CUDA_TRY(cudaEventRecord(p->ev_start, st));
+        PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_in, p->ev_start, 0));
+        PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_out, p->ev_start, 0));
+        for (int32_t k = 0; k < nbatch; ++k) {
+            const int b = k & 1;
+            void *xa = p->d_hb[2 * b], *xb = p->d_hb[2 * b + 1];
+            if (k >= 2) PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_in, p->ev_free[b], 0));
+            PEPP_CUDA_TRY(cudaMemcpyAsync(xa, x_hosts[k], p->esz * p->ncols, cudaMemcpyHostToDevice, p->cs_in));
+            PEPP_CUDA_TRY(cudaEventRecord(p->ev_in[b], p->cs_in));
+            PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_in[b], 0));
+            void* yout = nullptr;
+            pepp_status_t s = host_iterations(p, xa, xb, iterations, flags, st, &yout);
+            if (s) return s;
+            PEPP_CUDA_TRY(cudaEventRecord(p->ev_out[b], st));
+            PEPP_CUDA_TRY(cudaStreamWaitEvent(p->cs_out, p->ev_out[b], 0));
+            if (cnt > 0)
+                PEPP_CUDA_TRY(cudaMemcpyAsync((char*)y_hosts[k] + lo * (int64_t)p->esz,
+                                              (const char*)yout + lo * (int64_t)p->esz, p->esz * cnt,
+                                              cudaMemcpyDeviceToHost, p->cs_out));
+            PEPP_CUDA_TRY(cudaEventRecord(p->ev_free[b], p->cs_out));
+        }
+        PEPP_CUDA_TRY(cudaEventRecord(p->ev_end, p->cs_out));
+        PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_end, 0));
+        return PEPP_OK;
+    };
+    const pepp_status_t s = enqueue();
+    // on success the caller's stream has joined the copy streams; on failure
+    // drain all three so no copy still touches the caller's host buffers
+    bool ok = cudaStreamSynchronize(st) == cudaSuccess;
+    if (s) {
+        ok &= cudaStreamSynchronize(p->cs_in) == cudaSuccess;
+        ok &= cudaStreamSynchronize(p->cs_out) == cudaSuccess;
     }
-    PEPP_CUDA_TRY(cudaEventRecord(p->ev_end, p->cs_out));
-    PEPP_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_end, 0));
-    if (cudaStreamSynchronize(st) != cudaSuccess) { (void)cudaGetLastError(); p->sticky = PEPP_E_CUDA; return PEPP_E_CUDA; }
-    return PEPP_OK;
+    if (!ok) { (void)cudaGetLastError(); p->sticky = PEPP_E_CUDA; return PEPP_E_CUDA; }
+    return s;
 }
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_destroy(pepp_spmv_plan_t* p) {
