@@ -239,6 +239,45 @@ __device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __
     return acc;
 }
 
+// Two unmasked stencil chunks of N slots each (a warp's chunks i and i+1):
+// every load of both issued before the first FMA — twice the bytes in flight
+// of one chunk. Per row the same products and the same slot-order sums as
+// sell_slots: results are bit-identical. Measured on config 4: fp64 605 ->
+// 587 µs (DRAM 99 % of the copy peak), fp32 420 -> 436 µs, so it is compiled
+// into the fp64 kernel only.
+template <int N, typename T>
+__device__ __forceinline__ void sell_stencil_pair(const T* __restrict__ val, const T* __restrict__ x, int offa,
+                                                  int rowa, int64_t basea, int offb, int rowb, int64_t baseb,
+                                                  T& acca, T& accb, uint64_t pol) {
+    int ca[N], cb[N];
+    T va[N], vb[N], xa[N], xb[N];
+#pragma unroll
+    for (int u = 0; u < N; ++u) {
+        ca[u] = rowa + __shfl_sync(0xffffffffu, offa, u);
+        cb[u] = rowb + __shfl_sync(0xffffffffu, offb, u);
+    }
+#pragma unroll
+    for (int u = 0; u < N; ++u) {
+        va[u] = ld_stream_v(val + basea + (int64_t)u * 32, pol);
+        vb[u] = ld_stream_v(val + baseb + (int64_t)u * 32, pol);
+    }
+#pragma unroll
+    for (int u = 0; u < N; ++u) { xa[u] = ld_x(x, ca[u]); xb[u] = ld_x(x, cb[u]); }
+    acca = T(0);
+    accb = T(0);
+#pragma unroll
+    for (int u = 0; u < N; ++u) { acca = fma(va[u], xa[u], acca); accb = fma(vb[u], xb[u], accb); }
+}
+
+#ifndef PEPP_SELL_PAIR_F64
+#define PEPP_SELL_PAIR_F64 1   // measured (tools/gpu_pair.sh): fp64 605 -> 587 us on config 4
+#endif
+#ifndef PEPP_SELL_PAIR_F32
+#define PEPP_SELL_PAIR_F32 0   // fp32 420 -> 436 us: off
+#endif
+template <typename T>
+constexpr bool sell_pairs() { return std::is_same<T, float>::value ? PEPP_SELL_PAIR_F32 : PEPP_SELL_PAIR_F64; }
+
 template <int IDX, typename T>
 __device__ __forceinline__ T sell_chunk(const T* __restrict__ val, const int* __restrict__ col,
                                         const int16_t* __restrict__ col16, int offl, int row0,
@@ -482,6 +521,33 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
     for (; i < end; i += step) {
         const Desc q2 = desc(i + 2 * step);
         const Lane l1 = lanes(i + step, q1);
+        if constexpr (sell_pairs<T>() && !SORTED && !PAT) {
+            // chunks i and i+1 both unmasked stencil chunks of one length <= 8:
+            // both at once, then the pipeline moves two chunks on
+            const int pl = q0.d & kSellLenMask;
+            if (q1.d == q0.d && (q0.d & kSellStencil) && !(q0.d & kSellMasked) && pl >= 1 && pl <= 8 &&
+                i + step < end) {
+                const int ra = l0.orow, rb = l1.orow;
+                T a = T(0), b = T(0);
+                switch (pl) {
+                case 1: sell_stencil_pair<1, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
+                case 2: sell_stencil_pair<2, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
+                case 3: sell_stencil_pair<3, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
+                case 4: sell_stencil_pair<4, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
+                case 5: sell_stencil_pair<5, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
+                case 6: sell_stencil_pair<6, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
+                case 7: sell_stencil_pair<7, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
+                default: sell_stencil_pair<8, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
+                }
+                y[ra] = a;   // unmasked chunks: all 32 rows exist
+                y[rb] = b;
+                const Desc q3 = desc(i + 3 * step);
+                l0 = lanes(i + 2 * step, q2);
+                q0 = q2; q1 = q3;
+                i += step;   // + the loop's step
+                continue;
+            }
+        }
         const int c = chunk_of(i);
         const int64_t base = q0.cp + lane;
         const int clen = q0.d & kSellLenMask;

@@ -492,8 +492,9 @@ def test_torch_graph_capture_global_mode(calibrate):
         x = _dev(x0)
         y = torch.full((20_000,), float("nan"), dtype=torch.float64, device="cuda")
         if calibrate:
-            for _ in range(40):
-                plan.exec(x, y)
+            for _ in range(400):   # until calibration (with refinement rounds) is over
+                if not plan.exec(x, y).calibrating:
+                    break
             plan.flush_history()
         before = [plan.history_stats(c)[0] for c in range(len(plan.candidates()))]
         s = torch.cuda.Stream()
@@ -582,8 +583,10 @@ def test_cold_start_from_persisted_history(tmp_path):
     with pepp.Plan.from_csr(A, history_path=hist) as plan:
         assert plan.info()["prior_key"] == 0
         calls_a = 0
-        while plan.exec(x, y).calibrating:
+        seen_a = set()
+        while (u := plan.exec(x, y)).calibrating:
             calls_a += 1
+            seen_a.add(u.name)
         best_a = plan.select()
     B = gen.laplacian2d(1200)
     xb = _dev(gen.vector(46, gen.REAL, B.nrows))
@@ -594,9 +597,13 @@ def test_cold_start_from_persisted_history(tmp_path):
         first = plan.exec(xb, yb)
         assert first.calibrating and (first.variant, first.param) == (best_a.variant, best_a.param)
         calls_b = 1
-        while plan.exec(xb, yb).calibrating:
+        seen_b = {first.name}
+        while (u := plan.exec(xb, yb)).calibrating:
             calls_b += 1
-        assert calls_b < calls_a          # the prior ruled some candidates out
+            seen_b.add(u.name)
+        # the prior ruled some candidates out: never timed on B (the number
+        # of calls also depends on the refinement of noisy contenders)
+        assert seen_b < seen_a
 
 
 def test_entry_points_restore_the_callers_device():
