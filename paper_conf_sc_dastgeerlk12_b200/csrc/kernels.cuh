@@ -239,22 +239,31 @@ __device__ __forceinline__ T sell_slots(const T* __restrict__ val, const int* __
     return acc;
 }
 
-// Two unmasked stencil chunks of N slots each (a warp's chunks i and i+1):
+// Two unmasked chunks of N slots each and one format (a warp's chunks i and i+1):
 // every load of both issued before the first FMA — twice the bytes in flight
 // of one chunk. Per row the same products and the same slot-order sums as
 // sell_slots: results are bit-identical. Measured on config 4: fp64 605 ->
 // 587 µs (DRAM 99 % of the copy peak), fp32 420 -> 436 µs, so it is compiled
 // into the fp64 kernel only.
-template <int N, typename T>
-__device__ __forceinline__ void sell_stencil_pair(const T* __restrict__ val, const T* __restrict__ x, int offa,
-                                                  int rowa, int64_t basea, int offb, int rowb, int64_t baseb,
-                                                  T& acca, T& accb, uint64_t pol) {
+template <int N, int IDX, typename T>
+__device__ __forceinline__ void sell_pair(const T* __restrict__ val, const int* __restrict__ col,
+                                          const int16_t* __restrict__ col16, const T* __restrict__ x, int offa,
+                                          int rowa, int64_t basea, int offb, int rowb, int64_t baseb, T& acca,
+                                          T& accb, uint64_t pol) {
     int ca[N], cb[N];
     T va[N], vb[N], xa[N], xb[N];
 #pragma unroll
     for (int u = 0; u < N; ++u) {
-        ca[u] = rowa + __shfl_sync(0xffffffffu, offa, u);
-        cb[u] = rowb + __shfl_sync(0xffffffffu, offb, u);
+        if (IDX == kIdxStencil) {
+            ca[u] = rowa + __shfl_sync(0xffffffffu, offa, u);
+            cb[u] = rowb + __shfl_sync(0xffffffffu, offb, u);
+        } else if (IDX == kIdx16) {
+            ca[u] = rowa + ld_stream_i16(col16 + basea + (int64_t)u * 32, pol);
+            cb[u] = rowb + ld_stream_i16(col16 + baseb + (int64_t)u * 32, pol);
+        } else {
+            ca[u] = ld_stream_i(col + basea + (int64_t)u * 32, pol);
+            cb[u] = ld_stream_i(col + baseb + (int64_t)u * 32, pol);
+        }
     }
 #pragma unroll
     for (int u = 0; u < N; ++u) {
@@ -268,6 +277,27 @@ __device__ __forceinline__ void sell_stencil_pair(const T* __restrict__ val, con
 #pragma unroll
     for (int u = 0; u < N; ++u) { acca = fma(va[u], xa[u], acca); accb = fma(vb[u], xb[u], accb); }
 }
+
+template <int IDX, typename T>
+__device__ __forceinline__ void sell_pair_len(int n, const T* __restrict__ val, const int* __restrict__ col,
+                                              const int16_t* __restrict__ col16, const T* __restrict__ x, int offa,
+                                              int rowa, int64_t basea, int offb, int rowb, int64_t baseb, T& a,
+                                              T& b, uint64_t pol) {
+    switch (n) {
+    case 1: sell_pair<1, IDX, T>(val, col, col16, x, offa, rowa, basea, offb, rowb, baseb, a, b, pol); break;
+    case 2: sell_pair<2, IDX, T>(val, col, col16, x, offa, rowa, basea, offb, rowb, baseb, a, b, pol); break;
+    case 3: sell_pair<3, IDX, T>(val, col, col16, x, offa, rowa, basea, offb, rowb, baseb, a, b, pol); break;
+    case 4: sell_pair<4, IDX, T>(val, col, col16, x, offa, rowa, basea, offb, rowb, baseb, a, b, pol); break;
+    case 5: sell_pair<5, IDX, T>(val, col, col16, x, offa, rowa, basea, offb, rowb, baseb, a, b, pol); break;
+    case 6: sell_pair<6, IDX, T>(val, col, col16, x, offa, rowa, basea, offb, rowb, baseb, a, b, pol); break;
+    case 7: sell_pair<7, IDX, T>(val, col, col16, x, offa, rowa, basea, offb, rowb, baseb, a, b, pol); break;
+    default: sell_pair<8, IDX, T>(val, col, col16, x, offa, rowa, basea, offb, rowb, baseb, a, b, pol); break;
+    }
+}
+
+#ifndef PEPP_SELL_PAIR_ALL
+#define PEPP_SELL_PAIR_ALL 0   // also pair 16- / 32-bit column chunks (experiment)
+#endif
 
 #ifndef PEPP_SELL_PAIR_F64
 #define PEPP_SELL_PAIR_F64 1   // measured (tools/gpu_pair.sh): fp64 605 -> 587 us on config 4
@@ -525,20 +555,16 @@ __global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, con
             // chunks i and i+1 both unmasked stencil chunks of one length <= 8:
             // both at once, then the pipeline moves two chunks on
             const int pl = q0.d & kSellLenMask;
-            if (q1.d == q0.d && (q0.d & kSellStencil) && !(q0.d & kSellMasked) && pl >= 1 && pl <= 8 &&
-                i + step < end) {
+            const bool fmt_ok = (q0.d & kSellStencil) || PEPP_SELL_PAIR_ALL;
+            if (q1.d == q0.d && fmt_ok && !(q0.d & kSellMasked) && pl >= 1 && pl <= 8 && i + step < end) {
                 const int ra = l0.orow, rb = l1.orow;
                 T a = T(0), b = T(0);
-                switch (pl) {
-                case 1: sell_stencil_pair<1, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
-                case 2: sell_stencil_pair<2, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
-                case 3: sell_stencil_pair<3, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
-                case 4: sell_stencil_pair<4, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
-                case 5: sell_stencil_pair<5, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
-                case 6: sell_stencil_pair<6, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
-                case 7: sell_stencil_pair<7, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
-                default: sell_stencil_pair<8, T>(val, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol); break;
-                }
+                if (q0.d & kSellStencil)
+                    sell_pair_len<kIdxStencil, T>(pl, val, col, col16, x, l0.offl, ra, q0.cp + lane, l1.offl, rb, q1.cp + lane, a, b, pol);
+                else if (q0.d & kSellCol16)
+                    sell_pair_len<kIdx16, T>(pl, val, col, col16, x, 0, ra, q0.cp + lane, 0, rb, q1.cp + lane, a, b, pol);
+                else
+                    sell_pair_len<kIdx32, T>(pl, val, col, col16, x, 0, ra, q0.cp + lane, 0, rb, q1.cp + lane, a, b, pol);
                 y[ra] = a;   // unmasked chunks: all 32 rows exist
                 y[rb] = b;
                 const Desc q3 = desc(i + 3 * step);
