@@ -23,7 +23,9 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--compress", type=int, default=0,
                     help="opts.compress_values (0 = the bench headline's layout, 1 = pattern-table chunks)")
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"], help="value type (f32: the paper's float instance)")
     a = ap.parse_args()
+    import numpy as np
     import torch
 
     import paper_conf_sc_dastgeerlk12_b200 as pepp
@@ -31,9 +33,13 @@ def main():
     R = len(rp) - 1
     A = bench.make_block(a.workload, 0, R)
     x0 = bench.x0_vector(a.workload, A.ncols)
+    if a.dtype == "f32":
+        import gen
+        A = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float32), A.r0, A.global_nrows, A.name)
+        x0 = x0.astype(np.float32)
     plan = pepp.Plan.from_csr(A, compress_values=bool(a.compress))
     xs = torch.from_numpy(x0).cuda()
-    y = torch.empty(R, dtype=torch.float64, device="cuda")
+    y = torch.empty(R, dtype=torch.float32 if a.dtype == "f32" else torch.float64, device="cuda")
     vs = [bench.parse_variant(v) for v in a.variants.split(",") if v] or \
         [pepp.Choice(c.variant, c.param) for c in plan.candidates()]
     for f in vs:
