@@ -147,13 +147,32 @@ class Plan:
             o.predict = cb
         C.check(L.pepp_spmv_plan(ctypes.byref(A), ctypes.byref(o), ctypes.byref(self._h)), "pepp_spmv_plan")
         self.nrows, self.ncols, self.nnz = nrows, ncols, nnz
+        self._global_rows = int(self._bounds[-1]) if self._bounds is not None else nrows
 
     # ---- calls ----
+    def _vec(self, t, n: int, name: str) -> int:
+        """Device address of an operand: a contiguous CUDA tensor of the plan's
+        value type with at least `n` entries, or a raw device address (int,
+        unchecked). Host arrays are refused (exec_host takes those): the C
+        entry points get plain pointers and cannot tell."""
+        if t is None or isinstance(t, int):
+            return t or 0
+        if isinstance(t, np.ndarray):
+            raise TypeError(f"{name}: a host array; pass a CUDA tensor (or use exec_host / exec_host_batch)")
+        want = "float32" if self.value_type == C.VALUE_F32 else "float64"
+        if not getattr(t, "is_cuda", False) or str(t.dtype).rpartition(".")[2] != want:
+            raise TypeError(f"{name}: expected a CUDA {want} tensor, got {getattr(t, 'device', '?')} {t.dtype}")
+        if not t.is_contiguous() or t.numel() < n:
+            raise ValueError(f"{name}: needs a contiguous tensor of >= {n} entries, got {tuple(t.shape)}")
+        return int(t.data_ptr())
+
     def exec(self, x, y, flags: int = Y_LOCAL, stream=None, force: Optional[Choice] = None) -> Choice:
-        """y = A·x (x, y: CUDA float64 tensors; y global-length). Asynchronous on ``stream``."""
+        """y = A·x (x: ncols entries, y: global rows; CUDA tensors of the plan's
+        value type). Asynchronous on ``stream``."""
         used = C.CHOICE_T()
         f = force._to() if force is not None else None
-        C.check(C.lib().pepp_spmv_exec(self._h, _ptr(x), _ptr(y), flags, _stream_handle(stream),
+        px, py = self._vec(x, self.ncols, "x"), self._vec(y, self._global_rows, "y")
+        C.check(C.lib().pepp_spmv_exec(self._h, px, py, flags, _stream_handle(stream),
                                        ctypes.byref(f) if f is not None else None, ctypes.byref(used)),
                 "pepp_spmv_exec")
         return Choice._from(used)
@@ -173,13 +192,16 @@ class Plan:
         """Capture `iterations` calls into a CUDA graph (mode 0: repeat y = A·x;
         mode 1: iterate, ping-pong y / work)."""
         g = ctypes.c_void_p()
-        C.check(C.lib().pepp_spmv_graph_create(self._h, _ptr(x), _ptr(y), _ptr(work), iterations, mode, flags,
+        px, py = self._vec(x, self.ncols, "x"), self._vec(y, self._global_rows, "y")
+        pw = self._vec(work, self._global_rows, "work")
+        C.check(C.lib().pepp_spmv_graph_create(self._h, px, py, pw, iterations, mode, flags,
                                                _stream_handle(stream), ctypes.byref(g)), "pepp_spmv_graph_create")
         return Graph(g, (x, y, work))
 
     def exchange(self, y, flags: int = Y_NEXT_INPUT, stream=None) -> None:
         """The exchange step alone (no-op on an unpartitioned plan)."""
-        C.check(C.lib().pepp_spmv_exchange(self._h, _ptr(y), flags, _stream_handle(stream)), "pepp_spmv_exchange")
+        C.check(C.lib().pepp_spmv_exchange(self._h, self._vec(y, self._global_rows, "y"), flags, _stream_handle(stream)),
+                "pepp_spmv_exchange")
 
     def p2p_buffers(self, nbuf: int = 2) -> list:
         """pepp_spmv_p2p_buffers (collective): `nbuf` plan-owned symmetric
@@ -204,7 +226,9 @@ class Plan:
                   stream=None) -> None:
         """Host buffers in and out, transfers inside the call (synchronous)."""
         want = np.float32 if self.value_type == C.VALUE_F32 else np.float64
-        assert x_host.dtype == want and y_host.dtype == want
+        for a, n, name in ((x_host, self.ncols, "x_host"), (y_host, self._global_rows, "y_host")):
+            if not isinstance(a, np.ndarray) or a.dtype != want or not a.flags.c_contiguous or a.size < n:
+                raise ValueError(f"{name}: needs a contiguous {np.dtype(want).name} array of >= {n} entries")
         C.check(C.lib().pepp_spmv_exec_host(self._h, _ptr(x_host), _ptr(y_host), iterations, flags,
                                             _stream_handle(stream)), "pepp_spmv_exec_host")
 
@@ -213,8 +237,12 @@ class Plan:
         """exec_host over independent right-hand sides, transfers overlapped
         with the computation (synchronous)."""
         want = np.float32 if self.value_type == C.VALUE_F32 else np.float64
-        assert len(x_hosts) == len(y_hosts)
-        assert all(a.dtype == want for a in x_hosts) and all(a.dtype == want for a in y_hosts)
+        if len(x_hosts) != len(y_hosts):
+            raise ValueError("x_hosts and y_hosts differ in length")
+        for arrs, n, name in ((x_hosts, self.ncols, "x_hosts"), (y_hosts, self._global_rows, "y_hosts")):
+            for a in arrs:
+                if not isinstance(a, np.ndarray) or a.dtype != want or not a.flags.c_contiguous or a.size < n:
+                    raise ValueError(f"{name}: needs contiguous {np.dtype(want).name} arrays of >= {n} entries")
         n = len(x_hosts)
         xs = (ctypes.c_void_p * max(n, 1))(*[_ptr(a) for a in x_hosts])
         ys = (ctypes.c_void_p * max(n, 1))(*[_ptr(a) for a in y_hosts])

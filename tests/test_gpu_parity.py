@@ -336,8 +336,10 @@ def test_error_codes():
         with pytest.raises(pepp.PeppError) as e:
             plan.exec(x, x)                       # x and y alias
         assert e.value.status == pepp._capi.PEPP_E_INVALID
-        with pytest.raises(pepp.PeppError):
-            plan.exec(x, x[10:])                  # overlap
+        z = torch.ones(512, dtype=torch.float64, device="cuda")
+        with pytest.raises(pepp.PeppError) as e:
+            plan.exec(z[:256], z[10:266])         # overlap (the C-ABI's check)
+        assert e.value.status == pepp._capi.PEPP_E_INVALID
     bad = gen.laplacian2d(16)
     bad.col = bad.col.copy()
     bad.col[7] = 256                              # column out of range
@@ -720,3 +722,26 @@ def test_value_compression_long_patterns(name):
         assert i1["sell_constval_frac"] >= 0.5
         assert np.array_equal(y1.view(np.int64), y0.view(np.int64))
         _check(A, x, y1, bool(np.all(x == np.round(x))))
+
+
+def test_binding_refuses_bad_operands():
+    """The binding checks what the C-ABI's plain pointers cannot carry: host
+    arrays, wrong dtype, non-contiguous or short tensors raise before any
+    launch; the plan stays usable."""
+    A = gen.laplacian2d(32)
+    x0 = gen.vector(3, gen.INT8, A.ncols)
+    with pepp.Plan.from_csr(A) as plan:
+        x, y = _dev(x0), torch.empty(A.nrows, dtype=torch.float64, device="cuda")
+        with pytest.raises(TypeError):
+            plan.exec(x0, y)                                   # host array
+        with pytest.raises(TypeError):
+            plan.exec(x.float(), y)                            # wrong value type
+        with pytest.raises(ValueError):
+            plan.exec(x[: A.ncols - 1], y)                     # short
+        with pytest.raises(ValueError):
+            plan.exec(torch.stack([x, x], 1)[:, 0], y)         # strided view
+        with pytest.raises(ValueError):
+            plan.exec_host(x0, np.empty(A.nrows - 1))
+        plan.exec(x, y)
+        torch.cuda.synchronize()
+        assert np.array_equal(y.cpu().numpy(), oracle.spmv(A, x0))
