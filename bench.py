@@ -458,6 +458,18 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
+    # one cold call (fresh plan, first launch of the process's kernels on this
+    # matrix) — reported for launch-bound workloads
+    cold_us = None
+    if not iterated and A.nnz < 10_000_000:
+        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        with torch.cuda.stream(stream):
+            c0.record(stream)
+            plan.exec(xs, bufs[0], flags=flags, stream=stream)
+            c1.record(stream)
+        c1.synchronize()
+        cold_us = round(c0.elapsed_time(c1) * 1e3, 2)
     for _ in range(args.warmup):
         one_step(False)
     torch.cuda.synchronize()
@@ -563,7 +575,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             e1.record(stream)
         e1.synchronize()
         us = e0.elapsed_time(e1) * 1e3 / (reps * ncalls)
-        graph_info = {"calls": ncalls, "us_per_call": round(us, 3),
+        graph_info = {"calls": ncalls, "us_per_call": round(us, 3), "cold_first_call_us": cold_us,
                       "gflops": round(2.0 * Z / (us * 1e-6) / 1e9, 3),
                       "note": "back-to-back calls replayed from one CUDA graph (pepp_spmv_graph_*); L2-warm"}
         g.close()
