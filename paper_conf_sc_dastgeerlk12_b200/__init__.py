@@ -31,7 +31,7 @@ __all__ = ["Plan", "Choice", "History", "Vector", "ACCESS_READ", "ACCESS_WRITE",
 lib_path = C.LIB_PATH
 
 
-@dataclass
+@dataclass(slots=True)
 class Choice:
     variant: int
     param: int = 0
@@ -71,6 +71,9 @@ def _stream_handle(stream) -> int:
         import torch
         if not torch.cuda.is_available():
             return 0   # legacy default stream (the library reports PEPP_E_CUDA where a device is needed)
+        raw = getattr(torch._C, "_cuda_getCurrentRawStream", None)   # torch's current stream, without a Stream object
+        if raw is not None:
+            return int(raw(torch._C._cuda_getDevice()))
         return int(torch.cuda.current_stream().cuda_stream)
     if isinstance(stream, int):
         return stream
@@ -148,6 +151,16 @@ class Plan:
         C.check(L.pepp_spmv_plan(ctypes.byref(A), ctypes.byref(o), ctypes.byref(self._h)), "pepp_spmv_plan")
         self.nrows, self.ncols, self.nnz = nrows, ncols, nnz
         self._global_rows = int(self._bounds[-1]) if self._bounds is not None else nrows
+        # per-call fast path of exec: the bound C function, a reused result struct,
+        # the torch dtype of the plan's value type (None without torch)
+        self._fexec = L.pepp_spmv_exec
+        self._used = C.CHOICE_T()
+        self._used_ref = ctypes.byref(self._used)
+        try:
+            import torch
+            self._tdtype = torch.float32 if f32 else torch.float64
+        except ImportError:
+            self._tdtype = None
 
     # ---- calls ----
     def _vec(self, t, n: int, name: str) -> int:
@@ -155,6 +168,9 @@ class Plan:
         value type with at least `n` entries, or a raw device address (int,
         unchecked). Host arrays are refused (exec_host takes those): the C
         entry points get plain pointers and cannot tell."""
+        td = self._tdtype
+        if td is not None and getattr(t, "dtype", None) is td and t.is_cuda and t.is_contiguous() and t.numel() >= n:
+            return t.data_ptr()   # the common case, checked cheaply
         if t is None or isinstance(t, int):
             return t or 0
         if isinstance(t, np.ndarray):
@@ -169,13 +185,13 @@ class Plan:
     def exec(self, x, y, flags: int = Y_LOCAL, stream=None, force: Optional[Choice] = None) -> Choice:
         """y = A·x (x: ncols entries, y: global rows; CUDA tensors of the plan's
         value type). Asynchronous on ``stream``."""
-        used = C.CHOICE_T()
-        f = force._to() if force is not None else None
+        f = ctypes.byref(force._to()) if force is not None else None
         px, py = self._vec(x, self.ncols, "x"), self._vec(y, self._global_rows, "y")
-        C.check(C.lib().pepp_spmv_exec(self._h, px, py, flags, _stream_handle(stream),
-                                       ctypes.byref(f) if f is not None else None, ctypes.byref(used)),
-                "pepp_spmv_exec")
-        return Choice._from(used)
+        st = stream.cuda_stream if hasattr(stream, "cuda_stream") else _stream_handle(stream)
+        r = self._fexec(self._h, px, py, flags, st, f, self._used_ref)
+        if r:
+            C.check(r, "pepp_spmv_exec")
+        return Choice._from(self._used)
 
     def exec_vec(self, x: "Vector", y: "Vector", flags: int = Y_LOCAL, stream=None,
                  force: Optional[Choice] = None) -> Choice:

@@ -153,6 +153,7 @@ struct pepp_spmv_plan_s {
     pepp_history* hist = nullptr;
     uint64_t key = 0;
     int64_t ncalls = 0;
+    bool calibrated = false;   // calibration (rounds + refinement) finished: exploit without rescanning
 
     // timing ring
     TimingRec ring[kTimingRing];
@@ -934,14 +935,12 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out, bool frozen
         const int32_t ms = std::max(1, p->opts.min_samples);
         const int32_t n = (int32_t)p->cands.size();
         auto hget = [&](int32_t c) { return pepp::history_get(p->hist, p->key, p->uids[c]); };
-        double best_mean = -1.0;
-        for (int32_t c = 0; c < n; ++c) {
+        double best_mean = -1.0, prior_best = -1.0;
+        for (int32_t c = 0; c < n && !p->calibrated; ++c) {
             const pepp::Welford* w = hget(c);
             if (p->eligible[c] && w && w->count > 0 && (best_mean < 0 || w->mean < best_mean)) best_mean = w->mean;
-        }
-        double prior_best = -1.0;
-        for (int32_t c = 0; c < n; ++c)
             if (p->eligible[c] && p->prior[c] > 0 && (prior_best < 0 || p->prior[c] < prior_best)) prior_best = p->prior[c];
+        }
         // ruled out: own samples > 4x the best own mean, or (never sampled) a
         // prior > 4x the best prior from the nearest recorded context
         auto ruled_out = [&](int32_t c, const pepp::Welford* w) {
@@ -954,7 +953,9 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out, bool frozen
             return k >= 2 ? pepp::kRefineRounds * ms : ms;
         };
         cand = -1;
-        for (int32_t r = 1; r <= rounds() && cand < 0; ++r) {
+        // once calibration has finished it stays finished (sample counts only
+        // grow): the per-call path skips the round scan (select < 1 µs)
+        for (int32_t r = 1; !p->calibrated && r <= rounds() && cand < 0; ++r) {
             // round r: every candidate not yet ruled out gets its r-th timed call
             // (calls still in flight count, so the host can run ahead of the GPU);
             // rounds past ms refine only the contenders (within kContendFactor
@@ -990,6 +991,7 @@ pepp_status_t select_choice(pepp_spmv_plan_t* p, pepp_choice_t* out, bool frozen
             }
         }
         if (cand < 0) {
+            p->calibrated = true;
             // exploitation: argmin of the measured means, ties within 1 % -> lower index (A10)
             double bt = 0.0;
             for (int32_t c = 0; c < n; ++c) {
