@@ -455,6 +455,144 @@ __device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int p
     }
 }
 
+// Stencil list (σ = 1 plans whose stencil chunks keep their values, i.e. not
+// pattern chunks): the unmasked stencil chunks of up to 8 slots, as entries
+// {chunk | pattern id << 26, chunk_ptr / 32} grouped by their offset pattern;
+// the distinct offset sets (<= 32) travel in the kernel's parameter space.
+// A warp walks its entries U at a time with the pattern's offsets held in
+// registers — no chunk descriptor, no per-lane offset load, no masks: per
+// chunk only the value stream, the x gathers and the y store. The other
+// chunks go through sell_kernel over the plan's genlist.
+constexpr int kSellMaxStencils = 32;
+#ifndef PEPP_SLIST_U_F64
+#define PEPP_SLIST_U_F64 8   // measured (tools/gpu_slist.sh): U = 2 / 4 / 8 -> 595 / 627 / 585 us, general walk 593
+#endif
+#ifndef PEPP_SLIST_U_F32
+#define PEPP_SLIST_U_F32 4   // U = 2 / 4 / 8 -> 373 / 360 / 459 us, general walk 421
+#endif
+template <typename T>
+constexpr int sell_slist_u() { return std::is_same<T, float>::value ? PEPP_SLIST_U_F32 : PEPP_SLIST_U_F64; }
+struct SellStencils {
+    int len[kSellMaxStencils];
+    int off[kSellMaxStencils][kSellMaxPatternLen];
+};
+
+template <int U>
+__device__ __forceinline__ void sell_slist_ids(const int2* __restrict__ list, int n, int k0, int stride,
+                                               int2 (&q)[U]) {
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+        const int kk = k0 + u * stride;
+        q[u] = kk < n ? __ldg(list + kk) : make_int2(-1, 0);
+    }
+}
+
+template <int U, int N, typename T>
+__device__ __forceinline__ void sell_slist_chunks(const int (&o)[N], const int2 (&q)[U], int lane,
+                                                  const T* __restrict__ val, const T* __restrict__ x,
+                                                  T* __restrict__ y, uint64_t pol) {
+    T v[U][N], xv[U][N];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+        const int64_t base = (int64_t)q[u].y * 32 + lane;
+#pragma unroll
+        for (int j = 0; j < N; ++j) v[u][j] = q[u].x >= 0 ? ld_stream_v(val + base + (int64_t)j * 32, pol) : T(0);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+        const int r = (q[u].x & ((1 << 26) - 1)) * 32 + lane;
+#pragma unroll
+        for (int j = 0; j < N; ++j) xv[u][j] = q[u].x >= 0 ? ld_x(x, r + o[j]) : T(0);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+        T acc = T(0);
+#pragma unroll
+        for (int j = 0; j < N; ++j) acc = fma(v[u][j], xv[u][j], acc);   // slot order = the row's CSR order
+        if (q[u].x >= 0) y[(q[u].x & ((1 << 26) - 1)) * 32 + lane] = acc;
+    }
+}
+
+// a run of groups whose entries all have pattern `pid` (N slots); returns
+// the list index of the first group that does not (q then holds it)
+template <int U, int N, typename T>
+__device__ __forceinline__ int sell_slist_run(const SellStencils& st, int pid, const int2* __restrict__ list, int n,
+                                              int k0, int stride, int2 (&q)[U], int lane, const T* __restrict__ val,
+                                              const T* __restrict__ x, T* __restrict__ y, uint64_t pol) {
+    int o[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) o[j] = st.off[pid][j];
+    for (; k0 < n; k0 += U * stride) {
+        bool uni = true;
+#pragma unroll
+        for (int u = 0; u < U; ++u) uni &= q[u].x < 0 || (q[u].x >> 26) == pid;
+        if (!uni) return k0;
+        int2 qn[U];
+        sell_slist_ids<U>(list, n, k0 + U * stride, stride, qn);
+        sell_slist_chunks<U, N, T>(o, q, lane, val, x, y, pol);
+#pragma unroll
+        for (int u = 0; u < U; ++u) q[u] = qn[u];
+    }
+    return k0;
+}
+
+template <int U, int N, typename T>
+__device__ __forceinline__ void sell_slist_one(const SellStencils& st, int2 e, int lane, const T* __restrict__ val,
+                                               const T* __restrict__ x, T* __restrict__ y, uint64_t pol) {
+    int o[N];
+    const int pid = e.x >> 26;
+#pragma unroll
+    for (int j = 0; j < N; ++j) o[j] = st.off[pid][j];
+    int2 q[U];
+    q[0] = e;
+#pragma unroll
+    for (int u = 1; u < U; ++u) q[u] = make_int2(-1, 0);
+    sell_slist_chunks<U, N, T>(o, q, lane, val, x, y, pol);
+}
+
+template <int BLOCK, int U, typename T>
+__global__ void __launch_bounds__(BLOCK) sell_slist_kernel(const int2* __restrict__ list, int n,
+                                                           const __grid_constant__ SellStencils st,
+                                                           const T* __restrict__ val, const T* __restrict__ x,
+                                                           T* __restrict__ y) {
+    const int lane = threadIdx.x & 31;
+    const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
+    const int nwarps = (gridDim.x * BLOCK) >> 5;
+    const uint64_t pol = evict_first_policy();
+    int2 e[U];
+    int k0 = warp;
+    sell_slist_ids<U>(list, n, k0, nwarps, e);
+    while (k0 < n) {
+        const int pid = e[0].x >> 26;
+        switch (st.len[pid]) {
+        case 1: k0 = sell_slist_run<U, 1, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
+        case 2: k0 = sell_slist_run<U, 2, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
+        case 3: k0 = sell_slist_run<U, 3, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
+        case 4: k0 = sell_slist_run<U, 4, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
+        case 5: k0 = sell_slist_run<U, 5, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
+        case 6: k0 = sell_slist_run<U, 6, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
+        case 7: k0 = sell_slist_run<U, 7, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
+        default: k0 = sell_slist_run<U, 8, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
+        }
+        if (k0 >= n) break;
+        for (int u = 0; u < U; ++u) {   // a group that straddles two patterns
+            if (e[u].x < 0) continue;
+            switch (st.len[e[u].x >> 26]) {
+            case 1: sell_slist_one<U, 1, T>(st, e[u], lane, val, x, y, pol); break;
+            case 2: sell_slist_one<U, 2, T>(st, e[u], lane, val, x, y, pol); break;
+            case 3: sell_slist_one<U, 3, T>(st, e[u], lane, val, x, y, pol); break;
+            case 4: sell_slist_one<U, 4, T>(st, e[u], lane, val, x, y, pol); break;
+            case 5: sell_slist_one<U, 5, T>(st, e[u], lane, val, x, y, pol); break;
+            case 6: sell_slist_one<U, 6, T>(st, e[u], lane, val, x, y, pol); break;
+            case 7: sell_slist_one<U, 7, T>(st, e[u], lane, val, x, y, pol); break;
+            default: sell_slist_one<U, 8, T>(st, e[u], lane, val, x, y, pol); break;
+            }
+        }
+        k0 += U * nwarps;
+        sell_slist_ids<U>(list, n, k0, nwarps, e);
+    }
+}
+
 struct NoPatterns {};
 template <bool PAT, typename T>
 using SellPatternArg = std::conditional_t<PAT, SellPatterns<T>, NoPatterns>;

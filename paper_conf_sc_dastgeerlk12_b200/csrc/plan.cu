@@ -33,6 +33,10 @@ constexpr int kBlock = 256;
 constexpr int kSellCapMin = 64;       // hybrid SELL: floor of the cap (prepare_sell_long)
 constexpr int64_t kChunkCost = 4;     // SELL per-chunk overhead in slot-equivalents (warp ranges, hybrid cap)
 constexpr int64_t kSellMidMax = 1024; // hybrid rows up to this length: one warp each (sell_mid_kernel)
+#ifndef PEPP_SLIST_F64
+#define PEPP_SLIST_F64 0
+#endif
+constexpr bool kSlistF64 = PEPP_SLIST_F64;   // stencil list for fp64 plans too (sell_stencil_list)
 constexpr int kMergeBlock = 256;
 constexpr int kMergeIPT = 7;
 constexpr int kMergeTile = kMergeBlock * kMergeIPT;
@@ -106,6 +110,9 @@ struct pepp_spmv_plan_s {
     int* d_patlist = nullptr;        // σ = 1: pattern chunks as (chunk << 5 | id), phase A of the kernel
     int* d_genlist = nullptr;        // σ = 1: the other chunks, phase B
     int npatc = 0, ngen = 0;
+    int2* d_stlist = nullptr;        // σ = 1, values streamed: stencil-list entries (sell_slist_kernel)
+    int nstc = 0, grid_slist = 0;
+    pepp::k::SellStencils stab{};    // the distinct offset sets of the stencil list (kernel parameter)
     pepp::k::SellPatterns<double> pat64{};   // the pattern table, passed by value to the SELL kernel
     pepp::k::SellPatterns<float> pat32{};
     int64_t sell_stencil_chunks = 0;
@@ -283,7 +290,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
                     p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist,
-                    p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, p->d_sell_part, p->d_sell_mid};
+                    p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, p->d_sell_part, p->d_sell_mid, p->d_stlist};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -484,6 +491,8 @@ pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
     return PEPP_OK;
 }
 
+pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p);
+
 pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     const int n = (int)p->nrows;
     p->nchunks = (n + 31) / 32;
@@ -614,6 +623,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
         if (n16 == 0) { cudaFree(p->d_scol16); p->d_scol16 = nullptr; p->dev_bytes -= (int64_t)sizeof(int16_t) * (p->sell_slots + 32); }
     }
     PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    if ((s = sell_stencil_list(p))) return s;
     p->sell_cpw = sigma > 1 ? std::max(1, sigma / 32) : 1;
     p->info.sell_sigma = sigma;
     p->info.sell_col16_frac = p->nchunks ? (double)p->sell_col16_chunks / (double)p->nchunks : 0.0;
@@ -622,6 +632,71 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->info.sell_fill = fill;
     p->info.sell_long_rows = p->nsell_long + p->nsell_mid;
     p->info.sell_cap = p->sell_cap == INT32_MAX ? 0 : p->sell_cap;
+    return PEPP_OK;
+}
+
+// Stencil list for σ = 1 plans whose stencil chunks stream their values (no
+// pattern table): unmasked stencil chunks of <= 8 slots, grouped by offset
+// set (<= kSellMaxStencils sets; chunks of further sets stay general), for
+// sell_slist_kernel; every other chunk goes to the genlist for sell_kernel.
+pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
+    using pepp::k::kSellLenMask;
+    const int nc = p->nchunks;
+    if (p->d_perm || p->d_patlist || p->sell_stencil_chunks == 0 || nc <= 0) return PEPP_OK;
+    if (const char* e = std::getenv("PEPP_NO_SLIST")) if (std::atoi(e)) return PEPP_OK;   // experiments only
+    // measured on config 4 (tools/gpu_slist2.sh, 3 alternating repeats): fp32
+    // 424 -> 361 µs (the issue-limited general walk loses its per-chunk
+    // instructions); fp64 584.0 -> 582.5 µs, i.e. nothing for a second launch,
+    // so the fp64 plans keep the one-kernel general walk (with paired chunks)
+    if (p->vt == PEPP_VALUE_F64 && !kSlistF64) return PEPP_OK;
+    const int64_t nsb = p->sell_slots / 32 + 8;
+    std::vector<int> clen(nc), soff(nsb);
+    std::vector<int64_t> cp(nc + 1);
+    PEPP_CUDA_TRY(cudaMemcpy(clen.data(), p->d_chunk_len, sizeof(int) * nc, cudaMemcpyDeviceToHost));
+    PEPP_CUDA_TRY(cudaMemcpy(cp.data(), p->d_chunk_ptr, sizeof(int64_t) * (nc + 1), cudaMemcpyDeviceToHost));
+    PEPP_CUDA_TRY(cudaMemcpy(soff.data(), p->d_soff, sizeof(int) * nsb, cudaMemcpyDeviceToHost));
+    pepp::k::SellStencils tab{};
+    int nset = 0;
+    std::vector<int2> lst;
+    std::vector<int> gen;
+    lst.reserve(nc);
+    for (int c = 0; c < nc; ++c) {
+        const int d = clen[c], len = d & kSellLenMask;
+        int pid = -1;
+        if ((d & pepp::k::kSellStencil) && !(d & pepp::k::kSellMasked) && len >= 1 && len <= pepp::k::kSellMaxPatternLen &&
+            c < (1 << 26) && (cp[c] >> 5) <= INT32_MAX) {
+            const int64_t sb = cp[c] >> 5;
+            for (int q = 0; q < nset && pid < 0; ++q) {
+                bool same = tab.len[q] == len;
+                for (int j = 0; same && j < len; ++j) same = tab.off[q][j] == soff[sb + j];
+                if (same) pid = q;
+            }
+            if (pid < 0 && nset < pepp::k::kSellMaxStencils) {
+                pid = nset++;
+                tab.len[pid] = len;
+                for (int j = 0; j < len; ++j) tab.off[pid][j] = soff[sb + j];
+            }
+        }
+        if (pid >= 0) lst.push_back(make_int2(c | (pid << 26), (int)(cp[c] >> 5)));
+        else gen.push_back(c);
+    }
+    if (lst.empty()) return PEPP_OK;
+    std::stable_sort(lst.begin(), lst.end(), [](const int2& a, const int2& b) { return (a.x >> 26) < (b.x >> 26); });
+    pepp_status_t s;
+    if ((s = dalloc(p, &p->d_stlist, (int64_t)lst.size()))) return s;
+    if ((s = dalloc(p, &p->d_genlist, (int64_t)gen.size()))) return s;
+    PEPP_CUDA_TRY(cudaMemcpy(p->d_stlist, lst.data(), sizeof(int2) * lst.size(), cudaMemcpyHostToDevice));
+    if (!gen.empty()) PEPP_CUDA_TRY(cudaMemcpy(p->d_genlist, gen.data(), sizeof(int) * gen.size(), cudaMemcpyHostToDevice));
+    p->nstc = (int)lst.size();
+    p->ngen = (int)gen.size();
+    p->stab = tab;
+    int occ = 0;
+    const void* fn = p->vt == PEPP_VALUE_F32 ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<float>(), float>
+                                             : (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<double>(), double>;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
+    (void)cudaGetLastError();
+    const int64_t need = ((int64_t)p->nstc + kBlock / 32 - 1) / (kBlock / 32);
+    p->grid_slist = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ));
     return PEPP_OK;
 }
 
@@ -810,7 +885,15 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                 (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
                 p->d_patlist, p->npatc, p->d_genlist);
-        else
+        else if (p->d_stlist) {   // stencil list (values streamed), then the other chunks
+            pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), T><<<p->grid_slist, kBlock, 0, st>>>(p->d_stlist, p->nstc, p->stab,
+                                                                                   (const T*)p->d_sval, x, y);
+            if (p->ngen > 0)   // the genlist walk of the PAT instance, with no pattern chunks (phase A empty)
+                pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, st>>>(
+                    (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
+                    p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
+                    nullptr, 0, p->d_genlist);
+        } else
             pepp::k::sell_kernel<kBlock, false, false, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, pepp::k::NoPatterns{}, (const T*)p->d_sval, x, y, 1, nullptr,
@@ -837,7 +920,7 @@ int launches_for(const pepp_spmv_plan_t* p, const Candidate& c) {
         if (c.param == kMergeWarpParam) return p->ntiles_w > 0 ? 2 + (p->nlongruns_w > 0) : 0;
         return p->ntiles > 0 ? 2 + (p->nlongruns > 0) : 0;
     case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
-    case PEPP_V_SELL: return 1 + (p->nsell_mid > 0) + (p->nsell_seg > 0);
+    case PEPP_V_SELL: return (p->d_stlist ? 1 + (p->ngen > 0) : 1) + (p->nsell_mid > 0) + (p->nsell_seg > 0);
     default: return 0;
     }
 }

@@ -38,13 +38,17 @@ def _run(plan, x, force=None):
     return y.cpu().numpy(), used
 
 
+@pytest.mark.parametrize("compress", [True, False])
 @pytest.mark.parametrize("case", sorted(CASES))
-def test_every_variant_fp32(case):
+def test_every_variant_fp32(case, compress):
+    """compress = False keeps stencil values streamed: the fp32 SELL plan then
+    runs its stencil chunks through the stencil-list kernel (sell_slist_kernel)
+    and the rest through the genlist walk."""
     A, x, exact = CASES[case]()
     A32, x32 = _f32(A), x.astype(np.float32)
     ref = oracle.spmv(A32, x32)
     assert ref.dtype == np.float32
-    with pepp.Plan.from_csr(A32, prune=False) as plan:
+    with pepp.Plan.from_csr(A32, prune=False, compress_values=compress) as plan:
         assert plan.value_type == pepp._capi.VALUE_F32
         forces = [pepp.Choice(c.variant, c.param) for c in plan.candidates()]
         assert {f.variant for f in forces} == {pepp.V_CSR_VECTOR, pepp.V_MERGE_PATH, pepp.V_SELL, pepp.V_CSR_STREAM}
@@ -96,3 +100,18 @@ def test_fp32_differs_from_fp64_where_float_rounds():
     with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_CSR_STREAM) as plan:
         y, _ = _run(plan, x)
     assert y[0] == np.float32(1.0) == oracle.spmv(A, x)[0]
+
+
+def test_fp32_stencil_list_large_bitwise():
+    """The fp32 stencil-list path at a size spanning many warps and the
+    straddling groups between offset sets (a 1024² Laplacian has 3 stencil
+    offset sets plus the general boundary chunks): integer inputs bit-exact,
+    launches = stencil-list kernel + genlist walk."""
+    A = gen.laplacian2d(1024)
+    A32 = _f32(A)
+    x32 = gen.vector(7, gen.INT8, A.ncols).astype(np.float32)
+    ref = oracle.spmv(A32, x32)
+    with pepp.Plan.from_csr(A32, variant_mask=1 << pepp.V_SELL, compress_values=False) as plan:
+        y, used = _run(plan, x32)
+        assert used.launches == 2
+        assert np.array_equal(y, ref)

@@ -73,6 +73,15 @@ def main() -> int:
         bad += 0 if np.array_equal(w.host(pepp.ACCESS_READ), oracle.spmv(A, oracle.spmv(A, x0))) else 1
         for c in (u, v, w):
             c.close()
+    # fp32 stencil list (values streamed) + its genlist walk
+    A32 = gen.laplacian2d(96)
+    A32 = gen.CSR(A32.nrows, A32.ncols, A32.row_ptr, A32.col, A32.val.astype(np.float32), A32.r0, A32.global_nrows, A32.name)
+    x32 = gen.vector(3, gen.INT8, A32.ncols).astype(np.float32)
+    with pepp.Plan.from_csr(A32, compress_values=False) as plan:
+        y32 = torch.full((A32.nrows,), float("nan"), dtype=torch.float32, device="cuda")
+        plan.exec(torch.from_numpy(x32).cuda(), y32, force=pepp.Choice(pepp.V_SELL, 0))
+        torch.cuda.synchronize()
+        bad += 0 if np.array_equal(y32.cpu().numpy(), oracle.spmv(A32, x32)) else 1
     # overlapped host batch (copy streams, two device slots)
     with pepp.Plan.from_csr(A) as plan:
         xs = [gen.vector(30 + k, gen.INT8, A.nrows) for k in range(3)]
