@@ -37,6 +37,10 @@ constexpr int64_t kSellMidMax = 1024; // hybrid rows up to this length: one warp
 #define PEPP_SLIST_F64 0
 #endif
 constexpr bool kSlistF64 = PEPP_SLIST_F64;   // stencil list for fp64 plans too (sell_stencil_list)
+#ifndef PEPP_SLIST_CONCURRENT
+#define PEPP_SLIST_CONCURRENT 1
+#endif
+constexpr bool kSlistConcurrent = PEPP_SLIST_CONCURRENT;   // genlist walk on a second stream
 constexpr int kMergeBlock = 256;
 constexpr int kMergeIPT = 7;
 constexpr int kMergeTile = kMergeBlock * kMergeIPT;
@@ -112,6 +116,8 @@ struct pepp_spmv_plan_s {
     int npatc = 0, ngen = 0;
     int2* d_stlist = nullptr;        // σ = 1, values streamed: stencil-list entries (sell_slist_kernel)
     int nstc = 0, grid_slist = 0;
+    cudaStream_t gside = nullptr;                // the genlist walk's stream (concurrent with the list kernel)
+    cudaEvent_t ev_gfork = nullptr, ev_gjoin = nullptr;
     pepp::k::SellStencils stab{};    // the distinct offset sets of the stencil list (kernel parameter)
     pepp::k::SellPatterns<double> pat64{};   // the pattern table, passed by value to the SELL kernel
     pepp::k::SellPatterns<float> pat32{};
@@ -305,6 +311,9 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->ev_fork) cudaEventDestroy(p->ev_fork);
     if (p->ev_join) cudaEventDestroy(p->ev_join);
     if (p->ev_scratch) cudaEventDestroy(p->ev_scratch);
+    if (p->ev_gfork) cudaEventDestroy(p->ev_gfork);
+    if (p->ev_gjoin) cudaEventDestroy(p->ev_gjoin);
+    if (p->gside) cudaStreamDestroy(p->gside);
     if (p->side) cudaStreamDestroy(p->side);
     for (void* b : p->d_hb) if (b) cudaFree(b);
     for (cudaEvent_t e : {p->ev_start, p->ev_end, p->ev_in[0], p->ev_in[1], p->ev_out[0], p->ev_out[1], p->ev_free[0], p->ev_free[1]})
@@ -690,6 +699,11 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
     p->nstc = (int)lst.size();
     p->ngen = (int)gen.size();
     p->stab = tab;
+    if (p->ngen > 0 && kSlistConcurrent) {
+        PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->gside, cudaStreamNonBlocking));
+        PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gfork, cudaEventDisableTiming));
+        PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gjoin, cudaEventDisableTiming));
+    }
     int occ = 0;
     const void* fn = p->vt == PEPP_VALUE_F32 ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<float>(), float>
                                              : (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<double>(), double>;
@@ -885,14 +899,23 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                 (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
                 p->d_patlist, p->npatc, p->d_genlist);
-        else if (p->d_stlist) {   // stencil list (values streamed), then the other chunks
+        else if (p->d_stlist) {   // stencil list (values streamed) and the other chunks (disjoint rows)
+            // the small, latency-bound genlist walk runs beside the list kernel
+            // on the plan's second stream when it has one (kSlistConcurrent)
+            cudaStream_t gs = p->gside ? p->gside : st;
+            if (p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
+                             cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
+                return PEPP_E_CUDA;
             pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), T><<<p->grid_slist, kBlock, 0, st>>>(p->d_stlist, p->nstc, p->stab,
                                                                                    (const T*)p->d_sval, x, y);
             if (p->ngen > 0)   // the genlist walk of the PAT instance, with no pattern chunks (phase A empty)
-                pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, st>>>(
+                pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, gs>>>(
                     (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                     p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
                     nullptr, 0, p->d_genlist);
+            if (p->gside && (cudaEventRecord(p->ev_gjoin, p->gside) != cudaSuccess ||
+                             cudaStreamWaitEvent(st, p->ev_gjoin, 0) != cudaSuccess))
+                return PEPP_E_CUDA;
         } else
             pepp::k::sell_kernel<kBlock, false, false, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,

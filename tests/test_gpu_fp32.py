@@ -115,3 +115,12 @@ def test_fp32_stencil_list_large_bitwise():
         y, used = _run(plan, x32)
         assert used.launches == 2
         assert np.array_equal(y, ref)
+        # the same path captured in a CUDA graph (the genlist walk's fork /
+        # join onto the plan's second stream becomes a graph branch)
+        xd = torch.from_numpy(x32).cuda()
+        yd = torch.full((A.nrows,), float("nan"), dtype=torch.float32, device="cuda")
+        g = plan.graph(xd, yd, iterations=3, mode=0)
+        g.launch()
+        torch.cuda.synchronize()
+        g.close()
+        assert np.array_equal(yd.cpu().numpy(), ref)
