@@ -34,7 +34,7 @@ constexpr int kSellCapMin = 64;       // hybrid SELL: floor of the cap (prepare_
 constexpr int64_t kChunkCost = 4;     // SELL per-chunk overhead in slot-equivalents (warp ranges, hybrid cap)
 constexpr int64_t kSellMidMax = 1024; // hybrid rows up to this length: one warp each (sell_mid_kernel)
 #ifndef PEPP_SLIST_F64
-#define PEPP_SLIST_F64 0
+#define PEPP_SLIST_F64 1
 #endif
 constexpr bool kSlistF64 = PEPP_SLIST_F64;   // stencil list for fp64 plans too (sell_stencil_list)
 #ifndef PEPP_SLIST_CONCURRENT
@@ -653,10 +653,11 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
     const int nc = p->nchunks;
     if (p->d_perm || p->d_patlist || p->sell_stencil_chunks == 0 || nc <= 0) return PEPP_OK;
     if (const char* e = std::getenv("PEPP_NO_SLIST")) if (std::atoi(e)) return PEPP_OK;   // experiments only
-    // measured on config 4 (tools/gpu_slist2.sh, 3 alternating repeats): fp32
-    // 424 -> 361 µs (the issue-limited general walk loses its per-chunk
-    // instructions); fp64 584.0 -> 582.5 µs, i.e. nothing for a second launch,
-    // so the fp64 plans keep the one-kernel general walk (with paired chunks)
+    // measured on config 4 (3 alternating repeats each): fp32 424 -> 361 µs
+    // (the issue-limited general walk loses its per-chunk instructions,
+    // tools/gpu_slist2.sh), 349 µs with the genlist walk concurrent; fp64
+    // 593-596 -> 578.5 µs with the concurrent genlist walk (tools/gpu_slist5.sh;
+    // 582.5 with it sequential)
     if (p->vt == PEPP_VALUE_F64 && !kSlistF64) return PEPP_OK;
     const int64_t nsb = p->sell_slots / 32 + 8;
     std::vector<int> clen(nc), soff(nsb);
