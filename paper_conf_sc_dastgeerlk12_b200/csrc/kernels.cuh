@@ -300,7 +300,7 @@ __device__ __forceinline__ void sell_pair_len(int n, const T* __restrict__ val, 
 #endif
 
 #ifndef PEPP_SELL_PAIR_F64
-#define PEPP_SELL_PAIR_F64 1   // measured (tools/gpu_pair.sh): fp64 605 -> 587 us on config 4
+#define PEPP_SELL_PAIR_F64 0   // pairing helped the general walk on config 4 (605 -> 587 us) but costs 9-slot banded chunks 11 % (200 -> 223 us, tools/gpu_banded.sh); the stencil list now carries config 4
 #endif
 #ifndef PEPP_SELL_PAIR_F32
 #define PEPP_SELL_PAIR_F32 0   // fp32 420 -> 436 us: off
@@ -464,6 +464,7 @@ __device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int p
 // chunk only the value stream, the x gathers and the y store. The other
 // chunks go through sell_kernel over the plan's genlist.
 constexpr int kSellMaxStencils = 32;
+constexpr int kSellMaxStencilLen = 16;   // slots of a stencil-list chunk (9-point / banded b = 4 fit)
 #ifndef PEPP_SLIST_U_F64
 #define PEPP_SLIST_U_F64 8   // measured (tools/gpu_slist.sh): U = 2 / 4 / 8 -> 595 / 627 / 585 us, general walk 593
 #endif
@@ -474,7 +475,7 @@ template <typename T>
 constexpr int sell_slist_u() { return std::is_same<T, float>::value ? PEPP_SLIST_U_F32 : PEPP_SLIST_U_F64; }
 struct SellStencils {
     int len[kSellMaxStencils];
-    int off[kSellMaxStencils][kSellMaxPatternLen];
+    int off[kSellMaxStencils][kSellMaxStencilLen];
 };
 
 template <int U>
@@ -491,25 +492,37 @@ template <int U, int N, typename T>
 __device__ __forceinline__ void sell_slist_chunks(const int (&o)[N], const int2 (&q)[U], int lane,
                                                   const T* __restrict__ val, const T* __restrict__ x,
                                                   T* __restrict__ y, uint64_t pol) {
-    T v[U][N], xv[U][N];
+    // at most ~40 values + gathers in flight per lane: long stencils take the
+    // group in sub-groups of H chunks
+    constexpr int H = U * N > 40 ? (40 / N > 0 ? 40 / N : 1) : U;
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-        const int64_t base = (int64_t)q[u].y * 32 + lane;
+    for (int u0 = 0; u0 < U; u0 += H) {
+        T v[H][N], xv[H][N];
 #pragma unroll
-        for (int j = 0; j < N; ++j) v[u][j] = q[u].x >= 0 ? ld_stream_v(val + base + (int64_t)j * 32, pol) : T(0);
-    }
+        for (int h = 0; h < H; ++h) {
+            const int u = u0 + h < U ? u0 + h : U - 1;
+            const bool ok = u0 + h < U && q[u].x >= 0;
+            const int64_t base = (int64_t)q[u].y * 32 + lane;
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-        const int r = (q[u].x & ((1 << 26) - 1)) * 32 + lane;
+            for (int j = 0; j < N; ++j) v[h][j] = ok ? ld_stream_v(val + base + (int64_t)j * 32, pol) : T(0);
+        }
 #pragma unroll
-        for (int j = 0; j < N; ++j) xv[u][j] = q[u].x >= 0 ? ld_x(x, r + o[j]) : T(0);
-    }
+        for (int h = 0; h < H; ++h) {
+            const int u = u0 + h < U ? u0 + h : U - 1;
+            const bool ok = u0 + h < U && q[u].x >= 0;
+            const int r = (q[u].x & ((1 << 26) - 1)) * 32 + lane;
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-        T acc = T(0);
+            for (int j = 0; j < N; ++j) xv[h][j] = ok ? ld_x(x, r + o[j]) : T(0);
+        }
 #pragma unroll
-        for (int j = 0; j < N; ++j) acc = fma(v[u][j], xv[u][j], acc);   // slot order = the row's CSR order
-        if (q[u].x >= 0) y[(q[u].x & ((1 << 26) - 1)) * 32 + lane] = acc;
+        for (int h = 0; h < H; ++h) {
+            const int u = u0 + h < U ? u0 + h : U - 1;
+            const bool ok = u0 + h < U && q[u].x >= 0;
+            T acc = T(0);
+#pragma unroll
+            for (int j = 0; j < N; ++j) acc = fma(v[h][j], xv[h][j], acc);   // slot order = the row's CSR order
+            if (ok) y[(q[u].x & ((1 << 26) - 1)) * 32 + lane] = acc;
+        }
     }
 }
 
@@ -550,7 +563,51 @@ __device__ __forceinline__ void sell_slist_one(const SellStencils& st, int2 e, i
     sell_slist_chunks<U, N, T>(o, q, lane, val, x, y, pol);
 }
 
-template <int BLOCK, int U, typename T>
+// NMAX: the longest offset set the plan's table holds (8 or 16): plans with
+// short stencils get the instance whose registers are sized for them
+template <int U, int NMAX, typename T>
+__device__ __forceinline__ int sell_slist_dispatch_run(int len, const SellStencils& st, int pid,
+                                                       const int2* __restrict__ list, int n, int k0, int stride,
+                                                       int2 (&e)[U], int lane, const T* __restrict__ val,
+                                                       const T* __restrict__ x, T* __restrict__ y, uint64_t pol) {
+#define PEPP_SLR(N) case N: return sell_slist_run<U, N, T>(st, pid, list, n, k0, stride, e, lane, val, x, y, pol);
+    switch (len) {
+    PEPP_SLR(1) PEPP_SLR(2) PEPP_SLR(3) PEPP_SLR(4) PEPP_SLR(5) PEPP_SLR(6) PEPP_SLR(7)
+    default: break;
+    }
+    if constexpr (NMAX > 8) {
+        switch (len) {
+        PEPP_SLR(8) PEPP_SLR(9) PEPP_SLR(10) PEPP_SLR(11) PEPP_SLR(12) PEPP_SLR(13) PEPP_SLR(14) PEPP_SLR(15)
+        default: break;
+        }
+        return sell_slist_run<U, 16, T>(st, pid, list, n, k0, stride, e, lane, val, x, y, pol);
+    }
+    return sell_slist_run<U, 8, T>(st, pid, list, n, k0, stride, e, lane, val, x, y, pol);
+#undef PEPP_SLR
+}
+
+template <int U, int NMAX, typename T>
+__device__ __forceinline__ void sell_slist_dispatch_one(int len, const SellStencils& st, int2 e, int lane,
+                                                        const T* __restrict__ val, const T* __restrict__ x,
+                                                        T* __restrict__ y, uint64_t pol) {
+#define PEPP_SLO(N) case N: sell_slist_one<U, N, T>(st, e, lane, val, x, y, pol); return;
+    switch (len) {
+    PEPP_SLO(1) PEPP_SLO(2) PEPP_SLO(3) PEPP_SLO(4) PEPP_SLO(5) PEPP_SLO(6) PEPP_SLO(7)
+    default: break;
+    }
+    if constexpr (NMAX > 8) {
+        switch (len) {
+        PEPP_SLO(8) PEPP_SLO(9) PEPP_SLO(10) PEPP_SLO(11) PEPP_SLO(12) PEPP_SLO(13) PEPP_SLO(14) PEPP_SLO(15)
+        default: break;
+        }
+        sell_slist_one<U, 16, T>(st, e, lane, val, x, y, pol);
+        return;
+    }
+    sell_slist_one<U, 8, T>(st, e, lane, val, x, y, pol);
+#undef PEPP_SLO
+}
+
+template <int BLOCK, int U, int NMAX, typename T>
 __global__ void __launch_bounds__(BLOCK) sell_slist_kernel(const int2* __restrict__ list, int n,
                                                            const __grid_constant__ SellStencils st,
                                                            const T* __restrict__ val, const T* __restrict__ x,
@@ -564,30 +621,10 @@ __global__ void __launch_bounds__(BLOCK) sell_slist_kernel(const int2* __restric
     sell_slist_ids<U>(list, n, k0, nwarps, e);
     while (k0 < n) {
         const int pid = e[0].x >> 26;
-        switch (st.len[pid]) {
-        case 1: k0 = sell_slist_run<U, 1, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
-        case 2: k0 = sell_slist_run<U, 2, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
-        case 3: k0 = sell_slist_run<U, 3, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
-        case 4: k0 = sell_slist_run<U, 4, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
-        case 5: k0 = sell_slist_run<U, 5, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
-        case 6: k0 = sell_slist_run<U, 6, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
-        case 7: k0 = sell_slist_run<U, 7, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
-        default: k0 = sell_slist_run<U, 8, T>(st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol); break;
-        }
+        k0 = sell_slist_dispatch_run<U, NMAX, T>(st.len[pid], st, pid, list, n, k0, nwarps, e, lane, val, x, y, pol);
         if (k0 >= n) break;
-        for (int u = 0; u < U; ++u) {   // a group that straddles two patterns
-            if (e[u].x < 0) continue;
-            switch (st.len[e[u].x >> 26]) {
-            case 1: sell_slist_one<U, 1, T>(st, e[u], lane, val, x, y, pol); break;
-            case 2: sell_slist_one<U, 2, T>(st, e[u], lane, val, x, y, pol); break;
-            case 3: sell_slist_one<U, 3, T>(st, e[u], lane, val, x, y, pol); break;
-            case 4: sell_slist_one<U, 4, T>(st, e[u], lane, val, x, y, pol); break;
-            case 5: sell_slist_one<U, 5, T>(st, e[u], lane, val, x, y, pol); break;
-            case 6: sell_slist_one<U, 6, T>(st, e[u], lane, val, x, y, pol); break;
-            case 7: sell_slist_one<U, 7, T>(st, e[u], lane, val, x, y, pol); break;
-            default: sell_slist_one<U, 8, T>(st, e[u], lane, val, x, y, pol); break;
-            }
-        }
+        for (int u = 0; u < U; ++u)   // a group that straddles two offset sets
+            if (e[u].x >= 0) sell_slist_dispatch_one<U, NMAX, T>(st.len[e[u].x >> 26], st, e[u], lane, val, x, y, pol);
         k0 += U * nwarps;
         sell_slist_ids<U>(list, n, k0, nwarps, e);
     }

@@ -116,6 +116,7 @@ struct pepp_spmv_plan_s {
     int npatc = 0, ngen = 0;
     int2* d_stlist = nullptr;        // σ = 1, values streamed: stencil-list entries (sell_slist_kernel)
     int nstc = 0, grid_slist = 0;
+    bool slist_long = false;                     // an offset set longer than 8: the 16-slot instance
     cudaStream_t gside = nullptr;                // the genlist walk's stream (concurrent with the list kernel)
     cudaEvent_t ev_gfork = nullptr, ev_gjoin = nullptr;
     pepp::k::SellStencils stab{};    // the distinct offset sets of the stencil list (kernel parameter)
@@ -645,7 +646,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
 }
 
 // Stencil list for σ = 1 plans whose stencil chunks stream their values (no
-// pattern table): unmasked stencil chunks of <= 8 slots, grouped by offset
+// pattern table): unmasked stencil chunks of <= 16 slots, grouped by offset
 // set (<= kSellMaxStencils sets; chunks of further sets stay general), for
 // sell_slist_kernel; every other chunk goes to the genlist for sell_kernel.
 pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
@@ -673,7 +674,7 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
     for (int c = 0; c < nc; ++c) {
         const int d = clen[c], len = d & kSellLenMask;
         int pid = -1;
-        if ((d & pepp::k::kSellStencil) && !(d & pepp::k::kSellMasked) && len >= 1 && len <= pepp::k::kSellMaxPatternLen &&
+        if ((d & pepp::k::kSellStencil) && !(d & pepp::k::kSellMasked) && len >= 1 && len <= pepp::k::kSellMaxStencilLen &&
             c < (1 << 26) && (cp[c] >> 5) <= INT32_MAX) {
             const int64_t sb = cp[c] >> 5;
             for (int q = 0; q < nset && pid < 0; ++q) {
@@ -690,7 +691,10 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
         if (pid >= 0) lst.push_back(make_int2(c | (pid << 26), (int)(cp[c] >> 5)));
         else gen.push_back(c);
     }
-    if (lst.empty()) return PEPP_OK;
+    // worth it only when the list carries most chunks: otherwise the genlist
+    // walk (the PAT instance, no pairing) would take the bulk (measured on
+    // banded b = 4, 9-slot chunks: 1833 -> 2065 µs at 10^8 rows)
+    if (lst.empty() || 2 * (int64_t)lst.size() < (int64_t)nc) return PEPP_OK;
     std::stable_sort(lst.begin(), lst.end(), [](const int2& a, const int2& b) { return (a.x >> 26) < (b.x >> 26); });
     pepp_status_t s;
     if ((s = dalloc(p, &p->d_stlist, (int64_t)lst.size()))) return s;
@@ -706,8 +710,15 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
         PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gjoin, cudaEventDisableTiming));
     }
     int occ = 0;
-    const void* fn = p->vt == PEPP_VALUE_F32 ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<float>(), float>
-                                             : (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<double>(), double>;
+    int lmax = 0;
+    for (int q = 0; q < nset; ++q) lmax = std::max(lmax, tab.len[q]);
+    p->slist_long = lmax > 8;
+    const bool lg = p->slist_long;
+    const void* fn = p->vt == PEPP_VALUE_F32
+        ? (lg ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<float>(), 16, float>
+              : (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<float>(), 8, float>)
+        : (lg ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<double>(), 16, double>
+              : (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<double>(), 8, double>);
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
     (void)cudaGetLastError();
     const int64_t need = ((int64_t)p->nstc + kBlock / 32 - 1) / (kBlock / 32);
@@ -907,8 +918,12 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
             if (p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
                              cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
                 return PEPP_E_CUDA;
-            pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), T><<<p->grid_slist, kBlock, 0, st>>>(p->d_stlist, p->nstc, p->stab,
-                                                                                   (const T*)p->d_sval, x, y);
+            if (p->slist_long)
+                pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), 16, T><<<p->grid_slist, kBlock, 0, st>>>(
+                    p->d_stlist, p->nstc, p->stab, (const T*)p->d_sval, x, y);
+            else
+                pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), 8, T><<<p->grid_slist, kBlock, 0, st>>>(
+                    p->d_stlist, p->nstc, p->stab, (const T*)p->d_sval, x, y);
             if (p->ngen > 0)   // the genlist walk of the PAT instance, with no pattern chunks (phase A empty)
                 pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, gs>>>(
                     (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
