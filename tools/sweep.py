@@ -4,7 +4,7 @@
 For banded (half-bandwidth 4) and uniform-random (16/row) square matrices
 with 10^4 ... 10^8 rows, build one plan, let the history-based selector
 calibrate through ordinary automatic calls, then compare its choice with an
-exhaustive per-candidate timing in the same process (median of several
+exhaustive per-candidate timing in the same process (mean of several
 calls, L2 flushed between calls). Also reports the cold pick: the first call
 of a fresh plan whose history file holds the previously swept matrices
 (nearest-context prior; the first matrix has none). One JSON line per matrix.
@@ -60,7 +60,8 @@ def main():
             plan = pepp.Plan.from_csr(A, history_path=hist_path)
             tplan = time.perf_counter() - t0
             del A
-            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.reps)]
+            reps = a.reps if R > 1_000_000 else 3 * a.reps   # short calls: more samples (cheap)
+            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
 
             def timed(force=None):
                 # calls issued back to back (no host sync in between): each L2
@@ -75,7 +76,10 @@ def main():
                     e1.record()
                 torch.cuda.synchronize()
                 ts = [e0.elapsed_time(e1) * 1e3 for e0, e1 in ev]
-                return statistics.median(ts), u
+                # the mean, as the selector's objective (reading A10): short
+                # calls time in ~2 µs steps, and a median of quantised samples
+                # cannot resolve candidates one step apart, a mean can
+                return statistics.fmean(ts), u
 
             # calibration through ordinary automatic calls (flush between calls);
             # the first call is the cold pick (predicted best from the prior)
