@@ -362,6 +362,9 @@ __device__ __forceinline__ T sell_pattern_slots(const SellPatterns<T>& pt, int p
 #define PEPP_PAT_U 4
 #endif
 constexpr int kPatU = PEPP_PAT_U;   // pattern chunks per warp iteration in phase A
+#ifndef PEPP_PAT_INFLIGHT
+#define PEPP_PAT_INFLIGHT 20   // x gathers in flight per lane in phase A (sub-groups beyond)
+#endif
 #ifndef PEPP_PAT_PREFETCH
 #define PEPP_PAT_PREFETCH 1   // L2 prefetch distance in groups (0 = off; 1 measured best: 265 -> 254 us on config 4)
 #endif
@@ -413,7 +416,7 @@ __device__ __forceinline__ int sell_pattern_run(const SellPatterns<T>& pt, int p
 #endif
         // at most ~20 gathers in flight per lane: long patterns take the
         // group in sub-groups of H chunks (keeps the kernel at 48 registers)
-        constexpr int H = N * kPatU > 20 ? (20 / N > 0 ? 20 / N : 1) : kPatU;
+        constexpr int H = N * kPatU > PEPP_PAT_INFLIGHT ? (PEPP_PAT_INFLIGHT / N > 0 ? PEPP_PAT_INFLIGHT / N : 1) : kPatU;
 #pragma unroll
         for (int u0 = 0; u0 < kPatU; u0 += H) {
             T xv[H][N];
