@@ -288,8 +288,8 @@ pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_choice_t* out);
       force->exchange when partitioned) select the implementation.
    used: optional; receives the choice that ran (launches = this library's
       kernels the call enqueued).
-   Some plans also use their own second stream inside a call (the hybrid-SELL
-   and stencil-list kernels' companions, the overlapped halo): it forks from
+   Some plans also use their own second stream inside a call (the genlist
+   walk beside the stencil-list kernel, the overlapped halo): it forks from
    `stream` after the caller's queued work and joins back before the call's
    last operation on `stream`, so completion of `stream` means y is written.
    Errors: PEPP_E_INVALID (NULL / aliasing / unknown forced variant or
