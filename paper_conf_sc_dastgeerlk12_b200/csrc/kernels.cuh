@@ -469,13 +469,18 @@ __device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int p
 constexpr int kSellMaxStencils = 32;
 constexpr int kSellMaxStencilLen = 16;   // slots of a stencil-list chunk (9-point / banded b = 4 fit)
 #ifndef PEPP_SLIST_U_F64
-#define PEPP_SLIST_U_F64 8   // measured (tools/gpu_slist.sh): U = 2 / 4 / 8 -> 595 / 627 / 585 us, general walk 593
+#define PEPP_SLIST_U_F64 12   // measured (tools/gpu_u64.sh, 2 repeats): U = 6 / 8 / 12 / 16 -> 565.6 / 573.4 / 562.5 / 567.6 us on config 4
 #endif
 #ifndef PEPP_SLIST_U_F32
 #define PEPP_SLIST_U_F32 4   // U = 2 / 4 / 8 -> 373 / 360 / 459 us, general walk 421
 #endif
-template <typename T>
-constexpr int sell_slist_u() { return std::is_same<T, float>::value ? PEPP_SLIST_U_F32 : PEPP_SLIST_U_F64; }
+#ifndef PEPP_SLIST_U_F64_LONG
+#define PEPP_SLIST_U_F64_LONG 8   // fp64, offset sets of 9-16 slots (banded / 9-point)
+#endif
+template <typename T, int NMAX = 8>
+constexpr int sell_slist_u() {
+    return std::is_same<T, float>::value ? PEPP_SLIST_U_F32 : (NMAX > 8 ? PEPP_SLIST_U_F64_LONG : PEPP_SLIST_U_F64);
+}
 struct SellStencils {
     int len[kSellMaxStencils];
     int off[kSellMaxStencils][kSellMaxStencilLen];

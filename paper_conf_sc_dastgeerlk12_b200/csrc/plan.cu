@@ -715,9 +715,9 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
     p->slist_long = lmax > 8;
     const bool lg = p->slist_long;
     const void* fn = p->vt == PEPP_VALUE_F32
-        ? (lg ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<float>(), 16, float>
+        ? (lg ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<float, 16>(), 16, float>
               : (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<float>(), 8, float>)
-        : (lg ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<double>(), 16, double>
+        : (lg ? (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<double, 16>(), 16, double>
               : (const void*)pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<double>(), 8, double>);
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kBlock, 0) != cudaSuccess || occ < 1) occ = 1;
     (void)cudaGetLastError();
@@ -919,7 +919,7 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                              cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
                 return PEPP_E_CUDA;
             if (p->slist_long)
-                pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), 16, T><<<p->grid_slist, kBlock, 0, st>>>(
+                pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T, 16>(), 16, T><<<p->grid_slist, kBlock, 0, st>>>(
                     p->d_stlist, p->nstc, p->stab, (const T*)p->d_sval, x, y);
             else
                 pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), 8, T><<<p->grid_slist, kBlock, 0, st>>>(
