@@ -469,10 +469,10 @@ __device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int p
 constexpr int kSellMaxStencils = 32;
 constexpr int kSellMaxStencilLen = 16;   // slots of a stencil-list chunk (9-point / banded b = 4 fit)
 #ifndef PEPP_SLIST_U_F64
-#define PEPP_SLIST_U_F64 12   // measured (tools/gpu_u64.sh, 2 repeats): U = 6 / 8 / 12 / 16 -> 565.6 / 573.4 / 562.5 / 567.6 us on config 4
+#define PEPP_SLIST_U_F64 12   // measured (tools/gpu_u64.sh, 2 repeats): U = 6 / 8 / 12 / 16 -> 565.6 / 573.4 / 562.5 / 567.6 us on config 4; tools/gpu_u_sweep2.sh: U = 10 / 12 / 14 -> 565.5-566.5 / 560.0-570.2 / 564.9 us
 #endif
 #ifndef PEPP_SLIST_U_F32
-#define PEPP_SLIST_U_F32 4   // U = 2 / 4 / 8 -> 373 / 360 / 459 us, general walk 421
+#define PEPP_SLIST_U_F32 5   // U = 2 / 4 / 8 -> 373 / 360 / 459 us, general walk 421; tools/gpu_u_sweep2.sh (2 repeats): U = 3 / 4 / 5 / 6 -> 360.5 / 350.2-350.4 / 340.6-340.7 / 345.7 (one 589 outlier) us
 #endif
 #ifndef PEPP_SLIST_U_F64_LONG
 #define PEPP_SLIST_U_F64_LONG 8   // fp64, offset sets of 9-16 slots (banded / 9-point)
