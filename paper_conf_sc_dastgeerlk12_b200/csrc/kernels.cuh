@@ -475,7 +475,7 @@ constexpr int kSellMaxStencilLen = 16;   // slots of a stencil-list chunk (9-poi
 #define PEPP_SLIST_U_F32 5   // U = 2 / 4 / 8 -> 373 / 360 / 459 us, general walk 421; tools/gpu_u_sweep2.sh (2 repeats): U = 3 / 4 / 5 / 6 -> 360.5 / 350.2-350.4 / 340.6-340.7 / 345.7 (one 589 outlier) us
 #endif
 #ifndef PEPP_SLIST_U_F64_LONG
-#define PEPP_SLIST_U_F64_LONG 8   // fp64, offset sets of 9-16 slots (banded / 9-point)
+#define PEPP_SLIST_U_F64_LONG 10   // fp64, offset sets of 9-16 slots (banded / 9-point); tools/gpu_ulong.sh (2 repeats, banded b = 4 at 10^8 rows): U = 6 / 8 / 10 / 12 -> 1404 / 1333-1334 / 1318.6 / 1325-1329 us
 #endif
 template <typename T, int NMAX = 8>
 constexpr int sell_slist_u() {

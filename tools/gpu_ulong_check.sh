@@ -1,0 +1,5 @@
+# U_LONG = 10 default: GPU suite, smoke, banded timing
+mkdir -p gpurun_out
+timeout 1200 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo pytest_rc=$?; tail -1 gpurun_out/pytest_gpu.log; grep "^FAILED" gpurun_out/pytest_gpu.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo smoke_rc=$?; tail -1 gpurun_out/smoke.log
+timeout 600 python tools/banded_ab.py --rows 1e7,1e8 2>&1 | grep banded | cut -c1-90
