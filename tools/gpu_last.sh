@@ -1,0 +1,4 @@
+# Last check of the committed build: default bench line
+mkdir -p gpurun_out
+timeout 900 python bench.py > gpurun_out/bench_default.log 2>&1; echo bench_rc=$?
+tail -1 gpurun_out/bench_default.log | python -c 'import sys,json; d=json.loads(sys.stdin.read()); print(d["value"], d["roofline"]["avg_launch_us"], d["e2e"]["value"], d["clocks"])'
