@@ -10,7 +10,11 @@ Every function is a thin ctypes call into ``oracle/oracle.c`` (plain C,
 one follows. Pins: ``tests/test_oracle_pins.py`` (dense brute force,
 permutation, diagonal, Laplacian closed forms, exact-sum bound, power-of-two
 scaling, partition brute force) — none of them re-calls this code to make its
-expected value.
+expected value. The tolerance and checker helpers (``bound``, ``bound_rows``,
+``bound_f32``, ``abs_rowsum``, ``iterate_bound``, ``within``, ``equal``) are
+pinned by ``tests/test_oracle_bound_pins.py`` against the hand-worked values
+of ``tests/golden/bounds_worked.txt`` and by sensitivity cases (a dropped
+term, or an error of 2x the bound, must be rejected).
 """
 from __future__ import annotations
 
@@ -187,6 +191,34 @@ def iterate_bound(A, zK: np.ndarray, K: int) -> np.ndarray:
     u = 2.0 ** -53
     g = w * u / (1 - w * u)
     return 2.0 * K * g * (1 + g) ** K * zK
+
+
+def within(y, ref, tol) -> np.ndarray:
+    """Per-element parity verdict (the checker every parity test applies).
+
+    Finite reference entries: ``|y - ref| <= tol`` (tol from ``bound`` /
+    ``bound_f32`` / ``iterate_bound``; an empty row has tol 0, so it must be
+    exactly 0). Non-finite reference entries (Inf/NaN in x reach the row
+    through a stored entry; IEEE-754 propagation is order-independent for a
+    row whose only non-finite terms are infinities of one sign or NaN):
+    ``y`` must be the same infinity, or NaN where ``ref`` is NaN. A NaN in
+    ``y`` against a finite ``ref`` always fails."""
+    y = np.asarray(y, dtype=np.float64)
+    ref = np.asarray(ref, dtype=np.float64)
+    tol = np.broadcast_to(np.asarray(tol, dtype=np.float64), ref.shape)
+    fin = np.isfinite(ref)
+    ok = np.zeros(ref.shape, dtype=bool)
+    with np.errstate(invalid="ignore"):
+        ok[fin] = np.abs(y[fin] - ref[fin]) <= tol[fin]
+    nf = ~fin
+    ok[nf] = (y[nf] == ref[nf]) | (np.isnan(y[nf]) & np.isnan(ref[nf]))
+    return ok
+
+
+def equal(y, ref) -> np.ndarray:
+    """Bit-exact verdict for integer-valued inputs (reading A7: +0 == -0),
+    with NaN equal to NaN (non-finite x)."""
+    return within(y, ref, 0.0)
 
 
 def partition_nnz(A, P: int) -> np.ndarray:
