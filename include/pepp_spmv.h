@@ -63,7 +63,7 @@
 extern "C" {
 #endif
 
-#define PEPP_ABI_VERSION 5
+#define PEPP_ABI_VERSION 6
 
 typedef enum {
     PEPP_OK = 0,
@@ -212,6 +212,13 @@ typedef struct {
     int32_t launches;         /* exec only: kernels of this library the call launched (SpMV kernels,
                                  fix-ups, halo pack/unpack or the fused push; NCCL's own not counted) */
     int32_t reserved;
+    int64_t layout_bytes;     /* bytes this candidate's kernels move from / to HBM per call with the plan's
+                                 layout as stored: matrix arrays as the variant streams them (values,
+                                 index stream or per-chunk stencil offsets, descriptors, lists, row
+                                 pointers), x read once (ncols) and y written once (nrows) — the
+                                 physical roofline numerator. SURVEY §8(d)'s algorithmic bytes
+                                 (nnz*12 + row_ptr + x + y) are pepp_plan_info_t.algorithmic_bytes:
+                                 a compressed layout streams fewer bytes than that for the same work. */
 } pepp_choice_t;
 
 /* Context instance (§III P@9781: "a tuple of concrete values for context
@@ -332,8 +339,14 @@ pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* y, int flags, void* 
    Rows of this block outside the ghosts a peer reads may also be written
    into that peer's buffer (with their correct values). Calls with any other
    y use the NCCL exchange. Boundary rows are summed in the oracle's order
-   (no FMA). Requires nranks > 1, the halo exchange and the head / interior /
-   tail split (pepp_plan_info_t.overlap == 1), else PEPP_E_UNSUPPORTED;
+   (no FMA). Readiness flows from each receiver to its senders and data from
+   senders to receivers, so the send and receive peer sets may differ
+   (nonsymmetric matrices). Requires nranks > 1, the halo exchange and, on
+   every rank that sends rows, the head / interior / tail split
+   (pepp_plan_info_t.overlap == 1; a rank that sends nothing computes its
+   whole block on `stream` and only signals). The ranks agree first (one
+   max-reduce): if any rank cannot take part, EVERY rank returns
+   PEPP_E_UNSUPPORTED and the plan stays usable with the NCCL halo.
    PEPP_E_STATE if already registered. A peer that stops calling makes the
    waiting kernel give up after 20 s and the plan's next call return
    PEPP_E_NCCL. Errors: PEPP_E_INVALID, PEPP_E_CUDA (IPC unavailable),
@@ -524,8 +537,16 @@ pepp_status_t pepp_history_save(const pepp_history* h, const char* path);
 pepp_status_t pepp_history_load(pepp_history* h, const char* path);
 
 /* Context key of a row-pointer array (host): bucketed (log2 rows, log2 nnz,
-   mean row length, CV, nparts) — the "context instance" used as history key. */
-uint64_t pepp_context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts);
+   mean row length, CV, nparts) plus the kernel instance — the "context
+   instance" used as history key (§III P@9781). `instance` is a bit set:
+   PEPP_KEY_F32 for an fp32 plan, PEPP_KEY_COMPRESS for a plan built with
+   opts.compress_values = 1 (both select different kernels, so their timings
+   must not be mixed with the fp64 / value-streaming plan's). A cold-start
+   prior (pepp_history_prior) is only taken from a key with the same rank
+   count and instance. */
+#define PEPP_KEY_F32      0x1
+#define PEPP_KEY_COMPRESS 0x2
+uint64_t pepp_context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts, int32_t instance);
 
 /* NCCL bootstrap helper: write a fresh 128-byte ncclUniqueId into id_out
    (NCCL is loaded on demand with dlopen; PEPP_E_NCCL if unavailable). */

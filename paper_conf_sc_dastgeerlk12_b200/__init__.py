@@ -41,6 +41,7 @@ class Choice:
     candidate: int = -1
     predicted_us: float = 0.0
     launches: int = 0
+    layout_bytes: int = 0
 
     @property
     def name(self) -> str:
@@ -49,7 +50,7 @@ class Choice:
     @staticmethod
     def _from(c: C.CHOICE_T) -> "Choice":
         return Choice(c.variant, c.param, c.exchange, c.nparts, bool(c.calibrating), c.candidate, c.predicted_us,
-                      c.launches)
+                      c.launches, c.layout_bytes)
 
     def _to(self) -> C.CHOICE_T:
         c = C.CHOICE_T()
@@ -487,8 +488,10 @@ def halo_ghosts(col: np.ndarray, nranks: int, rank: int, row_bounds: Sequence[in
     return counts, g[:total.value]
 
 
-def context_key(nrows: int, ncols: int, nnz: int, cv: float, nparts: int = 1) -> int:
-    return int(C.lib().pepp_context_key(nrows, ncols, nnz, cv, nparts))
+def context_key(nrows: int, ncols: int, nnz: int, cv: float, nparts: int = 1, *, f32: bool = False,
+                compress: bool = False) -> int:
+    inst = (C.KEY_F32 if f32 else 0) | (C.KEY_COMPRESS if compress else 0)
+    return int(C.lib().pepp_context_key(nrows, ncols, nnz, cv, nparts, inst))
 
 
 def nccl_unique_id() -> bytes:

@@ -18,6 +18,7 @@ Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, EXEC_NO_TIMING = 0x0, 0x1, 0x2, 0x10
 ACCESS_READ, ACCESS_WRITE, ACCESS_READWRITE = 1, 2, 3
 VALUE_F64, VALUE_F32 = 0, 1
 DEVICE_SIMULATED = -2
+KEY_F32, KEY_COMPRESS = 0x1, 0x2
 VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell", V_CSR_STREAM: "csr_stream"}
 EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_P2P: "p2p", X_AUTO: "auto"}
 
@@ -61,13 +62,13 @@ class OPTS_T(ctypes.Structure):
 class CHOICE_T(ctypes.Structure):
     _fields_ = [("variant", c_i32), ("param", c_i32), ("nparts", c_i32), ("exchange", c_i32),
                 ("calibrating", c_i32), ("candidate", c_i32), ("predicted_us", c_f64),
-                ("launches", c_i32), ("reserved", c_i32)]
+                ("launches", c_i32), ("reserved", c_i32), ("layout_bytes", c_i64)]
 
     def as_dict(self) -> dict:
         return {"variant": VARIANT_NAMES.get(self.variant, str(self.variant)), "variant_id": self.variant,
                 "param": self.param, "nparts": self.nparts, "exchange": EXCHANGE_NAMES.get(self.exchange, "?"),
                 "calibrating": bool(self.calibrating), "candidate": self.candidate,
-                "predicted_us": self.predicted_us, "launches": self.launches}
+                "predicted_us": self.predicted_us, "launches": self.launches, "layout_bytes": self.layout_bytes}
 
 
 # (name, restype, argtypes) for every entry point of include/pepp_spmv.h
@@ -108,7 +109,7 @@ SIGNATURES = {
     "pepp_history_prior": (c_i32, [c_vp, c_u64, c_i32, c_vp, c_vp, ctypes.POINTER(c_u64)]),
     "pepp_history_save": (c_i32, [c_vp, ctypes.c_char_p]),
     "pepp_history_load": (c_i32, [c_vp, ctypes.c_char_p]),
-    "pepp_context_key": (c_u64, [c_i64, c_i64, c_i64, c_f64, c_i32]),
+    "pepp_context_key": (c_u64, [c_i64, c_i64, c_i64, c_f64, c_i32, c_i32]),
     "pepp_nccl_unique_id": (c_i32, [c_vp]),
     "pepp_nccl_selftest": (c_i32, [c_i32]),
     "pepp_abi_version": (c_i32, []),
@@ -130,7 +131,7 @@ class PeppError(RuntimeError):
         super().__init__(f"{where}: {status_str(status)} ({status})" + (f": {detail}" if detail else ""))
 
 
-ABI_VERSION = 5   # PEPP_ABI_VERSION of include/pepp_spmv.h
+ABI_VERSION = 6   # PEPP_ABI_VERSION of include/pepp_spmv.h
 
 
 def lib() -> ctypes.CDLL:

@@ -218,7 +218,7 @@ bool history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t
                    uint64_t* from_key) {
     auto field = [](uint64_t k, int shift, uint64_t mask) { return (int64_t)((k >> shift) & mask); };
     auto dist = [&](uint64_t a, uint64_t b) -> int64_t {
-        if ((a >> 27) != (b >> 27)) return -1;   // ranks + tag must match
+        if ((a >> 27) != (b >> 27)) return -1;   // ranks + instance + tag must match
         return std::llabs(field(a, 0, 0x7f) - field(b, 0, 0x7f)) + std::llabs(field(a, 7, 0x7f) - field(b, 7, 0x7f)) +
                std::llabs(field(a, 14, 0x7f) - field(b, 14, 0x7f)) + std::llabs(field(a, 21, 0x3f) - field(b, 21, 0x3f));
     };
@@ -243,7 +243,7 @@ bool history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t
     return true;
 }
 
-uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts) {
+uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts, int32_t instance) {
     // bucketed context instance: half-octave buckets of rows / cols / nnz,
     // quarter buckets of the row-length CV (capped), and the partition count.
     auto hb = [](int64_t v) -> uint64_t { return (uint64_t)std::floor(2.0 * std::log2((double)v + 1.0)); };
@@ -254,7 +254,8 @@ uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32
     k |= (hb(nnz) & 0x7f) << 14;
     k |= (cvb & 0x3f) << 21;
     k |= ((uint64_t)nparts & 0xffff) << 27;
-    k |= (uint64_t)0x5EBBu << 48;   // tag: fp64 CSR SpMV
+    k |= ((uint64_t)instance & 0x1f) << 43;   // kernel instance: value type, value compression
+    k |= (uint64_t)0x5EBBu << 48;   // tag: CSR SpMV
     return k;
 }
 
@@ -338,6 +339,7 @@ extern "C" PEPP_API pepp_status_t pepp_history_load(pepp_history* h, const char*
     return PEPP_OK;
 }
 
-extern "C" PEPP_API uint64_t pepp_context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts) {
-    return pepp::context_key(nrows, ncols, nnz, cv, nparts);
+extern "C" PEPP_API uint64_t pepp_context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts,
+                                              int32_t instance) {
+    return pepp::context_key(nrows, ncols, nnz, cv, nparts, instance);
 }

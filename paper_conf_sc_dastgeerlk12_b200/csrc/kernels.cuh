@@ -1555,20 +1555,29 @@ __global__ void scatter_kernel(int64_t n, const int* __restrict__ idx, const T* 
 // head/tail SpMV kernels + NCCL send/recv + pack/unpack of the in-order path.
 //
 // Protocol (per plan, `epoch` e = number of P2P calls so far, device
-// resident so CUDA graphs replay it correctly). Flags live in the receiver's
-// signal block, one slot per sender:
-//   ready[q]  = e+1 : rank q began call e, so everything q's streams did
-//                   before (calls < e, which read q's buffers — e.g. the
-//                   previous x — and the caller's own writes, e.g. filling
-//                   x_0) is complete: q's y of call e may now be written;
-//   arrive[q] = e+1 : rank q's rows of call e have landed in this rank's y.
-// Call e on rank r: every CTA writes ready = e+1 into each send-peer's block
-// (idempotent; no CTA waits for another CTA of the grid), waits for the
-// send-peers' ready >= e+1, computes its rows and pushes them; the last CTA
-// (grid-wide counter) fences, writes arrive = e+1 into each send-peer's
-// block, waits for arrive >= e+1 from every receive-peer, resets the counter
-// and bumps the epoch. Kernel completion therefore means exactly what the
-// NCCL halo's stream completion means: own rows and every ghost are in y.
+// resident so CUDA graphs replay it correctly). Each rank's signal block
+// holds ready[P] and arrive[P], one slot per peer:
+//   my.ready[q]  = e+1 : rank q (which RECEIVES from me) began call e, so
+//                        everything q's streams did before (calls < e, which
+//                        read q's buffers — e.g. the previous x — and the
+//                        caller's own writes, e.g. filling x_0) is complete:
+//                        I may now write into q's y of call e;
+//   my.arrive[q] = e+1 : rank q (which SENDS to me) has landed its rows of
+//                        call e in my y.
+// Readiness flows from receiver to sender and data + arrival from sender to
+// receiver, so the send and receive peer sets need not match (nonsymmetric
+// matrices: upwind stencils, one-sided bands). Call e on rank r: every CTA
+// writes ready = e+1 into the block of each rank r receives from
+// (idempotent; no CTA waits for another CTA of the grid), waits for
+// my.ready[q] >= e+1 from every rank q r sends to, computes its rows and
+// pushes them; the last CTA (grid-wide counter) fences, writes arrive = e+1
+// into each send-peer's block, waits for my.arrive[q] >= e+1 from every
+// receive-peer, resets the counter and bumps the epoch. Kernel completion
+// therefore means exactly what the NCCL halo's stream completion means: own
+// rows and every ghost are in y. Deadlock freedom: call e waits only for
+// the peers' call e (ready: published first thing; arrive: published after
+// their own ready waits, which depend only on call e starting everywhere),
+// and call e starts after call e-1 completed — by induction on e, no cycle.
 // Every wait is bounded (%globaltimer, timeout_ns: 20 s, PEPP_P2P_TIMEOUT_MS): a peer that never
 // arrives sets *err (host-mapped) instead of hanging the GPU.
 //
@@ -1587,11 +1596,11 @@ struct P2PArgs {
     int64_t push_lo[kP2PMaxPush], push_hi[kP2PMaxPush];
     T* push_dst[kP2PMaxPush];          // the peer's buffer (global indexing)
     int nsend;                         // peers this rank writes to
-    unsigned long long* peer_ready[kP2PMaxPeers];    // &peer.ready[me]
-    unsigned long long* peer_arrive[kP2PMaxPeers];   // &peer.arrive[me]
-    unsigned long long* my_ready[kP2PMaxPeers];      // &my.ready[send peer]
+    unsigned long long* ready_in[kP2PMaxPeers];      // &my.ready[send peer]       (waited on)
+    unsigned long long* arrive_out[kP2PMaxPeers];    // &send_peer.arrive[me]      (published)
     int nrecv;                         // peers this rank receives from
-    unsigned long long* my_arrive[kP2PMaxPeers];     // &my.arrive[recv peer]
+    unsigned long long* ready_out[kP2PMaxPeers];     // &recv_peer.ready[me]       (published)
+    unsigned long long* arrive_in[kP2PMaxPeers];     // &my.arrive[recv peer]      (waited on)
     unsigned long long* epoch;         // my signal block
     unsigned int* done;                // my signal block: CTAs finished this call
     int* err;                          // host-mapped error flag
@@ -1636,9 +1645,9 @@ __global__ void __launch_bounds__(256) halo_push_kernel(const int* __restrict__ 
     if (threadIdx.x == 0) {
         const unsigned long long e = *(volatile unsigned long long*)a.epoch;
         s_epoch = e;
-        for (int j = 0; j < a.nsend; ++j) st_release_sys(a.peer_ready[j], e + 1);
+        for (int j = 0; j < a.nrecv; ++j) st_release_sys(a.ready_out[j], e + 1);
         bool ok = true;
-        for (int j = 0; j < a.nsend; ++j) ok &= wait_geq(a.my_ready[j], e + 1, t0, a.timeout_ns);
+        for (int j = 0; j < a.nsend; ++j) ok &= wait_geq(a.ready_in[j], e + 1, t0, a.timeout_ns);
         if (!ok) atomicExch(a.err, 1);
     }
     __syncthreads();
@@ -1660,9 +1669,9 @@ __global__ void __launch_bounds__(256) halo_push_kernel(const int* __restrict__ 
     if (!s_last || threadIdx.x != 0) return;
     __threadfence_system();
     const unsigned long long e = s_epoch;
-    for (int j = 0; j < a.nsend; ++j) st_release_sys(a.peer_arrive[j], e + 1);
+    for (int j = 0; j < a.nsend; ++j) st_release_sys(a.arrive_out[j], e + 1);
     bool ok = true;
-    for (int j = 0; j < a.nrecv; ++j) ok &= wait_geq(a.my_arrive[j], e + 1, global_ns(), a.timeout_ns);
+    for (int j = 0; j < a.nrecv; ++j) ok &= wait_geq(a.arrive_in[j], e + 1, global_ns(), a.timeout_ns);
     if (!ok) atomicExch(a.err, 1);
     *a.done = 0u;
     *(volatile unsigned long long*)a.epoch = e + 1;

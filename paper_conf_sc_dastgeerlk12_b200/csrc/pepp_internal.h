@@ -8,6 +8,19 @@
 
 #define PEPP_API __attribute__((visibility("default")))
 
+// NVTX ranges around plan / exec / exchange / host calls (header-only NVTX3:
+// a no-op unless a profiler injects itself, e.g. ncu --nvtx or nsys)
+#include <nvtx3/nvToolsExt.h>
+namespace pepp {
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
+}  // namespace pepp
+#define PEPP_NVTX(name) ::pepp::NvtxRange pepp_nvtx_range_(name)
+
 namespace pepp {
 
 struct Welford {
@@ -31,7 +44,7 @@ constexpr int32_t kRefineRounds = 3;
 bool history_contender(const Welford* w, double best_mean);
 int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible,
                      int32_t min_samples, int32_t* calibrating, double* predicted_us);
-uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts);
+uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts, int32_t instance);
 bool history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t* ids, double* prior,
                    uint64_t* from_key);
 void halo_ghost_list(const int32_t* col, int64_t nnz, int64_t lo, int64_t hi, std::vector<int32_t>& out);

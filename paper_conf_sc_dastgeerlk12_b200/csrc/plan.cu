@@ -31,7 +31,10 @@ using pepp::ncclComm_t;
 
 constexpr int kBlock = 256;
 constexpr int kSellCapMin = 64;       // hybrid SELL: floor of the cap (prepare_sell_long)
-constexpr int64_t kChunkCost = 4;     // SELL per-chunk overhead in slot-equivalents (warp ranges, hybrid cap)
+#ifndef PEPP_EXP_CHUNK_COST   // experiments only: build-time override (PEPP_NVCC_EXTRA=-DPEPP_EXP_CHUNK_COST=n)
+#define PEPP_EXP_CHUNK_COST 4
+#endif
+constexpr int64_t kChunkCost = PEPP_EXP_CHUNK_COST;   // SELL per-chunk overhead in slot-equivalents (warp ranges, hybrid cap)
 constexpr int64_t kSellMidMax = 1024; // hybrid rows up to this length: one warp each (sell_mid_kernel)
 #ifndef PEPP_SLIST_F64
 #define PEPP_SLIST_F64 1
@@ -135,6 +138,8 @@ struct pepp_spmv_plan_s {
     unsigned int* d_sell_cnt = nullptr;
     int nsell_mid = 0;
     int* d_sell_mid = nullptr;       // rows of cap < length <= kSellLongSeg: sell_mid_kernel, warp per row
+    int64_t sell_long_nnz = 0;       // entries of the rows the mid / long-row kernels sum
+    int64_t sell_bytes = 0;          // DRAM bytes one SELL call streams with this layout (layout_bytes)
     void* d_sell_part = nullptr;     // segment partials (8-byte slots)
 
     // merge path
@@ -175,6 +180,7 @@ struct pepp_spmv_plan_s {
     int ring_count = 0;
     std::vector<int32_t> pending;   // timed calls in flight per candidate
     std::vector<int32_t> uids;      // stable candidate identity in the history: variant << 20 | param
+    std::vector<int64_t> cand_bytes;// per candidate: bytes its kernels move per call (layout as stored + x + y)
     std::vector<double> prior;      // cold-start means from the nearest recorded context (-1 = none)
     std::vector<int32_t> order;     // calibration order (predicted best first)
     std::vector<double> predicted;  // opts.predict per candidate (-1 = none)
@@ -212,10 +218,10 @@ struct pepp_spmv_plan_s {
     int64_t p2p_push_lo[pepp::k::kP2PMaxPush] = {}, p2p_push_hi[pepp::k::kP2PMaxPush] = {};
     void* p2p_push_dst[kP2PMaxBuf][pepp::k::kP2PMaxPush] = {};
     int p2p_nsend = 0, p2p_nrecv = 0;
-    unsigned long long* p2p_peer_ready[pepp::k::kP2PMaxPeers] = {};
-    unsigned long long* p2p_peer_arrive[pepp::k::kP2PMaxPeers] = {};
-    unsigned long long* p2p_my_ready[pepp::k::kP2PMaxPeers] = {};
-    unsigned long long* p2p_my_arrive[pepp::k::kP2PMaxPeers] = {};
+    unsigned long long* p2p_ready_in[pepp::k::kP2PMaxPeers] = {};    // per send peer
+    unsigned long long* p2p_arrive_out[pepp::k::kP2PMaxPeers] = {};  // per send peer
+    unsigned long long* p2p_ready_out[pepp::k::kP2PMaxPeers] = {};   // per receive peer
+    unsigned long long* p2p_arrive_in[pepp::k::kP2PMaxPeers] = {};   // per receive peer
     int p2p_grid = 1;
     unsigned long long p2p_timeout_ns = 20ull * 1000 * 1000 * 1000;
 
@@ -345,8 +351,7 @@ pepp_status_t sell_warp_ranges(pepp_spmv_plan_t* p) {
     if (nc > 0) PEPP_CUDA_TRY(cudaMemcpy(len.data(), p->d_chunk_len, sizeof(int) * nc, cudaMemcpyDeviceToHost));
     const int nwin = nc / cpw, nfull = nwin * cpw;
     auto chunk_of = [&](int i) { return i < nfull ? (i % nwin) * cpw + i / nwin : i; };
-    int64_t kChunkOverhead = kChunkCost;   // descriptor + per-lane loads + y store, in slot-equivalents
-    if (const char* e = std::getenv("PEPP_SELL_CHUNK_COST")) kChunkOverhead = std::atoi(e);   // experiments only
+    const int64_t kChunkOverhead = kChunkCost;   // descriptor + per-lane loads + y store, in slot-equivalents
     int64_t total = 0;
     for (int i = 0; i < nc; ++i) total += (len[chunk_of(i)] & pepp::k::kSellLenMask) + kChunkOverhead;
     std::vector<int> ws(W + 1, nc);
@@ -460,7 +465,9 @@ pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
         const int64_t rel = (int64_t)std::ceil(8.0 * p->info.mean_row);
         cap = std::max<int64_t>(cap, std::min(share, rel));
     }
-    if (const char* e = std::getenv("PEPP_SELL_CAP")) cap = std::max(1, std::atoi(e));   // experiments only
+#ifdef PEPP_EXP_SELL_CAP   // experiments only: a fixed cap, set at build time (PEPP_NVCC_EXTRA=-DPEPP_EXP_SELL_CAP=n)
+    cap = std::max(1, PEPP_EXP_SELL_CAP);
+#endif
     p->sell_cap = (int)std::min<int64_t>(cap, INT32_MAX);
     if (p->info.max_row <= cap) return PEPP_OK;
     const int64_t n = p->nrows;
@@ -469,8 +476,7 @@ pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
     std::vector<int4> seg;
     std::vector<int2> lrow;
     std::vector<int> mid;
-    int64_t mid_max = kSellMidMax;
-    if (const char* e = std::getenv("PEPP_SELL_MIDMAX")) mid_max = std::atoi(e);   // experiments only
+    const int64_t mid_max = kSellMidMax;
     for (int64_t r = 0; r < n; ++r) {
         const int b = rp[r], e = rp[r + 1];
         if (e - b <= cap) continue;
@@ -503,6 +509,51 @@ pepp_status_t prepare_sell_long(pepp_spmv_plan_t* p, int64_t* nnz_long) {
 
 pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p);
 
+// Bytes one SELL call moves from / to HBM with the layout as stored — the
+// physical roofline numerator (bench.py `roofline`): per chunk of the
+// general walk its descriptor (chunk_ptr 8 B + chunk_len 4 B, + a 4 B list
+// entry when walked through a list), its values (slots x value size, none
+// for a pattern-table chunk), its index stream (stencil: one 4 B offset per
+// slot for the whole chunk; 16-bit deltas: 2 B per slot; else 4 B per slot),
+// row lengths of masked chunks (4 B per row) and the permutation (4 B per
+// row, σ > 1); stencil-list chunks: values + one 8 B list entry; hybrid rows
+// (mid / long kernels): their CSR entries (value + 4 B column), 2 row
+// pointers and a 4 B row id or a 16 B segment + 2 x 8 B partial; plus x
+// read once (ncols) and y written once (nrows). Padding slots count: they
+// are streamed.
+pepp_status_t sell_layout_bytes(pepp_spmv_plan_t* p) {
+    using pepp::k::kSellLenMask;
+    const int nc = p->nchunks;
+    const int64_t es = (int64_t)p->esz;
+    std::vector<int> clen(nc);
+    if (nc) PEPP_CUDA_TRY(cudaMemcpy(clen.data(), p->d_chunk_len, sizeof(int) * nc, cudaMemcpyDeviceToHost));
+    std::vector<uint8_t> in_list(nc, 0);
+    if (p->d_stlist && p->nstc) {
+        std::vector<int2> l(p->nstc);
+        PEPP_CUDA_TRY(cudaMemcpy(l.data(), p->d_stlist, sizeof(int2) * p->nstc, cudaMemcpyDeviceToHost));
+        for (const int2& e : l) in_list[e.x & ((1 << 26) - 1)] = 1;
+    }
+    const bool lists = p->d_genlist != nullptr;   // general chunks reached through a 4 B list entry
+    int64_t b = 0;
+    for (int c = 0; c < nc; ++c) {
+        const int d = clen[c];
+        const int64_t len = d & kSellLenMask, slots = 32 * len;
+        if (in_list[c]) { b += slots * es + 8; continue; }
+        if (d & pepp::k::kSellPattern) { b += 4; continue; }   // patlist entry; offsets and values are kernel parameters
+        b += 12 + (lists ? 4 : 0) + slots * es;
+        if (d & pepp::k::kSellStencil) b += 4 * len;
+        else if (d & pepp::k::kSellCol16) b += 2 * slots;
+        else b += 4 * slots;
+        if (d & pepp::k::kSellMasked) b += 4 * 32;
+    }
+    if (p->d_perm) b += 4 * p->nrows;
+    b += p->sell_long_nnz * (es + 4) + (int64_t)p->nsell_mid * (4 + 8) + (int64_t)p->nsell_long * 8 +
+         (int64_t)p->nsell_seg * (16 + 16);
+    b += p->ncols * es + p->nrows * es;
+    p->sell_bytes = b;
+    return PEPP_OK;
+}
+
 pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     const int n = (int)p->nrows;
     p->nchunks = (n + 31) / 32;
@@ -514,6 +565,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     const int tb = 256, gb = (n + tb - 1) / tb;
     int64_t nnz_long = 0;
     if ((s = prepare_sell_long(p, &nnz_long))) return s;
+    p->sell_long_nnz = nnz_long;
     const int cap = p->sell_cap;
 
     auto fill_ratio = [&](const int* perm, double* fill) -> pepp_status_t {
@@ -634,6 +686,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     }
     PEPP_CUDA_TRY(cudaStreamSynchronize(st));
     if ((s = sell_stencil_list(p))) return s;
+    if ((s = sell_layout_bytes(p))) return s;
     p->sell_cpw = sigma > 1 ? std::max(1, sigma / 32) : 1;
     p->info.sell_sigma = sigma;
     p->info.sell_col16_frac = p->nchunks ? (double)p->sell_col16_chunks / (double)p->nchunks : 0.0;
@@ -653,7 +706,6 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
     using pepp::k::kSellLenMask;
     const int nc = p->nchunks;
     if (p->d_perm || p->d_patlist || p->sell_stencil_chunks == 0 || nc <= 0) return PEPP_OK;
-    if (const char* e = std::getenv("PEPP_NO_SLIST")) if (std::atoi(e)) return PEPP_OK;   // experiments only
     // measured on config 4 (3 alternating repeats each): fp32 424 -> 361 µs
     // (the issue-limited general walk loses its per-chunk instructions,
     // tools/gpu_slist2.sh), 349 µs with the genlist walk concurrent; fp64
@@ -1031,6 +1083,7 @@ void fill_choice(const pepp_spmv_plan_t* p, int cand, int calibrating, double pr
     out->calibrating = calibrating;
     out->candidate = cand;
     out->predicted_us = pred;
+    out->layout_bytes = p->cand_bytes[cand];
 }
 
 // frozen: the call is being captured into a CUDA graph — no event queries (a
@@ -1138,6 +1191,7 @@ pepp_status_t nccl_ok(const pepp_spmv_plan_t* p, int r) { (void)p; return r == 0
 int nccl_value_type(const pepp_spmv_plan_t* p) { return p->vt == PEPP_VALUE_F32 ? pepp::NCCL_FLOAT32 : pepp::NCCL_FLOAT64; }
 
 pepp_status_t exchange_allgather(pepp_spmv_plan_t* p, void* y, cudaStream_t st) {
+    PEPP_NVTX("pepp exchange allgatherv");
     const Nccl* n = p->nccl;
     char* yb = (char*)y;
     if (nccl_ok(p, n->GroupStart())) return PEPP_E_NCCL;
@@ -1161,6 +1215,7 @@ void pack_unpack(pepp_spmv_plan_t* p, T* y, bool pack, cudaStream_t st) {
 }
 
 pepp_status_t exchange_halo(pepp_spmv_plan_t* p, void* y, cudaStream_t st) {
+    PEPP_NVTX("pepp exchange halo");
     const Nccl* n = p->nccl;
     char* yb = (char*)y;
     const int64_t es = (int64_t)p->esz;
@@ -1367,6 +1422,13 @@ pepp_status_t nccl_barrier(pepp_spmv_plan_t* p, cudaStream_t st) {
 pepp_status_t p2p_export(pepp_spmv_plan_t* p, int nbuf, cudaStream_t st, P2PHandles* mine) {
     const int P = p->opts.nranks;
     pepp_status_t s;
+    if (!p->side) {   // a rank without a head / tail split (it sends nothing) still forks a side stream
+        int lo = 0, hi = 0;
+        PEPP_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        PEPP_CUDA_TRY(cudaStreamCreateWithPriority(&p->side, cudaStreamNonBlocking, hi));
+        PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming));
+        PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_join, cudaEventDisableTiming));
+    }
     // symmetric buffers + signal block (zeroed before any peer can see them)
     for (int b = 0; b < nbuf; ++b) {
         if ((s = dalloc_bytes(p, &p->p2p_buf[b], p->global_rows * (int64_t)p->esz))) return s;
@@ -1384,7 +1446,7 @@ pepp_status_t p2p_export(pepp_spmv_plan_t* p, int nbuf, cudaStream_t st, P2PHand
     return PEPP_OK;
 }
 
-// map the send-peers' buffers and signal blocks; build the push ranges
+// map the send-peers' buffers and the signal blocks of send and receive peers; build the push ranges
 pepp_status_t p2p_import(pepp_spmv_plan_t* p, int nbuf, const std::vector<P2PHandles>& all) {
     const int P = p->opts.nranks, me = p->opts.rank;
     std::vector<int> sendp, recvp;   // peers this rank writes to (its send list) / receives from
@@ -1396,6 +1458,16 @@ pepp_status_t p2p_import(pepp_spmv_plan_t* p, int nbuf, const std::vector<P2PHan
     recvp.erase(std::unique(recvp.begin(), recvp.end()), recvp.end());
     if ((int)sendp.size() > pepp::k::kP2PMaxPeers || (int)recvp.size() > pepp::k::kP2PMaxPeers) return PEPP_E_UNSUPPORTED;
     std::vector<std::vector<void*>> peer_buf(P);
+    std::vector<unsigned long long*> peer_sig(P, nullptr);   // mapped signal blocks (send and receive peers)
+    auto open_sig = [&](int q) -> pepp_status_t {
+        if (peer_sig[q]) return PEPP_OK;
+        void* sig = nullptr;
+        PEPP_CUDA_TRY(cudaIpcOpenMemHandle(&sig, all[q].sig, cudaIpcMemLazyEnablePeerAccess));
+        p->p2p_opened.push_back(sig);
+        peer_sig[q] = (unsigned long long*)sig;
+        return PEPP_OK;
+    };
+    pepp_status_t s;
     for (size_t j = 0; j < sendp.size(); ++j) {
         const int q = sendp[j];
         peer_buf[q].assign(nbuf, nullptr);
@@ -1403,15 +1475,16 @@ pepp_status_t p2p_import(pepp_spmv_plan_t* p, int nbuf, const std::vector<P2PHan
             PEPP_CUDA_TRY(cudaIpcOpenMemHandle(&peer_buf[q][b], all[q].buf[b], cudaIpcMemLazyEnablePeerAccess));
             p->p2p_opened.push_back(peer_buf[q][b]);
         }
-        void* sig = nullptr;
-        PEPP_CUDA_TRY(cudaIpcOpenMemHandle(&sig, all[q].sig, cudaIpcMemLazyEnablePeerAccess));
-        p->p2p_opened.push_back(sig);
-        auto* qs = (unsigned long long*)sig;
-        p->p2p_peer_ready[j] = qs + me;            // q's ready[me]
-        p->p2p_peer_arrive[j] = qs + P + me;       // q's arrive[me]
-        p->p2p_my_ready[j] = p->d_sig + q;         // my ready[q]
+        if ((s = open_sig(q))) return s;
+        p->p2p_ready_in[j] = p->d_sig + q;              // my ready[q]: q may now be written
+        p->p2p_arrive_out[j] = peer_sig[q] + P + me;    // q's arrive[me]
     }
-    for (size_t j = 0; j < recvp.size(); ++j) p->p2p_my_arrive[j] = p->d_sig + P + recvp[j];
+    for (size_t j = 0; j < recvp.size(); ++j) {
+        const int q = recvp[j];
+        if ((s = open_sig(q))) return s;
+        p->p2p_ready_out[j] = peer_sig[q] + me;         // q's ready[me]: q may write into me
+        p->p2p_arrive_in[j] = p->d_sig + P + q;         // my arrive[q]
+    }
     p->p2p_nsend = (int)sendp.size();
     p->p2p_nrecv = (int)recvp.size();
     // push ranges: each peer's send range cut to the head and the tail segments
@@ -1489,12 +1562,14 @@ pepp_status_t p2p_launch_t(pepp_spmv_plan_t* p, int b, const T* x, T* y, cudaStr
     }
     a.nsend = p->p2p_nsend;
     for (int j = 0; j < a.nsend; ++j) {
-        a.peer_ready[j] = p->p2p_peer_ready[j];
-        a.peer_arrive[j] = p->p2p_peer_arrive[j];
-        a.my_ready[j] = p->p2p_my_ready[j];
+        a.ready_in[j] = p->p2p_ready_in[j];
+        a.arrive_out[j] = p->p2p_arrive_out[j];
     }
     a.nrecv = p->p2p_nrecv;
-    for (int j = 0; j < a.nrecv; ++j) a.my_arrive[j] = p->p2p_my_arrive[j];
+    for (int j = 0; j < a.nrecv; ++j) {
+        a.ready_out[j] = p->p2p_ready_out[j];
+        a.arrive_in[j] = p->p2p_arrive_in[j];
+    }
     const int P = p->opts.nranks;
     a.epoch = p->d_sig + 2 * P;
     a.done = (unsigned int*)(p->d_sig + 2 * P + 1);
@@ -1502,6 +1577,14 @@ pepp_status_t p2p_launch_t(pepp_spmv_plan_t* p, int b, const T* x, T* y, cudaStr
     a.timeout_ns = p->p2p_timeout_ns;
     pepp::k::halo_push_kernel<T><<<p->p2p_grid, 256, 0, st>>>(p->d_rp, p->d_col, (const T*)p->d_val, x, y, a);
     return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
+}
+
+// a rank can run the fused push when the rows it sends lie in its head /
+// tail split (sub-plans) or when it sends nothing (it then only signals)
+bool p2p_capable(const pepp_spmv_plan_t* p) {
+    if (p->sub[1]) return true;
+    for (const auto& t : p->send_x) if (t.count) return false;
+    return true;
 }
 
 // index of the registered buffer y points to, -1 if none
@@ -1524,7 +1607,9 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     if (o->variant_mask != 0 && (o->variant_mask & ((1u << PEPP_V_COUNT) - 1)) == 0) return PEPP_E_INVALID;
 
     p->opts = *o;
-    if (const char* e = std::getenv("PEPP_RESERVE_SMS")) p->reserve_sms = std::atoi(e);   // experiments only (tools/overlap_cost.py)
+#ifdef PEPP_EXP_RESERVE_SMS   // experiments only (tools/overlap_cost.py): SMs a top-level plan's persistent grids leave free
+    if (!p->reserve_sms) p->reserve_sms = PEPP_EXP_RESERVE_SMS;
+#endif
     p->nrows = A->nrows; p->ncols = A->ncols; p->nnz = A->nnz; p->first = A->first;
     p->pad = (int)(((A->first % 4) + 4) % 4);
     if (o->nranks > 1) {
@@ -1653,6 +1738,21 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     }
     p->eligible.assign(p->cands.size(), 1);
     p->pending.assign(p->cands.size(), 0);
+    {   // bytes each candidate moves per call (pepp_choice_t.layout_bytes)
+        const int64_t es = (int64_t)p->esz;
+        const int64_t csr = A->nnz * (es + 4) + (A->nrows + 1) * 4 + A->ncols * es + A->nrows * es;
+        for (const Candidate& c : p->cands) {
+            int64_t b = csr;
+            if (c.variant == PEPP_V_SELL) b = p->sell_bytes;
+            else if (c.variant == PEPP_V_MERGE_PATH) {
+                const int64_t nt = c.param == kMergeWarpParam ? p->ntiles_w : p->ntiles;
+                b += (nt + 1) * 8 + nt * 2 * (4 + 8);   // tile coordinates, carries written and read back
+            } else if (c.variant == PEPP_V_CSR_STREAM) {
+                b += (int64_t)p->nitems * 16 + (int64_t)p->nlong * 16;
+            }
+            p->cand_bytes.push_back(b);
+        }
+    }
     I.ncandidates = (int32_t)p->cands.size();
 
     p->grid_csr[1] = grid_for((const void*)pepp::k::csr_vector_kernel<2, kBlock, double>, kBlock, A->nrows, kBlock / 2, p->sm_count);
@@ -1679,7 +1779,10 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     }
 
     // ---- history ----
-    p->key = pepp::context_key(A->nrows, A->ncols, A->nnz, I.cv_row, o->nranks);
+    // the instance bits keep fp32 / value-compressed plans (different kernels,
+    // ~1.6x apart on config 4) from sharing history records with fp64 ones
+    p->key = pepp::context_key(A->nrows, A->ncols, A->nnz, I.cv_row, o->nranks,
+                               (p->vt == PEPP_VALUE_F32 ? PEPP_KEY_F32 : 0) | (o->compress_values ? PEPP_KEY_COMPRESS : 0));
     I.key = p->key;
     p->hist = pepp::history_new();
     if (!p->hist) return PEPP_E_NOMEM;
@@ -1803,7 +1906,10 @@ pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flag
     PEPP_CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_fork, 0));
     // interior first (the host may block inside a synchronous exchange)
     pepp_choice_t u{};
-    pepp_status_t s = pepp_spmv_exec(p->sub[1], x, yb + p->sub_r0[1] * (int64_t)p->esz, sf, st, nullptr, &u);
+    // a rank that sends nothing (no split) computes its whole block as the
+    // "interior" through its own selection (PEPP_Y_LOCAL: no exchange)
+    pepp_status_t s = p->sub[1] ? pepp_spmv_exec(p->sub[1], x, yb + p->sub_r0[1] * (int64_t)p->esz, sf, st, nullptr, &u)
+                                : pepp_spmv_exec(p, x, y, sf | PEPP_Y_LOCAL, st, nullptr, &u);
     const int b = p2p_index(p, y);
     if (b >= 0) {
         // fused: head + tail rows computed, pushed into the peers' buffer b and
@@ -1833,6 +1939,7 @@ pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flag
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_plan(const pepp_csr_t* A, const pepp_spmv_opts_t* opts,
                                                 pepp_spmv_plan_t** out) {
+    PEPP_NVTX("pepp_spmv_plan");
     if (!out) return PEPP_E_INVALID;
     *out = nullptr;
     if (!A) return PEPP_E_INVALID;
@@ -1866,6 +1973,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_cho
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void* x, void* y, int flags,
                                                 void* stream, const pepp_choice_t* force, pepp_choice_t* used) {
+    PEPP_NVTX("pepp_spmv_exec");
     if (!p) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
     if ((!x && p->ncols > 0) || (!y && p->global_rows > 0)) return PEPP_E_INVALID;
@@ -1884,7 +1992,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         if (cudaStreamIsCapturing(st, &cs) != cudaSuccess) { (void)cudaGetLastError(); cs = cudaStreamCaptureStatusNone; }
         capturing = cs != cudaStreamCaptureStatusNone;
     }
-    if (!force && p->sub[1] && (flags & PEPP_Y_NEXT_INPUT) && !(flags & PEPP_Y_REPLICATED) && p->exchange == PEPP_X_HALO) {
+    if (!force && (flags & PEPP_Y_NEXT_INPUT) && !(flags & PEPP_Y_REPLICATED) && p->exchange == PEPP_X_HALO &&
+        (p->sub[1] || p2p_index(p, y) >= 0)) {
         pepp_status_t s = capturing ? PEPP_OK : scratch_acquire(p, st);
         if (!s) s = exec_overlap(p, x, y, flags, st, used);
         if (!s && !capturing) s = scratch_release(p, st);
@@ -1970,9 +2079,11 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_graph_create(pepp_spmv_plan_t* p, co
     if (p->sticky) return p->sticky;
     DeviceScope dscope(p->device);
     if (!dscope.ok) return PEPP_E_CUDA;
-    // choose once, outside the capture (calibration calls would not be timed)
+    // choose once, outside the capture: the best measured candidate so far,
+    // else the heuristic (frozen: a calibration pick would be baked into
+    // every replay untimed)
     pepp_choice_t ch{};
-    pepp_status_t s = select_choice(p, &ch);
+    pepp_status_t s = select_choice(p, &ch, /*frozen=*/true);
     if (s) return s;
     cudaStream_t st = (cudaStream_t)stream;
     cudaStream_t cap = nullptr;
@@ -2040,10 +2151,16 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_vec(pepp_spmv_plan_t* p, pepp_v
     double *dx = nullptr, *dy = nullptr;
     pepp_status_t s = pepp_vector_acquire_device(x, PEPP_ACCESS_READ, stream, &dx);
     if (s) return s;
-    // y is written (A4): with an exchange, other ranks' rows are written too;
-    // without one, rows outside this block are left untouched, so a
-    // partitioned LOCAL call keeps y's device copy as the valid one
-    s = pepp_vector_acquire_device(y, PEPP_ACCESS_WRITE, stream, &dy);
+    // y is written (A4). Every global row is written only when the call ends
+    // with an allgather (PEPP_Y_REPLICATED, or NEXT_INPUT on an allgather
+    // plan) or the plan is unpartitioned; a partitioned LOCAL or halo call
+    // writes this block's rows (+ ghosts) and leaves the rest as they were,
+    // so y is READWRITE there: its device copy must hold the current values
+    // of the rows the call does not write before the whole buffer becomes the
+    // valid copy
+    const bool all_rows = p->opts.nranks == 1 || (flags & PEPP_Y_REPLICATED) ||
+                          ((flags & PEPP_Y_NEXT_INPUT) && p->exchange == PEPP_X_ALLGATHER);
+    s = pepp_vector_acquire_device(y, all_rows ? PEPP_ACCESS_WRITE : PEPP_ACCESS_READWRITE, stream, &dy);
     if (s) return s;
     s = pepp_spmv_exec(p, dx, dy, flags, stream, force, used);
     const pepp_status_t s1 = pepp_vector_release_device(x, stream);
@@ -2052,6 +2169,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_vec(pepp_spmv_plan_t* p, pepp_v
 }
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* y, int flags, void* stream) {
+    PEPP_NVTX("pepp_spmv_exchange");
     if (!p) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
     if (p->opts.nranks == 1 || !(flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED))) return PEPP_OK;
@@ -2092,6 +2210,7 @@ void host_rows(const pepp_spmv_plan_t* p, int flags, int64_t* lo, int64_t* cnt) 
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const void* x_host, void* y_host,
                                                      int32_t iterations, int flags, void* stream) {
+    PEPP_NVTX("pepp_spmv_exec_host");
     if (!p || !x_host || !y_host || iterations < 1) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
     if (iterations > 1 && p->ncols != p->global_rows) return PEPP_E_INVALID;
@@ -2130,6 +2249,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host(pepp_spmv_plan_t* p, const
 extern "C" PEPP_API pepp_status_t pepp_spmv_exec_host_batch(pepp_spmv_plan_t* p, int32_t nbatch,
                                                            const void* const* x_hosts, void* const* y_hosts,
                                                            int32_t iterations, int flags, void* stream) {
+    PEPP_NVTX("pepp_spmv_exec_host_batch");
     if (!p || nbatch < 0 || (nbatch > 0 && (!x_hosts || !y_hosts)) || iterations < 1) return PEPP_E_INVALID;
     for (int32_t k = 0; k < nbatch; ++k) if (!x_hosts[k] || !y_hosts[k]) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
@@ -2214,16 +2334,25 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_destroy(pepp_spmv_plan_t* p) {
 }
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_p2p_buffers(pepp_spmv_plan_t* p, int32_t nbuf, void** bufs) {
+    PEPP_NVTX("pepp_spmv_p2p_buffers");
     if (!p || !bufs || nbuf < 1 || nbuf > kP2PMaxBuf) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
     if (p->p2p_nbuf) return PEPP_E_STATE;
-    if (p->opts.nranks < 2 || p->exchange != PEPP_X_HALO || !p->sub[1]) return PEPP_E_UNSUPPORTED;
+    if (p->opts.nranks < 2) return PEPP_E_UNSUPPORTED;
     DeviceScope dscope(p->device);
     if (!dscope.ok) { pepp::set_last_error("cannot select the plan's device", "DeviceScope", __LINE__); return PEPP_E_CUDA; }
     cudaStream_t st = nullptr;
     PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
-    pepp_status_t s = p2p_register(p, nbuf, st);
+    // agreement first (collective on every path): a rank that cannot take
+    // part — no halo exchange, or rows it sends outside a head / tail split —
+    // makes every rank return PEPP_E_UNSUPPORTED before any rank enters the
+    // registration collectives
+    int64_t cant = (p->exchange != PEPP_X_HALO || !p2p_capable(p)) ? 1 : 0;
+    pepp_status_t s = nccl_allmax(p, st, &cant);
+    if (!s && cant) s = PEPP_E_UNSUPPORTED;
+    else if (!s) s = p2p_register(p, nbuf, st);
     cudaStreamDestroy(st);
+    if (s == PEPP_E_UNSUPPORTED) return s;   // nothing changed: the plan stays usable (NCCL halo)
     if (s) { p->sticky = s; return s; }
     for (int b = 0; b < nbuf; ++b) bufs[b] = p->p2p_buf[b];
     p->info.p2p_buffers = nbuf;

@@ -47,65 +47,35 @@ def test_library_exports_every_declared_symbol():
 def test_abi_version_and_status_strings():
     from paper_conf_sc_dastgeerlk12_b200 import _capi
     L = _capi.lib()
-    assert L.pepp_abi_version() == _capi.ABI_VERSION == 5
+    assert L.pepp_abi_version() == _capi.ABI_VERSION == 6
     for s in [0, -1, -2, -3, -4, -5, -6]:
         assert L.pepp_status_str(s).decode().startswith("PEPP_")
 
 
 def test_struct_layouts_match_c():
+    """Every field of every ctypes mirror sits at the C offset (generated from
+    the mirrors' _fields_, so a field added on one side only fails here)."""
     from paper_conf_sc_dastgeerlk12_b200 import _capi as C
-    probe = r"""
-#include <stdio.h>
-#include <stddef.h>
-#include "pepp_spmv.h"
-#define P(T, f) printf(#T "." #f " %zu\n", offsetof(T, f));
-int main(void) {
-  printf("csr %zu\nopts %zu\nchoice %zu\ninfo %zu\n", sizeof(pepp_csr_t), sizeof(pepp_spmv_opts_t),
-         sizeof(pepp_choice_t), sizeof(pepp_plan_info_t));
-  P(pepp_csr_t, on_device) P(pepp_spmv_opts_t, row_bounds) P(pepp_spmv_opts_t, exchange)
-  P(pepp_spmv_opts_t, history_path) P(pepp_spmv_opts_t, prune) P(pepp_choice_t, predicted_us) P(pepp_choice_t, launches) P(pepp_plan_info_t, key)
-  P(pepp_plan_info_t, sell_fill) P(pepp_plan_info_t, halo_send) P(pepp_plan_info_t, sell_col16_frac) P(pepp_plan_info_t, prior_key) P(pepp_plan_info_t, sell_stencil_frac)
-  P(pepp_spmv_opts_t, overlap) P(pepp_plan_info_t, overlap) P(pepp_plan_info_t, overlap_head) P(pepp_plan_info_t, overlap_tail)
-  P(pepp_spmv_opts_t, predict) P(pepp_spmv_opts_t, predict_user) P(pepp_plan_info_t, predicted)
-  P(pepp_spmv_opts_t, compress_values) P(pepp_plan_info_t, sell_constval_frac) P(pepp_plan_info_t, p2p_buffers) P(pepp_plan_info_t, sell_long_rows) P(pepp_plan_info_t, sell_cap)
-  printf("x_p2p %d\n", (int)PEPP_X_P2P);
-  return 0;
-}
-"""
+    structs = {"pepp_csr_t": C.CSR_T, "pepp_spmv_opts_t": C.OPTS_T, "pepp_choice_t": C.CHOICE_T,
+               "pepp_plan_info_t": C.INFO_T}
+    lines = []
+    for cname, py in structs.items():
+        lines.append(f'printf("{cname} %zu\\n", sizeof({cname}));')
+        for f, _ in py._fields_:
+            lines.append(f'printf("{cname}.{f} %zu\\n", offsetof({cname}, {f}));')
+    probe = ("#include <stdio.h>\n#include <stddef.h>\n#include \"pepp_spmv.h\"\nint main(void) {\n" +
+             "\n".join(lines) + '\nprintf("x_p2p %d\\n", (int)PEPP_X_P2P);\nreturn 0;\n}\n')
     with tempfile.TemporaryDirectory() as d:
         c = os.path.join(d, "p.c")
         open(c, "w").write(probe)
         exe = os.path.join(d, "p")
         subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), c, "-o", exe])
         vals = dict(l.rsplit(" ", 1) for l in subprocess.check_output([exe], text=True).splitlines())
-    assert int(vals["csr"]) == ctypes.sizeof(C.CSR_T)
-    assert int(vals["opts"]) == ctypes.sizeof(C.OPTS_T)
-    assert int(vals["choice"]) == ctypes.sizeof(C.CHOICE_T)
-    assert int(vals["info"]) == ctypes.sizeof(C.INFO_T)
-    assert int(vals["pepp_csr_t.on_device"]) == C.CSR_T.on_device.offset
-    assert int(vals["pepp_spmv_opts_t.row_bounds"]) == C.OPTS_T.row_bounds.offset
-    assert int(vals["pepp_spmv_opts_t.exchange"]) == C.OPTS_T.exchange.offset
-    assert int(vals["pepp_spmv_opts_t.history_path"]) == C.OPTS_T.history_path.offset
-    assert int(vals["pepp_spmv_opts_t.prune"]) == C.OPTS_T.prune.offset
-    assert int(vals["pepp_choice_t.predicted_us"]) == C.CHOICE_T.predicted_us.offset
-    assert int(vals["pepp_choice_t.launches"]) == C.CHOICE_T.launches.offset
-    assert int(vals["pepp_plan_info_t.key"]) == C.INFO_T.key.offset
-    assert int(vals["pepp_plan_info_t.sell_fill"]) == C.INFO_T.sell_fill.offset
-    assert int(vals["pepp_plan_info_t.halo_send"]) == C.INFO_T.halo_send.offset
-    assert int(vals["pepp_plan_info_t.sell_col16_frac"]) == C.INFO_T.sell_col16_frac.offset
-    assert int(vals["pepp_plan_info_t.prior_key"]) == C.INFO_T.prior_key.offset
-    assert int(vals["pepp_plan_info_t.sell_stencil_frac"]) == C.INFO_T.sell_stencil_frac.offset
-    for f in ("overlap", "overlap_head", "overlap_tail"):
-        assert int(vals["pepp_plan_info_t." + f]) == getattr(C.INFO_T, f).offset
-    assert int(vals["pepp_spmv_opts_t.overlap"]) == C.OPTS_T.overlap.offset
-    assert int(vals["pepp_spmv_opts_t.predict"]) == C.OPTS_T.predict.offset
-    assert int(vals["pepp_spmv_opts_t.predict_user"]) == C.OPTS_T.predict_user.offset
-    assert int(vals["pepp_plan_info_t.predicted"]) == C.INFO_T.predicted.offset
-    assert int(vals["pepp_spmv_opts_t.compress_values"]) == C.OPTS_T.compress_values.offset
-    assert int(vals["pepp_plan_info_t.sell_constval_frac"]) == C.INFO_T.sell_constval_frac.offset
-    assert int(vals["pepp_plan_info_t.p2p_buffers"]) == C.INFO_T.p2p_buffers.offset
-    assert int(vals["pepp_plan_info_t.sell_long_rows"]) == C.INFO_T.sell_long_rows.offset
-    assert int(vals["pepp_plan_info_t.sell_cap"]) == C.INFO_T.sell_cap.offset
+    for cname, py in structs.items():
+        assert int(vals[cname]) == ctypes.sizeof(py), cname
+        for f, _ in py._fields_:
+            assert int(vals[f"{cname}.{f}"]) == getattr(py, f).offset, f"{cname}.{f}"
+    # and the C structs have no field the mirrors lack (sizes match, offsets ascend)
     assert int(vals["x_p2p"]) == C.X_P2P
 
 

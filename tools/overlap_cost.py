@@ -89,11 +89,12 @@ def main():
         # as the overlapped call runs it: interior on the caller's stream (its
         # persistent grid leaving `reserve` SMs), head + tail on a high-priority
         # side stream, fork / join (the exchange itself is not modelled)
+        # (round 1 swept the reserve with a PEPP_RESERVE_SMS environment knob;
+        # round 2 removed run-time experiment knobs from the library: rebuild
+        # with -DPEPP_EXP_RESERVE_SMS=n for a sweep)
         side = torch.cuda.Stream(priority=-1)
-        for reserve in (0, 2, 4):
-            os.environ["PEPP_RESERVE_SMS"] = str(reserve)
+        for reserve in (int(os.environ.get("PEPP_EXP_RESERVE_SMS", "0")),):
             inner = pepp.Plan.from_csr(gen.row_block(A, r0 + n, r1 - n))
-            del os.environ["PEPP_RESERVE_SMS"]
             edges = [(pepp.Plan.from_csr(gen.row_block(A, s, e)), s, e) for s, e in [(r0, r0 + n), (r1 - n, r1)]]
 
             def conc():
