@@ -15,8 +15,11 @@ exchange + history update).
                   [--workload lap8192|uniform1m|zipf4m|lap64] [--iters I] [--variant csr_vector:4|merge_path|sell]
 
 One JSON line on rank 0. Multi-GPU: launched by torchrun (RANK / WORLD_SIZE /
-LOCAL_RANK / MASTER_* from the environment); times are device events, max
-over ranks.
+LOCAL_RANK / MASTER_* from the environment), or `--gpus N` alone re-executes
+itself under torch.distributed.run with N ranks; times are device events, max
+over ranks. The default line also carries BASELINE configs 1-3 (`configs`:
+per-SpMV time, layout-bytes roofline fraction, selector ratio, plan time,
+cold single call with the matrix upload).
 """
 from __future__ import annotations
 
@@ -149,8 +152,9 @@ def measured_peak() -> tuple[float, str]:
 
 
 def traffic_for(kernel: str, workload: str, dtype: str = "f64"):
-    """dram read+write bytes per launch from the committed ncu --set full
-    summary, if any (entries are per workload and fp64 unless keyed 'name:f32')."""
+    """DRAM read+write bytes per launch from the committed ncu --set full
+    capture of this kernel on this workload (profiles/traffic.json, written by
+    tools/ncu_summary.py), if any — a cross-check of the layout bytes only."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     try:
         d = json.load(open(p))
@@ -159,22 +163,27 @@ def traffic_for(kernel: str, workload: str, dtype: str = "f64"):
         return None
 
 
-def roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, workload, dtype="f64") -> dict:
-    """Roofline of the dominant kernel: algorithmic bytes / launch time vs the
-    measured peak; `traffic` = ncu DRAM bytes per launch (may be below the
-    algorithmic bytes when the variant stores a compressed layout, e.g. SELL
-    16-bit column deltas), with the DRAM-traffic fraction beside it."""
-    traffic = traffic_for(kname, workload, dtype)
+def roofline_obj(kname, layout_bytes, alg_bytes, peak, peak_src, avg_kernel_s, workload, dtype="f64") -> dict:
+    """Roofline of the dominant kernel: the bytes its layout moves per launch
+    (pepp_choice_t.layout_bytes: the matrix arrays as stored and streamed, x
+    read once, y written once) / its average launch time (CUDA events on the
+    launching stream, timed region), against the measured copy peak.
+    `effective_gbs` = SURVEY §8(d)'s algorithmic bytes (nnz*12 + row_ptr +
+    x + y, the metric's CSR-equivalent count) / the same time — a compressed
+    layout does the same work with fewer bytes, so that figure can exceed
+    the peak and is not a roofline fraction. `traffic` = ncu DRAM bytes per
+    launch from the committed capture (profiles/traffic.json), a cross-check:
+    `traffic_vs_layout` should be ~1 (gathers that miss L2 push it above)."""
+    achieved = layout_bytes / avg_kernel_s / 1e9
     d = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "peak_source": peak_src,
          "unit": "GB/s", "frac": round(achieved / peak, 4), "avg_launch_us": round(avg_kernel_s * 1e6, 2),
-         "bytes_per_launch": local_bytes, "traffic": traffic}
+         "bytes_per_launch": int(layout_bytes), "bytes_source": "plan layout (pepp_choice_t.layout_bytes)",
+         "effective_gbs": round(alg_bytes / avg_kernel_s / 1e9, 1), "algorithmic_bytes_per_launch": int(alg_bytes)}
+    traffic = traffic_for(kname, workload, dtype)
+    d["traffic"] = traffic
     if traffic:
-        d["traffic_gbs"] = round(traffic / avg_kernel_s / 1e9, 1)
-        d["traffic_frac"] = round(traffic / avg_kernel_s / 1e9 / peak, 4)
-        if traffic < local_bytes:
-            d["note"] = ("achieved counts the metric's algorithmic bytes (nnz*12 B + row_ptr + x + y); the kernel's "
-                         "layout moves fewer (traffic, ncu DRAM bytes per launch), so frac can exceed 1: "
-                         "traffic_frac is the DRAM-side fraction of the measured peak")
+        d["traffic_vs_layout"] = round(traffic / layout_bytes, 4)
+        d["traffic_source"] = "ncu --set full capture committed in profiles/ (traffic.json)"
     return d
 
 
@@ -279,6 +288,7 @@ def value_compressed_leg(args, A, xs, bufs, stream, iters, iterated, flush, peak
             return {"applies": False, "note": "no constant-coefficient chunks in this matrix"}
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(iters)]
         used: dict = {}
+        lbytes: dict = {}
 
         def step(record):
             with torch.cuda.stream(stream):
@@ -294,6 +304,7 @@ def value_compressed_leg(args, A, xs, bufs, stream, iters, iterated, flush, peak
                     if record:
                         ev[k][1].record(stream)
                         used[u.name] = used.get(u.name, 0) + 1
+                        lbytes[u.name] = u.layout_bytes
                     if iterated:
                         src = bufs[k & 1]
         for _ in range(args.warmup):
@@ -306,21 +317,143 @@ def value_compressed_leg(args, A, xs, bufs, stream, iters, iterated, flush, peak
         avg_s = statistics.mean(ms) / 1e3
         chosen = max(used, key=used.get)
         kname = chosen + ("+constval" if chosen.startswith("sell") else "")
+        lb = lbytes[chosen]
         traffic = traffic_for(kname, args.workload, args.dtype)
         d = {"applies": True, "kernel": kname, "constval_frac": info["sell_constval_frac"],
              "avg_launch_us": round(avg_s * 1e6, 2), "gflops": round(2.0 * A.nnz / avg_s / 1e9, 3),
-             "traffic": traffic, "choices": used,
-             "note": "opts.compress_values = 1: constant stencil chunks read only x and write y; lossless"}
+             "layout_bytes": lb, "achieved_gbs": round(lb / avg_s / 1e9, 1),
+             "frac": round(lb / avg_s / 1e9 / peak, 4), "traffic": traffic, "choices": used,
+             "note": "opts.compress_values = 1: constant stencil chunks read only x and write y; lossless; "
+                     "frac = layout bytes (x read once, y written, lists) / launch time / measured peak"}
         if traffic:
-            d["traffic_gbs"] = round(traffic / avg_s / 1e9, 1)
-            d["traffic_frac"] = round(traffic / avg_s / 1e9 / peak, 4)
+            d["traffic_vs_layout"] = round(traffic / lb, 4)
         return d
     finally:
         plan.close()
 
 
+LEG_WORKLOADS = ("lap64", "uniform1m", "zipf4m")   # BASELINE configs 1, 2, 3
+
+
+def config_leg(name: str, args, dev, stream, peak: float, with_cpu: bool) -> dict:
+    """One of BASELINE's single-SpMV configs measured beside the headline (rank
+    0, N = 1): plan time (matrix upload + layouts), the automatic choice's
+    median time per SpMV after calibration (kernel events, L2 flushed between
+    calls), its layout bytes / time against the measured peak, every
+    candidate forced (selector ratio = chosen / best), a cold single call with
+    the matrix upload (plan + pepp_spmv_exec_host: x in, y out), and the CPU
+    oracle's time for one SpMV (break-even call count = plan / (cpu - gpu))."""
+    import torch
+
+    import paper_conf_sc_dastgeerlk12_b200 as pepp
+    R = len(global_rowptr(name)) - 1
+    A = make_block(name, 0, R)
+    x0 = x0_vector(name, A.ncols)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    plan = pepp.Plan.from_csr(A)
+    torch.cuda.synchronize()
+    plan_ms = (time.perf_counter() - t0) * 1e3
+    try:
+        yh = torch.empty(A.nrows, dtype=torch.float64).pin_memory().numpy()
+        xh = torch.from_numpy(x0).pin_memory().numpy()
+        t1 = time.perf_counter()
+        plan.exec_host(xh, yh, iterations=1, stream=stream)      # first call: cold, with its copies
+        cold_call_ms = (time.perf_counter() - t1) * 1e3
+        xs = torch.from_numpy(x0).to(dev)
+        y = torch.empty(A.nrows, dtype=torch.float64, device=dev)
+        small = A.nnz < 100_000
+        flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+        ncal = 200 if small else 40
+        with torch.cuda.stream(stream):
+            for _ in range(ncal):   # calibration (history-based selection settles)
+                plan.exec(xs, y, stream=stream)
+        stream.synchronize()
+        n = 200 if small else 30
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
+        used: dict = {}
+        lb: dict = {}
+        with torch.cuda.stream(stream):
+            for a, b in ev:
+                flush.zero_()
+                a.record(stream)
+                u = plan.exec(xs, y, stream=stream)
+                b.record(stream)
+                used[u.name] = used.get(u.name, 0) + 1
+                lb[u.name] = u.layout_bytes
+        stream.synchronize()
+        us = statistics.median(a.elapsed_time(b) for a, b in ev) * 1e3
+        chosen = max(used, key=used.get)
+        per = {}
+        for c in plan.candidates():
+            f = pepp.Choice(c.variant, c.param)
+            m = 40 if small else 10
+            pairs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(m)]
+            with torch.cuda.stream(stream):
+                for a, b in pairs:
+                    flush.zero_()
+                    a.record(stream)
+                    plan.exec(xs, y, stream=stream, force=f)
+                    b.record(stream)
+            stream.synchronize()
+            per[f.name] = statistics.median(a.elapsed_time(b) for a, b in pairs[2:]) * 1e3
+        best = min(per, key=per.get)
+        graph_us = None
+        if small:   # launch-bound: the same call replayed from a CUDA graph
+            g = plan.graph(xs, y, iterations=1000, mode=0, stream=stream)
+            with torch.cuda.stream(stream):
+                g.launch(stream)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                for _ in range(5):
+                    g.launch(stream)
+                e1.record(stream)
+            e1.synchronize()
+            graph_us = round(e0.elapsed_time(e1) * 1e3 / 5000, 3)
+            g.close()
+        alg = A.nnz * 12 + (A.nrows + 1) * 4 + A.ncols * 8 + A.nrows * 8
+        d = {"desc": WORKLOADS[name]["desc"], "rows": A.nrows, "nnz": A.nnz, "chosen": chosen,
+             "us_per_spmv": round(us, 2), "gflops": round(2.0 * A.nnz / (us * 1e-6) / 1e9, 2),
+             "layout_bytes": lb[chosen], "achieved_gbs": round(lb[chosen] / (us * 1e-6) / 1e9, 1),
+             "frac": round(lb[chosen] / (us * 1e-6) / 1e9 / peak, 4),
+             "effective_gbs": round(alg / (us * 1e-6) / 1e9, 1),
+             "selector": {"best": best, "best_us": round(per[best], 2), "ratio": round(per.get(chosen, us) / per[best], 4),
+                          "candidates_us": {k: round(v, 2) for k, v in per.items()}},
+             "plan_ms": round(plan_ms, 1), "cold_call_incl_copies_ms": round(cold_call_ms, 3),
+             "e2e_single_call_incl_upload_ms": round(plan_ms + cold_call_ms, 1),
+             "graph_us_per_call": graph_us}
+        if small:
+            d["note"] = "launch-latency bound (20 K nnz): frac not a roofline claim; see graph_us_per_call"
+        if with_cpu:
+            import oracle
+            t2 = time.perf_counter()
+            reps = 0
+            while reps < 3 or time.perf_counter() - t2 < 0.5:
+                oracle.spmv(A, x0, parallel=True)
+                reps += 1
+            cpu_ms = (time.perf_counter() - t2) * 1e3 / reps
+            d["cpu_oracle_ms"] = round(cpu_ms, 3)
+            gap = cpu_ms - us * 1e-3
+            d["break_even_calls"] = round(plan_ms / gap, 1) if gap > 0 else None
+        return d
+    finally:
+        plan.close()
+        torch.cuda.empty_cache()
+
+
 # --------------------------------------------------------------- arms
 METRIC = "SpMV GFLOP/s (aggregate over ranks); achieved HBM GB/s in 'hbm'"
+
+
+def config_of(args, R: int, Z: int) -> dict:
+    """The workload description both arms print (same dict, same keys)."""
+    wl = WORKLOADS[args.workload]
+    iters = args.iters or wl["iters"]
+    alg = Z * 12 + (R + 1) * 4 + R * 16
+    l2 = (f"inputs larger than L2 ({alg / 1e9:.1f} GB/SpMV)" if wl["iterated"]
+          else "L2 flushed (512 MB memset) between SpMVs; kernel events only" if alg < 4 * (1 << 30)
+          else f"inputs larger than L2 ({alg / 1e9:.1f} GB/SpMV)")
+    return {"workload": args.workload, "desc": wl["desc"], "spmv_per_step": iters, "rows": R, "nnz": Z, "l2": l2}
 
 
 def run_reference(args, rank: int, world: int) -> None:
@@ -346,7 +479,7 @@ def run_reference(args, rank: int, world: int) -> None:
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(1000 * t / args.steps, 3), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": args.workload, "desc": wl["desc"], "rows": A.nrows, "nnz": A.nnz},
+            "config": config_of(args, A.nrows, A.nnz),
             "cpu_baseline": {"value": round(val, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
                              "sample": sample, "host": host_cpu()},
             "e2e": {"value": round(val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -390,10 +523,16 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     force = parse_variant(args.variant)
     # --variant pins the choice everywhere (timed steps and the e2e leg): the
     # plan is built with that variant only
+    # plan = matrix upload (host -> device) + validation + every variant's
+    # layout (a1-a3), timed: the cost a caller pays once before any call
+    torch.cuda.synchronize()
+    t_plan = time.perf_counter()
     plan = pepp.Plan.from_csr(A, nranks=world, rank=rank, row_bounds=bounds if world > 1 else None,
                               nccl_unique_id=uid, prune=not args.no_prune,
                               variant_mask=(1 << force.variant) if force is not None else 0,
                               compress_values=args.value_compression)
+    torch.cuda.synchronize()
+    plan_ms = (time.perf_counter() - t_plan) * 1e3
     info = plan.info()
     flags = pepp.Y_NEXT_INPUT if iterated else pepp.Y_LOCAL
     overlapped = bool(world > 1 and iterated and force is None and info["overlap"])
@@ -401,17 +540,27 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     stream = torch.cuda.Stream(device=dev)
     xs = torch.from_numpy(x0).to(dev)
     p2p = overlapped and not args.no_p2p
+    p2p_note = None
+    bufs = None
     if p2p:
         # symmetric buffers: the boundary kernel pushes the halo straight into
-        # the neighbours' copies over peer memory (PEPP_X_P2P), no NCCL per iteration
-        bufs = plan.p2p_buffers(2)
-    else:
+        # the neighbours' copies over peer memory (PEPP_X_P2P), no NCCL per
+        # iteration. The library's registration is agreed on by every rank:
+        # if any rank cannot map its peers (no CUDA IPC / peer access) or
+        # cannot take part, all ranks get the same error and the plan keeps
+        # the NCCL halo — fall back to it here.
+        try:
+            bufs = plan.p2p_buffers(2)
+        except pepp.PeppError as e:
+            p2p, p2p_note = False, f"p2p unavailable, NCCL halo used: {e}"[:300]
+    if bufs is None:
         bufs = [torch.empty(R, dtype=tdt, device=dev) for _ in range(2)]
     flush = None if iterated or Z * 12 > 4 * (1 << 30) else torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     ev_pool = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(iters)]
     launches = {"n": 0}
     used_count: dict = {}
+    used_bytes: dict = {}
 
     def one_step(record: bool):
         """`iters` SpMVs through the C-ABI. Iterated: x0 -> b0 -> b1 -> b0 ...
@@ -438,6 +587,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
                 if record:
                     b.record(stream)
                     used_count[u.name] = used_count.get(u.name, 0) + 1
+                    used_bytes[u.name] = u.layout_bytes
                     launches["n"] += u.launches   # the library's own count of its kernels in this call
                 if not overlapped and flags != pepp.Y_LOCAL and world > 1:
                     plan.exchange(dst, flags, stream=stream)
@@ -510,11 +660,15 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
 
     # roofline of the dominant kernel on this rank (rank 0 reports)
     avg_kernel_s = statistics.mean(kern_ms) / 1e3
-    local_bytes = A.nnz * (4 + esz) + (A.nrows + 1) * 4 + (A.nrows + info["halo_recv"]) * esz + A.nrows * esz
+    local_alg = A.nnz * (4 + esz) + (A.nrows + 1) * 4 + (A.nrows + info["halo_recv"]) * esz + A.nrows * esz
     if world == 1:
-        local_bytes = alg_bytes_global
-    achieved = local_bytes / avg_kernel_s / 1e9
+        local_alg = alg_bytes_global
     chosen = max(used_count, key=used_count.get) if used_count else "?"
+    layout_bytes = used_bytes.get(chosen, local_alg)
+    if overlapped:   # the call's `used` is the interior sub-plan's: use the whole block's layout of that variant
+        for c in plan.candidates():
+            if c.name == chosen:
+                layout_bytes = c.layout_bytes
 
     # ---- the value-compressed layout (opts.compress_values), reported beside the headline ----
     vc = None
@@ -602,6 +756,26 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     if rank == 0 and world == 1 and not args.no_cpu and not f32:
         cpu = cpu_baseline(A, x0, 2 if A.nnz > 10_000_000 else 200)
 
+    # transfer- and plan-inclusive view (the paper's Fig. 5 setting, P@35591-35720)
+    step_s = te / e2e_steps
+    with_plan = {"plan_ms": round(plan_ms, 1),
+                 "first_step_incl_plan_gflops": round(2.0 * Z * e2e_iters / (plan_ms / 1e3 + step_s) / 1e9, 3),
+                 "note": "one e2e step (host x in, iterations, host y out) plus the plan that uploads the matrix"}
+    if cpu:
+        t_cpu = 2.0 * Z / (cpu["value"] * 1e9)
+        t_gpu = secs / nspmv
+        with_plan["break_even_spmvs_vs_cpu_oracle"] = round(plan_ms / 1e3 / (t_cpu - t_gpu), 1) if t_cpu > t_gpu else None
+
+    # BASELINE configs 1-3 beside the headline (rank 0, N = 1, default workload)
+    legs = None
+    if rank == 0 and world == 1 and args.workload == "lap8192" and not args.no_legs and not f32 and force is None:
+        legs = {}
+        for name in LEG_WORKLOADS:
+            try:
+                legs[name] = config_leg(name, args, dev, stream, peak, with_cpu=not args.no_cpu)
+            except Exception as e:   # reported, never fatal for the headline
+                legs[name] = {"error": repr(e)[:300]}
+
     if rank == 0:
         kname = chosen
         if kname.startswith("sell") and info["sell_constval_frac"] > 0:
@@ -611,15 +785,17 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             "value": round(gflops, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
-            "config": {"workload": args.workload, "desc": wl["desc"], "spmv_per_step": iters,
-                       "rows": R, "nnz": Z, "l2": "inputs larger than L2 (5.4 GB/SpMV)" if iterated
-                       else "L2 flushed (512 MB memset) between SpMVs; kernel events only",
-                       "exchange": "p2p (fused boundary kernel, peer-memory stores)" if p2p
-                       else pepp._capi.EXCHANGE_NAMES.get(info["exchange"], "?"),
-                       "variant": args.variant or "auto (history-based per call)"},
+            "config": config_of(args, R, Z),
+            "run": {"exchange": ("p2p (fused boundary kernel, peer-memory stores)" if p2p
+                                 else pepp._capi.EXCHANGE_NAMES.get(info["exchange"], "?")),
+                    "p2p_fallback": p2p_note,
+                    "variant": args.variant or "auto (history-based per call)",
+                    "plan_ms": round(plan_ms, 1),
+                    "plan_note": "pepp_spmv_plan wall time on rank 0: host -> device copy of the matrix, "
+                                 "validation, context extraction and every variant's layout (a1-a3); paid once"},
             "hbm": {"achieved_gbs": round(gbs, 1), "frac_of_measured": round(gbs / (world * peak), 4),
                     "frac_of_8tbs": round(gbs / (world * 8000.0), 4), "algorithmic_bytes_per_spmv": alg_bytes_global},
-            "roofline": dict(roofline_obj(kname, achieved, peak, peak_src, avg_kernel_s, local_bytes, args.workload, args.dtype),
+            "roofline": dict(roofline_obj(kname, layout_bytes, local_alg, peak, peak_src, avg_kernel_s, args.workload, args.dtype),
                              **({"launch_includes": "interior kernel + the fused boundary/push kernel (P2P halo)"
                                  if p2p else "head + interior + tail kernels and the overlapped halo exchange"}
                                 if overlapped else {})),
@@ -627,7 +803,9 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
                     "d2h_bytes_per_step": A.nrows * esz, "spmv_per_step": e2e_iters,
                     "steps": e2e_steps,
                     "api": "pepp_spmv_exec_host_batch (per step: pinned host x -> device, iterations, device -> "
-                           "pinned host y; step k+1's input copy and step k-1's output copy overlap step k)"},
+                           "pinned host y; step k+1's input copy and step k-1's output copy overlap step k)",
+                    "with_plan": with_plan},
+            "configs": legs,
             "gpu_launches": launches["n"],
             "graph": graph_info,
             "selector": sel,
@@ -664,6 +842,7 @@ def main():
     ap.add_argument("--no-value-compression", action="store_true", help=argparse.SUPPRESS)   # the default now
     ap.add_argument("--no-vc-leg", action="store_true", help="skip the value-compressed leg")
     ap.add_argument("--no-library", action="store_true", help="skip the cuSPARSE context measurement")
+    ap.add_argument("--no-legs", action="store_true", help="skip the BASELINE config 1-3 legs of the default line")
     ap.add_argument("--no-p2p", action="store_true",
                     help="N > 1: NCCL halo per iteration instead of the fused peer-memory push (PEPP_X_P2P)")
     ap.add_argument("--dtype", choices=["f64", "f32"], default="f64",
@@ -671,9 +850,28 @@ def main():
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
 
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # `python bench.py --gpus N` on its own: one process per GPU, launched
+        # the way the driver launches N > 1 (torch.distributed.run, 127.0.0.1)
+        import socket
+        sk = socket.socket()
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+        sk.close()
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(args.gpus),
+               "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+        sys.exit(subprocess.call(cmd))
+
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world} (one process per GPU)")
+    if world > 1:
+        # NCCL's communicator init lines (rank, nranks, transport) in the log:
+        # evidence of the N-rank communicators the library and torch build
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     # Test-only knobs (tests/test_gpu_bench_multirank.py): run every rank on one
     # device with gloo for torch.distributed (the library then needs
     # PEPP_NCCL_LIB pointing at the NCCL stand-in). Never set by the driver.

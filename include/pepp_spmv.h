@@ -346,7 +346,13 @@ pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* y, int flags, void* 
    (pepp_plan_info_t.overlap == 1; a rank that sends nothing computes its
    whole block on `stream` and only signals). The ranks agree first (one
    max-reduce): if any rank cannot take part, EVERY rank returns
-   PEPP_E_UNSUPPORTED and the plan stays usable with the NCCL halo.
+   PEPP_E_UNSUPPORTED and the plan stays usable with the NCCL halo. A CUDA
+   failure on any rank (IPC export or peer mapping) is also agreed on: every
+   rank returns PEPP_E_CUDA, the partial registration is undone and the plan
+   stays usable with the NCCL halo (callers fall back; bench.py does). Only
+   a failing collective (PEPP_E_NCCL) leaves the plan in a sticky error.
+   Test hook: environment PEPP_FAULT_P2P_EXPORT=<rank> makes that rank's
+   export fail (fault injection for the fallback test; no other effect).
    PEPP_E_STATE if already registered. A peer that stops calling makes the
    waiting kernel give up after 20 s and the plan's next call return
    PEPP_E_NCCL. Errors: PEPP_E_INVALID, PEPP_E_CUDA (IPC unavailable),

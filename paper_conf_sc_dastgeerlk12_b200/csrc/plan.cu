@@ -1418,10 +1418,28 @@ pepp_status_t nccl_barrier(pepp_spmv_plan_t* p, cudaStream_t st) {
     return nccl_allmax(p, st, &v);
 }
 
+// undo a registration every rank agreed had failed: nothing of it is in use
+// on any rank, so the plan stays usable with the NCCL halo
+void p2p_reset(pepp_spmv_plan_t* p) {
+    for (void* m : p->p2p_opened) cudaIpcCloseMemHandle(m);
+    p->p2p_opened.clear();
+    for (void*& b : p->p2p_buf)
+        if (b) { cudaFree(b); b = nullptr; p->dev_bytes -= p->global_rows * (int64_t)p->esz; }
+    if (p->d_sig) { cudaFree(p->d_sig); p->d_sig = nullptr; p->dev_bytes -= (int64_t)sizeof(unsigned long long) * (2 * p->opts.nranks + 2); }
+    if (p->h_err) { cudaFreeHost(p->h_err); p->h_err = nullptr; }
+    p->d_err = nullptr;
+    p->p2p_nbuf = p->p2p_npush = p->p2p_nsend = p->p2p_nrecv = 0;
+    (void)cudaGetLastError();
+}
+
 // this rank's half: buffers, signal block, error flag, IPC export
 pepp_status_t p2p_export(pepp_spmv_plan_t* p, int nbuf, cudaStream_t st, P2PHandles* mine) {
     const int P = p->opts.nranks;
     pepp_status_t s;
+    // test-only fault injection (tests/test_gpu_partitioned.py): this rank's
+    // export fails, so every rank must return the error and fall back
+    if (const char* f = std::getenv("PEPP_FAULT_P2P_EXPORT"))
+        if (std::atoi(f) == p->opts.rank) { pepp::set_last_error("injected export failure", "PEPP_FAULT_P2P_EXPORT", __LINE__); return PEPP_E_CUDA; }
     if (!p->side) {   // a rank without a head / tail split (it sends nothing) still forks a side stream
         int lo = 0, hi = 0;
         PEPP_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
@@ -1540,8 +1558,8 @@ pepp_status_t p2p_register(pepp_spmv_plan_t* p, int nbuf, cudaStream_t st) {
     // mapped its peers and zeroed its flags)
     int64_t fail = s ? 1 : 0;
     pepp_status_t sb = nccl_allmax(p, st, &fail);
-    if (s) return s;
-    if (sb) return sb;
+    if (sb) return PEPP_E_NCCL;   // no agreement: the caller makes the plan's error sticky
+    if (s) return s;              // agreed failure (every rank returns an error)
     if (fail) { pepp::set_last_error("a peer rank could not map its peers' buffers", "p2p_register", __LINE__); return PEPP_E_CUDA; }
     p->p2p_nbuf = nbuf;
     return PEPP_OK;
@@ -2353,6 +2371,12 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_p2p_buffers(pepp_spmv_plan_t* p, int
     else if (!s) s = p2p_register(p, nbuf, st);
     cudaStreamDestroy(st);
     if (s == PEPP_E_UNSUPPORTED) return s;   // nothing changed: the plan stays usable (NCCL halo)
+    if (s && s != PEPP_E_NCCL) {
+        // every rank saw the failure through the agreement max-reduce: undo,
+        // and the plan keeps working with the NCCL halo (not sticky)
+        p2p_reset(p);
+        return s;
+    }
     if (s) { p->sticky = s; return s; }
     for (int b = 0; b < nbuf; ++b) bufs[b] = p->p2p_buf[b];
     p->info.p2p_buffers = nbuf;

@@ -28,23 +28,40 @@ def _port() -> int:
     return p
 
 
-def test_bench_two_ranks_one_gpu():
+@pytest.mark.parametrize("launch,fault", [("torchrun", False), ("self", False), ("self", True)])
+def test_bench_two_ranks_one_gpu(launch, fault):
+    """launch = torchrun: the driver's command line; self: `python bench.py
+    --gpus 2` with no WORLD_SIZE re-executes itself under
+    torch.distributed.run. fault: rank 1's CUDA-IPC export is made to fail
+    (PEPP_FAULT_P2P_EXPORT=1): every rank gets the agreed error and the bench
+    falls back to the NCCL halo (reported in run.p2p_fallback)."""
     sys.path.insert(0, HERE)
     from test_gpu_partitioned import _build_fake
     env = dict(os.environ, PEPP_NCCL_LIB=_build_fake(), PEPP_BENCH_ONE_DEVICE="1", PEPP_BENCH_DIST_BACKEND="gloo")
-    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
-           "127.0.0.1", "--master-port", str(_port()), os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "1",
-           "--warmup", "3", "--workload", "lap2048", "--no-sweep"]
+    env.pop("WORLD_SIZE", None)
+    if fault:
+        env["PEPP_FAULT_P2P_EXPORT"] = "1"
+    tail = [os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "1", "--warmup", "3", "--workload", "lap2048",
+            "--no-sweep"]
+    if launch == "torchrun":
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
+               "127.0.0.1", "--master-port", str(_port()), *tail]
+    else:
+        cmd = [sys.executable, *tail]
     out = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=900, cwd=ROOT)
     assert out.returncode == 0, out.stderr[-3000:]
     lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, out.stdout[-2000:]
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["steps"] == 1 and d["value"] > 0
-    # halo pushed by the fused boundary kernel into the peer's buffer (PEPP_X_P2P, CUDA IPC on one device)
-    assert d["config"]["exchange"].startswith("p2p")
+    if not fault:
+        # halo pushed by the fused boundary kernel into the peer's buffer (PEPP_X_P2P, CUDA IPC on one device)
+        assert d["run"]["exchange"].startswith("p2p") and d["run"]["p2p_fallback"] is None
+    else:
+        assert d["run"]["exchange"] == "halo" and "PEPP_E_CUDA" in d["run"]["p2p_fallback"], d["run"]
     # rank 0's block sends its last grid row: interior kernel + the fused tail/push kernel per SpMV
     assert d["plan"]["overlap"] == 1 and d["plan"]["overlap_head"] == 0 and d["plan"]["overlap_tail"] == 2048
     assert d["e2e"]["value"] > 0 and d["gpu_launches"] >= 200
     assert "launch_includes" in d["roofline"]
     assert d["cpu_baseline"] is None          # rank 0 at N = 1 only
+    assert d["configs"] is None               # the config 1-3 legs run at N = 1 only

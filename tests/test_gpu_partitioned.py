@@ -32,8 +32,28 @@ def _build_fake() -> str:
     return LIB
 
 
+def _one_sided_band(n, wrap):
+    """Row i: columns i, i+1, i+2 (mod n when `wrap`), integer values. Not
+    structurally symmetric: rank r reads only rank r+1's first rows, so its
+    send and receive peer sets differ (3 ranks with wrap: send to r-1,
+    receive from r+1; 2 ranks without wrap: rank 1 sends, rank 0 sends
+    nothing)."""
+    import gen
+    rp, cols, vals = [0], [], []
+    for i in range(n):
+        cs = sorted({(i + d) % n for d in range(3)} if wrap else {i + d for d in range(3) if i + d < n})
+        cols += cs
+        vals += [float((i + j) % 7 - 3) or 1.0 for j in range(len(cs))]
+        rp.append(len(cols))
+    return gen.CSR(n, n, np.array(rp, np.int64), np.array(cols, np.int32), np.array(vals), 0, n)
+
+
 def _matrix(name):
     import gen
+    if name == "cyclic":
+        return _one_sided_band(3000, True)
+    if name == "upper":
+        return _one_sided_band(3000, False)
     if name == "lap":
         return gen.laplacian2d(96)
     if name == "zipf":
@@ -245,18 +265,18 @@ def _worker_p2p(rank, world, lib, uid, name, K, outq, f32=False, real=False):
         outq.put((rank, {"error": repr(e) + traceback.format_exc()}))
 
 
-def _run_p2p(name, K=6, f32=False, real=False):
+def _run_p2p(name, K=6, f32=False, real=False, world=2):
     import torch.multiprocessing as mp
     lib = _build_fake()
-    uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_p2p_{int(f32)}{int(real)}".encode() + b"\0" * 128)[:128]
+    uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_p2p_{int(f32)}{int(real)}_{world}".encode() + b"\0" * 128)[:128]
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker_p2p, args=(r, 2, lib, uid, name, K, q, f32, real)) for r in range(2)]
+    procs = [ctx.Process(target=_worker_p2p, args=(r, world, lib, uid, name, K, q, f32, real)) for r in range(world)]
     for p in procs:
         p.start()
     out = {}
     try:
-        for _ in range(2):
+        for _ in range(world):
             r, res = q.get(timeout=300)
             out[r] = res
     finally:   # never leave a worker (and its GPU context) behind
@@ -265,9 +285,33 @@ def _run_p2p(name, K=6, f32=False, real=False):
             if p.is_alive():
                 p.kill()
                 p.join(10)
-    for r in range(2):
+    for r in range(world):
         assert "error" not in out[r], out[r]["error"]
     return out
+
+
+@pytest.mark.parametrize("name,world", [("cyclic", 3), ("upper", 2)])
+def test_p2p_fused_halo_nonsymmetric_peers(name, world):
+    """Send and receive peer sets differ (readiness must flow from
+    receiver to sender): 3 ranks on a one-sided cyclic band (rank r sends to
+    r-1 only and receives from r+1 only), and 2 ranks on a one-sided band
+    where rank 0 sends nothing (it computes its whole block and only
+    signals). NaN-initialised buffers, integer inputs: own rows + ghosts
+    bit-exact vs the oracle after every iteration, every call PEPP_X_P2P."""
+    import paper_conf_sc_dastgeerlk12_b200 as pepp
+    out = _run_p2p(name, world=world)
+    owners = {r: out[r]["own"] for r in range(world)}
+    for r in range(world):
+        assert out[r]["ok"], (r, out[r]["used"])
+        assert out[r]["used"] == [pepp.X_P2P], out[r]
+        gi, gv = out[r]["ghosts"]
+        for g, v in zip(gi, gv):
+            q = max(o for o in owners if owners[o][0] <= g)
+            o0, ov = owners[q]
+            assert v == ov[g - o0]
+    if name == "upper":
+        assert len(out[1]["ghosts"][0]) == 0 and len(out[0]["ghosts"][0]) > 0
+        assert out[0]["overlap"][0] == 0 and out[1]["overlap"][0] == 1   # rank 0: no split, it sends nothing
 
 
 @pytest.mark.parametrize("name,f32,real", [("lap", False, False), ("banded", False, False), ("lap", True, False),
