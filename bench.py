@@ -535,11 +535,13 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
     plan_ms = (time.perf_counter() - t_plan) * 1e3
     info = plan.info()
     flags = pepp.Y_NEXT_INPUT if iterated else pepp.Y_LOCAL
-    overlapped = bool(world > 1 and iterated and force is None and info["overlap"])
+    # N > 1, iterated: the exchange happens inside each call, as the plan's
+    # distribution choice (P', exchange — opts.dist_select) or its overlapped halo
+    overlapped = bool(world > 1 and iterated and force is None)
 
     stream = torch.cuda.Stream(device=dev)
     xs = torch.from_numpy(x0).to(dev)
-    p2p = overlapped and not args.no_p2p
+    p2p = overlapped and bool(info["overlap"]) and not args.no_p2p
     p2p_note = None
     bufs = None
     if p2p:
@@ -555,6 +557,7 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             p2p, p2p_note = False, f"p2p unavailable, NCCL halo used: {e}"[:300]
     if bufs is None:
         bufs = [torch.empty(R, dtype=tdt, device=dev) for _ in range(2)]
+    final_info = plan.info()   # after the P2P registration (its timing may change the distribution choice)
     flush = None if iterated or Z * 12 > 4 * (1 << 30) else torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     ev_pool = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(iters)]
@@ -786,8 +789,15 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             "warmup": args.warmup, "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
             "config": config_of(args, R, Z),
-            "run": {"exchange": ("p2p (fused boundary kernel, peer-memory stores)" if p2p
-                                 else pepp._capi.EXCHANGE_NAMES.get(info["exchange"], "?")),
+            "run": {"exchange": ("p2p (fused boundary kernel, peer-memory stores)"
+                                 if final_info["dist_exchange"] == pepp.X_P2P or (p2p and not final_info["dist_candidates"])
+                                 else pepp._capi.EXCHANGE_NAMES.get(final_info["dist_exchange"] if final_info["dist_candidates"]
+                                                                    else info["exchange"], "?")),
+                    "nparts": final_info["dist_nparts"] if final_info["dist_candidates"] else world,
+                    "distribution": ([{"nparts": a, "exchange": pepp._capi.EXCHANGE_NAMES.get(b, "?"),
+                                       "agreed_us": round(c, 2)} for a, b, c in plan.dist_stats()]
+                                     if final_info["dist_candidates"] else None),
+                    "dist_probe_ms": round(final_info["dist_probe_ms"], 1),
                     "p2p_fallback": p2p_note,
                     "variant": args.variant or "auto (history-based per call)",
                     "plan_ms": round(plan_ms, 1),
@@ -796,8 +806,8 @@ def run_ours(args, rank: int, world: int, local_rank: int) -> None:
             "hbm": {"achieved_gbs": round(gbs, 1), "frac_of_measured": round(gbs / (world * peak), 4),
                     "frac_of_8tbs": round(gbs / (world * 8000.0), 4), "algorithmic_bytes_per_spmv": alg_bytes_global},
             "roofline": dict(roofline_obj(kname, layout_bytes, local_alg, peak, peak_src, avg_kernel_s, args.workload, args.dtype),
-                             **({"launch_includes": "interior kernel + the fused boundary/push kernel (P2P halo)"
-                                 if p2p else "head + interior + tail kernels and the overlapped halo exchange"}
+                             **({"launch_includes": "the whole call: its kernels and its exchange, as the plan's "
+                                                    "distribution choice runs them (run.nparts / run.exchange)"}
                                 if overlapped else {})),
             "e2e": {"value": round(e2e_val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": A.ncols * esz,
                     "d2h_bytes_per_step": A.nrows * esz, "spmv_per_step": e2e_iters,

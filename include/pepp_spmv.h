@@ -63,7 +63,7 @@
 extern "C" {
 #endif
 
-#define PEPP_ABI_VERSION 6
+#define PEPP_ABI_VERSION 7
 
 typedef enum {
     PEPP_OK = 0,
@@ -196,6 +196,24 @@ typedef struct {
                                  (constant-coefficient stencils). Lossless: the same products and
                                  sums in the same order (bit-identical y); only the bytes read
                                  change. 0 = every stored slot's value is streamed. */
+    int32_t dist_select;      /* nranks > 1, use_history = 1: 1 (default) = the partition count P and the
+                                 exchange are timed choices too (§8(a) a4; the runtime picks "which
+                                 implementation/device to use by considering previous historical
+                                 execution information as well as ... load balance, data locality and
+                                 potential data-transfer cost", §V-D P@38827). Candidates: P' in the
+                                 powers of two dividing nranks (the call runs on ranks 0..P'-1, each on
+                                 the union of nranks/P' consecutive row blocks, shipped to it over NCCL
+                                 at plan time) x exchange in {halo, allgather} (only opts.exchange when
+                                 it is not AUTO), plus the fused peer-memory push once
+                                 pepp_spmv_p2p_buffers registers buffers. pepp_spmv_plan (and
+                                 pepp_spmv_p2p_buffers) time each candidate with plan-owned scratch
+                                 vectors — its kernels first calibrated, then min_samples timed
+                                 calls — and all ranks agree on the max-over-ranks means (one NCCL
+                                 max-reduce): every later PEPP_Y_NEXT_INPUT call runs the argmin
+                                 (PEPP_Y_REPLICATED: the argmin among allgather candidates;
+                                 PEPP_Y_LOCAL: always P' = nranks). A loaded history_path with
+                                 min_samples records of every candidate on every rank skips the
+                                 timing. 0 = P' = nranks, exchange by the plan's footprint rule. */
 } pepp_spmv_opts_t;
 
 /* Selection result. `candidate` indexes pepp_spmv_candidates(). The plan's
@@ -255,6 +273,13 @@ typedef struct pepp_plan_info_s {
                                  part of the SELL work = (nnz/32 + 4 x chunks) / warps of one
                                  resident wave; rows up to 1024 long above it: one warp each,
                                  longer: 4096-entry segments */
+    int32_t dist_candidates;  /* distribution candidates (P', exchange) timed (0 = none: nranks == 1 or
+                                 dist_select = 0) — pepp_spmv_dist_stats lists them */
+    int32_t dist_nparts;      /* chosen P' for PEPP_Y_NEXT_INPUT calls (nranks when not selected) */
+    int32_t dist_exchange;    /* chosen exchange for PEPP_Y_NEXT_INPUT calls (PEPP_X_P2P when the
+                                 registered buffers' fused push won) */
+    int32_t dist_repl_nparts; /* chosen P' for PEPP_Y_REPLICATED calls (allgather) */
+    double dist_probe_ms;     /* wall time the plan-time timing of the candidates took */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */
@@ -291,8 +316,10 @@ pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_choice_t* out);
       PEPP_Y_REPLICATED the exchange then fills ghost / all entries from the
       other ranks (NCCL, same stream). Entries not covered by `flags` are
       left untouched.
-   force: NULL = automatic selection; else force->variant/param (and
-      force->exchange when partitioned) select the implementation.
+   force: NULL = automatic selection; else force->variant/param (and, when
+      partitioned, force->exchange and force->nparts: P' > 0 and < nranks runs
+      the call on ranks 0..P'-1 as a distribution candidate does; nparts <= 0
+      or == nranks means this rank's own block) select the implementation.
    used: optional; receives the choice that ran (launches = this library's
       kernels the call enqueued).
    Some plans also use their own second stream inside a call (the genlist
@@ -358,6 +385,13 @@ pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* y, int flags, void* 
    PEPP_E_NCCL. Errors: PEPP_E_INVALID, PEPP_E_CUDA (IPC unavailable),
    PEPP_E_NCCL, PEPP_E_NOMEM. */
 pepp_status_t pepp_spmv_p2p_buffers(pepp_spmv_plan_t* p, int32_t nbuf, void** bufs);
+
+/* Distribution candidates of a partitioned plan (opts.dist_select): for
+   each i < *n (up to cap): nparts[i] = P', exchange[i] = pepp_exchange_t,
+   agreed_us[i] = the max-over-ranks mean time of one PEPP_Y_NEXT_INPUT call
+   the ranks agreed on (0 if never timed). Host only. */
+pepp_status_t pepp_spmv_dist_stats(const pepp_spmv_plan_t* p, int32_t cap, int32_t* nparts, int32_t* exchange,
+                                   double* agreed_us, int32_t* n);
 
 /* Host-buffer entry point (the paper's measurement setting, where operand
    transfers are part of the call: Fig. 5 "communication overhead of copying
@@ -530,6 +564,18 @@ pepp_status_t pepp_history_stats(const pepp_history* h, uint64_t key, int32_t ca
 pepp_status_t pepp_history_select(const pepp_history* h, uint64_t key, int32_t ncand,
                                   const uint8_t* eligible, int32_t min_samples,
                                   int32_t* cand, int32_t* calibrating, double* predicted_us);
+/* Distribution choice policy (§8(a) a4, P and exchange; host only, the
+   rule pepp_spmv_plan applies after its NCCL max-reduce): means is
+   [nranks][nd] row-major, each rank's own measured mean time per candidate;
+   a partitioned call takes as long as its slowest rank, so candidate d's
+   agreed time is max over ranks of means[r][d]; *choice = argmin of the
+   agreed times over eligible candidates (eligible NULL = all; a candidate
+   with agreed time 0 or Inf is skipped), ties within 1 % going to the lower
+   index (reading A10). agreed: optional [nd] output. PEPP_E_INVALID on NULL
+   or negative / NaN input, PEPP_E_STATE if nothing is eligible. */
+pepp_status_t pepp_dist_choose(int32_t nranks, int32_t nd, const double* means, const uint8_t* eligible,
+                               int32_t* choice, double* agreed);
+
 /* Cold-start prior (static composition from recorded runs, P@10069, P@10489):
    the nearest context key to `key` (L1 distance over the bucket fields of
    pepp_context_key; same rank count) that has samples for some of the
@@ -552,6 +598,7 @@ pepp_status_t pepp_history_load(pepp_history* h, const char* path);
    count and instance. */
 #define PEPP_KEY_F32      0x1
 #define PEPP_KEY_COMPRESS 0x2
+#define PEPP_KEY_DIST     0x4   /* the distribution (P', exchange) records of a partitioned plan */
 uint64_t pepp_context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts, int32_t instance);
 
 /* NCCL bootstrap helper: write a fresh 128-byte ncclUniqueId into id_out

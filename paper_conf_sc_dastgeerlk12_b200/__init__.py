@@ -23,7 +23,7 @@ from ._capi import (ACCESS_READ, ACCESS_READWRITE, ACCESS_WRITE, DEVICE_SIMULATE
                     X_HALO, X_NONE, X_P2P, Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, VARIANT_NAMES)
 
 __all__ = ["Plan", "Choice", "History", "Vector", "ACCESS_READ", "ACCESS_WRITE", "ACCESS_READWRITE",
-           "DEVICE_SIMULATED", "partition_rows", "halo_ghosts", "context_key", "nccl_unique_id",
+           "DEVICE_SIMULATED", "partition_rows", "halo_ghosts", "context_key", "nccl_unique_id", "dist_choose",
            "lib_path", "PeppError", "V_CSR_VECTOR", "V_MERGE_PATH", "V_SELL", "V_CSR_STREAM", "X_AUTO", "X_NONE",
            "X_ALLGATHER", "X_HALO", "X_P2P", "Y_LOCAL", "Y_NEXT_INPUT", "Y_REPLICATED", "EXEC_NO_TIMING",
            "VARIANT_NAMES"]
@@ -36,7 +36,7 @@ class Choice:
     variant: int
     param: int = 0
     exchange: int = X_AUTO
-    nparts: int = 1
+    nparts: int = 0          # force: 0 = this rank's own block (P' = nranks); P' < nranks = a distribution
     calibrating: bool = False
     candidate: int = -1
     predicted_us: float = 0.0
@@ -97,7 +97,7 @@ class Plan:
                  nranks: int = 1, rank: int = 0, row_bounds: Optional[Sequence[int]] = None,
                  nccl_unique_id: Optional[bytes] = None, exchange: int = X_AUTO,
                  history_path: Optional[str] = None, prune: bool = True, overlap: bool = True,
-                 predict=None, compress_values: bool = True):
+                 predict=None, compress_values: bool = True, dist_select: bool = True):
         L = C.lib()
         self._h = ctypes.c_void_p()
         on_dev = not isinstance(row_ptr, np.ndarray)
@@ -138,6 +138,7 @@ class Plan:
         o.prune = 1 if prune else 0
         o.overlap = 1 if overlap else 0
         o.compress_values = 1 if compress_values else 0
+        o.dist_select = 1 if dist_select else 0
         cb = None
         if predict is not None:
             # predict(context: dict, variant: int, param: int) -> µs (<= 0: no prediction);
@@ -282,6 +283,16 @@ class Plan:
         i = C.INFO_T()
         C.check(C.lib().pepp_spmv_plan_info(self._h, ctypes.byref(i)), "pepp_spmv_plan_info")
         return i.as_dict()
+
+    def dist_stats(self) -> list[tuple[int, int, float]]:
+        """(P', exchange, agreed mean µs) per distribution candidate (opts.dist_select)."""
+        n = ctypes.c_int32()
+        C.check(C.lib().pepp_spmv_dist_stats(self._h, 0, None, None, None, ctypes.byref(n)), "pepp_spmv_dist_stats")
+        k = max(1, n.value)
+        pa, ex, us = np.zeros(k, np.int32), np.zeros(k, np.int32), np.zeros(k, np.float64)
+        C.check(C.lib().pepp_spmv_dist_stats(self._h, k, pa.ctypes.data, ex.ctypes.data, us.ctypes.data,
+                                             ctypes.byref(n)), "pepp_spmv_dist_stats")
+        return [(int(pa[i]), int(ex[i]), float(us[i])) for i in range(n.value)]
 
     def flush_history(self) -> None:
         C.check(C.lib().pepp_spmv_flush_history(self._h), "pepp_spmv_flush_history")
@@ -486,6 +497,20 @@ def halo_ghosts(col: np.ndarray, nranks: int, rank: int, row_bounds: Sequence[in
                                      counts.ctypes.data, g.ctypes.data, g.size, ctypes.byref(total)),
             "pepp_halo_ghosts")
     return counts, g[:total.value]
+
+
+def dist_choose(means, eligible=None) -> tuple[int, np.ndarray]:
+    """pepp_dist_choose: means [nranks][nd] (each rank's own mean µs per
+    distribution candidate) -> (argmin of the max-over-ranks means, agreed)."""
+    m = np.ascontiguousarray(means, dtype=np.float64)
+    if m.ndim != 2:
+        raise ValueError("means must be [nranks][nd]")
+    e = None if eligible is None else np.ascontiguousarray([1 if v else 0 for v in eligible], dtype=np.uint8)
+    ag = np.zeros(m.shape[1])
+    c = ctypes.c_int32()
+    C.check(C.lib().pepp_dist_choose(m.shape[0], m.shape[1], m.ctypes.data, e.ctypes.data if e is not None else None,
+                                     ctypes.byref(c), ag.ctypes.data), "pepp_dist_choose")
+    return c.value, ag
 
 
 def context_key(nrows: int, ncols: int, nnz: int, cv: float, nparts: int = 1, *, f32: bool = False,

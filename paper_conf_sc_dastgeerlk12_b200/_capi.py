@@ -18,7 +18,7 @@ Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, EXEC_NO_TIMING = 0x0, 0x1, 0x2, 0x10
 ACCESS_READ, ACCESS_WRITE, ACCESS_READWRITE = 1, 2, 3
 VALUE_F64, VALUE_F32 = 0, 1
 DEVICE_SIMULATED = -2
-KEY_F32, KEY_COMPRESS = 0x1, 0x2
+KEY_F32, KEY_COMPRESS, KEY_DIST = 0x1, 0x2, 0x4
 VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell", V_CSR_STREAM: "csr_stream"}
 EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_P2P: "p2p", X_AUTO: "auto"}
 
@@ -40,7 +40,9 @@ class INFO_T(ctypes.Structure):
                 ("prior_key", c_u64), ("sell_stencil_frac", c_f64),
                 ("overlap", c_i32), ("overlap_head", c_i64), ("overlap_tail", c_i64), ("predicted", c_i32),
                 ("sell_constval_frac", c_f64), ("p2p_buffers", c_i32),
-                ("sell_long_rows", c_i64), ("sell_cap", c_i64)]
+                ("sell_long_rows", c_i64), ("sell_cap", c_i64), ("dist_candidates", c_i32),
+                ("dist_nparts", c_i32), ("dist_exchange", c_i32), ("dist_repl_nparts", c_i32),
+                ("dist_probe_ms", c_f64)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -56,7 +58,7 @@ class OPTS_T(ctypes.Structure):
                 ("rank", c_i32), ("row_bounds", c_vp), ("nccl_comm", c_vp), ("nccl_unique_id", c_vp),
                 ("exchange", c_i32), ("history_path", ctypes.c_char_p), ("prune", c_i32),
                 ("overlap", c_i32), ("predict", PREDICT_FN), ("predict_user", c_vp),
-                ("compress_values", c_i32)]
+                ("compress_values", c_i32), ("dist_select", c_i32)]
 
 
 class CHOICE_T(ctypes.Structure):
@@ -86,6 +88,8 @@ SIGNATURES = {
     "pepp_spmv_plan_info": (c_i32, [c_vp, ctypes.POINTER(INFO_T)]),
     "pepp_spmv_candidates": (c_i32, [c_vp, ctypes.POINTER(CHOICE_T), c_i32, ctypes.POINTER(c_i32)]),
     "pepp_spmv_flush_history": (c_i32, [c_vp]),
+    "pepp_spmv_dist_stats": (c_i32, [c_vp, c_i32, c_vp, c_vp, c_vp, ctypes.POINTER(c_i32)]),
+    "pepp_dist_choose": (c_i32, [c_i32, c_i32, c_vp, c_vp, ctypes.POINTER(c_i32), c_vp]),
     "pepp_spmv_history_stats": (c_i32, [c_vp, c_i32, ctypes.POINTER(c_i64), ctypes.POINTER(c_f64), ctypes.POINTER(c_f64)]),
     "pepp_spmv_graph_create": (c_i32, [c_vp, c_vp, c_vp, c_vp, c_i32, c_i32, ctypes.c_int, c_vp, ctypes.POINTER(c_vp)]),
     "pepp_spmv_graph_launch": (c_i32, [c_vp, c_vp]),
@@ -131,7 +135,7 @@ class PeppError(RuntimeError):
         super().__init__(f"{where}: {status_str(status)} ({status})" + (f": {detail}" if detail else ""))
 
 
-ABI_VERSION = 6   # PEPP_ABI_VERSION of include/pepp_spmv.h
+ABI_VERSION = 7   # PEPP_ABI_VERSION of include/pepp_spmv.h
 
 
 def lib() -> ctypes.CDLL:

@@ -62,6 +62,7 @@ extern "C" PEPP_API void pepp_spmv_opts_default(pepp_spmv_opts_t* o) {
     o->prune = 1;
     o->overlap = 1;
     o->compress_values = 1;
+    o->dist_select = 1;
 }
 
 // ---------------------------------------------------------------- partition
@@ -243,6 +244,17 @@ bool history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t
     return true;
 }
 
+int32_t dist_argmin(int32_t nd, const double* agreed, const uint8_t* eligible) {
+    // argmin of the agreed means, ties within 1 % -> lower index (reading A10)
+    int32_t c = -1;
+    double bt = 0.0;
+    for (int32_t d = 0; d < nd; ++d) {
+        if ((eligible && !eligible[d]) || !(agreed[d] > 0.0) || std::isinf(agreed[d])) continue;
+        if (c < 0 || agreed[d] < bt * 0.99) { c = d; bt = agreed[d]; }
+    }
+    return c;
+}
+
 uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts, int32_t instance) {
     // bucketed context instance: half-octave buckets of rows / cols / nnz,
     // quarter buckets of the row-length CV (capped), and the partition count.
@@ -297,6 +309,24 @@ extern "C" PEPP_API pepp_status_t pepp_history_select(const pepp_history* h, uin
     if (!any) return PEPP_E_INVALID;
     *cand = pepp::history_pick(h, key, ncand, eligible, min_samples < 1 ? 1 : min_samples, calibrating, predicted_us);
     return PEPP_OK;
+}
+
+extern "C" PEPP_API pepp_status_t pepp_dist_choose(int32_t nranks, int32_t nd, const double* means,
+                                                  const uint8_t* eligible, int32_t* choice, double* agreed) {
+    if (nranks < 1 || nd < 1 || !means || !choice) return PEPP_E_INVALID;
+    std::vector<double> ag(nd, 0.0);
+    for (int32_t d = 0; d < nd; ++d) {
+        double m = 0.0;
+        for (int32_t r = 0; r < nranks; ++r) {
+            const double v = means[(int64_t)r * nd + d];
+            if (!(v >= 0.0)) return PEPP_E_INVALID;       // NaN or negative
+            m = std::max(m, v);
+        }
+        ag[d] = m;
+    }
+    if (agreed) std::copy(ag.begin(), ag.end(), agreed);
+    *choice = pepp::dist_argmin(nd, ag.data(), eligible);
+    return *choice < 0 ? PEPP_E_STATE : PEPP_OK;
 }
 
 extern "C" PEPP_API pepp_status_t pepp_history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t* ids,

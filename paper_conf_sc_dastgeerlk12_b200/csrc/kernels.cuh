@@ -1536,6 +1536,13 @@ __global__ void gather_kernel(int64_t n, const int* __restrict__ idx, const T* _
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         dst[i] = src[idx[i]];
 }
+// union row pointer of shipped row blocks (distribution candidates): a
+// block's narrowed row pointer (local offsets + its alignment pad) widened
+// and moved to the union's nonzero offset: out[i] = rp[i] + delta
+__global__ void rowptr_widen_kernel(int64_t n, const int* __restrict__ rp, int64_t delta, int64_t* __restrict__ out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = (int64_t)rp[i] + delta;
+}
 template <typename T>
 __global__ void scatter_kernel(int64_t n, const int* __restrict__ idx, const T* __restrict__ src,
                                T* __restrict__ dst) {

@@ -44,6 +44,8 @@ constexpr int32_t kRefineRounds = 3;
 bool history_contender(const Welford* w, double best_mean);
 int32_t history_pick(const pepp_history* h, uint64_t key, int32_t ncand, const uint8_t* eligible,
                      int32_t min_samples, int32_t* calibrating, double* predicted_us);
+// distribution choice (P and exchange): argmin of the agreed (max over ranks) means
+int32_t dist_argmin(int32_t nd, const double* agreed, const uint8_t* eligible);
 uint64_t context_key(int64_t nrows, int64_t ncols, int64_t nnz, double cv, int32_t nparts, int32_t instance);
 bool history_prior(const pepp_history* h, uint64_t key, int32_t n, const int32_t* ids, double* prior,
                    uint64_t* from_key);

@@ -16,6 +16,7 @@
 #include <cub/device/device_scan.cuh>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -79,6 +80,22 @@ struct PeerXfer {            // halo traffic with one peer
     int64_t contig_start;    // >= 0: the entries are y[contig_start, contig_start+count)
     int* d_idx = nullptr;    // else: global indices into y (device)
     void* d_buf = nullptr;   // pack / unpack buffer (value type)
+};
+
+// Distribution candidates (opts.dist_select, §8(a) a4: P and exchange are
+// timed choices). P' < nranks: ranks 0..P'-1 each compute the union of
+// nranks/P' consecutive row blocks (shipped to them at plan time).
+struct DistPart {
+    int32_t parts = 0;
+    std::vector<int64_t> bounds;             // [parts + 1] global row boundaries under P'
+    pepp_spmv_plan_t* plan = nullptr;        // this rank's block under P' (rank < P'), else none
+    std::vector<PeerXfer> recv_x, send_x;    // after a P' call: own rows + own ghosts from their P' owners
+    std::vector<PeerXfer> recv_g, send_g;    // after a P' = nranks call: what a P' call reads (its block +
+                                             // its ghosts) beyond own rows + own ghosts, from their owners
+};
+struct DistCand {
+    int32_t parts;                           // P'
+    int32_t ex;                              // PEPP_X_HALO / PEPP_X_ALLGATHER
 };
 
 }  // namespace
@@ -179,6 +196,7 @@ struct pepp_spmv_plan_s {
     int ring_head = 0;   // oldest pending
     int ring_count = 0;
     std::vector<int32_t> pending;   // timed calls in flight per candidate
+    std::vector<uint8_t> warmed;    // per candidate: its warm-up call (first timed call, not recorded) is done
     std::vector<int32_t> uids;      // stable candidate identity in the history: variant << 20 | param
     std::vector<int64_t> cand_bytes;// per candidate: bytes its kernels move per call (layout as stored + x + y)
     std::vector<double> prior;      // cold-start means from the nearest recorded context (-1 = none)
@@ -225,6 +243,16 @@ struct pepp_spmv_plan_s {
     int p2p_grid = 1;
     unsigned long long p2p_timeout_ns = 20ull * 1000 * 1000 * 1000;
 
+    // distribution choice (opts.dist_select)
+    std::vector<DistPart> dparts;                // P' < nranks
+    std::vector<DistCand> dcands;                // (P', exchange) candidates, P' = nranks first
+    std::vector<double> dist_agreed;             // agreed (max over ranks) mean µs per candidate
+    int dist_next = -1, dist_repl = -1;          // chosen for PEPP_Y_NEXT_INPUT / PEPP_Y_REPLICATED calls
+    bool p2p_use = true;                         // registered buffers: the fused push won (or no choice made)
+    double p2p_agreed = 0.0;
+    uint64_t dist_key = 0;
+    int64_t global_nnz = 0;
+
     // plan-owned x / y for pepp_spmv_exec_host (allocated on first use)
     void* d_hx = nullptr;
     void* d_hy = nullptr;
@@ -246,6 +274,10 @@ namespace {
             return PEPP_E_CUDA;                               \
         }                                                     \
     } while (0)
+
+double now_ms() {
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
 
 // Every entry point works on the plan's device and leaves the caller's
 // current device as it found it.
@@ -307,6 +339,11 @@ void free_plan(pepp_spmv_plan_t* p) {
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
+    for (auto& dp : p->dparts) {
+        for (auto* v : {&dp.recv_x, &dp.send_x, &dp.recv_g, &dp.send_g})
+            for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
+        free_plan(dp.plan);
+    }
     for (auto& r : p->ring) { if (r.start) cudaEventDestroy(r.start); if (r.stop) cudaEventDestroy(r.stop); }
     for (void* m : p->p2p_opened) cudaIpcCloseMemHandle(m);
     for (void* b : p->p2p_buf) if (b) cudaFree(b);
@@ -1037,8 +1074,15 @@ void harvest(pepp_spmv_plan_t* p, bool block) {
         cudaError_t q = cudaEventQuery(r.stop);
         if (q == cudaErrorNotReady) { (void)cudaGetLastError(); break; }
         float ms = 0.f;
-        if (q == cudaSuccess && cudaEventElapsedTime(&ms, r.start, r.stop) == cudaSuccess)
-            pepp::history_add(p->hist, p->key, p->uids[r.cand], (double)ms * 1000.0);
+        if (q == cudaSuccess && cudaEventElapsedTime(&ms, r.start, r.stop) == cudaSuccess) {
+            // a candidate's first timed call in this plan is a warm-up, not a
+            // sample: it can carry one-off costs (lazy module load of its
+            // kernels, the SM clock ramping up from idle, cold TLBs) that, in
+            // a 3-sample mean, once pushed the best candidate past a 1.7x
+            // slower one on config 4 (round-2 bench, sell[1] vs csr_vector[2])
+            if (r.cand >= 0 && r.cand < (int)p->warmed.size() && !p->warmed[r.cand]) p->warmed[r.cand] = 1;
+            else pepp::history_add(p->hist, p->key, p->uids[r.cand], (double)ms * 1000.0);
+        }
         (void)cudaGetLastError();
         r.pending = false;
         if (r.cand >= 0 && r.cand < (int)p->pending.size()) --p->pending[r.cand];
@@ -1190,13 +1234,15 @@ pepp_status_t nccl_ok(const pepp_spmv_plan_t* p, int r) { (void)p; return r == 0
 
 int nccl_value_type(const pepp_spmv_plan_t* p) { return p->vt == PEPP_VALUE_F32 ? pepp::NCCL_FLOAT32 : pepp::NCCL_FLOAT64; }
 
-pepp_status_t exchange_allgather(pepp_spmv_plan_t* p, void* y, cudaStream_t st) {
+// grouped broadcasts: block j = y[bounds[j], bounds[j+1]) from rank j to
+// every rank of the plan's communicator (allgatherv of nb blocks, nb <= ranks)
+pepp_status_t exchange_blocks(pepp_spmv_plan_t* p, const int64_t* bounds, int nb, void* y, cudaStream_t st) {
     PEPP_NVTX("pepp exchange allgatherv");
     const Nccl* n = p->nccl;
     char* yb = (char*)y;
     if (nccl_ok(p, n->GroupStart())) return PEPP_E_NCCL;
-    for (int r = 0; r < p->opts.nranks; ++r) {
-        const int64_t b = p->row_bounds[r], cnt = p->row_bounds[r + 1] - b;
+    for (int r = 0; r < nb; ++r) {
+        const int64_t b = bounds[r], cnt = bounds[r + 1] - b;
         if (cnt == 0) continue;
         char* at = yb + b * (int64_t)p->esz;
         if (n->Broadcast(at, at, (size_t)cnt, nccl_value_type(p), r, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
@@ -1204,9 +1250,13 @@ pepp_status_t exchange_allgather(pepp_spmv_plan_t* p, void* y, cudaStream_t st) 
     return nccl_ok(p, n->GroupEnd());
 }
 
+pepp_status_t exchange_allgather(pepp_spmv_plan_t* p, void* y, cudaStream_t st) {
+    return exchange_blocks(p, p->row_bounds.data(), p->opts.nranks, y, st);
+}
+
 template <typename T>
-void pack_unpack(pepp_spmv_plan_t* p, T* y, bool pack, cudaStream_t st) {
-    for (auto& t : pack ? p->send_x : p->recv_x) {
+void pack_unpack(std::vector<PeerXfer>& lst, T* y, bool pack, cudaStream_t st) {
+    for (auto& t : lst) {
         if (t.contig_start >= 0 || t.count == 0) continue;
         const int g = (int)std::min<int64_t>(1024, (t.count + 255) / 256);
         if (pack) pepp::k::gather_kernel<T><<<g, 256, 0, st>>>(t.count, t.d_idx, y, (T*)t.d_buf);
@@ -1214,28 +1264,35 @@ void pack_unpack(pepp_spmv_plan_t* p, T* y, bool pack, cudaStream_t st) {
     }
 }
 
-pepp_status_t exchange_halo(pepp_spmv_plan_t* p, void* y, cudaStream_t st) {
-    PEPP_NVTX("pepp exchange halo");
+// point-to-point transfer lists (halo ghosts, or a distribution's scatter):
+// pack scattered send entries, grouped send/recv, unpack scattered receives
+pepp_status_t exchange_xfer(pepp_spmv_plan_t* p, std::vector<PeerXfer>& recv, std::vector<PeerXfer>& send, void* y,
+                            cudaStream_t st) {
     const Nccl* n = p->nccl;
     char* yb = (char*)y;
     const int64_t es = (int64_t)p->esz;
-    if (p->vt == PEPP_VALUE_F32) pack_unpack<float>(p, (float*)y, true, st);
-    else pack_unpack<double>(p, (double*)y, true, st);
+    if (p->vt == PEPP_VALUE_F32) pack_unpack<float>(send, (float*)y, true, st);
+    else pack_unpack<double>(send, (double*)y, true, st);
     if (n->GroupStart()) return PEPP_E_NCCL;
-    for (auto& t : p->send_x) {
+    for (auto& t : send) {
         if (!t.count) continue;
         const void* src = t.contig_start >= 0 ? (const void*)(yb + t.contig_start * es) : t.d_buf;
         if (n->Send(src, (size_t)t.count, nccl_value_type(p), t.peer, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
     }
-    for (auto& t : p->recv_x) {
+    for (auto& t : recv) {
         if (!t.count) continue;
         void* dst = t.contig_start >= 0 ? (void*)(yb + t.contig_start * es) : t.d_buf;
         if (n->Recv(dst, (size_t)t.count, nccl_value_type(p), t.peer, p->comm, st)) { n->GroupEnd(); return PEPP_E_NCCL; }
     }
     if (n->GroupEnd()) return PEPP_E_NCCL;
-    if (p->vt == PEPP_VALUE_F32) pack_unpack<float>(p, (float*)y, false, st);
-    else pack_unpack<double>(p, (double*)y, false, st);
+    if (p->vt == PEPP_VALUE_F32) pack_unpack<float>(recv, (float*)y, false, st);
+    else pack_unpack<double>(recv, (double*)y, false, st);
     return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
+}
+
+pepp_status_t exchange_halo(pepp_spmv_plan_t* p, void* y, cudaStream_t st) {
+    PEPP_NVTX("pepp exchange halo");
+    return exchange_xfer(p, p->recv_x, p->send_x, y, st);
 }
 
 // plan-time halo setup: ghosts (what I receive) from my columns; what I send
@@ -1319,6 +1376,85 @@ pepp_status_t setup_halo(pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts
     p->info.halo_recv = tr;
     p->info.halo_send = ts;
     return PEPP_OK;
+}
+
+// Transfer lists for `needed` (sorted distinct global rows this rank must
+// hold after a call) whose owners are the blocks [bounds[q], bounds[q+1]),
+// q < nb: one count and one index exchange over the plan's communicator
+// (every rank takes part, also ranks that need nothing), as in setup_halo.
+pepp_status_t setup_xfer(pepp_spmv_plan_t* p, const std::vector<int32_t>& needed, const std::vector<int64_t>& bounds,
+                         std::vector<PeerXfer>& recv, std::vector<PeerXfer>& send, cudaStream_t st) {
+    const int P = p->opts.nranks, me = p->opts.rank;
+    std::vector<int64_t> rcount(P, 0), scount(P, 0);
+    std::vector<std::vector<int32_t>> rlist(P);
+    for (int32_t c : needed) {
+        const int q = (int)(std::upper_bound(bounds.begin(), bounds.end(), (int64_t)c) - bounds.begin()) - 1;
+        if (q >= 0 && q < P && q != me) rlist[q].push_back(c);
+    }
+    for (int q = 0; q < P; ++q) rcount[q] = (int64_t)rlist[q].size();
+    DevTmp<int64_t> d_rc, d_sc;
+    PEPP_CUDA_TRY(d_rc.alloc(P));
+    PEPP_CUDA_TRY(d_sc.alloc(P));
+    PEPP_CUDA_TRY(cudaMemcpy(d_rc.p, rcount.data(), sizeof(int64_t) * P, cudaMemcpyHostToDevice));
+    PEPP_CUDA_TRY(cudaMemset(d_sc.p, 0, sizeof(int64_t) * P));
+    const Nccl* n = p->nccl;
+    if (n->GroupStart()) return PEPP_E_NCCL;
+    for (int q = 0; q < P; ++q) {
+        if (q == me) continue;
+        n->Send(d_rc.p + q, 1, pepp::NCCL_INT64, q, p->comm, st);
+        n->Recv(d_sc.p + q, 1, pepp::NCCL_INT64, q, p->comm, st);
+    }
+    if (n->GroupEnd()) return PEPP_E_NCCL;
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    PEPP_CUDA_TRY(cudaMemcpy(scount.data(), d_sc.p, sizeof(int64_t) * P, cudaMemcpyDeviceToHost));
+    scount[me] = 0;
+    std::vector<DevTmp<int>> d_r(P), d_s(P);
+    for (int q = 0; q < P; ++q) {
+        if (rcount[q]) {
+            PEPP_CUDA_TRY(d_r[q].alloc(rcount[q]));
+            PEPP_CUDA_TRY(cudaMemcpy(d_r[q].p, rlist[q].data(), sizeof(int) * rcount[q], cudaMemcpyHostToDevice));
+        }
+        if (scount[q]) PEPP_CUDA_TRY(d_s[q].alloc(scount[q]));
+    }
+    if (n->GroupStart()) return PEPP_E_NCCL;
+    for (int q = 0; q < P; ++q) {
+        if (rcount[q]) n->Send(d_r[q].p, (size_t)rcount[q], pepp::NCCL_INT32, q, p->comm, st);
+        if (scount[q]) n->Recv(d_s[q].p, (size_t)scount[q], pepp::NCCL_INT32, q, p->comm, st);
+    }
+    if (n->GroupEnd()) return PEPP_E_NCCL;
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    auto make = [&](int q, const std::vector<int32_t>& lst, DevTmp<int>& d_list, std::vector<PeerXfer>& out) -> pepp_status_t {
+        PeerXfer t;
+        t.peer = q;
+        t.count = (int64_t)lst.size();
+        const bool contig = !lst.empty() && (int64_t)lst.back() - lst.front() + 1 == t.count;
+        t.contig_start = contig ? lst.front() : -1;
+        if (!contig && t.count) {
+            DevTmp<double> buf;   // 8-byte slots hold either value type
+            PEPP_CUDA_TRY(buf.alloc(t.count));
+            t.d_idx = d_list.release();
+            t.d_buf = buf.release();
+        }
+        out.push_back(t);
+        return PEPP_OK;
+    };
+    for (int q = 0; q < P; ++q) {
+        if (rcount[q]) { pepp_status_t s = make(q, rlist[q], d_r[q], recv); if (s) return s; }
+        if (scount[q]) {
+            std::vector<int32_t> sl(scount[q]);
+            PEPP_CUDA_TRY(cudaMemcpy(sl.data(), d_s[q].p, sizeof(int) * scount[q], cudaMemcpyDeviceToHost));
+            pepp_status_t s = make(q, sl, d_s[q], send);
+            if (s) return s;
+        }
+    }
+    return PEPP_OK;
+}
+
+int xfer_kernels(const std::vector<PeerXfer>& recv, const std::vector<PeerXfer>& send) {
+    int n = 0;
+    for (const auto* v : {&send, &recv})
+        for (const auto& t : *v) n += t.contig_start < 0 && t.count > 0;
+    return n;
 }
 
 pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spmv_plan_t* p);
@@ -1416,6 +1552,230 @@ pepp_status_t nccl_allmax(pepp_spmv_plan_t* p, cudaStream_t st, int64_t* v) {
 pepp_status_t nccl_barrier(pepp_spmv_plan_t* p, cudaStream_t st) {
     int64_t v = 0;
     return nccl_allmax(p, st, &v);
+}
+
+// elementwise max over ranks of a host vector of doubles (agreement on times)
+pepp_status_t nccl_allmax_f64(pepp_spmv_plan_t* p, cudaStream_t st, std::vector<double>& v) {
+    if (v.empty()) return PEPP_OK;
+    DevTmp<double> d;
+    PEPP_CUDA_TRY(d.alloc(v.size()));
+    PEPP_CUDA_TRY(cudaMemcpyAsync(d.p, v.data(), sizeof(double) * v.size(), cudaMemcpyHostToDevice, st));
+    if (p->nccl->AllReduce(d.p, d.p, v.size(), pepp::NCCL_FLOAT64, pepp::NCCL_OP_MAX, p->comm, st)) return PEPP_E_NCCL;
+    PEPP_CUDA_TRY(cudaMemcpyAsync(v.data(), d.p, sizeof(double) * v.size(), cudaMemcpyDeviceToHost, st));
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    return PEPP_OK;
+}
+
+// every rank's value of v (grouped broadcasts of one int64 per rank)
+pepp_status_t nccl_allgather_i64(pepp_spmv_plan_t* p, cudaStream_t st, int64_t v, std::vector<int64_t>& all) {
+    const int P = p->opts.nranks, me = p->opts.rank;
+    all.assign(P, 0);
+    all[me] = v;
+    DevTmp<int64_t> d;
+    PEPP_CUDA_TRY(d.alloc(P));
+    PEPP_CUDA_TRY(cudaMemcpyAsync(d.p, all.data(), sizeof(int64_t) * P, cudaMemcpyHostToDevice, st));
+    if (p->nccl->GroupStart()) return PEPP_E_NCCL;
+    for (int r = 0; r < P; ++r)
+        if (p->nccl->Broadcast(d.p + r, d.p + r, 1, pepp::NCCL_INT64, r, p->comm, st)) { p->nccl->GroupEnd(); return PEPP_E_NCCL; }
+    if (p->nccl->GroupEnd()) return PEPP_E_NCCL;
+    PEPP_CUDA_TRY(cudaMemcpyAsync(all.data(), d.p, sizeof(int64_t) * P, cudaMemcpyDeviceToHost, st));
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    return PEPP_OK;
+}
+
+pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spmv_plan_t* p);
+
+// Distribution candidates P' < nranks (opts.dist_select; §8(a) a4 "P" and
+// §V-D P@38827 "which ... device to use ... data locality and potential
+// data-transfer cost"). For every P' = 2^i dividing nranks (and whose blocks
+// fit the int32 device indexing), P'-block j is the union of the nranks/P'
+// consecutive row blocks j*k .. j*k+k-1 (k = nranks/P'; its boundaries are
+// row_bounds[j*k], so with the A9 rule they are exactly A9's P'-way split).
+// Each rank ships its block (narrowed row pointer, columns, values) to rank
+// r / k over NCCL; rank j < P' widens the row pointers to one union row
+// pointer and plans the union (P' ranks, halo exchange among them). Every
+// rank then learns, for the HALO form, where its own rows and own ghosts
+// come from after a P' call (setup_xfer). Collective over all ranks.
+pepp_status_t setup_dist_parts(const pepp_spmv_opts_t* o, pepp_spmv_plan_t* p, const std::vector<int32_t>& ghosts,
+                               cudaStream_t st) {
+    const int N = o->nranks, me = o->rank;
+    const int64_t es = (int64_t)p->esz;
+    std::vector<int64_t> nnz_all, pad_all;
+    pepp_status_t s;
+    if ((s = nccl_allgather_i64(p, st, p->nnz, nnz_all))) return s;
+    if ((s = nccl_allgather_i64(p, st, p->pad, pad_all))) return s;
+    p->global_nnz = 0;
+    for (int64_t z : nnz_all) p->global_nnz += z;
+    for (int parts = 1; parts < N; parts *= 2) {
+        if (N % parts) continue;
+        const int k = N / parts;
+        bool fits = true;   // the same verdict on every rank (global facts only)
+        for (int j = 0; j < parts; ++j) {
+            int64_t z = 0;
+            for (int r = j * k; r < (j + 1) * k; ++r) z += nnz_all[r];
+            fits &= z + 8 < (int64_t)INT32_MAX && p->row_bounds[(j + 1) * k] - p->row_bounds[j * k] < (int64_t)INT32_MAX;
+        }
+        if (!fits) continue;
+        DistPart dp;
+        dp.parts = parts;
+        dp.bounds.resize(parts + 1);
+        for (int j = 0; j <= parts; ++j) dp.bounds[j] = p->row_bounds[(int64_t)j * k];
+        // ---- ship the blocks: rank r -> rank r / k
+        const int dest = me / k;
+        const bool recv_side = me < parts;
+        int64_t urows = 0, unnz = 0;
+        std::vector<int64_t> zoff(k + 1, 0);   // union nonzero offset of each source block
+        if (recv_side) {
+            urows = dp.bounds[me + 1] - dp.bounds[me];
+            for (int i = 0; i < k; ++i) zoff[i + 1] = zoff[i] + nnz_all[me * k + i];
+            unnz = zoff[k];
+        }
+        DevTmp<int64_t> u_rp;
+        DevTmp<int> u_col;
+        DevTmp<unsigned char> u_val;
+        std::vector<DevTmp<int>> rp32(k);
+        if (recv_side) {
+            PEPP_CUDA_TRY(u_rp.alloc(urows + 1));
+            PEPP_CUDA_TRY(u_col.alloc(unnz));
+            PEPP_CUDA_TRY(u_val.alloc((size_t)std::max<int64_t>(1, unnz) * es));
+            for (int i = 0; i < k; ++i) {
+                const int src = me * k + i;
+                PEPP_CUDA_TRY(rp32[i].alloc(p->row_bounds[src + 1] - p->row_bounds[src] + 1));
+            }
+        }
+        const Nccl* n = p->nccl;
+        if (n->GroupStart()) return PEPP_E_NCCL;
+        if (dest != me) {
+            n->Send(p->d_rp, (size_t)(p->nrows + 1), pepp::NCCL_INT32, dest, p->comm, st);
+            if (p->nnz) {
+                n->Send(p->d_col + p->pad, (size_t)p->nnz, pepp::NCCL_INT32, dest, p->comm, st);
+                n->Send((char*)p->d_val + p->pad * es, (size_t)(p->nnz * es), pepp::NCCL_INT8, dest, p->comm, st);
+            }
+        }
+        if (recv_side) {
+            for (int i = 0; i < k; ++i) {
+                const int src = me * k + i;
+                const int64_t rows = p->row_bounds[src + 1] - p->row_bounds[src], z = nnz_all[src];
+                if (src == me) {   // this rank's own block is part of its union (j = 0 only)
+                    PEPP_CUDA_TRY(cudaMemcpyAsync(rp32[i].p, p->d_rp, sizeof(int) * (rows + 1), cudaMemcpyDeviceToDevice, st));
+                    if (z) {
+                        PEPP_CUDA_TRY(cudaMemcpyAsync(u_col.p + zoff[i], p->d_col + p->pad, sizeof(int) * z, cudaMemcpyDeviceToDevice, st));
+                        PEPP_CUDA_TRY(cudaMemcpyAsync(u_val.p + zoff[i] * es, (char*)p->d_val + p->pad * es, (size_t)(z * es),
+                                                      cudaMemcpyDeviceToDevice, st));
+                    }
+                    continue;
+                }
+                n->Recv(rp32[i].p, (size_t)(rows + 1), pepp::NCCL_INT32, src, p->comm, st);
+                if (z) {
+                    n->Recv(u_col.p + zoff[i], (size_t)z, pepp::NCCL_INT32, src, p->comm, st);
+                    n->Recv(u_val.p + zoff[i] * es, (size_t)(z * es), pepp::NCCL_INT8, src, p->comm, st);
+                }
+            }
+        }
+        if (n->GroupEnd()) return PEPP_E_NCCL;
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        if (recv_side) {
+            // union row pointer: block i's rows at union row offset ro, entries
+            // rebased from (local offset + pad_src) to zoff[i]; the last entry
+            // of one block is the first of the next (same value), so the
+            // blocks are written in order and each writes rows + 1 entries
+            int64_t ro = 0;
+            for (int i = 0; i < k; ++i) {
+                const int src = me * k + i;
+                const int64_t rows = p->row_bounds[src + 1] - p->row_bounds[src];
+                const int g = (int)std::min<int64_t>(1024, (rows + 1 + 255) / 256);
+                pepp::k::rowptr_widen_kernel<<<g, 256, 0, st>>>(rows + 1, rp32[i].p, zoff[i] - pad_all[src], u_rp.p + ro);
+                PEPP_CUDA_TRY(cudaGetLastError());
+                PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+                ro += rows;
+            }
+            pepp_csr_t U{};
+            U.nrows = urows;
+            U.ncols = p->ncols;
+            U.nnz = unnz;
+            U.first = 0;
+            U.row_ptr = u_rp.p;
+            U.col_idx = u_col.p;
+            U.values = u_val.p;
+            U.on_device = 1;
+            U.value_type = p->vt;
+            pepp_spmv_opts_t so = *o;
+            so.nranks = parts;
+            so.rank = me;
+            so.row_bounds = parts > 1 ? dp.bounds.data() : nullptr;
+            so.nccl_comm = parts > 1 ? (void*)p->comm : nullptr;
+            so.nccl_unique_id = nullptr;
+            so.exchange = parts > 1 ? PEPP_X_HALO : PEPP_X_NONE;   // explicit: no AUTO all-reduce among a subset
+            so.history_path = nullptr;
+            so.overlap = 0;
+            so.validate = 0;
+            so.dist_select = 0;
+            so.device = p->device;
+            pepp_spmv_plan_t* q = new (std::nothrow) pepp_spmv_plan_t();
+            if (!q) return PEPP_E_NOMEM;
+            q->device = -1;
+            if ((s = plan_impl(&U, &so, q))) { free_plan(q); return s; }
+            dp.plan = q;
+        }
+        p->dparts.push_back(std::move(dp));   // owned by the plan from here on (freed with it)
+        // ---- HALO form: own rows + own ghosts from their P' owners
+        {
+            DistPart& D = p->dparts.back();
+            std::vector<int32_t> need;
+            const int64_t lo = p->row_offset, hi = p->row_offset + p->nrows;
+            const int64_t clo = recv_side ? D.bounds[me] : 0, chi = recv_side ? D.bounds[me + 1] : 0;
+            need.reserve(p->nrows + ghosts.size());
+            size_t gi = 0;
+            auto add = [&](int64_t r) { if (r < clo || r >= chi) need.push_back((int32_t)r); };
+            for (int64_t r = lo; r < hi; ++r) {
+                while (gi < ghosts.size() && ghosts[gi] < r) add(ghosts[gi++]);
+                add(r);
+            }
+            while (gi < ghosts.size()) add(ghosts[gi++]);
+            if ((s = setup_xfer(p, need, D.bounds, D.recv_x, D.send_x, st))) return s;
+            // gather form: after a P' = nranks call (own rows + own ghosts
+            // valid), what a P' call on this rank reads on top of that — the
+            // rest of its P' block and its P' ghosts — from their owners
+            std::vector<int32_t> gneed;
+            if (recv_side && D.plan) {
+                std::vector<int32_t> pcols(D.plan->nnz), pghost;
+                if (D.plan->nnz)
+                    PEPP_CUDA_TRY(cudaMemcpy(pcols.data(), D.plan->d_col + D.plan->pad, sizeof(int) * D.plan->nnz,
+                                             cudaMemcpyDeviceToHost));
+                pepp::halo_ghost_list(pcols.data(), D.plan->nnz, clo, chi, pghost);
+                auto held = [&](int64_t r) {
+                    return (r >= lo && r < hi) || std::binary_search(ghosts.begin(), ghosts.end(), (int32_t)r);
+                };
+                size_t pg = 0;
+                for (int64_t r = clo; r < chi || pg < pghost.size();) {
+                    int64_t nxt;
+                    if (pg < pghost.size() && (r >= chi || pghost[pg] < r)) nxt = pghost[pg++];
+                    else nxt = r++;
+                    if (!held(nxt)) gneed.push_back((int32_t)nxt);
+                }
+                std::sort(gneed.begin(), gneed.end());
+                gneed.erase(std::unique(gneed.begin(), gneed.end()), gneed.end());
+            }
+            if ((s = setup_xfer(p, gneed, p->row_bounds, D.recv_g, D.send_g, st))) return s;
+        }
+    }
+    return PEPP_OK;
+}
+
+// after a NEXT_INPUT exchange that ran with P'' = `parts_done` partitions:
+// when the plan's chosen distribution for NEXT_INPUT calls is a P' < nranks
+// other than P'', bring what a P' call reads to the P' ranks (the gather
+// lists), so that y serves the plan's next call whichever path it takes
+pepp_status_t dist_complete(pepp_spmv_plan_t* p, void* y, cudaStream_t st, int parts_done, int* launches) {
+    if (p->dist_next < 0) return PEPP_OK;
+    const int parts = p->dcands[p->dist_next].parts;
+    if (parts == p->opts.nranks || parts == parts_done) return PEPP_OK;
+    for (auto& dp : p->dparts)
+        if (dp.parts == parts) {
+            if (launches) *launches += xfer_kernels(dp.recv_g, dp.send_g);
+            return exchange_xfer(p, dp.recv_g, dp.send_g, y, st);
+        }
+    return PEPP_OK;
 }
 
 // undo a registration every rank agreed had failed: nothing of it is in use
@@ -1756,6 +2116,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     }
     p->eligible.assign(p->cands.size(), 1);
     p->pending.assign(p->cands.size(), 0);
+    p->warmed.assign(p->cands.size(), 0);
     {   // bytes each candidate moves per call (pepp_choice_t.layout_bytes)
         const int64_t es = (int64_t)p->esz;
         const int64_t csr = A->nnz * (es + 4) + (A->nrows + 1) * 4 + A->ncols * es + A->nrows * es;
@@ -1870,10 +2231,16 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         if ((s = setup_overlap(A, o, p))) return s;
     p->send_local.clear();
     p->send_local.shrink_to_fit();
+    // distribution candidates (P' < nranks) for the plan-time timing (dist_probe)
+    if (o->nranks > 1 && o->dist_select && o->use_history && p->ncols == p->global_rows)
+        if ((s = setup_dist_parts(o, p, ghosts, st))) return s;
     I.device_bytes = p->dev_bytes;
     for (auto* q : p->sub) if (q) I.device_bytes += q->dev_bytes;
+    for (auto& dp : p->dparts) if (dp.plan) I.device_bytes += dp.plan->dev_bytes;
     return PEPP_OK;
 }
+
+pepp_status_t dist_probe(pepp_spmv_plan_t* p);
 
 }  // namespace
 
@@ -1916,7 +2283,7 @@ pepp_status_t scratch_release(pepp_spmv_plan_t* p, cudaStream_t st) {
 // stream joins the side stream. Critical path: max(interior, head + tail +
 // exchange) instead of kernel + exchange.
 pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flags, cudaStream_t st,
-                           pepp_choice_t* used) {
+                           pepp_choice_t* used, bool allow_p2p) {
     char* yb = (char*)y + p->row_offset * (int64_t)p->esz;
     const int sf = flags & PEPP_EXEC_NO_TIMING;
     // the side stream starts after everything the caller queued (x is ready)
@@ -1928,7 +2295,7 @@ pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flag
     // "interior" through its own selection (PEPP_Y_LOCAL: no exchange)
     pepp_status_t s = p->sub[1] ? pepp_spmv_exec(p->sub[1], x, yb + p->sub_r0[1] * (int64_t)p->esz, sf, st, nullptr, &u)
                                 : pepp_spmv_exec(p, x, y, sf | PEPP_Y_LOCAL, st, nullptr, &u);
-    const int b = p2p_index(p, y);
+    const int b = allow_p2p ? p2p_index(p, y) : -1;
     if (b >= 0) {
         // fused: head + tail rows computed, pushed into the peers' buffer b and
         // signalled by one kernel (PEPP_X_P2P)
@@ -1952,6 +2319,55 @@ pepp_status_t exec_overlap(pepp_spmv_plan_t* p, const void* x, void* y, int flag
     u.exchange = b >= 0 ? PEPP_X_P2P : PEPP_X_HALO;
     if (used) *used = u;
     return PEPP_OK;
+}
+
+// One call under a distribution candidate with P' < nranks: ranks 0..P'-1
+// compute their P' block (its own history-based variant selection), then
+// the exchange: the P' blocks all-gathered to every rank (PEPP_X_ALLGATHER,
+// or any PEPP_Y_REPLICATED call), or (PEPP_X_HALO) the halo among the P'
+// ranks followed by every rank receiving its own rows and own ghosts from
+// their P' owners — so the call leaves y as a P' = nranks call would for
+// this rank's own block (own rows + the entries its next call reads).
+pepp_status_t exec_dist(pepp_spmv_plan_t* p, DistPart& dp, int ex, const void* x, void* y, int flags, cudaStream_t st,
+                        const pepp_choice_t* force, pepp_choice_t* used) {
+    pepp_choice_t u{};
+    pepp_status_t s = PEPP_OK;
+    if (dp.plan) {
+        pepp_choice_t f{};
+        const pepp_choice_t* fp = nullptr;
+        if (force && force->variant >= 0) { f = *force; f.nparts = 0; f.exchange = PEPP_X_AUTO; fp = &f; }
+        s = pepp_spmv_exec(dp.plan, x, y, flags & PEPP_EXEC_NO_TIMING, st, fp, &u);
+        if (s) return s;
+    }
+    if ((flags & PEPP_Y_REPLICATED) || ex == PEPP_X_ALLGATHER) {
+        ex = PEPP_X_ALLGATHER;
+        s = exchange_blocks(p, dp.bounds.data(), dp.parts, y, st);
+    } else {
+        if (dp.plan && dp.parts > 1) {
+            s = exchange_halo(dp.plan, y, st);
+            u.launches += halo_kernels(dp.plan);
+        }
+        if (!s) s = exchange_xfer(p, dp.recv_x, dp.send_x, y, st);
+        u.launches += xfer_kernels(dp.recv_x, dp.send_x);
+        if (!s) s = dist_complete(p, y, st, dp.parts, &u.launches);
+    }
+    if (s) return s;
+    u.nparts = dp.parts;
+    u.exchange = ex;
+    if (used) *used = u;
+    return PEPP_OK;
+}
+
+// the plans whose kernels a distribution candidate runs on this rank are
+// still calibrating their variant choice (so the candidate is not timed yet)
+bool dist_busy(const pepp_spmv_plan_t* p, int parts, int ex) {
+    auto busy = [](const pepp_spmv_plan_t* q) { return q && q->opts.use_history && !q->calibrated && q->cands.size() > 1; };
+    if (parts == p->opts.nranks) {
+        if (ex == PEPP_X_HALO && p->sub[1]) return busy(p->sub[0]) || busy(p->sub[1]) || busy(p->sub[2]);
+        return busy(p);
+    }
+    for (const auto& dp : p->dparts) if (dp.parts == parts) return busy(dp.plan);
+    return false;
 }
 }  // namespace
 
@@ -1978,6 +2394,14 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_plan(const pepp_csr_t* A, const pepp
     } catch (...) {
         s = PEPP_E_INVALID;
     }
+    // P and exchange as timed choices: every candidate timed, ranks agree
+    if (s == PEPP_OK && p->opts.nranks > 1 && p->opts.dist_select && p->opts.use_history && p->ncols == p->global_rows) {
+        try {
+            s = dist_probe(p);
+        } catch (const std::bad_alloc&) {
+            s = PEPP_E_NOMEM;
+        }
+    }
     if (s != PEPP_OK) { free_plan(p); return s; }
     *out = p;
     return PEPP_OK;
@@ -1986,7 +2410,12 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_plan(const pepp_csr_t* A, const pepp
 extern "C" PEPP_API pepp_status_t pepp_spmv_select(pepp_spmv_plan_t* p, pepp_choice_t* out) {
     if (!p || !out) return PEPP_E_INVALID;
     if (p->sticky) return p->sticky;
-    return select_choice(p, out);
+    const pepp_status_t s = select_choice(p, out);
+    if (!s && p->dist_next >= 0) {   // partitioned: the distribution a PEPP_Y_NEXT_INPUT call runs
+        out->nparts = p->info.dist_nparts;
+        out->exchange = p->info.dist_exchange;
+    }
+    return s;
 }
 
 extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void* x, void* y, int flags,
@@ -2010,24 +2439,59 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
         if (cudaStreamIsCapturing(st, &cs) != cudaSuccess) { (void)cudaGetLastError(); cs = cudaStreamCaptureStatusNone; }
         capturing = cs != cudaStreamCaptureStatusNone;
     }
-    if (!force && (flags & PEPP_Y_NEXT_INPUT) && !(flags & PEPP_Y_REPLICATED) && p->exchange == PEPP_X_HALO &&
-        (p->sub[1] || p2p_index(p, y) >= 0)) {
+    // ---- partitioned calls: the distribution (P', exchange) of this call
+    const int N = p->opts.nranks;
+    const bool fvar = force && force->variant >= 0;   // variant forced (PEPP_V_AUTO = selected as usual)
+    const bool part_call = N > 1 && (flags & (PEPP_Y_NEXT_INPUT | PEPP_Y_REPLICATED));
+    const bool next_only = (flags & PEPP_Y_NEXT_INPUT) && !(flags & PEPP_Y_REPLICATED);
+    int ex_call = p->exchange;                        // exchange of a P' = nranks call
+    bool allow_p2p = p->dcands.empty() || p->p2p_use;
+    DistPart* dpart = nullptr;
+    if (part_call) {
+        if (force && force->nparts > 0 && force->nparts != N) {   // a forced P' < nranks
+            for (auto& dp : p->dparts) if (dp.parts == force->nparts) dpart = &dp;
+            if (!dpart) return PEPP_E_INVALID;
+            ex_call = force->exchange == PEPP_X_ALLGATHER ? PEPP_X_ALLGATHER : PEPP_X_HALO;
+        } else if (force && (force->exchange == PEPP_X_ALLGATHER || force->exchange == PEPP_X_HALO)) {
+            ex_call = force->exchange;
+            allow_p2p = false;
+        } else if (force && force->exchange == PEPP_X_P2P) {
+            allow_p2p = true;
+        } else if (!force && !p->dcands.empty() && !(next_only && allow_p2p && p2p_index(p, y) >= 0)) {
+            // the distribution the plan-time timing chose (opts.dist_select)
+            const int d = (flags & PEPP_Y_REPLICATED) ? p->dist_repl : p->dist_next;
+            if (d >= 0) {
+                if (p->dcands[d].parts != N)
+                    for (auto& dp : p->dparts) if (dp.parts == p->dcands[d].parts) dpart = &dp;
+                ex_call = p->dcands[d].ex;
+            }
+            allow_p2p = false;
+        }
+    }
+    if (dpart) {
         pepp_status_t s = capturing ? PEPP_OK : scratch_acquire(p, st);
-        if (!s) s = exec_overlap(p, x, y, flags, st, used);
+        if (!s) s = exec_dist(p, *dpart, ex_call, x, y, flags, st, force, used);
+        if (!s && !capturing) s = scratch_release(p, st);
+        if (s) p->sticky = s;
+        else ++p->ncalls;
+        return s;
+    }
+    if (!fvar && next_only && ex_call == PEPP_X_HALO && (p->sub[1] || (allow_p2p && p2p_index(p, y) >= 0))) {
+        pepp_status_t s = capturing ? PEPP_OK : scratch_acquire(p, st);
+        if (!s) s = exec_overlap(p, x, y, flags, st, used, allow_p2p);
+        if (!s) s = dist_complete(p, y, st, N, used ? &used->launches : nullptr);
         if (!s && !capturing) s = scratch_release(p, st);
         if (s) p->sticky = s;
         else ++p->ncalls;
         return s;
     }
     pepp_choice_t ch{};
-    if (force) {
+    if (fvar) {
         int idx = -1;
         for (size_t i = 0; i < p->cands.size(); ++i)
             if (p->cands[i].variant == force->variant && (force->param <= 0 || p->cands[i].param == force->param)) { idx = (int)i; break; }
         if (idx < 0) return PEPP_E_INVALID;
         fill_choice(p, idx, 0, 0.0, &ch);
-        if (p->opts.nranks > 1 && (force->exchange == PEPP_X_ALLGATHER || force->exchange == PEPP_X_HALO))
-            ch.exchange = force->exchange;
         if (!capturing) harvest(p, false);
     } else {
         pepp_status_t s = select_choice(p, &ch, capturing);
@@ -2067,10 +2531,9 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
     }
     ch.exchange = PEPP_X_NONE;
     if (exchanging) {
-        const bool ag = (flags & PEPP_Y_REPLICATED) || p->exchange == PEPP_X_ALLGATHER;
-        const int ex = (force && (force->exchange == PEPP_X_ALLGATHER || force->exchange == PEPP_X_HALO))
-                           ? force->exchange : (ag ? PEPP_X_ALLGATHER : PEPP_X_HALO);
+        const int ex = ((flags & PEPP_Y_REPLICATED) || ex_call == PEPP_X_ALLGATHER) ? PEPP_X_ALLGATHER : PEPP_X_HALO;
         s = ex == PEPP_X_ALLGATHER ? exchange_allgather(p, y, st) : exchange_halo(p, y, st);
+        if (!s && ex == PEPP_X_HALO) s = dist_complete(p, y, st, N, &ch.launches);
         if (s) { p->sticky = s; return s; }
         ch.exchange = ex;
         if (ex == PEPP_X_HALO) ch.launches += halo_kernels(p);
@@ -2080,6 +2543,159 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
     if (used) *used = ch;
     return PEPP_OK;
 }
+
+namespace {
+constexpr int32_t kDistVariant = 5;   // history uid of a distribution candidate: kDistVariant << 20 | P' << 4 | exchange
+
+int32_t dist_uid(int parts, int ex) { return (kDistVariant << 20) | ((parts & 0xFFFF) << 4) | (ex & 0xF); }
+
+// Time one candidate (P', ex) on this rank: NEXT_INPUT calls on scratch
+// vectors until every rank's plans for it finished calibrating their variant
+// choice (agreed every 4 calls), then `ms` timed calls (events on the
+// stream around the whole call: kernels + exchange). Collective.
+pepp_status_t dist_time(pepp_spmv_plan_t* p, int parts, int ex, void* a, void* b, cudaStream_t st, int ms,
+                        double* samples) {
+    pepp_choice_t f{};
+    f.variant = PEPP_V_AUTO;
+    f.param = 0;
+    f.nparts = parts;
+    f.exchange = ex;
+    pepp_status_t s;
+    for (int it = 0;; it += 4) {
+        for (int j = 0; j < 4; ++j) {
+            if ((s = pepp_spmv_exec(p, a, b, PEPP_Y_NEXT_INPUT, st, &f, nullptr))) return s;
+            std::swap(a, b);
+        }
+        int64_t busy = dist_busy(p, parts, ex == PEPP_X_P2P ? PEPP_X_HALO : ex) ? 1 : 0;
+        if ((s = nccl_allmax(p, st, &busy))) return s;
+        if (!busy || it >= 256) break;
+    }
+    std::vector<cudaEvent_t> ev(2 * ms, nullptr);
+    struct Ev { std::vector<cudaEvent_t>& v; ~Ev() { for (auto e : v) if (e) cudaEventDestroy(e); } } guard{ev};
+    for (auto& e : ev) PEPP_CUDA_TRY(cudaEventCreate(&e));
+    for (int j = 0; j < ms; ++j) {
+        PEPP_CUDA_TRY(cudaEventRecord(ev[2 * j], st));
+        if ((s = pepp_spmv_exec(p, a, b, PEPP_Y_NEXT_INPUT | PEPP_EXEC_NO_TIMING, st, &f, nullptr))) return s;
+        PEPP_CUDA_TRY(cudaEventRecord(ev[2 * j + 1], st));
+        std::swap(a, b);
+    }
+    PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+    for (int j = 0; j < ms; ++j) {
+        float t = 0.f;
+        PEPP_CUDA_TRY(cudaEventElapsedTime(&t, ev[2 * j], ev[2 * j + 1]));
+        samples[j] = (double)t * 1000.0;
+    }
+    return PEPP_OK;
+}
+
+// Plan-time choice of (P', exchange) for a partitioned plan (opts.dist_select;
+// §8(a) a4; dynamic composition from recorded history, §III P@10254). The
+// candidates: P' = nranks first, then every prepared P' < nranks, descending,
+// each with halo and allgather (only opts.exchange when it is not AUTO). If
+// this rank's loaded history lacks min_samples records of some candidate on
+// any rank, every candidate is timed (dist_time) on plan-owned zero vectors
+// (SpMV time does not depend on the values) and the samples are max-reduced
+// over ranks (a partitioned call lasts as long as its slowest rank) and
+// recorded; then the agreed means (this rank's history means, max-reduced)
+// give the argmin for NEXT_INPUT calls and, among allgather candidates, for
+// REPLICATED calls — identical on every rank (pepp::dist_argmin, the rule of
+// pepp_dist_choose).
+pepp_status_t dist_probe(pepp_spmv_plan_t* p) {
+    PEPP_NVTX("pepp dist probe");
+    const int N = p->opts.nranks;
+    const double t0 = now_ms();
+    std::vector<int> exs;
+    if (p->opts.exchange == PEPP_X_HALO || p->opts.exchange == PEPP_X_ALLGATHER) exs = {p->opts.exchange};
+    else exs = {PEPP_X_HALO, PEPP_X_ALLGATHER};
+    p->dcands.clear();
+    for (int ex : exs) p->dcands.push_back({N, ex});
+    for (auto it = p->dparts.rbegin(); it != p->dparts.rend(); ++it)
+        for (int ex : exs) p->dcands.push_back({it->parts, ex});
+    const int nd = (int)p->dcands.size();
+    const int ms = std::max(1, p->opts.min_samples);
+    p->dist_key = pepp::context_key(p->global_rows, p->ncols, p->global_nnz, 0.0, N,
+                                    (p->vt == PEPP_VALUE_F32 ? PEPP_KEY_F32 : 0) |
+                                    (p->opts.compress_values ? PEPP_KEY_COMPRESS : 0) | PEPP_KEY_DIST);
+    cudaStream_t st = nullptr;
+    PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+    struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{st};
+    pepp_status_t s;
+    int64_t need = 0;
+    for (const auto& c : p->dcands) {
+        const pepp::Welford* w = pepp::history_get(p->hist, p->dist_key, dist_uid(c.parts, c.ex));
+        need |= !w || w->count < ms;
+    }
+    if ((s = nccl_allmax(p, st, &need))) return s;
+    if (need) {
+        DevTmp<unsigned char> a, b;
+        const size_t bytes = (size_t)std::max<int64_t>(1, p->global_rows) * p->esz;
+        PEPP_CUDA_TRY(a.alloc(bytes));
+        PEPP_CUDA_TRY(b.alloc(bytes));
+        PEPP_CUDA_TRY(cudaMemsetAsync(a.p, 0, bytes, st));
+        PEPP_CUDA_TRY(cudaMemsetAsync(b.p, 0, bytes, st));
+        std::vector<double> samples((size_t)nd * ms, 0.0);
+        for (int d = 0; d < nd; ++d)
+            if ((s = dist_time(p, p->dcands[d].parts, p->dcands[d].ex, a.p, b.p, st, ms, &samples[(size_t)d * ms]))) return s;
+        if ((s = nccl_allmax_f64(p, st, samples))) return s;
+        for (int d = 0; d < nd; ++d)
+            for (int j = 0; j < ms; ++j)
+                pepp::history_add(p->hist, p->dist_key, dist_uid(p->dcands[d].parts, p->dcands[d].ex), samples[(size_t)d * ms + j]);
+    }
+    std::vector<double> mean(nd, 0.0);
+    for (int d = 0; d < nd; ++d) {
+        const pepp::Welford* w = pepp::history_get(p->hist, p->dist_key, dist_uid(p->dcands[d].parts, p->dcands[d].ex));
+        mean[d] = w ? w->mean : 0.0;
+    }
+    if ((s = nccl_allmax_f64(p, st, mean))) return s;
+    p->dist_agreed = mean;
+    std::vector<uint8_t> ag(nd);
+    for (int d = 0; d < nd; ++d) ag[d] = p->dcands[d].ex == PEPP_X_ALLGATHER;
+    p->dist_next = pepp::dist_argmin(nd, mean.data(), nullptr);
+    p->dist_repl = pepp::dist_argmin(nd, mean.data(), ag.data());
+    if (p->dist_next < 0) p->dist_next = 0;
+    pepp_plan_info_t& I = p->info;
+    I.dist_candidates = nd;
+    I.dist_nparts = p->dcands[p->dist_next].parts;
+    I.dist_exchange = p->dcands[p->dist_next].ex;
+    I.dist_repl_nparts = p->dist_repl >= 0 ? p->dcands[p->dist_repl].parts : N;
+    I.dist_probe_ms = now_ms() - t0;
+    return PEPP_OK;
+}
+
+// The fused push as a distribution candidate (P' = nranks, PEPP_X_P2P), timed
+// on the just-registered buffers like dist_probe's candidates and compared
+// with the agreed best (1 % tie rule: the NCCL candidates come first).
+pepp_status_t p2p_probe(pepp_spmv_plan_t* p) {
+    PEPP_NVTX("pepp p2p probe");
+    const int N = p->opts.nranks, ms = std::max(1, p->opts.min_samples);
+    cudaStream_t st = nullptr;
+    PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+    struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{st};
+    pepp_status_t s;
+    const int32_t uid = dist_uid(N, PEPP_X_P2P);
+    const pepp::Welford* w = pepp::history_get(p->hist, p->dist_key, uid);
+    int64_t need = !w || w->count < ms;
+    if ((s = nccl_allmax(p, st, &need))) return s;
+    if (need && p->p2p_nbuf < 2) return PEPP_OK;   // one buffer: no ping-pong to time it with; the push is used
+    if (need) {
+        std::vector<double> samples(ms, 0.0);
+        const bool keep = p->p2p_use;
+        p->p2p_use = true;
+        s = dist_time(p, N, PEPP_X_P2P, p->p2p_buf[0], p->p2p_buf[1 % p->p2p_nbuf], st, ms, samples.data());
+        p->p2p_use = keep;
+        if (s) return s;
+        if ((s = nccl_allmax_f64(p, st, samples))) return s;
+        for (double v : samples) pepp::history_add(p->hist, p->dist_key, uid, v);
+    }
+    std::vector<double> m(1, pepp::history_get(p->hist, p->dist_key, uid)->mean);
+    if ((s = nccl_allmax_f64(p, st, m))) return s;
+    p->p2p_agreed = m[0];
+    const double best = p->dist_next >= 0 ? p->dist_agreed[p->dist_next] : 0.0;
+    p->p2p_use = !(best > 0.0) || m[0] < best * 0.99;
+    if (p->p2p_use) { p->info.dist_nparts = N; p->info.dist_exchange = PEPP_X_P2P; }
+    return PEPP_OK;
+}
+}  // namespace
 
 struct pepp_spmv_graph_s {
     cudaGraph_t graph = nullptr;
@@ -2197,6 +2813,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* 
     cudaStream_t st = (cudaStream_t)stream;
     const bool ag = (flags & PEPP_Y_REPLICATED) || p->exchange == PEPP_X_ALLGATHER;
     pepp_status_t s = ag ? exchange_allgather(p, y, st) : exchange_halo(p, y, st);
+    if (!s && !ag) s = dist_complete(p, y, st, p->opts.nranks, nullptr);
     if (s) p->sticky = s;
     return s;
 }
@@ -2378,6 +2995,8 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_p2p_buffers(pepp_spmv_plan_t* p, int
         return s;
     }
     if (s) { p->sticky = s; return s; }
+    // the fused push is a timed distribution candidate too (collective)
+    if (!p->dcands.empty() && (s = p2p_probe(p))) { p->sticky = s; return s; }
     for (int b = 0; b < nbuf; ++b) bufs[b] = p->p2p_buf[b];
     p->info.p2p_buffers = nbuf;
     p->info.device_bytes = p->dev_bytes;
@@ -2403,11 +3022,26 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_candidates(const pepp_spmv_plan_t* p
     return PEPP_OK;
 }
 
+extern "C" PEPP_API pepp_status_t pepp_spmv_dist_stats(const pepp_spmv_plan_t* p, int32_t cap, int32_t* nparts,
+                                                      int32_t* exchange, double* agreed_us, int32_t* n) {
+    if (!p || !n || cap < 0) return PEPP_E_INVALID;
+    const int32_t nd = (int32_t)p->dcands.size(), tot = nd + (nd && p->p2p_nbuf ? 1 : 0);
+    *n = tot;
+    for (int32_t i = 0; i < tot && i < cap; ++i) {
+        const bool pp = i == nd;
+        if (nparts) nparts[i] = pp ? p->opts.nranks : p->dcands[i].parts;
+        if (exchange) exchange[i] = pp ? PEPP_X_P2P : p->dcands[i].ex;
+        if (agreed_us) agreed_us[i] = pp ? p->p2p_agreed : p->dist_agreed[i];
+    }
+    return PEPP_OK;
+}
+
 extern "C" PEPP_API pepp_status_t pepp_spmv_flush_history(pepp_spmv_plan_t* p) {
     if (!p) return PEPP_E_INVALID;
     DeviceScope dscope(p->device);
     harvest(p, true);
     for (auto* q : p->sub) if (q) harvest(q, true);
+    for (auto& dp : p->dparts) if (dp.plan) harvest(dp.plan, true);
     return PEPP_OK;
 }
 

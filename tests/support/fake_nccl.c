@@ -4,9 +4,12 @@
  * processes sharing ONE GPU can run the library's partitioned path (real
  * NCCL refuses two ranks on one device). Semantics follow NCCL's: calls
  * between ncclGroupStart/End are matched in order per peer; a call outside a
- * group is a group of one. Data moves through a shared, file-backed mapping
- * with a process-shared sense-reversing barrier; the device <-> host copies
- * are synchronous (the stream is synchronised first). Selected by the
+ * group is a group of one; point-to-point groups involve only the peers they
+ * name (per-pair mailboxes with published / consumed message counters, no
+ * barrier), collectives (broadcast, all-reduce) every rank. Data moves
+ * through a shared, file-backed mapping with a process-shared barrier for
+ * the collectives; the device <-> host copies are synchronous (the stream is
+ * synchronised first). MAXR ranks, PEPP_FAKE_NCCL_BOX_MB per pair message. Selected by the
  * library when PEPP_NCCL_LIB points at this .so.
  *
  * Build: gcc -O2 -shared -fPIC fake_nccl.c -I$CUDA/include -L$CUDA/lib64 -lcudart
@@ -63,7 +66,8 @@ static __thread Comm* g_pending = NULL;   /* the communicator with queued ops (o
 static Barrier* bar(Comm* c) { return (Barrier*)c->base; }
 static unsigned char* box(Comm* c, int src, int dst) { return c->base + 4096 + ((size_t)src * MAXR + dst) * c->box; }
 static unsigned char* bcast(Comm* c, int root) { return c->base + 4096 + (size_t)MAXR * MAXR * c->box + (size_t)root * c->box; }
-static unsigned char* arslot(Comm* c, int r) { return c->base + 2048 + (size_t)r * 128; }
+#define ARMAX 65536   /* all-reduce payload per rank and group */
+static unsigned char* arslot(Comm* c, int r) { return c->base + 4096 + (size_t)MAXR * MAXR * c->box + (size_t)MAXR * c->box + (size_t)r * ARMAX; }
 
 static void barrier(Comm* c) {
     Barrier* b = bar(c);
@@ -104,7 +108,7 @@ EXPORT int ncclCommInitRank(ncclComm_t* out, int nranks, ncclUniqueId id, int ra
     snprintf(c->path, sizeof(c->path), "%s", id.internal);
     const char* e = getenv("PEPP_FAKE_NCCL_BOX_MB");
     c->box = (size_t)(e ? atoi(e) : 16) << 20;
-    c->size = 4096 + (size_t)MAXR * MAXR * c->box + (size_t)MAXR * c->box;
+    c->size = 4096 + (size_t)MAXR * MAXR * c->box + (size_t)MAXR * c->box + (size_t)MAXR * ARMAX;
     int fd = open(c->path, O_RDWR | O_CREAT, 0600);
     if (fd < 0) { free(c); return 2; }
     if (ftruncate(fd, (off_t)c->size) != 0) { close(fd); free(c); return 2; }
@@ -130,44 +134,77 @@ EXPORT int ncclCommDestroy(ncclComm_t c) {
 
 EXPORT int ncclCommGetAsyncError(ncclComm_t c, int* err) { (void)c; *err = 0; return 0; }
 
+/* per (src, dst) mailbox state: messages published / consumed (one message =
+   all sends src -> dst of one group, concatenated in call order) */
+static volatile int* pub(Comm* c, int src, int dst) { return (volatile int*)(c->base + 3072) + src * MAXR + dst; }
+static volatile int* con(Comm* c, int src, int dst) { return (volatile int*)(c->base + 3072 + 256) + src * MAXR + dst; }
+
 static int flush(Comm* c) {
     size_t out[MAXR] = {0}, in[MAXR] = {0}, bc[MAXR] = {0};
-    for (int i = 0; i < c->nops; ++i)
+    int has_coll = 0, sends_to[MAXR] = {0}, recvs_from[MAXR] = {0};
+    for (int i = 0; i < c->nops; ++i) {
         if (cudaStreamSynchronize(c->ops[i].stream) != cudaSuccess) return 1;
-    size_t arc = 0;
-    for (int i = 0; i < c->nops; ++i) {            /* phase 1: publish */
         Op* o = &c->ops[i];
-        if (o->kind == OP_SEND) {
-            if (out[o->peer] + o->bytes > c->box) return 3;
-            cudaMemcpy(box(c, c->rank, o->peer) + out[o->peer], o->sbuf, o->bytes, cudaMemcpyDeviceToHost);
-            out[o->peer] += o->bytes;
-        } else if (o->kind == OP_BCAST) {
-            if (bc[o->peer] + o->bytes > c->box) return 3;
-            if (c->rank == o->peer)
-                cudaMemcpy(bcast(c, o->peer) + bc[o->peer], o->sbuf, o->bytes, cudaMemcpyDeviceToHost);
-            bc[o->peer] += o->bytes;
-        } else if (o->kind == OP_AR) {
-            if (arc + o->bytes > 128) return 3;
-            cudaMemcpy(arslot(c, c->rank) + arc, o->sbuf, o->bytes, cudaMemcpyDeviceToHost);
-            arc += o->bytes;
-        }
+        if (o->kind == OP_BCAST || o->kind == OP_AR) has_coll = 1;
+        else if (o->kind == OP_SEND) sends_to[o->peer] = 1;
+        else recvs_from[o->peer] = 1;
     }
-    barrier(c);
+    /* point-to-point: like NCCL, only the two peers take part (no barrier):
+       wait until the previous message to that peer was consumed, write, publish */
+    for (int q = 0; q < c->nranks; ++q) {
+        if (!sends_to[q]) continue;
+        while (__atomic_load_n(pub(c, c->rank, q), __ATOMIC_ACQUIRE) != __atomic_load_n(con(c, c->rank, q), __ATOMIC_ACQUIRE))
+            sched_yield();
+        for (int i = 0; i < c->nops; ++i) {
+            Op* o = &c->ops[i];
+            if (o->kind != OP_SEND || o->peer != q) continue;
+            if (out[q] + o->bytes > c->box) return 3;
+            cudaMemcpy(box(c, c->rank, q) + out[q], o->sbuf, o->bytes, cudaMemcpyDeviceToHost);
+            out[q] += o->bytes;
+        }
+        __atomic_add_fetch(pub(c, c->rank, q), 1, __ATOMIC_RELEASE);
+    }
+    size_t arc = 0;
+    if (has_coll) {
+        for (int i = 0; i < c->nops; ++i) {            /* collectives, phase 1: publish */
+            Op* o = &c->ops[i];
+            if (o->kind == OP_BCAST) {
+                if (bc[o->peer] + o->bytes > c->box) return 3;
+                if (c->rank == o->peer)
+                    cudaMemcpy(bcast(c, o->peer) + bc[o->peer], o->sbuf, o->bytes, cudaMemcpyDeviceToHost);
+                bc[o->peer] += o->bytes;
+            } else if (o->kind == OP_AR) {
+                if (arc + o->bytes > ARMAX) return 3;
+                cudaMemcpy(arslot(c, c->rank) + arc, o->sbuf, o->bytes, cudaMemcpyDeviceToHost);
+                arc += o->bytes;
+            }
+        }
+        barrier(c);
+    }
     memset(bc, 0, sizeof(bc));
     arc = 0;
-    for (int i = 0; i < c->nops; ++i) {            /* phase 2: consume */
+    for (int q = 0; q < c->nranks; ++q) {            /* point-to-point receives, in call order per peer */
+        if (!recvs_from[q]) continue;
+        while (__atomic_load_n(pub(c, q, c->rank), __ATOMIC_ACQUIRE) == __atomic_load_n(con(c, q, c->rank), __ATOMIC_ACQUIRE))
+            sched_yield();
+        for (int i = 0; i < c->nops; ++i) {
+            Op* o = &c->ops[i];
+            if (o->kind != OP_RECV || o->peer != q) continue;
+            cudaMemcpy(o->rbuf, box(c, q, c->rank) + in[q], o->bytes, cudaMemcpyHostToDevice);
+            in[q] += o->bytes;
+        }
+        __atomic_add_fetch(con(c, q, c->rank), 1, __ATOMIC_RELEASE);
+    }
+    for (int i = 0; i < c->nops && has_coll; ++i) {            /* collectives, phase 2: consume */
         Op* o = &c->ops[i];
-        if (o->kind == OP_RECV) {
-            cudaMemcpy(o->rbuf, box(c, o->peer, c->rank) + in[o->peer], o->bytes, cudaMemcpyHostToDevice);
-            in[o->peer] += o->bytes;
-        } else if (o->kind == OP_BCAST) {
+        if (o->kind == OP_BCAST) {
             if (c->rank != o->peer)
                 cudaMemcpy(o->rbuf, bcast(c, o->peer) + bc[o->peer], o->bytes, cudaMemcpyHostToDevice);
             else if (o->rbuf != o->sbuf)
                 cudaMemcpy(o->rbuf, o->sbuf, o->bytes, cudaMemcpyDeviceToDevice);
             bc[o->peer] += o->bytes;
         } else if (o->kind == OP_AR) {
-            unsigned char tmp[128];
+            static __thread unsigned char tmp[ARMAX];
             for (size_t k = 0; k < o->count; ++k) {
                 double dv = 0; int64_t iv = 0;
                 for (int r = 0; r < c->nranks; ++r) {
@@ -191,15 +228,26 @@ static int flush(Comm* c) {
        visible to work the caller enqueues next on any stream (real NCCL
        orders it on the op's stream) */
     if (cudaDeviceSynchronize() != cudaSuccess) return 1;
-    barrier(c);
+    if (has_coll) barrier(c);   /* the collective slots may be reused by the next group */
     c->nops = 0;
     return cudaGetLastError() == cudaSuccess ? 0 : 1;
+}
+
+static int flush_checked(Comm* c) {
+    int r = flush(c);
+    if (r) {
+        cudaError_t e = cudaGetLastError();
+        fprintf(stderr, "[fake nccl] rank %d/%d: group of %d ops failed (%d; cuda: %s)\n", c->rank, c->nranks, c->nops, r,
+                cudaGetErrorString(e));
+        c->nops = 0;
+    }
+    return r;
 }
 
 static int enqueue(Comm* c, Op o) {
     if (c->nops >= MAXOPS) return 3;
     c->ops[c->nops++] = o;
-    if (g_depth == 0) return flush(c);
+    if (g_depth == 0) return flush_checked(c);
     g_pending = c;
     return 0;
 }
@@ -207,7 +255,7 @@ static int enqueue(Comm* c, Op o) {
 EXPORT int ncclGroupStart(void) { ++g_depth; return 0; }
 EXPORT int ncclGroupEnd(void) {
     if (g_depth <= 0) return 4;
-    if (--g_depth == 0 && g_pending) { Comm* c = g_pending; g_pending = NULL; return flush(c); }
+    if (--g_depth == 0 && g_pending) { Comm* c = g_pending; g_pending = NULL; return flush_checked(c); }
     return 0;
 }
 

@@ -146,3 +146,50 @@ def test_two_rank_iterated_spmv_matches_oracle(name, exchange):
     assert nans == 0 and equal
     if exchange == "halo" and name == "lap":
         assert nghost == 24          # one grid row of ghosts per neighbour
+
+
+def _dist_worker(rank, world, port, outq):
+    """Each rank holds its OWN (injected) timings of the distribution
+    candidates; the agreement the plan makes over NCCL (an elementwise max
+    all-reduce of the mean vector, then pepp::dist_argmin) is made here over
+    gloo with the library's host rule: every rank must reach the same choice,
+    equal to pepp_dist_choose on the stacked [rank][candidate] matrix."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    try:
+        import sys
+        root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+        sys.path.insert(0, root)
+        import paper_conf_sc_dastgeerlk12_b200 as pepp
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        rng = np.random.default_rng(100 + rank)
+        mine = rng.uniform(50, 150, size=6)           # this rank's clock
+        t = torch.from_numpy(mine.copy())
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        agreed = t.numpy()
+        c_local, ag = pepp.dist_choose(agreed[None, :])
+        allm = [torch.zeros(6, dtype=torch.float64) for _ in range(world)]
+        dist.all_gather(allm, torch.from_numpy(mine))
+        c_ref, ag_ref = pepp.dist_choose(np.stack([m.numpy() for m in allm]))
+        outq.put((rank, (c_local, c_ref, bool(np.array_equal(ag, ag_ref)))))
+        dist.destroy_process_group()
+    except Exception as e:
+        import traceback
+        outq.put((rank, repr(e) + traceback.format_exc()))
+
+
+def test_two_rank_distribution_agreement():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_dist_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = dict(q.get(timeout=120) for _ in range(2))
+    for p in procs:
+        p.join(30)
+    for r in range(2):
+        assert isinstance(out[r], tuple), out[r]
+        c_local, c_ref, same = out[r]
+        assert c_local == c_ref and same
+    assert out[0][0] == out[1][0]

@@ -304,9 +304,10 @@ def test_selector_calibrates_then_picks_fastest_measured():
                 break
             seen.append(u.candidate)
         # round 1 visits every candidate; later rounds skip the ones ruled out,
-        # rounds 4..9 (refinement) only the contenders within 10 % of the best
+        # rounds 4..9 (refinement) only the contenders within 10 % of the best;
+        # each candidate's first timed call is a warm-up (not recorded): +1 each
         assert seen[:n] == list(range(n))
-        assert len(seen) <= 9 * n
+        assert len(seen) <= 10 * n
         plan.flush_history()
         means = [plan.history_stats(c)[1] for c in range(n)]
         ch = plan.select()

@@ -219,7 +219,7 @@ def _worker_p2p(rank, world, lib, uid, name, K, outq, f32=False, real=False):
         x0 = (gen.vector(5, gen.REAL, n) if real else gen.vector(3, gen.INT8, n)).astype(dt)
         res = {}
         with pepp.Plan.from_csr(blk, nranks=world, rank=rank, row_bounds=bounds, nccl_unique_id=uid,
-                                exchange=pepp.X_HALO) as plan:
+                                exchange=pepp.X_HALO, dist_select=False) as plan:
             info = plan.info()
             bufs = plan.p2p_buffers(2)
             res["p2p_buffers"] = plan.info()["p2p_buffers"]
@@ -333,3 +333,150 @@ def test_two_ranks_p2p_fused_halo(name, f32, real):
         assert len(gi) > 0 and np.array_equal(gv, ov[gi - o0])   # what arrived is what the owner computed
         assert out[r]["used"] == [pepp.X_P2P], out[r]
         assert out[r]["p2p_buffers"] == 2
+
+
+# ------------------------------------------- distribution choice (row a4)
+def _worker_dist(rank, world, lib, uid, name, K, outq, p2p):
+    """opts.dist_select: the plan times every (P', exchange) candidate, the
+    ranks agree, and NEXT_INPUT / REPLICATED calls run the agreed argmin; every
+    candidate forced must give the same bits (integer inputs)."""
+    os.environ["PEPP_NCCL_LIB"] = lib
+    try:
+        import sys
+        sys.path.insert(0, os.path.dirname(HERE))
+        import torch
+
+        import gen
+        import oracle
+        import paper_conf_sc_dastgeerlk12_b200 as pepp
+        torch.cuda.set_device(0)
+        A = _matrix(name)
+        n = A.nrows
+        bounds = pepp.partition_rows(A.row_ptr, world)
+        r0, r1 = int(bounds[rank]), int(bounds[rank + 1])
+        blk = gen.row_block(A, r0, r1)
+        x0 = gen.vector(3, gen.INT8, n)
+        _, ghosts = pepp.halo_ghosts(blk.col, world, rank, bounds)
+        rows = np.concatenate([np.arange(r0, r1), ghosts.astype(np.int64)])
+        refs = [x0]
+        for _ in range(K):
+            refs.append(oracle.spmv(A, refs[-1]))
+        res = {"ok": True, "forced": {}}
+        with pepp.Plan.from_csr(blk, nranks=world, rank=rank, row_bounds=bounds, nccl_unique_id=uid) as plan:
+            info = plan.info()
+            res["info"] = {k: info[k] for k in ("dist_candidates", "dist_nparts", "dist_exchange", "dist_repl_nparts")}
+            res["stats"] = plan.dist_stats()
+            if p2p:
+                bufs = plan.p2p_buffers(2)
+                info = plan.info()
+                res["info_p2p"] = {k: info[k] for k in ("dist_nparts", "dist_exchange")}
+                res["stats"] = plan.dist_stats()
+            else:
+                bufs = [torch.empty(n, dtype=torch.float64, device="cuda") for _ in range(2)]
+            sel = plan.select()
+            res["select"] = (sel.nparts, sel.exchange)
+            # automatic: the agreed distribution, iterated
+            x = torch.from_numpy(x0).cuda()
+            src = x
+            used = set()
+            for k in range(1, K + 1):
+                dst = bufs[k & 1]
+                dst.fill_(float("nan"))
+                u = plan.exec(src, dst, flags=pepp.Y_NEXT_INPUT)
+                used.add((u.nparts, u.exchange))
+                torch.cuda.synchronize()
+                res["ok"] &= bool(np.array_equal(dst.cpu().numpy()[rows], refs[k][rows]))
+                src = dst
+            res["used"] = sorted(used)
+            # replicated: every row on every rank
+            yr = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+            u = plan.exec(x, yr, flags=pepp.Y_REPLICATED)
+            torch.cuda.synchronize()
+            res["repl"] = (u.nparts, u.exchange, bool(np.array_equal(yr.cpu().numpy(), refs[1])))
+            # every candidate forced: same bits (own rows + ghosts after NEXT_INPUT, all rows after REPLICATED)
+            for parts, ex, _ in plan.dist_stats():
+                if ex == pepp.X_P2P:
+                    continue
+                f = pepp.Choice(pepp._capi.V_AUTO, 0, exchange=ex, nparts=parts)
+                a = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+                b = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+                plan.exec(x, a, flags=pepp.Y_NEXT_INPUT, force=f)
+                plan.exec(a, b, flags=pepp.Y_NEXT_INPUT, force=f)
+                c = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+                plan.exec(b, c, flags=pepp.Y_REPLICATED, force=f)
+                torch.cuda.synchronize()
+                res["forced"][(parts, ex)] = (bool(np.array_equal(b.cpu().numpy()[rows], refs[2][rows])) and
+                                              bool(np.array_equal(c.cpu().numpy(), refs[3])))
+            # host entry point, iterated, the exchange inside (REPLICATED output)
+            yh = np.full(n, np.nan)
+            plan.exec_host(x0, yh, iterations=K, flags=pepp.Y_REPLICATED)
+            res["host"] = bool(np.array_equal(yh, refs[K]))
+        outq.put((rank, res))
+    except Exception as e:
+        import traceback
+        outq.put((rank, {"error": repr(e) + traceback.format_exc()}))
+
+
+def _run_dist(name, world, K=5, p2p=False):
+    import torch.multiprocessing as mp
+    lib = _build_fake()
+    uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_dist_{world}_{int(p2p)}".encode() + b"\0" * 128)[:128]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker_dist, args=(r, world, lib, uid, name, K, q, p2p)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = {}
+    try:
+        for _ in range(world):
+            r, res = q.get(timeout=600)
+            out[r] = res
+    finally:
+        for p in procs:
+            p.join(timeout=60)
+            if p.is_alive():
+                p.kill()
+                p.join(10)
+    for r in range(world):
+        assert "error" not in out[r], out[r]["error"]
+    return out
+
+
+@pytest.mark.parametrize("name,world,p2p", [("lap", 2, False), ("zipf", 2, False), ("lap", 4, False),
+                                            ("lap", 2, True)])
+def test_distribution_choice_agreed_and_bitwise(name, world, p2p):
+    """Row a4 (P and exchange as timed choices): the plan times every
+    (P', exchange) candidate — P' in {nranks, nranks/2, ..., 1} x {halo,
+    allgather}, plus the fused push once buffers are registered — on every
+    rank; all ranks agree on the same choice (max-over-ranks means); the
+    automatic calls use it; every candidate forced gives the oracle's bits
+    (own rows + ghosts after NEXT_INPUT, every row after REPLICATED); the
+    host entry point too. 4 ranks exercise P' = 2 (point-to-point groups
+    among a subset of the ranks)."""
+    import paper_conf_sc_dastgeerlk12_b200 as pepp
+    out = _run_dist(name, world, p2p=p2p)
+    expect_parts = []
+    pp = world
+    while pp >= 1:
+        expect_parts.append(pp)
+        pp //= 2
+    for r in range(world):
+        res = out[r]
+        assert res["ok"] and res["host"], (r, res)
+        assert res["repl"][2] and res["repl"][1] == pepp.X_ALLGATHER
+        assert res["info"]["dist_candidates"] == 2 * len(expect_parts)
+        assert sorted({c[0] for c in res["stats"]}) == sorted(expect_parts)
+        assert all(c[2] > 0 for c in res["stats"])                # every candidate timed
+        assert all(res["forced"].values()) and len(res["forced"]) == 2 * len(expect_parts), res["forced"]
+        if p2p:
+            assert res["stats"][-1][1] == pepp.X_P2P
+    # every rank made the same choice, from the same agreed means
+    for key in ("info", "stats", "select", "used"):
+        assert all(out[r][key] == out[0][key] for r in range(world)), key
+    choice = out[0]["info"] if not p2p else out[0]["info_p2p"]
+    assert [tuple(u) for u in out[0]["used"]] == [(choice["dist_nparts"], choice["dist_exchange"])]
+    # the choice is the argmin of the agreed means (1 % tie rule)
+    stats = out[0]["stats"]
+    best = min(range(len(stats)), key=lambda i: stats[i][2])
+    chosen = [i for i, c in enumerate(stats) if (c[0], c[1]) == (choice["dist_nparts"], choice["dist_exchange"])][0]
+    assert stats[chosen][2] <= stats[best][2] * 1.0101

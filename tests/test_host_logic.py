@@ -190,3 +190,37 @@ def test_cold_start_prior_from_nearest_context():
     # a context with a different rank count never serves as a prior
     q3 = pepp.context_key(1 << 20, 1 << 20, 16 << 20, 0.0, nparts=4)
     assert H.prior(q3, ids) is None
+
+
+# ------------------------------------------------ distribution choice (a4)
+def test_dist_choose_max_over_ranks_then_argmin():
+    """P and exchange as timed choices (§8(a) a4, §V-D P@38827): a
+    partitioned call lasts as long as its slowest rank, so candidate d's
+    agreed time is the max over ranks; the choice is its argmin (A10 tie
+    rule). Injected times: rank 1 is slow on candidate 0, so candidate 2
+    (never the fastest on either rank alone) wins."""
+    means = [[10.0, 30.0, 12.0, 50.0],
+             [25.0, 11.0, 13.0, 40.0]]
+    c, agreed = pepp.dist_choose(means)
+    assert list(agreed) == [25.0, 30.0, 13.0, 50.0]
+    assert c == 2
+    # eligibility (e.g. REPLICATED calls: allgather candidates only)
+    c, _ = pepp.dist_choose(means, eligible=[True, True, False, True])
+    assert c == 0
+    # ties within 1 % go to the lower index; 2 % apart does not tie
+    c, _ = pepp.dist_choose([[100.0, 99.5]])
+    assert c == 0
+    c, _ = pepp.dist_choose([[100.0, 98.0]])
+    assert c == 1
+    # untimed (0) candidates are skipped
+    c, _ = pepp.dist_choose([[0.0, 5.0], [0.0, 6.0]])
+    assert c == 1
+
+
+def test_dist_choose_rejects_bad_input():
+    with pytest.raises(pepp.PeppError):
+        pepp.dist_choose([[1.0, float("nan")]])
+    with pytest.raises(pepp.PeppError):
+        pepp.dist_choose([[-1.0, 2.0]])
+    with pytest.raises(pepp.PeppError):
+        pepp.dist_choose([[1.0, 2.0]], eligible=[False, False])
