@@ -193,7 +193,7 @@ def parse_variant(s: str | None):
         return None
     name, _, prm = s.partition(":")
     v = {"csr_vector": pepp.V_CSR_VECTOR, "merge_path": pepp.V_MERGE_PATH, "sell": pepp.V_SELL,
-         "csr_stream": pepp.V_CSR_STREAM}[name]
+         "csr_stream": pepp.V_CSR_STREAM, "panel": pepp.V_PANEL}[name]
     return pepp.Choice(v, int(prm) if prm else 0)
 
 

@@ -63,7 +63,7 @@
 extern "C" {
 #endif
 
-#define PEPP_ABI_VERSION 7
+#define PEPP_ABI_VERSION 8
 
 typedef enum {
     PEPP_OK = 0,
@@ -84,7 +84,11 @@ typedef enum {
     PEPP_V_MERGE_PATH = 1,    /* merge-path over (row ends, nnz), smem-staged, deterministic carry fix-up */
     PEPP_V_SELL = 2,          /* SELL-C-σ, C = 32, column-major chunks; param = σ */
     PEPP_V_CSR_STREAM = 3,    /* CSR-stream fed by a TMA (cp.async.bulk) shared-memory pipeline; param = nnz per item */
-    PEPP_V_COUNT = 4
+    PEPP_V_PANEL = 4,         /* column panels for x far beyond L2 (random columns): the matrix stored panel-major,
+                                 one launch per panel of 2^param columns, (row, panel) pairs summed in order
+                                 (deterministic, no atomics); a candidate only when ncols x value size > 96 MB
+                                 and the mean row span exceeds half a panel; param = log2 panel width */
+    PEPP_V_COUNT = 5
 } pepp_variant_t;
 
 /* Exchange that makes y usable as the next x when the call is partitioned */

@@ -19,12 +19,12 @@ from typing import Optional, Sequence
 import numpy as np
 
 from . import _capi as C
-from ._capi import (ACCESS_READ, ACCESS_READWRITE, ACCESS_WRITE, DEVICE_SIMULATED, EXEC_NO_TIMING, PeppError, V_CSR_STREAM, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, X_ALLGATHER, X_AUTO,
+from ._capi import (ACCESS_READ, ACCESS_READWRITE, ACCESS_WRITE, DEVICE_SIMULATED, EXEC_NO_TIMING, PeppError, V_CSR_STREAM, V_CSR_VECTOR, V_MERGE_PATH, V_PANEL, V_SELL, X_ALLGATHER, X_AUTO,
                     X_HALO, X_NONE, X_P2P, Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, VARIANT_NAMES)
 
 __all__ = ["Plan", "Choice", "History", "Vector", "ACCESS_READ", "ACCESS_WRITE", "ACCESS_READWRITE",
            "DEVICE_SIMULATED", "partition_rows", "halo_ghosts", "context_key", "nccl_unique_id", "dist_choose",
-           "lib_path", "PeppError", "V_CSR_VECTOR", "V_MERGE_PATH", "V_SELL", "V_CSR_STREAM", "X_AUTO", "X_NONE",
+           "lib_path", "PeppError", "V_CSR_VECTOR", "V_MERGE_PATH", "V_SELL", "V_CSR_STREAM", "V_PANEL", "X_AUTO", "X_NONE",
            "X_ALLGATHER", "X_HALO", "X_P2P", "Y_LOCAL", "Y_NEXT_INPUT", "Y_REPLICATED", "EXEC_NO_TIMING",
            "VARIANT_NAMES"]
 

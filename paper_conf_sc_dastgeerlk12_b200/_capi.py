@@ -12,14 +12,15 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libpepp_spmv.so")
 
 PEPP_OK, PEPP_E_INVALID, PEPP_E_CUDA, PEPP_E_NCCL, PEPP_E_NOMEM, PEPP_E_UNSUPPORTED, PEPP_E_STATE = 0, -1, -2, -3, -4, -5, -6
-V_AUTO, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, V_CSR_STREAM, V_COUNT = -1, 0, 1, 2, 3, 4
+V_AUTO, V_CSR_VECTOR, V_MERGE_PATH, V_SELL, V_CSR_STREAM, V_PANEL, V_COUNT = -1, 0, 1, 2, 3, 4, 5
 X_AUTO, X_NONE, X_ALLGATHER, X_HALO, X_P2P = -1, 0, 1, 2, 3
 Y_LOCAL, Y_NEXT_INPUT, Y_REPLICATED, EXEC_NO_TIMING = 0x0, 0x1, 0x2, 0x10
 ACCESS_READ, ACCESS_WRITE, ACCESS_READWRITE = 1, 2, 3
 VALUE_F64, VALUE_F32 = 0, 1
 DEVICE_SIMULATED = -2
 KEY_F32, KEY_COMPRESS, KEY_DIST = 0x1, 0x2, 0x4
-VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell", V_CSR_STREAM: "csr_stream"}
+VARIANT_NAMES = {V_CSR_VECTOR: "csr_vector", V_MERGE_PATH: "merge_path", V_SELL: "sell", V_CSR_STREAM: "csr_stream",
+                 V_PANEL: "panel"}
 EXCHANGE_NAMES = {X_NONE: "none", X_ALLGATHER: "allgather", X_HALO: "halo", X_P2P: "p2p", X_AUTO: "auto"}
 
 c_i32, c_i64, c_u32, c_u64, c_f64, c_vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_uint64,
@@ -135,7 +136,7 @@ class PeppError(RuntimeError):
         super().__init__(f"{where}: {status_str(status)} ({status})" + (f": {detail}" if detail else ""))
 
 
-ABI_VERSION = 7   # PEPP_ABI_VERSION of include/pepp_spmv.h
+ABI_VERSION = 8   # PEPP_ABI_VERSION of include/pepp_spmv.h
 
 
 def lib() -> ctypes.CDLL:

@@ -1097,6 +1097,100 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
                  ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
 }
 
+// =====================================================================
+// Variant 4: column panels — random columns whose x is far larger than L2.
+// With x beyond L2 (e.g. 10^8 columns = 800 MB) every random gather of the
+// row-major variants is a DRAM access of its own (~50 G gathers/s). Here the
+// columns are cut into panels of 2^P entries (x panel <= 64 MB, L2-resident
+// while it is used) and the matrix is stored panel-major: for panel k, the
+// (row, entries) pairs of the rows that have entries in it, in row order,
+// each pair's entries contiguous (pcol / pval, their CSR order). One launch
+// per panel, one thread per pair: the row's panel entries summed
+// sequentially (product rounded by FMA, ascending column), then
+// y[row] += that sum — rows are owned by one thread per panel and the
+// panels run in order, so no atomics and the same bits on every call (y is
+// zeroed first; row i's result is (((0 + s_0) + s_1) + ...) over the panels
+// holding its entries).
+// =====================================================================
+template <typename T>
+__global__ void __launch_bounds__(256) panel_kernel(int j0, int j1, const int* __restrict__ prow,
+                                                    const int* __restrict__ pstart, const int* __restrict__ pcol,
+                                                    const T* __restrict__ pval, const T* __restrict__ x,
+                                                    T* __restrict__ y) {
+    const uint64_t pol = evict_first_policy();
+    for (int j = j0 + blockIdx.x * blockDim.x + threadIdx.x; j < j1; j += gridDim.x * blockDim.x) {
+        const int r = __ldg(prow + j), s = __ldg(pstart + j), e = __ldg(pstart + j + 1);
+        T acc = T(0);
+        for (int k = s; k < e; ++k) acc = fma(ld_stream_v(pval + k, pol), __ldg(x + ld_stream_i(pcol + k, pol)), acc);
+        y[r] += acc;
+    }
+}
+
+// plan-time helpers of the panel layout
+// sum over rows of (largest - smallest column): the plan's test whether rows
+// reach across x (random columns) or stay near the diagonal (bands, stencils)
+__global__ void row_span_kernel(int64_t nrows, const int* __restrict__ rp, const int* __restrict__ col,
+                                unsigned long long* __restrict__ total) {
+    unsigned long long acc = 0;
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < nrows; r += (int64_t)gridDim.x * blockDim.x) {
+        int lo = INT32_MAX, hi = -1;
+        for (int k = rp[r]; k < rp[r + 1]; ++k) { lo = min(lo, col[k]); hi = max(hi, col[k]); }
+        if (hi >= lo) acc += (unsigned long long)(hi - lo);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if ((threadIdx.x & 31) == 0) atomicAdd(total, acc);
+}
+
+// entry positions k of the plan's CSR copy (k in [pad, pad + nnz)) ->
+// slot k - pad: its panel key, its row, and k itself (the sort's payload)
+__global__ void panel_keys_kernel(int64_t nrows, const int* __restrict__ rp, const int* __restrict__ col, int lg, int pad,
+                                  unsigned char* __restrict__ key, int* __restrict__ row_of, int* __restrict__ idx) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < nrows; r += (int64_t)gridDim.x * blockDim.x)
+        for (int k = rp[r]; k < rp[r + 1]; ++k) {
+            key[k - pad] = (unsigned char)(col[k] >> lg);
+            row_of[k - pad] = (int)r;
+            idx[k - pad] = k;
+        }
+}
+// sorted keys -> first position of each present panel
+__global__ void panel_bounds_kernel(int64_t n, const unsigned char* __restrict__ skey, int64_t* __restrict__ zoff) {
+    for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n; p += (int64_t)gridDim.x * blockDim.x)
+        if (p == 0 || skey[p] != skey[p - 1]) zoff[skey[p]] = p;
+}
+// per panel k: the first pair whose entries start at or after zoff[k]
+__global__ void panel_pair_offsets_kernel(int npanels, const int64_t* __restrict__ zoff, const int* __restrict__ pstart,
+                                          int64_t npairs, int* __restrict__ poff) {
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k > npanels) return;
+    int64_t lo = 0, hi = npairs;
+    while (lo < hi) {
+        const int64_t m = (lo + hi) / 2;
+        if ((int64_t)pstart[m] < zoff[k]) lo = m + 1;
+        else hi = m;
+    }
+    poff[k] = (int)lo;
+}
+template <typename T>
+__global__ void panel_gather_kernel(int64_t n, int pad, const int* __restrict__ sidx, const int* __restrict__ col,
+                                    const T* __restrict__ val, const int* __restrict__ row_of,
+                                    const unsigned char* __restrict__ skey, int* __restrict__ pcol, T* __restrict__ pval,
+                                    int* __restrict__ prow_full, unsigned char* __restrict__ head) {
+    for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n; p += (int64_t)gridDim.x * blockDim.x) {
+        const int k = sidx[p];
+        pcol[p] = col[k];
+        pval[p] = val[k];
+        const int r = row_of[k - pad];
+        prow_full[p] = r;
+        head[p] = p == 0 || skey[p] != skey[p - 1] || row_of[sidx[p - 1] - pad] != r;
+    }
+}
+__global__ void panel_pairs_kernel(int64_t npairs, const int* __restrict__ starts, const int* __restrict__ prow_full,
+                                   int* __restrict__ prow) {
+    for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < npairs; j += (int64_t)gridDim.x * blockDim.x)
+        prow[j] = prow_full[starts[j]];
+}
+
 constexpr int kStreamVecFlag = 0x40000000;   // item.y flag: the item holds a row longer than VEC
 
 template <int NB, int RMAX, typename T>

@@ -14,6 +14,8 @@
 
 #include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
+#include <cub/device/device_select.cuh>
+#include <thrust/iterator/counting_iterator.h>
 
 #include <algorithm>
 #include <chrono>
@@ -80,6 +82,17 @@ struct PeerXfer {            // halo traffic with one peer
     int64_t contig_start;    // >= 0: the entries are y[contig_start, contig_start+count)
     int* d_idx = nullptr;    // else: global indices into y (device)
     void* d_buf = nullptr;   // pack / unpack buffer (value type)
+};
+
+// Column-panel layout (PEPP_V_PANEL) for one panel width 2^lg
+struct PanelLayout {
+    int lg = 0, npanels = 0;
+    int64_t npairs = 0;
+    int* d_prow = nullptr;        // [npairs] row of each (row, panel) pair, panel-major, row order within a panel
+    int* d_pstart = nullptr;      // [npairs + 1] first entry of each pair in pcol / pval
+    int* d_pcol = nullptr;        // [nnz] columns, panel-major
+    void* d_pval = nullptr;       // [nnz] values (plan value type)
+    std::vector<int> poff;        // [npanels + 1] pair range of each panel
 };
 
 // Distribution candidates (opts.dist_select, §8(a) a4: P and exchange are
@@ -158,6 +171,9 @@ struct pepp_spmv_plan_s {
     int64_t sell_long_nnz = 0;       // entries of the rows the mid / long-row kernels sum
     int64_t sell_bytes = 0;          // DRAM bytes one SELL call streams with this layout (layout_bytes)
     void* d_sell_part = nullptr;     // segment partials (8-byte slots)
+
+    // column panels (x beyond L2)
+    std::vector<PanelLayout> panels;
 
     // merge path
     int ntiles = 0;
@@ -339,6 +355,8 @@ void free_plan(pepp_spmv_plan_t* p) {
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
         for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
+    for (auto& pl : p->panels)
+        for (void* b : {(void*)pl.d_prow, (void*)pl.d_pstart, (void*)pl.d_pcol, pl.d_pval}) if (b) cudaFree(b);
     for (auto& dp : p->dparts) {
         for (auto* v : {&dp.recv_x, &dp.send_x, &dp.recv_g, &dp.send_g})
             for (auto& t : *v) { if (t.d_idx) cudaFree(t.d_idx); if (t.d_buf) cudaFree(t.d_buf); }
@@ -815,6 +833,121 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
     return PEPP_OK;
 }
 
+// ---------------------------------------------------------------- panel prep
+// The column-panel layout (variant PEPP_V_PANEL) pays only where x is far
+// larger than L2 and the rows reach across it (random columns): x > 96 MB
+// and a mean row span (last - first column) above half a panel. One layout
+// per panel width 2^lg (x panel of 32 MB and, when memory is modest, 64 MB):
+// a stable radix sort of the entries by panel (CSR order kept within a
+// panel), the (row, panel) pairs by head flags (cub select), their pair
+// ranges per panel by binary search.
+constexpr int64_t kPanelMinX = 96ll << 20;
+
+pepp_status_t prepare_panels(pepp_spmv_plan_t* p, cudaStream_t st, std::vector<int>* lgs) {
+    lgs->clear();
+    const int64_t n = p->nnz, R = p->nrows;
+    if (p->ncols * (int64_t)p->esz <= kPanelMinX || n == 0 || R == 0) return PEPP_OK;
+    // mean row span
+    {
+        DevTmp<unsigned long long> d_span;
+        PEPP_CUDA_TRY(d_span.alloc(1));
+        PEPP_CUDA_TRY(cudaMemsetAsync(d_span.p, 0, sizeof(unsigned long long), st));
+        pepp::k::row_span_kernel<<<std::min<int64_t>((R + 255) / 256, (int64_t)p->sm_count * 8), 256, 0, st>>>(
+            R, p->d_rp, p->d_col, d_span.p);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        unsigned long long span = 0;
+        PEPP_CUDA_TRY(cudaMemcpyAsync(&span, d_span.p, sizeof(span), cudaMemcpyDeviceToHost, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        const int lg0 = p->esz == 8 ? 22 : 23;   // 32 MB of x per panel
+        if ((double)span / (double)R < (double)(1ll << (lg0 - 1))) return PEPP_OK;
+        lgs->push_back(lg0);
+        if ((double)n * 2.0 * (4.0 + (double)p->esz) <= 48e9) lgs->push_back(lg0 + 1);   // and 64 MB, memory permitting
+    }
+    std::vector<int> ok;
+    for (int lg : *lgs) {
+        const int npanels = (int)((p->ncols + (1ll << lg) - 1) >> lg);
+        if (npanels < 2 || npanels > 255) continue;
+        PanelLayout L;
+        L.lg = lg;
+        L.npanels = npanels;
+        pepp_status_t s;
+        DevTmp<unsigned char> key, skey, head;
+        DevTmp<int> idx, sidx, row_of, prow_full, starts;
+        DevTmp<int> nsel;
+        DevTmp<unsigned char> tmp;
+        PEPP_CUDA_TRY(key.alloc(n));
+        PEPP_CUDA_TRY(skey.alloc(n));
+        PEPP_CUDA_TRY(idx.alloc(n));
+        PEPP_CUDA_TRY(sidx.alloc(n));
+        PEPP_CUDA_TRY(row_of.alloc(n));
+        const int gb = (int)std::min<int64_t>((R + 255) / 256, (int64_t)p->sm_count * 16);
+        pepp::k::panel_keys_kernel<<<gb, 256, 0, st>>>(R, p->d_rp, p->d_col, lg, p->pad, key.p, row_of.p, idx.p);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        int end_bit = 1;
+        while ((1 << end_bit) < npanels) ++end_bit;
+        size_t tb = 0;
+        PEPP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, key.p, skey.p, idx.p, sidx.p, (int)n, 0, end_bit, st));
+        PEPP_CUDA_TRY(tmp.alloc(tb));
+        PEPP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp.p, tb, key.p, skey.p, idx.p, sidx.p, (int)n, 0, end_bit, st));
+        { DevTmp<unsigned char> k2; std::swap(k2.p, key.p); DevTmp<int> i2; std::swap(i2.p, idx.p); }   // free early
+        if ((s = dalloc(p, &L.d_pcol, n))) return s;
+        if ((s = dalloc_bytes(p, &L.d_pval, n * (int64_t)p->esz))) { cudaFree(L.d_pcol); return s; }
+        PEPP_CUDA_TRY(prow_full.alloc(n));
+        PEPP_CUDA_TRY(head.alloc(n));
+        const int gn = (int)std::min<int64_t>((n + 255) / 256, (int64_t)p->sm_count * 32);
+        if (p->vt == PEPP_VALUE_F32)
+            pepp::k::panel_gather_kernel<float><<<gn, 256, 0, st>>>(n, p->pad, sidx.p, p->d_col, (const float*)p->d_val,
+                                                                   row_of.p, skey.p, L.d_pcol, (float*)L.d_pval, prow_full.p, head.p);
+        else
+            pepp::k::panel_gather_kernel<double><<<gn, 256, 0, st>>>(n, p->pad, sidx.p, p->d_col, (const double*)p->d_val,
+                                                                    row_of.p, skey.p, L.d_pcol, (double*)L.d_pval, prow_full.p, head.p);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        PEPP_CUDA_TRY(starts.alloc(n + 1));
+        PEPP_CUDA_TRY(nsel.alloc(1));
+        thrust::counting_iterator<int> it(0);
+        size_t tb2 = 0;
+        PEPP_CUDA_TRY(cub::DeviceSelect::Flagged(nullptr, tb2, it, head.p, starts.p, nsel.p, (int)n, st));
+        DevTmp<unsigned char> tmp2;
+        PEPP_CUDA_TRY(tmp2.alloc(tb2));
+        PEPP_CUDA_TRY(cub::DeviceSelect::Flagged(tmp2.p, tb2, it, head.p, starts.p, nsel.p, (int)n, st));
+        int np = 0;
+        PEPP_CUDA_TRY(cudaMemcpyAsync(&np, nsel.p, sizeof(int), cudaMemcpyDeviceToHost, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        L.npairs = np;
+        if ((s = dalloc(p, &L.d_prow, np))) { cudaFree(L.d_pcol); cudaFree(L.d_pval); return s; }
+        if ((s = dalloc(p, &L.d_pstart, (int64_t)np + 1))) { cudaFree(L.d_pcol); cudaFree(L.d_pval); cudaFree(L.d_prow); return s; }
+        const int nn = (int)n;
+        PEPP_CUDA_TRY(cudaMemcpyAsync(L.d_pstart, starts.p, sizeof(int) * np, cudaMemcpyDeviceToDevice, st));
+        PEPP_CUDA_TRY(cudaMemcpyAsync(L.d_pstart + np, &nn, sizeof(int), cudaMemcpyHostToDevice, st));
+        pepp::k::panel_pairs_kernel<<<(int)std::min<int64_t>(((int64_t)np + 255) / 256, (int64_t)p->sm_count * 32), 256, 0, st>>>(
+            np, starts.p, prow_full.p, L.d_prow);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        // pair ranges per panel
+        DevTmp<int64_t> zoff;
+        DevTmp<int> poff;
+        PEPP_CUDA_TRY(zoff.alloc(npanels + 1));
+        PEPP_CUDA_TRY(poff.alloc(npanels + 1));
+        std::vector<int64_t> hz(npanels + 1, -1);
+        PEPP_CUDA_TRY(cudaMemcpyAsync(zoff.p, hz.data(), sizeof(int64_t) * (npanels + 1), cudaMemcpyHostToDevice, st));
+        pepp::k::panel_bounds_kernel<<<gn, 256, 0, st>>>(n, skey.p, zoff.p);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        PEPP_CUDA_TRY(cudaMemcpyAsync(hz.data(), zoff.p, sizeof(int64_t) * (npanels + 1), cudaMemcpyDeviceToHost, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        hz[npanels] = n;
+        for (int k = npanels - 1; k >= 0; --k) if (hz[k] < 0) hz[k] = hz[k + 1];   // empty panels
+        PEPP_CUDA_TRY(cudaMemcpyAsync(zoff.p, hz.data(), sizeof(int64_t) * (npanels + 1), cudaMemcpyHostToDevice, st));
+        pepp::k::panel_pair_offsets_kernel<<<(npanels + 1 + 255) / 256, 256, 0, st>>>(npanels, zoff.p, L.d_pstart, np, poff.p);
+        PEPP_CUDA_TRY(cudaGetLastError());
+        L.poff.resize(npanels + 1);
+        PEPP_CUDA_TRY(cudaMemcpyAsync(L.poff.data(), poff.p, sizeof(int) * (npanels + 1), cudaMemcpyDeviceToHost, st));
+        PEPP_CUDA_TRY(cudaStreamSynchronize(st));
+        p->panels.push_back(std::move(L));
+        ok.push_back(lg);
+    }
+    *lgs = ok;
+    return PEPP_OK;
+}
+
 // ---------------------------------------------------------------- merge prep
 // Runs of >= kLongRun consecutive tiles that carry into the same row (the row
 // open at a tile's end is tile_coord[t+1].x, fixed by the structure).
@@ -1033,6 +1166,19 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
             pepp::k::sell_long_kernel<256, T><<<p->nsell_seg, 256, 0, st>>>(
                 p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, (T*)p->d_sell_part, p->d_col, val, x, y);
         break;
+    case PEPP_V_PANEL: {
+        const PanelLayout* L = nullptr;
+        for (const auto& pl : p->panels) if (pl.lg == c.param) L = &pl;
+        if (!L) return PEPP_E_INVALID;
+        if (cudaMemsetAsync(y, 0, sizeof(T) * p->nrows, st) != cudaSuccess) return PEPP_E_CUDA;
+        for (int k = 0; k < L->npanels; ++k) {
+            const int j0 = L->poff[k], j1 = L->poff[k + 1];
+            if (j1 <= j0) continue;
+            const int g = (int)std::min<int64_t>(((int64_t)j1 - j0 + 255) / 256, (int64_t)p->sm_count * 16);
+            pepp::k::panel_kernel<T><<<g, 256, 0, st>>>(j0, j1, L->d_prow, L->d_pstart, L->d_pcol, (const T*)L->d_pval, x, y);
+        }
+        break;
+    }
     default:
         return PEPP_E_INVALID;
     }
@@ -1049,6 +1195,14 @@ int launches_for(const pepp_spmv_plan_t* p, const Candidate& c) {
         return p->ntiles > 0 ? 2 + (p->nlongruns > 0) : 0;
     case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
     case PEPP_V_SELL: return (p->d_stlist ? 1 + (p->ngen > 0) : 1) + (p->nsell_mid > 0) + (p->nsell_seg > 0);
+    case PEPP_V_PANEL:
+        for (const auto& pl : p->panels)
+            if (pl.lg == c.param) {
+                int k = 0;
+                for (int i = 0; i < pl.npanels; ++i) k += pl.poff[i + 1] > pl.poff[i];
+                return k;
+            }
+        return 0;
     default: return 0;
     }
 }
@@ -2114,6 +2268,12 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
         if ((s = prepare_stream(p, st))) return s;
         p->cands.push_back({PEPP_V_CSR_STREAM, kStreamNB});
     }
+    if (mask & (1u << PEPP_V_PANEL)) {   // only where x is far beyond L2 and rows reach across it
+        std::vector<int> lgs;
+        if ((s = prepare_panels(p, st, &lgs))) return s;
+        for (int lg : lgs) p->cands.push_back({PEPP_V_PANEL, lg});
+    }
+    if (p->cands.empty()) return PEPP_E_UNSUPPORTED;
     p->eligible.assign(p->cands.size(), 1);
     p->pending.assign(p->cands.size(), 0);
     p->warmed.assign(p->cands.size(), 0);
@@ -2128,6 +2288,12 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
                 b += (nt + 1) * 8 + nt * 2 * (4 + 8);   // tile coordinates, carries written and read back
             } else if (c.variant == PEPP_V_CSR_STREAM) {
                 b += (int64_t)p->nitems * 16 + (int64_t)p->nlong * 16;
+            } else if (c.variant == PEPP_V_PANEL) {
+                // entries (column + value), pairs (row + start), y zeroed then
+                // read and written once per pair, x read once
+                int64_t np = 0;
+                for (const auto& pl : p->panels) if (pl.lg == c.param) np = pl.npairs;
+                b = A->nnz * (es + 4) + np * (8 + 2 * es) + A->nrows * es + A->ncols * es;
             }
             p->cand_bytes.push_back(b);
         }

@@ -303,10 +303,12 @@ def test_selector_calibrates_then_picks_fastest_measured():
             if not u.calibrating:
                 break
             seen.append(u.candidate)
-        # round 1 visits every candidate; later rounds skip the ones ruled out,
-        # rounds 4..9 (refinement) only the contenders within 10 % of the best;
-        # each candidate's first timed call is a warm-up (not recorded): +1 each
-        assert seen[:n] == list(range(n))
+        # round 1 visits every candidate in index order (a candidate whose
+        # warm-up call — its first timed call, not recorded — already came back
+        # is issued again right away); later rounds skip the ones ruled out,
+        # rounds 4..9 (refinement) only the contenders within 10 % of the best
+        first_seen = list(dict.fromkeys(seen))
+        assert first_seen == list(range(n))
         assert len(seen) <= 10 * n
         plan.flush_history()
         means = [plan.history_stats(c)[1] for c in range(n)]
