@@ -750,3 +750,73 @@ def test_binding_refuses_bad_operands():
         plan.exec(x, y)
         torch.cuda.synchronize()
         assert np.array_equal(y.cpu().numpy(), oracle.spmv(A, x0))
+
+
+# ------------------------------------------------- column panels (variant 4)
+def _wide(nrows, ncols, seed, val_mode, dt=np.float64):
+    A = gen.uniform(nrows, ncols, 16, seed=seed, val_mode=val_mode)
+    return A if dt == np.float64 else gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float32), A.r0,
+                                              A.global_nrows)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_panel_variant_parity(dt):
+    """x beyond the 96 MB threshold with random columns: the column-panel
+    candidates exist (32 and 64 MB panels) and match the oracle — integer
+    inputs bit-exact, real inputs within the bound, the same bits on every
+    call (panel order fixed, no atomics), Inf/NaN in x propagated exactly."""
+    ncols = (1 << 24) if dt == np.float64 else (1 << 25)          # x = 128 MB
+    tdt = torch.float64 if dt == np.float64 else torch.float32
+    A = _wide(150_000, ncols, 61, gen.INT4, dt)
+    x = gen.vector(62, gen.INT8, ncols).astype(dt)
+    ref = oracle.spmv(A, x)
+    with pepp.Plan.from_csr(A) as plan:
+        pan = [c for c in plan.candidates() if c.variant == pepp.V_PANEL]
+        assert [c.param for c in pan] == ([22, 23] if dt == np.float64 else [23, 24])
+        xd = torch.from_numpy(x).cuda()
+        y = torch.full((A.nrows,), float("nan"), dtype=tdt, device="cuda")
+        for c in pan:
+            f = pepp.Choice(c.variant, c.param)
+            plan.exec(xd, y, force=f)
+            torch.cuda.synchronize()
+            y1 = y.cpu().numpy()
+            assert oracle.equal(y1, ref).all(), c.name
+            plan.exec(xd, y, force=f)
+            torch.cuda.synchronize()
+            assert np.array_equal(y.cpu().numpy(), y1)
+            assert c.layout_bytes > A.nnz * (4 + np.dtype(dt).itemsize)
+        # real values
+        R = gen.with_values(_wide(150_000, ncols, 61, gen.INT4), 63, gen.REAL)
+        R = R if dt == np.float64 else gen.CSR(R.nrows, R.ncols, R.row_ptr, R.col, R.val.astype(np.float32), R.r0,
+                                               R.global_nrows)
+        xr = gen.vector(64, gen.REAL, ncols).astype(dt)
+    with pepp.Plan.from_csr(R) as plan:
+        xd = torch.from_numpy(xr).cuda()
+        y = torch.empty(R.nrows, dtype=tdt, device="cuda")
+        refr = oracle.spmv(R, xr)
+        tol = oracle.bound(R, xr.astype(np.float64)) if dt == np.float64 else oracle.bound_f32(R, xr)
+        for c in plan.candidates():
+            if c.variant != pepp.V_PANEL:
+                continue
+            plan.exec(xd, y, force=pepp.Choice(c.variant, c.param))
+            torch.cuda.synchronize()
+            assert oracle.within(y.cpu().numpy().astype(np.float64), refr.astype(np.float64), tol).all(), c.name
+        # non-finite x
+        xn = xr.copy()
+        xn[::997] = np.inf
+        xn[5::1999] = np.nan
+        refn = oracle.spmv(R, xn)
+        plan.exec(torch.from_numpy(xn).cuda(), y, force=pepp.Choice(pepp.V_PANEL, 0))
+        torch.cuda.synchronize()
+        yn = y.cpu().numpy().astype(np.float64)
+        fin = np.isfinite(refn)
+        assert np.array_equal(np.isnan(yn), np.isnan(refn)) and np.array_equal(yn[np.isinf(refn)], refn[np.isinf(refn)])
+        assert oracle.within(yn[fin], refn[fin].astype(np.float64), tol[fin]).all()
+
+
+def test_panel_variant_absent_where_it_cannot_pay():
+    """Banded / stencil rows (span << a panel) and small x get no panel candidate."""
+    with pepp.Plan.from_csr(gen.laplacian2d(2048)) as plan:        # x = 32 MB
+        assert not any(c.variant == pepp.V_PANEL for c in plan.candidates())
+    with pepp.Plan.from_csr(gen.banded(20_000_000, 4, seed=100)) as plan:   # x = 160 MB, span 8
+        assert not any(c.variant == pepp.V_PANEL for c in plan.candidates())
