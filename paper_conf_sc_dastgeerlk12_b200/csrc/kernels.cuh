@@ -644,8 +644,11 @@ using SellPatternArg = std::conditional_t<PAT, SellPatterns<T>, NoPatterns>;
 
 // PAT: the plan has pattern chunks (phase A + genlist); PAT = false compiles
 // the general kernel without them (no extra registers, no 3 KB parameter).
+#ifndef PEPP_PAT_MINB
+#define PEPP_PAT_MINB 1   // experiments: minimum resident blocks per SM for the PAT (value-compressed) instances
+#endif
 template <int BLOCK, bool SORTED, bool PAT, typename T>
-__global__ void __launch_bounds__(BLOCK) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
+__global__ void __launch_bounds__(BLOCK, (PAT && !SORTED) ? PEPP_PAT_MINB : 1) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
                                                      const int* __restrict__ chunk_len,
                                                      const int* __restrict__ rowlen,
                                                      const int* __restrict__ perm,

@@ -11,7 +11,8 @@ import gen
 import paper_conf_sc_dastgeerlk12_b200 as pepp
 
 peak = json.load(open("MEASURED_PEAKS.json"))["hbm_gbs"] if os.path.exists("MEASURED_PEAKS.json") else 6545.0
-for n, dt in [(8192, "f64"), (8192, "f32"), (4096, "f64")]:
+for n, dt in [tuple(a.split(":")) for a in (sys.argv[1:] or ["8192:f64", "8192:f32", "4096:f64"])]:
+    n = int(n)
     A = gen.laplacian2d(n)
     if dt == "f32":
         A = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float32), A.r0, A.global_nrows)

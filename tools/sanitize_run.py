@@ -89,6 +89,16 @@ def main() -> int:
         plan.exec_host_batch(xs, ys, iterations=2)
         for xk, yk in zip(xs, ys):
             bad += 0 if np.array_equal(yk, oracle.spmv(A, oracle.spmv(A, xk))) else 1
+    # column panels (x > 96 MB, random columns): both panel widths
+    W = gen.uniform(20_000, 1 << 24, 8, seed=61, val_mode=gen.INT4)
+    xw = gen.vector(62, gen.INT8, W.ncols)
+    with pepp.Plan.from_csr(W, variant_mask=1 << pepp.V_PANEL) as plan:
+        yw = torch.full((W.nrows,), float("nan"), dtype=torch.float64, device="cuda")
+        xwd = torch.from_numpy(xw).cuda()
+        for c in plan.candidates():
+            plan.exec(xwd, yw, force=pepp.Choice(c.variant, c.param))
+            torch.cuda.synchronize()
+            bad += 0 if np.array_equal(yw.cpu().numpy(), oracle.spmv(W, xw)) else 1
     print("sanitize_run: mismatches =", bad)
     return 1 if bad else 0
 
