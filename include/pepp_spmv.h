@@ -293,7 +293,15 @@ typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a t
 /* Human-readable name of a status code (static storage; never NULL). */
 const char* pepp_status_str(pepp_status_t s);
 
-/* Fill *opts with the defaults documented above. */
+/* Fill *opts with the defaults documented above. The composition tool's
+   global switches (the paper's disableImpls, P@16687, and useHistoryModels,
+   "per component or global", P@28058) can be given as environment defaults,
+   read here only (fields a caller sets afterwards win — the per-component
+   form): PEPP_VARIANT = comma list of csr_vector, merge_path, sell,
+   csr_stream, panel (the allowed variants -> variant_mask; no known name =
+   all); PEPP_USE_HISTORY = 0 / 1 (use_history); PEPP_HISTORY_PATH = file
+   (history_path; the string must stay in the environment while the options
+   are used). */
 void pepp_spmv_opts_default(pepp_spmv_opts_t* opts);
 
 /* Build a plan for A on opts->device. Copies A; the plan owns all device

@@ -91,8 +91,8 @@ class Plan:
     plan copies them.
     """
 
-    def __init__(self, nrows: int, ncols: int, row_ptr, col, val, *, variant_mask: int = 0,
-                 use_history: bool = True, validate: bool = True, sell_sigma: int = 0,
+    def __init__(self, nrows: int, ncols: int, row_ptr, col, val, *, variant_mask: Optional[int] = None,
+                 use_history: Optional[bool] = None, validate: bool = True, sell_sigma: int = 0,
                  device: Optional[int] = None, min_samples: int = 3, sample_period: int = 8,
                  nranks: int = 1, rank: int = 0, row_bounds: Optional[Sequence[int]] = None,
                  nccl_unique_id: Optional[bytes] = None, exchange: int = X_AUTO,
@@ -116,8 +116,12 @@ class Plan:
                     _ptr(val) if nnz else 0, 1 if on_dev else 0, self.value_type)
         o = C.OPTS_T()
         L.pepp_spmv_opts_default(ctypes.byref(o))
-        o.variant_mask = variant_mask
-        o.use_history = 1 if use_history else 0
+        # None keeps pepp_spmv_opts_default's value (which honours the global
+        # switches PEPP_VARIANT / PEPP_USE_HISTORY / PEPP_HISTORY_PATH)
+        if variant_mask is not None:
+            o.variant_mask = variant_mask
+        if use_history is not None:
+            o.use_history = 1 if use_history else 0
         o.validate = 1 if validate else 0
         o.sell_sigma = sell_sigma
         o.device = -1 if device is None else device
@@ -134,7 +138,8 @@ class Plan:
             o.nccl_unique_id = ctypes.addressof(self._uid)
         o.exchange = exchange
         self._hp = history_path.encode() if history_path else None
-        o.history_path = self._hp
+        if self._hp is not None:
+            o.history_path = self._hp
         o.prune = 1 if prune else 0
         o.overlap = 1 if overlap else 0
         o.compress_values = 1 if compress_values else 0

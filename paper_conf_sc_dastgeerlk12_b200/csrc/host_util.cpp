@@ -12,9 +12,11 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <unordered_map>
+#include <string>
 #include <vector>
 
 namespace {
@@ -63,6 +65,29 @@ extern "C" PEPP_API void pepp_spmv_opts_default(pepp_spmv_opts_t* o) {
     o->overlap = 1;
     o->compress_values = 1;
     o->dist_select = 1;
+    // the composition tool's global switches (§IV: disableImpls P@16687,
+    // useHistoryModels "per component or global" P@28058) as environment
+    // defaults: they set the defaults only — options a caller sets after
+    // this call (the per-component form) win
+    if (const char* v = std::getenv("PEPP_VARIANT")) {
+        uint32_t m = 0;
+        std::string list(v);
+        size_t i = 0;
+        while (i <= list.size()) {
+            size_t j = list.find(',', i);
+            if (j == std::string::npos) j = list.size();
+            const std::string t = list.substr(i, j - i);
+            if (t == "csr_vector") m |= 1u << PEPP_V_CSR_VECTOR;
+            else if (t == "merge_path") m |= 1u << PEPP_V_MERGE_PATH;
+            else if (t == "sell") m |= 1u << PEPP_V_SELL;
+            else if (t == "csr_stream") m |= 1u << PEPP_V_CSR_STREAM;
+            else if (t == "panel") m |= 1u << PEPP_V_PANEL;
+            i = j + 1;
+        }
+        o->variant_mask = m;   // unknown names only: 0 = every variant
+    }
+    if (const char* v = std::getenv("PEPP_USE_HISTORY")) o->use_history = std::atoi(v) != 0;
+    if (const char* v = std::getenv("PEPP_HISTORY_PATH")) if (*v) o->history_path = v;
 }
 
 // ---------------------------------------------------------------- partition

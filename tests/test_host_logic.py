@@ -224,3 +224,24 @@ def test_dist_choose_rejects_bad_input():
         pepp.dist_choose([[-1.0, 2.0]])
     with pytest.raises(pepp.PeppError):
         pepp.dist_choose([[1.0, 2.0]], eligible=[False, False])
+
+
+def test_global_switches_from_environment():
+    """The paper's global tool switches (disableImpls P@16687, useHistoryModels
+    P@28058) as environment defaults of pepp_spmv_opts_default; explicit
+    options set afterwards win (the per-component form)."""
+    import subprocess
+    import sys
+    code = ("import ctypes, paper_conf_sc_dastgeerlk12_b200._capi as C; o = C.OPTS_T(); "
+            "C.lib().pepp_spmv_opts_default(ctypes.byref(o)); "
+            "print(o.variant_mask, o.use_history, (o.history_path or b'').decode())")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    base = {k: v for k, v in os.environ.items() if not k.startswith("PEPP_")}
+    out = subprocess.run([sys.executable, "-c", code], env=base, capture_output=True, text=True, cwd=root)
+    assert out.stdout.split() == ["0", "1"], out.stderr
+    env = dict(base, PEPP_VARIANT="sell,merge_path", PEPP_USE_HISTORY="0", PEPP_HISTORY_PATH="/tmp/h.txt")
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, cwd=root)
+    assert out.stdout.split() == [str((1 << pepp.V_SELL) | (1 << pepp.V_MERGE_PATH)), "0", "/tmp/h.txt"], out.stderr
+    env = dict(base, PEPP_VARIANT="nonsense")
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, cwd=root)
+    assert out.stdout.split()[0] == "0"
