@@ -71,3 +71,36 @@ def test_reported_launches_match_profiler():
                     torch.cuda.synchronize()
                 seen = sum(e.count for e in prof.key_averages() if "pepp::" in e.key)
                 assert u.launches == seen > 0, (A.name, f.name, u.launches, seen)
+
+
+def test_graph_of_uncalibrated_plan_captures_frozen_choice():
+    """pepp_spmv_graph_create on a plan that has timed nothing yet
+    captures the frozen choice (best measured, else the static heuristic —
+    SELL on the Laplacian: mean <= 12, CV <= 0.5), not the first calibration
+    candidate (vector-CSR TPR 2), which would be replayed untimed."""
+    from torch.profiler import ProfilerActivity, profile
+    A = gen.laplacian2d(256)
+    x = torch.from_numpy(gen.vector(3, gen.INT8, A.ncols)).cuda()
+    y = torch.empty(A.nrows, dtype=torch.float64, device="cuda")
+    with pepp.Plan.from_csr(A, prune=False) as plan:
+        g = plan.graph(x, y, iterations=2, mode=0)
+        torch.cuda.synchronize()
+        with profile(activities=[ProfilerActivity.CUDA]) as prof:
+            g.launch()
+            torch.cuda.synchronize()
+        names = [e.key for e in prof.key_averages() if "pepp::" in e.key]
+        g.close()
+    assert names and all("sell" in n for n in names), names
+
+
+def test_context_key_separates_value_type_and_compression():
+    """fp32 and value-compressed plans of the same matrix keep
+    their own history records (different kernels, ~1.6x apart)."""
+    A = gen.laplacian2d(128)
+    A32 = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float32), A.r0, A.global_nrows)
+    keys = set()
+    for M in (A, A32):
+        for cv in (False, True):
+            with pepp.Plan.from_csr(M, compress_values=cv) as plan:
+                keys.add(plan.info()["key"])
+    assert len(keys) == 4

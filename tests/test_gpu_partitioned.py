@@ -107,6 +107,19 @@ def _worker(rank, world, lib, uid, name, exchange, K, outq, f32=False, overlap=T
             plan.exec_host(x0, yh, iterations=K, flags=pepp.Y_REPLICATED)
             A64 = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float64))
             res["host"] = bool(np.array_equal(yh.astype(np.float64), oracle.iterate(A64, x0.astype(np.float64), K)))
+            if not f32:   # smart containers on a partitioned plan: a LOCAL call writes only
+                #             this block's rows; the host copy of the other rows must survive the copy-back
+                r0, r1 = int(bounds[rank]), int(bounds[rank + 1])
+                xv = pepp.Vector(n, host=x0.astype(np.float64).copy())
+                yhost = np.full(n, -99.0)
+                yv = pepp.Vector(n, host=yhost)
+                plan.exec_vec(xv, yv, flags=pepp.Y_LOCAL)
+                got = yv.host(pepp.ACCESS_READ)
+                own = oracle.spmv(A64, x0.astype(np.float64))[r0:r1]
+                res["vec_local"] = bool(np.array_equal(got[r0:r1], own) and np.all(got[:r0] == -99.0)
+                                        and np.all(got[r1:] == -99.0))
+                xv.close()
+                yv.close()
             res["exchange"] = info["exchange"]
             res["halo_recv"] = info["halo_recv"]
             res["halo_send"] = info["halo_send"]
@@ -149,6 +162,7 @@ def test_two_ranks_one_gpu_iterated_spmv_bitwise(name, exchange):
     out = _run(name, exchange)
     for r in range(2):
         assert out[r]["iter"] and out[r]["host"], (r, out[r])
+        assert out[r]["vec_local"], r
     ex = {out[0]["exchange"], out[1]["exchange"]}
     assert len(ex) == 1                       # every rank resolved the same exchange
     if exchange != -1:
