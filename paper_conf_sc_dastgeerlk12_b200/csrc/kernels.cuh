@@ -1129,9 +1129,10 @@ __global__ void __launch_bounds__(256) panel_kernel(int j0, int j1, const int* _
     const uint64_t pol = evict_first_policy();
     for (int j = j0 + blockIdx.x * blockDim.x + threadIdx.x; j < j1; j += gridDim.x * blockDim.x) {
         const int r = __ldg(prow + j), s = __ldg(pstart + j), e = __ldg(pstart + j + 1);
+        const T yv = y[r];   // issued before the entries: in flight with them, not after the FMA chain
         T acc = T(0);
         for (int k = s; k < e; ++k) acc = fma(ld_stream_v(pval + k, pol), __ldg(x + ld_stream_i(pcol + k, pol)), acc);
-        y[r] += acc;   // the row's panels in order: (((0 + s_0) + s_1) + ...)
+        y[r] = yv + acc;   // the row's panels in order: (((0 + s_0) + s_1) + ...)
     }
 }
 

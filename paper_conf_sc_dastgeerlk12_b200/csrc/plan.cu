@@ -884,7 +884,10 @@ pepp_status_t prepare_panels(pepp_spmv_plan_t* p, cudaStream_t st, std::vector<i
         unsigned long long span = 0;
         PEPP_CUDA_TRY(cudaMemcpyAsync(&span, d_span.p, sizeof(span), cudaMemcpyDeviceToHost, st));
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-        const int lg0 = p->esz == 8 ? 22 : 23;   // 32 MB of x per panel
+#ifndef PEPP_PANEL_LG0
+#define PEPP_PANEL_LG0 22   // experiments: log2 entries of the first fp64 panel width (32 MB of x)
+#endif
+        const int lg0 = p->esz == 8 ? PEPP_PANEL_LG0 : PEPP_PANEL_LG0 + 1;   // 32 MB of x per panel
         if ((double)span / (double)R < (double)(1ll << (lg0 - 1))) return PEPP_OK;
         lgs->push_back(lg0);
         if ((double)n * 2.0 * (4.0 + (double)p->esz) <= 48e9) lgs->push_back(lg0 + 1);   // and 64 MB, memory permitting

@@ -24,7 +24,10 @@ for n in sizes:
     plan_s = time.perf_counter() - t0
     del A
     res = {"rows": n, "plan_s": round(plan_s, 2), "device_gb": round(plan.info()["device_bytes"] / 1e9, 1)}
+    only = os.environ.get("PANEL_ONLY")
     for c in plan.candidates():
+        if only and c.variant != pepp.V_PANEL:
+            continue
         f = pepp.Choice(c.variant, c.param)
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(6)]
         for a, b in ev:
