@@ -120,16 +120,6 @@ def bound_f32(A, x) -> np.ndarray:
     return 2.0 * row_lengths(A).astype(np.float64) * 2.0 ** -23 * s
 
 
-def spmv_raw(nrows, first, row_ptr, col, val, x, parallel=False) -> np.ndarray:
-    rp, c, v = _args(row_ptr, col, val)
-    xx = _c(x, np.float64)
-    y = np.empty(nrows, dtype=np.float64)
-    f = lib().oracle_spmv_rows_parallel if parallel else lib().oracle_spmv_seq
-    if nrows:
-        f(nrows, first, _ptr(rp), _ptr(c), _ptr(v), _ptr(xx), _ptr(y))
-    return y
-
-
 def spmv_rows(A, x, rows) -> np.ndarray:
     """y_i for sampled rows i only (full-size parity)."""
     rp, c, v = _args(A.row_ptr, A.col, A.val)
