@@ -896,7 +896,8 @@ pepp_status_t prepare_panels(pepp_spmv_plan_t* p, cudaStream_t st, std::vector<i
     for (int lg : *lgs) {
         const int npanels = (int)((p->ncols + (1ll << lg) - 1) >> lg);
         if (npanels < 2 || npanels > 255) continue;
-        PanelLayout L;
+        p->panels.emplace_back();   // owned by the plan from here on: freed with it on any error path
+        PanelLayout& L = p->panels.back();
         L.lg = lg;
         L.npanels = npanels;
         pepp_status_t s;
@@ -920,7 +921,7 @@ pepp_status_t prepare_panels(pepp_spmv_plan_t* p, cudaStream_t st, std::vector<i
         PEPP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp.p, tb, key.p, skey.p, idx.p, sidx.p, (int)n, 0, end_bit, st));
         { DevTmp<unsigned char> k2; std::swap(k2.p, key.p); DevTmp<int> i2; std::swap(i2.p, idx.p); }   // free early
         if ((s = dalloc(p, &L.d_pcol, n))) return s;
-        if ((s = dalloc_bytes(p, &L.d_pval, n * (int64_t)p->esz))) { cudaFree(L.d_pcol); return s; }
+        if ((s = dalloc_bytes(p, &L.d_pval, n * (int64_t)p->esz))) return s;
         PEPP_CUDA_TRY(prow_full.alloc(n));
         PEPP_CUDA_TRY(head.alloc(n));
         const int gn = (int)std::min<int64_t>((n + 255) / 256, (int64_t)p->sm_count * 32);
@@ -943,8 +944,8 @@ pepp_status_t prepare_panels(pepp_spmv_plan_t* p, cudaStream_t st, std::vector<i
         PEPP_CUDA_TRY(cudaMemcpyAsync(&np, nsel.p, sizeof(int), cudaMemcpyDeviceToHost, st));
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
         L.npairs = np;
-        if ((s = dalloc(p, &L.d_prow, np))) { cudaFree(L.d_pcol); cudaFree(L.d_pval); return s; }
-        if ((s = dalloc(p, &L.d_pstart, (int64_t)np + 1))) { cudaFree(L.d_pcol); cudaFree(L.d_pval); cudaFree(L.d_prow); return s; }
+        if ((s = dalloc(p, &L.d_prow, np))) return s;
+        if ((s = dalloc(p, &L.d_pstart, (int64_t)np + 1))) return s;
         const int nn = (int)n;
         PEPP_CUDA_TRY(cudaMemcpyAsync(L.d_pstart, starts.p, sizeof(int) * np, cudaMemcpyDeviceToDevice, st));
         PEPP_CUDA_TRY(cudaMemcpyAsync(L.d_pstart + np, &nn, sizeof(int), cudaMemcpyHostToDevice, st));
@@ -970,7 +971,6 @@ pepp_status_t prepare_panels(pepp_spmv_plan_t* p, cudaStream_t st, std::vector<i
         L.poff.resize(npanels + 1);
         PEPP_CUDA_TRY(cudaMemcpyAsync(L.poff.data(), poff.p, sizeof(int) * (npanels + 1), cudaMemcpyDeviceToHost, st));
         PEPP_CUDA_TRY(cudaStreamSynchronize(st));
-        p->panels.push_back(std::move(L));
         ok.push_back(lg);
     }
     *lgs = ok;
