@@ -615,8 +615,11 @@ __device__ __forceinline__ void sell_slist_dispatch_one(int len, const SellStenc
 #undef PEPP_SLO
 }
 
+#ifndef PEPP_SLIST_MINB_F32
+#define PEPP_SLIST_MINB_F32 1   // experiments: minimum resident blocks per SM for the fp32 list kernel
+#endif
 template <int BLOCK, int U, int NMAX, typename T>
-__global__ void __launch_bounds__(BLOCK) sell_slist_kernel(const int2* __restrict__ list, int n,
+__global__ void __launch_bounds__(BLOCK, std::is_same<T, float>::value ? PEPP_SLIST_MINB_F32 : 1) sell_slist_kernel(const int2* __restrict__ list, int n,
                                                            const __grid_constant__ SellStencils st,
                                                            const T* __restrict__ val, const T* __restrict__ x,
                                                            T* __restrict__ y) {
