@@ -350,7 +350,7 @@ def test_two_ranks_p2p_fused_halo(name, f32, real):
 
 
 # ------------------------------------------- distribution choice (row a4)
-def _worker_dist(rank, world, lib, uid, name, K, outq, p2p):
+def _worker_dist(rank, world, lib, uid, name, K, outq, p2p, f32=False):
     """opts.dist_select: the plan times every (P', exchange) candidate, the
     ranks agree, and NEXT_INPUT / REPLICATED calls run the agreed argmin; every
     candidate forced must give the same bits (integer inputs)."""
@@ -368,8 +368,13 @@ def _worker_dist(rank, world, lib, uid, name, K, outq, p2p):
         n = A.nrows
         bounds = pepp.partition_rows(A.row_ptr, world)
         r0, r1 = int(bounds[rank]), int(bounds[rank + 1])
-        blk = gen.row_block(A, r0, r1)
+        dt = np.float32 if f32 else np.float64
+        tdt = torch.float32 if f32 else torch.float64
+        Ad = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(dt), A.r0, A.global_nrows)
+        blk = gen.row_block(Ad, r0, r1)
         x0 = gen.vector(3, gen.INT8, n)
+        if f32:
+            K = min(K, 4)   # |x| stays below 2^24: the fp32 results are exact too
         _, ghosts = pepp.halo_ghosts(blk.col, world, rank, bounds)
         rows = np.concatenate([np.arange(r0, r1), ghosts.astype(np.int64)])
         refs = [x0]
@@ -386,11 +391,11 @@ def _worker_dist(rank, world, lib, uid, name, K, outq, p2p):
                 res["info_p2p"] = {k: info[k] for k in ("dist_nparts", "dist_exchange")}
                 res["stats"] = plan.dist_stats()
             else:
-                bufs = [torch.empty(n, dtype=torch.float64, device="cuda") for _ in range(2)]
+                bufs = [torch.empty(n, dtype=tdt, device="cuda") for _ in range(2)]
             sel = plan.select()
             res["select"] = (sel.nparts, sel.exchange)
             # automatic: the agreed distribution, iterated
-            x = torch.from_numpy(x0).cuda()
+            x = torch.from_numpy(x0.astype(dt)).cuda()
             src = x
             used = set()
             for k in range(1, K + 1):
@@ -399,45 +404,45 @@ def _worker_dist(rank, world, lib, uid, name, K, outq, p2p):
                 u = plan.exec(src, dst, flags=pepp.Y_NEXT_INPUT)
                 used.add((u.nparts, u.exchange))
                 torch.cuda.synchronize()
-                res["ok"] &= bool(np.array_equal(dst.cpu().numpy()[rows], refs[k][rows]))
+                res["ok"] &= bool(np.array_equal(dst.cpu().numpy().astype(np.float64)[rows], refs[k][rows]))
                 src = dst
             res["used"] = sorted(used)
             # replicated: every row on every rank
-            yr = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+            yr = torch.full((n,), float("nan"), dtype=tdt, device="cuda")
             u = plan.exec(x, yr, flags=pepp.Y_REPLICATED)
             torch.cuda.synchronize()
-            res["repl"] = (u.nparts, u.exchange, bool(np.array_equal(yr.cpu().numpy(), refs[1])))
+            res["repl"] = (u.nparts, u.exchange, bool(np.array_equal(yr.cpu().numpy().astype(np.float64), refs[1])))
             # every candidate forced: same bits (own rows + ghosts after NEXT_INPUT, all rows after REPLICATED)
             for parts, ex, _ in plan.dist_stats():
                 if ex == pepp.X_P2P:
                     continue
                 f = pepp.Choice(pepp._capi.V_AUTO, 0, exchange=ex, nparts=parts)
-                a = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
-                b = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+                a = torch.full((n,), float("nan"), dtype=tdt, device="cuda")
+                b = torch.full((n,), float("nan"), dtype=tdt, device="cuda")
                 plan.exec(x, a, flags=pepp.Y_NEXT_INPUT, force=f)
                 plan.exec(a, b, flags=pepp.Y_NEXT_INPUT, force=f)
-                c = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+                c = torch.full((n,), float("nan"), dtype=tdt, device="cuda")
                 plan.exec(b, c, flags=pepp.Y_REPLICATED, force=f)
                 torch.cuda.synchronize()
-                res["forced"][(parts, ex)] = (bool(np.array_equal(b.cpu().numpy()[rows], refs[2][rows])) and
-                                              bool(np.array_equal(c.cpu().numpy(), refs[3])))
+                res["forced"][(parts, ex)] = (bool(np.array_equal(b.cpu().numpy().astype(np.float64)[rows], refs[2][rows]))
+                                              and bool(np.array_equal(c.cpu().numpy().astype(np.float64), refs[3])))
             # host entry point, iterated, the exchange inside (REPLICATED output)
-            yh = np.full(n, np.nan)
-            plan.exec_host(x0, yh, iterations=K, flags=pepp.Y_REPLICATED)
-            res["host"] = bool(np.array_equal(yh, refs[K]))
+            yh = np.full(n, np.nan, dtype=dt)
+            plan.exec_host(x0.astype(dt), yh, iterations=K, flags=pepp.Y_REPLICATED)
+            res["host"] = bool(np.array_equal(yh.astype(np.float64), refs[K]))
         outq.put((rank, res))
     except Exception as e:
         import traceback
         outq.put((rank, {"error": repr(e) + traceback.format_exc()}))
 
 
-def _run_dist(name, world, K=5, p2p=False):
+def _run_dist(name, world, K=5, p2p=False, f32=False):
     import torch.multiprocessing as mp
     lib = _build_fake()
-    uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_dist_{world}_{int(p2p)}".encode() + b"\0" * 128)[:128]
+    uid = (f"/tmp/pepp_fake_nccl_{os.getpid()}_{name}_dist_{world}_{int(p2p)}{int(f32)}".encode() + b"\0" * 128)[:128]
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker_dist, args=(r, world, lib, uid, name, K, q, p2p)) for r in range(world)]
+    procs = [ctx.Process(target=_worker_dist, args=(r, world, lib, uid, name, K, q, p2p, f32)) for r in range(world)]
     for p in procs:
         p.start()
     out = {}
@@ -456,9 +461,10 @@ def _run_dist(name, world, K=5, p2p=False):
     return out
 
 
-@pytest.mark.parametrize("name,world,p2p", [("lap", 2, False), ("zipf", 2, False), ("lap", 4, False),
-                                            ("lap", 2, True)])
-def test_distribution_choice_agreed_and_bitwise(name, world, p2p):
+@pytest.mark.parametrize("name,world,p2p,f32", [("lap", 2, False, False), ("zipf", 2, False, False),
+                                                ("lap", 4, False, False), ("lap", 2, True, False),
+                                                ("banded", 2, False, True)])
+def test_distribution_choice_agreed_and_bitwise(name, world, p2p, f32):
     """Row a4 (P and exchange as timed choices): the plan times every
     (P', exchange) candidate — P' in {nranks, nranks/2, ..., 1} x {halo,
     allgather}, plus the fused push once buffers are registered — on every
@@ -468,7 +474,7 @@ def test_distribution_choice_agreed_and_bitwise(name, world, p2p):
     host entry point too. 4 ranks exercise P' = 2 (point-to-point groups
     among a subset of the ranks)."""
     import paper_conf_sc_dastgeerlk12_b200 as pepp
-    out = _run_dist(name, world, p2p=p2p)
+    out = _run_dist(name, world, p2p=p2p, f32=f32)
     expect_parts = []
     pp = world
     while pp >= 1:
