@@ -463,7 +463,7 @@ def _run_dist(name, world, K=5, p2p=False, f32=False):
 
 @pytest.mark.parametrize("name,world,p2p,f32", [("lap", 2, False, False), ("zipf", 2, False, False),
                                                 ("lap", 4, False, False), ("lap", 2, True, False),
-                                                ("banded", 2, False, True)])
+                                                ("banded", 2, False, True), ("zipf", 3, False, False)])
 def test_distribution_choice_agreed_and_bitwise(name, world, p2p, f32):
     """Row a4 (P and exchange as timed choices): the plan times every
     (P', exchange) candidate — P' in {nranks, nranks/2, ..., 1} x {halo,
@@ -475,11 +475,7 @@ def test_distribution_choice_agreed_and_bitwise(name, world, p2p, f32):
     among a subset of the ranks)."""
     import paper_conf_sc_dastgeerlk12_b200 as pepp
     out = _run_dist(name, world, p2p=p2p, f32=f32)
-    expect_parts = []
-    pp = world
-    while pp >= 1:
-        expect_parts.append(pp)
-        pp //= 2
+    expect_parts = [world] + [pp for pp in (4, 2, 1) if pp < world and world % pp == 0]   # powers of two dividing N
     for r in range(world):
         res = out[r]
         assert res["ok"] and res["host"], (r, res)
