@@ -1895,10 +1895,21 @@ pepp_status_t setup_dist_parts(const pepp_spmv_opts_t* o, pepp_spmv_plan_t* p, c
             so.dist_select = 0;
             so.device = p->device;
             pepp_spmv_plan_t* q = new (std::nothrow) pepp_spmv_plan_t();
-            if (!q) return PEPP_E_NOMEM;
-            q->device = -1;
-            if ((s = plan_impl(&U, &so, q))) { free_plan(q); return s; }
+            s = q ? PEPP_OK : PEPP_E_NOMEM;
+            if (q) {
+                q->device = -1;
+                if ((s = plan_impl(&U, &so, q))) { free_plan(q); q = nullptr; }
+            }
             dp.plan = q;
+        }
+        {   // agreement: a rank whose P' plan failed (e.g. out of memory for the union of
+            // its blocks) must not leave the others inside the next collectives
+            int64_t code = -(int64_t)s;
+            const pepp_status_t sa = nccl_allmax(p, st, &code);
+            if (sa || code) {
+                free_plan(dp.plan);
+                return sa ? sa : (s ? s : (pepp_status_t)(-code));
+            }
         }
         p->dparts.push_back(std::move(dp));   // owned by the plan from here on (freed with it)
         // ---- HALO form: own rows + own ghosts from their P' owners
