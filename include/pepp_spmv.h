@@ -398,10 +398,15 @@ pepp_status_t pepp_spmv_exchange(pepp_spmv_plan_t* p, void* y, int flags, void* 
    PEPP_E_NCCL, PEPP_E_NOMEM. */
 pepp_status_t pepp_spmv_p2p_buffers(pepp_spmv_plan_t* p, int32_t nbuf, void** bufs);
 
-/* Distribution candidates of a partitioned plan (opts.dist_select): for
-   each i < *n (up to cap): nparts[i] = P', exchange[i] = pepp_exchange_t,
-   agreed_us[i] = the max-over-ranks mean time of one PEPP_Y_NEXT_INPUT call
-   the ranks agreed on (0 if never timed). Host only. */
+/* Distribution candidates of a partitioned plan (opts.dist_select; the
+   runtime's choice of "which implementation/device to use" from history
+   and data-transfer cost, §V-D P@38827; §8(a) a4): for each i < *n (up to
+   cap): nparts[i] = P', exchange[i] = pepp_exchange_t (the last entry is
+   PEPP_X_P2P once pepp_spmv_p2p_buffers registered buffers), agreed_us[i] =
+   the max-over-ranks mean time of one PEPP_Y_NEXT_INPUT call the ranks
+   agreed on (0 if never timed). nparts / exchange / agreed_us: WRITE, host,
+   cap entries each, or NULL; *n: WRITE, the total. Host only.
+   PEPP_E_INVALID on NULL p or n, negative cap. */
 pepp_status_t pepp_spmv_dist_stats(const pepp_spmv_plan_t* p, int32_t cap, int32_t* nparts, int32_t* exchange,
                                    double* agreed_us, int32_t* n);
 
