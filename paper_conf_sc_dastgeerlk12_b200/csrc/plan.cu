@@ -2391,8 +2391,24 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
             if (!have_prior && p->info.predicted) { p->prior = p->predicted; have_prior = true; }
         }
         if (have_prior) {
+            // a recorded neighbour context orders the calibration by its means;
+            // a *variant* it never recorded at all (e.g. the column panels,
+            // which only exist once x leaves L2, so a smaller neighbour cannot
+            // have timed them) is tried first — optimism under uncertainty: its
+            // one calibration call costs less than missing a new best variant
+            // (round-2 sweep: cold picks 2.15x / 2.35x off on the two largest
+            // random matrices without it). Predictions keep their own order.
+            std::vector<uint8_t> unseen(n, 0);
+            if (p->prior_key) {
+                for (int32_t c = 0; c < n; ++c) {
+                    bool seen = false;
+                    for (int32_t d = 0; d < n && !seen; ++d) seen = p->cands[d].variant == p->cands[c].variant && p->prior[d] > 0;
+                    unseen[c] = !seen;
+                }
+            }
             std::stable_sort(p->order.begin(), p->order.end(), [&](int32_t a, int32_t b) {
-                const double pa = p->prior[a] > 0 ? p->prior[a] : 1e300, pb = p->prior[b] > 0 ? p->prior[b] : 1e300;
+                const double pa = unseen[a] ? 0.0 : p->prior[a] > 0 ? p->prior[a] : 1e300;
+                const double pb = unseen[b] ? 0.0 : p->prior[b] > 0 ? p->prior[b] : 1e300;
                 return pa < pb;
             });
         }
