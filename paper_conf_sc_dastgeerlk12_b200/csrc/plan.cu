@@ -147,6 +147,16 @@ struct pepp_spmv_plan_s {
     int* d_patlist = nullptr;        // σ = 1: pattern chunks as (chunk << 5 | id), phase A of the kernel
     int* d_genlist = nullptr;        // σ = 1: the other chunks, phase B
     int npatc = 0, ngen = 0;
+    // pattern tiles (sell_ptile_kernel): runs of pattern chunks cut into
+    // tiles whose x ranges are bulk-copied; the pattern chunks no tile holds
+    // stay in d_patrest for phase A of the genlist walk
+    int2* d_ptiles = nullptr;
+    int nptiles = 0, grid_ptile = 0, ptile_rows = 0, ptile_stage = 0;
+    int64_t ptile_chunks = 0;
+    size_t ptile_smem = 0;
+    pepp::k::PatTiles ptt{};
+    int* d_patrest = nullptr;
+    int npatrest = 0;
     int2* d_stlist = nullptr;        // σ = 1, values streamed: stencil-list entries (sell_slist_kernel)
     int nstc = 0, grid_slist = 0;
     bool slist_long = false;                     // an offset set longer than 8: the 16-slot instance
@@ -350,7 +360,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
-                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist,
+                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist, p->d_ptiles, p->d_patrest,
                     p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, p->d_sell_part, p->d_sell_mid, p->d_stlist};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
@@ -423,6 +433,148 @@ pepp_status_t sell_warp_ranges(pepp_spmv_plan_t* p) {
     return PEPP_OK;
 }
 
+// Pattern tiles (sell_ptile_kernel, σ = 1 value-compressed plans): the
+// pattern list (sorted by id, chunk order within an id) is cut into tiles of
+// consecutive chunks of one pattern, <= ptile_rows rows each. Per pattern the
+// distinct offsets are grouped into clusters (gap <= kPtileGap elements: one
+// bulk copy of a few extra elements is cheaper than another copy); cluster c
+// copies x[r0 + clo_c, r0 + clo_c + round16(nr + cext_c)) — clo_c rounded
+// down to 16 B (r0 is a multiple of 32 rows, so the rounding is the same for
+// every tile). A tile whose rounded ranges leave [0, ncols) keeps its chunks
+// in the phase-A list (d_patrest). Stage size = the largest pattern's
+// clusters at ptile_rows rows; ptile_rows = the largest multiple of 32 rows
+// (<= kPtileRangeBytes of x per range) whose S stages fit the shared-memory budget.
+#ifndef PEPP_PTILE
+#define PEPP_PTILE 1
+#endif
+#ifndef PEPP_PTILE_S
+#define PEPP_PTILE_S 4   // stages of sell_ptile_kernel
+#endif
+#ifndef PEPP_PTILE_RANGE_KB
+#define PEPP_PTILE_RANGE_KB 16   // x bytes per cluster range: rows per tile = 16 KB / value size (fewer if the stages do not fit)
+#endif
+#ifndef PEPP_PTILE_BLOCK
+#define PEPP_PTILE_BLOCK 288   // one producer warp + 8 consumer warps
+#endif
+constexpr bool kPatTiles = PEPP_PTILE;
+constexpr int kPtileS = PEPP_PTILE_S, kPtileBlock = PEPP_PTILE_BLOCK, kPtileRangeBytes = PEPP_PTILE_RANGE_KB * 1024;
+constexpr int kPtileGap = 64;
+#ifndef PEPP_PTILE_SMEM_KB
+#define PEPP_PTILE_SMEM_KB 200   // per CTA
+#endif
+constexpr size_t kPtileSmemBudget = (size_t)PEPP_PTILE_SMEM_KB * 1024;
+
+template <typename T>
+pepp_status_t sell_pattern_tiles(pepp_spmv_plan_t* p, const pepp::k::SellPatterns<T>& pt, const std::vector<int>& pat) {
+    constexpr int A = 16 / (int)sizeof(T);
+    auto rdn = [](int64_t v) { return (v >= 0 ? v / A : -((-v + A - 1) / A)) * A; };
+    auto rup = [](int64_t v) { return ((v + A - 1) / A) * A; };
+    pepp::k::PatTiles tt{};
+    int npat = 0;
+    for (int e : pat) npat = std::max(npat, (e & 31) + 1);
+    // clusters per pattern, and the stage elements beyond the rows (sum of cext + rounding)
+    std::vector<int64_t> extra(npat, 0);
+    for (int q = 0; q < npat; ++q) {
+        const int len = pt.len[q];
+        std::vector<int> o(pt.off[q], pt.off[q] + len);
+        std::sort(o.begin(), o.end());
+        o.erase(std::unique(o.begin(), o.end()), o.end());
+        int nc = 0;
+        std::vector<int> lo, hi;
+        for (size_t i = 0; i < o.size(); ++i) {
+            if (nc && (int64_t)o[i] - hi.back() <= kPtileGap) { hi.back() = o[i]; continue; }
+            lo.push_back(o[i]);
+            hi.push_back(o[i]);
+            ++nc;
+        }
+        tt.ncl[q] = nc;
+        for (int c = 0; c < nc; ++c) {
+            const int64_t clo = rdn(lo[c]), cext = (int64_t)hi[c] - clo;
+            if (clo < INT32_MIN / 2 || clo > INT32_MAX / 2 || cext > (1 << 20)) return PEPP_OK;   // no tiles
+            tt.clo[q][c] = (int)clo;
+            tt.cext[q][c] = (int)cext;
+            extra[q] += rup(cext) + A;   // round16(nr + cext) <= nr + round16(cext) (nr a multiple of 32)
+        }
+    }
+    int64_t emax = 0;
+    for (int q = 0; q < npat; ++q) emax = std::max(emax, extra[q] + 0);
+    int maxcl = 1;
+    for (int q = 0; q < npat; ++q) maxcl = std::max(maxcl, tt.ncl[q]);
+    // S x (stage + y stage) + barriers within the budget
+    int rows = kPtileRangeBytes / (int)sizeof(T);
+    auto stage_of = [&](int r) { return (int64_t)maxcl * r + emax; };
+    while (rows >= 32 && (size_t)kPtileS * (size_t)stage_of(rows) * sizeof(T) + 24 * kPtileS + 64 > kPtileSmemBudget) rows -= 32;
+    if (rows < 32) return PEPP_OK;
+    const int64_t stage = rup(stage_of(rows));
+    for (int q = 0; q < npat; ++q) {
+        int64_t d = 0;
+        for (int c = 0; c < tt.ncl[q]; ++c) { tt.cdst[q][c] = (int)d; d += rup(rows + tt.cext[q][c]); }
+        for (int j = 0; j < pt.len[q]; ++j) {
+            int c = 0;
+            while (c + 1 < tt.ncl[q] && pt.off[q][j] >= tt.clo[q][c + 1]) ++c;
+            tt.sidx[q][j] = tt.cdst[q][c] + (pt.off[q][j] - tt.clo[q][c]);
+        }
+    }
+    // the tiles: runs of consecutive chunks of one pattern
+    std::vector<int2> tiles;
+    std::vector<int> rest;
+    const int cmax = rows / 32;
+    // 0: fits; 1: a range starts below x[0]; 2: a range (or the rows) ends past the end
+    auto misfit = [&](int64_t r0, int nr, int q) {
+        if (r0 + nr > p->nrows) return 2;
+        for (int c = 0; c < tt.ncl[q]; ++c) {
+            const int64_t a = r0 + tt.clo[q][c], b = a + rup(nr + tt.cext[q][c]);
+            if (a < 0) return 1;
+            if (b > p->ncols) return 2;
+        }
+        return 0;
+    };
+    int64_t tiled = 0;
+    for (size_t i = 0; i < pat.size();) {
+        const int q = pat[i] & 31;
+        size_t j = i + 1;
+        while (j < pat.size() && (int)(j - i) < cmax && (pat[j] & 31) == q && (pat[j] >> 5) == (pat[i] >> 5) + (int)(j - i)) ++j;
+        // trim chunks off the run's start / end until its ranges lie inside x
+        size_t a = i, b = j;
+        for (int m; a < b && (m = misfit((int64_t)(pat[a] >> 5) * 32, (int)(b - a) * 32, q)) != 0;) {
+            if (m == 1) rest.push_back(pat[a++]);
+            else rest.push_back(pat[--b]);
+        }
+        if (a < b) {
+            tiles.push_back(make_int2(pat[a] >> 5, ((int)(b - a) << 5) | q));
+            tiled += (int64_t)(b - a);
+        }
+        i = j;
+    }
+    if (tiles.empty()) return PEPP_OK;
+    pepp_status_t s;
+    if ((s = dalloc(p, &p->d_ptiles, (int64_t)tiles.size()))) return s;
+    PEPP_CUDA_TRY(cudaMemcpy(p->d_ptiles, tiles.data(), sizeof(int2) * tiles.size(), cudaMemcpyHostToDevice));
+    if (!rest.empty()) {
+        if ((s = dalloc(p, &p->d_patrest, (int64_t)rest.size()))) return s;
+        PEPP_CUDA_TRY(cudaMemcpy(p->d_patrest, rest.data(), sizeof(int) * rest.size(), cudaMemcpyHostToDevice));
+    }
+    p->nptiles = (int)tiles.size();
+    p->npatrest = (int)rest.size();
+    p->ptile_chunks = tiled;
+    p->ptile_rows = rows;
+    p->ptile_stage = (int)stage;
+    p->ptt = tt;
+    p->ptile_smem = (size_t)kPtileS * (size_t)stage * sizeof(T) + 24 * kPtileS;
+    const void* fn = (const void*)pepp::k::sell_ptile_kernel<kPtileBlock, kPtileS, T>;
+    PEPP_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->ptile_smem));
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kPtileBlock, p->ptile_smem) != cudaSuccess || occ < 1) occ = 1;
+    (void)cudaGetLastError();
+    p->grid_ptile = (int)std::max<int64_t>(1, std::min<int64_t>(p->nptiles, (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ));
+    if (p->ngen + p->npatrest > 0 && kSlistConcurrent && !p->gside) {
+        PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->gside, cudaStreamNonBlocking));
+        PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gfork, cudaEventDisableTiming));
+        PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gjoin, cudaEventDisableTiming));
+    }
+    return PEPP_OK;
+}
+
 // Value + index compression: constant stencil chunks (cflag) with the same
 // (length, offsets, value bits) become one entry of the pattern table; the
 // chunk keeps its length, trades kSellStencil for kSellPattern, and its
@@ -489,6 +641,7 @@ pepp_status_t sell_patterns(pepp_spmv_plan_t* p, int64_t nsb, const void* d_scon
         if (!gen.empty()) PEPP_CUDA_TRY(cudaMemcpy(p->d_genlist, gen.data(), sizeof(int) * gen.size(), cudaMemcpyHostToDevice));
         p->npatc = (int)pat.size();
         p->ngen = (int)gen.size();
+        if (kPatTiles && (s = sell_pattern_tiles<T>(p, *pt, pat))) return s;
     }
     return PEPP_OK;
 }
@@ -628,6 +781,7 @@ pepp_status_t sell_layout_bytes(pepp_spmv_plan_t* p) {
         if (d & pepp::k::kSellMasked) b += 4 * 32;
     }
     if (p->d_perm) b += 4 * p->nrows;
+    b += 8 * (int64_t)p->nptiles - 4 * p->ptile_chunks;   // tiled pattern chunks: one 8 B tile entry per tile
     b += p->sell_long_nnz * (es + 4) + (int64_t)p->nsell_mid * (4 + 8) + (int64_t)p->nsell_long * 8 +
          (int64_t)p->nsell_seg * (16 + 16);
     b += p->ncols * es + p->nrows * es;
@@ -773,6 +927,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->info.sell_col16_frac = p->nchunks ? (double)p->sell_col16_chunks / (double)p->nchunks : 0.0;
     p->info.sell_stencil_frac = p->nchunks ? (double)p->sell_stencil_chunks / (double)p->nchunks : 0.0;
     p->info.sell_constval_frac = p->nchunks ? (double)p->sell_const_chunks / (double)p->nchunks : 0.0;
+    p->info.sell_ptile_frac = p->nchunks ? (double)p->ptile_chunks / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
     p->info.sell_long_rows = p->nsell_long + p->nsell_mid;
     p->info.sell_cap = p->sell_cap == INT32_MAX ? 0 : p->sell_cap;
@@ -1157,7 +1312,25 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
                 p->d_scol16, p->d_soff, pepp::k::NoPatterns{}, (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws,
                 nullptr, 0, nullptr);
-        else if (p->d_patlist)   // pattern chunks (value compression): phase A + the rest through genlist
+        else if (p->d_patlist && p->nptiles && ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0) {
+            // pattern tiles (bulk-copied x ranges) on st; the grid-edge chunks
+            // and the untiled pattern chunks through the genlist walk beside it
+            cudaStream_t gs = p->gside ? p->gside : st;
+            const bool side = p->ngen + p->npatrest > 0;
+            if (side && p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
+                                     cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
+                return PEPP_E_CUDA;
+            pepp::k::sell_ptile_kernel<kPtileBlock, kPtileS, T><<<p->grid_ptile, kPtileBlock, p->ptile_smem, st>>>(
+                sell_pattern_table<T>(p), p->ptt, p->d_ptiles, p->nptiles, p->ptile_stage, x, y);
+            if (side)
+                pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, gs>>>(
+                    (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
+                    p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
+                    p->d_patrest, p->npatrest, p->d_genlist);
+            if (side && p->gside && (cudaEventRecord(p->ev_gjoin, p->gside) != cudaSuccess ||
+                                     cudaStreamWaitEvent(st, p->ev_gjoin, 0) != cudaSuccess))
+                return PEPP_E_CUDA;
+        } else if (p->d_patlist)   // pattern chunks (value compression): phase A + the rest through genlist
             pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
@@ -1223,7 +1396,9 @@ int launches_for(const pepp_spmv_plan_t* p, const Candidate& c) {
         if (c.param == kMergeWarpParam) return p->ntiles_w > 0 ? 2 + (p->nlongruns_w > 0) : 0;
         return p->ntiles > 0 ? 2 + (p->nlongruns > 0) : 0;
     case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
-    case PEPP_V_SELL: return (p->d_stlist ? 1 + (p->ngen > 0) : 1) + (p->nsell_mid > 0) + (p->nsell_seg > 0);
+    case PEPP_V_SELL:
+        return (p->d_stlist ? 1 + (p->ngen > 0) : (p->d_patlist && p->nptiles) ? 1 + (p->ngen + p->npatrest > 0) : 1) +
+               (p->nsell_mid > 0) + (p->nsell_seg > 0);
     case PEPP_V_PANEL:
         for (const auto& pl : p->panels)
             if (pl.lg == c.param) {

@@ -315,7 +315,9 @@ def test_selector_calibrates_then_picks_fastest_measured():
         ch = plan.select()
         assert not ch.calibrating
         best = min(means)
-        assert means[ch.candidate] <= best * 1.01 + 1e-9
+        # the tie rule (reading A10): a later candidate replaces the pick only
+        # when it is more than 1 % faster, so the pick is within best / 0.99
+        assert means[ch.candidate] * 0.99 <= best + 1e-9
         u = plan.exec(x, y)
         assert u.candidate == ch.candidate
 

@@ -1,0 +1,123 @@
+"""GPU parity of the pattern-tile kernel (sell_ptile_kernel): value-compressed
+σ = 1 plans compute runs of pattern chunks from x ranges bulk-copied into
+shared memory. Per row the same FMAs in the same slot order as the
+register path, so y must be bit-identical to the streamed layout (and to
+the oracle on integer inputs, within the north-star bound on real ones).
+Covers: 2-D / 3-D stencils (1-5 offset clusters), fp64 and fp32, x / y
+views that are not 16-byte aligned (the register path runs instead), tiles
+whose ranges would leave x (kept in the phase-A list), and the fraction of
+chunks the tiles hold."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_sc_dastgeerlk12_b200 as pepp  # noqa: E402
+from test_gpu_parity import _check, _stencil_grid  # noqa: E402
+
+
+def _y(A, x, compress, dt=torch.float64, shift=0):
+    """y through a SELL-only plan; `shift` > 0 runs the call on views that
+    start `shift` elements into their buffers (not 16-byte aligned)."""
+    with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_SELL, prune=False, compress_values=compress) as plan:
+        xb = torch.zeros(A.ncols + shift, dtype=dt, device="cuda")
+        xb[shift:] = torch.from_numpy(np.ascontiguousarray(x)).to(dt).cuda()
+        yb = torch.full((A.nrows + shift,), float("nan"), dtype=dt, device="cuda")
+        xv, yv = xb[shift:], yb[shift:]
+        for _ in range(3):   # calibration calls, then the measured one
+            plan.exec(xv, yv)
+        torch.cuda.synchronize()
+        return yv.cpu().numpy(), plan.info()
+
+
+def _bits(a):
+    return a.view(np.int64 if a.dtype == np.float64 else np.int32)
+
+
+@pytest.mark.parametrize("n", [96, 1024])
+def test_ptile_laplacian_bit_identical(n):
+    A = gen.laplacian2d(n)
+    for x in (gen.vector(3, gen.INT8, A.ncols), gen.vector(4, gen.REAL, A.ncols)):
+        y1, i1 = _y(A, x, True)
+        y0, i0 = _y(A, x, False)
+        assert i0["sell_ptile_frac"] == 0.0
+        assert i1["sell_ptile_frac"] > (0.9 if n == 1024 else 0.3)
+        assert i1["sell_ptile_frac"] <= i1["sell_constval_frac"]
+        assert np.array_equal(_bits(y1), _bits(y0))
+        _check(A, x, y1, bool(np.all(x == np.round(x))))
+
+
+def test_ptile_misaligned_views_fall_back_bit_identical():
+    """x / y one element into their buffers: not 16-byte aligned, so the
+    bulk copies cannot run; the call takes the register path — same bits."""
+    A = gen.laplacian2d(300)
+    x = gen.vector(5, gen.REAL, A.ncols)
+    ya, ia = _y(A, x, True)
+    for shift in (1, 2):
+        yb, _ = _y(A, x, True, shift=shift)
+        assert np.array_equal(_bits(ya), _bits(yb)), shift
+    assert ia["sell_ptile_frac"] > 0.5
+    _check(A, x, ya, False)
+
+
+@pytest.mark.parametrize("name", ["lap3d_7pt", "grid_8pt", "lap1d", "edge"])
+def test_ptile_stencils(name):
+    """3-D 7-point (5 offset clusters: ±n², ±n, {-1, 0, 1}); a 3x3 stencil
+    minus a corner (3 clusters of 2-3 offsets); a 1-D 3-point stencil; and
+    `edge`: 1600 rows with columns i+1..i+3 of 1603, one run of 50 chunks
+    whose rounded range would end at x[1604]: its last chunk is trimmed off
+    into the phase-A list (exactly 49 of 50 chunks tiled) — all
+    bit-identical to the streamed layout."""
+    if name == "lap3d_7pt":
+        offs = [(0, 0, 0), (-1, 0, 0), (1, 0, 0), (0, -1, 0), (0, 1, 0), (0, 0, -1), (0, 0, 1)]
+        A = _stencil_grid(96, offs, 6.0, -1.0, dims=3)
+    elif name == "grid_8pt":
+        offs = [(a, b) for a in (-1, 0, 1) for b in (-1, 0, 1) if (a, b) != (1, 1)]
+        A = _stencil_grid(700, offs, 8.0, -1.0)
+    elif name == "lap1d":
+        A = _stencil_grid(200_003, [(-1,), (0,), (1,)], 2.0, -1.0, dims=1)
+    else:
+        n = 1600
+        col = (np.arange(n)[:, None] + np.array([1, 2, 3])[None, :]).ravel().astype(np.int32)
+        val = np.tile(np.array([-1.0, 2.0, -1.0]), n)
+        A = gen.CSR(n, n + 3, np.arange(0, 3 * n + 1, 3, dtype=np.int64), col, val, 0, n)
+    for x in (gen.vector(3, gen.INT8, A.ncols), gen.vector(4, gen.REAL, A.ncols)):
+        y1, i1 = _y(A, x, True)
+        y0, _ = _y(A, x, False)
+        if name == "edge":
+            assert i1["sell_ptile_frac"] == pytest.approx(49 / 50)
+        else:
+            assert i1["sell_ptile_frac"] > 0.3
+        assert np.array_equal(_bits(y1), _bits(y0))
+        _check(A, x, y1, bool(np.all(x == np.round(x))))
+
+
+def test_ptile_fp32_bit_identical_and_within_bound():
+    A = gen.laplacian2d(1000)
+    x = gen.vector(8, gen.REAL, A.ncols).astype(np.float32)
+    A32 = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float32), A.r0, A.global_nrows)
+    y1, i1 = _y(A32, x, True, dt=torch.float32)
+    y0, _ = _y(A32, x, False, dt=torch.float32)
+    assert i1["sell_ptile_frac"] > 0.9
+    assert np.array_equal(_bits(y1), _bits(y0))
+    b = oracle.bound_f32(A32, x)
+    yr = oracle.spmv_f32(A32, x)
+    assert np.all(np.abs(y1.astype(np.float64) - yr.astype(np.float64)) <= b)
+
+
+def test_ptile_nonfinite_x():
+    """Inf / NaN in x reach exactly the rows whose stencil touches them."""
+    A = gen.laplacian2d(512)
+    x = gen.vector(9, gen.REAL, A.ncols)
+    x[[5, 40_000, 131_000]] = [np.inf, np.nan, -np.inf]
+    y1, _ = _y(A, x, True)
+    y0, _ = _y(A, x, False)
+    assert np.array_equal(_bits(y1), _bits(y0))
+    yr = oracle.spmv(A, x)
+    assert np.array_equal(np.isnan(y1), np.isnan(yr)) and np.array_equal(np.isinf(y1), np.isinf(yr))
