@@ -284,9 +284,10 @@ typedef struct pepp_plan_info_s {
                                  registered buffers' fused push won) */
     int32_t dist_repl_nparts; /* chosen P' for PEPP_Y_REPLICATED calls (allgather) */
     double dist_probe_ms;     /* wall time the plan-time timing of the candidates took */
-    double sell_ptile_frac;   /* fraction of SELL chunks in pattern tiles (compress_values, σ = 1):
-                                 runs of pattern chunks whose x ranges are bulk-copied into shared
-                                 memory (sell_ptile_kernel) when x and y are 16-byte aligned */
+    double sell_ptile_frac;   /* fraction of SELL chunks in tiles (σ = 1): runs of stencil chunks
+                                 (pattern chunks with compress_values, else stencil-list chunks whose
+                                 values stream) computed from x ranges and values bulk-copied into
+                                 shared memory (sell_tile_kernel) when x and y are 16-byte aligned */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

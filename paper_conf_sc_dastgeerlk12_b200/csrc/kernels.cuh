@@ -1116,30 +1116,34 @@ __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.w
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
 // =====================================================================
-// Value-compressed SELL, pattern tiles (B200-native phase A). A pattern chunk
-// (sell_patterns: 32 rows sharing their column offsets and their values)
-// reads only x and writes y: y[r] = sum_j v_j x[r + o_j] — a constant-
-// coefficient stencil. Runs of consecutive chunks of one pattern are cut at
-// plan time into tiles of <= trows rows. For a tile starting at row r0 the
-// x elements it needs form, per cluster of nearby offsets (gap <= 64), one
-// contiguous range [r0 + lo, r0 + nr - 1 + hi]; one thread of the CTA copies
-// each range into shared memory with cp.async.bulk (rounded out to 16 B:
-// r0 is a multiple of 32, so the rounding is a per-pattern constant),
-// completion counted on the stage's mbarrier, S stages deep. The CTA then
-// computes the tile's rows from shared memory (per row the same FMAs in the
-// same slot order as sell_pattern_slots: bit-identical) into a y stage that
-// one thread writes back with a bulk store. The x elements are read once
-// from DRAM (a 5-point stencil's three ranges of a tile meet again in L2 as
-// the grid's front advances: ±n grid rows are ~64 KB apart) and nothing goes
-// through the L1 gather path that held phase A at ~0.6 of the copy peak
-// (one 32-sector request per cycle per SM: ~26 sectors per chunk).
+// SELL tiles (B200-native): runs of consecutive stencil chunks of one
+// offset set. A stencil chunk's 32 rows share their column offsets o_j, so
+// y[r] = sum_j v_j(r) x[r + o_j]; for a run of chunks starting at row r0
+// the x elements needed form, per cluster of nearby offsets (gap <= 64),
+// one contiguous range [r0 + lo, r0 + nr - 1 + hi], and the chunks' values
+// (slot-major per chunk, chunks consecutive in the SELL value array) one
+// contiguous block. A producer warp copies each range (rounded out to 16 B:
+// r0 is a multiple of 32, so the rounding is a per-set constant) and, when
+// the values are streamed (VALS), the value block into a shared-memory
+// stage with cp.async.bulk, completion counted on the stage's mbarrier,
+// S stages deep; consumer warps compute the tile's rows from shared memory
+// — per row the same FMAs in the same slot order as the register paths
+// (sell_pattern_slots / sell_slist_chunks: bit-identical) — and store y.
+// !VALS: pattern chunks (value compression, the values are kernel
+// parameters; only x is read and y written). x elements are read once
+// from DRAM (a 5-point stencil's three ranges meet again in L2 as the grid's
+// front advances: ±n grid rows are ~64 KB apart), and nothing goes through
+// the L1 gather path that held the register form at ~0.6 of the copy peak
+// (one 32-B sector request per SM cycle: ~26 sectors per chunk).
 // =====================================================================
+constexpr int kTileMaxSets = 32, kTileMaxLen = 16;
 struct PatTiles {
-    int ncl[kSellMaxPatterns];                          // offset clusters of the pattern
-    int clo[kSellMaxPatterns][kSellMaxPatternLen];      // cluster c: first x element, relative to r0 (16-B aligned)
-    int cext[kSellMaxPatterns][kSellMaxPatternLen];     // elements copied = round16(nr + cext)
-    int cdst[kSellMaxPatterns][kSellMaxPatternLen];     // cluster c's element offset within a stage
-    int sidx[kSellMaxPatterns][kSellMaxPatternLen];     // slot j: stage element of the tile's row 0
+    int len[kTileMaxSets];                       // slots of set q
+    int ncl[kTileMaxSets];                       // offset clusters of set q
+    int clo[kTileMaxSets][kTileMaxLen];          // cluster c: first x element, relative to r0 (16-B aligned)
+    int cext[kTileMaxSets][kTileMaxLen];         // elements copied = round16(nr + cext)
+    int cdst[kTileMaxSets][kTileMaxLen];         // cluster c's element offset within a stage
+    int sidx[kTileMaxSets][kTileMaxLen];         // slot j: stage element of the tile's row 0
 };
 
 #ifndef PEPP_PTILE_U
@@ -1151,59 +1155,67 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 
 // Consumer thread c of NC: rows c, c + NC, ... of the tile, U at a time
 // (all shared-memory loads of the U rows first), written straight to y.
-template <int NC, int N, typename T>
-__device__ __forceinline__ void ptile_rows(const SellPatterns<T>& pt, const PatTiles& tt, int pid, const T* sx,
-                                           T* __restrict__ y, int nr, int c) {
-    constexpr int U = PEPP_PTILE_U;
+// VALS: slot j of row i is sv[(i / 32) * 32N + 32 j + i % 32].
+template <int NC, int N, bool VALS, typename T>
+__device__ __forceinline__ void tile_rows(const SellPatterns<T>& pt, const PatTiles& tt, int q, const T* sx,
+                                          const T* sv, T* __restrict__ y, int nr, int c) {
+    constexpr int U = !VALS ? PEPP_PTILE_U : (N <= 4 ? 4 : N <= 8 ? 2 : 1);
     int b[N];
     T w[N];
 #pragma unroll
-    for (int j = 0; j < N; ++j) { b[j] = tt.sidx[pid][j]; w[j] = pt.val[pid][j]; }
+    for (int j = 0; j < N; ++j) { b[j] = tt.sidx[q][j]; w[j] = VALS ? T(0) : pt.val[q][j]; }
     for (int i0 = c; i0 < nr; i0 += NC * U) {
-        T xv[U][N];
+        T xv[U][N], vv[VALS ? U : 1][N];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             const int i = i0 + u * NC < nr ? i0 + u * NC : i0;
 #pragma unroll
             for (int j = 0; j < N; ++j) xv[u][j] = sx[b[j] + i];
+            if constexpr (VALS) {
+                const T* v = sv + (i >> 5) * (32 * N) + (i & 31);
+#pragma unroll
+                for (int j = 0; j < N; ++j) vv[u][j] = v[32 * j];
+            }
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             T acc = T(0);
 #pragma unroll
-            for (int j = 0; j < N; ++j) acc = fma(w[j], xv[u][j], acc);   // slot order = the row's CSR order
+            for (int j = 0; j < N; ++j) acc = fma(VALS ? vv[u][j] : w[j], xv[u][j], acc);   // slot order = CSR order
             if (i0 + u * NC < nr) y[i0 + u * NC] = acc;
         }
     }
 }
 
-// tiles[t] = {first chunk, chunks << 5 | pattern id}; persistent CTAs walk
-// t = blockIdx.x, + gridDim.x, ... (the grid's front advances through the
-// rows together, so the ranges of neighbouring tiles meet in L2).
-// Warp-specialized: warp 0 (one elected lane) is the producer — it waits
-// until stage s is released (empty[s]), writes the tile's list entry to the
-// stage, and issues its bulk copies (completion on full[s]); the list entry
-// of its next tile is loaded one tile ahead. The other BLOCK/32 - 1 warps
-// consume: wait full[s], read the entry, compute their rows, store y with
-// coalesced st.global, release the stage (one arrive per warp). No CTA-wide
-// barrier in the loop, so the producer keeps S stages in flight while the
-// consumers work (a CTA-barrier form with a bulk store of y measured
-// 270-600 µs on config 4: the barriers put the compute and the issue of
-// every tile on one serial path).
-// Shared memory: S x stage (x ranges, stage_elems) | S full | S empty | S entries.
-template <int BLOCK, int S, typename T>
-__global__ void __launch_bounds__(BLOCK, 1) sell_ptile_kernel(const __grid_constant__ SellPatterns<T> pt,
-                                                              const __grid_constant__ PatTiles tt,
-                                                              const int2* __restrict__ tiles, int ntiles,
-                                                              int stage_elems, const T* __restrict__ x,
-                                                              T* __restrict__ y) {
+// tiles[t] = {first chunk, chunks << 5 | set id, value block / 32 (VALS), 0};
+// persistent CTAs walk t = blockIdx.x, + gridDim.x, ... (the grid's front
+// advances through the rows together, so the ranges of neighbouring tiles
+// meet in L2). Warp-specialized: warp 0 (one lane) is the producer — it
+// waits until stage s is released (empty[s]), writes the tile's list entry
+// to the stage and issues its bulk copies (completion on full[s]); the list
+// entry of its next tile is loaded one tile ahead. The other BLOCK/32 - 1
+// warps consume: wait full[s], read the entry, compute their rows, store y
+// with coalesced st.global, release the stage (one arrive per warp). No
+// CTA-wide barrier in the loop, so the producer keeps S stages in flight
+// while the consumers work (a CTA-barrier form with a bulk store of y
+// measured 270-600 µs on config 4: the barriers put the compute and the
+// issue of every tile on one serial path).
+// Shared memory: S x stage (x ranges; VALS: then the value block at
+// vstage) | S full | S empty | S entries.
+template <int BLOCK, int S, bool VALS, typename T>
+__global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_constant__ SellPatterns<T> pt,
+                                                             const __grid_constant__ PatTiles tt,
+                                                             const int4* __restrict__ tiles, int ntiles,
+                                                             int stage_elems, int vstage,
+                                                             const T* __restrict__ val, const T* __restrict__ x,
+                                                             T* __restrict__ y) {
     extern __shared__ __align__(128) unsigned char ptile_smem[];
     constexpr int A = 16 / sizeof(T);
     constexpr int NCW = BLOCK / 32 - 1, NC = NCW * 32;
     T* sx = reinterpret_cast<T*>(ptile_smem);
     uint64_t* full = reinterpret_cast<uint64_t*>(sx + (size_t)S * stage_elems);
     uint64_t* empty = full + S;
-    int2* ent = reinterpret_cast<int2*>(empty + S);
+    int4* ent = reinterpret_cast<int4*>(empty + S);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int G = gridDim.x;
     if (tid == 0) {
@@ -1213,23 +1225,25 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_ptile_kernel(const __grid_const
     __syncthreads();
     if (warp == 0) {
         if (lane != 0) return;
-        int2 e = blockIdx.x < ntiles ? __ldg(tiles + blockIdx.x) : make_int2(0, 0);
+        int4 e = blockIdx.x < ntiles ? __ldg(tiles + blockIdx.x) : make_int4(0, 0, 0, 0);
         for (int it = 0;; ++it) {
             const int t = blockIdx.x + it * G;
             if (t >= ntiles) break;
             const int s = it % S;
-            const int2 en = t + G < ntiles ? __ldg(tiles + t + G) : make_int2(0, 0);
+            const int4 en = t + G < ntiles ? __ldg(tiles + t + G) : make_int4(0, 0, 0, 0);
             if (it >= S) mbar_wait(&empty[s], (uint32_t)(((it / S) - 1) & 1));
             const int64_t r0 = (int64_t)e.x * 32;
-            const int nr = (e.y >> 5) * 32, pid = e.y & 31, nc = tt.ncl[pid];
+            const int nr = (e.y >> 5) * 32, q = e.y & 31, nc = tt.ncl[q];
             ent[s] = e;
             uint32_t bytes = 0;
-            for (int c = 0; c < nc; ++c) bytes += (uint32_t)(((nr + tt.cext[pid][c] + A - 1) / A) * A) * sizeof(T);
-            mbar_arrive_expect_tx(&full[s], bytes);
+            for (int c = 0; c < nc; ++c) bytes += (uint32_t)(((nr + tt.cext[q][c] + A - 1) / A) * A) * sizeof(T);
+            const uint32_t vbytes = VALS ? (uint32_t)nr * tt.len[q] * sizeof(T) : 0;
+            mbar_arrive_expect_tx(&full[s], bytes + vbytes);
             T* dst = sx + (size_t)s * stage_elems;
             for (int c = 0; c < nc; ++c)
-                tma_load_1d_nohint(dst + tt.cdst[pid][c], x + r0 + tt.clo[pid][c],
-                                   (uint32_t)(((nr + tt.cext[pid][c] + A - 1) / A) * A) * sizeof(T), &full[s]);
+                tma_load_1d_nohint(dst + tt.cdst[q][c], x + r0 + tt.clo[q][c],
+                                   (uint32_t)(((nr + tt.cext[q][c] + A - 1) / A) * A) * sizeof(T), &full[s]);
+            if (VALS) tma_load_1d_nohint(dst + vstage, val + (int64_t)e.z * 32, vbytes, &full[s]);
             e = en;
         }
         return;
@@ -1240,20 +1254,26 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_ptile_kernel(const __grid_const
         if (t >= ntiles) break;
         const int s = it % S;
         mbar_wait(&full[s], (uint32_t)((it / S) & 1));
-        const int2 e = ent[s];
-        const int nr = (e.y >> 5) * 32, pid = e.y & 31;
+        const int4 e = ent[s];
+        const int nr = (e.y >> 5) * 32, q = e.y & 31;
         const T* xs = sx + (size_t)s * stage_elems;
+        const T* vs = xs + vstage;
         T* yt = y + (int64_t)e.x * 32;
-        switch (pt.len[pid]) {
-        case 1: ptile_rows<NC, 1, T>(pt, tt, pid, xs, yt, nr, c); break;
-        case 2: ptile_rows<NC, 2, T>(pt, tt, pid, xs, yt, nr, c); break;
-        case 3: ptile_rows<NC, 3, T>(pt, tt, pid, xs, yt, nr, c); break;
-        case 4: ptile_rows<NC, 4, T>(pt, tt, pid, xs, yt, nr, c); break;
-        case 5: ptile_rows<NC, 5, T>(pt, tt, pid, xs, yt, nr, c); break;
-        case 6: ptile_rows<NC, 6, T>(pt, tt, pid, xs, yt, nr, c); break;
-        case 7: ptile_rows<NC, 7, T>(pt, tt, pid, xs, yt, nr, c); break;
-        default: ptile_rows<NC, 8, T>(pt, tt, pid, xs, yt, nr, c); break;
+#define PEPP_TR(N) case N: tile_rows<NC, N, VALS, T>(pt, tt, q, xs, vs, yt, nr, c); break;
+        switch (tt.len[q]) {
+        PEPP_TR(1) PEPP_TR(2) PEPP_TR(3) PEPP_TR(4) PEPP_TR(5) PEPP_TR(6) PEPP_TR(7)
+        default:
+            if constexpr (VALS) {
+                switch (tt.len[q]) {
+                PEPP_TR(8) PEPP_TR(9) PEPP_TR(10) PEPP_TR(11) PEPP_TR(12) PEPP_TR(13) PEPP_TR(14) PEPP_TR(15)
+                default: tile_rows<NC, 16, VALS, T>(pt, tt, q, xs, vs, yt, nr, c); break;
+                }
+            } else {
+                tile_rows<NC, 8, VALS, T>(pt, tt, q, xs, vs, yt, nr, c);
+            }
+            break;
         }
+#undef PEPP_TR
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[s]);   // this warp's reads of stage s are done
     }

@@ -84,6 +84,16 @@ struct PeerXfer {            // halo traffic with one peer
     void* d_buf = nullptr;   // pack / unpack buffer (value type)
 };
 
+// SELL tiles (sell_tile_kernel) of one kind: pattern chunks, or stencil
+// chunks whose values stream (sell_build_tiles)
+struct TileLayout {
+    int4* d_tiles = nullptr;      // {first chunk, chunks << 5 | set id, value block / 32, 0}
+    int ntiles = 0, grid = 0, rows = 0, stage = 0, vstage = 0;
+    int64_t chunks = 0;           // chunks the tiles hold
+    size_t smem = 0;              // dynamic shared memory per CTA
+    pepp::k::PatTiles tt{};
+};
+
 // Column-panel layout (PEPP_V_PANEL) for one panel width 2^lg
 struct PanelLayout {
     int lg = 0, npanels = 0;
@@ -150,13 +160,12 @@ struct pepp_spmv_plan_s {
     // pattern tiles (sell_ptile_kernel): runs of pattern chunks cut into
     // tiles whose x ranges are bulk-copied; the pattern chunks no tile holds
     // stay in d_patrest for phase A of the genlist walk
-    int2* d_ptiles = nullptr;
-    int nptiles = 0, grid_ptile = 0, ptile_rows = 0, ptile_stage = 0;
-    int64_t ptile_chunks = 0;
-    size_t ptile_smem = 0;
-    pepp::k::PatTiles ptt{};
+    TileLayout ptl;                  // pattern tiles
     int* d_patrest = nullptr;
     int npatrest = 0;
+    TileLayout stl;                  // stencil tiles (values streamed) over the stencil list
+    int2* d_strest = nullptr;        // stencil-list entries no tile holds (sell_slist_kernel)
+    int nstrest = 0;
     int2* d_stlist = nullptr;        // σ = 1, values streamed: stencil-list entries (sell_slist_kernel)
     int nstc = 0, grid_slist = 0;
     bool slist_long = false;                     // an offset set longer than 8: the 16-slot instance
@@ -360,7 +369,7 @@ void free_plan(pepp_spmv_plan_t* p) {
     if (p->device >= 0) cudaSetDevice(p->device);
     void* bufs[] = {p->d_rp, p->d_col, p->d_val, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm,
                     p->d_scol, p->d_scol16, p->d_soff, p->d_sval, p->d_tile, p->d_carry_row, p->d_carry_val, p->d_hx, p->d_hy,
-                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist, p->d_ptiles, p->d_patrest,
+                    p->d_items, p->d_longrows, p->d_stream_carry, p->d_tile_w, p->d_carry_row_w, p->d_carry_val_w, p->d_longruns, p->d_longruns_w, p->d_sell_ws, p->d_patlist, p->d_genlist, p->ptl.d_tiles, p->stl.d_tiles, p->d_patrest, p->d_strest,
                     p->d_sell_seg, p->d_sell_lrow, p->d_sell_cnt, p->d_sell_part, p->d_sell_mid, p->d_stlist};
     for (void* b : bufs) if (b) cudaFree(b);
     for (auto* v : {&p->recv_x, &p->send_x})
@@ -433,91 +442,120 @@ pepp_status_t sell_warp_ranges(pepp_spmv_plan_t* p) {
     return PEPP_OK;
 }
 
-// Pattern tiles (sell_ptile_kernel, σ = 1 value-compressed plans): the
-// pattern list (sorted by id, chunk order within an id) is cut into tiles of
-// consecutive chunks of one pattern, <= ptile_rows rows each. Per pattern the
-// distinct offsets are grouped into clusters (gap <= kPtileGap elements: one
+// SELL tiles (sell_tile_kernel, σ = 1 plans): a list of stencil chunks
+// (pattern chunks of value-compressed plans, or the stencil list's chunks
+// whose values stream), sorted by set id, chunk order within a set, is cut
+// into tiles of consecutive chunks of one set, <= rows rows each. Per set the
+// distinct offsets are grouped into clusters (gap <= kTileGap elements: one
 // bulk copy of a few extra elements is cheaper than another copy); cluster c
 // copies x[r0 + clo_c, r0 + clo_c + round16(nr + cext_c)) — clo_c rounded
 // down to 16 B (r0 is a multiple of 32 rows, so the rounding is the same for
-// every tile). A tile whose rounded ranges leave [0, ncols) keeps its chunks
-// in the phase-A list (d_patrest). Stage size = the largest pattern's
-// clusters at ptile_rows rows; ptile_rows = the largest multiple of 32 rows
-// (<= kPtileRangeBytes of x per range) whose S stages fit the shared-memory budget.
+// every tile). Chunks whose rounded ranges would leave [0, ncols) are
+// trimmed off a run's start / end into the caller's rest list. Stage = the
+// largest set's clusters at `rows` rows (+ rows x longest set values when
+// they stream); rows = the largest multiple of 32 (<= range bytes of x per
+// cluster) whose S stages fit the shared-memory budget.
 #ifndef PEPP_PTILE
-#define PEPP_PTILE 1
+#define PEPP_PTILE 1   // value-compressed plans: pattern tiles
+#endif
+#ifndef PEPP_STILE
+#define PEPP_STILE 3   // values streamed: stencil tiles (bit 0: fp32 plans, bit 1: fp64 plans); config 4: fp32 340 -> 281 us, fp64 605 -> 553 us (same box)
 #endif
 #ifndef PEPP_PTILE_S
-#define PEPP_PTILE_S 4   // stages of sell_ptile_kernel
+#define PEPP_PTILE_S 4   // stages, pattern tiles
+#endif
+#ifndef PEPP_STILE_S
+#define PEPP_STILE_S 3   // stages, stencil tiles (values streamed)
 #endif
 #ifndef PEPP_PTILE_RANGE_KB
 #define PEPP_PTILE_RANGE_KB 16   // x bytes per cluster range: rows per tile = 16 KB / value size (fewer if the stages do not fit)
 #endif
+#ifndef PEPP_STILE_RANGE_KB
+#define PEPP_STILE_RANGE_KB 8
+#endif
 #ifndef PEPP_PTILE_BLOCK
 #define PEPP_PTILE_BLOCK 288   // one producer warp + 8 consumer warps
 #endif
-constexpr bool kPatTiles = PEPP_PTILE;
-constexpr int kPtileS = PEPP_PTILE_S, kPtileBlock = PEPP_PTILE_BLOCK, kPtileRangeBytes = PEPP_PTILE_RANGE_KB * 1024;
-constexpr int kPtileGap = 64;
 #ifndef PEPP_PTILE_SMEM_KB
 #define PEPP_PTILE_SMEM_KB 200   // per CTA
 #endif
+constexpr bool kPatTiles = PEPP_PTILE;
+constexpr int kStencilTiles = PEPP_STILE;
+constexpr int kPtileS = PEPP_PTILE_S, kStileS = PEPP_STILE_S, kPtileBlock = PEPP_PTILE_BLOCK;
+constexpr int kTileGap = 64;
 constexpr size_t kPtileSmemBudget = (size_t)PEPP_PTILE_SMEM_KB * 1024;
 
+#ifndef PEPP_TILE_SIDE_BPS
+#define PEPP_TILE_SIDE_BPS 8   // blocks per SM (cap) of the walks beside a tile kernel; measured 1 / 2 / 8: vc config 4 207.5 / 197.9 / 197.0 us, fp32 list 293 / 282 / 282 us
+#endif
+int tile_side_grid(const pepp_spmv_plan_t* p, int grid) {
+    return std::max(1, std::min(grid, PEPP_TILE_SIDE_BPS * std::max(1, p->sm_count - p->reserve_sms)));
+}
+
+template <int S, bool VALS, typename T>
+const void* tile_kernel_fn() { return (const void*)pepp::k::sell_tile_kernel<kPtileBlock, S, VALS, T>; }
+
+// ents[i] = {chunk, set id, value block / 32, -}; sorted by set id then chunk.
+// Fills *L and appends the indices of untiled entries to *rest.
 template <typename T>
-pepp_status_t sell_pattern_tiles(pepp_spmv_plan_t* p, const pepp::k::SellPatterns<T>& pt, const std::vector<int>& pat) {
+pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, const int (*offs)[pepp::k::kTileMaxLen],
+                               const std::vector<int4>& ents, bool vals, TileLayout* L, std::vector<size_t>* rest) {
+    using pepp::k::kTileMaxLen;
     constexpr int A = 16 / (int)sizeof(T);
+    const int S = vals ? kStileS : kPtileS;
+    const int range_bytes = (vals ? PEPP_STILE_RANGE_KB : PEPP_PTILE_RANGE_KB) * 1024;
     auto rdn = [](int64_t v) { return (v >= 0 ? v / A : -((-v + A - 1) / A)) * A; };
     auto rup = [](int64_t v) { return ((v + A - 1) / A) * A; };
+    *L = TileLayout{};
     pepp::k::PatTiles tt{};
-    int npat = 0;
-    for (int e : pat) npat = std::max(npat, (e & 31) + 1);
-    // clusters per pattern, and the stage elements beyond the rows (sum of cext + rounding)
-    std::vector<int64_t> extra(npat, 0);
-    for (int q = 0; q < npat; ++q) {
-        const int len = pt.len[q];
-        std::vector<int> o(pt.off[q], pt.off[q] + len);
+    if (nsets > pepp::k::kTileMaxSets) return PEPP_OK;
+    int64_t emax = 0;
+    int maxcl = 1, maxlen = 1;
+    for (int q = 0; q < nsets; ++q) {
+        const int len = lens[q];
+        if (len < 1 || len > kTileMaxLen) return PEPP_OK;
+        tt.len[q] = len;
+        maxlen = std::max(maxlen, len);
+        std::vector<int> o(offs[q], offs[q] + len);
         std::sort(o.begin(), o.end());
         o.erase(std::unique(o.begin(), o.end()), o.end());
-        int nc = 0;
-        std::vector<int> lo, hi;
-        for (size_t i = 0; i < o.size(); ++i) {
-            if (nc && (int64_t)o[i] - hi.back() <= kPtileGap) { hi.back() = o[i]; continue; }
-            lo.push_back(o[i]);
-            hi.push_back(o[i]);
-            ++nc;
+        std::vector<int64_t> lo, hi;
+        for (int v : o) {
+            if (!lo.empty() && (int64_t)v - hi.back() <= kTileGap) { hi.back() = v; continue; }
+            lo.push_back(v);
+            hi.push_back(v);
         }
+        const int nc = (int)lo.size();
         tt.ncl[q] = nc;
+        maxcl = std::max(maxcl, nc);
+        int64_t extra = 0;
         for (int c = 0; c < nc; ++c) {
-            const int64_t clo = rdn(lo[c]), cext = (int64_t)hi[c] - clo;
+            const int64_t clo = rdn(lo[c]), cext = hi[c] - clo;
             if (clo < INT32_MIN / 2 || clo > INT32_MAX / 2 || cext > (1 << 20)) return PEPP_OK;   // no tiles
             tt.clo[q][c] = (int)clo;
             tt.cext[q][c] = (int)cext;
-            extra[q] += rup(cext) + A;   // round16(nr + cext) <= nr + round16(cext) (nr a multiple of 32)
+            extra += rup(cext) + A;   // round16(nr + cext) <= nr + round16(cext) (nr a multiple of 32)
         }
+        emax = std::max(emax, extra);
     }
-    int64_t emax = 0;
-    for (int q = 0; q < npat; ++q) emax = std::max(emax, extra[q] + 0);
-    int maxcl = 1;
-    for (int q = 0; q < npat; ++q) maxcl = std::max(maxcl, tt.ncl[q]);
-    // S x (stage + y stage) + barriers within the budget
-    int rows = kPtileRangeBytes / (int)sizeof(T);
-    auto stage_of = [&](int r) { return (int64_t)maxcl * r + emax; };
-    while (rows >= 32 && (size_t)kPtileS * (size_t)stage_of(rows) * sizeof(T) + 24 * kPtileS + 64 > kPtileSmemBudget) rows -= 32;
+    // S stages (x ranges, + values) and barriers / entries within the budget
+    int rows = std::max(32, range_bytes / (int)sizeof(T) / 32 * 32);
+    auto xpart = [&](int r) { return rup((int64_t)maxcl * r + emax); };
+    auto stage_of = [&](int r) { return xpart(r) + (vals ? (int64_t)r * maxlen : 0); };
+    while (rows >= 32 && (size_t)S * (size_t)stage_of(rows) * sizeof(T) + 32 * S + 64 > kPtileSmemBudget) rows -= 32;
     if (rows < 32) return PEPP_OK;
-    const int64_t stage = rup(stage_of(rows));
-    for (int q = 0; q < npat; ++q) {
+    for (int q = 0; q < nsets; ++q) {
         int64_t d = 0;
         for (int c = 0; c < tt.ncl[q]; ++c) { tt.cdst[q][c] = (int)d; d += rup(rows + tt.cext[q][c]); }
-        for (int j = 0; j < pt.len[q]; ++j) {
+        for (int j = 0; j < tt.len[q]; ++j) {
             int c = 0;
-            while (c + 1 < tt.ncl[q] && pt.off[q][j] >= tt.clo[q][c + 1]) ++c;
-            tt.sidx[q][j] = tt.cdst[q][c] + (pt.off[q][j] - tt.clo[q][c]);
+            while (c + 1 < tt.ncl[q] && offs[q][j] >= tt.clo[q][c + 1]) ++c;
+            tt.sidx[q][j] = tt.cdst[q][c] + (offs[q][j] - tt.clo[q][c]);
         }
     }
-    // the tiles: runs of consecutive chunks of one pattern
-    std::vector<int2> tiles;
-    std::vector<int> rest;
+    // the tiles: runs of consecutive chunks of one set (their values are
+    // consecutive too: σ = 1, chunk_ptr advances by 32 x len)
+    std::vector<int4> tiles;
     const int cmax = rows / 32;
     // 0: fits; 1: a range starts below x[0]; 2: a range (or the rows) ends past the end
     auto misfit = [&](int64_t r0, int nr, int q) {
@@ -529,49 +567,81 @@ pepp_status_t sell_pattern_tiles(pepp_spmv_plan_t* p, const pepp::k::SellPattern
         }
         return 0;
     };
+    auto next_of = [&](size_t i, size_t k) {   // entry k continues entry i's run
+        return ents[k].y == ents[i].y && (int64_t)ents[k].x == (int64_t)ents[i].x + (int64_t)(k - i) &&
+               (!vals || (int64_t)ents[k].z == (int64_t)ents[i].z + (int64_t)(k - i) * tt.len[ents[i].y]);
+    };
     int64_t tiled = 0;
-    for (size_t i = 0; i < pat.size();) {
-        const int q = pat[i] & 31;
+    for (size_t i = 0; i < ents.size();) {
+        const int q = ents[i].y;
         size_t j = i + 1;
-        while (j < pat.size() && (int)(j - i) < cmax && (pat[j] & 31) == q && (pat[j] >> 5) == (pat[i] >> 5) + (int)(j - i)) ++j;
-        // trim chunks off the run's start / end until its ranges lie inside x
+        while (j < ents.size() && (int)(j - i) < cmax && next_of(i, j)) ++j;
         size_t a = i, b = j;
-        for (int m; a < b && (m = misfit((int64_t)(pat[a] >> 5) * 32, (int)(b - a) * 32, q)) != 0;) {
-            if (m == 1) rest.push_back(pat[a++]);
-            else rest.push_back(pat[--b]);
+        for (int m; a < b && (m = misfit((int64_t)ents[a].x * 32, (int)(b - a) * 32, q)) != 0;) {
+            if (m == 1) rest->push_back(a++);
+            else rest->push_back(--b);
         }
         if (a < b) {
-            tiles.push_back(make_int2(pat[a] >> 5, ((int)(b - a) << 5) | q));
+            tiles.push_back(make_int4(ents[a].x, ((int)(b - a) << 5) | q, ents[a].z, 0));
             tiled += (int64_t)(b - a);
         }
         i = j;
     }
-    if (tiles.empty()) return PEPP_OK;
+    if (tiles.empty()) { rest->clear(); return PEPP_OK; }
     pepp_status_t s;
-    if ((s = dalloc(p, &p->d_ptiles, (int64_t)tiles.size()))) return s;
-    PEPP_CUDA_TRY(cudaMemcpy(p->d_ptiles, tiles.data(), sizeof(int2) * tiles.size(), cudaMemcpyHostToDevice));
-    if (!rest.empty()) {
-        if ((s = dalloc(p, &p->d_patrest, (int64_t)rest.size()))) return s;
-        PEPP_CUDA_TRY(cudaMemcpy(p->d_patrest, rest.data(), sizeof(int) * rest.size(), cudaMemcpyHostToDevice));
-    }
-    p->nptiles = (int)tiles.size();
-    p->npatrest = (int)rest.size();
-    p->ptile_chunks = tiled;
-    p->ptile_rows = rows;
-    p->ptile_stage = (int)stage;
-    p->ptt = tt;
-    p->ptile_smem = (size_t)kPtileS * (size_t)stage * sizeof(T) + 24 * kPtileS;
-    const void* fn = (const void*)pepp::k::sell_ptile_kernel<kPtileBlock, kPtileS, T>;
-    PEPP_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->ptile_smem));
+    if ((s = dalloc(p, &L->d_tiles, (int64_t)tiles.size()))) return s;
+    PEPP_CUDA_TRY(cudaMemcpy(L->d_tiles, tiles.data(), sizeof(int4) * tiles.size(), cudaMemcpyHostToDevice));
+    L->ntiles = (int)tiles.size();
+    L->chunks = tiled;
+    L->rows = rows;
+    L->stage = (int)stage_of(rows);
+    L->vstage = vals ? (int)xpart(rows) : 0;
+    L->tt = tt;
+    L->smem = (size_t)S * (size_t)L->stage * sizeof(T) + 32 * S;
+    const void* fn = vals ? (S == kStileS ? tile_kernel_fn<kStileS, true, T>() : nullptr) : tile_kernel_fn<kPtileS, false, T>();
+    PEPP_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem));
     int occ = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kPtileBlock, p->ptile_smem) != cudaSuccess || occ < 1) occ = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kPtileBlock, L->smem) != cudaSuccess || occ < 1) occ = 1;
     (void)cudaGetLastError();
-    p->grid_ptile = (int)std::max<int64_t>(1, std::min<int64_t>(p->nptiles, (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ));
-    if (p->ngen + p->npatrest > 0 && kSlistConcurrent && !p->gside) {
-        PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->gside, cudaStreamNonBlocking));
-        PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gfork, cudaEventDisableTiming));
-        PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gjoin, cudaEventDisableTiming));
+    L->grid = (int)std::max<int64_t>(1, std::min<int64_t>(L->ntiles, (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ));
+    return PEPP_OK;
+}
+
+pepp_status_t ensure_side_stream(pepp_spmv_plan_t* p) {
+    if (!kSlistConcurrent || p->gside) return PEPP_OK;
+    PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->gside, cudaStreamNonBlocking));
+    PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gfork, cudaEventDisableTiming));
+    PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gjoin, cudaEventDisableTiming));
+    return PEPP_OK;
+}
+
+// pattern tiles from the pattern list (entries chunk << 5 | id); untiled
+// entries -> d_patrest (phase A of the genlist walk)
+template <typename T>
+pepp_status_t sell_pattern_tiles(pepp_spmv_plan_t* p, const pepp::k::SellPatterns<T>& pt, const std::vector<int>& pat) {
+    int npat = 0;
+    for (int e : pat) npat = std::max(npat, (e & 31) + 1);
+    int lens[pepp::k::kTileMaxSets] = {0};
+    int offs[pepp::k::kTileMaxSets][pepp::k::kTileMaxLen] = {{0}};
+    for (int q = 0; q < npat; ++q) {
+        lens[q] = pt.len[q];
+        for (int j = 0; j < pt.len[q]; ++j) offs[q][j] = pt.off[q][j];
     }
+    std::vector<int4> ents(pat.size());
+    for (size_t i = 0; i < pat.size(); ++i) ents[i] = make_int4(pat[i] >> 5, pat[i] & 31, 0, 0);
+    std::vector<size_t> rest;
+    pepp_status_t s;
+    if ((s = sell_build_tiles<T>(p, npat, lens, offs, ents, false, &p->ptl, &rest))) return s;
+    if (!p->ptl.ntiles) return PEPP_OK;
+    std::sort(rest.begin(), rest.end());   // the pattern list's order (grouped by id)
+    if (!rest.empty()) {
+        std::vector<int> r(rest.size());
+        for (size_t i = 0; i < rest.size(); ++i) r[i] = pat[rest[i]];
+        if ((s = dalloc(p, &p->d_patrest, (int64_t)r.size()))) return s;
+        PEPP_CUDA_TRY(cudaMemcpy(p->d_patrest, r.data(), sizeof(int) * r.size(), cudaMemcpyHostToDevice));
+    }
+    p->npatrest = (int)rest.size();
+    if (p->ngen + p->npatrest > 0) return ensure_side_stream(p);
     return PEPP_OK;
 }
 
@@ -781,7 +851,8 @@ pepp_status_t sell_layout_bytes(pepp_spmv_plan_t* p) {
         if (d & pepp::k::kSellMasked) b += 4 * 32;
     }
     if (p->d_perm) b += 4 * p->nrows;
-    b += 8 * (int64_t)p->nptiles - 4 * p->ptile_chunks;   // tiled pattern chunks: one 8 B tile entry per tile
+    b += 16 * (int64_t)p->ptl.ntiles - 4 * p->ptl.chunks;   // tiled pattern chunks: one 16 B tile entry per tile
+    b += 16 * (int64_t)p->stl.ntiles - 8 * p->stl.chunks;   // tiled stencil-list chunks: likewise
     b += p->sell_long_nnz * (es + 4) + (int64_t)p->nsell_mid * (4 + 8) + (int64_t)p->nsell_long * 8 +
          (int64_t)p->nsell_seg * (16 + 16);
     b += p->ncols * es + p->nrows * es;
@@ -927,7 +998,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->info.sell_col16_frac = p->nchunks ? (double)p->sell_col16_chunks / (double)p->nchunks : 0.0;
     p->info.sell_stencil_frac = p->nchunks ? (double)p->sell_stencil_chunks / (double)p->nchunks : 0.0;
     p->info.sell_constval_frac = p->nchunks ? (double)p->sell_const_chunks / (double)p->nchunks : 0.0;
-    p->info.sell_ptile_frac = p->nchunks ? (double)p->ptile_chunks / (double)p->nchunks : 0.0;
+    p->info.sell_ptile_frac = p->nchunks ? (double)(p->ptl.chunks + p->stl.chunks) / (double)p->nchunks : 0.0;
     p->info.sell_fill = fill;
     p->info.sell_long_rows = p->nsell_long + p->nsell_mid;
     p->info.sell_cap = p->sell_cap == INT32_MAX ? 0 : p->sell_cap;
@@ -992,6 +1063,29 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
     p->nstc = (int)lst.size();
     p->ngen = (int)gen.size();
     p->stab = tab;
+    // stencil tiles over the list (the untiled entries -> d_strest)
+    if (kStencilTiles & (p->vt == PEPP_VALUE_F32 ? 1 : 2)) {
+        std::vector<int4> ents(lst.size());
+        for (size_t i = 0; i < lst.size(); ++i)
+            ents[i] = make_int4(lst[i].x & ((1 << 26) - 1), lst[i].x >> 26, lst[i].y, 0);
+        std::vector<size_t> rest;
+        int offs[pepp::k::kTileMaxSets][pepp::k::kTileMaxLen] = {{0}};
+        for (int q = 0; q < nset; ++q)
+            for (int j = 0; j < tab.len[q]; ++j) offs[q][j] = tab.off[q][j];
+        pepp_status_t st2 = p->vt == PEPP_VALUE_F32
+            ? sell_build_tiles<float>(p, nset, tab.len, offs, ents, true, &p->stl, &rest)
+            : sell_build_tiles<double>(p, nset, tab.len, offs, ents, true, &p->stl, &rest);
+        if (st2) return st2;
+        if (p->stl.ntiles && !rest.empty()) {
+            std::sort(rest.begin(), rest.end());
+            std::vector<int2> r(rest.size());
+            for (size_t i = 0; i < rest.size(); ++i) r[i] = lst[rest[i]];
+            if ((s = dalloc(p, &p->d_strest, (int64_t)r.size()))) return s;
+            PEPP_CUDA_TRY(cudaMemcpy(p->d_strest, r.data(), sizeof(int2) * r.size(), cudaMemcpyHostToDevice));
+            p->nstrest = (int)r.size();
+        }
+        if (p->stl.ntiles && p->nstrest && (s = ensure_side_stream(p))) return s;
+    }
     if (p->ngen > 0 && kSlistConcurrent) {
         PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->gside, cudaStreamNonBlocking));
         PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gfork, cudaEventDisableTiming));
@@ -1312,7 +1406,7 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                 (int)p->nrows, p->nchunks, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, p->d_perm, p->d_scol,
                 p->d_scol16, p->d_soff, pepp::k::NoPatterns{}, (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws,
                 nullptr, 0, nullptr);
-        else if (p->d_patlist && p->nptiles && ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0) {
+        else if (p->d_patlist && p->ptl.ntiles && ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0) {
             // pattern tiles (bulk-copied x ranges) on st; the grid-edge chunks
             // and the untiled pattern chunks through the genlist walk beside it
             cudaStream_t gs = p->gside ? p->gside : st;
@@ -1320,10 +1414,10 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
             if (side && p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
                                      cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
                 return PEPP_E_CUDA;
-            pepp::k::sell_ptile_kernel<kPtileBlock, kPtileS, T><<<p->grid_ptile, kPtileBlock, p->ptile_smem, st>>>(
-                sell_pattern_table<T>(p), p->ptt, p->d_ptiles, p->nptiles, p->ptile_stage, x, y);
+            pepp::k::sell_tile_kernel<kPtileBlock, kPtileS, false, T><<<p->ptl.grid, kPtileBlock, p->ptl.smem, st>>>(
+                sell_pattern_table<T>(p), p->ptl.tt, p->ptl.d_tiles, p->ptl.ntiles, p->ptl.stage, 0, nullptr, x, y);
             if (side)
-                pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, gs>>>(
+                pepp::k::sell_kernel<kBlock, false, true, T><<<tile_side_grid(p, p->grid_sell), kBlock, 0, gs>>>(
                     (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                     p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
                     p->d_patrest, p->npatrest, p->d_genlist);
@@ -1335,7 +1429,34 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                 (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
                 p->d_patlist, p->npatc, p->d_genlist);
-        else if (p->d_stlist) {   // stencil list (values streamed) and the other chunks (disjoint rows)
+        else if (p->d_stlist && p->stl.ntiles && ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0) {
+            // stencil tiles (bulk-copied x ranges and values) on st; the grid-edge
+            // chunks and the untiled list entries beside it on the side stream
+            cudaStream_t gs = p->gside ? p->gside : st;
+            const bool side = p->ngen + p->nstrest > 0;
+            if (side && p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
+                                     cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
+                return PEPP_E_CUDA;
+            pepp::k::sell_tile_kernel<kPtileBlock, kStileS, true, T><<<p->stl.grid, kPtileBlock, p->stl.smem, st>>>(
+                sell_pattern_table<T>(p), p->stl.tt, p->stl.d_tiles, p->stl.ntiles, p->stl.stage, p->stl.vstage,
+                (const T*)p->d_sval, x, y);
+            if (p->nstrest) {
+                if (p->slist_long)
+                    pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T, 16>(), 16, T><<<tile_side_grid(p, p->grid_slist), kBlock, 0, gs>>>(
+                        p->d_strest, p->nstrest, p->stab, (const T*)p->d_sval, x, y);
+                else
+                    pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), 8, T><<<tile_side_grid(p, p->grid_slist), kBlock, 0, gs>>>(
+                        p->d_strest, p->nstrest, p->stab, (const T*)p->d_sval, x, y);
+            }
+            if (p->ngen > 0)
+                pepp::k::sell_kernel<kBlock, false, true, T><<<tile_side_grid(p, p->grid_sell), kBlock, 0, gs>>>(
+                    (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
+                    p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
+                    nullptr, 0, p->d_genlist);
+            if (side && p->gside && (cudaEventRecord(p->ev_gjoin, p->gside) != cudaSuccess ||
+                                     cudaStreamWaitEvent(st, p->ev_gjoin, 0) != cudaSuccess))
+                return PEPP_E_CUDA;
+        } else if (p->d_stlist) {   // stencil list (values streamed) and the other chunks (disjoint rows)
             // the small, latency-bound genlist walk runs beside the list kernel
             // on the plan's second stream when it has one (kSlistConcurrent)
             cudaStream_t gs = p->gside ? p->gside : st;
@@ -1397,7 +1518,8 @@ int launches_for(const pepp_spmv_plan_t* p, const Candidate& c) {
         return p->ntiles > 0 ? 2 + (p->nlongruns > 0) : 0;
     case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
     case PEPP_V_SELL:
-        return (p->d_stlist ? 1 + (p->ngen > 0) : (p->d_patlist && p->nptiles) ? 1 + (p->ngen + p->npatrest > 0) : 1) +
+        return (p->d_stlist ? (p->stl.ntiles ? 1 + (p->nstrest > 0) : 1) + (p->ngen > 0)
+                            : (p->d_patlist && p->ptl.ntiles) ? 1 + (p->ngen + p->npatrest > 0) : 1) +
                (p->nsell_mid > 0) + (p->nsell_seg > 0);
     case PEPP_V_PANEL:
         for (const auto& pl : p->panels)

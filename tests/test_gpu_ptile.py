@@ -1,7 +1,9 @@
-"""GPU parity of the pattern-tile kernel (sell_ptile_kernel): value-compressed
-σ = 1 plans compute runs of pattern chunks from x ranges bulk-copied into
-shared memory. Per row the same FMAs in the same slot order as the
-register path, so y must be bit-identical to the streamed layout (and to
+"""GPU parity of the SELL tile kernel (sell_tile_kernel): σ = 1 plans compute
+runs of stencil chunks from x ranges (and, when the values stream, the
+chunks' value block) bulk-copied into shared memory — pattern tiles for
+value-compressed plans, stencil tiles over the stencil list otherwise. Per
+row the same FMAs in the same slot order as the register paths, so y must
+be bit-identical between the layouts and the register paths (and equal to
 the oracle on integer inputs, within the north-star bound on real ones).
 Covers: 2-D / 3-D stencils (1-5 offset clusters), fp64 and fp32, x / y
 views that are not 16-byte aligned (the register path runs instead), tiles
@@ -46,8 +48,9 @@ def test_ptile_laplacian_bit_identical(n):
     for x in (gen.vector(3, gen.INT8, A.ncols), gen.vector(4, gen.REAL, A.ncols)):
         y1, i1 = _y(A, x, True)
         y0, i0 = _y(A, x, False)
-        assert i0["sell_ptile_frac"] == 0.0
         assert i1["sell_ptile_frac"] > (0.9 if n == 1024 else 0.3)
+        if n == 1024:   # (96-wide grid rows straddle chunks: too few stencil chunks for the list)
+            assert i0["sell_ptile_frac"] > 0.9
         assert i1["sell_ptile_frac"] <= i1["sell_constval_frac"]
         assert np.array_equal(_bits(y1), _bits(y0))
         _check(A, x, y1, bool(np.all(x == np.round(x))))
@@ -58,12 +61,13 @@ def test_ptile_misaligned_views_fall_back_bit_identical():
     bulk copies cannot run; the call takes the register path — same bits."""
     A = gen.laplacian2d(300)
     x = gen.vector(5, gen.REAL, A.ncols)
-    ya, ia = _y(A, x, True)
-    for shift in (1, 2):
-        yb, _ = _y(A, x, True, shift=shift)
-        assert np.array_equal(_bits(ya), _bits(yb)), shift
-    assert ia["sell_ptile_frac"] > 0.5
-    _check(A, x, ya, False)
+    for compress in (True, False):
+        ya, ia = _y(A, x, compress)
+        for shift in (1, 2):
+            yb, _ = _y(A, x, compress, shift=shift)
+            assert np.array_equal(_bits(ya), _bits(yb)), (compress, shift)
+        assert ia["sell_ptile_frac"] > 0.5
+        _check(A, x, ya, False)
 
 
 @pytest.mark.parametrize("name", ["lap3d_7pt", "grid_8pt", "lap1d", "edge"])
@@ -90,6 +94,8 @@ def test_ptile_stencils(name):
     for x in (gen.vector(3, gen.INT8, A.ncols), gen.vector(4, gen.REAL, A.ncols)):
         y1, i1 = _y(A, x, True)
         y0, _ = _y(A, x, False)
+        y2, _ = _y(A, x, False, shift=1)   # register stencil-list path
+        assert np.array_equal(_bits(y0), _bits(y2))
         if name == "edge":
             assert i1["sell_ptile_frac"] == pytest.approx(49 / 50)
         else:
@@ -103,8 +109,10 @@ def test_ptile_fp32_bit_identical_and_within_bound():
     x = gen.vector(8, gen.REAL, A.ncols).astype(np.float32)
     A32 = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, A.val.astype(np.float32), A.r0, A.global_nrows)
     y1, i1 = _y(A32, x, True, dt=torch.float32)
-    y0, _ = _y(A32, x, False, dt=torch.float32)
-    assert i1["sell_ptile_frac"] > 0.9
+    y0, i0 = _y(A32, x, False, dt=torch.float32)
+    assert i1["sell_ptile_frac"] > 0.9 and i0["sell_ptile_frac"] > 0.9
+    y2, _ = _y(A32, x, False, dt=torch.float32, shift=1)   # register stencil-list path
+    assert np.array_equal(_bits(y0), _bits(y2))
     assert np.array_equal(_bits(y1), _bits(y0))
     b = oracle.bound_f32(A32, x)
     yr = oracle.spmv_f32(A32, x)
