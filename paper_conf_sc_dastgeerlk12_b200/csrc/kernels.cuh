@@ -1156,14 +1156,23 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // Consumer thread c of NC: rows c, c + NC, ... of the tile, U at a time
 // (all shared-memory loads of the U rows first), written straight to y.
 // VALS: slot j of row i is sv[(i / 32) * 32N + 32 j + i % 32].
+#ifndef PEPP_TILE_CHECKS
+#define PEPP_TILE_CHECKS 0   // 1: bounds traps in sell_tile_kernel (debug builds, tools/r2/gpu_tile_checks.sh)
+#endif
 template <int NC, int N, bool VALS, typename T>
 __device__ __forceinline__ void tile_rows(const SellPatterns<T>& pt, const PatTiles& tt, int q, const T* sx,
-                                          const T* sv, T* __restrict__ y, int nr, int c) {
+                                          const T* sv, T* __restrict__ y, int nr, int c, int xspan) {
     constexpr int U = !VALS ? PEPP_PTILE_U : (N <= 4 ? 4 : N <= 8 ? 2 : 1);
     int b[N];
     T w[N];
 #pragma unroll
     for (int j = 0; j < N; ++j) { b[j] = tt.sidx[q][j]; w[j] = VALS ? T(0) : pt.val[q][j]; }
+#if PEPP_TILE_CHECKS
+    for (int j = 0; j < N; ++j)
+        if (b[j] < 0 || b[j] + nr > xspan) __trap();   // every slot's reads inside the stage's x part
+#else
+    (void)xspan;
+#endif
     for (int i0 = c; i0 < nr; i0 += NC * U) {
         T xv[U][N], vv[VALS ? U : 1][N];
 #pragma unroll
@@ -1208,7 +1217,7 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
                                                              const int4* __restrict__ tiles, int ntiles,
                                                              int stage_elems, int vstage,
                                                              const T* __restrict__ val, const T* __restrict__ x,
-                                                             T* __restrict__ y) {
+                                                             T* __restrict__ y, int64_t xlen) {
     extern __shared__ __align__(128) unsigned char ptile_smem[];
     constexpr int A = 16 / sizeof(T);
     constexpr int NCW = BLOCK / 32 - 1, NC = NCW * 32;
@@ -1240,6 +1249,15 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
             const uint32_t vbytes = VALS ? (uint32_t)nr * tt.len[q] * sizeof(T) : 0;
             mbar_arrive_expect_tx(&full[s], bytes + vbytes);
             T* dst = sx + (size_t)s * stage_elems;
+#if PEPP_TILE_CHECKS
+            // debug build (compute-sanitizer is not available on the GPU pool):
+            // every copy inside x / its stage, the value block after the ranges
+            for (int c = 0; c < nc; ++c) {
+                const int64_t a = r0 + tt.clo[q][c], n = ((nr + tt.cext[q][c] + A - 1) / A) * A;
+                if (a < 0 || a + n > xlen || tt.cdst[q][c] + n > (VALS ? vstage : stage_elems)) __trap();
+            }
+            if (VALS && vstage + (int64_t)nr * tt.len[q] > stage_elems) __trap();
+#endif
             for (int c = 0; c < nc; ++c)
                 tma_load_1d_nohint(dst + tt.cdst[q][c], x + r0 + tt.clo[q][c],
                                    (uint32_t)(((nr + tt.cext[q][c] + A - 1) / A) * A) * sizeof(T), &full[s]);
@@ -1259,17 +1277,17 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
         const T* xs = sx + (size_t)s * stage_elems;
         const T* vs = xs + vstage;
         T* yt = y + (int64_t)e.x * 32;
-#define PEPP_TR(N) case N: tile_rows<NC, N, VALS, T>(pt, tt, q, xs, vs, yt, nr, c); break;
+#define PEPP_TR(N) case N: tile_rows<NC, N, VALS, T>(pt, tt, q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems); break;
         switch (tt.len[q]) {
         PEPP_TR(1) PEPP_TR(2) PEPP_TR(3) PEPP_TR(4) PEPP_TR(5) PEPP_TR(6) PEPP_TR(7)
         default:
             if constexpr (VALS) {
                 switch (tt.len[q]) {
                 PEPP_TR(8) PEPP_TR(9) PEPP_TR(10) PEPP_TR(11) PEPP_TR(12) PEPP_TR(13) PEPP_TR(14) PEPP_TR(15)
-                default: tile_rows<NC, 16, VALS, T>(pt, tt, q, xs, vs, yt, nr, c); break;
+                default: tile_rows<NC, 16, VALS, T>(pt, tt, q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems); break;
                 }
             } else {
-                tile_rows<NC, 8, VALS, T>(pt, tt, q, xs, vs, yt, nr, c);
+                tile_rows<NC, 8, VALS, T>(pt, tt, q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems);
             }
             break;
         }

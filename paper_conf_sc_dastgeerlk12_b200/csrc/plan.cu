@@ -488,6 +488,9 @@ constexpr size_t kPtileSmemBudget = (size_t)PEPP_PTILE_SMEM_KB * 1024;
 #ifndef PEPP_TILE_SIDE_BPS
 #define PEPP_TILE_SIDE_BPS 8   // blocks per SM (cap) of the walks beside a tile kernel; measured 1 / 2 / 8: vc config 4 207.5 / 197.9 / 197.0 us, fp32 list 293 / 282 / 282 us
 #endif
+#ifndef PEPP_EXP_TILE_SIDE
+#define PEPP_EXP_TILE_SIDE 0   // experiments only: 1 = the side walks after the tile kernel on its stream, 2 = skipped (wrong y)
+#endif
 int tile_side_grid(const pepp_spmv_plan_t* p, int grid) {
     return std::max(1, std::min(grid, PEPP_TILE_SIDE_BPS * std::max(1, p->sm_count - p->reserve_sms)));
 }
@@ -1084,9 +1087,9 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
             PEPP_CUDA_TRY(cudaMemcpy(p->d_strest, r.data(), sizeof(int2) * r.size(), cudaMemcpyHostToDevice));
             p->nstrest = (int)r.size();
         }
-        if (p->stl.ntiles && p->nstrest && (s = ensure_side_stream(p))) return s;
+        if (p->stl.ntiles && (p->nstrest || p->ngen) && (s = ensure_side_stream(p))) return s;
     }
-    if (p->ngen > 0 && kSlistConcurrent) {
+    if (p->ngen > 0 && kSlistConcurrent && !p->gside) {
         PEPP_CUDA_TRY(cudaStreamCreateWithFlags(&p->gside, cudaStreamNonBlocking));
         PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gfork, cudaEventDisableTiming));
         PEPP_CUDA_TRY(cudaEventCreateWithFlags(&p->ev_gjoin, cudaEventDisableTiming));
@@ -1409,13 +1412,13 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
         else if (p->d_patlist && p->ptl.ntiles && ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0) {
             // pattern tiles (bulk-copied x ranges) on st; the grid-edge chunks
             // and the untiled pattern chunks through the genlist walk beside it
-            cudaStream_t gs = p->gside ? p->gside : st;
-            const bool side = p->ngen + p->npatrest > 0;
+            cudaStream_t gs = p->gside && PEPP_EXP_TILE_SIDE == 0 ? p->gside : st;
+            const bool side = p->ngen + p->npatrest > 0 && PEPP_EXP_TILE_SIDE != 2;
             if (side && p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
                                      cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
                 return PEPP_E_CUDA;
             pepp::k::sell_tile_kernel<kPtileBlock, kPtileS, false, T><<<p->ptl.grid, kPtileBlock, p->ptl.smem, st>>>(
-                sell_pattern_table<T>(p), p->ptl.tt, p->ptl.d_tiles, p->ptl.ntiles, p->ptl.stage, 0, nullptr, x, y);
+                sell_pattern_table<T>(p), p->ptl.tt, p->ptl.d_tiles, p->ptl.ntiles, p->ptl.stage, 0, nullptr, x, y, p->ncols);
             if (side)
                 pepp::k::sell_kernel<kBlock, false, true, T><<<tile_side_grid(p, p->grid_sell), kBlock, 0, gs>>>(
                     (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
@@ -1432,14 +1435,14 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
         else if (p->d_stlist && p->stl.ntiles && ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0) {
             // stencil tiles (bulk-copied x ranges and values) on st; the grid-edge
             // chunks and the untiled list entries beside it on the side stream
-            cudaStream_t gs = p->gside ? p->gside : st;
-            const bool side = p->ngen + p->nstrest > 0;
+            cudaStream_t gs = p->gside && PEPP_EXP_TILE_SIDE == 0 ? p->gside : st;
+            const bool side = p->ngen + p->nstrest > 0 && PEPP_EXP_TILE_SIDE != 2;
             if (side && p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
                                      cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
                 return PEPP_E_CUDA;
             pepp::k::sell_tile_kernel<kPtileBlock, kStileS, true, T><<<p->stl.grid, kPtileBlock, p->stl.smem, st>>>(
                 sell_pattern_table<T>(p), p->stl.tt, p->stl.d_tiles, p->stl.ntiles, p->stl.stage, p->stl.vstage,
-                (const T*)p->d_sval, x, y);
+                (const T*)p->d_sval, x, y, p->ncols);
             if (p->nstrest) {
                 if (p->slist_long)
                     pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T, 16>(), 16, T><<<tile_side_grid(p, p->grid_slist), kBlock, 0, gs>>>(

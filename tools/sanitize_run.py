@@ -82,6 +82,20 @@ def main() -> int:
         plan.exec(torch.from_numpy(x32).cuda(), y32, force=pepp.Choice(pepp.V_SELL, 0))
         torch.cuda.synchronize()
         bad += 0 if np.array_equal(y32.cpu().numpy(), oracle.spmv(A32, x32)) else 1
+    # SELL tiles (bulk-copied ranges, producer / consumer mbarrier ring):
+    # pattern tiles and stencil tiles, fp64 and fp32, more tiles than CTAs
+    L = gen.laplacian2d(256)
+    for dt in (np.float64, np.float32):
+        Ld = gen.CSR(L.nrows, L.ncols, L.row_ptr, L.col, L.val.astype(dt), L.r0, L.global_nrows, L.name)
+        xl = gen.vector(5, gen.INT8, L.ncols).astype(dt)
+        for cz in (True, False):
+            with pepp.Plan.from_csr(Ld, compress_values=cz, variant_mask=1 << pepp.V_SELL) as plan:
+                yl = torch.full((L.nrows,), float("nan"), dtype=torch.from_numpy(xl).dtype, device="cuda")
+                for _ in range(3):
+                    plan.exec(torch.from_numpy(xl).cuda(), yl)
+                torch.cuda.synchronize()
+                ok = plan.info()["sell_ptile_frac"] > 0.5 and np.array_equal(yl.cpu().numpy(), oracle.spmv(Ld, xl) if dt == np.float64 else oracle.spmv_f32(Ld, xl))
+                bad += 0 if ok else 1
     # overlapped host batch (copy streams, two device slots)
     with pepp.Plan.from_csr(A) as plan:
         xs = [gen.vector(30 + k, gen.INT8, A.nrows) for k in range(3)]
