@@ -1144,6 +1144,14 @@ struct PatTiles {
     int cext[kTileMaxSets][kTileMaxLen];         // elements copied = round16(nr + cext)
     int cdst[kTileMaxSets][kTileMaxLen];         // cluster c's element offset within a stage
     int sidx[kTileMaxSets][kTileMaxLen];         // slot j: stage element of the tile's row 0
+    // multi-line tiles (!VALS; tile entry .z = K > 0): the set's offsets are
+    // a_j·D + b_j with a_j in [amin, amax] (a grid stencil, D = the line
+    // stride); a tile is K lines of nr rows, r0 + l·D (l < K), and loads the
+    // K + W lines (W = amax - amin) x[r0 + lbase + m·D, + round16(nr + lext))
+    // once each into stage line m (stride lws) — x crosses L2 -> SM
+    // (K + W) / K times instead of once per cluster per line
+    int D[kTileMaxSets], W[kTileMaxSets], lbase[kTileMaxSets], lext[kTileMaxSets], lws[kTileMaxSets];
+    int msidx[kTileMaxSets][kTileMaxLen];        // slot j: stage element of line 0's row 0
 };
 
 #ifndef PEPP_PTILE_U
@@ -1160,13 +1168,13 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 #define PEPP_TILE_CHECKS 0   // 1: bounds traps in sell_tile_kernel (debug builds, tools/r2/gpu_tile_checks.sh)
 #endif
 template <int NC, int N, bool VALS, typename T>
-__device__ __forceinline__ void tile_rows(const SellPatterns<T>& pt, const PatTiles& tt, int q, const T* sx,
+__device__ __forceinline__ void tile_rows(const SellPatterns<T>& pt, const int* sidx, int q, const T* sx,
                                           const T* sv, T* __restrict__ y, int nr, int c, int xspan) {
     constexpr int U = !VALS ? PEPP_PTILE_U : (N <= 4 ? 4 : N <= 8 ? 2 : 1);
     int b[N];
     T w[N];
 #pragma unroll
-    for (int j = 0; j < N; ++j) { b[j] = tt.sidx[q][j]; w[j] = VALS ? T(0) : pt.val[q][j]; }
+    for (int j = 0; j < N; ++j) { b[j] = sidx[j]; w[j] = VALS ? T(0) : pt.val[q][j]; }
 #if PEPP_TILE_CHECKS
     for (int j = 0; j < N; ++j)
         if (b[j] < 0 || b[j] + nr > xspan) __trap();   // every slot's reads inside the stage's x part
@@ -1244,6 +1252,22 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
             const int64_t r0 = (int64_t)e.x * 32;
             const int nr = (e.y >> 5) * 32, q = e.y & 31, nc = tt.ncl[q];
             ent[s] = e;
+            if (!VALS && e.z > 0) {   // multi-line tile: K + W lines, each once
+                const int nl = e.z + tt.W[q];
+                const uint32_t lb = (uint32_t)(((nr + tt.lext[q] + A - 1) / A) * A) * sizeof(T);
+                mbar_arrive_expect_tx(&full[s], lb * nl);
+                T* dst = sx + (size_t)s * stage_elems;
+                const T* src = x + r0 + tt.lbase[q];
+                for (int m = 0; m < nl; ++m) {
+#if PEPP_TILE_CHECKS
+                    const int64_t a = r0 + tt.lbase[q] + (int64_t)m * tt.D[q];
+                    if (a < 0 || a + lb / sizeof(T) > xlen || (int64_t)m * tt.lws[q] + lb / sizeof(T) > stage_elems) __trap();
+#endif
+                    tma_load_1d_nohint(dst + m * tt.lws[q], src + (int64_t)m * tt.D[q], lb, &full[s]);
+                }
+                e = en;
+                continue;
+            }
             uint32_t bytes = 0;
             for (int c = 0; c < nc; ++c) bytes += (uint32_t)(((nr + tt.cext[q][c] + A - 1) / A) * A) * sizeof(T);
             const uint32_t vbytes = VALS ? (uint32_t)nr * tt.len[q] * sizeof(T) : 0;
@@ -1277,17 +1301,33 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
         const T* xs = sx + (size_t)s * stage_elems;
         const T* vs = xs + vstage;
         T* yt = y + (int64_t)e.x * 32;
-#define PEPP_TR(N) case N: tile_rows<NC, N, VALS, T>(pt, tt, q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems); break;
+        if (!VALS && e.z > 0) {   // multi-line tile: line l's rows from stage line l (+ the slots' line offsets)
+            for (int l = 0; l < e.z; ++l) {
+                const T* xl = xs + l * tt.lws[q];
+                T* yl = yt + (int64_t)l * tt.D[q];
+                const int span = stage_elems - l * tt.lws[q];
+#define PEPP_TM(N) case N: tile_rows<NC, N, VALS, T>(pt, tt.msidx[q], q, xl, vs, yl, nr, c, span); break;
+                switch (tt.len[q]) {
+                PEPP_TM(1) PEPP_TM(2) PEPP_TM(3) PEPP_TM(4) PEPP_TM(5) PEPP_TM(6) PEPP_TM(7)
+                default: tile_rows<NC, 8, VALS, T>(pt, tt.msidx[q], q, xl, vs, yl, nr, c, span); break;
+                }
+#undef PEPP_TM
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+            continue;
+        }
+#define PEPP_TR(N) case N: tile_rows<NC, N, VALS, T>(pt, tt.sidx[q], q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems); break;
         switch (tt.len[q]) {
         PEPP_TR(1) PEPP_TR(2) PEPP_TR(3) PEPP_TR(4) PEPP_TR(5) PEPP_TR(6) PEPP_TR(7)
         default:
             if constexpr (VALS) {
                 switch (tt.len[q]) {
                 PEPP_TR(8) PEPP_TR(9) PEPP_TR(10) PEPP_TR(11) PEPP_TR(12) PEPP_TR(13) PEPP_TR(14) PEPP_TR(15)
-                default: tile_rows<NC, 16, VALS, T>(pt, tt, q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems); break;
+                default: tile_rows<NC, 16, VALS, T>(pt, tt.sidx[q], q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems); break;
                 }
             } else {
-                tile_rows<NC, 8, VALS, T>(pt, tt, q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems);
+                tile_rows<NC, 8, VALS, T>(pt, tt.sidx[q], q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems);
             }
             break;
         }

@@ -18,6 +18,8 @@
 #include <thrust/iterator/counting_iterator.h>
 
 #include <algorithm>
+#include <map>
+#include <tuple>
 #include <chrono>
 #include <cmath>
 #include <cstdio>
@@ -90,6 +92,7 @@ struct TileLayout {
     int4* d_tiles = nullptr;      // {first chunk, chunks << 5 | set id, value block / 32, 0}
     int ntiles = 0, grid = 0, rows = 0, stage = 0, vstage = 0;
     int64_t chunks = 0;           // chunks the tiles hold
+    int64_t lines = 0;            // multi-line tiles among them
     size_t smem = 0;              // dynamic shared memory per CTA
     pepp::k::PatTiles tt{};
 };
@@ -462,7 +465,7 @@ pepp_status_t sell_warp_ranges(pepp_spmv_plan_t* p) {
 #define PEPP_STILE 3   // values streamed: stencil tiles (bit 0: fp32 plans, bit 1: fp64 plans); config 4: fp32 340 -> 281 us, fp64 605 -> 553 us (same box)
 #endif
 #ifndef PEPP_PTILE_S
-#define PEPP_PTILE_S 4   // stages, pattern tiles
+#define PEPP_PTILE_S 2   // stages, pattern tiles (multi-line tiles: K + W lines of 16 KB per stage)
 #endif
 #ifndef PEPP_STILE_S
 #define PEPP_STILE_S 3   // stages, stencil tiles (values streamed)
@@ -484,6 +487,15 @@ constexpr int kStencilTiles = PEPP_STILE;
 constexpr int kPtileS = PEPP_PTILE_S, kStileS = PEPP_STILE_S, kPtileBlock = PEPP_PTILE_BLOCK;
 constexpr int kTileGap = 64;
 constexpr size_t kPtileSmemBudget = (size_t)PEPP_PTILE_SMEM_KB * 1024;
+#ifndef PEPP_MTILE_K
+#define PEPP_MTILE_K 3   // lines per multi-line pattern tile (< 2: off); tools/r2/gpu_mtile.sh, config 4 fp64 / fp32 µs:
+                         // off 199.3 / 105.3; K=4, 8 KB lines, S=4 183.6 / 119.7; K=6 S=3 197.5 / 115.9;
+                         // K=8 S=2 181.0 / 116.3; K=2, 16 KB 214.9 / 116.8; K=3, 16 KB, S=2 181.6 / 102.6 (kept)
+#endif
+#ifndef PEPP_MTILE_LINE_KB
+#define PEPP_MTILE_LINE_KB 16   // x bytes per line (rows per line = 16 KB / value size)
+#endif
+constexpr int kMarchK = PEPP_MTILE_K, kMarchLineBytes = PEPP_MTILE_LINE_KB * 1024;
 
 #ifndef PEPP_TILE_SIDE_BPS
 #define PEPP_TILE_SIDE_BPS 8   // blocks per SM (cap) of the walks beside a tile kernel; measured 1 / 2 / 8: vc config 4 207.5 / 197.9 / 197.0 us, fp32 list 293 / 282 / 282 us
@@ -514,6 +526,7 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
     if (nsets > pepp::k::kTileMaxSets) return PEPP_OK;
     int64_t emax = 0;
     int maxcl = 1, maxlen = 1;
+    std::vector<std::pair<std::vector<int64_t>, std::vector<int64_t>>> clusters(nsets);
     for (int q = 0; q < nsets; ++q) {
         const int len = lens[q];
         if (len < 1 || len > kTileMaxLen) return PEPP_OK;
@@ -531,6 +544,7 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
         const int nc = (int)lo.size();
         tt.ncl[q] = nc;
         maxcl = std::max(maxcl, nc);
+        clusters[q] = {lo, hi};
         int64_t extra = 0;
         for (int c = 0; c < nc; ++c) {
             const int64_t clo = rdn(lo[c]), cext = hi[c] - clo;
@@ -541,12 +555,70 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
         }
         emax = std::max(emax, extra);
     }
-    // S stages (x ranges, + values) and barriers / entries within the budget
-    int rows = std::max(32, range_bytes / (int)sizeof(T) / 32 * 32);
+    // multi-line tiles (pattern tiles of grid stencils): per set, D = the
+    // largest |cluster centre|, a_c = round(centre_c / D), b_c = lo_c - a_c·D;
+    // usable when D keeps 16-B alignment, every |b_c| <= D / 4 and the lines
+    // stay short (lext <= 4096) — e.g. 5- / 9-point 2-D (W = 2), 7-point 3-D
+    // (D = n², ±n inside the line)
+    std::vector<int> amin_of(nsets, 0);
+    std::vector<std::vector<int>> a_of(nsets);
+    bool march = !vals && kMarchK >= 2;
+    int wmax = 0, lextmax = 0;
+    for (int q = 0; q < nsets && march; ++q) {
+        const auto& lo = clusters[q].first;
+        const auto& hi = clusters[q].second;
+        int64_t D = 0;
+        for (size_t c = 0; c < lo.size(); ++c) D = std::max<int64_t>(D, std::llabs((lo[c] + hi[c]) / 2));
+        tt.D[q] = 0;
+        if (D < 64 || D % A || D > INT32_MAX / 8) continue;   // no line structure: regular tiles
+        int amin = INT32_MAX, amax = INT32_MIN;
+        int64_t bmin = INT64_MAX, bmax = INT64_MIN;
+        bool ok = true;
+        std::vector<int> a(lo.size());
+        for (size_t c = 0; c < lo.size(); ++c) {
+            const double ctr = 0.5 * (double)(lo[c] + hi[c]);
+            a[c] = (int)std::llround(ctr / (double)D);
+            const int64_t b = lo[c] - (int64_t)a[c] * D;
+            ok &= std::llabs(b) <= D / 4;
+            amin = std::min(amin, a[c]);
+            amax = std::max(amax, a[c]);
+            bmin = std::min(bmin, b);
+            bmax = std::max(bmax, b + (hi[c] - lo[c]));
+        }
+        bmin = rdn(bmin);
+        if (!ok || amax - amin > 4 || bmax - bmin > 4096) continue;
+        tt.D[q] = (int)D;
+        tt.W[q] = amax - amin;
+        tt.lbase[q] = (int)((int64_t)amin * D + bmin);
+        tt.lext[q] = (int)(bmax - bmin);
+        amin_of[q] = amin;
+        a_of[q] = a;
+        wmax = std::max(wmax, tt.W[q]);
+        lextmax = std::max(lextmax, tt.lext[q]);
+    }
+    if (march) {
+        march = false;
+        for (int q = 0; q < nsets; ++q) march |= tt.D[q] > 0;
+    }
+    // S stages (x ranges, + values) and barriers / entries within the budget;
+    // with lines, rows per line = kMarchLineBytes of x and K + W lines per stage
+    int rows = std::max(32, (march ? kMarchLineBytes : range_bytes) / (int)sizeof(T) / 32 * 32);
     auto xpart = [&](int r) { return rup((int64_t)maxcl * r + emax); };
-    auto stage_of = [&](int r) { return xpart(r) + (vals ? (int64_t)r * maxlen : 0); };
+    auto mpart = [&](int r) { return march ? (int64_t)(kMarchK + wmax) * rup(r + lextmax) : 0; };
+    auto stage_of = [&](int r) { return std::max(xpart(r), mpart(r)) + (vals ? (int64_t)r * maxlen : 0); };
     while (rows >= 32 && (size_t)S * (size_t)stage_of(rows) * sizeof(T) + 32 * S + 64 > kPtileSmemBudget) rows -= 32;
     if (rows < 32) return PEPP_OK;
+    for (int q = 0; q < nsets && march; ++q) {
+        if (!tt.D[q]) continue;
+        tt.lws[q] = (int)rup(rows + lextmax);
+        const auto& lo = clusters[q].first;
+        for (int j = 0; j < tt.len[q]; ++j) {
+            size_t c = 0;
+            while (c + 1 < lo.size() && offs[q][j] >= lo[c + 1]) ++c;
+            const int64_t a = a_of[q][c];
+            tt.msidx[q][j] = (int)((a - amin_of[q]) * tt.lws[q] + (offs[q][j] - a * tt.D[q] - (tt.lbase[q] - (int64_t)amin_of[q] * tt.D[q])));
+        }
+    }
     for (int q = 0; q < nsets; ++q) {
         int64_t d = 0;
         for (int c = 0; c < tt.ncl[q]; ++c) { tt.cdst[q][c] = (int)d; d += rup(rows + tt.cext[q][c]); }
@@ -591,6 +663,50 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
         i = j;
     }
     if (tiles.empty()) { rest->clear(); return PEPP_OK; }
+    if (march) {
+        // columns: tiles of one set and length whose first rows differ by D,
+        // cut into blocks of <= K lines; a block of >= 2 lines becomes one
+        // multi-line tile when all its K + W lines lie inside x
+        std::map<std::tuple<int, int, int64_t>, std::vector<size_t>> cols;
+        for (size_t t = 0; t < tiles.size(); ++t) {
+            const int q = tiles[t].y & 31;
+            if (!tt.D[q]) continue;
+            const int64_t r0 = (int64_t)tiles[t].x * 32;
+            cols[{q, tiles[t].y >> 5, r0 % tt.D[q]}].push_back(t);
+        }
+        std::vector<uint8_t> absorbed(tiles.size(), 0);
+        std::vector<int4> multi;
+        for (auto& kv : cols) {
+            auto& v = kv.second;   // ascending r0 (tiles are in chunk order within a set)
+            const int q = std::get<0>(kv.first), nr = std::get<1>(kv.first) * 32;
+            const int64_t D = tt.D[q];
+            const int64_t lb = rup(nr + tt.lext[q]);
+            for (size_t i = 0; i < v.size();) {
+                size_t j = i + 1;
+                while (j < v.size() && (int)(j - i) < kMarchK &&
+                       (int64_t)tiles[v[j]].x * 32 == (int64_t)tiles[v[i]].x * 32 + (int64_t)(j - i) * D) ++j;
+                const int K = (int)(j - i);
+                const int64_t r0 = (int64_t)tiles[v[i]].x * 32;
+                const int64_t a = r0 + tt.lbase[q], b = a + (int64_t)(K + tt.W[q] - 1) * D + lb;
+                if (K >= 2 && a >= 0 && b <= p->ncols) {
+                    multi.push_back(make_int4(tiles[v[i]].x, tiles[v[i]].y, K, 0));
+                    for (size_t k = i; k < j; ++k) absorbed[v[k]] = 1;
+                }
+                i = j;
+            }
+        }
+        if (!multi.empty()) {
+            std::vector<int4> all;
+            for (size_t t = 0; t < tiles.size(); ++t) if (!absorbed[t]) all.push_back(tiles[t]);
+            all.insert(all.end(), multi.begin(), multi.end());
+            // set, then first row: the grid's front advances through x together
+            std::stable_sort(all.begin(), all.end(), [](const int4& u, const int4& w) {
+                return (u.y & 31) != (w.y & 31) ? (u.y & 31) < (w.y & 31) : u.x < w.x;
+            });
+            tiles.swap(all);
+            L->lines = (int64_t)multi.size();
+        }
+    }
     pepp_status_t s;
     if ((s = dalloc(p, &L->d_tiles, (int64_t)tiles.size()))) return s;
     PEPP_CUDA_TRY(cudaMemcpy(L->d_tiles, tiles.data(), sizeof(int4) * tiles.size(), cudaMemcpyHostToDevice));
