@@ -707,6 +707,17 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
             L->lines = (int64_t)multi.size();
         }
     }
+    const size_t smem = (size_t)S * (size_t)stage_of(rows) * sizeof(T) + 32 * S;
+    const void* fn = vals ? tile_kernel_fn<kStileS, true, T>() : tile_kernel_fn<kPtileS, false, T>();
+    // the attribute is per kernel, not per plan: set the budget every plan's
+    // tiles fit in (a plan setting its own, smaller size would make another
+    // plan's launches of the same kernel fail)
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPtileSmemBudget) != cudaSuccess) {
+        (void)cudaGetLastError();   // the device cannot give a CTA that much shared memory: no tiles
+        *L = TileLayout{};
+        rest->clear();
+        return PEPP_OK;
+    }
     pepp_status_t s;
     if ((s = dalloc(p, &L->d_tiles, (int64_t)tiles.size()))) return s;
     PEPP_CUDA_TRY(cudaMemcpy(L->d_tiles, tiles.data(), sizeof(int4) * tiles.size(), cudaMemcpyHostToDevice));
@@ -716,9 +727,7 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
     L->stage = (int)stage_of(rows);
     L->vstage = vals ? (int)xpart(rows) : 0;
     L->tt = tt;
-    L->smem = (size_t)S * (size_t)L->stage * sizeof(T) + 32 * S;
-    const void* fn = vals ? (S == kStileS ? tile_kernel_fn<kStileS, true, T>() : nullptr) : tile_kernel_fn<kPtileS, false, T>();
-    PEPP_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem));
+    L->smem = smem;
     int occ = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kPtileBlock, L->smem) != cudaSuccess || occ < 1) occ = 1;
     (void)cudaGetLastError();
@@ -1627,8 +1636,10 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
     return cudaGetLastError() == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
 }
 
-// kernels launch_t enqueues for candidate c (mirrors its conditions)
-int launches_for(const pepp_spmv_plan_t* p, const Candidate& c) {
+// kernels launch_t enqueues for candidate c (mirrors its conditions; the
+// tile kernels run only on 16-byte aligned x and y)
+int launches_for(const pepp_spmv_plan_t* p, const Candidate& c, const void* x, const void* y) {
+    const bool al = ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0;
     if (p->nrows == 0) return 0;
     switch (c.variant) {
     case PEPP_V_CSR_VECTOR: return 1;
@@ -1637,8 +1648,8 @@ int launches_for(const pepp_spmv_plan_t* p, const Candidate& c) {
         return p->ntiles > 0 ? 2 + (p->nlongruns > 0) : 0;
     case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
     case PEPP_V_SELL:
-        return (p->d_stlist ? (p->stl.ntiles ? 1 + (p->nstrest > 0) : 1) + (p->ngen > 0)
-                            : (p->d_patlist && p->ptl.ntiles) ? 1 + (p->ngen + p->npatrest > 0) : 1) +
+        return (p->d_stlist ? (p->stl.ntiles && al ? 1 + (p->nstrest > 0) : 1) + (p->ngen > 0)
+                            : (p->d_patlist && p->ptl.ntiles && al) ? 1 + (p->ngen + p->npatrest > 0) : 1) +
                (p->nsell_mid > 0) + (p->nsell_seg > 0);
     case PEPP_V_PANEL:
         for (const auto& pl : p->panels)
@@ -3157,7 +3168,7 @@ extern "C" PEPP_API pepp_status_t pepp_spmv_exec(pepp_spmv_plan_t* p, const void
     }
     pepp_status_t s = launch(p, p->cands[ch.candidate], x, (char*)y + p->row_offset * (int64_t)p->esz, st);
     if (s) { p->sticky = s; return s; }
-    ch.launches = launches_for(p, p->cands[ch.candidate]);
+    ch.launches = launches_for(p, p->cands[ch.candidate], x, (char*)y + p->row_offset * (int64_t)p->esz);
     if (rec) {
         if (cudaEventRecord(rec->stop, st) == cudaSuccess) {
             rec->cand = ch.candidate;

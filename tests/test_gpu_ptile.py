@@ -129,3 +129,23 @@ def test_ptile_nonfinite_x():
     assert np.array_equal(_bits(y1), _bits(y0))
     yr = oracle.spmv(A, x)
     assert np.array_equal(np.isnan(y1), np.isnan(yr)) and np.array_equal(np.isinf(y1), np.isinf(yr))
+
+
+def test_tile_plans_with_different_stage_sizes_interleave():
+    """The kernel's dynamic shared-memory limit is a per-kernel attribute:
+    a plan with smaller tiles created after one with larger tiles must not
+    make the first plan's launches fail (4-rank distribution hang, round 2)."""
+    A = gen.laplacian2d(1024)                                     # multi-line pattern tiles (5 lines / stage)
+    B = _stencil_grid(300_000, [(-1,), (0,), (1,)], 2.0, -1.0, dims=1)   # one cluster: a small stage
+    xa, xb = gen.vector(3, gen.INT8, A.ncols), gen.vector(4, gen.INT8, B.ncols)
+    with pepp.Plan.from_csr(A, variant_mask=1 << pepp.V_SELL) as pa, \
+            pepp.Plan.from_csr(B, variant_mask=1 << pepp.V_SELL) as pb:
+        ya = torch.full((A.nrows,), float("nan"), dtype=torch.float64, device="cuda")
+        yb = torch.full((B.nrows,), float("nan"), dtype=torch.float64, device="cuda")
+        for _ in range(3):
+            pa.exec(torch.from_numpy(xa).cuda(), ya)
+            pb.exec(torch.from_numpy(xb).cuda(), yb)
+        torch.cuda.synchronize()
+        assert pa.info()["sell_ptile_frac"] > 0.9 and pb.info()["sell_ptile_frac"] > 0.9
+        assert np.array_equal(ya.cpu().numpy(), oracle.spmv(A, xa))
+        assert np.array_equal(yb.cpu().numpy(), oracle.spmv(B, xb))
