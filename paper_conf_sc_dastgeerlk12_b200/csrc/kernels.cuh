@@ -645,66 +645,19 @@ struct NoPatterns {};
 template <bool PAT, typename T>
 using SellPatternArg = std::conditional_t<PAT, SellPatterns<T>, NoPatterns>;
 
-// PAT: the plan has pattern chunks (phase A + genlist); PAT = false compiles
-// the general kernel without them (no extra registers, no 3 KB parameter).
-#ifndef PEPP_PAT_MINB
-#define PEPP_PAT_MINB 1   // experiments: minimum resident blocks per SM for the PAT (value-compressed) instances
-#endif
-template <int BLOCK, bool SORTED, bool PAT, typename T>
-__global__ void __launch_bounds__(BLOCK, (PAT && !SORTED) ? PEPP_PAT_MINB : 1) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
-                                                     const int* __restrict__ chunk_len,
-                                                     const int* __restrict__ rowlen,
-                                                     const int* __restrict__ perm,
-                                                     const int* __restrict__ col,
-                                                     const int16_t* __restrict__ col16,
-                                                     const int* __restrict__ soff,
-                                                     const __grid_constant__ SellPatternArg<PAT, T> pt,
-                                                     const T* __restrict__ val,
-                                                     const T* __restrict__ x,
-                                                     T* __restrict__ y,
-                                                     int cpw,
-                                                     const int* __restrict__ wstart,
-                                                     const int* __restrict__ patlist, int npatc,
-                                                     const int* __restrict__ genlist) {
-    const int lane = threadIdx.x & 31;
-    const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
-    const int nwarps = (gridDim.x * BLOCK) >> 5;
-    const uint64_t pol = evict_first_policy();
-    // Phase A (σ = 1 plans with pattern chunks): the pattern chunks, listed
-    // as (chunk << 5 | pattern id), in a tight loop — no descriptor, no
-    // per-lane loads: 1 list entry (prefetched one step ahead), the x
-    // gathers, the FMAs and the y store per chunk. Phase B below then walks
-    // only the other chunks (`genlist`, `nchunks` of them).
-    if constexpr (!SORTED && PAT) if (npatc > 0) {
-        // Runs of one pattern go through sell_pattern_run<N> (no per-chunk
-        // branch on the pattern length); a group of list entries that
-        // straddles two patterns (the list is sorted by id: at most one per
-        // pattern change per warp) takes the one-chunk path.
-        int e[kPatU];
-        int k0 = warp;
-        sell_pattern_ids(patlist, npatc, k0, nwarps, e);
-        while (k0 < npatc) {
-            const int pid = e[0] & 31;
-            switch (pt.len[pid]) {
-            case 1: k0 = sell_pattern_run<1, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            case 2: k0 = sell_pattern_run<2, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            case 3: k0 = sell_pattern_run<3, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            case 4: k0 = sell_pattern_run<4, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            case 5: k0 = sell_pattern_run<5, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            case 6: k0 = sell_pattern_run<6, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            case 7: k0 = sell_pattern_run<7, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            default: k0 = sell_pattern_run<8, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            }
-            if (k0 >= npatc) break;
-            for (int u = 0; u < kPatU; ++u) {   // the mixed group
-                if (e[u] < 0) continue;
-                const int r = (e[u] >> 5) * 32 + lane;
-                y[r] = sell_pattern_chunk<T>(pt, e[u] & 31, r, x);
-            }
-            k0 += kPatU * nwarps;
-            sell_pattern_ids(patlist, npatc, k0, nwarps, e);
-        }
-    }
+// Phase B of sell_kernel (and the grid-edge walk inside the tile kernel):
+// warp `warp` of `nwarps` walks its chunks (σ = 1: i = warp, + nwarps, ...
+// over `genlist` when PAT, else over all chunks; σ > 1: the plan-time range
+// wstart[warp] .. wstart[warp + 1] of the transposed window order).
+template <bool SORTED, bool PAT, typename T>
+__device__ __forceinline__ void sell_walk(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
+                                          const int* __restrict__ chunk_len, const int* __restrict__ rowlen,
+                                          const int* __restrict__ perm, const int* __restrict__ col,
+                                          const int16_t* __restrict__ col16, const int* __restrict__ soff,
+                                          const SellPatternArg<PAT, T>& pt, const T* __restrict__ val,
+                                          const T* __restrict__ x, T* __restrict__ y, int cpw,
+                                          const int* __restrict__ wstart, const int* __restrict__ genlist, int warp,
+                                          int nwarps, int lane, uint64_t pol) {
     const int nfull = SORTED ? (nchunks / cpw) * cpw : 0;
     const int nwin = SORTED ? nchunks / cpw : 1;
     auto chunk_of = [&](int i) -> int {
@@ -779,6 +732,70 @@ __global__ void __launch_bounds__(BLOCK, (PAT && !SORTED) ? PEPP_PAT_MINB : 1) s
         if (c * 32 + lane < nrows) y[l0.orow] = acc;
         q0 = q1; q1 = q2; l0 = l1;
     }
+}
+
+// PAT: the plan has pattern chunks (phase A + genlist); PAT = false compiles
+// the general kernel without them (no extra registers, no 3 KB parameter).
+#ifndef PEPP_PAT_MINB
+#define PEPP_PAT_MINB 1   // experiments: minimum resident blocks per SM for the PAT (value-compressed) instances
+#endif
+template <int BLOCK, bool SORTED, bool PAT, typename T>
+__global__ void __launch_bounds__(BLOCK, (PAT && !SORTED) ? PEPP_PAT_MINB : 1) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
+                                                     const int* __restrict__ chunk_len,
+                                                     const int* __restrict__ rowlen,
+                                                     const int* __restrict__ perm,
+                                                     const int* __restrict__ col,
+                                                     const int16_t* __restrict__ col16,
+                                                     const int* __restrict__ soff,
+                                                     const __grid_constant__ SellPatternArg<PAT, T> pt,
+                                                     const T* __restrict__ val,
+                                                     const T* __restrict__ x,
+                                                     T* __restrict__ y,
+                                                     int cpw,
+                                                     const int* __restrict__ wstart,
+                                                     const int* __restrict__ patlist, int npatc,
+                                                     const int* __restrict__ genlist) {
+    const int lane = threadIdx.x & 31;
+    const int warp = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
+    const int nwarps = (gridDim.x * BLOCK) >> 5;
+    const uint64_t pol = evict_first_policy();
+    // Phase A (σ = 1 plans with pattern chunks): the pattern chunks, listed
+    // as (chunk << 5 | pattern id), in a tight loop — no descriptor, no
+    // per-lane loads: 1 list entry (prefetched one step ahead), the x
+    // gathers, the FMAs and the y store per chunk. Phase B below then walks
+    // only the other chunks (`genlist`, `nchunks` of them).
+    if constexpr (!SORTED && PAT) if (npatc > 0) {
+        // Runs of one pattern go through sell_pattern_run<N> (no per-chunk
+        // branch on the pattern length); a group of list entries that
+        // straddles two patterns (the list is sorted by id: at most one per
+        // pattern change per warp) takes the one-chunk path.
+        int e[kPatU];
+        int k0 = warp;
+        sell_pattern_ids(patlist, npatc, k0, nwarps, e);
+        while (k0 < npatc) {
+            const int pid = e[0] & 31;
+            switch (pt.len[pid]) {
+            case 1: k0 = sell_pattern_run<1, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 2: k0 = sell_pattern_run<2, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 3: k0 = sell_pattern_run<3, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 4: k0 = sell_pattern_run<4, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 5: k0 = sell_pattern_run<5, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 6: k0 = sell_pattern_run<6, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 7: k0 = sell_pattern_run<7, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            default: k0 = sell_pattern_run<8, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            }
+            if (k0 >= npatc) break;
+            for (int u = 0; u < kPatU; ++u) {   // the mixed group
+                if (e[u] < 0) continue;
+                const int r = (e[u] >> 5) * 32 + lane;
+                y[r] = sell_pattern_chunk<T>(pt, e[u] & 31, r, x);
+            }
+            k0 += kPatU * nwarps;
+            sell_pattern_ids(patlist, npatc, k0, nwarps, e);
+        }
+    }
+    sell_walk<SORTED, PAT, T>(nrows, nchunks, chunk_ptr, chunk_len, rowlen, perm, col, col16, soff, pt, val, x, y, cpw,
+                              wstart, genlist, warp, nwarps, lane, pol);
 }
 
 // =====================================================================
@@ -1219,16 +1236,31 @@ __device__ __forceinline__ void tile_rows(const SellPatterns<T>& pt, const int* 
 // issue of every tile on one serial path).
 // Shared memory: S x stage (x ranges; VALS: then the value block at
 // vstage) | S full | S empty | S entries.
-template <int BLOCK, int S, bool VALS, typename T>
+// The chunks outside the tiles (grid edges: `genlist`), walked by the tile
+// kernel's last NWK warps with the general SELL walk (sell_walk) while the
+// producer / consumers run the tiles — beside the tiles on every SM instead
+// of a second kernel on a second stream (which added 16-20 µs per call).
+struct TileWalk {
+    int nrows = 0, ngen = 0;
+    const int64_t* chunk_ptr = nullptr;
+    const int* chunk_len = nullptr;
+    const int* rowlen = nullptr;
+    const int* col = nullptr;
+    const int16_t* col16 = nullptr;
+    const int* soff = nullptr;
+    const int* genlist = nullptr;
+};
+
+template <int BLOCK, int S, bool VALS, typename T, int NWK>
 __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_constant__ SellPatterns<T> pt,
                                                              const __grid_constant__ PatTiles tt,
                                                              const int4* __restrict__ tiles, int ntiles,
                                                              int stage_elems, int vstage,
                                                              const T* __restrict__ val, const T* __restrict__ x,
-                                                             T* __restrict__ y, int64_t xlen) {
+                                                             T* __restrict__ y, int64_t xlen, const TileWalk wk) {
     extern __shared__ __align__(128) unsigned char ptile_smem[];
     constexpr int A = 16 / sizeof(T);
-    constexpr int NCW = BLOCK / 32 - 1, NC = NCW * 32;
+    constexpr int NCW = BLOCK / 32 - 1 - NWK, NC = NCW * 32;
     T* sx = reinterpret_cast<T*>(ptile_smem);
     uint64_t* full = reinterpret_cast<uint64_t*>(sx + (size_t)S * stage_elems);
     uint64_t* empty = full + S;
@@ -1240,6 +1272,13 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
+    if (warp > NCW) {   // the walkers: the chunks outside the tiles
+        if (wk.ngen > 0)
+            sell_walk<false, true, T>(wk.nrows, wk.ngen, wk.chunk_ptr, wk.chunk_len, wk.rowlen, nullptr, wk.col, wk.col16,
+                                      wk.soff, pt, val, x, y, 1, nullptr, wk.genlist, blockIdx.x * NWK + (warp - NCW - 1),
+                                      gridDim.x * NWK, lane, evict_first_policy());
+        return;
+    }
     if (warp == 0) {
         if (lane != 0) return;
         int4 e = blockIdx.x < ntiles ? __ldg(tiles + blockIdx.x) : make_int4(0, 0, 0, 0);
@@ -1290,7 +1329,7 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
         }
         return;
     }
-    const int c = tid - 32;
+    const int c = tid - 32;   // consumer index (warps 1 .. NCW)
     for (int it = 0;; ++it) {
         const int t = blockIdx.x + it * G;
         if (t >= ntiles) break;

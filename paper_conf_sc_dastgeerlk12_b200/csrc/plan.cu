@@ -507,8 +507,23 @@ int tile_side_grid(const pepp_spmv_plan_t* p, int grid) {
     return std::max(1, std::min(grid, PEPP_TILE_SIDE_BPS * std::max(1, p->sm_count - p->reserve_sms)));
 }
 
+// warps per tile CTA walking the grid-edge chunks (0: a second kernel on the
+// side stream); config 4 µs, one box, walkers 0 / 2 / 4 — values streamed
+// fp64 571.6 / 556.3 / 557.6, fp32 291.5 / 275.6 / 276.5; pattern tiles fp64
+// 187.6 / 196.3 / 172.7, fp32 116.3 / 140.4 / 99.8 (with few walkers the walk
+// outlasts the short pattern-tile kernel); pattern-tile walkers 4 / 6 / 8:
+// fp64 172.4 / 173.9 / 176.7 µs, 4096² 57.3 / 52.4 / 52.6 µs
+#ifndef PEPP_TILE_WALKERS_S
+#define PEPP_TILE_WALKERS_S 4   // stencil tiles (values streamed)
+#endif
+#ifndef PEPP_TILE_WALKERS_P
+#define PEPP_TILE_WALKERS_P 6   // pattern tiles
+#endif
+template <bool VALS> constexpr int tile_walkers() { return VALS ? PEPP_TILE_WALKERS_S : PEPP_TILE_WALKERS_P; }
+template <bool VALS> constexpr int tile_block() { return kPtileBlock + 32 * tile_walkers<VALS>(); }
+
 template <int S, bool VALS, typename T>
-const void* tile_kernel_fn() { return (const void*)pepp::k::sell_tile_kernel<kPtileBlock, S, VALS, T>; }
+const void* tile_kernel_fn() { return (const void*)pepp::k::sell_tile_kernel<tile_block<VALS>(), S, VALS, T, tile_walkers<VALS>()>; }
 
 // ents[i] = {chunk, set id, value block / 32, -}; sorted by set id then chunk.
 // Fills *L and appends the indices of untiled entries to *rest.
@@ -729,7 +744,7 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
     L->tt = tt;
     L->smem = smem;
     int occ = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kPtileBlock, L->smem) != cudaSuccess || occ < 1) occ = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, vals ? tile_block<true>() : tile_block<false>(), L->smem) != cudaSuccess || occ < 1) occ = 1;
     (void)cudaGetLastError();
     L->grid = (int)std::max<int64_t>(1, std::min<int64_t>(L->ntiles, (int64_t)std::max(1, p->sm_count - p->reserve_sms) * occ));
     return PEPP_OK;
@@ -1474,6 +1489,41 @@ template <typename T> const pepp::k::SellPatterns<T>& sell_pattern_table(const p
 template <> const pepp::k::SellPatterns<double>& sell_pattern_table<double>(const pepp_spmv_plan_t* p) { return p->pat64; }
 template <> const pepp::k::SellPatterns<float>& sell_pattern_table<float>(const pepp_spmv_plan_t* p) { return p->pat32; }
 
+// the side stream of a tile call: forked after the work already on st
+pepp_status_t side_fork(pepp_spmv_plan_t* p, cudaStream_t st, cudaStream_t* gs) {
+    *gs = p->gside && PEPP_EXP_TILE_SIDE == 0 ? p->gside : st;
+    if (*gs != st && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess || cudaStreamWaitEvent(*gs, p->ev_gfork, 0) != cudaSuccess))
+        return PEPP_E_CUDA;
+    return PEPP_OK;
+}
+pepp_status_t side_join(pepp_spmv_plan_t* p, cudaStream_t st) {
+    if (p->gside && PEPP_EXP_TILE_SIDE == 0 &&
+        (cudaEventRecord(p->ev_gjoin, p->gside) != cudaSuccess || cudaStreamWaitEvent(st, p->ev_gjoin, 0) != cudaSuccess))
+        return PEPP_E_CUDA;
+    return PEPP_OK;
+}
+
+// one tile-kernel launch; with `walk`, its walker warps take the genlist
+template <bool VALS, typename T>
+pepp_status_t tile_launch(pepp_spmv_plan_t* p, const TileLayout& L, bool walk, const T* x, T* y, cudaStream_t st) {
+    pepp::k::TileWalk wk;
+    if (walk && p->ngen > 0 && PEPP_EXP_TILE_SIDE != 2) {
+        wk.nrows = (int)p->nrows;
+        wk.ngen = p->ngen;
+        wk.chunk_ptr = p->d_chunk_ptr;
+        wk.chunk_len = p->d_chunk_len;
+        wk.rowlen = p->d_rowlen;
+        wk.col = p->d_scol;
+        wk.col16 = p->d_scol16;
+        wk.soff = p->d_soff;
+        wk.genlist = p->d_genlist;
+    }
+    pepp::k::sell_tile_kernel<tile_block<VALS>(), VALS ? kStileS : kPtileS, VALS, T, tile_walkers<VALS>()>
+        <<<L.grid, tile_block<VALS>(), L.smem, st>>>(sell_pattern_table<T>(p), L.tt, L.d_tiles, L.ntiles, L.stage, L.vstage,
+                                             (const T*)p->d_sval, x, y, p->ncols, wk);
+    return PEPP_OK;
+}
+
 template <typename T>
 pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y, cudaStream_t st) {
     if (p->nrows == 0) return PEPP_OK;
@@ -1535,55 +1585,51 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
                 p->d_scol16, p->d_soff, pepp::k::NoPatterns{}, (const T*)p->d_sval, x, y, p->sell_cpw, p->d_sell_ws,
                 nullptr, 0, nullptr);
         else if (p->d_patlist && p->ptl.ntiles && ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0) {
-            // pattern tiles (bulk-copied x ranges) on st; the grid-edge chunks
-            // and the untiled pattern chunks through the genlist walk beside it
-            cudaStream_t gs = p->gside && PEPP_EXP_TILE_SIDE == 0 ? p->gside : st;
-            const bool side = p->ngen + p->npatrest > 0 && PEPP_EXP_TILE_SIDE != 2;
-            if (side && p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
-                                     cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
-                return PEPP_E_CUDA;
-            pepp::k::sell_tile_kernel<kPtileBlock, kPtileS, false, T><<<p->ptl.grid, kPtileBlock, p->ptl.smem, st>>>(
-                sell_pattern_table<T>(p), p->ptl.tt, p->ptl.d_tiles, p->ptl.ntiles, p->ptl.stage, 0, nullptr, x, y, p->ncols);
-            if (side)
+            // pattern tiles (bulk-copied x ranges); the grid-edge chunks by the
+            // tile kernel's walker warps, or — with untiled pattern chunks
+            // left (phase A) or no walkers — by the genlist walk beside it
+            const bool inwalk = tile_walkers<false>() > 0 && p->npatrest == 0;
+            pepp_status_t s2 = tile_launch<false, T>(p, p->ptl, inwalk, x, y, st);
+            if (s2) return s2;
+            if (!inwalk && p->ngen + p->npatrest > 0) {
+                cudaStream_t gs;
+                if ((s2 = side_fork(p, st, &gs))) return s2;
                 pepp::k::sell_kernel<kBlock, false, true, T><<<tile_side_grid(p, p->grid_sell), kBlock, 0, gs>>>(
                     (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                     p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
                     p->d_patrest, p->npatrest, p->d_genlist);
-            if (side && p->gside && (cudaEventRecord(p->ev_gjoin, p->gside) != cudaSuccess ||
-                                     cudaStreamWaitEvent(st, p->ev_gjoin, 0) != cudaSuccess))
-                return PEPP_E_CUDA;
+                if ((s2 = side_join(p, st))) return s2;
+            }
         } else if (p->d_patlist)   // pattern chunks (value compression): phase A + the rest through genlist
             pepp::k::sell_kernel<kBlock, false, true, T><<<p->grid_sell, kBlock, 0, st>>>(
                 (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
                 p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
                 p->d_patlist, p->npatc, p->d_genlist);
         else if (p->d_stlist && p->stl.ntiles && ((((uintptr_t)x) | ((uintptr_t)y)) & 15) == 0) {
-            // stencil tiles (bulk-copied x ranges and values) on st; the grid-edge
-            // chunks and the untiled list entries beside it on the side stream
-            cudaStream_t gs = p->gside && PEPP_EXP_TILE_SIDE == 0 ? p->gside : st;
-            const bool side = p->ngen + p->nstrest > 0 && PEPP_EXP_TILE_SIDE != 2;
-            if (side && p->gside && (cudaEventRecord(p->ev_gfork, st) != cudaSuccess ||
-                                     cudaStreamWaitEvent(p->gside, p->ev_gfork, 0) != cudaSuccess))
-                return PEPP_E_CUDA;
-            pepp::k::sell_tile_kernel<kPtileBlock, kStileS, true, T><<<p->stl.grid, kPtileBlock, p->stl.smem, st>>>(
-                sell_pattern_table<T>(p), p->stl.tt, p->stl.d_tiles, p->stl.ntiles, p->stl.stage, p->stl.vstage,
-                (const T*)p->d_sval, x, y, p->ncols);
-            if (p->nstrest) {
-                if (p->slist_long)
-                    pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T, 16>(), 16, T><<<tile_side_grid(p, p->grid_slist), kBlock, 0, gs>>>(
-                        p->d_strest, p->nstrest, p->stab, (const T*)p->d_sval, x, y);
-                else
-                    pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), 8, T><<<tile_side_grid(p, p->grid_slist), kBlock, 0, gs>>>(
-                        p->d_strest, p->nstrest, p->stab, (const T*)p->d_sval, x, y);
+            // stencil tiles (bulk-copied x ranges and values); the grid-edge
+            // chunks by the walker warps; untiled list entries (and, without
+            // walkers, the grid-edge chunks) beside it on the side stream
+            const bool inwalk = tile_walkers<true>() > 0;
+            pepp_status_t s2 = tile_launch<true, T>(p, p->stl, inwalk, x, y, st);
+            if (s2) return s2;
+            if (p->nstrest || (!inwalk && p->ngen > 0)) {
+                cudaStream_t gs;
+                if ((s2 = side_fork(p, st, &gs))) return s2;
+                if (p->nstrest) {
+                    if (p->slist_long)
+                        pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T, 16>(), 16, T><<<tile_side_grid(p, p->grid_slist), kBlock, 0, gs>>>(
+                            p->d_strest, p->nstrest, p->stab, (const T*)p->d_sval, x, y);
+                    else
+                        pepp::k::sell_slist_kernel<kBlock, pepp::k::sell_slist_u<T>(), 8, T><<<tile_side_grid(p, p->grid_slist), kBlock, 0, gs>>>(
+                            p->d_strest, p->nstrest, p->stab, (const T*)p->d_sval, x, y);
+                }
+                if (!inwalk && p->ngen > 0)
+                    pepp::k::sell_kernel<kBlock, false, true, T><<<tile_side_grid(p, p->grid_sell), kBlock, 0, gs>>>(
+                        (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
+                        p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
+                        nullptr, 0, p->d_genlist);
+                if ((s2 = side_join(p, st))) return s2;
             }
-            if (p->ngen > 0)
-                pepp::k::sell_kernel<kBlock, false, true, T><<<tile_side_grid(p, p->grid_sell), kBlock, 0, gs>>>(
-                    (int)p->nrows, p->ngen, p->d_chunk_ptr, p->d_chunk_len, p->d_rowlen, nullptr,
-                    p->d_scol, p->d_scol16, p->d_soff, sell_pattern_table<T>(p), (const T*)p->d_sval, x, y, 1, nullptr,
-                    nullptr, 0, p->d_genlist);
-            if (side && p->gside && (cudaEventRecord(p->ev_gjoin, p->gside) != cudaSuccess ||
-                                     cudaStreamWaitEvent(st, p->ev_gjoin, 0) != cudaSuccess))
-                return PEPP_E_CUDA;
         } else if (p->d_stlist) {   // stencil list (values streamed) and the other chunks (disjoint rows)
             // the small, latency-bound genlist walk runs beside the list kernel
             // on the plan's second stream when it has one (kSlistConcurrent)
@@ -1648,8 +1694,11 @@ int launches_for(const pepp_spmv_plan_t* p, const Candidate& c, const void* x, c
         return p->ntiles > 0 ? 2 + (p->nlongruns > 0) : 0;
     case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
     case PEPP_V_SELL:
-        return (p->d_stlist ? (p->stl.ntiles && al ? 1 + (p->nstrest > 0) : 1) + (p->ngen > 0)
-                            : (p->d_patlist && p->ptl.ntiles && al) ? 1 + (p->ngen + p->npatrest > 0) : 1) +
+        return (p->d_stlist ? (p->stl.ntiles && al ? 1 + (p->nstrest > 0) + (tile_walkers<true>() == 0 && p->ngen > 0)
+                                                   : 1 + (p->ngen > 0))
+                            : (p->d_patlist && p->ptl.ntiles && al)
+                                  ? 1 + ((tile_walkers<false>() == 0 || p->npatrest > 0) && p->ngen + p->npatrest > 0)
+                                  : 1) +
                (p->nsell_mid > 0) + (p->nsell_seg > 0);
     case PEPP_V_PANEL:
         for (const auto& pl : p->panels)
