@@ -103,18 +103,26 @@ def test_fp32_differs_from_fp64_where_float_rounds():
 
 
 def test_fp32_stencil_list_large_bitwise():
-    """The fp32 stencil-list path at a size spanning many warps and the
+    """The fp32 stencil path at a size spanning many warps and the
     straddling groups between offset sets (a 1024² Laplacian has 3 stencil
-    offset sets plus the general boundary chunks): integer inputs bit-exact,
-    launches = stencil-list kernel + genlist walk."""
+    offset sets plus the general boundary chunks): integer inputs bit-exact;
+    one launch (the tile kernel, its walker warps taking the boundary chunks)
+    — two (stencil-list kernel + genlist walk) when x / y are not 16-byte
+    aligned."""
     A = gen.laplacian2d(1024)
     A32 = _f32(A)
     x32 = gen.vector(7, gen.INT8, A.ncols).astype(np.float32)
     ref = oracle.spmv(A32, x32)
     with pepp.Plan.from_csr(A32, variant_mask=1 << pepp.V_SELL, compress_values=False) as plan:
         y, used = _run(plan, x32)
-        assert used.launches == 2
+        assert used.launches == 1
         assert np.array_equal(y, ref)
+        xo = torch.zeros(A.ncols + 1, dtype=torch.float32, device="cuda")
+        xo[1:] = torch.from_numpy(x32).cuda()
+        yo = torch.full((A.nrows + 1,), float("nan"), dtype=torch.float32, device="cuda")
+        u = plan.exec(xo[1:], yo[1:])
+        torch.cuda.synchronize()
+        assert u.launches == 2 and np.array_equal(yo[1:].cpu().numpy(), ref)
         # the same path captured in a CUDA graph (the genlist walk's fork /
         # join onto the plan's second stream becomes a graph branch)
         xd = torch.from_numpy(x32).cuda()
