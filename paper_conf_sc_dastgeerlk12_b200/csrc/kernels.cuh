@@ -305,6 +305,9 @@ __device__ __forceinline__ void sell_pair_len(int n, const T* __restrict__ val, 
 #ifndef PEPP_SELL_PAIR_F32
 #define PEPP_SELL_PAIR_F32 0   // fp32 420 -> 436 us: off
 #endif
+#ifndef PEPP_SELL_PAIR_SORTED
+#define PEPP_SELL_PAIR_SORTED 0   // pair equal chunks in σ > 1 walks: config 3 358 -> 373 us, skew 249 -> 268 us (84 vs fewer registers): off
+#endif
 template <typename T>
 constexpr bool sell_pairs() { return std::is_same<T, float>::value ? PEPP_SELL_PAIR_F32 : PEPP_SELL_PAIR_F64; }
 
@@ -693,11 +696,13 @@ __device__ __forceinline__ void sell_walk(int nrows, int nchunks, const int64_t*
     for (; i < end; i += step) {
         const Desc q2 = desc(i + 2 * step);
         const Lane l1 = lanes(i + step, q1);
-        if constexpr (sell_pairs<T>() && !SORTED && !PAT) {
+        if constexpr ((sell_pairs<T>() && !SORTED && !PAT) || (PEPP_SELL_PAIR_SORTED && SORTED && !PAT)) {
             // chunks i and i+1 both unmasked stencil chunks of one length <= 8:
-            // both at once, then the pipeline moves two chunks on
+            // both at once, then the pipeline moves two chunks on (σ > 1: the
+            // transposed window order puts chunks of equal length next to each
+            // other, any index format)
             const int pl = q0.d & kSellLenMask;
-            const bool fmt_ok = (q0.d & kSellStencil) || PEPP_SELL_PAIR_ALL;
+            const bool fmt_ok = (q0.d & kSellStencil) || PEPP_SELL_PAIR_ALL || SORTED;
             if (q1.d == q0.d && fmt_ok && !(q0.d & kSellMasked) && pl >= 1 && pl <= 8 && i + step < end) {
                 const int ra = l0.orow, rb = l1.orow;
                 T a = T(0), b = T(0);
