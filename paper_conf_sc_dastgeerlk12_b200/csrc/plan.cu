@@ -19,6 +19,8 @@
 
 #include <algorithm>
 #include <map>
+#include <mutex>
+#include <thread>
 #include <tuple>
 #include <chrono>
 #include <cmath>
@@ -356,6 +358,91 @@ struct DevTmp {
     cudaError_t alloc(size_t n) { return cudaMalloc((void**)&p, sizeof(T) * (n ? n : 1)); }
     T* release() { T* r = p; p = nullptr; return r; }
 };
+
+// Host -> device upload of a large pageable operand (the matrix at plan
+// time). A plain cudaMemcpy from pageable memory runs at ~10 GB/s on the
+// GPU boxes (the driver stages it through one pinned buffer with one CPU
+// thread); registering the caller's pages costs more than it saves (4 GB:
+// 0.85 s + 0.18 s to unregister against 0.39 s; tools/r2/h2d_probe.py).
+// Here kStageThreads host threads each copy their own chunks into their own
+// pair of pinned buffers (process-wide, allocated once) and issue the DMA on
+// their own stream; `st` then waits for every worker stream. Small, device
+// and already-pinned operands go straight through cudaMemcpyAsync.
+constexpr size_t kStageChunk = 16u << 20, kStageMin = 64u << 20;
+constexpr int kStageThreads = 8;
+struct StagePool {
+    std::mutex mu;
+    std::vector<void*> buf;   // kStageThreads x 2 pinned chunks (never freed: process lifetime)
+};
+StagePool& stage_pool() {
+    static StagePool* sp = new StagePool;
+    return *sp;
+}
+
+pepp_status_t upload(void* dst, const void* src, size_t bytes, cudaMemcpyKind kind, cudaStream_t st) {
+    if (!bytes) return PEPP_OK;
+    cudaPointerAttributes at{};
+    const bool pageable = kind == cudaMemcpyHostToDevice && cudaPointerGetAttributes(&at, src) == cudaSuccess &&
+                          at.type == cudaMemoryTypeUnregistered;
+    (void)cudaGetLastError();
+    if (!pageable || bytes < kStageMin) return cudaMemcpyAsync(dst, src, bytes, kind, st) == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
+    StagePool& sp = stage_pool();
+    std::lock_guard<std::mutex> lock(sp.mu);   // one staged upload at a time per process
+    if (sp.buf.empty()) {
+        for (int i = 0; i < 2 * kStageThreads; ++i) {
+            void* b = nullptr;
+            if (cudaHostAlloc(&b, kStageChunk, cudaHostAllocDefault) != cudaSuccess) {
+                (void)cudaGetLastError();
+                for (void* q : sp.buf) cudaFreeHost(q);
+                sp.buf.clear();
+                return cudaMemcpyAsync(dst, src, bytes, kind, st) == cudaSuccess ? PEPP_OK : PEPP_E_CUDA;
+            }
+            sp.buf.push_back(b);
+        }
+    }
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return PEPP_E_CUDA;
+    // the worker streams start after the work already queued on st (the
+    // destination's memset)
+    cudaEvent_t ev_start = nullptr;
+    if (cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventRecord(ev_start, st) != cudaSuccess)
+        return PEPP_E_CUDA;
+    const size_t nchunks = (bytes + kStageChunk - 1) / kStageChunk;
+    std::vector<int> fail(kStageThreads, 0);
+    std::vector<cudaStream_t> ws(kStageThreads, nullptr);
+    auto work = [&](int w) {
+        if (cudaSetDevice(dev) != cudaSuccess || cudaStreamCreateWithFlags(&ws[w], cudaStreamNonBlocking) != cudaSuccess ||
+            cudaStreamWaitEvent(ws[w], ev_start, 0) != cudaSuccess) { fail[w] = 1; return; }
+        cudaEvent_t ev[2] = {nullptr, nullptr};
+        for (auto& e : ev)
+            if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { fail[w] = 1; return; }
+        int k = 0;
+        for (size_t c = (size_t)w; c < nchunks && !fail[w]; c += kStageThreads, ++k) {
+            const int b = k & 1;
+            if (k >= 2 && cudaEventSynchronize(ev[b]) != cudaSuccess) { fail[w] = 1; break; }   // buffer b free again
+            const size_t off = c * kStageChunk, n = std::min(kStageChunk, bytes - off);
+            void* pin = sp.buf[2 * w + b];
+            std::memcpy(pin, (const char*)src + off, n);
+            if (cudaMemcpyAsync((char*)dst + off, pin, n, cudaMemcpyHostToDevice, ws[w]) != cudaSuccess ||
+                cudaEventRecord(ev[b], ws[w]) != cudaSuccess) fail[w] = 1;
+        }
+        // the pinned buffers are reused by the next upload: wait for this one's DMAs
+        if (cudaStreamSynchronize(ws[w]) != cudaSuccess) fail[w] = 1;
+        for (auto& e : ev) if (e) cudaEventDestroy(e);
+    };
+    std::vector<std::thread> th;
+    for (int w = 0; w < kStageThreads; ++w) th.emplace_back(work, w);
+    for (auto& t : th) t.join();
+    bool bad = false;
+    for (int w = 0; w < kStageThreads; ++w) {
+        bad |= fail[w] != 0;
+        if (ws[w]) cudaStreamDestroy(ws[w]);
+    }
+    cudaEventDestroy(ev_start);
+    if (bad) { (void)cudaGetLastError(); return PEPP_E_CUDA; }
+    return PEPP_OK;
+}
 
 template <typename T>
 pepp_status_t dalloc(pepp_spmv_plan_t* p, T** ptr, int64_t n) {
@@ -2708,8 +2795,8 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     PEPP_CUDA_TRY(cudaMemsetAsync(p->d_val, 0, p->esz * nstore, st));
     const cudaMemcpyKind kind = A->on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
     if (A->nnz) {
-        PEPP_CUDA_TRY(cudaMemcpyAsync(p->d_col + p->pad, A->col_idx, sizeof(int) * A->nnz, kind, st));
-        PEPP_CUDA_TRY(cudaMemcpyAsync((char*)p->d_val + p->pad * p->esz, A->values, p->esz * A->nnz, kind, st));
+        if ((s = upload(p->d_col + p->pad, A->col_idx, sizeof(int) * A->nnz, kind, st))) return s;
+        if ((s = upload((char*)p->d_val + p->pad * p->esz, A->values, p->esz * A->nnz, kind, st))) return s;
     }
     DevTmp<int64_t> rp64;
     DevTmp<pepp::k::RowStats> stats;
@@ -2718,7 +2805,7 @@ pepp_status_t plan_impl(const pepp_csr_t* A, const pepp_spmv_opts_t* o, pepp_spm
     int64_t* d_rp64 = rp64.p;
     pepp::k::RowStats* d_stats = stats.p;
     PEPP_CUDA_TRY(cudaMemsetAsync(d_stats, 0, sizeof(pepp::k::RowStats), st));
-    PEPP_CUDA_TRY(cudaMemcpyAsync(d_rp64, A->row_ptr, sizeof(int64_t) * (A->nrows + 1), kind, st));
+    if ((s = upload(d_rp64, A->row_ptr, sizeof(int64_t) * (A->nrows + 1), kind, st))) return s;
     {
         const int tb = 256;
         const int gb = (int)std::min<int64_t>((A->nrows + 1 + tb - 1) / tb, (int64_t)p->sm_count * 8);
