@@ -1346,7 +1346,10 @@ pepp_status_t sell_stencil_list(pepp_spmv_plan_t* p) {
 // a stable radix sort of the entries by panel (CSR order kept within a
 // panel), the (row, panel) pairs by head flags (cub select), their pair
 // ranges per panel by binary search.
-constexpr int64_t kPanelMinX = 96ll << 20;
+#ifndef PEPP_PANEL_MIN_MB
+#define PEPP_PANEL_MIN_MB 96   // checked below it (tools/r2/panel_mid.py, threshold 24 MB): uniform 16/row at 6e6 / 1e7 / 1.2e7 rows
+#endif                         // panel[22] 862 / 1347 / 1536 us vs sell[1] 413 / 860 / 1450 us
+constexpr int64_t kPanelMinX = (int64_t)PEPP_PANEL_MIN_MB << 20;
 
 pepp_status_t prepare_panels(pepp_spmv_plan_t* p, cudaStream_t st, std::vector<int>* lgs) {
     lgs->clear();
