@@ -63,7 +63,7 @@
 extern "C" {
 #endif
 
-#define PEPP_ABI_VERSION 9
+#define PEPP_ABI_VERSION 10
 
 typedef enum {
     PEPP_OK = 0,
@@ -288,6 +288,8 @@ typedef struct pepp_plan_info_s {
                                  (pattern chunks with compress_values, else stencil-list chunks whose
                                  values stream) computed from x ranges and values bulk-copied into
                                  shared memory (sell_tile_kernel) when x and y are 16-byte aligned */
+    int64_t sell_tile_multiline; /* multi-line pattern tiles (grid stencils: K tiles D rows apart
+                                 loading their K + W x lines once each; 0 = none) */
 } pepp_plan_info_t;
 
 typedef struct pepp_spmv_plan_s pepp_spmv_plan_t;  /* opaque plan (C forbids a typedef and a function sharing the name pepp_spmv_plan) */

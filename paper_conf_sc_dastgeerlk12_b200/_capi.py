@@ -43,7 +43,8 @@ class INFO_T(ctypes.Structure):
                 ("sell_constval_frac", c_f64), ("p2p_buffers", c_i32),
                 ("sell_long_rows", c_i64), ("sell_cap", c_i64), ("dist_candidates", c_i32),
                 ("dist_nparts", c_i32), ("dist_exchange", c_i32), ("dist_repl_nparts", c_i32),
-                ("dist_probe_ms", c_f64), ("sell_ptile_frac", c_f64)]
+                ("dist_probe_ms", c_f64), ("sell_ptile_frac", c_f64),
+                ("sell_tile_multiline", c_i64)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -136,7 +137,7 @@ class PeppError(RuntimeError):
         super().__init__(f"{where}: {status_str(status)} ({status})" + (f": {detail}" if detail else ""))
 
 
-ABI_VERSION = 9   # PEPP_ABI_VERSION of include/pepp_spmv.h
+ABI_VERSION = 10   # PEPP_ABI_VERSION of include/pepp_spmv.h
 
 
 def lib() -> ctypes.CDLL:

@@ -1229,6 +1229,7 @@ pepp_status_t prepare_sell(pepp_spmv_plan_t* p, cudaStream_t st) {
     p->info.sell_stencil_frac = p->nchunks ? (double)p->sell_stencil_chunks / (double)p->nchunks : 0.0;
     p->info.sell_constval_frac = p->nchunks ? (double)p->sell_const_chunks / (double)p->nchunks : 0.0;
     p->info.sell_ptile_frac = p->nchunks ? (double)(p->ptl.chunks + p->stl.chunks) / (double)p->nchunks : 0.0;
+    p->info.sell_tile_multiline = p->ptl.lines;
     p->info.sell_fill = fill;
     p->info.sell_long_rows = p->nsell_long + p->nsell_mid;
     p->info.sell_cap = p->sell_cap == INT32_MAX ? 0 : p->sell_cap;

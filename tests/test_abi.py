@@ -47,7 +47,7 @@ def test_library_exports_every_declared_symbol():
 def test_abi_version_and_status_strings():
     from paper_conf_sc_dastgeerlk12_b200 import _capi
     L = _capi.lib()
-    assert L.pepp_abi_version() == _capi.ABI_VERSION == 9
+    assert L.pepp_abi_version() == _capi.ABI_VERSION == 10
     for s in [0, -1, -2, -3, -4, -5, -6]:
         assert L.pepp_status_str(s).decode().startswith("PEPP_")
 

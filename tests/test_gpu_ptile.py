@@ -149,3 +149,31 @@ def test_tile_plans_with_different_stage_sizes_interleave():
         assert pa.info()["sell_ptile_frac"] > 0.9 and pb.info()["sell_ptile_frac"] > 0.9
         assert np.array_equal(ya.cpu().numpy(), oracle.spmv(A, xa))
         assert np.array_equal(yb.cpu().numpy(), oracle.spmv(B, xb))
+
+
+@pytest.mark.parametrize("name", ["lap2d", "nine_point", "lap3d"])
+def test_multiline_pattern_tiles(name):
+    """Grid stencils whose rows align with the chunks (grid line a multiple
+    of 32) become multi-line pattern tiles — 5-point (W = 2), a 3x3 stencil
+    minus a corner (8 slots, the pattern-table limit; clusters of 3, 3 and 2
+    offsets), the 3-D 7-point (D = n², ±n inside the line): the plan
+    reports them, and y is bit-identical to the streamed layout and to the
+    oracle."""
+    if name == "lap2d":
+        A = gen.laplacian2d(512)
+    elif name == "nine_point":
+        offs = [(a, b) for a in (-1, 0, 1) for b in (-1, 0, 1) if (a, b) != (1, 1)]
+        A = _stencil_grid(512, offs, 8.0, -1.0)
+    else:
+        offs = [(0, 0, 0), (-1, 0, 0), (1, 0, 0), (0, -1, 0), (0, 1, 0), (0, 0, -1), (0, 0, 1)]
+        A = _stencil_grid(96, offs, 6.0, -1.0, dims=3)   # x-lines of 3 chunks: the middle one is interior
+    x = gen.vector(3, gen.INT8, A.ncols)
+    y1, i1 = _y(A, x, True)
+    y0, _ = _y(A, x, False)
+    assert i1["sell_tile_multiline"] > 0, i1
+    assert np.array_equal(_bits(y1), _bits(y0))
+    _check(A, x, y1, True)
+    xr = gen.vector(4, gen.REAL, A.ncols)
+    y1, _ = _y(A, xr, True)
+    y2, _ = _y(A, xr, True, shift=1)   # register path
+    assert np.array_equal(_bits(y1), _bits(y2))
