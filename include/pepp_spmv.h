@@ -311,7 +311,10 @@ const char* pepp_status_str(pepp_status_t s);
 void pepp_spmv_opts_default(pepp_spmv_opts_t* opts);
 
 /* Build a plan for A on opts->device. Copies A; the plan owns all device
-   memory it allocates. Collective over ranks when opts->nranks > 1 (every
+   memory it allocates. Host arrays of A are only read during the call;
+   pageable ones of 64 MB or more are staged through a process-wide pool of
+   pinned buffers (16 x 16 MB, allocated on first use and kept for the
+   process) by 8 host threads. Collective over ranks when opts->nranks > 1 (every
    rank must call it with its own row block). On error *out is NULL.
    Errors: PEPP_E_INVALID (NULL args, broken CSR invariants, bad options),
    PEPP_E_CUDA (no device / CUDA failure), PEPP_E_NOMEM, PEPP_E_NCCL,
