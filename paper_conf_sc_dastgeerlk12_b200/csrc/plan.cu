@@ -709,6 +709,12 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
     auto mpart = [&](int r) { return march ? (int64_t)(kMarchK + wmax) * rup(r + lextmax) : 0; };
     auto stage_of = [&](int r) { return std::max(xpart(r), mpart(r)) + (vals ? (int64_t)r * maxlen : 0); };
     while (rows >= 32 && (size_t)S * (size_t)stage_of(rows) * sizeof(T) + 32 * S + 64 > kPtileSmemBudget) rows -= 32;
+    if (rows < 32 && march) {   // lines too long for K + W per stage (wide 3-D grids): single-line tiles
+        march = false;
+        for (int q = 0; q < nsets; ++q) tt.D[q] = 0;
+        rows = std::max(32, range_bytes / (int)sizeof(T) / 32 * 32);
+        while (rows >= 32 && (size_t)S * (size_t)stage_of(rows) * sizeof(T) + 32 * S + 64 > kPtileSmemBudget) rows -= 32;
+    }
     if (rows < 32) return PEPP_OK;
     for (int q = 0; q < nsets && march; ++q) {
         if (!tt.D[q]) continue;
