@@ -424,6 +424,15 @@ def config_leg(name: str, args, dev, stream, peak: float, with_cpu: bool) -> dic
              "graph_us_per_call": graph_us}
         if small:
             d["note"] = "launch-latency bound (20 K nnz): frac not a roofline claim; see graph_us_per_call"
+        if name in ("uniform1m", "zipf4m", "skew"):
+            # random columns: one x gather (a 32-B sector for 8 B) per stored
+            # entry; the ceiling is the measured random-gather rate from an
+            # L2-resident x, not HBM bandwidth
+            gps = A.nnz / (us * 1e-6)
+            d["gather_bound"] = {"gathers_per_spmv": int(A.nnz), "achieved_g_per_s": round(gps / 1e9, 1),
+                                 "ceiling_g_per_s": GATHER_CEILING_G, "frac": round(gps / 1e9 / GATHER_CEILING_G, 4),
+                                 "ceiling_source": "tools/experiments/gather_probe.cu: random 8-B gathers from an "
+                                                   "L2-resident x on this B200 pool, any load path (DESIGN §6)"}
         if with_cpu:
             import oracle
             t2 = time.perf_counter()
@@ -440,6 +449,8 @@ def config_leg(name: str, args, dev, stream, peak: float, with_cpu: bool) -> dic
         plan.close()
         torch.cuda.empty_cache()
 
+
+GATHER_CEILING_G = 255.0   # G random 8-B gathers / s from L2 (measured)
 
 # --------------------------------------------------------------- arms
 METRIC = "SpMV GFLOP/s (aggregate over ranks); achieved HBM GB/s in 'hbm'"
