@@ -1156,7 +1156,12 @@ __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wa
 // from DRAM (a 5-point stencil's three ranges meet again in L2 as the grid's
 // front advances: ±n grid rows are ~64 KB apart), and nothing goes through
 // the L1 gather path that held the register form at ~0.6 of the copy peak
-// (one 32-B sector request per SM cycle: ~26 sectors per chunk).
+// (one 32-B sector request per SM cycle: ~26 sectors per chunk). Grid
+// stencils' pattern tiles come as multi-line tiles (PatTiles.D: K lines of a
+// column, each x line copied once). The chunks outside the tiles (grid
+// edges) are walked by the CTA's last warps with the general SELL walk.
+// One persistent CTA per SM: warp 0 producer, warps 1-8 consumers, then
+// the walkers (DESIGN §6 "SELL tiles" has the measured design steps).
 // =====================================================================
 constexpr int kTileMaxSets = 32, kTileMaxLen = 16;
 struct PatTiles {
