@@ -338,7 +338,10 @@ __device__ __forceinline__ T sell_chunk(const T* __restrict__ val, const int* __
 // by value as a kernel parameter (constant bank: uniform LDC reads, no
 // memory stream). The chunk reads only x and writes y.
 constexpr int kSellMaxPatterns = 32;
-constexpr int kSellMaxPatternLen = 8;
+#ifndef PEPP_PAT_MAXLEN
+#define PEPP_PAT_MAXLEN 16   // slots of a pattern-table entry (9-point / 3-D stencils up to 16 slots)
+#endif
+constexpr int kSellMaxPatternLen = PEPP_PAT_MAXLEN;
 template <typename T>
 struct SellPatterns {
     int len[kSellMaxPatterns];
@@ -457,8 +460,22 @@ __device__ __forceinline__ T sell_pattern_chunk(const SellPatterns<T>& pt, int p
     case 6: return sell_pattern_slots<6, T>(pt, pid, row0, x);
     case 7: return sell_pattern_slots<7, T>(pt, pid, row0, x);
     case 8: return sell_pattern_slots<8, T>(pt, pid, row0, x);
-    default: return T(0);
+    default: break;
     }
+    if constexpr (kSellMaxPatternLen > 8) {
+        switch (pt.len[pid]) {
+        case 9: return sell_pattern_slots<9, T>(pt, pid, row0, x);
+        case 10: return sell_pattern_slots<10, T>(pt, pid, row0, x);
+        case 11: return sell_pattern_slots<11, T>(pt, pid, row0, x);
+        case 12: return sell_pattern_slots<12, T>(pt, pid, row0, x);
+        case 13: return sell_pattern_slots<13, T>(pt, pid, row0, x);
+        case 14: return sell_pattern_slots<14, T>(pt, pid, row0, x);
+        case 15: return sell_pattern_slots<15, T>(pt, pid, row0, x);
+        case 16: return sell_pattern_slots<16, T>(pt, pid, row0, x);
+        default: break;
+        }
+    }
+    return T(0);
 }
 
 // Stencil list (σ = 1 plans whose stencil chunks keep their values, i.e. not
@@ -742,7 +759,7 @@ __device__ __forceinline__ void sell_walk(int nrows, int nchunks, const int64_t*
 // PAT: the plan has pattern chunks (phase A + genlist); PAT = false compiles
 // the general kernel without them (no extra registers, no 3 KB parameter).
 #ifndef PEPP_PAT_MINB
-#define PEPP_PAT_MINB 1   // experiments: minimum resident blocks per SM for the PAT (value-compressed) instances
+#define PEPP_PAT_MINB 2   // minimum resident blocks per SM for the σ = 1 PAT (value-compressed) instance: with 16-slot patterns it would take 208 registers (1 block per SM)
 #endif
 template <int BLOCK, bool SORTED, bool PAT, typename T>
 __global__ void __launch_bounds__(BLOCK, (PAT && !SORTED) ? PEPP_PAT_MINB : 1) sell_kernel(int nrows, int nchunks, const int64_t* __restrict__ chunk_ptr,
@@ -787,7 +804,23 @@ __global__ void __launch_bounds__(BLOCK, (PAT && !SORTED) ? PEPP_PAT_MINB : 1) s
             case 5: k0 = sell_pattern_run<5, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
             case 6: k0 = sell_pattern_run<6, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
             case 7: k0 = sell_pattern_run<7, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
-            default: k0 = sell_pattern_run<8, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            case 8: k0 = sell_pattern_run<8, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+            default:
+                if constexpr (kSellMaxPatternLen > 8) {
+                    switch (pt.len[pid]) {
+                    case 9: k0 = sell_pattern_run<9, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+                    case 10: k0 = sell_pattern_run<10, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+                    case 11: k0 = sell_pattern_run<11, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+                    case 12: k0 = sell_pattern_run<12, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+                    case 13: k0 = sell_pattern_run<13, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+                    case 14: k0 = sell_pattern_run<14, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+                    case 15: k0 = sell_pattern_run<15, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+                    default: k0 = sell_pattern_run<16, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y); break;
+                    }
+                } else {
+                    k0 = sell_pattern_run<8, T>(pt, pid, patlist, npatc, k0, nwarps, e, lane, x, y);
+                }
+                break;
             }
             if (k0 >= npatc) break;
             for (int u = 0; u < kPatU; ++u) {   // the mixed group
@@ -1197,7 +1230,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 template <int NC, int N, bool VALS, typename T>
 __device__ __forceinline__ void tile_rows(const SellPatterns<T>& pt, const int* sidx, int q, const T* sx,
                                           const T* sv, T* __restrict__ y, int nr, int c, int xspan) {
-    constexpr int U = !VALS ? PEPP_PTILE_U : (N <= 4 ? 4 : N <= 8 ? 2 : 1);
+    constexpr int U = !VALS ? (N <= 8 ? PEPP_PTILE_U : 2) : (N <= 4 ? 4 : N <= 8 ? 2 : 1);
     int b[N];
     T w[N];
 #pragma unroll
@@ -1357,8 +1390,15 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
                 const int span = stage_elems - l * tt.lws[q];
 #define PEPP_TM(N) case N: tile_rows<NC, N, VALS, T>(pt, tt.msidx[q], q, xl, vs, yl, nr, c, span); break;
                 switch (tt.len[q]) {
-                PEPP_TM(1) PEPP_TM(2) PEPP_TM(3) PEPP_TM(4) PEPP_TM(5) PEPP_TM(6) PEPP_TM(7)
-                default: tile_rows<NC, 8, VALS, T>(pt, tt.msidx[q], q, xl, vs, yl, nr, c, span); break;
+                PEPP_TM(1) PEPP_TM(2) PEPP_TM(3) PEPP_TM(4) PEPP_TM(5) PEPP_TM(6) PEPP_TM(7) PEPP_TM(8)
+                default:
+                    if constexpr (kSellMaxPatternLen > 8) {
+                        switch (tt.len[q]) {
+                        PEPP_TM(9) PEPP_TM(10) PEPP_TM(11) PEPP_TM(12) PEPP_TM(13) PEPP_TM(14) PEPP_TM(15)
+                        default: tile_rows<NC, 16, VALS, T>(pt, tt.msidx[q], q, xl, vs, yl, nr, c, span); break;
+                        }
+                    }
+                    break;
                 }
 #undef PEPP_TM
             }
@@ -1371,6 +1411,11 @@ __global__ void __launch_bounds__(BLOCK, 1) sell_tile_kernel(const __grid_consta
         PEPP_TR(1) PEPP_TR(2) PEPP_TR(3) PEPP_TR(4) PEPP_TR(5) PEPP_TR(6) PEPP_TR(7)
         default:
             if constexpr (VALS) {
+                switch (tt.len[q]) {
+                PEPP_TR(8) PEPP_TR(9) PEPP_TR(10) PEPP_TR(11) PEPP_TR(12) PEPP_TR(13) PEPP_TR(14) PEPP_TR(15)
+                default: tile_rows<NC, 16, VALS, T>(pt, tt.sidx[q], q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems); break;
+                }
+            } else if constexpr (kSellMaxPatternLen > 8) {
                 switch (tt.len[q]) {
                 PEPP_TR(8) PEPP_TR(9) PEPP_TR(10) PEPP_TR(11) PEPP_TR(12) PEPP_TR(13) PEPP_TR(14) PEPP_TR(15)
                 default: tile_rows<NC, 16, VALS, T>(pt, tt.sidx[q], q, xs, vs, yt, nr, c, VALS ? vstage : stage_elems); break;

@@ -1586,6 +1586,19 @@ template <typename T> const pepp::k::SellPatterns<T>& sell_pattern_table(const p
 template <> const pepp::k::SellPatterns<double>& sell_pattern_table<double>(const pepp_spmv_plan_t* p) { return p->pat64; }
 template <> const pepp::k::SellPatterns<float>& sell_pattern_table<float>(const pepp_spmv_plan_t* p) { return p->pat32; }
 
+// The walker warps are a handful per SM: they take the chunks outside the
+// tiles only when those are few next to the tiled ones (grid edges). A plan
+// whose tiles are a small part (e.g. a few constant-stencil regions in an
+// otherwise general matrix) walks the rest with the full-grid SELL kernel on
+// the side stream — with the walkers, 524 K general chunks of a 9-point
+// stencil beside 250 tiled ones took 34.8 ms instead of ~0.3 ms.
+#ifndef PEPP_WALK_RATIO
+#define PEPP_WALK_RATIO 16   // walkers when (chunks outside the tiles) x 16 <= tiled chunks
+#endif
+bool walkers_suffice(const pepp_spmv_plan_t* p, const TileLayout& L) {
+    return (int64_t)p->ngen * PEPP_WALK_RATIO <= L.chunks;
+}
+
 // the side stream of a tile call: forked after the work already on st
 pepp_status_t side_fork(pepp_spmv_plan_t* p, cudaStream_t st, cudaStream_t* gs) {
     *gs = p->gside && PEPP_EXP_TILE_SIDE == 0 ? p->gside : st;
@@ -1685,7 +1698,7 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
             // pattern tiles (bulk-copied x ranges); the grid-edge chunks by the
             // tile kernel's walker warps, or — with untiled pattern chunks
             // left (phase A) or no walkers — by the genlist walk beside it
-            const bool inwalk = tile_walkers<false>() > 0 && p->npatrest == 0;
+            const bool inwalk = tile_walkers<false>() > 0 && p->npatrest == 0 && walkers_suffice(p, p->ptl);
             pepp_status_t s2 = tile_launch<false, T>(p, p->ptl, inwalk, x, y, st);
             if (s2) return s2;
             if (!inwalk && p->ngen + p->npatrest > 0) {
@@ -1706,7 +1719,7 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
             // stencil tiles (bulk-copied x ranges and values); the grid-edge
             // chunks by the walker warps; untiled list entries (and, without
             // walkers, the grid-edge chunks) beside it on the side stream
-            const bool inwalk = tile_walkers<true>() > 0;
+            const bool inwalk = tile_walkers<true>() > 0 && walkers_suffice(p, p->stl);
             pepp_status_t s2 = tile_launch<true, T>(p, p->stl, inwalk, x, y, st);
             if (s2) return s2;
             if (p->nstrest || (!inwalk && p->ngen > 0)) {
@@ -1791,10 +1804,12 @@ int launches_for(const pepp_spmv_plan_t* p, const Candidate& c, const void* x, c
         return p->ntiles > 0 ? 2 + (p->nlongruns > 0) : 0;
     case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
     case PEPP_V_SELL:
-        return (p->d_stlist ? (p->stl.ntiles && al ? 1 + (p->nstrest > 0) + (tile_walkers<true>() == 0 && p->ngen > 0)
+        return (p->d_stlist ? (p->stl.ntiles && al ? 1 + (p->nstrest > 0) +
+                                                         ((tile_walkers<true>() == 0 || !walkers_suffice(p, p->stl)) && p->ngen > 0)
                                                    : 1 + (p->ngen > 0))
                             : (p->d_patlist && p->ptl.ntiles && al)
-                                  ? 1 + ((tile_walkers<false>() == 0 || p->npatrest > 0) && p->ngen + p->npatrest > 0)
+                                  ? 1 + ((tile_walkers<false>() == 0 || p->npatrest > 0 || !walkers_suffice(p, p->ptl)) &&
+                                         p->ngen + p->npatrest > 0)
                                   : 1) +
                (p->nsell_mid > 0) + (p->nsell_seg > 0);
     case PEPP_V_PANEL:

@@ -177,3 +177,42 @@ def test_multiline_pattern_tiles(name):
     y1, _ = _y(A, xr, True)
     y2, _ = _y(A, xr, True, shift=1)   # register path
     assert np.array_equal(_bits(y1), _bits(y2))
+
+
+def test_nine_point_value_compression_multiline():
+    """A 9-slot constant stencil (3x3) is a pattern-table entry (up to 16
+    slots): value-compressed, multi-line tiles, bit-identical to the streamed
+    layout and to the oracle."""
+    offs = [(a, b) for a in (-1, 0, 1) for b in (-1, 0, 1)]
+    A = _stencil_grid(512, offs, 8.0, -1.0)
+    x = gen.vector(3, gen.INT8, A.ncols)
+    y1, i1 = _y(A, x, True)
+    y0, i0 = _y(A, x, False)
+    assert i1["sell_constval_frac"] > 0.8 and i1["sell_tile_multiline"] > 0 and i0["sell_constval_frac"] == 0.0
+    assert np.array_equal(_bits(y1), _bits(y0))
+    _check(A, x, y1, True)
+
+
+def test_few_tiles_many_general_chunks():
+    """A plan whose pattern tiles are a small part of the matrix (a constant
+    block in an otherwise random-valued band): the chunks outside the tiles
+    are walked by the full-grid SELL kernel beside the tile kernel (two
+    launches), not by the tile kernel's few walker warps; y equals the oracle."""
+    B = gen.banded(1 << 20, 4, seed=11, val_mode=gen.INT4)
+    rp = np.asarray(B.row_ptr)
+    val = B.val.copy()
+    for r in range(64, 4096):                       # a constant 9-point block: 125 full chunks
+        s, e = int(rp[r]), int(rp[r + 1])
+        val[s:e] = np.where(B.col[s:e] == r, 8.0, -1.0)
+    C = gen.CSR(B.nrows, B.ncols, B.row_ptr, B.col, val, 0, B.nrows)
+    x = gen.vector(5, gen.INT8, C.ncols)
+    with pepp.Plan.from_csr(C, variant_mask=1 << pepp.V_SELL) as plan:
+        xd = torch.from_numpy(x).cuda()
+        y = torch.full((C.nrows,), float("nan"), dtype=torch.float64, device="cuda")
+        for _ in range(3):
+            u = plan.exec(xd, y)
+        torch.cuda.synchronize()
+        info = plan.info()
+        assert 0 < info["sell_ptile_frac"] < 0.01, info
+        assert u.launches == 2
+        assert np.array_equal(y.cpu().numpy(), oracle.spmv(C, x))
