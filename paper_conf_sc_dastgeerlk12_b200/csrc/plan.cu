@@ -583,6 +583,13 @@ constexpr size_t kPtileSmemBudget = (size_t)PEPP_PTILE_SMEM_KB * 1024;
 #define PEPP_MTILE_LINE_KB 16   // x bytes per line (rows per line = 16 KB / value size)
 #endif
 constexpr int kMarchK = PEPP_MTILE_K, kMarchLineBytes = PEPP_MTILE_LINE_KB * 1024;
+#ifndef PEPP_TILE_MIN_ROWS_VALS
+#define PEPP_TILE_MIN_ROWS_VALS 768    // mean rows per tile below which a plan keeps the register path (values streamed)
+#endif
+#ifndef PEPP_TILE_MIN_ROWS_PAT
+#define PEPP_TILE_MIN_ROWS_PAT 1536    // ... (pattern tiles)
+#endif
+constexpr int kTileMinRowsVals = PEPP_TILE_MIN_ROWS_VALS, kTileMinRowsPat = PEPP_TILE_MIN_ROWS_PAT;
 
 #ifndef PEPP_TILE_SIDE_BPS
 #define PEPP_TILE_SIDE_BPS 8   // blocks per SM (cap) of the walks beside a tile kernel; measured 1 / 2 / 8: vc config 4 207.5 / 197.9 / 197.0 us, fp32 list 293 / 282 / 282 us
@@ -771,6 +778,15 @@ pepp_status_t sell_build_tiles(pepp_spmv_plan_t* p, int nsets, const int* lens, 
         i = j;
     }
     if (tiles.empty()) { rest->clear(); return PEPP_OK; }
+    // tiles pay only on long runs (tools/r2/tile_vs_reg.py, tile / register
+    // µs): 2-D Laplacians n = 512 / 1024 / 2048 / 4096 — values streamed 1.01 /
+    // 0.74 / 0.88 / 0.87, value-compressed 1.35 / 1.21 / 0.82 / 0.69; 3-D
+    // 7-point (5 clusters, runs of 2-8 chunks) 1.3-2.3. Short runs leave the
+    // chunks to the register paths.
+    if (tiled * 32 < (int64_t)tiles.size() * (vals ? kTileMinRowsVals : kTileMinRowsPat)) {
+        rest->clear();
+        return PEPP_OK;
+    }
     if (march) {
         // columns: tiles of one set and length whose first rows differ by D,
         // cut into blocks of <= K lines; a block of >= 2 lines becomes one
@@ -1593,10 +1609,12 @@ template <> const pepp::k::SellPatterns<float>& sell_pattern_table<float>(const 
 // the side stream — with the walkers, 524 K general chunks of a 9-point
 // stencil beside 250 tiled ones took 34.8 ms instead of ~0.3 ms.
 #ifndef PEPP_WALK_RATIO
-#define PEPP_WALK_RATIO 16   // walkers when (chunks outside the tiles) x 16 <= tiled chunks
-#endif
+#define PEPP_WALK_RATIO 16   // walkers when (chunks outside the tiles) x 16 <= tiled chunks,
+#endif                       // or at most 8 of them per walker warp
+template <bool VALS>
 bool walkers_suffice(const pepp_spmv_plan_t* p, const TileLayout& L) {
-    return (int64_t)p->ngen * PEPP_WALK_RATIO <= L.chunks;
+    const int64_t walkers = (int64_t)tile_walkers<VALS>() * L.grid;
+    return (int64_t)p->ngen * PEPP_WALK_RATIO <= L.chunks || (int64_t)p->ngen <= 8 * walkers;
 }
 
 // the side stream of a tile call: forked after the work already on st
@@ -1698,7 +1716,7 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
             // pattern tiles (bulk-copied x ranges); the grid-edge chunks by the
             // tile kernel's walker warps, or — with untiled pattern chunks
             // left (phase A) or no walkers — by the genlist walk beside it
-            const bool inwalk = tile_walkers<false>() > 0 && p->npatrest == 0 && walkers_suffice(p, p->ptl);
+            const bool inwalk = tile_walkers<false>() > 0 && p->npatrest == 0 && walkers_suffice<false>(p, p->ptl);
             pepp_status_t s2 = tile_launch<false, T>(p, p->ptl, inwalk, x, y, st);
             if (s2) return s2;
             if (!inwalk && p->ngen + p->npatrest > 0) {
@@ -1719,7 +1737,7 @@ pepp_status_t launch_t(pepp_spmv_plan_t* p, const Candidate& c, const T* x, T* y
             // stencil tiles (bulk-copied x ranges and values); the grid-edge
             // chunks by the walker warps; untiled list entries (and, without
             // walkers, the grid-edge chunks) beside it on the side stream
-            const bool inwalk = tile_walkers<true>() > 0 && walkers_suffice(p, p->stl);
+            const bool inwalk = tile_walkers<true>() > 0 && walkers_suffice<true>(p, p->stl);
             pepp_status_t s2 = tile_launch<true, T>(p, p->stl, inwalk, x, y, st);
             if (s2) return s2;
             if (p->nstrest || (!inwalk && p->ngen > 0)) {
@@ -1805,10 +1823,10 @@ int launches_for(const pepp_spmv_plan_t* p, const Candidate& c, const void* x, c
     case PEPP_V_CSR_STREAM: return p->nitems > 0 ? 1 + (p->nlong > 0) : 0;
     case PEPP_V_SELL:
         return (p->d_stlist ? (p->stl.ntiles && al ? 1 + (p->nstrest > 0) +
-                                                         ((tile_walkers<true>() == 0 || !walkers_suffice(p, p->stl)) && p->ngen > 0)
+                                                         ((tile_walkers<true>() == 0 || !walkers_suffice<true>(p, p->stl)) && p->ngen > 0)
                                                    : 1 + (p->ngen > 0))
                             : (p->d_patlist && p->ptl.ntiles && al)
-                                  ? 1 + ((tile_walkers<false>() == 0 || p->npatrest > 0 || !walkers_suffice(p, p->ptl)) &&
+                                  ? 1 + ((tile_walkers<false>() == 0 || p->npatrest > 0 || !walkers_suffice<false>(p, p->ptl)) &&
                                          p->ngen + p->npatrest > 0)
                                   : 1) +
                (p->nsell_mid > 0) + (p->nsell_seg > 0);

@@ -84,7 +84,7 @@ def main() -> int:
         bad += 0 if np.array_equal(y32.cpu().numpy(), oracle.spmv(A32, x32)) else 1
     # SELL tiles (bulk-copied ranges, producer / consumer mbarrier ring):
     # pattern tiles and stencil tiles, fp64 and fp32, more tiles than CTAs
-    L = gen.laplacian2d(256)
+    L = gen.laplacian2d(2048)   # long runs: tiles in both layouts
     for dt in (np.float64, np.float32):
         Ld = gen.CSR(L.nrows, L.ncols, L.row_ptr, L.col, L.val.astype(dt), L.r0, L.global_nrows, L.name)
         xl = gen.vector(5, gen.INT8, L.ncols).astype(dt)
