@@ -941,7 +941,11 @@ pepp_status_t sell_patterns(pepp_spmv_plan_t* p, int64_t nsb, const void* d_scon
         cp[c] = pid;
         ++used;
     }
-    if (!used) return PEPP_OK;
+    // value compression only where it covers most chunks: a minority of
+    // pattern chunks would keep the plan off the stencil list / stencil tiles
+    // for all its other stencil chunks (the list and the pattern table are
+    // alternatives), which costs more than the few values it saves
+    if (!used || 2 * used < (int64_t)nc) { *pt = pepp::k::SellPatterns<T>{}; return PEPP_OK; }
     PEPP_CUDA_TRY(cudaMemcpy(p->d_chunk_len, clen.data(), sizeof(int) * nc, cudaMemcpyHostToDevice));
     PEPP_CUDA_TRY(cudaMemcpy(p->d_chunk_ptr, cp.data(), sizeof(int64_t) * nc, cudaMemcpyHostToDevice));
     p->sell_const_chunks = used;
