@@ -162,7 +162,7 @@ struct pepp_spmv_plan_s {
     int* d_patlist = nullptr;        // σ = 1: pattern chunks as (chunk << 5 | id), phase A of the kernel
     int* d_genlist = nullptr;        // σ = 1: the other chunks, phase B
     int npatc = 0, ngen = 0;
-    // pattern tiles (sell_ptile_kernel): runs of pattern chunks cut into
+    // pattern tiles (sell_tile_kernel<…, VALS = false>): runs of pattern chunks cut into
     // tiles whose x ranges are bulk-copied; the pattern chunks no tile holds
     // stay in d_patrest for phase A of the genlist walk
     TileLayout ptl;                  // pattern tiles
