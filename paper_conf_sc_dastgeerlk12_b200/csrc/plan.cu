@@ -614,7 +614,10 @@ int tile_side_grid(const pepp_spmv_plan_t* p, int grid) {
 #define PEPP_TILE_WALKERS_P 6   // pattern tiles
 #endif
 template <bool VALS> constexpr int tile_walkers() { return VALS ? PEPP_TILE_WALKERS_S : PEPP_TILE_WALKERS_P; }
-template <bool VALS> constexpr int tile_block() { return kPtileBlock + 32 * tile_walkers<VALS>(); }
+#ifndef PEPP_STILE_BLOCK
+#define PEPP_STILE_BLOCK 416   // producer + 12 consumer warps for stencil tiles (values streamed): config 4 fp64 549-552 vs 561-564 us with 8 (3 alternating repeats, tools/r2/gpu_sblock.sh), fp32 equal
+#endif
+template <bool VALS> constexpr int tile_block() { return (VALS ? PEPP_STILE_BLOCK : kPtileBlock) + 32 * tile_walkers<VALS>(); }
 
 template <int S, bool VALS, typename T>
 const void* tile_kernel_fn() { return (const void*)pepp::k::sell_tile_kernel<tile_block<VALS>(), S, VALS, T, tile_walkers<VALS>()>; }
